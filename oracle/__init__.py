@@ -1,0 +1,150 @@
+"""ctypes wrapper of the CPU oracle (oracle/oracle.c).
+
+TEST INFRASTRUCTURE, NOT PRODUCT CODE: only tests/, __graft_entry__.smoke() and
+bench.py's cpu_baseline / ``--impl reference`` legs may import this package.  It
+never imports the product package and the product package never imports it.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+import subprocess
+import threading
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "oracle.c")
+_LIB = os.path.join(_HERE, "liboracle.so")
+_lock = threading.Lock()
+_lib = None
+
+REC = 14  # uint64 words per FPM result record (see oracle.c)
+
+
+def build(force: bool = False) -> str:
+    """Compile liboracle.so with gcc (-O2 -fopenmp); returns its path."""
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+        tmp = _LIB + f".tmp{os.getpid()}"
+        subprocess.check_call(["gcc", "-O2", "-g", "-fopenmp", "-fPIC", "-shared", "-std=c11",
+                               "-Wall", "-Wno-unused-function", "-o", tmp, _SRC])
+        os.replace(tmp, _LIB)
+    return _LIB
+
+
+def lib():
+    global _lib
+    with _lock:
+        if _lib is None:
+            L = C.CDLL(build())
+            u32p = np.ctypeslib.ndpointer(np.uint32, flags="C_CONTIGUOUS")
+            u64p = np.ctypeslib.ndpointer(np.uint64, flags="C_CONTIGUOUS")
+            L.og_build.restype = C.c_void_p
+            L.og_build.argtypes = [C.c_uint32, C.c_uint64, u32p, u32p, C.c_void_p]
+            L.og_free.argtypes = [C.c_void_p]
+            L.og_n.restype = C.c_uint32; L.og_n.argtypes = [C.c_void_p]
+            L.og_m.restype = C.c_uint64; L.og_m.argtypes = [C.c_void_p]
+            L.og_csr.argtypes = [C.c_void_p, u64p, u32p]
+            L.og_kclique.restype = C.c_uint64
+            L.og_kclique.argtypes = [C.c_void_p, C.c_uint32, C.c_int, C.c_int]
+            L.og_kclique_roots.argtypes = [C.c_void_p, C.c_uint32, C.c_uint64, u32p, u64p, C.c_int]
+            L.og_match.restype = C.c_int
+            L.og_match.argtypes = [C.c_void_p, C.c_uint32, C.c_uint32, u32p, C.c_void_p, C.c_int,
+                                   C.POINTER(C.c_uint64), C.POINTER(C.c_uint64), C.POINTER(C.c_uint64)]
+            L.og_fpm.restype = C.c_int64
+            L.og_fpm.argtypes = [C.c_void_p, C.c_uint32, C.c_uint64, C.c_int, C.c_int, C.c_uint64,
+                                 u64p, C.c_uint64]
+            L.og_pattern_mni.restype = C.c_int
+            L.og_pattern_mni.argtypes = [C.c_void_p, C.c_uint32, C.c_uint32, u32p, C.c_void_p, C.c_int,
+                                         C.POINTER(C.c_uint64)]
+            _lib = L
+    return _lib
+
+
+class Graph:
+    """O-0 normalised undirected simple graph held by the oracle."""
+
+    def __init__(self, n: int, src, dst, labels=None):
+        L = lib()
+        src = np.ascontiguousarray(src, dtype=np.uint32)
+        dst = np.ascontiguousarray(dst, dtype=np.uint32)
+        assert src.shape == dst.shape
+        self._labels = None if labels is None else np.ascontiguousarray(labels, dtype=np.uint32)
+        lp = None if self._labels is None else self._labels.ctypes.data
+        self._h = L.og_build(int(n), int(src.size), src, dst, lp)
+        if not self._h:
+            raise ValueError("oracle: invalid edge list (vertex id >= n)")
+
+    def __del__(self):
+        h = getattr(self, "_h", None)
+        if h:
+            lib().og_free(h)
+            self._h = None
+
+    @property
+    def n(self) -> int:
+        return lib().og_n(self._h)
+
+    @property
+    def m(self) -> int:
+        return lib().og_m(self._h)
+
+    def csr(self):
+        off = np.empty(self.n + 1, np.uint64)
+        adj = np.empty(2 * self.m, np.uint32)
+        lib().og_csr(self._h, off, adj)
+        return off, adj
+
+    def kclique(self, k: int, order: str = "degree", threads: int = 0) -> int:
+        return int(lib().og_kclique(self._h, k, 0 if order == "degree" else 1, threads))
+
+    def kclique_roots(self, k: int, roots, threads: int = 0) -> np.ndarray:
+        roots = np.ascontiguousarray(roots, dtype=np.uint32)
+        out = np.zeros(roots.size, np.uint64)
+        lib().og_kclique_roots(self._h, k, roots.size, roots, out, threads)
+        return out
+
+    def match(self, nv: int, edges, plabels=None, threads: int = 0):
+        """Return (count, mappings, |Aut_L|)."""
+        e = np.ascontiguousarray(np.asarray(edges, dtype=np.uint32).reshape(-1))
+        pl = None if plabels is None else np.ascontiguousarray(plabels, dtype=np.uint32)
+        c, mp, a = C.c_uint64(), C.c_uint64(), C.c_uint64()
+        st = lib().og_match(self._h, nv, e.size // 2, e, None if pl is None else pl.ctypes.data,
+                            threads, C.byref(c), C.byref(mp), C.byref(a))
+        if st != 0:
+            raise ValueError(f"oracle og_match status {st}")
+        return int(c.value), int(mp.value), int(a.value)
+
+    def fpm(self, l: int, minsup: int, method: str = "shapes", threads: int = 0,
+            pattern_cap: int = 1 << 16):
+        """Frequent patterns as a sorted list of (ne, nv, labels, edges, support, instances).
+
+        ``instances`` is the number of connected edge sets mapped to the pattern."""
+        cap = 1 << 14
+        while True:
+            out = np.zeros(cap * REC, np.uint64)
+            n = lib().og_fpm(self._h, l, minsup, 0 if method == "shapes" else 1, threads, cap, out,
+                             pattern_cap)
+            if n < 0:
+                raise ValueError(f"oracle og_fpm status {n}")
+            if n <= cap:
+                break
+            cap = n
+        res = []
+        for i in range(n):
+            r = out[i * REC:(i + 1) * REC]
+            ne, nv = int(r[0]), int(r[1])
+            res.append((ne, nv, tuple(int(x) for x in r[2:2 + nv]),
+                        tuple((int(r[6 + 2 * e]), int(r[7 + 2 * e])) for e in range(ne)), int(r[12]),
+                        int(r[13])))
+        return res
+
+    def pattern_mni(self, nv: int, edges, plabels=None, threads: int = 0) -> int:
+        e = np.ascontiguousarray(np.asarray(edges, dtype=np.uint32).reshape(-1))
+        pl = None if plabels is None else np.ascontiguousarray(plabels, dtype=np.uint32)
+        s = C.c_uint64()
+        st = lib().og_pattern_mni(self._h, nv, e.size // 2, e, None if pl is None else pl.ctypes.data,
+                                  threads, C.byref(s))
+        if st != 0:
+            raise ValueError(f"oracle og_pattern_mni status {st}")
+        return int(s.value)

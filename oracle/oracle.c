@@ -1,0 +1,669 @@
+/*
+ * oracle/oracle.c -- the CPU ORACLE for the GAMMA hot path.
+ *
+ * TEST INFRASTRUCTURE, NOT PRODUCT CODE.  Only tests/, __graft_entry__.smoke()
+ * and bench.py's cpu_baseline / --impl reference legs may load this library.
+ * It shares no code, header, table or helper with the CUDA path
+ * (paper_conf_icde_hu0o23_b200/csrc); the only shared inputs are the raw arrays
+ * drawn by gamma_gen/.
+ *
+ * Every function is the plain definition, written slowly and checkably:
+ *   og_build       O-0  undirected simple graph from raw samples
+ *                       (§IV "CSR ... made up of adjacency lists";
+ *                        L119, L204: one label per vertex, no edge labels)
+ *   og_kclique     O-1  |{S subset of V : |S|=k, S a clique}|
+ *   og_match       O-2  #injective label-preserving edge-preserving maps / |Aut_L(P)|
+ *                       ("all subgraphs isomorphic to a pattern P";
+ *                        Alg. 1)
+ *   og_fpm_*       O-3  edge-induced patterns with <= l edges and MNI support >= minsup
+ *                       (Alg. 2; MNI per
+ *                        DESIGN.md reading R1)
+ *
+ * Readings of the paper that these functions take are listed in DESIGN.md
+ * ("Readings").  Parity-pinning tests: tests/test_oracle_*.py.
+ */
+#include <stdint.h>
+#include <stdlib.h>
+#include <string.h>
+#include <omp.h>
+
+#define OG_OK 0
+#define OG_EINVAL -1
+#define OG_ENOMEM -2
+#define OG_ENOTDIV -3
+
+typedef struct {
+  uint32_t n;
+  uint64_t m;        /* undirected edges after O-0 */
+  uint64_t *off;     /* n+1 offsets into adj */
+  uint32_t *adj;     /* 2m entries, every list ascending by vertex id */
+  uint32_t *lab;     /* n labels (all 0 when none given) */
+} og_graph;
+
+static int cmp_u64(const void *a, const void *b) {
+  uint64_t x = *(const uint64_t *)a, y = *(const uint64_t *)b;
+  return (x > y) - (x < y);
+}
+static int cmp_u32(const void *a, const void *b) {
+  uint32_t x = *(const uint32_t *)a, y = *(const uint32_t *)b;
+  return (x > y) - (x < y);
+}
+
+static void set_threads(int threads) {
+  if (threads > 0) omp_set_num_threads(threads);
+}
+
+/* ---------------------------------------------------------------------------
+ * O-0: symmetrise, drop self-loops, drop duplicates, sort every list.
+ * ------------------------------------------------------------------------- */
+og_graph *og_build(uint32_t n, uint64_t m_raw, const uint32_t *src, const uint32_t *dst,
+                   const uint32_t *labels) {
+  og_graph *g = (og_graph *)calloc(1, sizeof(og_graph));
+  if (!g) return NULL;
+  g->n = n;
+  uint64_t *key = (uint64_t *)malloc((m_raw ? m_raw : 1) * sizeof(uint64_t));
+  uint64_t k = 0;
+  for (uint64_t i = 0; i < m_raw; i++) {
+    uint32_t u = src[i], v = dst[i];
+    if (u >= n || v >= n) { free(key); free(g); return NULL; }
+    if (u == v) continue;                       /* no self-loops */
+    uint32_t a = u < v ? u : v, b = u < v ? v : u;
+    key[k++] = ((uint64_t)a << 32) | b;         /* one key per undirected edge */
+  }
+  qsort(key, k, sizeof(uint64_t), cmp_u64);
+  uint64_t m = 0;
+  for (uint64_t i = 0; i < k; i++)              /* drop duplicates */
+    if (i == 0 || key[i] != key[i - 1]) key[m++] = key[i];
+  g->m = m;
+  uint64_t *deg = (uint64_t *)calloc((size_t)n + 1, sizeof(uint64_t));
+  for (uint64_t i = 0; i < m; i++) { deg[key[i] >> 32]++; deg[key[i] & 0xffffffffu]++; }
+  g->off = (uint64_t *)malloc(((size_t)n + 1) * sizeof(uint64_t));
+  g->off[0] = 0;
+  for (uint32_t v = 0; v < n; v++) g->off[v + 1] = g->off[v] + deg[v];
+  g->adj = (uint32_t *)malloc((m > 0 ? 2 * m : 1) * sizeof(uint32_t));
+  for (uint32_t v = 0; v < n; v++) deg[v] = g->off[v];   /* reuse as fill cursor */
+  for (uint64_t i = 0; i < m; i++) {
+    uint32_t a = (uint32_t)(key[i] >> 32), b = (uint32_t)(key[i] & 0xffffffffu);
+    g->adj[deg[a]++] = b;
+    g->adj[deg[b]++] = a;
+  }
+  for (uint32_t v = 0; v < n; v++)
+    qsort(g->adj + g->off[v], g->off[v + 1] - g->off[v], sizeof(uint32_t), cmp_u32);
+  g->lab = (uint32_t *)malloc(((size_t)n ? n : 1) * sizeof(uint32_t));
+  for (uint32_t v = 0; v < n; v++) g->lab[v] = labels ? labels[v] : 0;
+  free(deg);
+  free(key);
+  return g;
+}
+
+void og_free(og_graph *g) {
+  if (!g) return;
+  free(g->off); free(g->adj); free(g->lab); free(g);
+}
+
+uint32_t og_n(const og_graph *g) { return g->n; }
+uint64_t og_m(const og_graph *g) { return g->m; }
+/* Copy out the symmetric CSR (off: n+1, adj: 2m). */
+void og_csr(const og_graph *g, uint64_t *off, uint32_t *adj) {
+  memcpy(off, g->off, ((size_t)g->n + 1) * sizeof(uint64_t));
+  memcpy(adj, g->adj, 2 * g->m * sizeof(uint32_t));
+}
+
+static uint64_t deg_of(const og_graph *g, uint32_t v) { return g->off[v + 1] - g->off[v]; }
+
+/* Is x in N(v)?  Plain binary search on the sorted list. */
+static int adjacent(const og_graph *g, uint32_t v, uint32_t x) {
+  uint64_t lo = g->off[v], hi = g->off[v + 1];
+  while (lo < hi) {
+    uint64_t mid = lo + (hi - lo) / 2;
+    uint32_t y = g->adj[mid];
+    if (y == x) return 1;
+    if (y < x) lo = mid + 1; else hi = mid;
+  }
+  return 0;
+}
+
+/* ---------------------------------------------------------------------------
+ * O-1: k-clique counting.  Each k-clique is counted once, at its lowest vertex
+ * under the order r(v) = (deg v, v) (order_mode 0) or r(v) = v (order_mode 1).
+ * Candidates are filtered by explicit adjacency checks (not list intersection).
+ * ------------------------------------------------------------------------- */
+static int r_less(const og_graph *g, int mode, uint32_t a, uint32_t b) {
+  if (mode == 1) return a < b;
+  uint64_t da = deg_of(g, a), db = deg_of(g, b);
+  return da < db || (da == db && a < b);
+}
+
+static uint64_t kcl_rec(const og_graph *g, int mode, uint32_t k, uint32_t size,
+                        const uint32_t *cand, uint64_t nc, uint32_t **buf) {
+  if (size == k - 1) return nc;   /* every remaining candidate completes a k-clique */
+  uint64_t total = 0;
+  uint32_t *next = buf[size];
+  for (uint64_t i = 0; i < nc; i++) {
+    uint32_t w = cand[i];
+    uint64_t nn = 0;
+    for (uint64_t j = 0; j < nc; j++) {
+      uint32_t x = cand[j];
+      if (r_less(g, mode, w, x) && adjacent(g, w, x)) next[nn++] = x;
+    }
+    total += kcl_rec(g, mode, k, size + 1, next, nn, buf);
+  }
+  return total;
+}
+
+static uint64_t max_degree(const og_graph *g) {
+  uint64_t md = 0;
+  for (uint32_t v = 0; v < g->n; v++) if (deg_of(g, v) > md) md = deg_of(g, v);
+  return md;
+}
+
+/* Count k-cliques whose lowest-ranked vertex is v (k >= 2). */
+static uint64_t kcl_root(const og_graph *g, int mode, uint32_t k, uint32_t v, uint32_t **buf) {
+  uint32_t *cand = buf[0];
+  uint64_t nc = 0;
+  for (uint64_t e = g->off[v]; e < g->off[v + 1]; e++)
+    if (r_less(g, mode, v, g->adj[e])) cand[nc++] = g->adj[e];
+  return kcl_rec(g, mode, k, 1, cand, nc, buf);
+}
+
+static uint32_t **alloc_bufs(uint32_t levels, uint64_t width) {
+  uint32_t **buf = (uint32_t **)malloc(levels * sizeof(uint32_t *));
+  for (uint32_t i = 0; i < levels; i++) buf[i] = (uint32_t *)malloc((width ? width : 1) * sizeof(uint32_t));
+  return buf;
+}
+static void free_bufs(uint32_t **buf, uint32_t levels) {
+  for (uint32_t i = 0; i < levels; i++) free(buf[i]);
+  free(buf);
+}
+
+uint64_t og_kclique(const og_graph *g, uint32_t k, int order_mode, int threads) {
+  if (k == 0) return 0;
+  if (k == 1) return g->n;
+  set_threads(threads);
+  uint64_t md = max_degree(g), total = 0;
+#pragma omp parallel reduction(+ : total)
+  {
+    uint32_t **buf = alloc_bufs(k + 1, md);
+#pragma omp for schedule(dynamic, 64)
+    for (int64_t v = 0; v < (int64_t)g->n; v++) total += kcl_root(g, order_mode, k, (uint32_t)v, buf);
+    free_bufs(buf, k + 1);
+  }
+  return total;
+}
+
+/* Per-root counts (order_mode 0 ranks) for sampled parity at full size. */
+void og_kclique_roots(const og_graph *g, uint32_t k, uint64_t nroots, const uint32_t *roots,
+                      uint64_t *counts, int threads) {
+  set_threads(threads);
+  uint64_t md = max_degree(g);
+#pragma omp parallel
+  {
+    uint32_t **buf = alloc_bufs(k + 1, md);
+#pragma omp for schedule(dynamic, 1)
+    for (int64_t i = 0; i < (int64_t)nroots; i++)
+      counts[i] = (k == 1) ? 1 : kcl_root(g, 0, k, roots[i], buf);
+    free_bufs(buf, k + 1);
+  }
+}
+
+/* ---------------------------------------------------------------------------
+ * O-2: labeled, non-induced subgraph matching.  count = mappings / |Aut_L(P)|.
+ * Matching order: BFS from pattern vertex 0 (deliberately not the GPU planner's
+ * order).  Candidates of pattern vertex q = N(phi(bfs parent of q)); every other
+ * backward edge checked by binary search; injectivity by linear scan.
+ * ------------------------------------------------------------------------- */
+#define OG_MAXV 8
+
+typedef struct {
+  uint32_t nv;
+  int adjm[OG_MAXV][OG_MAXV];
+  int labeled;
+  uint32_t plab[OG_MAXV];
+  uint32_t order[OG_MAXV];     /* BFS order */
+  uint32_t parent[OG_MAXV];    /* BFS parent of order[i] (i>0) */
+} og_pat;
+
+static int pat_init(og_pat *p, uint32_t nv, uint32_t ne, const uint32_t *edges, const uint32_t *plabels) {
+  if (nv < 1 || nv > OG_MAXV) return OG_EINVAL;
+  memset(p, 0, sizeof(*p));
+  p->nv = nv;
+  for (uint32_t e = 0; e < ne; e++) {
+    uint32_t a = edges[2 * e], b = edges[2 * e + 1];
+    if (a >= nv || b >= nv || a == b) return OG_EINVAL;
+    p->adjm[a][b] = p->adjm[b][a] = 1;
+  }
+  p->labeled = plabels != NULL;
+  for (uint32_t i = 0; i < nv; i++) p->plab[i] = plabels ? plabels[i] : 0;
+  /* BFS from vertex 0 */
+  int seen[OG_MAXV] = {0};
+  uint32_t head = 0, tail = 0;
+  p->order[tail++] = 0; seen[0] = 1;
+  while (head < tail) {
+    uint32_t x = p->order[head++];
+    for (uint32_t y = 0; y < nv; y++)
+      if (p->adjm[x][y] && !seen[y]) { seen[y] = 1; p->parent[tail] = x; p->order[tail++] = y; }
+  }
+  if (tail != nv) return OG_EINVAL;   /* disconnected */
+  return OG_OK;
+}
+
+/* |Aut_L(P)| by brute force over all nv! permutations (Heap's algorithm). */
+static uint64_t pat_aut(const og_pat *p) {
+  uint32_t nv = p->nv, perm[OG_MAXV], c[OG_MAXV];
+  for (uint32_t i = 0; i < nv; i++) { perm[i] = i; c[i] = 0; }
+  uint64_t count = 0;
+  for (;;) {
+    int ok = 1;
+    for (uint32_t i = 0; i < nv && ok; i++) {
+      if (p->plab[perm[i]] != p->plab[i]) ok = 0;
+      for (uint32_t j = 0; j < nv && ok; j++)
+        if (p->adjm[perm[i]][perm[j]] != p->adjm[i][j]) ok = 0;
+    }
+    count += ok;
+    /* next permutation (Heap) */
+    uint32_t i = 1;
+    while (i < nv && c[i] >= i) { c[i] = 0; i++; }
+    if (i >= nv) break;
+    uint32_t j = (i % 2) ? c[i] : 0;
+    uint32_t t = perm[j]; perm[j] = perm[i]; perm[i] = t;
+    c[i]++;
+  }
+  return count;
+}
+
+static uint64_t match_rec(const og_graph *g, const og_pat *p, uint32_t pos, uint32_t *phi) {
+  if (pos == p->nv) return 1;
+  uint32_t q = p->order[pos], par = p->parent[pos];
+  uint32_t base = phi[par];
+  uint64_t total = 0;
+  for (uint64_t e = g->off[base]; e < g->off[base + 1]; e++) {
+    uint32_t x = g->adj[e];
+    if (p->labeled && g->lab[x] != p->plab[q]) continue;
+    int ok = 1;
+    for (uint32_t i = 0; i < pos && ok; i++) if (phi[p->order[i]] == x) ok = 0;   /* injective */
+    for (uint32_t i = 0; i < pos && ok; i++) {
+      uint32_t b = p->order[i];
+      if (b != par && p->adjm[q][b] && !adjacent(g, phi[b], x)) ok = 0;           /* backward edges */
+    }
+    if (!ok) continue;
+    phi[q] = x;
+    total += match_rec(g, p, pos + 1, phi);
+  }
+  return total;
+}
+
+int og_match(const og_graph *g, uint32_t nv, uint32_t ne, const uint32_t *edges,
+             const uint32_t *plabels, int threads, uint64_t *count, uint64_t *mappings,
+             uint64_t *aut) {
+  og_pat p;
+  int st = pat_init(&p, nv, ne, edges, plabels);
+  if (st) return st;
+  set_threads(threads);
+  uint64_t total = 0;
+  uint32_t r = p.order[0];
+#pragma omp parallel for schedule(dynamic, 64) reduction(+ : total)
+  for (int64_t v = 0; v < (int64_t)g->n; v++) {
+    if (p.labeled && g->lab[v] != p.plab[r]) continue;
+    uint32_t phi[OG_MAXV];
+    phi[r] = (uint32_t)v;
+    total += match_rec(g, &p, 1, phi);
+  }
+  uint64_t a = pat_aut(&p);
+  if (aut) *aut = a;
+  if (mappings) *mappings = total;
+  if (total % a) return OG_ENOTDIV;
+  if (count) *count = total / a;
+  return OG_OK;
+}
+
+/* ---------------------------------------------------------------------------
+ * O-3: frequent pattern mining, edge-induced patterns of 1..l edges (l <= 3),
+ * MNI support.
+ *
+ * Canonical code of a connected edge set S with vertex set W (|W| = nv <= 4):
+ *   min over bijections pi : {0..nv-1} -> W  of
+ *     ( lab(pi(0)), ..., lab(pi(nv-1)),  sorted list of pairs (i<j) with {pi(i),pi(j)} in S )
+ *   compared lexicographically (labels first, then the sorted edge-pair list).
+ * Domain of canonical position i: union over every minimizing pi of {pi(i)}.
+ * sup(P) = min_i |domain(P, i)|  (MNI).  Output: every P with sup >= minsup.
+ * ------------------------------------------------------------------------- */
+#define FPM_MAXNV 4
+#define FPM_MAXE 3
+
+typedef struct {
+  uint32_t nv, ne;
+  uint32_t lab[FPM_MAXNV];
+  uint32_t e[FPM_MAXE][2];
+} og_code;
+
+static int code_cmp(const og_code *x, const og_code *y) {
+  if (x->nv != y->nv) return x->nv < y->nv ? -1 : 1;
+  for (uint32_t i = 0; i < x->nv; i++)
+    if (x->lab[i] != y->lab[i]) return x->lab[i] < y->lab[i] ? -1 : 1;
+  if (x->ne != y->ne) return x->ne < y->ne ? -1 : 1;
+  for (uint32_t i = 0; i < x->ne; i++) {
+    if (x->e[i][0] != y->e[i][0]) return x->e[i][0] < y->e[i][0] ? -1 : 1;
+    if (x->e[i][1] != y->e[i][1]) return x->e[i][1] < y->e[i][1] ? -1 : 1;
+  }
+  return 0;
+}
+
+/* Hash table of patterns -> domain bitsets (nv * ceil(n/64) words each). */
+typedef struct {
+  uint64_t cap;          /* slots, power of two */
+  og_code *key;
+  int *used;             /* 0 empty, 1 being written, 2 ready */
+  uint64_t **dom;        /* dom[slot] = FPM_MAXNV bitsets of `words` words */
+  uint64_t *inst;        /* inst[slot] = number of edge sets mapped to the pattern */
+  uint64_t words;
+  omp_lock_t lock;
+  int overflow;
+} og_ptab;
+
+static uint64_t code_hash(const og_code *c) {
+  uint64_t h = 1469598103934665603ull;
+  const uint32_t *w = (const uint32_t *)c;
+  for (size_t i = 0; i < sizeof(og_code) / 4; i++) { h ^= w[i]; h *= 1099511628211ull; }
+  return h;
+}
+
+static int64_t ptab_get(og_ptab *t, const og_code *c) {
+  uint64_t h = code_hash(c) & (t->cap - 1);
+  for (uint64_t probe = 0; probe < t->cap; probe++, h = (h + 1) & (t->cap - 1)) {
+    int u = __atomic_load_n(&t->used[h], __ATOMIC_ACQUIRE);
+    if (u == 2) { if (code_cmp(&t->key[h], c) == 0) return (int64_t)h; continue; }
+    /* empty or in flight: take the lock and re-check */
+    omp_set_lock(&t->lock);
+    u = t->used[h];
+    if (u == 2) {
+      omp_unset_lock(&t->lock);
+      if (code_cmp(&t->key[h], c) == 0) return (int64_t)h;
+      continue;
+    }
+    t->key[h] = *c;
+    t->dom[h] = (uint64_t *)calloc(FPM_MAXNV * t->words, sizeof(uint64_t));
+    __atomic_store_n(&t->used[h], 2, __ATOMIC_RELEASE);
+    omp_unset_lock(&t->lock);
+    return (int64_t)h;
+  }
+  t->overflow = 1;
+  return -1;
+}
+
+/* Canonicalise the edge set {ed[0..ne-1]} on vertex set W (nv vertices) and
+ * OR every minimizing assignment into the pattern's domains. */
+static void fpm_record(const og_graph *g, og_ptab *t, uint32_t nv, const uint32_t *W, uint32_t ne,
+                       const uint32_t (*ed)[2]) {
+  static const uint8_t perms4[24][4] = {
+      {0,1,2,3},{0,1,3,2},{0,2,1,3},{0,2,3,1},{0,3,1,2},{0,3,2,1},{1,0,2,3},{1,0,3,2},
+      {1,2,0,3},{1,2,3,0},{1,3,0,2},{1,3,2,0},{2,0,1,3},{2,0,3,1},{2,1,0,3},{2,1,3,0},
+      {2,3,0,1},{2,3,1,0},{3,0,1,2},{3,0,2,1},{3,1,0,2},{3,1,2,0},{3,2,0,1},{3,2,1,0}};
+  og_code best; int have = 0;
+  uint32_t bestpi[24][FPM_MAXNV]; int nbest = 0;
+  for (int pi = 0; pi < 24; pi++) {
+    const uint8_t *P = perms4[pi];
+    int valid = 1;   /* permutation of the first nv symbols only */
+    for (uint32_t i = 0; i < nv; i++) if (P[i] >= nv) valid = 0;
+    if (!valid) continue;
+    /* position i holds data vertex W[P[i]] */
+    og_code c; memset(&c, 0, sizeof(c));
+    c.nv = nv; c.ne = ne;
+    uint32_t pos_of[FPM_MAXNV];
+    for (uint32_t i = 0; i < nv; i++) { c.lab[i] = g->lab[W[P[i]]]; pos_of[P[i]] = i; }
+    for (uint32_t e = 0; e < ne; e++) {
+      uint32_t a = 0, b = 0;
+      for (uint32_t w = 0; w < nv; w++) { if (W[w] == ed[e][0]) a = pos_of[w]; if (W[w] == ed[e][1]) b = pos_of[w]; }
+      c.e[e][0] = a < b ? a : b; c.e[e][1] = a < b ? b : a;
+    }
+    /* sort the edge pairs (insertion sort, ne <= 3) */
+    for (uint32_t i = 1; i < ne; i++)
+      for (uint32_t j = i; j > 0; j--) {
+        uint32_t *x = c.e[j - 1], *y = c.e[j];
+        if (x[0] > y[0] || (x[0] == y[0] && x[1] > y[1])) {
+          uint32_t t0 = x[0], t1 = x[1]; x[0] = y[0]; x[1] = y[1]; y[0] = t0; y[1] = t1;
+        }
+      }
+    int cmp = have ? code_cmp(&c, &best) : -1;
+    if (cmp < 0) { best = c; have = 1; nbest = 0; }
+    if (cmp <= 0) {
+      for (uint32_t i = 0; i < nv; i++) bestpi[nbest][i] = W[P[i]];
+      nbest++;
+    }
+  }
+  int64_t slot = ptab_get(t, &best);
+  if (slot < 0) return;
+  uint64_t *dom = t->dom[slot];
+  __atomic_fetch_add(&t->inst[slot], 1, __ATOMIC_RELAXED);
+  for (int b = 0; b < nbest; b++)
+    for (uint32_t i = 0; i < nv; i++) {
+      uint32_t v = bestpi[b][i];
+      __atomic_fetch_or(&dom[i * t->words + v / 64], 1ull << (v % 64), __ATOMIC_RELAXED);
+    }
+}
+
+/* Shape-by-shape enumeration of every connected edge set with 1..l edges, each
+ * exactly once:
+ *   1 edge:   {u,v}, u<v
+ *   2 edges:  wedge, centre c with an unordered neighbour pair {a,b}
+ *   3 edges:  triangle u<v<w; 3-star, centre c with a neighbour triple a<b<d;
+ *             3-path a-b-c-d keyed by its middle edge {b,c} (b<c), a in N(b)-{c},
+ *             d in N(c)-{b}, a != d. */
+static void fpm_enum_shapes(const og_graph *g, og_ptab *t, uint32_t l) {
+#pragma omp parallel for schedule(dynamic, 64)
+  for (int64_t vv = 0; vv < (int64_t)g->n; vv++) {
+    uint32_t v = (uint32_t)vv;
+    uint64_t s = g->off[v], e = g->off[v + 1];
+    for (uint64_t i = s; i < e; i++) {
+      uint32_t u = g->adj[i];
+      if (u > v) {   /* edge {v,u} */
+        uint32_t W[2] = {v, u}; uint32_t ed[1][2] = {{v, u}};
+        fpm_record(g, t, 2, W, 1, ed);
+      }
+    }
+    if (l >= 2)
+      for (uint64_t i = s; i < e; i++)
+        for (uint64_t j = i + 1; j < e; j++) {   /* wedge a-v-b */
+          uint32_t a = g->adj[i], b = g->adj[j];
+          uint32_t W[3] = {v, a, b}; uint32_t ed[2][2] = {{v, a}, {v, b}};
+          fpm_record(g, t, 3, W, 2, ed);
+        }
+    if (l >= 3) {
+      for (uint64_t i = s; i < e; i++)
+        for (uint64_t j = i + 1; j < e; j++)
+          for (uint64_t q = j + 1; q < e; q++) {   /* 3-star */
+            uint32_t a = g->adj[i], b = g->adj[j], d = g->adj[q];
+            uint32_t W[4] = {v, a, b, d}; uint32_t ed[3][2] = {{v, a}, {v, b}, {v, d}};
+            fpm_record(g, t, 4, W, 3, ed);
+          }
+      for (uint64_t i = s; i < e; i++) {
+        uint32_t u = g->adj[i];
+        if (u <= v) continue;
+        for (uint64_t j = i + 1; j < e; j++) {   /* triangle v<u<w */
+          uint32_t w = g->adj[j];
+          if (adjacent(g, u, w)) {
+            uint32_t W[3] = {v, u, w}; uint32_t ed[3][2] = {{v, u}, {v, w}, {u, w}};
+            fpm_record(g, t, 3, W, 3, ed);
+          }
+        }
+        /* 3-paths with middle edge {v,u}, v<u: a-v-u-d */
+        for (uint64_t x = s; x < e; x++) {
+          uint32_t a = g->adj[x];
+          if (a == u) continue;
+          for (uint64_t y = g->off[u]; y < g->off[u + 1]; y++) {
+            uint32_t d = g->adj[y];
+            if (d == v || d == a) continue;
+            uint32_t W[4] = {a, v, u, d}; uint32_t ed[3][2] = {{a, v}, {v, u}, {u, d}};
+            fpm_record(g, t, 4, W, 3, ed);
+          }
+        }
+      }
+    }
+  }
+}
+
+/* Brute-force enumeration (tiny graphs only): every set of 1..l distinct edges
+ * whose edge set is connected, taken by its minimum edge id e1 < e2 < e3.  Edges
+ * are ids into the list of undirected edges (u<v) in CSR order. */
+static int edges_connected(uint32_t ne, const uint32_t (*ed)[2]) {
+  uint32_t comp[FPM_MAXE]; for (uint32_t i = 0; i < ne; i++) comp[i] = i;
+  for (int it = 0; it < 3; it++)
+    for (uint32_t i = 0; i < ne; i++)
+      for (uint32_t j = 0; j < ne; j++)
+        if (ed[i][0] == ed[j][0] || ed[i][0] == ed[j][1] || ed[i][1] == ed[j][0] || ed[i][1] == ed[j][1]) {
+          uint32_t c = comp[i] < comp[j] ? comp[i] : comp[j]; comp[i] = comp[j] = c;
+        }
+  for (uint32_t i = 0; i < ne; i++) if (comp[i] != 0) return 0;
+  return 1;
+}
+
+static void fpm_enum_brute(const og_graph *g, og_ptab *t, uint32_t l) {
+  uint64_t m = g->m, k = 0;
+  uint32_t (*E)[2] = (uint32_t (*)[2])malloc((m ? m : 1) * sizeof(*E));
+  for (uint32_t v = 0; v < g->n; v++)
+    for (uint64_t i = g->off[v]; i < g->off[v + 1]; i++)
+      if (g->adj[i] > v) { E[k][0] = v; E[k][1] = g->adj[i]; k++; }
+#pragma omp parallel for schedule(dynamic, 1)
+  for (int64_t a = 0; a < (int64_t)m; a++) {
+    for (uint64_t b = (uint64_t)a; b < (l >= 2 ? m : (uint64_t)a + 1); b++) {
+      for (uint64_t c = b; c < (l >= 3 ? m : b + 1); c++) {
+        uint64_t ids[3] = {(uint64_t)a, b, c};
+        uint32_t ne = 1 + (b > (uint64_t)a) + (c > b);
+        if ((b == (uint64_t)a && c != b)) continue;   /* only a<b<c or prefixes */
+        uint32_t ed[3][2]; uint32_t q = 0;
+        ed[q][0] = E[ids[0]][0]; ed[q][1] = E[ids[0]][1]; q++;
+        if (b > (uint64_t)a) { ed[q][0] = E[b][0]; ed[q][1] = E[b][1]; q++; }
+        if (c > b) { ed[q][0] = E[c][0]; ed[q][1] = E[c][1]; q++; }
+        if (!edges_connected(ne, (const uint32_t (*)[2])ed)) continue;
+        uint32_t W[4], nv = 0;
+        for (uint32_t e = 0; e < ne; e++)
+          for (int s = 0; s < 2; s++) {
+            uint32_t x = ed[e][s]; int f = 0;
+            for (uint32_t w = 0; w < nv; w++) if (W[w] == x) f = 1;
+            if (!f) W[nv++] = x;
+          }
+        if (nv > FPM_MAXNV) continue;
+        fpm_record(g, t, nv, W, ne, (const uint32_t (*)[2])ed);
+      }
+    }
+  }
+  free(E);
+}
+
+/* Result record layout (uint64 x 14):
+ *   [0]=ne [1]=nv [2..5]=labels [6..11]=edge pairs (a0,b0,a1,b1,a2,b2) [12]=support
+ *   [13]=number of edge sets (instances) mapped to the pattern. */
+#define OG_REC 14
+
+typedef struct { og_code c; uint64_t sup; uint64_t inst; } og_fres;
+
+static int fres_cmp(const void *a, const void *b) {
+  const og_fres *x = (const og_fres *)a, *y = (const og_fres *)b;
+  if (x->c.ne != y->c.ne) return x->c.ne < y->c.ne ? -1 : 1;
+  return code_cmp(&x->c, &y->c);
+}
+
+/* Run FPM.  method 0: shape enumeration, 1: brute-force edge subsets.
+ * Writes up to max_out records into out; returns the number of frequent patterns
+ * (which may exceed max_out), or <0 on error. */
+int64_t og_fpm(const og_graph *g, uint32_t l, uint64_t minsup, int method, int threads,
+               uint64_t max_out, uint64_t *out, uint64_t pattern_cap) {
+  if (l < 1 || l > FPM_MAXE || minsup < 1) return OG_EINVAL;
+  set_threads(threads);
+  og_ptab t; memset(&t, 0, sizeof(t));
+  t.cap = 1; while (t.cap < (pattern_cap ? pattern_cap : (1u << 16))) t.cap <<= 1;
+  t.key = (og_code *)calloc(t.cap, sizeof(og_code));
+  t.used = (int *)calloc(t.cap, sizeof(int));
+  t.dom = (uint64_t **)calloc(t.cap, sizeof(uint64_t *));
+  t.inst = (uint64_t *)calloc(t.cap, sizeof(uint64_t));
+  t.words = ((uint64_t)g->n + 63) / 64;
+  omp_init_lock(&t.lock);
+  if (method == 0) fpm_enum_shapes(g, &t, l); else fpm_enum_brute(g, &t, l);
+  int64_t nres = 0;
+  og_fres *res = (og_fres *)malloc(t.cap * sizeof(og_fres));
+  for (uint64_t h = 0; h < t.cap; h++) {
+    if (t.used[h] != 2) continue;
+    og_fres r; memset(&r, 0, sizeof(r)); r.c = t.key[h];
+    uint64_t sup = UINT64_MAX;
+    for (uint32_t i = 0; i < r.c.nv; i++) {
+      uint64_t cnt = 0;
+      for (uint64_t w = 0; w < t.words; w++) cnt += (uint64_t)__builtin_popcountll(t.dom[h][i * t.words + w]);
+      if (cnt < sup) sup = cnt;
+    }
+    r.sup = sup;
+    r.inst = t.inst[h];
+    if (sup >= minsup) res[nres++] = r;
+    free(t.dom[h]);
+  }
+  qsort(res, (size_t)nres, sizeof(og_fres), fres_cmp);
+  for (int64_t i = 0; i < nres && (uint64_t)i < max_out; i++) {
+    uint64_t *o = out + i * OG_REC;
+    memset(o, 0, OG_REC * sizeof(uint64_t));
+    o[0] = res[i].c.ne; o[1] = res[i].c.nv;
+    for (int j = 0; j < FPM_MAXNV; j++) o[2 + j] = j < (int)res[i].c.nv ? res[i].c.lab[j] : 0;
+    for (uint32_t e = 0; e < res[i].c.ne; e++) { o[6 + 2 * e] = res[i].c.e[e][0]; o[7 + 2 * e] = res[i].c.e[e][1]; }
+    o[12] = res[i].sup;
+    o[13] = res[i].inst;
+  }
+  int ovf = t.overflow;
+  free(res); free(t.key); free(t.used); free(t.dom); free(t.inst);
+  omp_destroy_lock(&t.lock);
+  return ovf ? OG_ENOMEM : nres;
+}
+
+/* MNI support of ONE labeled pattern, by subgraph-matching enumeration (O-2's
+ * enumerator, without symmetry breaking): domain(i) = {phi(i)} over all mappings.
+ * Used for sampled FPM parity at full size and as an independent pin of og_fpm. */
+int og_pattern_mni(const og_graph *g, uint32_t nv, uint32_t ne, const uint32_t *edges,
+                   const uint32_t *plabels, int threads, uint64_t *support) {
+  og_pat p;
+  int st = pat_init(&p, nv, ne, edges, plabels);
+  if (st) return st;
+  set_threads(threads);
+  uint64_t words = ((uint64_t)g->n + 63) / 64;
+  uint64_t *dom = (uint64_t *)calloc(nv * words, sizeof(uint64_t));
+  uint32_t r = p.order[0];
+#pragma omp parallel for schedule(dynamic, 64)
+  for (int64_t v = 0; v < (int64_t)g->n; v++) {
+    if (p.labeled && g->lab[v] != p.plab[r]) continue;
+    /* explicit DFS stack over match_rec's recursion so every mapping is visited */
+    uint32_t phi[OG_MAXV]; uint64_t it[OG_MAXV];
+    phi[r] = (uint32_t)v;
+    uint32_t pos = 1;
+    if (p.nv == 1) { __atomic_fetch_or(&dom[r * words + v / 64], 1ull << (v % 64), __ATOMIC_RELAXED); continue; }
+    it[1] = g->off[phi[p.parent[1]]];
+    while (pos >= 1) {
+      uint32_t q = p.order[pos], par = p.parent[pos], base = phi[par];
+      int advanced = 0;
+      while (it[pos] < g->off[base + 1]) {
+        uint32_t x = g->adj[it[pos]++];
+        if (p.labeled && g->lab[x] != p.plab[q]) continue;
+        int ok = 1;
+        for (uint32_t i = 0; i < pos && ok; i++) if (phi[p.order[i]] == x) ok = 0;
+        for (uint32_t i = 0; i < pos && ok; i++) {
+          uint32_t b = p.order[i];
+          if (b != par && p.adjm[q][b] && !adjacent(g, phi[b], x)) ok = 0;
+        }
+        if (!ok) continue;
+        phi[q] = x;
+        if (pos + 1 == p.nv) {
+          for (uint32_t i = 0; i < p.nv; i++)
+            __atomic_fetch_or(&dom[i * words + phi[i] / 64], 1ull << (phi[i] % 64), __ATOMIC_RELAXED);
+          continue;
+        }
+        advanced = 1;
+        break;
+      }
+      if (advanced) { pos++; it[pos] = g->off[phi[p.parent[pos]]]; }
+      else pos--;
+    }
+  }
+  uint64_t sup = UINT64_MAX;
+  for (uint32_t i = 0; i < nv; i++) {
+    uint64_t c = 0;
+    for (uint64_t w = 0; w < words; w++) c += (uint64_t)__builtin_popcountll(dom[i * words + w]);
+    if (c < sup) sup = c;
+  }
+  free(dom);
+  *support = sup;
+  return OG_OK;
+}

@@ -1,0 +1,121 @@
+"""Pins of oracle O-0 (graph normalisation) and O-1 (k-clique counting).
+
+Each pin is fixed by mathematics, not by the oracle: closed forms (K_n, Turan,
+wheels, cycles, grids, Petersen), brute force over all k-subsets, additivity over
+disjoint unions and independence of the orientation order.  (PAPER.md L15, L269,
+L449 name kCL; the count is the plain definition -- DESIGN.md reading R9.)
+"""
+from math import comb
+
+import numpy as np
+import pytest
+
+import gamma_gen as gg
+import brute
+
+
+def G(oracle_mod, g, labels=None):
+    n, (s, d) = g
+    return oracle_mod.Graph(n, s, d, labels)
+
+
+def test_normalisation_matches_set_definition(oracle_mod):
+    src = np.array([0, 1, 1, 2, 2, 3, 3, 4, 0, 5], np.uint32)
+    dst = np.array([1, 0, 1, 3, 3, 2, 4, 4, 5, 0], np.uint32)
+    g = oracle_mod.Graph(6, src, dst)
+    E = brute.normalise(src, dst)
+    assert g.m == len(E)
+    off, adj = g.csr()
+    got = set()
+    for v in range(6):
+        lst = adj[off[v]:off[v + 1]].tolist()
+        assert lst == sorted(set(lst)), "sorted, no duplicates"
+        assert v not in lst, "no self-loops"
+        got |= {frozenset((v, u)) for u in lst}
+    assert got == E
+    # symmetric
+    for v in range(6):
+        for u in adj[off[v]:off[v + 1]]:
+            assert v in adj[off[u]:off[u + 1]]
+
+
+@pytest.mark.parametrize("n", range(1, 11))
+def test_complete_graph(oracle_mod, n):
+    g = G(oracle_mod, gg.complete(n))
+    for k in range(1, n + 2):
+        assert g.kclique(k) == comb(n, k)
+
+
+@pytest.mark.parametrize("n,r", [(6, 2), (6, 3), (8, 4), (9, 3), (12, 4), (10, 5)])
+def test_turan(oracle_mod, n, r):
+    g = G(oracle_mod, gg.turan(n, r))
+    for k in range(2, r + 2):
+        assert g.kclique(k) == comb(r, k) * (n // r) ** k
+
+
+@pytest.mark.parametrize("n", [4, 5, 6, 9, 20])
+def test_wheel(oracle_mod, n):
+    g = G(oracle_mod, gg.wheel(n))
+    assert g.kclique(3) == n
+    assert g.kclique(4) == 0
+
+
+def test_triangle_free(oracle_mod):
+    assert G(oracle_mod, gg.cycle(3)).kclique(3) == 1
+    for n in (4, 5, 7, 30):
+        assert G(oracle_mod, gg.cycle(n)).kclique(3) == 0
+    assert G(oracle_mod, gg.grid(5, 7)).kclique(3) == 0
+    assert G(oracle_mod, gg.petersen()).kclique(3) == 0
+    assert G(oracle_mod, gg.complete_bipartite(4, 5)).kclique(3) == 0
+
+
+def test_k1_k2(oracle_mod):
+    n = 50
+    s, d = gg.er(n, 200, 3)
+    g = oracle_mod.Graph(n, s, d)
+    assert g.kclique(1) == 50
+    assert g.kclique(2) == len(brute.normalise(s, d))
+
+
+def test_empty(oracle_mod):
+    g = oracle_mod.Graph(5, np.zeros(0, np.uint32), np.zeros(0, np.uint32))
+    assert g.m == 0 and g.kclique(3) == 0 and g.kclique(1) == 5
+
+
+@pytest.mark.parametrize("seed", [1, 2, 3, 4, 5])
+def test_brute_force_random(oracle_mod, seed):
+    n = 14
+    s, d = gg.er(n, 60, seed)
+    E = brute.normalise(s, d)
+    g = oracle_mod.Graph(n, s, d)
+    for k in range(3, 7):
+        assert g.kclique(k) == brute.kcliques(n, E, k)
+
+
+def test_additivity_disjoint_union(oracle_mod):
+    parts = [gg.complete(6), gg.wheel(7), gg.turan(8, 4)]
+    u = G(oracle_mod, gg.disjoint_union(*parts))
+    for k in (3, 4):
+        assert u.kclique(k) == sum(G(oracle_mod, p).kclique(k) for p in parts)
+
+
+@pytest.mark.parametrize("seed", [1, 2])
+def test_order_independence_rmat(oracle_mod, seed):
+    s, d = gg.rmat(10, 12000, 0.57, 0.19, 0.19, seed)
+    g = oracle_mod.Graph(1 << 10, s, d)
+    for k in (3, 4, 5):
+        assert g.kclique(k, "degree") == g.kclique(k, "id")
+
+
+def test_roots_partition_total(oracle_mod):
+    s, d = gg.rmat(9, 5000, 0.57, 0.19, 0.19, 7)
+    g = oracle_mod.Graph(1 << 9, s, d)
+    roots = np.arange(1 << 9, dtype=np.uint32)
+    for k in (3, 4):
+        assert int(g.kclique_roots(k, roots).sum()) == g.kclique(k)
+
+
+def test_threads_invariance(oracle_mod):
+    n, s, d, _ = gg.config_graph("c1", scale=10)
+    g = oracle_mod.Graph(n, s, d)
+    assert g.kclique(4, threads=1) == g.kclique(4, threads=0)

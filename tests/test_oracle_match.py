@@ -1,0 +1,120 @@
+"""Pins of oracle O-2 (labeled, non-induced subgraph matching; Alg. 1
+L174-182; readings R4-R6, R10).
+
+Closed forms on K_n, K_{a,b}, grids, wheels, Petersen, C_4; |Aut_L| against brute
+force; the label-sum identity; brute force over edge subsets on tiny graphs.
+"""
+from math import comb
+
+import numpy as np
+import pytest
+
+import gamma_gen as gg
+import brute
+
+Q = gg.QUERIES
+
+
+def G(oracle_mod, g, labels=None):
+    n, (s, d) = g
+    return oracle_mod.Graph(n, s, d, labels)
+
+
+def count(g, name, plab=None):
+    nv, e = Q[name]
+    return g.match(nv, e, plab)[0]
+
+
+@pytest.mark.parametrize("n", [4, 5, 6, 8])
+def test_complete(oracle_mod, n):
+    g = G(oracle_mod, gg.complete(n))
+    assert count(g, "c4") == 3 * comb(n, 4)
+    assert count(g, "diamond") == 6 * comb(n, 4)
+    assert count(g, "tailed_triangle") == 12 * comb(n, 4)
+    assert count(g, "house") == 60 * comb(n, 5)
+
+
+@pytest.mark.parametrize("a,b", [(2, 2), (3, 4), (5, 3)])
+def test_complete_bipartite(oracle_mod, a, b):
+    g = G(oracle_mod, gg.complete_bipartite(a, b))
+    assert count(g, "c4") == comb(a, 2) * comb(b, 2)
+    for q in ("diamond", "tailed_triangle", "house"):
+        assert count(g, q) == 0
+
+
+@pytest.mark.parametrize("a,b", [(2, 2), (3, 5), (6, 4)])
+def test_grid(oracle_mod, a, b):
+    g = G(oracle_mod, gg.grid(a, b))
+    assert count(g, "c4") == (a - 1) * (b - 1)
+    for q in ("diamond", "tailed_triangle", "house"):
+        assert count(g, q) == 0
+
+
+@pytest.mark.parametrize("n", [5, 6, 9])
+def test_wheel(oracle_mod, n):
+    g = G(oracle_mod, gg.wheel(n))
+    assert count(g, "c4") == n
+    assert count(g, "diamond") == n
+    assert count(g, "tailed_triangle") == n * n
+    assert count(g, "house") == 2 * n
+
+
+def test_petersen_c4(oracle_mod):
+    assert count(G(oracle_mod, gg.petersen()), "c4") == 0
+    assert count(G(oracle_mod, gg.cycle(4)), "c4") == 1
+
+
+def test_aut():
+    assert [brute.aut(*Q[q]) for q in ("c4", "diamond", "tailed_triangle", "house")] == [8, 4, 2, 2]
+    assert brute.aut(*Q["c4"], plab=[0, 1, 0, 1]) == 4
+
+
+def test_oracle_aut_and_mappings(oracle_mod):
+    g = G(oracle_mod, gg.complete(6))
+    for q, a in (("c4", 8), ("diamond", 4), ("tailed_triangle", 2), ("house", 2)):
+        nv, e = Q[q]
+        c, mp, aut = g.match(nv, e)
+        assert aut == a and mp == c * a
+    nv, e = Q["c4"]
+    assert g.match(nv, e, [0, 1, 0, 1])[2] == 4
+
+
+def test_single_vertex_pattern(oracle_mod):
+    lab = np.array([0, 1, 1, 2, 1], np.uint32)
+    g = G(oracle_mod, gg.path(5), lab)
+    assert g.match(1, [], [1])[0] == 3
+    assert g.match(1, [])[0] == 5
+
+
+@pytest.mark.parametrize("q", ["c4", "diamond", "tailed_triangle", "house"])
+def test_label_sum_identity(oracle_mod, q):
+    import itertools
+    nv, e = Q[q]
+    n = 12
+    s, d = gg.er(n, 40, 11)
+    lab = gg.labels(n, 2, 5)
+    g = oracle_mod.Graph(n, s, d, lab)
+    total = sum(g.match(nv, e, list(pl))[1] for pl in itertools.product(range(2), repeat=nv))
+    g0 = oracle_mod.Graph(n, s, d)
+    assert total == g0.match(nv, e)[1]
+
+
+@pytest.mark.parametrize("seed", [1, 2, 3])
+@pytest.mark.parametrize("q", ["c4", "diamond", "tailed_triangle", "house"])
+def test_brute_force_subsets(oracle_mod, seed, q):
+    nv, e = Q[q]
+    n = 9
+    s, d = gg.er(n, 22, seed)
+    E = brute.normalise(s, d)
+    lab = gg.labels(n, 2, seed).tolist()
+    g = oracle_mod.Graph(n, s, d, np.array(lab, np.uint32))
+    assert g.match(nv, e)[0] == brute.distinct_subgraphs(n, E, nv, e)
+    plab = [i % 2 for i in range(nv)]
+    assert g.match(nv, e, plab)[0] == brute.distinct_subgraphs(n, E, nv, e, plab, lab)
+    assert g.match(nv, e, plab)[1] == brute.mappings(n, E, nv, e, plab, lab)
+
+
+def test_disconnected_pattern_rejected(oracle_mod):
+    g = G(oracle_mod, gg.complete(5))
+    with pytest.raises(ValueError):
+        g.match(4, [(0, 1), (2, 3)])
