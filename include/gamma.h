@@ -1,0 +1,194 @@
+/*
+ * gamma.h -- C ABI of the B200-native GAMMA hot path (embedding-table extension).
+ *
+ * What the calls compute (PAPER.md = /root/reference/PAPER.md, line numbers):
+ *   gamma_kclique  k-clique counting, the kCL task of PAPER.md L15, L269, L449, run
+ *                  as vertex extension (Def. 3.1) with early pruning to
+ *                  common neighbours (L146) over a degree-ordered DAG.
+ *   gamma_match    subgraph matching, "all subgraphs of G_d isomorphic to a pattern
+ *                  P" (L112), by worst-case-optimal-join vertex extension + filtering
+ *                  (Alg. 1).  Non-induced, labeled, counted as distinct
+ *                  subgraphs (readings R4-R6).
+ *   gamma_fpm      frequent pattern mining, "all patterns P whose support is at least a
+ *                  given threshold" (L113, L144), by edge extension + aggregation +
+ *                  filtering (Alg. 2), edge-induced, MNI support (R1-R3).
+ *   gamma_load_*   the CSR graph_data G_d of Fig. 3 (L158) / §IV (L199): adjacency
+ *                  lists and vertex labels, built on the GPU from raw edge samples.
+ *
+ * Conventions (all entry points):
+ *   - Return GAMMA_OK (0) or a negative gamma_status; outputs are written only on
+ *     GAMMA_OK.  gamma_last_error() gives a thread-local message for the last
+ *     failure on the calling thread (valid until the next call on that thread).
+ *   - Input arrays are BORROWED for the duration of the call and may be host or
+ *     device pointers (classified with cudaPointerGetAttributes); they are copied.
+ *   - Handles and result objects are OWNED by the library and released with the
+ *     matching *_free / *_destroy call.  No C++ exception crosses this ABI.
+ *   - One gamma_ctx per thread / process.  All device work runs on ctx's stream.
+ *   - There is no CPU fallback: with no usable CUDA device every call that computes
+ *     returns GAMMA_E_CUDA.
+ *   - Vertex ids are uint32 in [0, n); counts are uint64.  A count that would wrap
+ *     uint64 returns GAMMA_E_OVERFLOW.
+ */
+#ifndef GAMMA_H_
+#define GAMMA_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define GAMMA_ABI_VERSION 1
+
+typedef int32_t gamma_status;
+enum {
+  GAMMA_OK = 0,
+  GAMMA_E_INVAL = -1,        /* bad argument, malformed graph or pattern            */
+  GAMMA_E_NOMEM = -2,        /* device allocation failed or HBM/spill budget too small */
+  GAMMA_E_CUDA = -3,         /* CUDA runtime / kernel error (incl. no device)        */
+  GAMMA_E_OVERFLOW = -4,     /* uint64 count overflow                                */
+  GAMMA_E_UNSUPPORTED = -5   /* valid request outside this version (k>32, induced=1) */
+};
+
+typedef struct gamma_ctx gamma_ctx;
+typedef struct gamma_graph gamma_graph;
+
+/* Context descriptor.  Zero-initialise, then set what you need. */
+typedef struct {
+  int32_t device;            /* CUDA device ordinal                                  */
+  int32_t rank, world;       /* root-chunk partition: this process handles share
+                                `rank` of `world` (world <= 1: everything)          */
+  void *stream;              /* cudaStream_t to run on; NULL: the ctx creates one    */
+  /* Optional device allocator (e.g. PyTorch's caching allocator).  NULL: the
+     library uses cudaMallocAsync / cudaFreeAsync on ctx's stream.                   */
+  void *(*dev_alloc)(size_t bytes, void *stream, void *user);
+  void (*dev_free)(void *ptr, void *user);
+  void *alloc_user;
+  /* Optional collective: in-place SUM of n uint64 values held in HOST memory across
+     all `world` ranks (e.g. torch.distributed all_reduce over NCCL).  NULL: results
+     of gamma_kclique / gamma_match are this rank's partial counts.                   */
+  gamma_status (*allreduce_sum_u64)(uint64_t *host_buf, size_t n, void *user);
+  void *coll_user;
+  uint64_t hbm_budget_bytes; /* cap on embedding-table bytes; 0: 80% of free HBM     */
+  uint64_t host_spill_bytes; /* pinned-host spill capacity for ET levels; 0: none    */
+  uint32_t flags;            /* GAMMA_FLAG_* below                                   */
+} gamma_ctx_desc;
+
+#define GAMMA_FLAG_TIME_KERNELS 0x1u   /* record per-launch CUDA-event times (stats) */
+#define GAMMA_FLAG_NO_FUSE      0x2u   /* materialise every ET level (no fused tail) */
+#define GAMMA_FLAG_SPILL        0x4u   /* BFS with host-resident levels
+                                          instead of the DFS-over-chunks policy      */
+#define GAMMA_FLAG_DEBUG_NOSTAGE 0x8u  /* test hook: never stage runs in shared memory
+                                          (exercises the hub / long-run code path)   */
+
+/* Create / destroy a context.  Errors: E_INVAL (NULL args), E_CUDA (no device). */
+gamma_status gamma_ctx_create(const gamma_ctx_desc *desc, gamma_ctx **out);
+void gamma_ctx_destroy(gamma_ctx *ctx);
+const char *gamma_last_error(void);
+int32_t gamma_abi_version(void);
+
+/* ---- Graph data G_d (A1) ------------------------------------------------------
+ * gamma_load_edges: build the graph from m raw samples (src[i], dst[i]) over n
+ * vertices: symmetrise, drop self-loops and duplicates, sort every adjacency list
+ * ascending (O-0), then orient each edge u->v iff
+ * (deg u, u) < (deg v, v) (the degree-ordered DAG used by kCL; R9).
+ * labels: n uint32 vertex labels or NULL (all 0).  src/dst/labels host or device.
+ * Errors: E_INVAL (vertex id >= n, n == 0), E_NOMEM, E_CUDA.                      */
+gamma_status gamma_load_edges(gamma_ctx *ctx, uint32_t n, const uint32_t *src,
+                              const uint32_t *dst, uint64_t m, const uint32_t *labels,
+                              gamma_graph **out);
+
+/* gamma_load_csr: adopt a symmetric CSR (row_ptr: n+1 uint64, col: row_ptr[n]
+ * uint32).  Validated on the device: every list strictly ascending, no self-loop,
+ * ids < n, and symmetric; else E_INVAL.  The DAG is derived as above.            */
+gamma_status gamma_load_csr(gamma_ctx *ctx, uint32_t n, const uint64_t *row_ptr,
+                            const uint32_t *col, const uint32_t *labels, gamma_graph **out);
+
+void gamma_graph_free(gamma_graph *g);
+
+typedef struct {
+  uint32_t n;
+  uint64_t m;                /* undirected edges                                     */
+  uint32_t max_degree, max_out_degree;
+  uint64_t device_bytes;     /* HBM held by the graph                                */
+  double build_ms;           /* device time of the last gamma_load_* (CUDA events)   */
+} gamma_graph_info;
+gamma_status gamma_graph_get_info(const gamma_graph *g, gamma_graph_info *info);
+
+/* Copy the symmetric CSR (row_ptr n+1, col 2m) or the DAG CSR (row_ptr n+1, col m)
+ * into caller buffers (host or device).  which: 0 symmetric, 1 DAG.               */
+gamma_status gamma_graph_copy_csr(const gamma_graph *g, int which, uint64_t *row_ptr,
+                                  uint32_t *col);
+
+/* ---- k-clique counting (A2-A8) ------------------------------------------------
+ * *count = number of vertex sets S, |S| = k, every pair adjacent.  k = 1 gives n,
+ * k = 2 gives m.  k > 32: E_UNSUPPORTED; k == 0: E_INVAL.  With world > 1 only
+ * this rank's roots are processed and the count is all-reduced if the ctx has a
+ * collective (else partial).                                                       */
+gamma_status gamma_kclique(gamma_graph *g, uint32_t k, uint64_t *count);
+
+/* Per-root counts: counts[i] = number of k-cliques whose lowest vertex under
+ * (deg, id) order is roots[i] (roots/counts host or device, nroots entries).  Used
+ * for sampled parity at full size; ignores rank/world.                            */
+gamma_status gamma_kclique_roots(gamma_graph *g, uint32_t k, uint64_t nroots,
+                                 const uint32_t *roots, uint64_t *counts);
+
+/* ---- Subgraph matching (Alg. 1) ----------------------------------------------- */
+typedef struct {
+  uint32_t nv, ne;           /* 1 <= nv <= 8, connected                              */
+  const uint32_t *edges;     /* 2*ne vertex ids (host memory)                        */
+  const uint32_t *labels;    /* nv labels or NULL (unlabeled: any vertex matches)    */
+  int32_t induced;           /* must be 0 in v1 (E_UNSUPPORTED otherwise)            */
+} gamma_pattern;
+
+/* *count = number of distinct subgraphs of G isomorphic to P (labels respected);
+ * mappings (nullable) = *count * |Aut_L(P)|.  Partitioned / reduced like kclique. */
+gamma_status gamma_match(gamma_graph *g, const gamma_pattern *p, uint64_t *count,
+                         uint64_t *mappings);
+
+/* ---- Frequent pattern mining (Alg. 2) ------------------------------------------ */
+typedef struct {
+  uint32_t nv, ne;
+  uint32_t labels[8];        /* labels in canonical vertex order                     */
+  uint8_t edges[8][2];       /* sorted (a<b) pairs in canonical positions            */
+  uint64_t support;          /* MNI support                                          */
+} gamma_fpm_pattern;
+
+typedef struct {
+  uint64_t n;
+  gamma_fpm_pattern *pats;   /* sorted by (ne, nv, labels, edges)                    */
+} gamma_fpm_result;
+
+/* All connected edge-induced patterns with 1..max_edges edges and MNI support >=
+ * minsup (max_edges in [1,3] in v1; minsup >= 1).  Result owned by the library.   */
+gamma_status gamma_fpm(gamma_graph *g, uint32_t max_edges, uint64_t minsup,
+                       gamma_fpm_result **out);
+void gamma_fpm_result_free(gamma_fpm_result *r);
+
+/* ---- Run statistics of the last gamma_kclique / gamma_match / gamma_fpm --------
+ * Per kernel class: launches, summed CUDA-event time (only with
+ * GAMMA_FLAG_TIME_KERNELS), algorithmic bytes (SURVEY.md §8(d) B_l; DESIGN.md
+ * "Algorithmic bytes"), and per-level embedding counts.                            */
+#define GAMMA_MAX_KERNEL_CLASSES 16
+#define GAMMA_MAX_LEVELS 34
+typedef struct {
+  uint32_t n_classes;
+  char name[GAMMA_MAX_KERNEL_CLASSES][32];
+  uint64_t launches[GAMMA_MAX_KERNEL_CLASSES];
+  double ms[GAMMA_MAX_KERNEL_CLASSES];
+  uint64_t alg_bytes[GAMMA_MAX_KERNEL_CLASSES];
+  uint64_t level_entries[GAMMA_MAX_LEVELS];  /* embeddings kept at each level       */
+  uint64_t list_elems;       /* adjacency elements the method fetches (sum |list|)   */
+  uint64_t chunks;           /* root chunks processed (after overflow splits)        */
+  uint64_t retries;          /* chunk splits caused by the HBM budget                */
+  uint64_t spilled_bytes;    /* bytes staged through pinned host memory              */
+  uint64_t total_launches;   /* every kernel this library launched in the call      */
+  double wall_ms;            /* host wall time of the call                           */
+} gamma_run_stats;
+gamma_status gamma_get_stats(const gamma_ctx *ctx, gamma_run_stats *out);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* GAMMA_H_ */

@@ -1,0 +1,258 @@
+"""B200-native GAMMA hot path: embedding-table extension for graph pattern mining.
+
+Thin Python binding over the C ABI in ``include/gamma.h`` (libgamma.so, built
+in-tree for sm_100a).  This module only marshals arguments: every step of the
+path (CSR build, extension, intersection, filtering, compaction, aggregation)
+runs in the library's CUDA kernels.  PyTorch supplies the device allocator, the
+stream and (for world > 1) the process group; there is no CPU fallback -- if the
+library or a CUDA device is missing, calls raise ``GammaError``/``ImportError``.
+
+The C names are re-exported 1:1 (``gamma_ctx_create``, ``gamma_load_edges``,
+``gamma_kclique``, ``gamma_match``, ``gamma_fpm`` ...) and wrapped by
+:class:`Context` / :class:`Graph`.
+"""
+from __future__ import annotations
+
+import ctypes as C
+from typing import Optional
+
+import numpy as np
+
+from . import _native as N
+
+_lib = N.load()
+
+# 1:1 C entry points
+for _name, _res, _args in N.SIGNATURES:
+    globals()[_name] = getattr(_lib, _name)
+
+__all__ = ["Context", "Graph", "GammaError", "library_path"] + [s[0] for s in N.SIGNATURES]
+
+
+def library_path() -> str:
+    return N.LIB_PATH
+
+
+class GammaError(RuntimeError):
+    def __init__(self, status: int, where: str):
+        msg = (_lib.gamma_last_error() or b"").decode(errors="replace")
+        super().__init__(f"{where}: status {status}: {msg}")
+        self.status = status
+
+
+def _check(st: int, where: str):
+    if st != N.GAMMA_OK:
+        raise GammaError(st, where)
+
+
+def _ptr(x, dtype):
+    """(pointer, keepalive, length) for a numpy array or torch tensor (host or CUDA)."""
+    if x is None:
+        return None, None, 0
+    try:
+        import torch
+        if isinstance(x, torch.Tensor):
+            want = {np.uint32: (torch.int32, torch.uint32), np.uint64: (torch.int64, torch.uint64)}[dtype]
+            assert x.dtype in want, f"expected {dtype.__name__}-compatible tensor, got {x.dtype}"
+            x = x.contiguous()
+            return x.data_ptr(), x, x.numel()
+    except ImportError:
+        pass
+    a = np.ascontiguousarray(x, dtype=dtype)
+    return a.ctypes.data, a, a.size
+
+
+class Context:
+    """A gamma_ctx bound to one CUDA device, its stream and allocator.
+
+    ``rank``/``world`` partition root chunks across processes; with a
+    ``torch.distributed`` process group initialised and ``world > 1`` the counts are
+    all-reduced (SUM) through it inside the C call (callback), else partial.
+    """
+
+    def __init__(self, device: int = 0, rank: Optional[int] = None, world: Optional[int] = None,
+                 use_torch: bool = True, hbm_budget_bytes: int = 0, host_spill_bytes: int = 0,
+                 time_kernels: bool = False, flags: int = 0, reduce: bool = True):
+        self._keep = []
+        d = N.gamma_ctx_desc()
+        d.device = device
+        self._torch = None
+        if use_torch:
+            import torch
+            self._torch = torch
+        dist_ok = False
+        if self._torch is not None:
+            import torch.distributed as dist
+            dist_ok = dist.is_available() and dist.is_initialized()
+            if rank is None and dist_ok:
+                rank, world = dist.get_rank(), dist.get_world_size()
+        d.rank = rank or 0
+        d.world = world or 1
+        if self._torch is not None and self._torch.cuda.is_available():
+            torch = self._torch
+            stream = torch.cuda.current_stream(device)
+            d.stream = C.c_void_p(stream.cuda_stream)
+            dev = device
+
+            def _alloc(size, strm, user):
+                try:
+                    return torch.cuda.caching_allocator_alloc(int(size), dev, int(strm or 0))
+                except Exception:   # noqa: BLE001 -- reported as E_NOMEM by the library
+                    return None
+
+            def _free(p, user):
+                torch.cuda.caching_allocator_delete(int(p))
+
+            fa, ff = N.ALLOC_FN(_alloc), N.FREE_FN(_free)
+            d.dev_alloc, d.dev_free = fa, ff
+            self._keep += [fa, ff]
+        if reduce and d.world > 1 and dist_ok:
+            import torch.distributed as dist
+            torch = self._torch
+            backend = dist.get_backend()
+
+            def _allreduce(buf, n, user):
+                try:
+                    vals = [buf[i] for i in range(n)]
+                    dev = torch.device("cuda", device) if backend == "nccl" else torch.device("cpu")
+                    t = torch.tensor(vals, dtype=torch.int64, device=dev)
+                    dist.all_reduce(t, op=dist.ReduceOp.SUM)
+                    for i, v in enumerate(t.cpu().tolist()):
+                        buf[i] = v
+                    return 0
+                except Exception:   # noqa: BLE001
+                    return N.GAMMA_E_CUDA
+
+            fr = N.ALLREDUCE_FN(_allreduce)
+            d.allreduce_sum_u64 = fr
+            self._keep.append(fr)
+        d.hbm_budget_bytes = hbm_budget_bytes
+        d.host_spill_bytes = host_spill_bytes
+        d.flags = flags | (N.GAMMA_FLAG_TIME_KERNELS if time_kernels else 0)
+        self.desc = d
+        h = C.c_void_p()
+        _check(_lib.gamma_ctx_create(C.byref(d), C.byref(h)), "gamma_ctx_create")
+        self._h = h
+        self.device, self.rank, self.world = device, d.rank, d.world
+
+    @property
+    def handle(self):
+        return self._h
+
+    def close(self):
+        if getattr(self, "_h", None):
+            _lib.gamma_ctx_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:   # noqa: BLE001
+            pass
+
+    def load_edges(self, n: int, src, dst, labels=None) -> "Graph":
+        ps, ks, m = _ptr(src, np.uint32)
+        pd, kd, m2 = _ptr(dst, np.uint32)
+        assert m == m2, "src and dst differ in length"
+        pl, kl, _ = _ptr(labels, np.uint32)
+        g = C.c_void_p()
+        _check(_lib.gamma_load_edges(self._h, int(n), ps, pd, int(m), pl, C.byref(g)), "gamma_load_edges")
+        return Graph(self, g)
+
+    def load_csr(self, n: int, row_ptr, col, labels=None) -> "Graph":
+        pr, kr, _ = _ptr(row_ptr, np.uint64)
+        pc, kc, _ = _ptr(col, np.uint32)
+        pl, kl, _ = _ptr(labels, np.uint32)
+        g = C.c_void_p()
+        _check(_lib.gamma_load_csr(self._h, int(n), pr, pc, pl, C.byref(g)), "gamma_load_csr")
+        return Graph(self, g)
+
+    def stats(self) -> dict:
+        s = N.gamma_run_stats()
+        _check(_lib.gamma_get_stats(self._h, C.byref(s)), "gamma_get_stats")
+        classes = {}
+        for i in range(s.n_classes):
+            name = bytes(s.name[i]).split(b"\0")[0].decode()
+            classes[name] = {"launches": int(s.launches[i]), "ms": float(s.ms[i]),
+                             "alg_bytes": int(s.alg_bytes[i])}
+        return {"classes": classes, "level_entries": [int(x) for x in s.level_entries],
+                "list_elems": int(s.list_elems), "chunks": int(s.chunks), "retries": int(s.retries),
+                "spilled_bytes": int(s.spilled_bytes), "total_launches": int(s.total_launches),
+                "wall_ms": float(s.wall_ms)}
+
+
+class Graph:
+    """A gamma_graph (symmetric CSR + degree-ordered DAG + labels) in HBM."""
+
+    def __init__(self, ctx: Context, h):
+        self.ctx = ctx
+        self._h = h
+
+    def free(self):
+        if getattr(self, "_h", None):
+            _lib.gamma_graph_free(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:   # noqa: BLE001
+            pass
+
+    def info(self) -> dict:
+        i = N.gamma_graph_info()
+        _check(_lib.gamma_graph_get_info(self._h, C.byref(i)), "gamma_graph_get_info")
+        return {"n": i.n, "m": i.m, "max_degree": i.max_degree, "max_out_degree": i.max_out_degree,
+                "device_bytes": i.device_bytes, "build_ms": i.build_ms}
+
+    def csr(self, which: str = "sym"):
+        inf = self.info()
+        w = 0 if which == "sym" else 1
+        ne = 2 * inf["m"] if w == 0 else inf["m"]
+        rp = np.empty(inf["n"] + 1, np.uint64)
+        col = np.empty(max(ne, 1), np.uint32)
+        _check(_lib.gamma_graph_copy_csr(self._h, w, rp.ctypes.data, col.ctypes.data), "gamma_graph_copy_csr")
+        return rp, col[:ne]
+
+    def kclique(self, k: int) -> int:
+        c = C.c_uint64()
+        _check(_lib.gamma_kclique(self._h, int(k), C.byref(c)), "gamma_kclique")
+        return int(c.value)
+
+    def kclique_roots(self, k: int, roots) -> np.ndarray:
+        pr, kr, nr = _ptr(roots, np.uint32)
+        out = np.zeros(nr, np.uint64)
+        _check(_lib.gamma_kclique_roots(self._h, int(k), nr, pr, out.ctypes.data), "gamma_kclique_roots")
+        return out
+
+    def match(self, nv: int, edges, labels=None, induced: bool = False):
+        """(count of distinct subgraphs, mappings = count * |Aut_L|)."""
+        e = np.ascontiguousarray(np.asarray(edges, dtype=np.uint32).reshape(-1))
+        p = N.gamma_pattern()
+        p.nv = nv
+        p.ne = e.size // 2
+        p.edges = e.ctypes.data_as(C.POINTER(C.c_uint32))
+        lab = None
+        if labels is not None:
+            lab = np.ascontiguousarray(labels, dtype=np.uint32)
+            p.labels = lab.ctypes.data_as(C.POINTER(C.c_uint32))
+        p.induced = 1 if induced else 0
+        c, mp = C.c_uint64(), C.c_uint64()
+        _check(_lib.gamma_match(self._h, C.byref(p), C.byref(c), C.byref(mp)), "gamma_match")
+        return int(c.value), int(mp.value)
+
+    def fpm(self, max_edges: int, minsup: int):
+        """Frequent patterns: sorted list of (ne, nv, labels, edges, support)."""
+        r = C.POINTER(N.gamma_fpm_result)()
+        _check(_lib.gamma_fpm(self._h, int(max_edges), int(minsup), C.byref(r)), "gamma_fpm")
+        try:
+            out = []
+            res = r.contents
+            for i in range(res.n):
+                pt = res.pats[i]
+                out.append((int(pt.ne), int(pt.nv), tuple(int(pt.labels[j]) for j in range(pt.nv)),
+                            tuple((int(pt.edges[e][0]), int(pt.edges[e][1])) for e in range(pt.ne)),
+                            int(pt.support)))
+            return out
+        finally:
+            _lib.gamma_fpm_result_free(r)

@@ -1,0 +1,347 @@
+// graph.cu -- A1: raw edge samples -> symmetric CSR (+ degree-ordered DAG, labels).
+//
+// PAPER.md L199 (§IV): "We adopt Compressed Sparse Row (CSR) to represent a data
+// graph G_d, which is made up of adjacency lists of all vertices"; L204: labels +
+// adjacency lists only.  O-0 normalisation (R13): symmetrise, drop
+// self-loops and duplicates, sort each list ascending.  DAG (R9, not in
+// the paper): keep u->v iff (deg u, u) < (deg v, v).
+//
+// B200 layout: one packed key per directed edge, (u << b) | v with b = bit width
+// of n, radix-sorted over exactly 2b bits (CUB onesweep, one pass per 8 bits);
+// duplicates removed by a unique pass; row_ptr / col produced by one fused
+// boundary kernel.  Everything stays in HBM; the only host sync is to learn m.
+#include <cub/device/device_radix_sort.cuh>
+#include <cub/device/device_select.cuh>
+
+#include "internal.cuh"
+
+namespace gamma_impl {
+
+namespace {
+
+constexpr int kThreads = 256;
+
+inline unsigned grid_for(uint64_t n, int threads = kThreads, unsigned cap = 148u * 64u) {
+  uint64_t b = (n + threads - 1) / threads;
+  if (b == 0) b = 1;
+  return (unsigned)(b < cap ? b : cap);
+}
+
+// Two directed keys per raw sample; self-loops and out-of-range ids become the
+// invalid key (all 2b bits set), which sorts after every valid key.
+__global__ void pack_keys_kernel(const uint32_t *__restrict__ src, const uint32_t *__restrict__ dst,
+                                 uint64_t m, uint32_t n, uint32_t b, uint64_t *__restrict__ keys,
+                                 unsigned long long *err) {
+  const uint64_t invalid = (b >= 32) ? ~0ull : ((1ull << (2 * b)) - 1);
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < m;
+       i += (uint64_t)gridDim.x * blockDim.x) {
+    uint32_t u = src[i], v = dst[i];
+    uint64_t k0 = invalid, k1 = invalid;
+    if (u >= n || v >= n) {
+      atomicOr(err, 1ull);
+    } else if (u != v) {
+      k0 = ((uint64_t)u << b) | v;
+      k1 = ((uint64_t)v << b) | u;
+    }
+    keys[2 * i] = k0;
+    keys[2 * i + 1] = k1;
+  }
+}
+
+// From M sorted, unique, valid keys (u << b | v): col[i] = v and row_ptr boundaries.
+__global__ void csr_from_keys_kernel(const uint64_t *__restrict__ keys, uint64_t M, uint32_t n,
+                                     uint32_t b, uint64_t *__restrict__ row_ptr,
+                                     uint32_t *__restrict__ col) {
+  const uint64_t mask = (b >= 32) ? 0xffffffffull : ((1ull << b) - 1);
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < M;
+       i += (uint64_t)gridDim.x * blockDim.x) {
+    uint64_t key = keys[i];
+    uint32_t u = (uint32_t)(key >> b);
+    col[i] = (uint32_t)(key & mask);
+    // rows (prev_u, u] start at i
+    int64_t prev_u = (i == 0) ? -1 : (int64_t)(keys[i - 1] >> b);
+    for (int64_t w = prev_u + 1; w <= (int64_t)u; w++) row_ptr[w] = i;
+    if (i == M - 1)
+      for (uint64_t w = (uint64_t)u + 1; w <= n; w++) row_ptr[w] = M;
+  }
+}
+
+__global__ void fill_u64_kernel(uint64_t *p, uint64_t n, uint64_t v) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n;
+       i += (uint64_t)gridDim.x * blockDim.x)
+    p[i] = v;
+}
+
+// DAG flag: keep directed edge u->v iff (deg u, u) < (deg v, v).
+struct DagKeep {
+  const uint64_t *row_ptr;
+  uint32_t b;
+  uint64_t mask;
+  __device__ __forceinline__ bool operator()(const uint64_t &key) const {
+    uint32_t u = (uint32_t)(key >> b), v = (uint32_t)(key & mask);
+    uint64_t du = row_ptr[u + 1] - row_ptr[u], dv = row_ptr[v + 1] - row_ptr[v];
+    return du < dv || (du == dv && u < v);
+  }
+};
+
+__global__ void max_degree_kernel(const uint64_t *__restrict__ rp, uint32_t n,
+                                  unsigned long long *out) {
+  unsigned long long best = 0;
+  for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n;
+       v += (uint64_t)gridDim.x * blockDim.x) {
+    unsigned long long d = rp[v + 1] - rp[v];
+    best = d > best ? d : best;
+  }
+  for (int o = 16; o > 0; o >>= 1) {
+    unsigned long long x = __shfl_down_sync(0xffffffffu, best, o);
+    best = x > best ? x : best;
+  }
+  if ((threadIdx.x & 31) == 0) atomicMax(out, best);
+}
+
+// Expand a CSR into keys (u << b | v) and validate: ids < n, no self-loop, strictly
+// ascending lists.  err bit 1: range/self-loop/order violation.
+__global__ void csr_to_keys_kernel(const uint64_t *__restrict__ rp, const uint32_t *__restrict__ col,
+                                   uint32_t n, uint32_t b, uint64_t *__restrict__ keys,
+                                   unsigned long long *err) {
+  // one warp per vertex
+  const int lane = threadIdx.x & 31;
+  for (uint64_t v = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5; v < n;
+       v += ((uint64_t)gridDim.x * blockDim.x) >> 5) {
+    uint64_t s = rp[v], e = rp[v + 1];
+    if (e < s) {
+      if (lane == 0) atomicOr(err, 1ull);
+      continue;
+    }
+    for (uint64_t i = s + lane; i < e; i += 32) {
+      uint32_t x = col[i];
+      bool bad = x >= n || x == (uint32_t)v || (i > s && col[i - 1] >= x);
+      if (bad) atomicOr(err, 1ull);
+      keys[i] = ((uint64_t)v << b) | (x < n ? x : 0);
+    }
+  }
+}
+
+// Symmetry: every (v, x) must have v in N(x).  Binary search per element.
+__global__ void csr_symmetry_kernel(const uint64_t *__restrict__ rp, const uint32_t *__restrict__ col,
+                                    uint32_t n, unsigned long long *err) {
+  const int lane = threadIdx.x & 31;
+  for (uint64_t v = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5; v < n;
+       v += ((uint64_t)gridDim.x * blockDim.x) >> 5) {
+    for (uint64_t i = rp[v] + lane; i < rp[v + 1]; i += 32) {
+      uint32_t x = col[i];
+      uint64_t lo = rp[x], hi = rp[x + 1];
+      while (lo < hi) {
+        uint64_t mid = (lo + hi) >> 1;
+        if (col[mid] < (uint32_t)v) lo = mid + 1; else hi = mid;
+      }
+      if (lo >= rp[x + 1] || col[lo] != (uint32_t)v) atomicOr(err, 2ull);
+    }
+  }
+}
+
+uint32_t bit_width(uint32_t n) {  // bits to represent n itself
+  uint32_t b = 0;
+  while (b < 32 && (uint64_t(1) << b) <= n) b++;
+  return b ? b : 1;
+}
+
+void sort_keys(gamma_ctx *ctx, const uint64_t *in, uint64_t *out, uint64_t nkeys, int end_bit) {
+  size_t tmp = 0;
+  GAMMA_CUDA(cub::DeviceRadixSort::SortKeys(nullptr, tmp, in, out, nkeys, 0, end_bit, ctx->stream));
+  DevBuf<uint8_t> t(ctx, tmp);
+  ctx->launch(KC_BUILD, [&] {
+    GAMMA_CUDA(cub::DeviceRadixSort::SortKeys(t.p, tmp, in, out, nkeys, 0, end_bit, ctx->stream));
+  });
+  // onesweep: histogram + one pass per 8 key bits (+ the launch counted above)
+  ctx->stats.launches[KC_BUILD] += (end_bit + 7) / 8;
+  ctx->stats.total_launches += (end_bit + 7) / 8;
+}
+
+// keys -> (row_ptr, col) on g for M keys.
+void keys_to_csr(gamma_ctx *ctx, const uint64_t *keys, uint64_t M, uint32_t n, uint32_t b,
+                 uint64_t *row_ptr, uint32_t *col) {
+  if (M == 0) {
+    ctx->launch(KC_BUILD, [&] {
+      fill_u64_kernel<<<grid_for(n + 1), kThreads, 0, ctx->stream>>>(row_ptr, (uint64_t)n + 1, 0);
+    });
+    return;
+  }
+  ctx->launch(KC_BUILD, [&] {
+    csr_from_keys_kernel<<<grid_for(M), kThreads, 0, ctx->stream>>>(keys, M, n, b, row_ptr, col);
+  });
+}
+
+uint32_t max_degree(gamma_ctx *ctx, const uint64_t *rp, uint32_t n) {
+  GAMMA_CUDA(cudaMemsetAsync(ctx->ctrl + CTRL_AUX0, 0, sizeof(uint64_t), ctx->stream));
+  ctx->launch(KC_BUILD, [&] {
+    max_degree_kernel<<<grid_for(n), kThreads, 0, ctx->stream>>>(
+        rp, n, (unsigned long long *)(ctx->ctrl + CTRL_AUX0));
+  });
+  uint64_t h = 0;
+  GAMMA_CUDA(cudaMemcpyAsync(&h, ctx->ctrl + CTRL_AUX0, sizeof(uint64_t), cudaMemcpyDeviceToHost, ctx->stream));
+  ctx->sync();
+  return (uint32_t)h;
+}
+
+struct BuildTimer {
+  gamma_ctx *ctx;
+  cudaEvent_t a = nullptr, b = nullptr;
+  explicit BuildTimer(gamma_ctx *c) : ctx(c) {
+    GAMMA_CUDA(cudaEventCreate(&a));
+    GAMMA_CUDA(cudaEventCreate(&b));
+    GAMMA_CUDA(cudaEventRecord(a, ctx->stream));
+  }
+  double stop() {
+    GAMMA_CUDA(cudaEventRecord(b, ctx->stream));
+    GAMMA_CUDA(cudaEventSynchronize(b));
+    float ms = 0;
+    GAMMA_CUDA(cudaEventElapsedTime(&ms, a, b));
+    return ms;
+  }
+  ~BuildTimer() {
+    if (a) cudaEventDestroy(a);
+    if (b) cudaEventDestroy(b);
+  }
+};
+
+}  // namespace
+
+void build_dag(gamma_graph *g, uint64_t *keys, uint64_t M) {
+  gamma_ctx *ctx = g->ctx;
+  const uint32_t b = g->bits;
+  const uint64_t mask = (b >= 32) ? 0xffffffffull : ((1ull << b) - 1);
+  DevBuf<uint64_t> dkeys(ctx, M / 2 + 1);
+  DevBuf<uint64_t> nsel(ctx, 1);
+  DagKeep op{g->row_ptr, b, mask};
+  size_t tmp = 0;
+  GAMMA_CUDA(cub::DeviceSelect::If(nullptr, tmp, keys, dkeys.p, nsel.p, (int64_t)M, op, ctx->stream));
+  DevBuf<uint8_t> t(ctx, tmp);
+  ctx->launch(KC_BUILD, [&] {
+    GAMMA_CUDA(cub::DeviceSelect::If(t.p, tmp, keys, dkeys.p, nsel.p, (int64_t)M, op, ctx->stream));
+  });
+  uint64_t mdag = 0;
+  GAMMA_CUDA(cudaMemcpyAsync(&mdag, nsel.p, sizeof(uint64_t), cudaMemcpyDeviceToHost, ctx->stream));
+  ctx->sync();
+  GAMMA_REQUIRE(mdag == g->m, GAMMA_E_CUDA, "DAG orientation kept " + std::to_string(mdag) +
+                                                " of " + std::to_string(g->m) + " edges");
+  DevBuf<uint64_t> dp(ctx, (size_t)g->n + 1);
+  DevBuf<uint32_t> dc(ctx, mdag ? mdag : 1);
+  keys_to_csr(ctx, dkeys.p, mdag, g->n, b, dp.p, dc.p);
+  g->dag_ptr = dp.release();
+  g->dag_col = dc.release();
+  g->device_bytes += ((uint64_t)g->n + 1) * 8 + mdag * 4;
+  g->max_out_degree = max_degree(ctx, g->dag_ptr, g->n);
+}
+
+void build_from_edges(gamma_graph *g, const uint32_t *src, const uint32_t *dst, uint64_t m,
+                      bool on_device) {
+  gamma_ctx *ctx = g->ctx;
+  BuildTimer timer(ctx);
+  const uint32_t n = g->n;
+  const uint32_t b = bit_width(n);
+  g->bits = b;
+  DevBuf<uint32_t> s_copy, d_copy;
+  if (!on_device && m) {
+    s_copy = to_device(ctx, src, m);
+    d_copy = to_device(ctx, dst, m);
+    src = s_copy.p;
+    dst = d_copy.p;
+  }
+  const uint64_t nkeys = 2 * m;
+  uint64_t M = 0;
+  DevBuf<uint64_t> uniq;
+  if (nkeys) {
+    DevBuf<uint64_t> keys(ctx, nkeys);
+    GAMMA_CUDA(cudaMemsetAsync(ctx->ctrl + CTRL_ERR, 0, sizeof(uint64_t), ctx->stream));
+    ctx->launch(KC_BUILD, [&] {
+      pack_keys_kernel<<<grid_for(m), kThreads, 0, ctx->stream>>>(
+          src, dst, m, n, b, keys.p, (unsigned long long *)(ctx->ctrl + CTRL_ERR));
+    });
+    s_copy.reset();
+    d_copy.reset();
+    DevBuf<uint64_t> sorted(ctx, nkeys);
+    sort_keys(ctx, keys.p, sorted.p, nkeys, (int)(2 * b));
+    keys.reset();
+    uniq = DevBuf<uint64_t>(ctx, nkeys);
+    DevBuf<uint64_t> nsel(ctx, 2);
+    size_t tmp = 0;
+    GAMMA_CUDA(cub::DeviceSelect::Unique(nullptr, tmp, sorted.p, uniq.p, nsel.p, (int64_t)nkeys, ctx->stream));
+    {
+      DevBuf<uint8_t> t(ctx, tmp);
+      ctx->launch(KC_BUILD, [&] {
+        GAMMA_CUDA(cub::DeviceSelect::Unique(t.p, tmp, sorted.p, uniq.p, nsel.p, (int64_t)nkeys, ctx->stream));
+      });
+    }
+    uint64_t h[2] = {0, 0};
+    GAMMA_CUDA(cudaMemcpyAsync(&h[0], nsel.p, sizeof(uint64_t), cudaMemcpyDeviceToHost, ctx->stream));
+    GAMMA_CUDA(cudaMemcpyAsync(&h[1], ctx->ctrl + CTRL_ERR, sizeof(uint64_t), cudaMemcpyDeviceToHost, ctx->stream));
+    ctx->sync();
+    GAMMA_REQUIRE(h[1] == 0, GAMMA_E_INVAL, "gamma_load_edges: vertex id >= n");
+    M = h[0];
+    if (M) {  // drop the (single, last) invalid key if present
+      uint64_t last = 0;
+      GAMMA_CUDA(cudaMemcpyAsync(&last, uniq.p + M - 1, sizeof(uint64_t), cudaMemcpyDeviceToHost, ctx->stream));
+      ctx->sync();
+      const uint64_t invalid = (b >= 32) ? ~0ull : ((1ull << (2 * b)) - 1);
+      if (last == invalid) M--;
+    }
+  }
+  GAMMA_REQUIRE(M % 2 == 0, GAMMA_E_CUDA, "asymmetric key set after unique");
+  g->m = M / 2;
+  DevBuf<uint64_t> rp(ctx, (size_t)n + 1);
+  DevBuf<uint32_t> col(ctx, M ? M : 1);
+  keys_to_csr(ctx, uniq.p, M, n, b, rp.p, col.p);
+  g->row_ptr = rp.release();
+  g->col = col.release();
+  g->device_bytes += ((uint64_t)n + 1) * 8 + M * 4;
+  g->max_degree = max_degree(ctx, g->row_ptr, n);
+  build_dag(g, uniq.p, M);
+  g->build_ms = timer.stop();
+}
+
+void build_from_csr(gamma_graph *g, const uint64_t *row_ptr, const uint32_t *col) {
+  gamma_ctx *ctx = g->ctx;
+  BuildTimer timer(ctx);
+  const uint32_t n = g->n;
+  g->bits = bit_width(n);
+  DevBuf<uint64_t> rp = to_device(ctx, row_ptr, (size_t)n + 1);
+  uint64_t M = 0, first = 0;
+  GAMMA_CUDA(cudaMemcpyAsync(&first, rp.p, sizeof(uint64_t), cudaMemcpyDeviceToHost, ctx->stream));
+  GAMMA_CUDA(cudaMemcpyAsync(&M, rp.p + n, sizeof(uint64_t), cudaMemcpyDeviceToHost, ctx->stream));
+  ctx->sync();
+  GAMMA_REQUIRE(first == 0, GAMMA_E_INVAL, "gamma_load_csr: row_ptr[0] != 0");
+  GAMMA_REQUIRE(M % 2 == 0, GAMMA_E_INVAL, "gamma_load_csr: odd number of directed edges");
+  GAMMA_REQUIRE(M == 0 || col, GAMMA_E_INVAL, "gamma_load_csr: NULL col");
+  DevBuf<uint32_t> cl = to_device(ctx, col, M ? M : 0);
+  if (!M) cl = DevBuf<uint32_t>(ctx, 1);
+  DevBuf<uint64_t> keys(ctx, M ? M : 1);
+  GAMMA_CUDA(cudaMemsetAsync(ctx->ctrl + CTRL_ERR, 0, sizeof(uint64_t), ctx->stream));
+  unsigned grid = grid_for((uint64_t)n * 32);
+  if (M) {
+    ctx->launch(KC_BUILD, [&] {
+      csr_to_keys_kernel<<<grid, kThreads, 0, ctx->stream>>>(rp.p, cl.p, n, g->bits, keys.p,
+                                                             (unsigned long long *)(ctx->ctrl + CTRL_ERR));
+    });
+    uint64_t err = 0;
+    GAMMA_CUDA(cudaMemcpyAsync(&err, ctx->ctrl + CTRL_ERR, sizeof(uint64_t), cudaMemcpyDeviceToHost, ctx->stream));
+    ctx->sync();
+    GAMMA_REQUIRE(err == 0, GAMMA_E_INVAL, "gamma_load_csr: list not strictly ascending, self-loop, or id >= n");
+    ctx->launch(KC_BUILD, [&] {
+      csr_symmetry_kernel<<<grid, kThreads, 0, ctx->stream>>>(rp.p, cl.p, n,
+                                                              (unsigned long long *)(ctx->ctrl + CTRL_ERR));
+    });
+    GAMMA_CUDA(cudaMemcpyAsync(&err, ctx->ctrl + CTRL_ERR, sizeof(uint64_t), cudaMemcpyDeviceToHost, ctx->stream));
+    ctx->sync();
+    GAMMA_REQUIRE(err == 0, GAMMA_E_INVAL, "gamma_load_csr: adjacency is not symmetric");
+  }
+  g->m = M / 2;
+  g->row_ptr = rp.release();
+  g->col = cl.release();
+  g->device_bytes += ((uint64_t)n + 1) * 8 + M * 4;
+  g->max_degree = max_degree(ctx, g->row_ptr, n);
+  build_dag(g, keys.p, M);
+  g->build_ms = timer.stop();
+}
+
+}  // namespace gamma_impl

@@ -1,0 +1,204 @@
+// internal.cuh -- shared internals of libgamma (CUDA side only; never included by
+// oracle/).  Context, graph, error plumbing, device allocation, launch timing.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+#include <vector>
+
+#include "gamma.h"
+
+namespace gamma_impl {
+
+// ---- thread-local error message -------------------------------------------------
+void set_error(const std::string &msg);
+void clear_error();
+
+struct Fail {
+  gamma_status st;
+  std::string msg;
+};
+
+#define GAMMA_CUDA(expr)                                                              \
+  do {                                                                                \
+    cudaError_t e_ = (expr);                                                          \
+    if (e_ != cudaSuccess)                                                            \
+      throw ::gamma_impl::Fail{GAMMA_E_CUDA, std::string(#expr) + ": " +              \
+                                                 cudaGetErrorString(e_)};             \
+  } while (0)
+
+#define GAMMA_REQUIRE(cond, status, msg)                                              \
+  do {                                                                                \
+    if (!(cond)) throw ::gamma_impl::Fail{(status), (msg)};                           \
+  } while (0)
+
+// Runs f(), converting Fail / std exceptions into a status + thread-local message.
+template <class F>
+gamma_status guarded(F &&f) {
+  try {
+    clear_error();
+    f();
+    return GAMMA_OK;
+  } catch (const Fail &e) {
+    set_error(e.msg);
+    return e.st;
+  } catch (const std::bad_alloc &) {
+    set_error("host allocation failed");
+    return GAMMA_E_NOMEM;
+  } catch (const std::exception &e) {
+    set_error(e.what());
+    return GAMMA_E_INVAL;
+  } catch (...) {
+    set_error("unknown error");
+    return GAMMA_E_INVAL;
+  }
+}
+
+// ---- per-kernel-class statistics -------------------------------------------------
+enum KernelClass {
+  KC_BUILD = 0,      // A1 CSR/DAG build kernels (incl. CUB sort)
+  KC_ROOTS,          // A2 root list / cost / partition
+  KC_EXTEND,         // A3-A6 extend (stage + intersect + filter + compact + write)
+  KC_COUNT,          // A4+A7 last-level intersect-and-count
+  KC_FUSED,          // A3-A7 fused last two levels (DFS tail)
+  KC_SM_EXTEND,      // SM extend
+  KC_SM_COUNT,       // SM last level
+  KC_FPM,            // FPM edge extension / canonical code / domain bits
+  KC_FPM_SUPPORT,    // FPM popc / min over orbits
+  KC_MISC,           // memsets, small helpers
+  KC_NUM
+};
+extern const char *kKernelClassName[KC_NUM];
+
+struct Ctrl;  // device control block (counters), defined in ctx.cu
+
+struct gamma_ctx_impl;
+}  // namespace gamma_impl
+
+struct gamma_ctx {
+  gamma_ctx_desc desc;
+  int device = 0;
+  int num_sms = 148;
+  size_t smem_optin = 0;
+  cudaStream_t stream = nullptr;
+  bool own_stream = false;
+  // device control block: counters reset per launch
+  uint64_t *ctrl = nullptr;  // CTRL_WORDS u64 on device
+  uint64_t *ctrl_host = nullptr;  // pinned mirror
+  // stats of the last call
+  gamma_run_stats stats;
+  // event pool for kernel timing
+  std::vector<cudaEvent_t> ev_pool;
+  std::vector<std::pair<int, std::pair<cudaEvent_t, cudaEvent_t>>> pending;
+  size_t ev_next = 0;
+
+  void *alloc(size_t bytes);
+  void free(void *p);
+  void reset_stats();
+  // Launch helper: brackets the launch with events when timing is on.
+  template <class F>
+  void launch(int kc, F &&f) {
+    cudaEvent_t a = nullptr, b = nullptr;
+    bool timing = (desc.flags & GAMMA_FLAG_TIME_KERNELS) != 0;
+    if (timing) {
+      a = next_event();
+      b = next_event();
+      cudaEventRecord(a, stream);
+    }
+    f();
+    GAMMA_CUDA(cudaGetLastError());
+    if (timing) {
+      cudaEventRecord(b, stream);
+      pending.push_back({kc, {a, b}});
+    }
+    stats.launches[kc]++;
+    stats.total_launches++;
+  }
+  cudaEvent_t next_event();
+  void collect_timings();  // after a stream sync
+  void sync() { GAMMA_CUDA(cudaStreamSynchronize(stream)); }
+};
+
+// control block layout (u64 words)
+enum {
+  CTRL_WORK = 0,      // dynamic work counter
+  CTRL_VCUR = 1,      // vid cursor of the level being written
+  CTRL_GCUR = 2,      // group cursor of the level being written
+  CTRL_OVF = 3,       // overflow flag
+  CTRL_COUNT = 4,     // result accumulator
+  CTRL_ELEMS = 5,     // adjacency elements fetched (algorithmic)
+  CTRL_ENTRIES = 6,   // entries produced (kept)
+  CTRL_ERR = 7,       // validation error flag
+  CTRL_AUX0 = 8,
+  CTRL_AUX1 = 9,
+  CTRL_WORDS = 16
+};
+
+struct gamma_graph {
+  gamma_ctx *ctx = nullptr;
+  uint32_t n = 0;
+  uint64_t m = 0;
+  uint32_t bits = 1;             // bits needed for a vertex id (ids < 2^bits)
+  uint64_t *row_ptr = nullptr;   // n+1
+  uint32_t *col = nullptr;       // 2m
+  uint64_t *dag_ptr = nullptr;   // n+1
+  uint32_t *dag_col = nullptr;   // m
+  uint32_t *labels = nullptr;    // n (nullptr: unlabeled, all 0)
+  uint32_t max_degree = 0, max_out_degree = 0;
+  uint64_t device_bytes = 0;
+  double build_ms = 0;
+};
+
+// RAII device buffer through the ctx allocator.
+template <class T>
+struct DevBuf {
+  gamma_ctx *ctx = nullptr;
+  T *p = nullptr;
+  size_t n = 0;
+  DevBuf() = default;
+  DevBuf(gamma_ctx *c, size_t count) : ctx(c), n(count) {
+    p = static_cast<T *>(c->alloc(count * sizeof(T) ? count * sizeof(T) : 16));
+  }
+  DevBuf(const DevBuf &) = delete;
+  DevBuf &operator=(const DevBuf &) = delete;
+  DevBuf(DevBuf &&o) noexcept : ctx(o.ctx), p(o.p), n(o.n) { o.p = nullptr; }
+  DevBuf &operator=(DevBuf &&o) noexcept {
+    reset();
+    ctx = o.ctx; p = o.p; n = o.n; o.p = nullptr;
+    return *this;
+  }
+  ~DevBuf() { reset(); }
+  void reset() {
+    if (p && ctx) ctx->free(p);
+    p = nullptr;
+  }
+  T *release() { T *q = p; p = nullptr; return q; }
+};
+
+namespace gamma_impl {
+// Is ptr a device (or managed) pointer usable by kernels?
+bool is_device_ptr(const void *ptr);
+// Copy n elements of an input array (host or device) into a fresh device buffer.
+template <class T>
+DevBuf<T> to_device(gamma_ctx *ctx, const T *src, size_t n) {
+  DevBuf<T> d(ctx, n);
+  if (n) GAMMA_CUDA(cudaMemcpyAsync(d.p, src, n * sizeof(T), cudaMemcpyDefault, ctx->stream));
+  return d;
+}
+void ctrl_reset(gamma_ctx *ctx);                 // zero all control words (async)
+void ctrl_fetch(gamma_ctx *ctx);                 // async D2H into ctrl_host + sync
+int occupancy_blocks(const void *kernel, int threads, size_t smem);
+uint64_t checked_add(uint64_t a, uint64_t b);    // throws E_OVERFLOW
+
+// A1: builders (graph.cu)
+void build_from_edges(gamma_graph *g, const uint32_t *src, const uint32_t *dst, uint64_t m,
+                      bool src_on_device);
+void build_from_csr(gamma_graph *g, const uint64_t *row_ptr, const uint32_t *col);
+void build_dag(gamma_graph *g, uint64_t *sorted_keys_dev, uint64_t nkeys);
+
+// kCL (kclique.cu)
+uint64_t kclique_count(gamma_graph *g, uint32_t k, const uint32_t *roots_dev, uint64_t nroots,
+                       uint64_t *per_root_dev);
+}  // namespace gamma_impl

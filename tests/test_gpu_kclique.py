@@ -1,0 +1,221 @@
+"""GPU parity of A1 (CSR/DAG build) and kCL (A2-A8) against the oracle, through the
+C ABI.  Tolerance 0: every output is an integer (north_star)."""
+from math import comb
+
+import numpy as np
+import pytest
+
+import gamma_gen as gg
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def G():
+    import torch
+    assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+    import paper_conf_icde_hu0o23_b200 as G
+    return G
+
+
+@pytest.fixture(scope="module")
+def ctx(G):
+    return G.Context(device=0)
+
+
+def load(ctx, n, s, d, lab=None):
+    return ctx.load_edges(n, s, d, lab)
+
+
+def test_library_is_in_tree(G):
+    import os
+    assert os.path.dirname(G.library_path()) == os.path.dirname(G.__file__)
+
+
+def test_csr_matches_oracle(ctx, oracle_mod):
+    for seed in (1, 2, 3):
+        n, s, d, _ = gg.config_graph("c1", seed=seed)
+        g = load(ctx, n, s, d)
+        o = oracle_mod.Graph(n, s, d)
+        rp, col = g.csr("sym")
+        orp, ocol = o.csr()
+        assert g.info()["m"] == o.m
+        assert np.array_equal(rp, orp) and np.array_equal(col, ocol)
+
+
+def test_csr_from_device_tensors(ctx, oracle_mod):
+    import torch
+    n, s, d, _ = gg.config_graph("c1", seed=4, scale=11)
+    g = ctx.load_edges(n, torch.from_numpy(s.view(np.int32)).cuda(), torch.from_numpy(d.view(np.int32)).cuda())
+    o = oracle_mod.Graph(n, s, d)
+    rp, col = g.csr("sym")
+    orp, ocol = o.csr()
+    assert np.array_equal(rp, orp) and np.array_equal(col, ocol)
+
+
+def test_dag_definition(ctx):
+    n, s, d, _ = gg.config_graph("c1", seed=1)
+    g = load(ctx, n, s, d)
+    rp, col = g.csr("sym")
+    drp, dcol = g.csr("dag")
+    deg = np.diff(rp.astype(np.int64))
+    m = g.info()["m"]
+    assert drp[-1] == m
+    for v in range(0, n, 7):
+        out = dcol[drp[v]:drp[v + 1]]
+        assert np.all(np.diff(out.astype(np.int64)) > 0)
+        nb = col[rp[v]:rp[v + 1]]
+        want = [u for u in nb if (deg[v], v) < (deg[u], u)]
+        assert out.tolist() == want
+    assert g.info()["max_out_degree"] == int(np.diff(drp.astype(np.int64)).max())
+
+
+def test_closed_forms(ctx):
+    cases = [(gg.complete(12), {k: comb(12, k) for k in range(1, 14)}),
+             (gg.turan(12, 4), {k: comb(4, k) * 3 ** k for k in range(2, 6)}),
+             (gg.wheel(9), {3: 9, 4: 0}),
+             (gg.cycle(3), {3: 1}),
+             (gg.grid(6, 7), {3: 0}),
+             (gg.petersen(), {3: 0})]
+    for (n, (s, d)), want in cases:
+        g = load(ctx, n, s, d)
+        for k, c in want.items():
+            assert g.kclique(k) == c, (n, k)
+
+
+def test_complete_large_k(ctx):
+    # K_24 holds 2^24 cliques over all sizes: deep levels without blowing up the test
+    n, (s, d) = gg.complete(24)
+    g = load(ctx, n, s, d)
+    for k in (5, 8, 12, 20, 24, 25, 32):
+        assert g.kclique(k) == comb(24, k)
+
+
+@pytest.mark.parametrize("seed", [1, 2, 3, 4, 5])
+def test_er_vs_oracle(ctx, oracle_mod, seed):
+    n = 1 << (10 + seed)
+    s, d = gg.er(n, 12 * n, seed)
+    g = load(ctx, n, s, d)
+    o = oracle_mod.Graph(n, s, d)
+    for k in (3, 4, 5):
+        assert g.kclique(k) == o.kclique(k)
+
+
+@pytest.mark.parametrize("seed", [1, 2, 3])
+def test_c1_vs_oracle(ctx, oracle_mod, seed):
+    n, s, d, _ = gg.config_graph("c1", seed=seed)
+    g = load(ctx, n, s, d)
+    o = oracle_mod.Graph(n, s, d)
+    for k in (1, 2, 3, 4, 5, 6):
+        assert g.kclique(k) == o.kclique(k), k
+
+
+def test_per_root_counts(ctx, oracle_mod):
+    n, s, d, _ = gg.config_graph("c1", seed=2, scale=11)
+    g = load(ctx, n, s, d)
+    o = oracle_mod.Graph(n, s, d)
+    roots = np.arange(n, dtype=np.uint32)
+    for k in (2, 3, 4, 5):
+        got = g.kclique_roots(k, roots)
+        want = o.kclique_roots(k, roots)
+        assert np.array_equal(got, want), k
+        assert int(got.sum()) == g.kclique(k)
+
+
+def test_budget_forced_splits(G, oracle_mod):
+    n, s, d, _ = gg.config_graph("c1", seed=1)
+    o = oracle_mod.Graph(n, s, d)
+    c = G.Context(hbm_budget_bytes=3 << 20)   # ~3 MB of ET: forces range splits
+    g = c.load_edges(n, s, d)
+    for k in (4, 5, 6):
+        assert g.kclique(k) == o.kclique(k)
+    st = c.stats()
+    assert st["retries"] > 0
+
+
+def test_simulated_ranks_partition(G, oracle_mod):
+    n, s, d, _ = gg.config_graph("c1", seed=3)
+    want = oracle_mod.Graph(n, s, d).kclique(5)
+    for world in (2, 3, 8):
+        tot = 0
+        for r in range(world):
+            c = G.Context(rank=r, world=world, reduce=False)
+            tot += c.load_edges(n, s, d).kclique(5)
+        assert tot == want
+
+
+def test_load_csr_roundtrip_and_validation(G, ctx, oracle_mod):
+    n, s, d, _ = gg.config_graph("c1", seed=5, scale=11)
+    o = oracle_mod.Graph(n, s, d)
+    rp, col = o.csr()
+    g = ctx.load_csr(n, rp, col)
+    assert g.kclique(4) == o.kclique(4)
+    bad = col.copy()
+    i = int(rp[5])
+    if rp[6] - rp[5] >= 2:
+        bad[i], bad[i + 1] = bad[i + 1], bad[i]      # unsorted list
+        with pytest.raises(G.GammaError):
+            ctx.load_csr(n, rp, bad)
+    # asymmetric: drop one direction
+    rp2, col2 = gg.path(3)[1]
+    with pytest.raises(G.GammaError):
+        ctx.load_csr(3, np.array([0, 1, 1, 1], np.uint64), np.array([1], np.uint32))
+
+
+def test_edge_cases(G, ctx):
+    g = ctx.load_edges(7, np.zeros(0, np.uint32), np.zeros(0, np.uint32))
+    assert g.kclique(1) == 7 and g.kclique(2) == 0 and g.kclique(3) == 0
+    g = ctx.load_edges(3, np.array([0, 1, 1], np.uint32), np.array([0, 1, 1], np.uint32))  # self-loops only
+    assert g.info()["m"] == 0 and g.kclique(3) == 0
+    with pytest.raises(G.GammaError):
+        ctx.load_edges(3, np.array([0], np.uint32), np.array([5], np.uint32))
+    n, (s, d) = gg.complete(5)
+    g = ctx.load_edges(n, s, d)
+    with pytest.raises(G.GammaError) as e:
+        g.kclique(33)
+    assert e.value.status == -5
+    with pytest.raises(G.GammaError):
+        g.kclique(0)
+
+
+def test_unstaged_long_run_path(G, oracle_mod):
+    """Runs longer than the shared-memory staging buffer take the global-memory
+    probe and the direct-reservation write path; the debug flag forces that path
+    for every group so it is checked on ordinary inputs."""
+    c = G.Context(flags=0x8)   # GAMMA_FLAG_DEBUG_NOSTAGE
+    for seed in (1, 2):
+        n, s, d, _ = gg.config_graph("c1", seed=seed)
+        g = c.load_edges(n, s, d)
+        o = oracle_mod.Graph(n, s, d)
+        for k in (3, 4, 5, 6):
+            assert g.kclique(k) == o.kclique(k)
+
+
+def test_hub_out_list_longer_than_staging(ctx, oracle_mod):
+    """A real vertex with d+(v) > 1024: v joined to 1100 vertices of K_{1100,1101}'s
+    larger side (those outrank v), plus a sprinkle of edges among them."""
+    a, b = 1100, 1101
+    U = np.arange(1, 1 + a)
+    F = np.arange(1 + a, 1 + a + b)
+    e = [(0, u) for u in U] + [(u, f) for u in U for f in F[:b]]
+    rng = np.random.default_rng(3)
+    extra = rng.choice(U, size=(3000, 2))
+    e = np.array(e + [tuple(x) for x in extra], dtype=np.uint32)
+    n = 1 + a + b
+    g = ctx.load_edges(n, e[:, 0].copy(), e[:, 1].copy())
+    assert g.info()["max_out_degree"] > 1024
+    o = oracle_mod.Graph(n, e[:, 0].copy(), e[:, 1].copy())
+    roots = np.array([0], np.uint32)
+    for k in (3, 4):
+        assert np.array_equal(g.kclique_roots(k, roots), o.kclique_roots(k, roots))
+
+
+@pytest.mark.slow
+def test_c2_full_size(ctx, oracle_mod):
+    """configs[1] at full size: cit-Patents-shaped R-MAT scale 22, k = 4, 5, 6."""
+    n, s, d, _ = gg.config_graph("c2", seed=1)
+    g = load(ctx, n, s, d)
+    o = oracle_mod.Graph(n, s, d)
+    assert g.info()["m"] == o.m
+    for k in (4, 5, 6):
+        assert g.kclique(k) == o.kclique(k), k
