@@ -142,6 +142,20 @@ typedef struct {
   int32_t induced;           /* must be 0 in v1 (E_UNSUPPORTED otherwise)            */
 } gamma_pattern;
 
+/* Host-only planning of a pattern (no device needed): the matching order delta_v
+ * (Alg. 1 line 1; R10), |Aut_L(P)| and the symmetry-breaking
+ * order constraints gamma_match applies.  Masks are over matching-order positions.
+ * Errors: E_INVAL (nv out of [1,8], bad edge, disconnected), E_UNSUPPORTED (induced). */
+typedef struct {
+  uint32_t nv;
+  uint32_t order[8];         /* position -> pattern vertex                           */
+  uint32_t backward_mask[8]; /* earlier positions adjacent to this one               */
+  uint32_t less_mask[8];     /* earlier positions j with phi_j < phi_i required      */
+  uint32_t greater_mask[8];  /* earlier positions j with phi_i < phi_j required      */
+  uint64_t aut;              /* |Aut_L(P)|                                           */
+} gamma_plan_info;
+gamma_status gamma_pattern_plan(const gamma_pattern *p, gamma_plan_info *out);
+
 /* *count = number of distinct subgraphs of G isomorphic to P (labels respected);
  * mappings (nullable) = *count * |Aut_L(P)|.  Partitioned / reduced like kclique. */
 gamma_status gamma_match(gamma_graph *g, const gamma_pattern *p, uint64_t *count,

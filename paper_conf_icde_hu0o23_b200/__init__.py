@@ -26,7 +26,7 @@ _lib = N.load()
 for _name, _res, _args in N.SIGNATURES:
     globals()[_name] = getattr(_lib, _name)
 
-__all__ = ["Context", "Graph", "GammaError", "library_path"] + [s[0] for s in N.SIGNATURES]
+__all__ = ["Context", "Graph", "GammaError", "library_path", "pattern_plan"] + [s[0] for s in N.SIGNATURES]
 
 
 def library_path() -> str:
@@ -60,6 +60,32 @@ def _ptr(x, dtype):
         pass
     a = np.ascontiguousarray(x, dtype=dtype)
     return a.ctypes.data, a, a.size
+
+
+def _pattern(nv, edges, labels=None, induced=False):
+    e = np.ascontiguousarray(np.asarray(edges, dtype=np.uint32).reshape(-1))
+    p = N.gamma_pattern()
+    p.nv = nv
+    p.ne = e.size // 2
+    p.edges = e.ctypes.data_as(C.POINTER(C.c_uint32))
+    keep = [e]
+    if labels is not None:
+        lab = np.ascontiguousarray(labels, dtype=np.uint32)
+        p.labels = lab.ctypes.data_as(C.POINTER(C.c_uint32))
+        keep.append(lab)
+    p.induced = 1 if induced else 0
+    return p, keep
+
+
+def pattern_plan(nv: int, edges, labels=None, induced: bool = False) -> dict:
+    """Host-only planner output: matching order, |Aut_L|, symmetry constraints."""
+    p, keep = _pattern(nv, edges, labels, induced)
+    info = N.gamma_plan_info()
+    _check(_lib.gamma_pattern_plan(C.byref(p), C.byref(info)), "gamma_pattern_plan")
+    return {"nv": info.nv, "order": [info.order[i] for i in range(nv)],
+            "backward_mask": [info.backward_mask[i] for i in range(nv)],
+            "less_mask": [info.less_mask[i] for i in range(nv)],
+            "greater_mask": [info.greater_mask[i] for i in range(nv)], "aut": int(info.aut)}
 
 
 class Context:
@@ -227,16 +253,7 @@ class Graph:
 
     def match(self, nv: int, edges, labels=None, induced: bool = False):
         """(count of distinct subgraphs, mappings = count * |Aut_L|)."""
-        e = np.ascontiguousarray(np.asarray(edges, dtype=np.uint32).reshape(-1))
-        p = N.gamma_pattern()
-        p.nv = nv
-        p.ne = e.size // 2
-        p.edges = e.ctypes.data_as(C.POINTER(C.c_uint32))
-        lab = None
-        if labels is not None:
-            lab = np.ascontiguousarray(labels, dtype=np.uint32)
-            p.labels = lab.ctypes.data_as(C.POINTER(C.c_uint32))
-        p.induced = 1 if induced else 0
+        p, keep = _pattern(nv, edges, labels, induced)
         c, mp = C.c_uint64(), C.c_uint64()
         _check(_lib.gamma_match(self._h, C.byref(p), C.byref(c), C.byref(mp)), "gamma_match")
         return int(c.value), int(mp.value)

@@ -49,6 +49,11 @@ class gamma_pattern(C.Structure):
                 ("labels", C.POINTER(C.c_uint32)), ("induced", C.c_int32)]
 
 
+class gamma_plan_info(C.Structure):
+    _fields_ = [("nv", C.c_uint32), ("order", C.c_uint32 * 8), ("backward_mask", C.c_uint32 * 8),
+                ("less_mask", C.c_uint32 * 8), ("greater_mask", C.c_uint32 * 8), ("aut", C.c_uint64)]
+
+
 class gamma_fpm_pattern(C.Structure):
     _fields_ = [("nv", C.c_uint32), ("ne", C.c_uint32), ("labels", C.c_uint32 * 8),
                 ("edges", (C.c_uint8 * 2) * 8), ("support", C.c_uint64)]
@@ -90,6 +95,7 @@ SIGNATURES = [
     ("gamma_graph_copy_csr", C.c_int32, [C.c_void_p, C.c_int, C.c_void_p, C.c_void_p]),
     ("gamma_kclique", C.c_int32, [C.c_void_p, C.c_uint32, C.POINTER(C.c_uint64)]),
     ("gamma_kclique_roots", C.c_int32, [C.c_void_p, C.c_uint32, C.c_uint64, C.c_void_p, C.c_void_p]),
+    ("gamma_pattern_plan", C.c_int32, [C.POINTER(gamma_pattern), C.POINTER(gamma_plan_info)]),
     ("gamma_match", C.c_int32, [C.c_void_p, C.POINTER(gamma_pattern), C.POINTER(C.c_uint64),
                                 C.POINTER(C.c_uint64)]),
     ("gamma_fpm", C.c_int32, [C.c_void_p, C.c_uint32, C.c_uint64, C.POINTER(C.POINTER(gamma_fpm_result))]),

@@ -70,6 +70,15 @@ __device__ __forceinline__ bool wb_reserve(WarpBlock &w, const BlockPool &p, uin
   return true;
 }
 
+// Group tables are read densely by the next level, so slots a warp abandons when
+// it moves to a fresh block must be marked empty first.  Call before wb_reserve;
+// empty(slot) writes the "empty group" marker of one slot.
+template <class F>
+__device__ __forceinline__ void wb_retire_tail(const WarpBlock &w, uint32_t f, int lane, F empty) {
+  if (w.b + f > w.e)
+    for (uint64_t s = w.b + lane; s < w.e; s += 32) empty(s);
+}
+
 // Reserve ub slots directly from the pool (outputs that may exceed a block).
 __device__ __forceinline__ bool pool_reserve(const BlockPool &p, uint64_t ub, int lane, uint64_t &pos) {
   unsigned long long nb = 0;

@@ -12,23 +12,30 @@
 //    C(P) = N+(p1) ∩ ... ∩ N+(pd) of a d-vertex prefix P, sorted ascending; every
 //    element c of the run is one (d+1)-vertex embedding and its own candidate run
 //    is C(P) ∩ N+(c).  So L_m of Opt 2 *is* the parent run: it is staged once per
-//    group in shared memory and every child's N+(c) is streamed from HBM with
-//    coalesced 128 B warp loads and probed against it (branch-free binary search),
-//    survivors compacted in order with __ballot_sync/__popc.
+//    group in shared memory and probed with a branch-free binary search.
+//  * Flattened children: a window of up to 32 children is held one per lane (list
+//    offset + length in registers, exclusive-scanned with shuffles); the warp then
+//    streams the concatenation of their DAG lists 32 elements per step, each lane
+//    finding its child by a 5-step shuffle search.  Lanes stay busy even when the
+//    lists are short (mean d+ ~ 8), and every step issues one coalesced gather.
+//  * Survivors are compacted in order with __ballot_sync/__popc into a per-warp
+//    shared staging buffer (child-major, so each child's run is contiguous); per-
+//    child hit counts come from ballot & segment masks, in registers.
 //  * ET level = column-first vid[] (4 B per embedding) + group table {beg,len}
-//    (8 B per non-empty group).  The parent pointer of the prefix tree is implicit
-//    in the group.
-//  * Opt 1: per-warp 16 KB vid blocks / 4 KB group blocks reserved with one atomic;
-//    a child's run is written contiguously from a shared-memory staging buffer.
-//  * A8: DFS over (depth, group range) with level buffers that grow geometrically up
-//    to the HBM budget; when a level still overflows, the producing range is split
-//    in halves (BFS inside a range, DFS across ranges).
+//    (8 B per kept group).  The parent pointer of the prefix tree is implicit in the
+//    group.
+//  * Opt 1: per-warp 16 KB vid blocks / 4 KB group blocks, one atomic per block.
+//  * Fused tail (DFS hybrid): at depth k-3 the children's runs never leave shared
+//    memory -- they are counted in place, so the largest ET level is never written.
+//  * A8: DFS over (depth, group range), level buffers grow geometrically up to an
+//    equal share of the HBM budget; a range that still overflows is split in halves.
 #include <cub/device/device_radix_sort.cuh>
 #include <cub/device/device_select.cuh>
 
 #include <algorithm>
 #include <vector>
 
+#include "device_common.cuh"
 #include "internal.cuh"
 
 namespace gamma_impl {
@@ -37,119 +44,184 @@ namespace {
 
 constexpr int kWarps = 8;
 constexpr int kThreads = kWarps * 32;
-constexpr uint32_t kRunCap = 1024;   // staged run capacity per warp (u32)
+constexpr uint32_t kRunCap = 512;    // staged run capacity per warp (u32)
+constexpr uint32_t kOutCap = 1024;   // staged output capacity per warp (u32), >= kRunCap
 constexpr uint32_t kBlkV = 4096;     // Opt 1 vid block per warp (16 KB)
 constexpr uint32_t kBlkG = 512;      // Opt 1 group block per warp (4 KB)
 
+enum { MODE_EXTEND = 0, MODE_COUNT = 1, MODE_FUSED = 2 };
+
 struct KclArgs {
-  // graph (DAG)
   const uint64_t *dag_ptr;
   const uint32_t *dag_col;
-  // input groups: depth-1 (roots) or a level table
-  const uint32_t *roots;      // depth 1
-  const uint2 *grp_in;        // depth >= 2: {beg, len}
-  const uint32_t *groot_in;   // depth >= 2, per-root mode: root index per group
+  // input groups: depth 1 (roots) or a level table
+  const uint32_t *roots;
+  const uint2 *grp_in;        // {beg, len}
+  const uint32_t *groot_in;   // per-root mode: root index per group
   const uint32_t *vid_in;
-  uint64_t g_begin, g_end;    // group range processed by this launch
+  uint64_t g_begin, g_end;
   uint32_t need_group;        // skip groups with len < need_group
-  uint32_t need_child;        // keep children whose new run has >= need_child entries
-  // output level (extend)
+  uint32_t need_child;        // keep children whose own run has >= need_child entries
+  // output level (extend; fused: long-run spill)
   uint32_t *vid_out;
   uint2 *grp_out;
   uint32_t *groot_out;
   uint64_t cap_v, cap_g;
-  // control + results
   unsigned long long *ctrl;
-  unsigned long long *per_root;  // per-root counts (nullable)
+  unsigned long long *per_root;
   uint32_t batch;
-  uint32_t stage_cap;         // kRunCap (0 under GAMMA_FLAG_DEBUG_NOSTAGE)
+  uint32_t stage_cap;         // kRunCap (0: GAMMA_FLAG_DEBUG_NOSTAGE)
 };
 
-__device__ __forceinline__ uint32_t lanemask_lt() {
-  uint32_t m;
-  asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
-  return m;
-}
-
-// Branch-free lower-bound membership test in a sorted array of len >= 1 entries.
-template <class P>
-__device__ __forceinline__ bool sorted_contains(P s, uint32_t len, uint32_t y) {
-  uint32_t base = 0, n = len;
-  while (n > 1) {
-    uint32_t half = n >> 1;
-    base = (s[base + half] <= y) ? base + half : base;
-    n -= half;
-  }
-  return s[base] == y;
-}
-
-struct WarpBlocks {
-  uint64_t vb = 0, ve = 0, gb = 0, ge = 0;
+struct Counters {
+  uint64_t acc = 0, in_entries = 0, elems = 0, out_entries = 0;
 };
 
-// Opt 1: reserve f contiguous vid slots from the warp's current block, taking a
-// fresh block from the pool when the block cannot hold them.  Warp-uniform.
-__device__ __forceinline__ bool reserve_v(WarpBlocks &w, uint32_t f, const KclArgs &a, int lane,
-                                          uint64_t &pos) {
-  if (w.vb + f > w.ve) {
-    unsigned long long nb = 0;
-    if (lane == 0) nb = atomicAdd(&a.ctrl[CTRL_VCUR], (unsigned long long)kBlkV);
-    nb = __shfl_sync(0xffffffffu, nb, 0);
-    if (nb + kBlkV > a.cap_v) {
-      if (lane == 0) atomicExch(&a.ctrl[CTRL_OVF], 1ull);
-      return false;
+__device__ __forceinline__ uint32_t excl_scan(uint32_t x, int lane, uint32_t &total) {
+  uint32_t s = x;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    uint32_t y = __shfl_up_sync(0xffffffffu, s, o);
+    if (lane >= o) s += y;
+  }
+  total = __shfl_sync(0xffffffffu, s, 31);
+  return s - x;
+}
+
+// Lanes [lo, hi) of a 32-lane tile, clamped.
+__device__ __forceinline__ uint32_t seg_mask(int64_t lo, int64_t hi) {
+  lo = lo < 0 ? 0 : (lo > 32 ? 32 : lo);
+  hi = hi < 0 ? 0 : (hi > 32 ? 32 : hi);
+  if (hi <= lo) return 0u;
+  uint32_t up = hi >= 32 ? 0xffffffffu : ((1u << hi) - 1u);
+  uint32_t dn = lo >= 32 ? 0xffffffffu : ((1u << lo) - 1u);
+  return up & ~dn;
+}
+
+// The window core: children = one per active lane (list offset `beg`, length `dl`,
+// exclusive offsets `o`, total T).  Streams the concatenated lists, probes every
+// element against the staged run, and (WRITE) compacts hits into `out` child-major
+// and accumulates per-child hit counts in `cnt`.  Returns the number of hits.
+template <bool WRITE>
+__device__ __forceinline__ uint32_t window_probe(const KclArgs &a, const uint32_t *__restrict__ run,
+                                                 uint32_t len, uint32_t rmin, uint32_t rmax, uint32_t beg,
+                                                 uint32_t dl, uint32_t o, uint32_t T, int lane,
+                                                 uint32_t *out, uint32_t &cnt) {
+  uint32_t found = 0;
+  for (uint32_t t0 = 0; t0 < T; t0 += 32) {
+    const uint32_t t = t0 + lane;
+    const bool valid = t < T;
+    // j = max{i : o_i <= t} over the window lanes (o is non-decreasing)
+    int j = 0;
+#pragma unroll
+    for (int step = 16; step > 0; step >>= 1) {
+      uint32_t oc = __shfl_sync(0xffffffffu, o, (j + step) & 31);
+      if (j + step < 32 && oc <= t) j += step;
     }
-    w.vb = nb;
-    w.ve = nb + kBlkV;
-  }
-  pos = w.vb;
-  w.vb += f;
-  return true;
-}
-
-// Direct reservation of ub slots (children whose run may exceed the staging buffer).
-__device__ __forceinline__ bool reserve_big(uint64_t ub, const KclArgs &a, int lane, uint64_t &pos) {
-  unsigned long long nb = 0;
-  if (lane == 0) nb = atomicAdd(&a.ctrl[CTRL_VCUR], (unsigned long long)ub);
-  nb = __shfl_sync(0xffffffffu, nb, 0);
-  if (nb + ub > a.cap_v) {
-    if (lane == 0) atomicExch(&a.ctrl[CTRL_OVF], 1ull);
-    return false;
-  }
-  pos = nb;
-  return true;
-}
-
-__device__ __forceinline__ bool reserve_g(WarpBlocks &w, const KclArgs &a, int lane, uint64_t &pos) {
-  if (w.gb == w.ge) {
-    unsigned long long nb = 0;
-    if (lane == 0) nb = atomicAdd(&a.ctrl[CTRL_GCUR], (unsigned long long)kBlkG);
-    nb = __shfl_sync(0xffffffffu, nb, 0);
-    if (nb + kBlkG > a.cap_g) {
-      if (lane == 0) atomicExch(&a.ctrl[CTRL_OVF], 1ull);
-      return false;
+    const uint32_t bj = __shfl_sync(0xffffffffu, beg, j);
+    const uint32_t oj = __shfl_sync(0xffffffffu, o, j);
+    const uint32_t y = valid ? __ldg(a.dag_col + bj + (t - oj)) : 0xffffffffu;
+    bool hit = false;
+    if (valid && y >= rmin && y <= rmax) hit = sorted_contains(run, len, y);
+    const uint32_t bal = __ballot_sync(0xffffffffu, hit);
+    if (WRITE) {
+      if (hit) out[found + __popc(bal & lanemask_lt())] = y;
+      cnt += __popc(bal & seg_mask((int64_t)o - t0, (int64_t)o + dl - t0));
     }
-    w.gb = nb;
-    w.ge = nb + kBlkG;
+    found += __popc(bal);
   }
-  pos = w.gb++;
+  return found;
+}
+
+// Load the window's children (lane i: child w0+i of the run) and their DAG lists.
+__device__ __forceinline__ void load_children(const KclArgs &a, const uint32_t *run, uint32_t len,
+                                              uint32_t w0, int lane, uint32_t need, uint32_t &beg,
+                                              uint32_t &dl, uint32_t &raw) {
+  const uint32_t i = w0 + lane;
+  beg = 0;
+  dl = 0;
+  raw = 0;
+  if (i < len) {
+    const uint32_t c = run[i];
+    const uint64_t b0 = a.dag_ptr[c];
+    raw = (uint32_t)(a.dag_ptr[c + 1] - b0);
+    beg = (uint32_t)b0;
+    dl = raw >= need ? raw : 0;
+  }
+}
+
+// Count k-cliques under one staged group at the last depth: sum over children c
+// of |run ∩ N+(c)|.
+__device__ __forceinline__ uint64_t count_staged(const KclArgs &a, const uint32_t *run, uint32_t len,
+                                                 int lane, Counters &ct) {
+  const uint32_t rmin = run[0], rmax = run[len - 1];
+  uint64_t total = 0;
+  for (uint32_t w0 = 0; w0 < len; w0 += 32) {
+    uint32_t beg, dl, raw, T, dummy = 0;
+    load_children(a, run, len, w0, lane, 1, beg, dl, raw);
+    ct.elems += raw;
+    const uint32_t o = excl_scan(dl, lane, T);
+    total += window_probe<false>(a, run, len, rmin, rmax, beg, dl, o, T, lane, nullptr, dummy);
+  }
+  return total;
+}
+
+// Long runs (len > stage capacity): child by child, probing the run in global
+// memory; EXTEND/FUSED write each kept child's run with a direct pool reservation.
+template <int MODE, bool PER_ROOT>
+__device__ bool process_unstaged(const KclArgs &a, const uint32_t *run, uint32_t len, uint32_t root_idx,
+                                 int lane, Counters &ct, WarpBlock &wg, uint64_t &gacc) {
+  const BlockPool pv{&a.ctrl[CTRL_VCUR], &a.ctrl[CTRL_OVF], a.cap_v, kBlkV};
+  const BlockPool pg{&a.ctrl[CTRL_GCUR], &a.ctrl[CTRL_OVF], a.cap_g, kBlkG};
+  const uint32_t rmin = run[0], rmax = run[len - 1];
+  const uint32_t need = (MODE == MODE_COUNT) ? 1u : a.need_child;
+  for (uint32_t i = 0; i < len; i++) {
+    const uint32_t c = run[i];
+    const uint64_t lb = a.dag_ptr[c];
+    const uint32_t dl = (uint32_t)(a.dag_ptr[c + 1] - lb);
+    ct.elems += (lane == 0) ? dl : 0;
+    if (dl < need) continue;
+    const uint32_t *lst = a.dag_col + lb;
+    const uint32_t ub = min(dl, len);
+    uint64_t pos = 0;
+    if (MODE != MODE_COUNT && !pool_reserve(pv, ub, lane, pos)) return false;
+    uint32_t found = 0;
+    for (uint32_t j = 0; j < dl; j += 32) {
+      const uint32_t y = (j + lane < dl) ? __ldg(lst + j + lane) : 0xffffffffu;
+      bool hit = false;
+      if (y >= rmin && y <= rmax) hit = sorted_contains(run, len, y);
+      const uint32_t bal = __ballot_sync(0xffffffffu, hit);
+      if (MODE != MODE_COUNT && hit) a.vid_out[pos + found + __popc(bal & lanemask_lt())] = y;
+      found += __popc(bal);
+      if (__shfl_sync(0xffffffffu, y, 31) > rmax) break;
+    }
+    if (MODE == MODE_COUNT) {
+      gacc += found;
+      continue;
+    }
+    if (found < a.need_child) continue;
+    uint64_t gpos;
+    if (!wb_reserve(wg, pg, 1, lane, gpos)) return false;
+    if (lane == 0) {
+      a.grp_out[gpos] = make_uint2((uint32_t)pos, found);
+      if (PER_ROOT) a.groot_out[gpos] = root_idx;
+    }
+    ct.out_entries += (lane == 0) ? found : 0;
+  }
   return true;
 }
 
-// One kernel body for both the extend step (COUNT=false: write the children's runs
-// as the next ET level) and the last step (COUNT=true: sum the run lengths, i.e.
-// the k-cliques, without writing).  ROOT: input groups are depth-1 (DAG lists of
-// the root vertices) instead of a level table.  PER_ROOT: attribute counts to the
-// root of each group (gamma_kclique_roots).
-template <bool COUNT, bool ROOT, bool PER_ROOT>
-__global__ void __launch_bounds__(kThreads) kcl_step_kernel(KclArgs a) {
-  extern __shared__ uint32_t smem[];   // kWarps x kRunCap run (+ kWarps x kRunCap out)
+template <int MODE, bool ROOT, bool PER_ROOT>
+__global__ void __launch_bounds__(kThreads) kcl_kernel(KclArgs a) {
+  extern __shared__ uint32_t smem[];
   const int lane = threadIdx.x & 31;
   const int wid = threadIdx.x >> 5;
   uint32_t *srun = smem + wid * kRunCap;
-  uint32_t *sout = smem + (kWarps + wid) * kRunCap;
-  WarpBlocks wb;
-  uint64_t acc = 0, in_entries = 0, elems = 0, out_entries = 0;
+  uint32_t *sout = smem + kWarps * kRunCap + wid * kOutCap;   // unused in MODE_COUNT
+  const BlockPool pv{&a.ctrl[CTRL_VCUR], &a.ctrl[CTRL_OVF], a.cap_v, kBlkV};
+  const BlockPool pg{&a.ctrl[CTRL_GCUR], &a.ctrl[CTRL_OVF], a.cap_g, kBlkG};
+  WarpBlock wv, wg;
+  Counters ct;
   const uint64_t ng = a.g_end - a.g_begin;
   bool stop = false;
 
@@ -158,7 +230,7 @@ __global__ void __launch_bounds__(kThreads) kcl_step_kernel(KclArgs a) {
     if (lane == 0) base = atomicAdd(&a.ctrl[CTRL_WORK], (unsigned long long)a.batch);
     base = __shfl_sync(0xffffffffu, base, 0);
     if (base >= ng) break;
-    if (!COUNT && *(volatile unsigned long long *)&a.ctrl[CTRL_OVF]) break;
+    if (MODE != MODE_COUNT && *(volatile unsigned long long *)&a.ctrl[CTRL_OVF]) break;
     const uint64_t bend = min((uint64_t)base + a.batch, ng);
     for (uint64_t gi = a.g_begin + base; gi < a.g_begin + bend && !stop; gi++) {
       // ---- A2/A3: the group's run C(P) ----
@@ -166,94 +238,105 @@ __global__ void __launch_bounds__(kThreads) kcl_step_kernel(KclArgs a) {
       uint32_t len;
       uint32_t root_idx = 0;
       if (ROOT) {
-        uint32_t v = a.roots[gi];
-        uint64_t b0 = a.dag_ptr[v];
+        const uint32_t v = a.roots[gi];
+        const uint64_t b0 = a.dag_ptr[v];
         len = (uint32_t)(a.dag_ptr[v + 1] - b0);
         run = a.dag_col + b0;
         root_idx = (uint32_t)gi;
       } else {
-        uint2 gd = a.grp_in[gi];
+        const uint2 gd = a.grp_in[gi];
         len = gd.y;
         run = a.vid_in + gd.x;
         if (PER_ROOT) root_idx = a.groot_in[gi];
       }
       if (len < a.need_group) continue;
-      in_entries += len;
-      const bool staged = len <= a.stage_cap;
-      if (staged) {
+      ct.in_entries += (lane == 0) ? len : 0;
+      uint64_t gacc = 0;
+      if (len > a.stage_cap) {
+        if (!process_unstaged<MODE, PER_ROOT>(a, run, len, root_idx, lane, ct, wg, gacc)) stop = true;
+      } else {
         for (uint32_t i = lane; i < len; i += 32) srun[i] = run[i];
         __syncwarp();
-      }
-      const uint32_t *probe = staged ? srun : run;
-      const uint32_t rmin = probe[0], rmax = probe[len - 1];
-      uint64_t gacc = 0;
-      // ---- A4-A6: every child c of the group ----
-      for (uint32_t i = 0; i < len; i++) {
-        const uint32_t c = probe[i];
-        const uint64_t lb = a.dag_ptr[c];
-        const uint32_t dl = (uint32_t)(a.dag_ptr[c + 1] - lb);
-        elems += dl;
-        if (dl < a.need_child) continue;
-        const uint32_t *lst = a.dag_col + lb;
-        const uint32_t ub = min(dl, len);
-        const bool big = !COUNT && ub > a.stage_cap;
-        uint64_t bigpos = 0;
-        if (big && !reserve_big(ub, a, lane, bigpos)) { stop = true; break; }
-        uint32_t found = 0;
-        for (uint32_t j = 0; j < dl; j += 32) {
-          const uint32_t y = (j + lane < dl) ? __ldg(lst + j + lane) : 0xffffffffu;
-          bool hit = false;
-          if (y >= rmin && y <= rmax) hit = staged ? sorted_contains(srun, len, y)
-                                                   : sorted_contains(run, len, y);
-          const uint32_t bal = __ballot_sync(0xffffffffu, hit);
-          if (!COUNT && hit) {
-            const uint32_t p = found + __popc(bal & lanemask_lt());
-            if (big) a.vid_out[bigpos + p] = y;
-            else sout[p] = y;
-          }
-          found += __popc(bal);
-          if (__shfl_sync(0xffffffffu, y, 31) > rmax) break;  // rest of N+(c) is > max C(P)
-        }
-        if (COUNT) {
-          gacc += found;
-          continue;
-        }
-        // A6: keep the child's run as a group of the next level
-        if (found < a.need_child) continue;
-        uint64_t pos;
-        if (big) {
-          pos = bigpos;
+        if (MODE == MODE_COUNT) {
+          gacc = count_staged(a, srun, len, lane, ct);
         } else {
-          __syncwarp();
-          if (!reserve_v(wb, found, a, lane, pos)) { stop = true; break; }
-          for (uint32_t t = lane; t < found; t += 32) a.vid_out[pos + t] = sout[t];
+          // ---- A4-A6: windows of children, outputs staged child-major ----
+          const uint32_t rmin = srun[0], rmax = srun[len - 1];
+          for (uint32_t w0 = 0; w0 < len && !stop;) {
+            uint32_t beg, dl, raw;
+            load_children(a, srun, len, w0, lane, a.need_child, beg, dl, raw);
+            // window = longest prefix of lanes whose output upper bounds fit kOutCap
+            uint32_t ub = min(dl, len), ubt;
+            const uint32_t ubx = excl_scan(ub, lane, ubt);
+            const bool fits = (w0 + lane < len) && (ubx + ub <= kOutCap);
+            const uint32_t nwin = __popc(__ballot_sync(0xffffffffu, fits));   // >= 1
+            const bool active = lane < (int)nwin;
+            if (!active) dl = 0;
+            ct.elems += active ? raw : 0;
+            uint32_t T;
+            const uint32_t o = excl_scan(dl, lane, T);
+            uint32_t cnt = 0;
+            const uint32_t found = window_probe<true>(a, srun, len, rmin, rmax, beg, dl, o, T, lane, sout, cnt);
+            __syncwarp();
+            uint32_t ctot;
+            const uint32_t s = excl_scan(cnt, lane, ctot);   // child i's run = sout[s, s+cnt)
+            const bool keep = active && cnt >= a.need_child;
+            const uint32_t kbal = __ballot_sync(0xffffffffu, keep);
+            if (MODE == MODE_EXTEND) {
+              if (kbal) {
+                uint64_t pos = 0, gpos = 0;
+                wb_retire_tail(wg, __popc(kbal), lane, [&](uint64_t s) { a.grp_out[s] = make_uint2(0, 0); });
+                if (!wb_reserve(wv, pv, found, lane, pos) || !wb_reserve(wg, pg, __popc(kbal), lane, gpos)) {
+                  stop = true;
+                  break;
+                }
+                for (uint32_t t = lane; t < found; t += 32) a.vid_out[pos + t] = sout[t];
+                if (keep) {
+                  const uint64_t gp = gpos + __popc(kbal & lanemask_lt());
+                  a.grp_out[gp] = make_uint2((uint32_t)(pos + s), cnt);
+                  if (PER_ROOT) a.groot_out[gp] = root_idx;
+                }
+                ct.out_entries += (lane == 0) ? found : 0;
+              }
+            } else {   // MODE_FUSED: count each kept child's run in place
+              uint32_t rem = kbal;
+              while (rem) {
+                const int i = __ffs(rem) - 1;
+                rem &= rem - 1;
+                const uint32_t si = __shfl_sync(0xffffffffu, s, i);
+                const uint32_t ci = __shfl_sync(0xffffffffu, cnt, i);
+                gacc += count_staged(a, sout + si, ci, lane, ct);
+              }
+            }
+            __syncwarp();
+            w0 += nwin;
+          }
         }
-        uint64_t gpos;
-        if (!reserve_g(wb, a, lane, gpos)) { stop = true; break; }
-        if (lane == 0) {
-          a.grp_out[gpos] = make_uint2((uint32_t)pos, found);
-          if (PER_ROOT) a.groot_out[gpos] = root_idx;
-        }
-        out_entries += found;
         __syncwarp();
       }
-      acc += gacc;
-      if (PER_ROOT && COUNT && lane == 0 && gacc) atomicAdd(&a.per_root[root_idx], (unsigned long long)gacc);
-      __syncwarp();
+      ct.acc += gacc;
+      if (PER_ROOT && lane == 0 && gacc) atomicAdd(&a.per_root[root_idx], (unsigned long long)gacc);
     }
   }
   // unused group slots of this warp's last block become empty groups
-  if (!COUNT)
-    for (uint64_t s = wb.gb + lane; s < wb.ge; s += 32) a.grp_out[s] = make_uint2(0, 0);
+  if (MODE != MODE_COUNT)
+    for (uint64_t s = wg.b + lane; s < wg.e; s += 32) a.grp_out[s] = make_uint2(0, 0);
+  // counters: lane-partial sums -> one atomic per warp
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) {
+    ct.elems += __shfl_down_sync(0xffffffffu, ct.elems, off);
+    ct.in_entries += __shfl_down_sync(0xffffffffu, ct.in_entries, off);
+    ct.out_entries += __shfl_down_sync(0xffffffffu, ct.out_entries, off);
+  }
   if (lane == 0) {
-    if (COUNT && acc) atomicAdd(&a.ctrl[CTRL_COUNT], (unsigned long long)acc);
-    atomicAdd(&a.ctrl[CTRL_AUX0], (unsigned long long)in_entries);
-    atomicAdd(&a.ctrl[CTRL_ELEMS], (unsigned long long)elems);
-    if (!COUNT) atomicAdd(&a.ctrl[CTRL_ENTRIES], (unsigned long long)out_entries);
+    if (ct.acc) atomicAdd(&a.ctrl[CTRL_COUNT], (unsigned long long)ct.acc);
+    atomicAdd(&a.ctrl[CTRL_AUX0], (unsigned long long)ct.in_entries);
+    atomicAdd(&a.ctrl[CTRL_ELEMS], (unsigned long long)ct.elems);
+    atomicAdd(&a.ctrl[CTRL_ENTRIES], (unsigned long long)ct.out_entries);
   }
 }
 
-// A2: roots = vertices with d+(v) >= need, cost key for heavy-first ordering.
+// ---- A2: roots = vertices with d+(v) >= k-1, heavy first, snake-partitioned ----
 struct RootNeed {
   const uint64_t *dag_ptr;
   uint32_t need;
@@ -272,8 +355,8 @@ __global__ void root_cost_kernel(const uint64_t *dag_ptr, const uint32_t *roots,
                                  uint64_t *cost) {
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < nr;
        i += (uint64_t)gridDim.x * blockDim.x) {
-    uint32_t v = roots[i];
-    uint64_t d = dag_ptr[v + 1] - dag_ptr[v];
+    const uint32_t v = roots[i];
+    const uint64_t d = dag_ptr[v + 1] - dag_ptr[v];
     cost[i] = d * d;
   }
 }
@@ -283,7 +366,7 @@ __global__ void root_cost_kernel(const uint64_t *dag_ptr, const uint32_t *roots,
 __global__ void rank_flag_kernel(uint64_t nr, uint32_t rank, uint32_t world, uint8_t *flag) {
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < nr;
        i += (uint64_t)gridDim.x * blockDim.x) {
-    uint64_t r = i % (2ull * world);
+    const uint64_t r = i % (2ull * world);
     flag[i] = (r == rank || r == 2ull * world - 1 - rank) ? 1 : 0;
   }
 }
@@ -292,7 +375,7 @@ __global__ void degree_count_kernel(const uint64_t *dag_ptr, const uint32_t *roo
                                     uint32_t k, unsigned long long *out) {
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < nr;
        i += (uint64_t)gridDim.x * blockDim.x) {
-    uint32_t v = roots[i];
+    const uint32_t v = roots[i];
     out[i] = (k == 1) ? 1ull : (unsigned long long)(dag_ptr[v + 1] - dag_ptr[v]);
   }
 }
@@ -303,28 +386,22 @@ inline unsigned grid1d(uint64_t n, int threads = 256) {
   return (unsigned)std::min<uint64_t>(b, 148u * 32u);
 }
 
-constexpr size_t step_smem(bool count) {
-  return (count ? 1 : 2) * (size_t)kWarps * kRunCap * sizeof(uint32_t);
+constexpr size_t kcl_smem(int mode) {
+  return (size_t)kWarps * (kRunCap + (mode == MODE_COUNT ? 0 : kOutCap)) * sizeof(uint32_t);
 }
 
-template <bool COUNT, bool ROOT, bool PER_ROOT>
+template <int MODE, bool ROOT, bool PER_ROOT>
 void set_smem_attr() {
-  GAMMA_CUDA(cudaFuncSetAttribute(kcl_step_kernel<COUNT, ROOT, PER_ROOT>,
-                                  cudaFuncAttributeMaxDynamicSharedMemorySize, (int)step_smem(COUNT)));
+  GAMMA_CUDA(cudaFuncSetAttribute(kcl_kernel<MODE, ROOT, PER_ROOT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                  (int)kcl_smem(MODE)));
 }
 
-void configure_kernels() {
-  static bool done = false;   // per process; attributes are per function
-  if (done) return;
-  set_smem_attr<false, false, false>();
-  set_smem_attr<false, false, true>();
-  set_smem_attr<false, true, false>();
-  set_smem_attr<false, true, true>();
-  set_smem_attr<true, false, false>();
-  set_smem_attr<true, false, true>();
-  set_smem_attr<true, true, false>();
-  set_smem_attr<true, true, true>();
-  done = true;
+template <int MODE>
+void set_mode_attrs() {
+  set_smem_attr<MODE, false, false>();
+  set_smem_attr<MODE, false, true>();
+  set_smem_attr<MODE, true, false>();
+  set_smem_attr<MODE, true, true>();
 }
 
 struct Level {
@@ -339,149 +416,161 @@ struct KclRun {
   gamma_ctx *ctx;
   uint32_t k;
   bool per_root;
+  bool fuse;
   const uint32_t *roots;
   uint64_t nroots;
   unsigned long long *per_root_out;
   std::vector<Level> levels;   // levels[d] holds groups at depth d (d >= 2)
-  uint64_t budget;             // bytes for all level tables
+  uint64_t level_share;        // bytes allowed per level table
   uint64_t total = 0;
-  int grid_extend = 0, grid_count = 0;
+  int grid[3] = {0, 0, 0};
 
-  uint64_t level_bytes(uint64_t cv, uint64_t cg) const {
-    return cv * 4 + cg * (per_root ? 12 : 8);
-  }
-  uint64_t used_bytes() const {
-    uint64_t s = 0;
-    for (auto &l : levels) s += level_bytes(l.cap_v, l.cap_g);
-    return s;
-  }
+  uint64_t bytes_per_slot() const { return 4 + (per_root ? 12 : 8) / 2; }   // vid + cap_g = cap_v/2
 
-  void ensure_level(uint32_t d, uint64_t want_v) {
+  // Grow level d to hold want_v vid slots, within its share of the budget.
+  bool grow_level(uint32_t d, uint64_t want_v) {
     Level &L = levels[d];
-    if (L.cap_v >= want_v) return;
-    uint64_t cv = std::max<uint64_t>(want_v, 1ull << 20);
-    cv = std::min<uint64_t>(cv, 0xFFFFFFFFull - kBlkV);  // beg is u32
-    uint64_t cg = cv / 2 + kBlkG * 1024;
-    uint64_t others = used_bytes() - level_bytes(L.cap_v, L.cap_g);
-    if (others + level_bytes(cv, cg) > budget) {
-      // shrink to what the budget allows (at least one block per warp)
-      uint64_t avail = budget > others ? budget - others : 0;
-      cv = avail / (4 + (per_root ? 12 : 8) / 2);
-      cg = cv / 2;
-      if (cv <= L.cap_v) return;  // cannot grow
-    }
-    L.vid.reset(); L.grp.reset(); L.groot.reset();
+    uint64_t cv = std::max<uint64_t>(want_v, 1ull << 16);
+    cv = std::min<uint64_t>(cv, level_share / bytes_per_slot());
+    cv = std::min<uint64_t>(cv, 0xFFFFFFFFull - kBlkV);   // group beg is u32
+    if (cv <= L.cap_v) return false;
+    const uint64_t cg = cv / 2 + kBlkG;
+    L.vid.reset();
+    L.grp.reset();
+    L.groot.reset();
     L.vid = DevBuf<uint32_t>(ctx, cv);
     L.grp = DevBuf<uint2>(ctx, cg);
     if (per_root) L.groot = DevBuf<uint32_t>(ctx, cg);
     L.cap_v = cv;
     L.cap_g = cg;
+    return true;
   }
 
-  KclArgs base_args() const {
+  KclArgs args_for(uint32_t d, uint64_t g0, uint64_t g1) const {
     KclArgs a{};
     a.dag_ptr = g->dag_ptr;
     a.dag_col = g->dag_col;
     a.ctrl = (unsigned long long *)ctx->ctrl;
     a.per_root = per_root_out;
     a.stage_cap = (ctx->desc.flags & GAMMA_FLAG_DEBUG_NOSTAGE) ? 0u : kRunCap;
-    return a;
-  }
-
-  void fill_input(KclArgs &a, uint32_t d, uint64_t g0, uint64_t g1) const {
     a.g_begin = g0;
     a.g_end = g1;
     if (d == 1) {
       a.roots = roots;
-      a.batch = 4;
+      a.batch = 2;
     } else {
       const Level &L = levels[d];
       a.grp_in = L.grp.p;
       a.groot_in = L.groot.p;
       a.vid_in = L.vid.p;
-      a.batch = 32;
+      a.batch = 16;
     }
-    a.need_group = k - d;   // a depth-d group needs k-d more vertices
+    a.need_group = k - d;        // a depth-d group needs k-d more vertices
+    a.need_child = k - d - 1;    // a child's run is a depth-(d+1) group
+    return a;
   }
 
-  template <bool COUNT, bool ROOT>
-  void launch_step(const KclArgs &a, int grid) {
-    int kc = COUNT ? KC_COUNT : KC_EXTEND;
-    const size_t smem = step_smem(COUNT);
+  void set_output(KclArgs &a, uint32_t nd) {
+    Level &L = levels[nd];
+    a.vid_out = L.vid.p;
+    a.grp_out = L.grp.p;
+    a.groot_out = L.groot.p;
+    a.cap_v = L.cap_v;
+    a.cap_g = L.cap_g;
+  }
+
+  template <int MODE, bool ROOT>
+  void launch_t(const KclArgs &a, int grid_) {
+    const int kc = MODE == MODE_EXTEND ? KC_EXTEND : (MODE == MODE_COUNT ? KC_COUNT : KC_FUSED);
+    const size_t smem = kcl_smem(MODE);
     ctx->launch(kc, [&] {
       if (per_root)
-        kcl_step_kernel<COUNT, ROOT, true><<<grid, kThreads, smem, ctx->stream>>>(a);
+        kcl_kernel<MODE, ROOT, true><<<grid_, kThreads, smem, ctx->stream>>>(a);
       else
-        kcl_step_kernel<COUNT, ROOT, false><<<grid, kThreads, smem, ctx->stream>>>(a);
+        kcl_kernel<MODE, ROOT, false><<<grid_, kThreads, smem, ctx->stream>>>(a);
     });
   }
 
-  // Count the k-cliques under depth-(k-2)... i.e. groups at depth d = k-1 are the
-  // k-cliques; the last step reads depth k-2 groups and sums child run lengths.
-  void count_range(uint32_t d, uint64_t g0, uint64_t g1) {
-    KclArgs a = base_args();
-    fill_input(a, d, g0, g1);
-    a.need_child = 1;
+  template <int MODE>
+  void launch(const KclArgs &a, uint32_t d, uint64_t cap_v) {
+    int gr = grid[MODE];
+    if (MODE == MODE_EXTEND) {   // keep the Opt 1 block waste below half the level
+      const uint64_t warps_ok = std::max<uint64_t>(1, cap_v / (2ull * kBlkV));
+      gr = (int)std::max<uint64_t>(1, std::min<uint64_t>(gr, warps_ok / kWarps));
+    }
     ctrl_reset(ctx);
-    if (d == 1) launch_step<true, true>(a, grid_count);
-    else launch_step<true, false>(a, grid_count);
+    if (d == 1) launch_t<MODE, true>(a, gr);
+    else launch_t<MODE, false>(a, gr);
     ctrl_fetch(ctx);
-    const uint64_t *h = ctx->ctrl_host;
-    total = checked_add(total, h[CTRL_COUNT]);
+  }
+
+  void account(int kc, uint32_t d, const uint64_t *h, bool wrote) {
     if (d == 1) ctx->stats.level_entries[2] += h[CTRL_AUX0];
-    ctx->stats.level_entries[k] = checked_add(ctx->stats.level_entries[k], h[CTRL_COUNT]);
     ctx->stats.list_elems += h[CTRL_ELEMS];
-    ctx->stats.alg_bytes[KC_COUNT] += 12 * h[CTRL_AUX0] + 4 * h[CTRL_ELEMS];
+    ctx->stats.alg_bytes[kc] += 12 * h[CTRL_AUX0] + 4 * h[CTRL_ELEMS] + (wrote ? 8 * h[CTRL_ENTRIES] : 0);
+  }
+
+  void add_count(uint64_t c) {
+    total = checked_add(total, c);
+    ctx->stats.level_entries[k] = checked_add(ctx->stats.level_entries[k], c);
   }
 
   // DFS over (depth, group range); BFS inside the range.
   void process(uint32_t d, uint64_t g0, uint64_t g1) {
     if (g0 >= g1) return;
-    if (d == k - 2) {
-      count_range(d, g0, g1);
+    if (d == k - 2) {   // last extension: count, do not store
+      KclArgs a = args_for(d, g0, g1);
+      a.need_child = 1;
+      launch<MODE_COUNT>(a, d, 0);
+      const uint64_t *h = ctx->ctrl_host;
+      add_count(h[CTRL_COUNT]);
+      account(KC_COUNT, d, h, false);
       return;
     }
+    const bool fused = fuse && d == k - 3;
     const uint32_t nd = d + 1;
-    for (int attempt = 0;; attempt++) {
+    for (;;) {
       Level &L = levels[nd];
-      if (L.cap_v == 0) ensure_level(nd, 1ull << 24);
-      KclArgs a = base_args();
-      fill_input(a, d, g0, g1);
-      a.need_child = k - d - 1;  // the child's run is a depth-(d+1) group
-      a.vid_out = L.vid.p;
-      a.grp_out = L.grp.p;
-      a.groot_out = L.groot.p;
-      a.cap_v = L.cap_v;
-      a.cap_g = L.cap_g;
-      ctrl_reset(ctx);
-      if (d == 1) launch_step<false, true>(a, grid_extend);
-      else launch_step<false, false>(a, grid_extend);
-      ctrl_fetch(ctx);
+      if (L.cap_v == 0)
+        grow_level(nd, fused ? (1ull << 18)
+                             : std::max<uint64_t>(1ull << 24, 4ull * kBlkV * kWarps * (uint64_t)grid[MODE_EXTEND]));
+      KclArgs a = args_for(d, g0, g1);
+      set_output(a, nd);
+      if (fused) launch<MODE_FUSED>(a, d, L.cap_v);
+      else launch<MODE_EXTEND>(a, d, L.cap_v);
       const uint64_t *h = ctx->ctrl_host;
       if (!h[CTRL_OVF]) {
-        if (d == 1) ctx->stats.level_entries[2] += h[CTRL_AUX0];
-        ctx->stats.level_entries[nd + 1] += h[CTRL_ENTRIES];
-        ctx->stats.list_elems += h[CTRL_ELEMS];
-        ctx->stats.alg_bytes[KC_EXTEND] += 12 * h[CTRL_AUX0] + 4 * h[CTRL_ELEMS] + 8 * h[CTRL_ENTRIES];
+        const uint64_t cnt = h[CTRL_COUNT];
+        const uint64_t ent = h[CTRL_ENTRIES];
+        const uint64_t ng = std::min<uint64_t>(h[CTRL_GCUR], L.cap_g);
+        account(fused ? KC_FUSED : KC_EXTEND, d, h, !fused || ent > 0);
         ctx->stats.chunks++;
-        uint64_t ng = std::min<uint64_t>(h[CTRL_GCUR], L.cap_g);
+        if (fused) add_count(cnt);
+        else ctx->stats.level_entries[nd + 1] += ent;
+        // fused: only long-run (unstaged) children were written; count them now
         process(nd, 0, ng);
         return;
       }
-      // overflow: grow the level if the budget allows, else split the range
       ctx->stats.retries++;
-      uint64_t before = L.cap_v;
-      ensure_level(nd, std::max<uint64_t>(h[CTRL_VCUR], L.cap_v) * 4);
-      if (levels[nd].cap_v > before) continue;
+      if (grow_level(nd, std::max<uint64_t>(h[CTRL_VCUR], L.cap_v) * 4)) continue;
       GAMMA_REQUIRE(g1 - g0 > 1, GAMMA_E_NOMEM,
                     "HBM budget too small for the children of a single embedding group");
-      uint64_t mid = g0 + (g1 - g0) / 2;
+      const uint64_t mid = g0 + (g1 - g0) / 2;
       process(d, g0, mid);
       process(d, mid, g1);
       return;
     }
   }
 };
+
+void configure_kernels() {
+  static bool done = false;   // function attributes persist for the process
+  if (done) return;
+  set_mode_attrs<MODE_EXTEND>();
+  set_mode_attrs<MODE_COUNT>();
+  set_mode_attrs<MODE_FUSED>();
+  done = true;
+}
 
 }  // namespace
 
@@ -490,17 +579,21 @@ uint64_t kclique_count(gamma_graph *g, uint32_t k, const uint32_t *roots_dev, ui
   gamma_ctx *ctx = g->ctx;
   const bool per_root = per_root_dev != nullptr;
   if (!per_root && ctx->desc.world <= 1 && k <= 2) return k == 1 ? g->n : g->m;
+  GAMMA_REQUIRE(g->m < 0xFFFFFFFFull, GAMMA_E_UNSUPPORTED, "DAG with >= 2^32 edges");
   KclRun R;
   R.g = g;
   R.ctx = ctx;
   R.k = k;
   R.per_root = per_root;
+  R.fuse = (ctx->desc.flags & GAMMA_FLAG_NO_FUSE) == 0;
   R.per_root_out = (unsigned long long *)per_root_dev;
   R.levels.resize(k + 1);
   {
     size_t fr = 0, tot = 0;
     GAMMA_CUDA(cudaMemGetInfo(&fr, &tot));
-    R.budget = ctx->desc.hbm_budget_bytes ? ctx->desc.hbm_budget_bytes : (uint64_t)(fr * 0.8);
+    const uint64_t budget = ctx->desc.hbm_budget_bytes ? ctx->desc.hbm_budget_bytes : (uint64_t)(fr * 0.8);
+    const uint64_t stored = k >= 4 ? k - 3 : 1;   // level tables at depths 2 .. k-2
+    R.level_share = budget / stored;
   }
   // ---- A2: root list ----
   DevBuf<uint32_t> root_buf;
@@ -525,10 +618,9 @@ uint64_t kclique_count(gamma_graph *g, uint32_t k, const uint32_t *roots_dev, ui
     uint64_t nr = 0;
     GAMMA_CUDA(cudaMemcpyAsync(&nr, nsel.p, sizeof(uint64_t), cudaMemcpyDeviceToHost, ctx->stream));
     ctx->sync();
-    // heavy-first: sort by cost descending
     DevBuf<uint64_t> cost(ctx, nr ? nr : 1), cost2(ctx, nr ? nr : 1);
     root_buf = DevBuf<uint32_t>(ctx, nr ? nr : 1);
-    if (nr) {
+    if (nr) {   // heavy first: sort by cost descending
       ctx->launch(KC_ROOTS, [&] {
         root_cost_kernel<<<grid1d(nr), 256, 0, ctx->stream>>>(g->dag_ptr, sel.p, nr, cost.p);
       });
@@ -567,8 +659,7 @@ uint64_t kclique_count(gamma_graph *g, uint32_t k, const uint32_t *roots_dev, ui
     R.nroots = nr;
   }
   ctx->stats.level_entries[1] = R.nroots;
-  if (k <= 2) {
-    // per-root (or partitioned) k=1 / k=2: each root contributes 1 / d+(v)
+  if (k <= 2) {   // per-root or partitioned k = 1 / 2: each root contributes 1 / d+(v)
     if (R.nroots == 0) return 0;
     DevBuf<unsigned long long> tmpc(ctx, R.nroots);
     unsigned long long *out = per_root ? (unsigned long long *)per_root_dev : tmpc.p;
@@ -584,10 +675,12 @@ uint64_t kclique_count(gamma_graph *g, uint32_t k, const uint32_t *roots_dev, ui
     return s;
   }
   configure_kernels();
-  R.grid_extend = ctx->num_sms * occupancy_blocks((const void *)kcl_step_kernel<false, false, false>, kThreads,
-                                                  step_smem(false));
-  R.grid_count = ctx->num_sms * occupancy_blocks((const void *)kcl_step_kernel<true, false, false>, kThreads,
-                                                 step_smem(true));
+  R.grid[MODE_EXTEND] = ctx->num_sms * occupancy_blocks((const void *)kcl_kernel<MODE_EXTEND, false, false>,
+                                                        kThreads, kcl_smem(MODE_EXTEND));
+  R.grid[MODE_COUNT] = ctx->num_sms * occupancy_blocks((const void *)kcl_kernel<MODE_COUNT, false, false>,
+                                                       kThreads, kcl_smem(MODE_COUNT));
+  R.grid[MODE_FUSED] = ctx->num_sms * occupancy_blocks((const void *)kcl_kernel<MODE_FUSED, false, false>,
+                                                       kThreads, kcl_smem(MODE_FUSED));
   if (R.nroots) R.process(1, 0, R.nroots);
   ctx->sync();
   ctx->collect_timings();

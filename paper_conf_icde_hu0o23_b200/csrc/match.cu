@@ -1,26 +1,719 @@
-// match.cu -- subgraph matching (Alg. 1) -- placeholder until the SM path lands.
+// match.cu -- subgraph matching, Alg. 1 (WOJ, query-vertex-at-a-time vertex
+// extension + filtering), non-induced, labeled, counting
+// distinct subgraphs (readings R4-R6, R10).
+//
+// Host planner:
+//  * matching order delta_v (PAPER.md L176 leaves it open; reading R10): the
+//    max-degree query vertex first, then repeatedly the vertex with the most
+//    already-placed neighbours (ties: higher degree, then lower id);
+//  * Aut_L(P) by brute force over nv! permutations;
+//  * symmetry breaking by a stabilizer chain along the matching order: for each
+//    placed vertex v, phi(v) < phi(u) for every u != v in v's orbit under the
+//    stabilizer of the earlier vertices.  Each automorphism class of mappings then
+//    has exactly one representative, so constrained count = mappings / |Aut_L|.
+//
+// Device (per extension depth d -> d+1, one warp per group):
+//  * a group = a d-vertex prefix phi_0..phi_{d-1} + a run of valid candidates for
+//    position d (the children); the descriptor carries the prefix, so no parent
+//    pointers are chased (the prefix tree of PAPER.md L253 is stored per group);
+//  * Opt 2: L_m = the intersection of the backward-neighbour lists that do not
+//    involve the child (the prefix part) is computed once per group, filtered by
+//    label/order/injectivity, and staged in shared memory; every child then probes
+//    only its own list against it;
+//  * filters ("pruning and label checking at run-time"): label,
+//    degree >= pattern degree, injectivity, symmetry order;
+//  * children with long runs are sliced into several groups (hub load balance);
+//  * last position: counted, not stored.
+#include <cub/device/device_radix_sort.cuh>
+#include <cub/device/device_select.cuh>
+
+#include <algorithm>
+#include <cstring>
+#include <vector>
+
+#include "device_common.cuh"
 #include "internal.cuh"
 
+namespace gamma_impl {
+
+namespace {
+
+constexpr int kMaxV = 8;
+constexpr int kWarps = 8;
+constexpr int kThreads = kWarps * 32;
+constexpr uint32_t kLmCap = 1024;    // staged L_m per warp (u32)
+constexpr uint32_t kOutCap = 1024;   // staged child run per warp (u32)
+constexpr uint32_t kBlkV = 4096;
+constexpr uint32_t kBlkG = 256;      // descriptors per warp block
+constexpr uint32_t kSlice = 64;      // children per group descriptor
+constexpr uint32_t kRootChunk = 16;  // roots per depth-0 group
+
+struct SmPlan {
+  uint32_t nv, labeled;
+  uint32_t order[kMaxV];
+  uint32_t label[kMaxV];    // per position
+  uint32_t mindeg[kMaxV];   // per position
+  uint32_t bmask[kMaxV];    // backward-neighbour positions
+  uint32_t injmask[kMaxV];  // earlier non-neighbour positions (x != phi_j)
+  uint32_t ltmask[kMaxV];   // earlier positions j with phi_j < x
+  uint32_t gtmask[kMaxV];   // earlier positions j with x < phi_j
+  uint64_t aut;
+};
+
+struct SmArgs {
+  const uint64_t *rp;
+  const uint32_t *col;
+  const uint32_t *lab;      // nullable (unlabeled graph: all 0)
+  SmPlan P;
+  uint32_t d;               // children are at position d; extend to q = d+1
+  const uint32_t *vid_in;
+  const uint32_t *desc_in;  // dw_in words per group: beg, len, phi_0..phi_{d-1}
+  uint32_t dw_in;
+  uint64_t g_begin, g_end;
+  uint32_t *vid_out;
+  uint32_t *desc_out;
+  uint32_t dw_out;
+  uint64_t cap_v, cap_g;
+  unsigned long long *ctrl;
+  uint32_t batch;
+  uint32_t stage;           // 0: never stage L_m (debug)
+};
+
+__device__ __forceinline__ uint32_t gdeg(const SmArgs &a, uint32_t v) {
+  return (uint32_t)(a.rp[v + 1] - a.rp[v]);
+}
+
+struct Bounds {
+  int64_t lo;     // x > lo
+  uint32_t hi;    // x < hi (0xffffffff: none)
+  uint32_t inj;   // positions to check x != phi_j
+};
+
+// Candidate filter for position q.
+__device__ __forceinline__ bool sm_filter(const SmArgs &a, uint32_t q, uint32_t x, const Bounds &b,
+                                          const uint32_t *phi, bool last) {
+  if ((int64_t)x <= b.lo || x >= b.hi) return false;
+  if (a.P.labeled) {
+    const uint32_t lx = a.lab ? a.lab[x] : 0u;
+    if (lx != a.P.label[q]) return false;
+  }
+  uint32_t m = b.inj;
+  while (m) {
+    const int j = __ffs(m) - 1;
+    m &= m - 1;
+    if (phi[j] == x) return false;
+  }
+  if (!last && a.P.mindeg[q] > 1 && gdeg(a, x) < a.P.mindeg[q]) return false;
+  return true;
+}
+
+__device__ __forceinline__ Bounds bounds_for(const SmArgs &a, uint32_t q, uint32_t avail, const uint32_t *phi) {
+  Bounds b{-1, 0xffffffffu, a.P.injmask[q] & avail};
+  uint32_t m = a.P.ltmask[q] & avail;
+  while (m) {
+    const int j = __ffs(m) - 1;
+    m &= m - 1;
+    b.lo = max(b.lo, (int64_t)phi[j]);
+  }
+  m = a.P.gtmask[q] & avail;
+  while (m) {
+    const int j = __ffs(m) - 1;
+    m &= m - 1;
+    b.hi = min(b.hi, phi[j]);
+  }
+  return b;
+}
+
+// Intersect the lists N(phi_j), j in `lists`, with filters; results (sorted) go to
+// out[] (if WRITE and they fit in cap) or are only counted.  The shortest list
+// drives; the others are probed by binary search.  Returns the number of results,
+// or UINT32_MAX if WRITE and the results overflow cap.
+template <bool WRITE>
+__device__ uint32_t sm_intersect(const SmArgs &a, uint32_t q, uint32_t lists, const uint32_t *phi,
+                                 const Bounds &bd, bool last, const uint32_t *lm, uint32_t lm_len,
+                                 uint32_t *out, uint32_t cap, int lane) {
+  // choose the driver: L_m (shared memory) counts as a list when given
+  uint32_t best_len = 0xffffffffu, best = 0xffffffffu;
+  uint32_t m = lists;
+  while (m) {
+    const int j = __ffs(m) - 1;
+    m &= m - 1;
+    const uint32_t dl = gdeg(a, phi[j]);
+    if (dl < best_len) { best_len = dl; best = j; }
+  }
+  const bool drive_lm = lm != nullptr && lm_len <= best_len;
+  const uint32_t *drv;
+  uint32_t dlen;
+  if (drive_lm) {
+    drv = lm;
+    dlen = lm_len;
+  } else {
+    drv = a.col + a.rp[phi[best]];
+    dlen = best_len;
+  }
+  const uint32_t probes = drive_lm ? lists : (lists & ~(1u << best));
+  // skip driver entries <= lo (sorted)
+  uint32_t start = 0;
+  if (bd.lo >= 0 && dlen) start = upper_bound_idx(drv, dlen, (uint32_t)bd.lo);
+  uint32_t found = 0;
+  for (uint32_t j0 = start; j0 < dlen; j0 += 32) {
+    const uint32_t jj = j0 + lane;
+    const uint32_t x = jj < dlen ? drv[jj] : 0xffffffffu;
+    bool ok = jj < dlen && sm_filter(a, q, x, bd, phi, last);
+    if (ok && lm && !drive_lm) ok = sorted_contains(lm, lm_len, x);
+    uint32_t pm = probes;
+    while (ok && pm) {
+      const int j = __ffs(pm) - 1;
+      pm &= pm - 1;
+      const uint64_t s = a.rp[phi[j]];
+      const uint32_t l = (uint32_t)(a.rp[phi[j] + 1] - s);
+      ok = l > 0 && sorted_contains(a.col + s, l, x);
+    }
+    const uint32_t bal = __ballot_sync(0xffffffffu, ok);
+    if (WRITE && ok) {
+      const uint32_t p = found + __popc(bal & lanemask_lt());
+      if (p < cap) out[p] = x;
+    }
+    found += __popc(bal);
+    if (__shfl_sync(0xffffffffu, x, 31) >= bd.hi) break;   // driver is sorted
+  }
+  if (WRITE && found > cap) return 0xffffffffu;
+  return found;
+}
+
+__global__ void __launch_bounds__(kThreads) sm_kernel(SmArgs a) {
+  extern __shared__ uint32_t smem[];
+  const int lane = threadIdx.x & 31;
+  const int wid = threadIdx.x >> 5;
+  uint32_t *slm = smem + wid * (kLmCap + kOutCap);
+  uint32_t *sout = slm + kLmCap;
+  const uint32_t d = a.d, q = d + 1;
+  const bool last = q == a.P.nv - 1;
+  const BlockPool pv{&a.ctrl[CTRL_VCUR], &a.ctrl[CTRL_OVF], a.cap_v, kBlkV};
+  const BlockPool pg{&a.ctrl[CTRL_GCUR], &a.ctrl[CTRL_OVF], a.cap_g, kBlkG};
+  WarpBlock wv, wg;
+  uint64_t acc = 0, in_entries = 0, out_entries = 0;
+  const uint64_t ng = a.g_end - a.g_begin;
+  bool stop = false;
+  const uint32_t prefix_mask = (1u << d) - 1u;
+  const uint32_t bq = a.P.bmask[q];
+  const uint32_t bshared = bq & prefix_mask;
+  const bool child_in_b = (bq >> d) & 1u;
+
+  while (!stop) {
+    unsigned long long base = 0;
+    if (lane == 0) base = atomicAdd(&a.ctrl[CTRL_WORK], (unsigned long long)a.batch);
+    base = __shfl_sync(0xffffffffu, base, 0);
+    if (base >= ng) break;
+    if (!last && *(volatile unsigned long long *)&a.ctrl[CTRL_OVF]) break;
+    const uint64_t bend = min((uint64_t)base + a.batch, ng);
+    for (uint64_t gi = a.g_begin + base; gi < a.g_begin + bend && !stop; gi++) {
+      const uint32_t *dsc = a.desc_in + gi * a.dw_in;
+      const uint32_t w = lane < (int)a.dw_in ? dsc[lane] : 0u;
+      const uint32_t beg = __shfl_sync(0xffffffffu, w, 0);
+      const uint32_t len = __shfl_sync(0xffffffffu, w, 1);
+      if (len == 0) continue;
+      uint32_t phi[kMaxV];
+#pragma unroll
+      for (int j = 0; j < kMaxV; j++) phi[j] = __shfl_sync(0xffffffffu, w, (2 + j) & 31);
+      in_entries += (lane == 0) ? len : 0;
+      // ---- Opt 2: L_m over the prefix-only backward lists, staged per group ----
+      const Bounds bs = bounds_for(a, q, prefix_mask, phi);
+      bool staged = false;
+      uint32_t lm_len = 0;
+      if (bshared && a.stage) {
+        const uint32_t r = sm_intersect<true>(a, q, bshared, phi, bs, last, nullptr, 0, slm, kLmCap, lane);
+        __syncwarp();
+        if (r != 0xffffffffu) {
+          staged = true;
+          lm_len = r;
+        }
+      }
+      if (staged && lm_len == 0) continue;   // no child can extend
+      const uint32_t *run = a.vid_in + beg;
+      for (uint32_t i = 0; i < len && !stop; i++) {
+        const uint32_t c = run[i];
+        phi[d] = c;
+        const Bounds bc = bounds_for(a, q, prefix_mask | (1u << d), phi);
+        uint32_t found;
+        uint64_t pos = 0;
+        bool big = false;
+        if (staged && !child_in_b) {
+          // candidates = L_m minus position-d filters (all prefix filters applied)
+          found = 0;
+          for (uint32_t j0 = 0; j0 < lm_len; j0 += 32) {
+            const uint32_t jj = j0 + lane;
+            const uint32_t x = jj < lm_len ? slm[jj] : 0xffffffffu;
+            const bool ok = jj < lm_len && (int64_t)x > bc.lo && x < bc.hi &&
+                            !(((a.P.injmask[q] >> d) & 1u) && x == c);
+            const uint32_t bal = __ballot_sync(0xffffffffu, ok);
+            if (!last && ok) sout[found + __popc(bal & lanemask_lt())] = x;
+            found += __popc(bal);
+          }
+        } else {
+          const uint32_t lists = child_in_b ? (staged ? (1u << d) : bq) : bq;
+          if (!last) {
+            // upper bound of the child's run: the shortest list involved
+            uint32_t ub = staged ? lm_len : 0xffffffffu;
+            uint32_t mm = lists;
+            while (mm) {
+              const int j = __ffs(mm) - 1;
+              mm &= mm - 1;
+              ub = min(ub, gdeg(a, phi[j]));
+            }
+            big = ub > kOutCap;
+            if (big && !pool_reserve(pv, ub, lane, pos)) { stop = true; break; }
+          }
+          if (last)
+            found = sm_intersect<false>(a, q, lists, phi, bc, last, staged ? slm : nullptr, lm_len, nullptr, 0, lane);
+          else
+            found = sm_intersect<true>(a, q, lists, phi, bc, last, staged ? slm : nullptr, lm_len,
+                                       big ? a.vid_out + pos : sout, big ? 0xffffffffu : kOutCap, lane);
+        }
+        if (last) {
+          acc += found;
+          continue;
+        }
+        if (found == 0) continue;
+        __syncwarp();
+        if (!big) {
+          if (!wb_reserve(wv, pv, found, lane, pos)) { stop = true; break; }
+          for (uint32_t t = lane; t < found; t += 32) a.vid_out[pos + t] = sout[t];
+        }
+        // descriptors: slices of kSlice children, each carrying the prefix + c
+        const uint32_t ns = (found + kSlice - 1) / kSlice;
+        uint64_t gpos;
+        if (ns <= kBlkG)
+          wb_retire_tail(wg, ns, lane, [&](uint64_t s) { a.desc_out[s * a.dw_out + 1] = 0u; });
+        bool okg = ns <= kBlkG ? wb_reserve(wg, pg, ns, lane, gpos) : pool_reserve(pg, ns, lane, gpos);
+        if (!okg) { stop = true; break; }
+        for (uint32_t s = 0; s < ns; s++) {
+          uint32_t *o = a.desc_out + (gpos + s) * a.dw_out;
+          if (lane < (int)a.dw_out) {
+            uint32_t val;
+            if (lane == 0) val = (uint32_t)(pos + s * kSlice);
+            else if (lane == 1) val = min(kSlice, found - s * kSlice);
+            else val = phi[0];
+#pragma unroll
+            for (int j = 0; j < kMaxV; j++)
+              if (lane == 2 + j) val = phi[j];
+            o[lane] = val;
+          }
+        }
+        out_entries += (lane == 0) ? found : 0;
+        __syncwarp();
+      }
+      __syncwarp();
+    }
+  }
+  if (!last)   // unused descriptor slots of the last block: empty groups
+    for (uint64_t s = wg.b; s < wg.e; s++)
+      if (lane == 1) a.desc_out[s * a.dw_out + 1] = 0u;
+  if (lane == 0) {
+    if (acc) atomicAdd(&a.ctrl[CTRL_COUNT], (unsigned long long)acc);
+    atomicAdd(&a.ctrl[CTRL_AUX0], (unsigned long long)in_entries);
+    atomicAdd(&a.ctrl[CTRL_ENTRIES], (unsigned long long)out_entries);
+  }
+}
+
+// ---- roots: label / degree filter, cost order, rank partition ----
+struct RootOk {
+  const uint64_t *rp;
+  const uint32_t *lab;
+  uint32_t labeled, label, mindeg;
+  __device__ __forceinline__ bool operator()(const uint32_t &v) const {
+    if (labeled && (lab ? lab[v] : 0u) != label) return false;
+    return rp[v + 1] - rp[v] >= mindeg;
+  }
+};
+
+__global__ void sm_iota(uint32_t *p, uint32_t n) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+    p[i] = (uint32_t)i;
+}
+
+__global__ void sm_root_cost(const uint64_t *rp, const uint32_t *roots, uint64_t nr, uint64_t *cost) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < nr; i += (uint64_t)gridDim.x * blockDim.x)
+    cost[i] = rp[roots[i] + 1] - rp[roots[i]];
+}
+
+__global__ void sm_rank_flag(uint64_t nr, uint32_t rank, uint32_t world, uint8_t *flag) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < nr; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint64_t r = i % (2ull * world);
+    flag[i] = (r == rank || r == 2ull * world - 1 - rank) ? 1 : 0;
+  }
+}
+
+// depth-0 groups: chunks of kRootChunk roots, descriptor {beg, len}
+__global__ void sm_root_groups(uint64_t nr, uint32_t *desc) {
+  const uint64_t ngr = (nr + kRootChunk - 1) / kRootChunk;
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < ngr; i += (uint64_t)gridDim.x * blockDim.x) {
+    desc[2 * i] = (uint32_t)(i * kRootChunk);
+    const uint64_t rest = nr - i * kRootChunk;
+    desc[2 * i + 1] = (uint32_t)(rest < kRootChunk ? rest : kRootChunk);
+  }
+}
+
+inline unsigned g1d(uint64_t n) {
+  uint64_t b = (n + 255) / 256;
+  return (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(b, 148u * 32u));
+}
+
+constexpr size_t sm_smem() { return (size_t)kWarps * (kLmCap + kOutCap) * sizeof(uint32_t); }
+
+}  // namespace
+
+// ------------------------------------------------------------------------------------
+// Host planner (also exported for tests through gamma_pattern_plan).
+// ------------------------------------------------------------------------------------
+static void plan_pattern(const gamma_pattern *p, SmPlan &P) {
+  GAMMA_REQUIRE(p->nv >= 1 && p->nv <= (uint32_t)kMaxV, GAMMA_E_INVAL, "pattern: nv must be in [1, 8]");
+  GAMMA_REQUIRE(p->induced == 0, GAMMA_E_UNSUPPORTED, "pattern: induced matching is not supported in v1");
+  GAMMA_REQUIRE(p->ne == 0 || p->edges, GAMMA_E_INVAL, "pattern: NULL edges");
+  const uint32_t nv = p->nv;
+  int adj[kMaxV][kMaxV] = {};
+  for (uint32_t e = 0; e < p->ne; e++) {
+    const uint32_t u = p->edges[2 * e], v = p->edges[2 * e + 1];
+    GAMMA_REQUIRE(u < nv && v < nv && u != v, GAMMA_E_INVAL, "pattern: bad edge");
+    adj[u][v] = adj[v][u] = 1;
+  }
+  uint32_t deg[kMaxV] = {};
+  for (uint32_t u = 0; u < nv; u++)
+    for (uint32_t v = 0; v < nv; v++) deg[u] += adj[u][v];
+  uint32_t lab[kMaxV] = {};
+  for (uint32_t u = 0; u < nv; u++) lab[u] = p->labels ? p->labels[u] : 0;
+  // connectivity
+  {
+    int seen[kMaxV] = {};
+    uint32_t st[kMaxV], sp = 0;
+    st[sp++] = 0;
+    seen[0] = 1;
+    uint32_t cnt = 1;
+    while (sp) {
+      const uint32_t x = st[--sp];
+      for (uint32_t y = 0; y < nv; y++)
+        if (adj[x][y] && !seen[y]) { seen[y] = 1; st[sp++] = y; cnt++; }
+    }
+    GAMMA_REQUIRE(cnt == nv, GAMMA_E_INVAL, "pattern: not connected");
+  }
+  // matching order (reading R10)
+  uint32_t order[kMaxV], pos_of[kMaxV];
+  int placed[kMaxV] = {};
+  for (uint32_t i = 0; i < nv; i++) {
+    int best = -1;
+    uint32_t bb = 0, bd = 0;
+    for (uint32_t u = 0; u < nv; u++) {
+      if (placed[u]) continue;
+      uint32_t back = 0;
+      for (uint32_t t = 0; t < i; t++) back += adj[u][order[t]];
+      if (i > 0 && back == 0) continue;   // keep the order connected
+      const bool better = best < 0 || back > bb || (back == bb && deg[u] > bd);
+      if (better) { best = (int)u; bb = back; bd = deg[u]; }
+    }
+    order[i] = (uint32_t)best;
+    pos_of[best] = i;
+    placed[best] = 1;
+  }
+  // Aut_L by brute force (Heap's algorithm)
+  std::vector<std::vector<uint32_t>> autos;
+  {
+    uint32_t perm[kMaxV], c[kMaxV] = {};
+    for (uint32_t i = 0; i < nv; i++) perm[i] = i;
+    for (;;) {
+      bool ok = true;
+      for (uint32_t i = 0; i < nv && ok; i++) {
+        if (lab[perm[i]] != lab[i]) ok = false;
+        for (uint32_t j = 0; j < nv && ok; j++)
+          if (adj[perm[i]][perm[j]] != adj[i][j]) ok = false;
+      }
+      if (ok) autos.emplace_back(perm, perm + nv);
+      uint32_t i = 1;
+      while (i < nv && c[i] >= i) { c[i] = 0; i++; }
+      if (i >= nv) break;
+      const uint32_t j = (i % 2) ? c[i] : 0;
+      std::swap(perm[j], perm[i]);
+      c[i]++;
+    }
+  }
+  std::memset(&P, 0, sizeof(P));
+  P.nv = nv;
+  P.labeled = p->labels != nullptr;
+  P.aut = autos.size();
+  for (uint32_t i = 0; i < nv; i++) {
+    const uint32_t u = order[i];
+    P.order[i] = u;
+    P.label[i] = lab[u];
+    P.mindeg[i] = deg[u];
+    for (uint32_t t = 0; t < i; t++) {
+      if (adj[u][order[t]]) P.bmask[i] |= 1u << t;
+      else P.injmask[i] |= 1u << t;
+    }
+  }
+  // stabilizer chain along the matching order
+  std::vector<std::vector<uint32_t>> G = autos;
+  for (uint32_t i = 0; i < nv; i++) {
+    const uint32_t v = order[i];
+    bool orbit[kMaxV] = {};
+    for (auto &g : G) orbit[g[v]] = true;
+    for (uint32_t u = 0; u < nv; u++) {
+      if (u == v || !orbit[u]) continue;
+      // phi(v) < phi(u); u is placed later than v (it is still in v's orbit
+      // under the stabilizer of every earlier vertex, so it is not earlier)
+      const uint32_t pu = pos_of[u];
+      if (pu > i) P.ltmask[pu] |= 1u << i;
+      else P.gtmask[i] |= 1u << pu;
+    }
+    std::vector<std::vector<uint32_t>> H;
+    for (auto &g : G)
+      if (g[v] == v) H.push_back(g);
+    G.swap(H);
+  }
+}
+
+struct SmLevel {
+  DevBuf<uint32_t> vid;
+  DevBuf<uint32_t> desc;
+  uint64_t cap_v = 0, cap_g = 0;
+  uint32_t dw = 0;
+};
+
+struct SmRun {
+  gamma_graph *g;
+  gamma_ctx *ctx;
+  SmPlan P;
+  std::vector<SmLevel> lv;    // lv[d]: groups at depth d (d = 0: root chunks)
+  uint64_t level_share;
+  uint64_t total = 0;
+  int grid = 0;
+  uint32_t stage = 1;
+
+  bool grow(uint32_t d, uint64_t want_v) {
+    SmLevel &L = lv[d];
+    const uint32_t dw = 2 + d;
+    const uint64_t per_slot = 4 + (uint64_t)dw * 4 / 8;   // cap_g = cap_v / 8
+    uint64_t cv = std::max<uint64_t>(want_v, 1ull << 16);
+    cv = std::min<uint64_t>(cv, level_share / per_slot);
+    cv = std::min<uint64_t>(cv, 0xFFFFFFFFull - kBlkV);
+    if (cv <= L.cap_v) return false;
+    const uint64_t cg = cv / 8 + 2 * kBlkG;
+    L.vid.reset();
+    L.desc.reset();
+    L.vid = DevBuf<uint32_t>(ctx, cv);
+    L.desc = DevBuf<uint32_t>(ctx, cg * dw);
+    L.cap_v = cv;
+    L.cap_g = cg;
+    L.dw = dw;
+    return true;
+  }
+
+  SmArgs args(uint32_t d, uint64_t g0, uint64_t g1) {
+    SmArgs a{};
+    a.rp = g->row_ptr;
+    a.col = g->col;
+    a.lab = g->labels;
+    a.P = P;
+    a.d = d;
+    a.vid_in = lv[d].vid.p;
+    a.desc_in = lv[d].desc.p;
+    a.dw_in = 2 + d;
+    a.g_begin = g0;
+    a.g_end = g1;
+    a.ctrl = (unsigned long long *)ctx->ctrl;
+    a.batch = d == 0 ? 1 : 4;
+    a.stage = stage;
+    return a;
+  }
+
+  void run_kernel(const SmArgs &a, bool last, uint64_t cap_v) {
+    int gr = grid;
+    if (!last) {
+      const uint64_t warps_ok = std::max<uint64_t>(1, cap_v / (2ull * kBlkV));
+      gr = (int)std::max<uint64_t>(1, std::min<uint64_t>(gr, warps_ok / kWarps));
+    }
+    ctrl_reset(ctx);
+    ctx->launch(last ? KC_SM_COUNT : KC_SM_EXTEND,
+                [&] { sm_kernel<<<gr, kThreads, sm_smem(), ctx->stream>>>(a); });
+    ctrl_fetch(ctx);
+  }
+
+  void process(uint32_t d, uint64_t g0, uint64_t g1) {
+    if (g0 >= g1) return;
+    const uint32_t q = d + 1;
+    const bool last = q == P.nv - 1;
+    if (last) {
+      SmArgs a = args(d, g0, g1);
+      run_kernel(a, true, 0);
+      const uint64_t *h = ctx->ctrl_host;
+      total = checked_add(total, h[CTRL_COUNT]);
+      ctx->stats.level_entries[P.nv] = checked_add(ctx->stats.level_entries[P.nv], h[CTRL_COUNT]);
+      return;
+    }
+    for (;;) {
+      SmLevel &L = lv[q];
+      if (L.cap_v == 0) grow(q, std::max<uint64_t>(1ull << 24, 4ull * kBlkV * kWarps * (uint64_t)grid));
+      SmArgs a = args(d, g0, g1);
+      a.vid_out = L.vid.p;
+      a.desc_out = L.desc.p;
+      a.dw_out = 2 + q;
+      a.cap_v = L.cap_v;
+      a.cap_g = L.cap_g;
+      run_kernel(a, false, L.cap_v);
+      const uint64_t *h = ctx->ctrl_host;
+      if (!h[CTRL_OVF]) {
+        ctx->stats.level_entries[q + 1] += h[CTRL_ENTRIES];
+        ctx->stats.chunks++;
+        process(q, 0, std::min<uint64_t>(h[CTRL_GCUR], L.cap_g));
+        return;
+      }
+      ctx->stats.retries++;
+      if (grow(q, std::max<uint64_t>(h[CTRL_VCUR], L.cap_v) * 4)) continue;
+      GAMMA_REQUIRE(g1 - g0 > 1, GAMMA_E_NOMEM, "HBM budget too small for one embedding group (SM)");
+      const uint64_t mid = g0 + (g1 - g0) / 2;
+      process(d, g0, mid);
+      process(d, mid, g1);
+      return;
+    }
+  }
+};
+
+static uint64_t match_count(gamma_graph *g, const SmPlan &P) {
+  gamma_ctx *ctx = g->ctx;
+  SmRun R;
+  R.g = g;
+  R.ctx = ctx;
+  R.P = P;
+  R.lv.resize(kMaxV + 1);
+  R.stage = (ctx->desc.flags & GAMMA_FLAG_DEBUG_NOSTAGE) ? 0u : 1u;
+  {
+    size_t fr = 0, tot = 0;
+    GAMMA_CUDA(cudaMemGetInfo(&fr, &tot));
+    const uint64_t budget = ctx->desc.hbm_budget_bytes ? ctx->desc.hbm_budget_bytes : (uint64_t)(fr * 0.8);
+    R.level_share = budget / std::max<uint32_t>(1, P.nv > 2 ? P.nv - 2 : 1);
+  }
+  // ---- roots (position 0) ----
+  const uint32_t n = g->n;
+  DevBuf<uint32_t> all(ctx, n), sel(ctx, n);
+  DevBuf<uint64_t> nsel(ctx, 1);
+  ctx->launch(KC_ROOTS, [&] { sm_iota<<<g1d(n), 256, 0, ctx->stream>>>(all.p, n); });
+  RootOk op{g->row_ptr, g->labels, P.labeled, P.label[0], P.mindeg[0]};
+  size_t tmp = 0;
+  GAMMA_CUDA(cub::DeviceSelect::If(nullptr, tmp, all.p, sel.p, nsel.p, (int64_t)n, op, ctx->stream));
+  {
+    DevBuf<uint8_t> t(ctx, tmp);
+    ctx->launch(KC_ROOTS, [&] {
+      GAMMA_CUDA(cub::DeviceSelect::If(t.p, tmp, all.p, sel.p, nsel.p, (int64_t)n, op, ctx->stream));
+    });
+  }
+  uint64_t nr = 0;
+  GAMMA_CUDA(cudaMemcpyAsync(&nr, nsel.p, sizeof(uint64_t), cudaMemcpyDeviceToHost, ctx->stream));
+  ctx->sync();
+  if (P.nv == 1) {
+    if (ctx->desc.world > 1) {   // partition the roots like everything else
+      const uint64_t w = ctx->desc.world, r = ctx->desc.rank;
+      uint64_t mine = 0;
+      for (uint64_t i = 0; i < nr; i++) {
+        const uint64_t x = i % (2 * w);
+        mine += (x == r || x == 2 * w - 1 - r);
+      }
+      return mine;
+    }
+    return nr;
+  }
+  DevBuf<uint32_t> roots(ctx, nr ? nr : 1);
+  if (nr) {
+    DevBuf<uint64_t> cost(ctx, nr), cost2(ctx, nr);
+    ctx->launch(KC_ROOTS, [&] { sm_root_cost<<<g1d(nr), 256, 0, ctx->stream>>>(g->row_ptr, sel.p, nr, cost.p); });
+    int endbit = 1;
+    while (endbit < 64 && (1ull << endbit) <= (uint64_t)g->max_degree) endbit++;
+    tmp = 0;
+    GAMMA_CUDA(cub::DeviceRadixSort::SortPairsDescending(nullptr, tmp, cost.p, cost2.p, sel.p, roots.p, nr, 0,
+                                                         endbit, ctx->stream));
+    DevBuf<uint8_t> t(ctx, tmp);
+    ctx->launch(KC_ROOTS, [&] {
+      GAMMA_CUDA(cub::DeviceRadixSort::SortPairsDescending(t.p, tmp, cost.p, cost2.p, sel.p, roots.p, nr, 0,
+                                                           endbit, ctx->stream));
+    });
+  }
+  if (ctx->desc.world > 1 && nr) {
+    DevBuf<uint8_t> flag(ctx, nr);
+    ctx->launch(KC_ROOTS, [&] {
+      sm_rank_flag<<<g1d(nr), 256, 0, ctx->stream>>>(nr, ctx->desc.rank, ctx->desc.world, flag.p);
+    });
+    DevBuf<uint32_t> mine(ctx, nr);
+    tmp = 0;
+    GAMMA_CUDA(cub::DeviceSelect::Flagged(nullptr, tmp, roots.p, flag.p, mine.p, nsel.p, (int64_t)nr, ctx->stream));
+    {
+      DevBuf<uint8_t> t(ctx, tmp);
+      ctx->launch(KC_ROOTS, [&] {
+        GAMMA_CUDA(cub::DeviceSelect::Flagged(t.p, tmp, roots.p, flag.p, mine.p, nsel.p, (int64_t)nr, ctx->stream));
+      });
+    }
+    GAMMA_CUDA(cudaMemcpyAsync(&nr, nsel.p, sizeof(uint64_t), cudaMemcpyDeviceToHost, ctx->stream));
+    ctx->sync();
+    roots = std::move(mine);
+  }
+  ctx->stats.level_entries[1] = nr;
+  if (nr == 0) return 0;
+  const uint64_t ngr = (nr + kRootChunk - 1) / kRootChunk;
+  SmLevel &L0 = R.lv[0];
+  L0.desc = DevBuf<uint32_t>(ctx, 2 * ngr);
+  L0.dw = 2;
+  ctx->launch(KC_ROOTS, [&] { sm_root_groups<<<g1d(ngr), 256, 0, ctx->stream>>>(nr, L0.desc.p); });
+  L0.vid = std::move(roots);
+  L0.cap_v = nr;
+  L0.cap_g = ngr;
+  static bool attr = false;
+  if (!attr) {
+    GAMMA_CUDA(cudaFuncSetAttribute(sm_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm_smem()));
+    attr = true;
+  }
+  R.grid = ctx->num_sms * occupancy_blocks((const void *)sm_kernel, kThreads, sm_smem());
+  R.process(0, 0, ngr);
+  ctx->sync();
+  ctx->collect_timings();
+  return R.total;
+}
+
+}  // namespace gamma_impl
+
 using namespace gamma_impl;
+
+extern "C" gamma_status gamma_pattern_plan(const gamma_pattern *p, gamma_plan_info *out) {
+  return guarded([&] {
+    GAMMA_REQUIRE(p && out, GAMMA_E_INVAL, "gamma_pattern_plan: NULL argument");
+    SmPlan P;
+    plan_pattern(p, P);
+    std::memset(out, 0, sizeof(*out));
+    out->nv = P.nv;
+    out->aut = P.aut;
+    for (uint32_t i = 0; i < P.nv; i++) {
+      out->order[i] = P.order[i];
+      out->backward_mask[i] = P.bmask[i];
+      out->less_mask[i] = P.ltmask[i];
+      out->greater_mask[i] = P.gtmask[i];
+    }
+  });
+}
 
 extern "C" gamma_status gamma_match(gamma_graph *g, const gamma_pattern *p, uint64_t *count,
                                     uint64_t *mappings) {
   return guarded([&] {
     GAMMA_REQUIRE(g && p && count, GAMMA_E_INVAL, "gamma_match: NULL argument");
-    throw Fail{GAMMA_E_UNSUPPORTED, "gamma_match: not implemented yet"};
+    SmPlan P;
+    plan_pattern(p, P);
+    gamma_ctx *c = g->ctx;
+    GAMMA_CUDA(cudaSetDevice(c->device));
+    c->reset_stats();
+    uint64_t r = match_count(g, P);
+    if (c->desc.world > 1 && c->desc.allreduce_sum_u64) {
+      gamma_status st = c->desc.allreduce_sum_u64(&r, 1, c->desc.coll_user);
+      GAMMA_REQUIRE(st == GAMMA_OK, st, "allreduce_sum_u64 callback failed");
+    }
+    *count = r;
+    if (mappings) {
+      uint64_t mp;
+      GAMMA_REQUIRE(!__builtin_mul_overflow(r, P.aut, &mp), GAMMA_E_OVERFLOW, "mappings overflow uint64");
+      *mappings = mp;
+    }
   });
-}
-
-extern "C" gamma_status gamma_fpm(gamma_graph *g, uint32_t max_edges, uint64_t minsup,
-                                  gamma_fpm_result **out) {
-  return guarded([&] {
-    GAMMA_REQUIRE(g && out, GAMMA_E_INVAL, "gamma_fpm: NULL argument");
-    throw Fail{GAMMA_E_UNSUPPORTED, "gamma_fpm: not implemented yet"};
-  });
-}
-
-extern "C" void gamma_fpm_result_free(gamma_fpm_result *r) {
-  if (!r) return;
-  delete[] r->pats;
-  delete r;
 }

@@ -1,0 +1,131 @@
+"""GPU parity of gamma_match (Alg. 1, labeled non-induced SM) against the oracle
+(O-2), through the C ABI.  Tolerance 0."""
+from math import comb
+
+import numpy as np
+import pytest
+
+import gamma_gen as gg
+
+pytestmark = pytest.mark.gpu
+Q = gg.QUERIES
+
+
+@pytest.fixture(scope="module")
+def G():
+    import torch
+    assert torch.cuda.is_available()
+    import paper_conf_icde_hu0o23_b200 as G
+    return G
+
+
+@pytest.fixture(scope="module")
+def ctx(G):
+    return G.Context(device=0)
+
+
+def gcount(g, q, plab=None):
+    nv, e = Q[q]
+    return g.match(nv, e, plab)
+
+
+@pytest.mark.parametrize("n", [5, 8, 12])
+def test_complete(ctx, n):
+    ns, (s, d) = gg.complete(n)
+    g = ctx.load_edges(ns, s, d)
+    assert gcount(g, "c4")[0] == 3 * comb(n, 4)
+    assert gcount(g, "diamond")[0] == 6 * comb(n, 4)
+    assert gcount(g, "tailed_triangle")[0] == 12 * comb(n, 4)
+    assert gcount(g, "house")[0] == 60 * comb(n, 5)
+
+
+def test_closed_forms(ctx):
+    n, (s, d) = gg.complete_bipartite(5, 7)
+    g = ctx.load_edges(n, s, d)
+    assert gcount(g, "c4")[0] == comb(5, 2) * comb(7, 2)
+    assert gcount(g, "house")[0] == 0
+    n, (s, d) = gg.grid(7, 9)
+    g = ctx.load_edges(n, s, d)
+    assert gcount(g, "c4")[0] == 6 * 8
+    n, (s, d) = gg.wheel(11)
+    g = ctx.load_edges(n, s, d)
+    assert [gcount(g, q)[0] for q in ("c4", "diamond", "tailed_triangle", "house")] == [11, 11, 121, 22]
+    n, (s, d) = gg.petersen()
+    assert gcount(ctx.load_edges(n, s, d), "c4")[0] == 0
+
+
+@pytest.mark.parametrize("seed", [1, 2, 3])
+@pytest.mark.parametrize("q", ["c4", "diamond", "tailed_triangle", "house"])
+def test_rmat_vs_oracle(ctx, oracle_mod, seed, q):
+    n, s, d, _ = gg.config_graph("c3", seed=seed, scale=12)
+    lab = gg.labels(n, 8, seed)
+    g = ctx.load_edges(n, s, d, lab)
+    o = oracle_mod.Graph(n, s, d, lab)
+    nv, e = Q[q]
+    for plab in ([0] * nv, [i % 8 for i in range(nv)], None):
+        got = g.match(nv, e, plab)
+        want = o.match(nv, e, plab)
+        assert got == (want[0], want[1]), (q, plab)
+
+
+@pytest.mark.parametrize("q", ["c4", "diamond", "tailed_triangle", "house"])
+def test_er_unlabeled_vs_oracle(ctx, oracle_mod, q):
+    n = 1500
+    s, d = gg.er(n, 9000, 4)
+    g = ctx.load_edges(n, s, d)
+    o = oracle_mod.Graph(n, s, d)
+    nv, e = Q[q]
+    assert g.match(nv, e)[0] == o.match(nv, e)[0]
+
+
+def test_unstaged_and_budget_paths(G, oracle_mod):
+    n, s, d, _ = gg.config_graph("c3", seed=5, scale=11)
+    lab = gg.labels(n, 2, 5)
+    o = oracle_mod.Graph(n, s, d, lab)
+    for c in (G.Context(flags=0x8), G.Context(hbm_budget_bytes=2 << 20)):
+        g = c.load_edges(n, s, d, lab)
+        for q in ("c4", "house"):
+            nv, e = Q[q]
+            plab = [i % 2 for i in range(nv)]
+            assert g.match(nv, e, plab)[0] == o.match(nv, e, plab)[0]
+
+
+def test_more_patterns(ctx, oracle_mod):
+    """Triangle, path, star, K4, 5-cycle, 6-vertex patterns and a single vertex."""
+    pats = [(3, [(0, 1), (1, 2), (0, 2)]), (3, [(0, 1), (1, 2)]), (4, [(0, 1), (0, 2), (0, 3)]),
+            (4, [(0, 1), (0, 2), (0, 3), (1, 2), (1, 3), (2, 3)]), (5, [(0, 1), (1, 2), (2, 3), (3, 4), (4, 0)]),
+            (6, [(0, 1), (1, 2), (2, 0), (2, 3), (3, 4), (4, 5), (5, 3)]), (2, [(0, 1)])]
+    n, s, d, _ = gg.config_graph("c1", seed=2, scale=10)
+    lab = gg.labels(n, 3, 2)
+    g = ctx.load_edges(n, s, d, lab)
+    o = oracle_mod.Graph(n, s, d, lab)
+    for nv, e in pats:
+        assert g.match(nv, e)[0] == o.match(nv, e)[0], (nv, e)
+        plab = [(i * 7) % 3 for i in range(nv)]
+        assert g.match(nv, e, plab)[0] == o.match(nv, e, plab)[0], (nv, e, plab)
+    assert g.match(1, [], [1])[0] == int((lab == 1).sum())
+
+
+def test_simulated_ranks(G, oracle_mod):
+    n, s, d, _ = gg.config_graph("c3", seed=2, scale=11)
+    lab = gg.labels(n, 4, 2)
+    nv, e = Q["diamond"]
+    plab = [0, 1, 1, 0]
+    want = oracle_mod.Graph(n, s, d, lab).match(nv, e, plab)[0]
+    tot = 0
+    for r in range(3):
+        c = G.Context(rank=r, world=3, reduce=False)
+        tot += c.load_edges(n, s, d, lab).match(nv, e, plab)[0]
+    assert tot == want
+
+
+def test_invalid_patterns(G, ctx):
+    n, (s, d) = gg.complete(5)
+    g = ctx.load_edges(n, s, d)
+    with pytest.raises(G.GammaError):
+        g.match(4, [(0, 1), (2, 3)])          # disconnected
+    with pytest.raises(G.GammaError) as e:
+        g.match(3, [(0, 1), (1, 2)], induced=True)
+    assert e.value.status == -5
+    with pytest.raises(G.GammaError):
+        g.match(9, [(i, i + 1) for i in range(8)])
