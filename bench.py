@@ -102,6 +102,18 @@ class ClockSampler:
                 "reasons": sorted(reasons), "samples": len(sm)}
 
 
+def max_over_ranks(value: float, world: int) -> float:
+    """Max of a per-rank number over the default process group (identity at world 1)."""
+    if world <= 1:
+        return float(value)
+    import torch
+    import torch.distributed as dist
+    dev = torch.device("cuda", torch.cuda.current_device()) if dist.get_backend() == "nccl" else torch.device("cpu")
+    t = torch.tensor([float(value)], dtype=torch.float64, device=dev)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
 def dist_env():
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -255,10 +267,7 @@ def run_gamma(args):
         times.append(e0.elapsed_time(e1))
         counts_seen = counts
     clk = clocks.stop()
-    t = torch.tensor([sum(times)], dtype=torch.float64, device="cuda")
-    if world > 1:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    total_ms = float(t.item())
+    total_ms = max_over_ranks(sum(times), world)
     emb_per_step = sum(counts_seen)   # all-reduced global counts
     value = emb_per_step * args.steps / (total_ms / 1000.0)
 
@@ -275,10 +284,7 @@ def run_gamma(args):
         torch.cuda.synchronize()
         barrier()
         e2e_times.append(e0.elapsed_time(e1))
-    te = torch.tensor([sum(e2e_times)], dtype=torch.float64, device="cuda")
-    if world > 1:
-        dist.all_reduce(te, op=dist.ReduceOp.MAX)
-    e2e_value = emb_per_step * len(e2e_times) / (float(te.item()) / 1000.0)
+    e2e_value = emb_per_step * len(e2e_times) / (max_over_ranks(sum(e2e_times), world) / 1000.0)
 
     if rank != 0:
         if world > 1:

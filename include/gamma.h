@@ -81,6 +81,8 @@ typedef struct {
                                           instead of the DFS-over-chunks policy      */
 #define GAMMA_FLAG_DEBUG_NOSTAGE 0x8u  /* test hook: never stage runs in shared memory
                                           (exercises the hub / long-run code path)   */
+#define GAMMA_FLAG_NO_BITMAP    0x10u  /* kCL: use the ET-level path for every root
+                                          (no local-bitmap DFS; ablation / testing)  */
 
 /* Create / destroy a context.  Errors: E_INVAL (NULL args), E_CUDA (no device). */
 gamma_status gamma_ctx_create(const gamma_ctx_desc *desc, gamma_ctx **out);

@@ -88,6 +88,29 @@ def pattern_plan(nv: int, edges, labels=None, induced: bool = False) -> dict:
             "greater_mask": [info.greater_mask[i] for i in range(nv)], "aut": int(info.aut)}
 
 
+def make_allreduce_callback(device: int = 0):
+    """The ctx's ``allreduce_sum_u64`` callback: an in-place SUM of n uint64 values
+    held in host memory, over the default torch.distributed process group (a CUDA
+    int64 tensor for NCCL, a CPU one for gloo).  Returns the ctypes function."""
+    import torch
+    import torch.distributed as dist
+    backend = dist.get_backend()
+
+    def _allreduce(buf, n, user):
+        try:
+            vals = [buf[i] for i in range(n)]
+            dev = torch.device("cuda", device) if backend == "nccl" else torch.device("cpu")
+            t = torch.tensor(vals, dtype=torch.int64, device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.SUM)
+            for i, v in enumerate(t.cpu().tolist()):
+                buf[i] = v
+            return 0
+        except Exception:   # noqa: BLE001 -- reported as a gamma_status
+            return N.GAMMA_E_CUDA
+
+    return N.ALLREDUCE_FN(_allreduce)
+
+
 class Context:
     """A gamma_ctx bound to one CUDA device, its stream and allocator.
 
@@ -133,23 +156,7 @@ class Context:
             d.dev_alloc, d.dev_free = fa, ff
             self._keep += [fa, ff]
         if reduce and d.world > 1 and dist_ok:
-            import torch.distributed as dist
-            torch = self._torch
-            backend = dist.get_backend()
-
-            def _allreduce(buf, n, user):
-                try:
-                    vals = [buf[i] for i in range(n)]
-                    dev = torch.device("cuda", device) if backend == "nccl" else torch.device("cpu")
-                    t = torch.tensor(vals, dtype=torch.int64, device=dev)
-                    dist.all_reduce(t, op=dist.ReduceOp.SUM)
-                    for i, v in enumerate(t.cpu().tolist()):
-                        buf[i] = v
-                    return 0
-                except Exception:   # noqa: BLE001
-                    return N.GAMMA_E_CUDA
-
-            fr = N.ALLREDUCE_FN(_allreduce)
+            fr = make_allreduce_callback(device)
             d.allreduce_sum_u64 = fr
             self._keep.append(fr)
         d.hbm_budget_bytes = hbm_budget_bytes

@@ -18,7 +18,7 @@ void clear_error() { g_err.clear(); }
 
 const char *kKernelClassName[KC_NUM] = {"build",  "roots",     "extend", "count",
                                         "fused",  "sm_extend", "sm_count", "fpm",
-                                        "fpm_support", "misc"};
+                                        "fpm_support", "misc", "bitmap"};
 
 bool is_device_ptr(const void *ptr) {
   if (!ptr) return false;

@@ -1,13 +1,580 @@
-// fpm.cu -- frequent pattern mining (Alg. 2) -- placeholder until the FPM path lands.
+// fpm.cu -- frequent pattern mining, Alg. 2: edge extension
+// (Def. 3.1 Ext_e, L131-139), aggregation by canonical label into the pattern
+// table (L142), filtering by sup >= minsup (L144) with removal of the instances of
+// infrequent patterns before the next extension (Alg. 2 line 4).
+// Readings: R1 support = MNI (orbits merged), R2 length = #edges,
+// R3 edge-induced, R7 canonical code = min over vertex orders of (labels, sorted
+// edge-pair list), R8 sup >= minsup, R11 each connected edge set generated once.
+//
+// B200 design:
+//  * e-ET root = every edge e1 (generated from its smaller endpoint); one warp per
+//    root vertex u, lanes over u's edges / over the candidate second edges.  Each
+//    connected edge set S = {e1 < e2 < e3} (edge order = (min,max) lexicographic) is
+//    produced exactly once: from its minimum edge e1; the second generated edge is
+//    the smallest edge of S adjacent to e1's... (see gen rule in fpm_enum_kernel).
+//  * The levels < l are regenerated per level rather than stored (DFS per root
+//    edge); Alg. 2's pruning is applied at every generated prefix by looking its
+//    pattern up in the pattern table (infrequent prefix => no extension).
+//  * Canonical code: sort the <= 4 vertex labels (the minimal label sequence), then
+//    enumerate only the label-consistent vertex orders and keep the minimal sorted
+//    edge-pair list; every minimizing order is an automorphic placement, so OR-ing
+//    the vertex of each position into that position's domain merges orbits (MNI).
+//  * Pattern table: lock-free open-addressing hash (code -> slot) in HBM; the MNI
+//    domain of slot position p is a bitmap over the vertices of p's label class
+//    (bit index = rank of the vertex inside its label class), carved from a pool
+//    at slot creation.  Support = min over positions of popcount (one warp/slot).
+#include <cub/device/device_radix_sort.cuh>
+
+#include <algorithm>
+#include <vector>
+
+#include "device_common.cuh"
 #include "internal.cuh"
+
+namespace gamma_impl {
+
+namespace {
+
+constexpr int kThreads = 256;
+
+__constant__ uint8_t c_perm4[24][4] = {
+    {0, 1, 2, 3}, {0, 1, 3, 2}, {0, 2, 1, 3}, {0, 2, 3, 1}, {0, 3, 1, 2}, {0, 3, 2, 1},
+    {1, 0, 2, 3}, {1, 0, 3, 2}, {1, 2, 0, 3}, {1, 2, 3, 0}, {1, 3, 0, 2}, {1, 3, 2, 0},
+    {2, 0, 1, 3}, {2, 0, 3, 1}, {2, 1, 0, 3}, {2, 1, 3, 0}, {2, 3, 0, 1}, {2, 3, 1, 0},
+    {3, 0, 1, 2}, {3, 0, 2, 1}, {3, 1, 0, 2}, {3, 1, 2, 0}, {3, 2, 0, 1}, {3, 2, 1, 0}};
+// index of position pair (a<b) in lexicographic pair order: (0,1)(0,2)(0,3)(1,2)(1,3)(2,3)
+__constant__ uint8_t c_pair[4][4] = {{0, 0, 1, 2}, {0, 0, 3, 4}, {1, 3, 0, 5}, {2, 4, 5, 0}};
+
+struct Table {
+  uint32_t *st;          // 0 empty, 1 being written, 2 ready
+  unsigned long long *klo, *khi;
+  unsigned long long *dom;   // 4 word offsets per slot into the pool
+  unsigned long long *support;
+  uint32_t *freq;        // 1 if support >= minsup (set after the slot's level)
+  uint64_t cap;          // power of two
+  uint32_t *pool;
+  uint64_t pool_words;
+  unsigned long long *pool_cur;
+};
+
+struct FpmArgs {
+  const uint64_t *rp;
+  const uint32_t *col;
+  const uint32_t *lab;       // nullable
+  const uint32_t *lrank;     // rank of v inside its label class
+  const uint32_t *csize;     // label class sizes
+  uint32_t n;
+  uint32_t level;            // edges per recorded embedding
+  uint32_t rank, world;      // root partition
+  Table T;
+  unsigned long long *ctrl;
+};
+
+__device__ __forceinline__ uint32_t labof(const FpmArgs &a, uint32_t v) { return a.lab ? a.lab[v] : 0u; }
+
+__device__ __forceinline__ uint64_t ekey(uint32_t x, uint32_t y) {
+  const uint32_t lo = x < y ? x : y, hi = x < y ? y : x;
+  return ((uint64_t)lo << 32) | hi;
+}
+
+__device__ __forceinline__ bool shares(uint64_t e, uint64_t f) {
+  const uint32_t a = (uint32_t)(e >> 32), b = (uint32_t)e, c = (uint32_t)(f >> 32), d = (uint32_t)f;
+  return a == c || a == d || b == c || b == d;
+}
+
+__device__ __forceinline__ uint64_t mix64(uint64_t x) {
+  x ^= x >> 33;
+  x *= 0xff51afd7ed558ccdull;
+  x ^= x >> 33;
+  x *= 0xc4ceb9fe1a85ec53ull;
+  x ^= x >> 33;
+  return x;
+}
+
+// Lookup (insert = false) or lookup-or-insert a pattern code; returns slot or -1.
+__device__ int64_t table_slot(const FpmArgs &a, uint64_t klo, uint64_t khi, uint32_t nv, const uint32_t *labs,
+                              bool insert) {
+  const Table &T = a.T;
+  uint64_t h = mix64(klo ^ mix64(khi)) & (T.cap - 1);
+  for (uint64_t probe = 0; probe < T.cap; probe++, h = (h + 1) & (T.cap - 1)) {
+    uint32_t s = *(volatile uint32_t *)&T.st[h];
+    if (s == 0) {
+      if (!insert) return -1;
+      s = atomicCAS(&T.st[h], 0u, 1u);
+      if (s == 0) {
+        T.klo[h] = klo;
+        T.khi[h] = khi;
+        // carve the position bitmaps (one per position, sized to the label class)
+        uint64_t words = 0, wpos[4] = {0, 0, 0, 0};
+        for (uint32_t p = 0; p < nv; p++) {
+          wpos[p] = (a.csize[labs[p]] + 31) / 32;
+          words += wpos[p];
+        }
+        unsigned long long off = atomicAdd(a.T.pool_cur, (unsigned long long)words);
+        if (off + words > T.pool_words) {
+          atomicExch(&a.ctrl[CTRL_OVF], 1ull);
+          off = ~0ull;
+        }
+        uint64_t o = off;
+        for (uint32_t p = 0; p < 4; p++) {
+          T.dom[h * 4 + p] = (off == ~0ull) ? ~0ull : o;
+          o += wpos[p];
+        }
+        T.support[h] = 0;
+        T.freq[h] = 0;
+        __threadfence();
+        atomicExch(&T.st[h], 2u);
+        return (int64_t)h;
+      }
+    }
+    while (s != 2) s = *(volatile uint32_t *)&T.st[h];
+    __threadfence();
+    if (T.klo[h] == klo && T.khi[h] == khi) return (int64_t)h;
+  }
+  atomicExch(&a.ctrl[CTRL_ERR], 1ull);   // table full
+  return -1;
+}
+
+// Canonical code of a connected edge set on nv <= 4 local vertices (W) with ne <= 3
+// edges (local index pairs E).  Returns (klo, khi) and the minimizing vertex orders
+// as a bitmask over c_perm4 rows.
+struct Canon {
+  uint64_t klo, khi;
+  uint32_t labs[4];
+  uint32_t minmask;
+};
+
+__device__ Canon canonical(const FpmArgs &a, const uint32_t *W, uint32_t nv, const uint8_t (*E)[2], uint32_t ne) {
+  Canon cn;
+  uint32_t lw[4];
+  for (uint32_t i = 0; i < 4; i++) lw[i] = i < nv ? labof(a, W[i]) : 0xffffffffu;
+  // minimal label sequence = sorted labels
+  uint32_t ls[4] = {lw[0], lw[1], lw[2], lw[3]};
+  for (int i = 1; i < 4; i++)
+    for (int j = i; j > 0 && ls[j - 1] > ls[j]; j--) {
+      const uint32_t t = ls[j - 1];
+      ls[j - 1] = ls[j];
+      ls[j] = t;
+    }
+  uint32_t best = 0xffffffffu, mask = 0;
+  for (int r = 0; r < 24; r++) {
+    // row r places local vertex c_perm4[r][p] at position p; only rows that keep
+    // positions >= nv fixed are vertex orders of the first nv vertices
+    bool ok = true;
+    for (uint32_t p = 0; p < 4 && ok; p++) {
+      const uint32_t lv = c_perm4[r][p];
+      if (p >= nv) ok = lv == p;
+      else ok = lv < nv && lw[lv] == ls[p];
+    }
+    if (!ok) continue;
+    uint32_t inv[4];
+    for (uint32_t p = 0; p < 4; p++) inv[c_perm4[r][p]] = p;
+    uint32_t idx[3] = {7, 7, 7};
+    for (uint32_t e = 0; e < ne; e++) idx[e] = c_pair[inv[E[e][0]]][inv[E[e][1]]];
+    // sort ne <= 3 pair indices
+    if (idx[0] > idx[1]) { const uint32_t t = idx[0]; idx[0] = idx[1]; idx[1] = t; }
+    if (idx[1] > idx[2]) { const uint32_t t = idx[1]; idx[1] = idx[2]; idx[2] = t; }
+    if (idx[0] > idx[1]) { const uint32_t t = idx[0]; idx[0] = idx[1]; idx[1] = t; }
+    const uint32_t key = idx[0] * 64 + idx[1] * 8 + idx[2];
+    if (key < best) {
+      best = key;
+      mask = 1u << r;
+    } else if (key == best) {
+      mask |= 1u << r;
+    }
+  }
+  cn.klo = 0;
+  for (uint32_t p = 0; p < 4; p++) {
+    cn.labs[p] = p < nv ? ls[p] : 0;
+    cn.klo |= (uint64_t)(cn.labs[p] & 0xffffu) << (16 * p);
+  }
+  cn.khi = (uint64_t)nv | ((uint64_t)ne << 4) | ((uint64_t)best << 8);
+  cn.minmask = mask;
+  return cn;
+}
+
+// Aggregation: OR the vertex of every position of every minimizing order into the
+// position's domain bitmap (read-before-atomic: most bits are already set).
+__device__ void record(const FpmArgs &a, const uint32_t *W, uint32_t nv, const uint8_t (*E)[2], uint32_t ne) {
+  const Canon cn = canonical(a, W, nv, E, ne);
+  const int64_t s = table_slot(a, cn.klo, cn.khi, nv, cn.labs, true);
+  if (s < 0) return;
+  uint64_t off[4];
+  for (uint32_t p = 0; p < 4; p++) off[p] = a.T.dom[s * 4 + p];
+  if (off[0] == ~0ull) return;
+  uint32_t m = cn.minmask;
+  while (m) {
+    const int r = __ffs(m) - 1;
+    m &= m - 1;
+    for (uint32_t p = 0; p < nv; p++) {
+      const uint32_t v = W[c_perm4[r][p]];
+      const uint32_t bit = a.lrank[v];
+      uint32_t *w = a.T.pool + off[p] + (bit >> 5);
+      const uint32_t b = 1u << (bit & 31);
+      if (!(*(volatile uint32_t *)w & b)) atomicOr(w, b);
+    }
+  }
+}
+
+// Is the pattern of this (prefix) edge set frequent?  (Alg. 2 line 4 pruning)
+__device__ bool frequent(const FpmArgs &a, const uint32_t *W, uint32_t nv, const uint8_t (*E)[2], uint32_t ne) {
+  const Canon cn = canonical(a, W, nv, E, ne);
+  const int64_t s = table_slot(a, cn.klo, cn.khi, nv, cn.labs, false);
+  return s >= 0 && a.T.freq[s];
+}
+
+// Local view of an edge set: distinct vertices W and local edge pairs E.
+struct ESet {
+  uint32_t W[4];
+  uint8_t E[3][2];
+  uint32_t nv, ne;
+};
+
+__device__ __forceinline__ uint32_t local_of(ESet &s, uint32_t x) {
+  for (uint32_t i = 0; i < s.nv; i++)
+    if (s.W[i] == x) return i;
+  s.W[s.nv] = x;
+  return s.nv++;
+}
+
+__device__ __forceinline__ void add_edge(ESet &s, uint64_t e) {
+  const uint32_t a = local_of(s, (uint32_t)(e >> 32));
+  const uint32_t b = local_of(s, (uint32_t)e);
+  s.E[s.ne][0] = (uint8_t)a;
+  s.E[s.ne][1] = (uint8_t)b;
+  s.ne++;
+}
+
+// One warp per root vertex u; roots e1 = (u, v), v > u.
+//   level 1: record e1.
+//   level 2: e2 > e1 adjacent to e1 (an edge at u or v), prefix {e1} frequent.
+//   level 3: from each frequent 2-edge prefix (a, b), a < b adjacent, add c with
+//            (c > b, c adjacent to a or b)  or  (a < c < b, c adjacent to b, not to a).
+//            Every connected {e1<e2<e3} arises exactly once: if e1~e2 from (e1,e2)+e3,
+//            else (e3 joins them) from (e1,e3)+e2.
+__global__ void __launch_bounds__(kThreads) fpm_enum_kernel(FpmArgs a) {
+  const int lane = threadIdx.x & 31;
+  uint64_t emb = 0;
+  for (;;) {
+    unsigned long long u0 = 0;
+    if (lane == 0) u0 = atomicAdd(&a.ctrl[CTRL_WORK], 1ull);
+    u0 = __shfl_sync(0xffffffffu, u0, 0);
+    if (u0 >= a.n) break;
+    const uint32_t u = (uint32_t)u0;
+    if (a.world > 1 && (u % a.world) != a.rank) continue;
+    const uint64_t us = a.rp[u], ue = a.rp[u + 1];
+    // first neighbour > u
+    uint64_t first = us;
+    {
+      uint64_t lo = us, hi = ue;
+      while (lo < hi) {
+        const uint64_t mid = (lo + hi) >> 1;
+        if (a.col[mid] <= u) lo = mid + 1; else hi = mid;
+      }
+      first = lo;
+    }
+    for (uint64_t i1 = first; i1 < ue; i1++) {
+      const uint32_t v = a.col[i1];
+      const uint64_t e1 = ekey(u, v);
+      if (a.level == 1) {
+        if (lane == 0) {
+          ESet s{};
+          add_edge(s, e1);
+          record(a, s.W, s.nv, s.E, s.ne);
+          emb++;
+        }
+        continue;
+      }
+      {
+        ESet s{};
+        add_edge(s, e1);
+        if (!frequent(a, s.W, s.nv, s.E, s.ne)) continue;   // uniform: same e1 in all lanes
+      }
+      // candidate second edges: incident to u or v (lists of u then v), e2 > e1
+      const uint64_t vs = a.rp[v], ve = a.rp[v + 1];
+      const uint64_t nu = ue - us, ncand = nu + (ve - vs);
+      for (uint64_t c0 = 0; c0 < ncand; c0 += 32) {
+        const uint64_t ci = c0 + lane;
+        if (ci >= ncand) continue;
+        const uint32_t x = ci < nu ? u : v;
+        const uint32_t y = ci < nu ? a.col[us + ci] : a.col[vs + (ci - nu)];
+        const uint64_t e2 = ekey(x, y);
+        if (e2 <= e1) continue;   // also drops e1 itself
+        ESet s2{};
+        add_edge(s2, e1);
+        add_edge(s2, e2);
+        if (a.level == 2) {
+          record(a, s2.W, s2.nv, s2.E, s2.ne);
+          emb++;
+          continue;
+        }
+        if (!frequent(a, s2.W, s2.nv, s2.E, s2.ne)) continue;
+        // third edges: incident to the 3 vertices of {e1, e2}; an edge joining two of
+        // them is seen from both ends -- keep it at its smaller end only
+        for (uint32_t wi = 0; wi < 3; wi++) {
+          const uint32_t w = s2.W[wi];
+          for (uint64_t j = a.rp[w]; j < a.rp[w + 1]; j++) {
+            const uint32_t z = a.col[j];
+            const bool inner = z == s2.W[0] || z == s2.W[1] || z == s2.W[2];
+            if (inner && z < w) continue;
+            const uint64_t e3 = ekey(w, z);
+            if (e3 == e1 || e3 == e2) continue;
+            const bool ok = (e3 > e2) || (e3 > e1 && shares(e3, e2) && !shares(e3, e1));
+            if (!ok) continue;
+            ESet s3 = s2;
+            add_edge(s3, e3);
+            record(a, s3.W, s3.nv, s3.E, s3.ne);
+            emb++;
+          }
+        }
+      }
+    }
+  }
+  for (int off = 16; off > 0; off >>= 1) emb += __shfl_down_sync(0xffffffffu, emb, off);
+  if (lane == 0 && emb) atomicAdd(&a.ctrl[CTRL_ENTRIES], (unsigned long long)emb);
+}
+
+// Support of every slot of the given level: min over positions of popcount; one
+// warp per slot.
+__global__ void fpm_support_kernel(FpmArgs a, uint32_t level, uint64_t minsup) {
+  const int lane = threadIdx.x & 31;
+  const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  for (uint64_t s = warp; s < a.T.cap; s += nwarps) {
+    if (a.T.st[s] != 2) continue;
+    const uint64_t khi = a.T.khi[s];
+    const uint32_t nv = (uint32_t)(khi & 0xf), ne = (uint32_t)((khi >> 4) & 0xf);
+    if (ne != level) continue;
+    uint64_t sup = ~0ull;
+    const uint64_t klo = a.T.klo[s];
+    for (uint32_t p = 0; p < nv; p++) {
+      const uint32_t lp = (uint32_t)((klo >> (16 * p)) & 0xffff);
+      const uint64_t words = (a.csize[lp] + 31) / 32;
+      const uint64_t off = a.T.dom[s * 4 + p];
+      uint64_t c = 0;
+      for (uint64_t w = lane; w < words; w += 32) c += __popc(a.T.pool[off + w]);
+      for (int o = 16; o > 0; o >>= 1) c += __shfl_down_sync(0xffffffffu, c, o);
+      c = __shfl_sync(0xffffffffu, c, 0);
+      sup = c < sup ? c : sup;
+    }
+    if (lane == 0) {
+      a.T.support[s] = sup;
+      a.T.freq[s] = sup >= minsup ? 1u : 0u;
+    }
+  }
+}
+
+__global__ void label_hist_kernel(const uint32_t *lab, uint32_t n, uint32_t *csize, uint32_t *lrank_tmp) {
+  for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x)
+    atomicAdd(&csize[lab ? lab[v] : 0u], 1u);
+}
+
+__global__ void label_keys_kernel(const uint32_t *lab, uint32_t n, uint64_t *keys) {
+  for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x)
+    keys[v] = ((uint64_t)(lab ? lab[v] : 0u) << 32) | v;
+}
+
+// sorted (label, v) keys -> rank of v inside its label class
+__global__ void label_rank_kernel(const uint64_t *sorted, uint32_t n, uint32_t *lrank) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t l = (uint32_t)(sorted[i] >> 32);
+    // class start: binary search for the first key with this label
+    uint64_t lo = 0, hi = i;
+    while (lo < hi) {
+      const uint64_t mid = (lo + hi) >> 1;
+      if ((uint32_t)(sorted[mid] >> 32) < l) lo = mid + 1; else hi = mid;
+    }
+    lrank[(uint32_t)sorted[i]] = (uint32_t)(i - lo);
+  }
+}
+
+__global__ void max_label_kernel(const uint32_t *lab, uint32_t n, unsigned long long *out) {
+  unsigned long long m = 0;
+  for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x)
+    m = lab[v] > m ? lab[v] : m;
+  for (int o = 16; o > 0; o >>= 1) {
+    const unsigned long long x = __shfl_down_sync(0xffffffffu, m, o);
+    m = x > m ? x : m;
+  }
+  if ((threadIdx.x & 31) == 0) atomicMax(out, m);
+}
+
+inline unsigned g1d(uint64_t n) {
+  const uint64_t b = (n + 255) / 256;
+  return (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(b, 148u * 32u));
+}
+
+}  // namespace
+
+static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::vector<gamma_fpm_pattern> &out) {
+  gamma_ctx *ctx = g->ctx;
+  const uint32_t n = g->n;
+  // ---- label classes: sizes and in-class ranks ----
+  uint32_t nlab = 1;
+  if (g->labels) {
+    GAMMA_CUDA(cudaMemsetAsync(ctx->ctrl + CTRL_AUX1, 0, 8, ctx->stream));
+    ctx->launch(KC_FPM, [&] {
+      max_label_kernel<<<g1d(n), 256, 0, ctx->stream>>>(g->labels, n, (unsigned long long *)(ctx->ctrl + CTRL_AUX1));
+    });
+    uint64_t ml = 0;
+    GAMMA_CUDA(cudaMemcpyAsync(&ml, ctx->ctrl + CTRL_AUX1, 8, cudaMemcpyDeviceToHost, ctx->stream));
+    ctx->sync();
+    GAMMA_REQUIRE(ml < 65536, GAMMA_E_UNSUPPORTED, "gamma_fpm: labels must be < 65536");
+    nlab = (uint32_t)ml + 1;
+  }
+  DevBuf<uint32_t> csize(ctx, nlab), lrank(ctx, n);
+  GAMMA_CUDA(cudaMemsetAsync(csize.p, 0, nlab * 4, ctx->stream));
+  ctx->launch(KC_FPM, [&] { label_hist_kernel<<<g1d(n), 256, 0, ctx->stream>>>(g->labels, n, csize.p, nullptr); });
+  {
+    DevBuf<uint64_t> k0(ctx, n), k1(ctx, n);
+    ctx->launch(KC_FPM, [&] { label_keys_kernel<<<g1d(n), 256, 0, ctx->stream>>>(g->labels, n, k0.p); });
+    size_t tmp = 0;
+    int endbit = 32;
+    while (endbit < 64 && (1ull << (endbit - 32)) <= nlab) endbit++;
+    GAMMA_CUDA(cub::DeviceRadixSort::SortKeys(nullptr, tmp, k0.p, k1.p, (uint64_t)n, 0, endbit, ctx->stream));
+    DevBuf<uint8_t> t(ctx, tmp);
+    ctx->launch(KC_FPM, [&] {
+      GAMMA_CUDA(cub::DeviceRadixSort::SortKeys(t.p, tmp, k0.p, k1.p, (uint64_t)n, 0, endbit, ctx->stream));
+    });
+    ctx->launch(KC_FPM, [&] { label_rank_kernel<<<g1d(n), 256, 0, ctx->stream>>>(k1.p, n, lrank.p); });
+  }
+  // ---- pattern table + domain pool ----
+  size_t fr = 0, tot = 0;
+  GAMMA_CUDA(cudaMemGetInfo(&fr, &tot));
+  const uint64_t budget = ctx->desc.hbm_budget_bytes ? ctx->desc.hbm_budget_bytes : (uint64_t)(fr * 0.6);
+  std::vector<uint32_t> hsize(nlab);
+  GAMMA_CUDA(cudaMemcpyAsync(hsize.data(), csize.p, nlab * 4, cudaMemcpyDeviceToHost, ctx->stream));
+  ctx->sync();
+  uint64_t maxw = 0;
+  for (auto c : hsize) maxw = std::max<uint64_t>(maxw, (c + 31) / 32);
+  // capacity: distinct patterns are bounded by the label combinations seen; start
+  // from min(#labels^2 * 64, 2^22) slots and size the pool to the budget
+  uint64_t cap = 1;
+  const uint64_t want = std::min<uint64_t>((uint64_t)nlab * nlab * 64 + 1024, 1ull << 22);
+  while (cap < want) cap <<= 1;
+  const uint64_t slot_bytes = 4 + 8 + 8 + 32 + 8 + 4;
+  const uint64_t pool_min = 4 * maxw + 64;
+  uint64_t pool_words = std::min<uint64_t>(cap * 2 * std::max<uint64_t>(maxw, 1), 1ull << 28);
+  DevBuf<uint32_t> st, freq, pool;
+  DevBuf<unsigned long long> klo, khi, dom, sup, pcur;
+  FpmArgs a{};
+  for (int attempt = 0;; attempt++) {
+  pool_words = std::max<uint64_t>(std::min<uint64_t>(pool_words, (budget - std::min(budget, cap * slot_bytes)) / 4),
+                                  pool_min);
+  st.reset(); freq.reset(); pool.reset(); klo.reset(); khi.reset(); dom.reset(); sup.reset(); pcur.reset();
+  st = DevBuf<uint32_t>(ctx, cap);
+  freq = DevBuf<uint32_t>(ctx, cap);
+  pool = DevBuf<uint32_t>(ctx, pool_words);
+  klo = DevBuf<unsigned long long>(ctx, cap);
+  khi = DevBuf<unsigned long long>(ctx, cap);
+  dom = DevBuf<unsigned long long>(ctx, cap * 4);
+  sup = DevBuf<unsigned long long>(ctx, cap);
+  pcur = DevBuf<unsigned long long>(ctx, 1);
+  GAMMA_CUDA(cudaMemsetAsync(st.p, 0, cap * 4, ctx->stream));
+  GAMMA_CUDA(cudaMemsetAsync(pool.p, 0, pool_words * 4, ctx->stream));
+  GAMMA_CUDA(cudaMemsetAsync(pcur.p, 0, 8, ctx->stream));
+  a.rp = g->row_ptr;
+  a.col = g->col;
+  a.lab = g->labels;
+  a.lrank = lrank.p;
+  a.csize = csize.p;
+  a.n = n;
+  a.rank = 0;
+  a.world = 1;   // FPM runs every root on every rank (replicas)
+  a.T = Table{st.p, klo.p, khi.p, dom.p, sup.p, freq.p, cap, pool.p, pool_words, pcur.p};
+  a.ctrl = (unsigned long long *)ctx->ctrl;
+  const int grid_enum = ctx->num_sms * occupancy_blocks((const void *)fpm_enum_kernel, kThreads, 0);
+  bool full = false, exhausted = false;
+  for (uint32_t l = 1; l <= max_edges; l++) {
+    a.level = l;
+    ctrl_reset(ctx);
+    ctx->launch(KC_FPM, [&] { fpm_enum_kernel<<<grid_enum, kThreads, 0, ctx->stream>>>(a); });
+    ctx->launch(KC_FPM_SUPPORT, [&] {
+      fpm_support_kernel<<<g1d(cap * 32), 256, 0, ctx->stream>>>(a, l, minsup);
+    });
+    ctrl_fetch(ctx);
+    const uint64_t *h = ctx->ctrl_host;
+    exhausted = h[CTRL_OVF] != 0;
+    full = h[CTRL_ERR] != 0;
+    if (full || exhausted) break;
+    ctx->stats.level_entries[l] = h[CTRL_ENTRIES];
+  }
+  if (!full && !exhausted) break;
+  // grow what ran out and start over (rare: sizes are only known after the fact)
+  ctx->stats.retries++;
+  const uint64_t max_bytes = budget;
+  if (full) {
+    GAMMA_REQUIRE(cap * 4 * slot_bytes + pool_min * 4 <= max_bytes, GAMMA_E_NOMEM,
+                  "gamma_fpm: pattern table full (raise hbm_budget_bytes)");
+    cap *= 4;
+  }
+  if (exhausted) {
+    GAMMA_REQUIRE(pool_words * 4 * 2 + cap * slot_bytes <= max_bytes || pool_words * 4 + cap * slot_bytes < max_bytes,
+                  GAMMA_E_NOMEM, "gamma_fpm: MNI domain pool exhausted (raise hbm_budget_bytes)");
+    GAMMA_REQUIRE(attempt < 12, GAMMA_E_NOMEM, "gamma_fpm: MNI domain pool exhausted");
+    pool_words *= 4;
+  }
+  }
+  // ---- collect the frequent patterns ----
+  std::vector<uint32_t> hst(cap), hfreq(cap);
+  std::vector<unsigned long long> hlo(cap), hhi(cap), hsup(cap);
+  GAMMA_CUDA(cudaMemcpyAsync(hst.data(), st.p, cap * 4, cudaMemcpyDeviceToHost, ctx->stream));
+  GAMMA_CUDA(cudaMemcpyAsync(hfreq.data(), freq.p, cap * 4, cudaMemcpyDeviceToHost, ctx->stream));
+  GAMMA_CUDA(cudaMemcpyAsync(hlo.data(), klo.p, cap * 8, cudaMemcpyDeviceToHost, ctx->stream));
+  GAMMA_CUDA(cudaMemcpyAsync(hhi.data(), khi.p, cap * 8, cudaMemcpyDeviceToHost, ctx->stream));
+  GAMMA_CUDA(cudaMemcpyAsync(hsup.data(), sup.p, cap * 8, cudaMemcpyDeviceToHost, ctx->stream));
+  ctx->sync();
+  static const uint8_t pairs[6][2] = {{0, 1}, {0, 2}, {0, 3}, {1, 2}, {1, 3}, {2, 3}};
+  for (uint64_t s = 0; s < cap; s++) {
+    if (hst[s] != 2 || !hfreq[s]) continue;
+    gamma_fpm_pattern p{};
+    p.nv = (uint32_t)(hhi[s] & 0xf);
+    p.ne = (uint32_t)((hhi[s] >> 4) & 0xf);
+    const uint32_t key = (uint32_t)(hhi[s] >> 8);
+    const uint32_t idx[3] = {key / 64, (key / 8) % 8, key % 8};
+    for (uint32_t i = 0; i < p.nv; i++) p.labels[i] = (uint32_t)((hlo[s] >> (16 * i)) & 0xffff);
+    for (uint32_t e = 0; e < p.ne; e++) {
+      const uint32_t id = idx[e];   // sorted pair indices first, unused slots hold 7
+      p.edges[e][0] = pairs[id][0];
+      p.edges[e][1] = pairs[id][1];
+    }
+    p.support = hsup[s];
+    out.push_back(p);
+  }
+  std::sort(out.begin(), out.end(), [](const gamma_fpm_pattern &x, const gamma_fpm_pattern &y) {
+    if (x.ne != y.ne) return x.ne < y.ne;
+    if (x.nv != y.nv) return x.nv < y.nv;
+    for (uint32_t i = 0; i < x.nv; i++)
+      if (x.labels[i] != y.labels[i]) return x.labels[i] < y.labels[i];
+    for (uint32_t e = 0; e < x.ne; e++) {
+      if (x.edges[e][0] != y.edges[e][0]) return x.edges[e][0] < y.edges[e][0];
+      if (x.edges[e][1] != y.edges[e][1]) return x.edges[e][1] < y.edges[e][1];
+    }
+    return false;
+  });
+  ctx->collect_timings();
+}
+
+}  // namespace gamma_impl
 
 using namespace gamma_impl;
 
-extern "C" gamma_status gamma_fpm(gamma_graph *g, uint32_t max_edges, uint64_t minsup,
-                                  gamma_fpm_result **out) {
+extern "C" gamma_status gamma_fpm(gamma_graph *g, uint32_t max_edges, uint64_t minsup, gamma_fpm_result **out) {
   return guarded([&] {
     GAMMA_REQUIRE(g && out, GAMMA_E_INVAL, "gamma_fpm: NULL argument");
-    throw Fail{GAMMA_E_UNSUPPORTED, "gamma_fpm: not implemented yet"};
+    GAMMA_REQUIRE(minsup >= 1, GAMMA_E_INVAL, "gamma_fpm: minsup must be >= 1");
+    GAMMA_REQUIRE(max_edges >= 1, GAMMA_E_INVAL, "gamma_fpm: max_edges must be >= 1");
+    GAMMA_REQUIRE(max_edges <= 3, GAMMA_E_UNSUPPORTED, "gamma_fpm: max_edges > 3 not supported in v1");
+    gamma_ctx *c = g->ctx;
+    GAMMA_CUDA(cudaSetDevice(c->device));
+    c->reset_stats();
+    std::vector<gamma_fpm_pattern> pats;
+    fpm_run(g, max_edges, minsup, pats);
+    auto *r = new gamma_fpm_result();
+    r->n = pats.size();
+    r->pats = new gamma_fpm_pattern[pats.size() ? pats.size() : 1];
+    std::copy(pats.begin(), pats.end(), r->pats);
+    *out = r;
   });
 }
 

@@ -68,6 +68,7 @@ enum KernelClass {
   KC_FPM,            // FPM edge extension / canonical code / domain bits
   KC_FPM_SUPPORT,    // FPM popc / min over orbits
   KC_MISC,           // memsets, small helpers
+  KC_BITMAP,         // kCL local-bitmap path (depth-2 list intersection + bitmap DFS)
   KC_NUM
 };
 extern const char *kKernelClassName[KC_NUM];
@@ -201,4 +202,9 @@ void build_dag(gamma_graph *g, uint64_t *sorted_keys_dev, uint64_t nkeys);
 // kCL (kclique.cu)
 uint64_t kclique_count(gamma_graph *g, uint32_t k, const uint32_t *roots_dev, uint64_t nroots,
                        uint64_t *per_root_dev);
+// kCL local-bitmap path for roots with |N+(v)| <= kBitmapMaxRun (kclique_bitmap.cu)
+constexpr uint32_t kBitmapMaxRun = 512;
+constexpr uint32_t kBitmapMaxK = 12;
+uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint64_t nroots,
+                        unsigned long long *per_root);
 }  // namespace gamma_impl

@@ -71,6 +71,7 @@ struct KclArgs {
   unsigned long long *per_root;
   uint32_t batch;
   uint32_t stage_cap;         // kRunCap (0: GAMMA_FLAG_DEBUG_NOSTAGE)
+  uint32_t root_len_gt;       // depth 1: only roots with |N+(v)| > this (bitmap path took the rest)
 };
 
 struct Counters {
@@ -250,6 +251,7 @@ __global__ void __launch_bounds__(kThreads) kcl_kernel(KclArgs a) {
         if (PER_ROOT) root_idx = a.groot_in[gi];
       }
       if (len < a.need_group) continue;
+      if (ROOT && len <= a.root_len_gt) continue;
       ct.in_entries += (lane == 0) ? len : 0;
       uint64_t gacc = 0;
       if (len > a.stage_cap) {
@@ -420,6 +422,7 @@ struct KclRun {
   const uint32_t *roots;
   uint64_t nroots;
   unsigned long long *per_root_out;
+  uint32_t root_len_gt = 0;
   std::vector<Level> levels;   // levels[d] holds groups at depth d (d >= 2)
   uint64_t level_share;        // bytes allowed per level table
   uint64_t total = 0;
@@ -453,6 +456,7 @@ struct KclRun {
     a.ctrl = (unsigned long long *)ctx->ctrl;
     a.per_root = per_root_out;
     a.stage_cap = (ctx->desc.flags & GAMMA_FLAG_DEBUG_NOSTAGE) ? 0u : kRunCap;
+    a.root_len_gt = root_len_gt;
     a.g_begin = g0;
     a.g_end = g1;
     if (d == 1) {
@@ -681,7 +685,12 @@ uint64_t kclique_count(gamma_graph *g, uint32_t k, const uint32_t *roots_dev, ui
                                                        kThreads, kcl_smem(MODE_COUNT));
   R.grid[MODE_FUSED] = ctx->num_sms * occupancy_blocks((const void *)kcl_kernel<MODE_FUSED, false, false>,
                                                        kThreads, kcl_smem(MODE_FUSED));
-  if (R.nroots) R.process(1, 0, R.nroots);
+  const bool bitmap = (ctx->desc.flags & GAMMA_FLAG_NO_BITMAP) == 0 && k >= 3 && k <= kBitmapMaxK;
+  if (bitmap && R.nroots) {
+    R.add_count(kclique_bitmap(g, k, R.roots, R.nroots, R.per_root_out));
+    R.root_len_gt = kBitmapMaxRun;
+  }
+  if (R.nroots && (!bitmap || g->max_out_degree > kBitmapMaxRun)) R.process(1, 0, R.nroots);
   ctx->sync();
   ctx->collect_timings();
   return R.total;

@@ -1,0 +1,304 @@
+// kclique_bitmap.cu -- k-clique counting, local-bitmap fast path (DFS inside a root).
+//
+// Opt 2 of PAPER.md (L269-278) computes L_m, the intersection of the prefix's
+// lists, once per group and intersects every child's list with it.  Under the
+// degree-ordered DAG, every candidate set below a root v is a subset of the root's
+// run R = N+(v): C(v, c1, ..., ct) = R ∩ N+(c1) ∩ ... ∩ N+(ct).  So this path
+// intersects each child's list with R exactly once (the depth-2 extension, the only
+// step that reads adjacency lists) and stores the result as a bitmap row over R's
+// positions; every deeper extension is then a W-word AND of rows, and the last one
+// is a popcount (the last extension is counted, not stored).  The
+// embedding table below the root is held as these bitmaps, in shared memory, and
+// walked depth-first per thread (BFS across roots, DFS inside a root).
+//
+// Teams: one warp per root for |R| <= 128 (rows of <= 4 words), one CTA per root for
+// 128 < |R| <= 512 (<= 16 words).  Longer runs (and k > 12) use the ET-level path
+// in kclique.cu.
+#include <algorithm>
+
+#include "device_common.cuh"
+#include "internal.cuh"
+
+namespace gamma_impl {
+
+namespace {
+
+constexpr int kMaxStack = 10;   // DFS levels below the first child: k <= 12
+
+struct BmArgs {
+  const uint64_t *dag_ptr;
+  const uint32_t *dag_col;
+  const uint32_t *roots;
+  uint64_t nroots;
+  uint32_t k;
+  uint32_t len_lo, len_hi;    // this launch handles roots with len_lo < |R| <= len_hi
+  unsigned long long *ctrl;
+  unsigned long long *per_root;
+};
+
+__device__ __forceinline__ uint32_t excl_scan32(uint32_t x, int lane, uint32_t &total) {
+  uint32_t s = x;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(0xffffffffu, s, o);
+    if (lane >= o) s += y;
+  }
+  total = __shfl_sync(0xffffffffu, s, 31);
+  return s - x;
+}
+
+// Position of y in sorted s[0..len) or -1.
+__device__ __forceinline__ int find_pos(const uint32_t *s, uint32_t len, uint32_t y) {
+  uint32_t base = 0, n = len;
+  while (n > 1) {
+    const uint32_t half = n >> 1;
+    base = (s[base + half] <= y) ? base + half : base;
+    n -= half;
+  }
+  return s[base] == y ? (int)base : -1;
+}
+
+template <int TW>
+__device__ __forceinline__ int next_bit(const uint32_t (&bm)[TW], uint32_t pos, uint32_t W) {
+#pragma unroll
+  for (int w = 0; w < TW; w++) {
+    if (w < (int)W && (uint32_t)(w + 1) * 32 > pos) {
+      uint32_t word = bm[w];
+      if ((uint32_t)w * 32 < pos) word &= ~0u << (pos & 31);
+      if (word) return w * 32 + __ffs(word) - 1;
+    }
+  }
+  return -1;
+}
+
+template <int TW>
+__device__ __forceinline__ uint32_t popc_and(const uint32_t (&x)[TW], const uint32_t *row, uint32_t W,
+                                             uint32_t (&out)[TW]) {
+  uint32_t c = 0;
+#pragma unroll
+  for (int w = 0; w < TW; w++) {
+    out[w] = (w < (int)W) ? (x[w] & row[w]) : 0u;
+    c += __popc(out[w]);
+  }
+  return c;
+}
+
+// Count the k-cliques whose two lowest vertices are (v, R[j1]): DFS over the bitmap
+// rows B (stride W words), starting from cur = B[j1].
+template <int TW>
+__device__ uint64_t dfs_from(const uint32_t *B, uint32_t W, uint32_t j1, uint32_t k) {
+  uint32_t cur[TW];
+  uint32_t c0 = 0;
+#pragma unroll
+  for (int w = 0; w < TW; w++) {
+    cur[w] = (w < (int)W) ? B[j1 * W + w] : 0u;
+    c0 += __popc(cur[w]);
+  }
+  if (k == 3) return c0;
+  if (c0 < k - 2) return 0;
+  uint64_t cnt = 0;
+  if (k == 4) {   // sum over j in cur of |cur ∩ B_j|
+    uint32_t pos = 0;
+    for (;;) {
+      const int j = next_bit<TW>(cur, pos, W);
+      if (j < 0) break;
+      pos = j + 1;
+      uint32_t nx[TW];
+      cnt += popc_and<TW>(cur, B + j * W, W, nx);
+    }
+    return cnt;
+  }
+  uint32_t stk[kMaxStack][TW];
+  uint32_t pos[kMaxStack];
+#pragma unroll
+  for (int w = 0; w < TW; w++) stk[0][w] = cur[w];
+  pos[0] = 0;
+  int s = 0;
+  while (s >= 0) {
+    uint32_t top[TW];
+#pragma unroll
+    for (int w = 0; w < TW; w++) top[w] = stk[s][w];
+    const int j = next_bit<TW>(top, pos[s], W);
+    if (j < 0) {
+      s--;
+      continue;
+    }
+    pos[s] = j + 1;
+    const uint32_t t = s + 3;            // vertices chosen after taking j
+    uint32_t nx[TW];
+    const uint32_t c = popc_and<TW>(top, B + j * W, W, nx);
+    if (t == k - 1) {
+      cnt += c;
+      continue;
+    }
+    if (c < k - t) continue;             // cannot complete a k-clique
+    s++;
+#pragma unroll
+    for (int w = 0; w < TW; w++) stk[s][w] = nx[w];
+    pos[s] = 0;
+  }
+  return cnt;
+}
+
+template <int TEAM_WARPS>
+__device__ __forceinline__ void team_sync() {
+  if (TEAM_WARPS == 1) __syncwarp();
+  else __syncthreads();
+}
+
+template <int TEAM_WARPS, int TW, bool PER_ROOT>
+__global__ void __launch_bounds__(256) kcl_bitmap_kernel(BmArgs a) {
+  extern __shared__ uint32_t smem[];
+  constexpr int kTeamThreads = TEAM_WARPS * 32;
+  constexpr int kRunMax = TW * 32;
+  const int lane = threadIdx.x & 31;
+  const int team = threadIdx.x / kTeamThreads;
+  const int tid = threadIdx.x % kTeamThreads;
+  const int wit = tid >> 5;   // warp index inside the team
+  uint32_t *R = smem + team * (kRunMax + kRunMax * TW + 1);
+  uint32_t *B = R + kRunMax;
+  uint32_t *slot = B + kRunMax * TW;   // work index broadcast (CTA teams)
+  uint64_t total = 0, elems = 0, entries = 0;
+
+  for (;;) {
+    unsigned long long gi = 0;
+    if (tid == 0) gi = atomicAdd(&a.ctrl[CTRL_WORK], 1ull);
+    if (TEAM_WARPS == 1) {
+      gi = __shfl_sync(0xffffffffu, gi, 0);
+    } else {
+      if (tid == 0) *slot = gi < 0xffffffffull ? (uint32_t)gi : 0xffffffffu;
+      __syncthreads();
+      gi = *slot;
+      __syncthreads();
+    }
+    if (gi >= a.nroots) break;
+    const uint32_t v = a.roots[gi];
+    const uint64_t b0 = a.dag_ptr[v];
+    const uint32_t L = (uint32_t)(a.dag_ptr[v + 1] - b0);
+    if (L <= a.len_lo || L > a.len_hi || L < a.k - 1) continue;   // uniform across the team
+    const uint32_t W = (L + 31) >> 5;
+    for (uint32_t i = tid; i < L; i += kTeamThreads) R[i] = a.dag_col[b0 + i];
+    for (uint32_t i = tid; i < L * W; i += kTeamThreads) B[i] = 0u;
+    if (tid == 0) entries += L;
+    team_sync<TEAM_WARPS>();
+    const uint32_t rmin = R[0], rmax = R[L - 1];
+    // ---- depth-2 extension: row i = positions of R ∩ N+(R[i]) (flattened windows) ----
+    uint64_t hits = 0;
+    for (uint32_t w0 = wit * 32; w0 < L; w0 += TEAM_WARPS * 32) {
+      const uint32_t i = w0 + lane;
+      uint32_t beg = 0, dl = 0;
+      if (i < L) {
+        const uint32_t c = R[i];
+        const uint64_t cb = a.dag_ptr[c];
+        dl = (uint32_t)(a.dag_ptr[c + 1] - cb);
+        beg = (uint32_t)cb;
+      }
+      elems += dl;
+      uint32_t T;
+      const uint32_t o = excl_scan32(dl, lane, T);
+      for (uint32_t t0 = 0; t0 < T; t0 += 32) {
+        const uint32_t t = t0 + lane;
+        int j = 0;
+#pragma unroll
+        for (int step = 16; step > 0; step >>= 1) {
+          const uint32_t oc = __shfl_sync(0xffffffffu, o, (j + step) & 31);
+          if (j + step < 32 && oc <= t) j += step;
+        }
+        const uint32_t bj = __shfl_sync(0xffffffffu, beg, j);
+        const uint32_t oj = __shfl_sync(0xffffffffu, o, j);
+        int p = -1;
+        if (t < T) {
+          const uint32_t y = __ldg(a.dag_col + bj + (t - oj));
+          if (y >= rmin && y <= rmax) p = find_pos(R, L, y);
+        }
+        if (p >= 0) atomicOr(&B[(w0 + j) * W + (p >> 5)], 1u << (p & 31));
+        hits += __popc(__ballot_sync(0xffffffffu, p >= 0)) * (lane == 0);
+      }
+    }
+    team_sync<TEAM_WARPS>();
+    // ---- deeper extensions: bitmap DFS, one first-level child per thread ----
+    uint64_t cnt = 0;
+    if (a.k == 3) {
+      cnt = hits;
+    } else {
+      for (uint32_t j1 = tid; j1 < L; j1 += kTeamThreads) cnt += dfs_from<TW>(B, W, j1, a.k);
+    }
+    total += cnt;
+    if (PER_ROOT) {
+#pragma unroll
+      for (int off = 16; off > 0; off >>= 1) cnt += __shfl_down_sync(0xffffffffu, cnt, off);
+      if (lane == 0 && cnt) atomicAdd(&a.per_root[gi], (unsigned long long)cnt);
+    }
+    team_sync<TEAM_WARPS>();   // R/B are rewritten by the next root
+  }
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) {
+    total += __shfl_down_sync(0xffffffffu, total, off);
+    elems += __shfl_down_sync(0xffffffffu, elems, off);
+    entries += __shfl_down_sync(0xffffffffu, entries, off);
+  }
+  if (lane == 0) {
+    if (total) atomicAdd(&a.ctrl[CTRL_COUNT], (unsigned long long)total);
+    atomicAdd(&a.ctrl[CTRL_ELEMS], (unsigned long long)elems);
+    atomicAdd(&a.ctrl[CTRL_AUX0], (unsigned long long)entries);
+  }
+}
+
+template <int TEAM_WARPS, int TW>
+constexpr size_t bm_smem() {
+  return (size_t)(256 / (TEAM_WARPS * 32)) * (TW * 32 + TW * 32 * TW + 1) * sizeof(uint32_t);
+}
+
+template <int TEAM_WARPS, int TW>
+uint64_t run_bitmap(gamma_ctx *ctx, const BmArgs &a0, bool per_root) {
+  static bool attr = false;
+  if (!attr) {
+    GAMMA_CUDA(cudaFuncSetAttribute(kcl_bitmap_kernel<TEAM_WARPS, TW, false>,
+                                    cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bm_smem<TEAM_WARPS, TW>()));
+    GAMMA_CUDA(cudaFuncSetAttribute(kcl_bitmap_kernel<TEAM_WARPS, TW, true>,
+                                    cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bm_smem<TEAM_WARPS, TW>()));
+    attr = true;
+  }
+  const size_t smem = bm_smem<TEAM_WARPS, TW>();
+  const int grid = ctx->num_sms * occupancy_blocks((const void *)kcl_bitmap_kernel<TEAM_WARPS, TW, false>, 256, smem);
+  ctrl_reset(ctx);
+  ctx->launch(KC_BITMAP, [&] {
+    if (per_root)
+      kcl_bitmap_kernel<TEAM_WARPS, TW, true><<<grid, 256, smem, ctx->stream>>>(a0);
+    else
+      kcl_bitmap_kernel<TEAM_WARPS, TW, false><<<grid, 256, smem, ctx->stream>>>(a0);
+  });
+  ctrl_fetch(ctx);
+  const uint64_t *h = ctx->ctrl_host;
+  ctx->stats.list_elems += h[CTRL_ELEMS];
+  ctx->stats.level_entries[2] += h[CTRL_AUX0];
+  ctx->stats.alg_bytes[KC_BITMAP] += 4 * h[CTRL_AUX0] + 4 * h[CTRL_ELEMS];
+  return h[CTRL_COUNT];
+}
+
+}  // namespace
+
+// Count k-cliques rooted at roots[0..nroots) whose run length is <= 512 (k <= 12);
+// longer runs are left to the ET path.  per_root (nullable) indexed like roots.
+uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint64_t nroots,
+                        unsigned long long *per_root) {
+  gamma_ctx *ctx = g->ctx;
+  BmArgs a{};
+  a.dag_ptr = g->dag_ptr;
+  a.dag_col = g->dag_col;
+  a.roots = roots;
+  a.nroots = nroots;
+  a.k = k;
+  a.ctrl = (unsigned long long *)ctx->ctrl;
+  a.per_root = per_root;
+  uint64_t total = 0;
+  a.len_lo = 128;
+  a.len_hi = 512;
+  if (g->max_out_degree > 128) total = checked_add(total, run_bitmap<8, 16>(ctx, a, per_root != nullptr));
+  a.len_lo = 0;
+  a.len_hi = 128;
+  total = checked_add(total, run_bitmap<1, 4>(ctx, a, per_root != nullptr));
+  return total;
+}
+
+}  // namespace gamma_impl

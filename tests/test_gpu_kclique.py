@@ -123,9 +123,9 @@ def test_per_root_counts(ctx, oracle_mod):
 
 
 def test_budget_forced_splits(G, oracle_mod):
-    n, s, d, _ = gg.config_graph("c1", seed=1)
+    n, s, d, _ = gg.config_graph("c1", seed=1, scale=11)
     o = oracle_mod.Graph(n, s, d)
-    c = G.Context(hbm_budget_bytes=3 << 20)   # ~3 MB of ET: forces range splits
+    c = G.Context(hbm_budget_bytes=3 << 20, flags=0x10)   # ET path, ~3 MB of ET: forces range splits
     g = c.load_edges(n, s, d)
     for k in (4, 5, 6):
         assert g.kclique(k) == o.kclique(k)
@@ -182,7 +182,7 @@ def test_unstaged_long_run_path(G, oracle_mod):
     """Runs longer than the shared-memory staging buffer take the global-memory
     probe and the direct-reservation write path; the debug flag forces that path
     for every group so it is checked on ordinary inputs."""
-    c = G.Context(flags=0x8)   # GAMMA_FLAG_DEBUG_NOSTAGE
+    c = G.Context(flags=0x8 | 0x10)   # GAMMA_FLAG_DEBUG_NOSTAGE | GAMMA_FLAG_NO_BITMAP
     for seed in (1, 2):
         n, s, d, _ = gg.config_graph("c1", seed=seed)
         g = c.load_edges(n, s, d)
@@ -191,10 +191,12 @@ def test_unstaged_long_run_path(G, oracle_mod):
             assert g.kclique(k) == o.kclique(k)
 
 
-def test_hub_out_list_longer_than_staging(ctx, oracle_mod):
-    """A real vertex with d+(v) > 1024: v joined to 1100 vertices of K_{1100,1101}'s
-    larger side (those outrank v), plus a sprinkle of edges among them."""
-    a, b = 1100, 1101
+@pytest.mark.parametrize("a", [200, 1100])
+def test_hub_out_list_longer_than_staging(ctx, oracle_mod, a):
+    """A real vertex with a long DAG out-list: v joined to the a vertices of one side
+    of K_{a,a+1} (those outrank v), plus a sprinkle of edges among them.  a=200
+    takes the CTA-team bitmap path, a=1100 the ET path with an unstaged run."""
+    b = a + 1
     U = np.arange(1, 1 + a)
     F = np.arange(1 + a, 1 + a + b)
     e = [(0, u) for u in U] + [(u, f) for u in U for f in F[:b]]
@@ -203,11 +205,25 @@ def test_hub_out_list_longer_than_staging(ctx, oracle_mod):
     e = np.array(e + [tuple(x) for x in extra], dtype=np.uint32)
     n = 1 + a + b
     g = ctx.load_edges(n, e[:, 0].copy(), e[:, 1].copy())
-    assert g.info()["max_out_degree"] > 1024
+    assert g.info()["max_out_degree"] >= a
     o = oracle_mod.Graph(n, e[:, 0].copy(), e[:, 1].copy())
     roots = np.array([0], np.uint32)
     for k in (3, 4):
         assert np.array_equal(g.kclique_roots(k, roots), o.kclique_roots(k, roots))
+
+
+@pytest.mark.parametrize("flags", [0, 0x10, 0x2 | 0x10])
+def test_paths_agree(G, oracle_mod, flags):
+    """Bitmap DFS (default), ET levels with the fused tail (NO_BITMAP), and ET levels
+    with every level materialised (NO_FUSE | NO_BITMAP) all equal the oracle."""
+    c = G.Context(flags=flags)
+    n, s, d, _ = gg.config_graph("c1", seed=4)
+    g = c.load_edges(n, s, d)
+    o = oracle_mod.Graph(n, s, d)
+    for k in (3, 4, 5, 6, 7):
+        assert g.kclique(k) == o.kclique(k), (flags, k)
+    roots = np.arange(0, n, 3, dtype=np.uint32)
+    assert np.array_equal(g.kclique_roots(5, roots), o.kclique_roots(5, roots))
 
 
 @pytest.mark.slow

@@ -62,7 +62,7 @@ def test_rmat_vs_oracle(ctx, oracle_mod, seed, q):
     g = ctx.load_edges(n, s, d, lab)
     o = oracle_mod.Graph(n, s, d, lab)
     nv, e = Q[q]
-    for plab in ([0] * nv, [i % 8 for i in range(nv)], None):
+    for plab in ([0] * nv, [i % 8 for i in range(nv)], [i % 2 for i in range(nv)]):
         got = g.match(nv, e, plab)
         want = o.match(nv, e, plab)
         assert got == (want[0], want[1]), (q, plab)
