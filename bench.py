@@ -5,10 +5,13 @@ Default workload (N=1): configs[1], k-clique counting k = 4, 5, 6 on the
 cit-Patents-shaped R-MAT (scale 22, a,b,c = 0.53,0.20,0.20, 16.6M raw samples,
 seed 1).  One step = the whole hot path on one synthetic batch: A1 CSR + DAG build
 from the raw edge samples resident in HBM, then gamma_kclique(k) for each k
-(A2-A8).  value = sum of the k-clique counts / device time of the step (max over
-ranks), L2 flushed (256 MiB write) between steps.
+(A2-A8).  value = matched embeddings (sum of the k-clique counts) / device time
+of the step (CUDA events, max over ranks), L2 flushed (256 MiB write) between steps.
 
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--workload c2|c1|heavy] [--impl gamma|reference]
+Other workloads (not the default line): c1 (configs[0]), heavy (kCL scaling
+workload), c3 (labeled SM, 4 queries x 2 labelings), c4 (FPM, l=3, MNI).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--workload c2|c1|heavy|c3|c4] [--impl gamma|reference]
 
 Multi-GPU: torchrun one rank per GPU; roots are partitioned (snake-LPT on cost),
 the CSR is replicated, one NCCL SUM all-reduce per count.
@@ -31,14 +34,35 @@ import numpy as np  # noqa: E402
 
 METRIC = "matched embeddings/s (kCL, SM, FPM) at 1/2/4/8 B200; % of HBM-BW roofline"
 UNIT = "embeddings/s"
+COMPUTE_CLASSES = ("extend", "count", "fused", "bitmap", "sm_extend", "sm_count", "fpm")
+
+SM_QUERIES = ["c4", "diamond", "tailed_triangle", "house"]
 
 WORKLOADS = {
-    # name: (gamma_gen config, ks, description)
-    "c2": ("c2", (4, 5, 6), "configs[1]: kCL k=4,5,6 on cit-Patents-shaped R-MAT scale 22 "
-                            "(a,b,c=0.53,0.20,0.20), 16.6M raw samples, seed 1"),
-    "c1": ("c1", (4,), "configs[0]: 4-clique count on R-MAT scale 12 (0.57,0.19,0.19), 90K samples, seed 1"),
-    "heavy": ("heavy", (4, 5), "heavy kCL: Graph500-skew R-MAT scale 22 (0.57,0.19,0.19), 20M samples, k=4,5"),
+    "c2": {"kind": "kcl", "cfg": "c2", "ks": (4, 5, 6),
+           "desc": "configs[1]: kCL k=4,5,6 on cit-Patents-shaped R-MAT scale 22 (a,b,c=0.53,0.20,0.20), "
+                   "16.6M raw samples, seed 1"},
+    "c1": {"kind": "kcl", "cfg": "c1", "ks": (4,),
+           "desc": "configs[0]: 4-clique count on R-MAT scale 12 (0.57,0.19,0.19), 90K samples, seed 1"},
+    "heavy": {"kind": "kcl", "cfg": "heavy", "ks": (4, 5),
+              "desc": "heavy kCL: Graph500-skew R-MAT scale 22 (0.57,0.19,0.19), 20M samples, k=4,5, seed 1"},
+    "c3": {"kind": "sm", "cfg": "c3",
+           "desc": "configs[2]: labeled SM (4-cycle, diamond, tailed triangle, house) x labels {all 0, i mod 8} "
+                   "on LiveJournal-shaped R-MAT scale 23 (0.50,0.20,0.20), 43.5M samples, L=8, seed 1"},
+    "c4": {"kind": "fpm", "cfg": "c4", "l": 3, "minsup": 3000,
+           "desc": "configs[3]: FPM l=3 edges, MNI minsup=3000, on cit-Patents-shaped R-MAT scale 22 "
+                   "(0.40,0.25,0.25), 16.6M samples, L=37, seed 1"},
 }
+
+
+def sm_runs():
+    import gamma_gen as gg
+    runs = []
+    for q in SM_QUERIES:
+        nv, e = gg.QUERIES[q]
+        runs.append((q, "all0", nv, e, [0] * nv))
+        runs.append((q, "imod8", nv, e, [i % 8 for i in range(nv)]))
+    return runs
 
 
 def peaks():
@@ -135,38 +159,68 @@ def load_traffic(kernel_class: str):
 
 def make_input(name, seed=1):
     import gamma_gen as gg
-    cfg, ks, desc = WORKLOADS[name]
-    n, s, d, lab = gg.config_graph(cfg, seed=seed)
-    return n, s, d, ks, desc
+    w = WORKLOADS[name]
+    n, s, d, lab = gg.config_graph(w["cfg"], seed=seed)
+    return n, s, d, lab, w
 
 
-def cpu_oracle_sample(n, s, d, ks, budget_s=12.0, seed=7):
-    """Time the oracle (as it stands) on a bounded, seeded sample of the workload:
-    the full CSR build, then per-root k-clique counts for a random sample of roots,
-    growing the sample until ~budget_s seconds of counting."""
+# ------------------------------------------------------------------------------------
+# CPU baseline: the oracle, as it stands, on a bounded seeded sample of the workload.
+# ------------------------------------------------------------------------------------
+def cpu_oracle_sample(n, s, d, lab, w, budget_s=12.0, seed=7):
     import oracle
     t0 = time.perf_counter()
-    g = oracle.Graph(n, s, d)
+    g = oracle.Graph(n, s, d, lab)
     t_build = time.perf_counter() - t0
+    cores = os.cpu_count()
     rng = np.random.default_rng(seed)
+    if w["kind"] == "fpm":
+        # the oracle's FPM has no per-root form: time it on the same generator at a
+        # smaller scale until the budget is used
+        import gamma_gen as gg
+        emb, t_count, scale = 0, 0.0, 12
+        while True:
+            ns, ss, ds, ls = gg.config_graph(w["cfg"], seed=seed, scale=scale)
+            gs = oracle.Graph(ns, ss, ds, ls)
+            t1 = time.perf_counter()
+            res = gs.fpm(w["l"], max(1, int(w["minsup"] * 2.0 ** (scale - 22))), pattern_cap=1 << 21)
+            dt = time.perf_counter() - t1
+            emb_l = sum(r[5] for r in res if r[0] == w["l"])
+            if t_count + dt > budget_s * 3 and t_count > 0:
+                break
+            emb, t_count = emb_l, dt
+            if dt >= budget_s / 4 or scale >= 22:
+                break
+            scale += 1
+        return {"value": emb / t_count if t_count else None, "unit": UNIT, "cores": cores, "kind": "oracle",
+                "sample": f"oracle FPM l={w['l']} on the same generator at scale {scale} (minsup scaled by "
+                          f"2^(scale-22)); embeddings counted = frequent-pattern instances at level {w['l']} "
+                          f"({emb}) in {t_count:.2f}s on {cores} OpenMP threads",
+                "embeddings": emb, "seconds": t_count}
     perm = rng.permutation(n).astype(np.uint32)
-    frac, emb, t_count, used = 0.001, 0, 0.0, 0
+    frac, emb, t_count, used = 0.0005, 0.0, 0.0, 0
     while True:
-        cnt = max(1, int(n * frac))
+        cnt = min(max(1, int(n * frac)), n - used)
         roots = perm[used:used + cnt]
         t1 = time.perf_counter()
-        for k in ks:
-            emb += int(g.kclique_roots(k, roots).sum())
+        if w["kind"] == "kcl":
+            for k in w["ks"]:
+                emb += int(g.kclique_roots(k, roots).sum())
+        else:
+            for (q, lname, nv, e, plab) in sm_runs():
+                mp = int(g.match_roots(nv, e, roots, plab).sum())
+                import paper_conf_icde_hu0o23_b200 as G   # |Aut_L| from the host planner (no GPU)
+                emb += mp / G.pattern_plan(nv, e, plab)["aut"]
         t_count += time.perf_counter() - t1
         used += cnt
         if t_count >= budget_s or used >= n:
             break
         frac *= 2
-    cores = os.cpu_count()
+    what = (f"k-clique counts k={list(w['ks'])}" if w["kind"] == "kcl" else
+            "SM mappings / |Aut_L| over the 8 (query, labeling) runs")
     return {"value": emb / t_count if t_count > 0 else None, "unit": UNIT, "cores": cores, "kind": "oracle",
-            "sample": f"oracle k-clique counts k={list(ks)} for a seeded random sample of {used} of {n} roots "
-                      f"({used / n:.2%}; full CSR build {t_build:.2f}s excluded), {emb} embeddings in "
-                      f"{t_count:.2f}s on {cores} OpenMP threads",
+            "sample": f"oracle {what} for a seeded random sample of {used} of {n} roots ({used / n:.2%}; full CSR "
+                      f"build {t_build:.2f}s excluded), {emb:.0f} embeddings in {t_count:.2f}s on {cores} OpenMP threads",
             "embeddings": emb, "seconds": t_count}
 
 
@@ -174,14 +228,11 @@ def run_reference(args):
     rank, world, _ = dist_env()
     if rank != 0:
         return 0
-    n, s, d, ks, desc = make_input(args.workload)
-    for _ in range(args.warmup):
-        pass   # the oracle has no warm state worth warming beyond the first sample
-    vals, secs, embs = [], [], 0
+    n, s, d, lab, w = make_input(args.workload)
+    vals, secs, samples = [], [], []
     per_step_budget = max(2.0, 60.0 / max(1, args.steps + args.warmup))
-    samples = []
     for i in range(args.warmup + args.steps):
-        r = cpu_oracle_sample(n, s, d, ks, budget_s=per_step_budget, seed=11 + i)
+        r = cpu_oracle_sample(n, s, d, lab, w, budget_s=per_step_budget, seed=11 + i)
         if i >= args.warmup:
             vals.append(r["value"])
             secs.append(r["seconds"])
@@ -190,7 +241,7 @@ def run_reference(args):
     out = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": args.gpus,
            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * statistics.median(secs),
            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32/u64 integer",
-           "data": "synthetic", "config": {"workload": desc, "k": list(ks), "parallelism": "cpu-oracle"},
+           "data": "synthetic", "config": {"workload": w["desc"], "parallelism": "cpu-oracle"},
            "cpu_baseline": {"value": v, "unit": UNIT, "cores": samples[0]["cores"], "kind": "oracle",
                             "sample": samples[0]["sample"]},
            "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
@@ -198,6 +249,9 @@ def run_reference(args):
     return 0
 
 
+# ------------------------------------------------------------------------------------
+# The product path.
+# ------------------------------------------------------------------------------------
 def run_gamma(args):
     import torch
     import torch.distributed as dist
@@ -208,70 +262,82 @@ def run_gamma(args):
     dev = torch.cuda.current_device()
     import paper_conf_icde_hu0o23_b200 as G
 
-    n, s, d, ks, desc = make_input(args.workload)
+    n, s, d, lab, w = make_input(args.workload)
     m_raw = s.size
     ctx = G.Context(device=dev, time_kernels=True)
     stream = torch.cuda.current_stream()
     src_dev = torch.from_numpy(s.view(np.int32)).cuda()
     dst_dev = torch.from_numpy(d.view(np.int32)).cuda()
+    lab_dev = None if lab is None else torch.from_numpy(lab.view(np.int32)).cuda()
     src_pin = torch.from_numpy(s.view(np.int32)).pin_memory()
     dst_pin = torch.from_numpy(d.view(np.int32)).pin_memory()
+    lab_pin = None if lab is None else torch.from_numpy(lab.view(np.int32)).pin_memory()
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+    agg = {"_total_launches": {"n": 0}}
 
-    agg = {}
+    def collect():
+        st = ctx.stats()
+        for name, c in st["classes"].items():
+            a = agg.setdefault(name, {"launches": 0, "ms": 0.0, "alg_bytes": 0})
+            for key in a:
+                a[key] += c[key]
+        agg["_total_launches"]["n"] += st["total_launches"]
+        return st
 
-    def step(src, dst, collect):
-        g = ctx.load_edges(n, src, dst)
-        counts = []
-        if collect:
-            st = ctx.stats()
-            for name, c in st["classes"].items():
-                a = agg.setdefault(name, {"launches": 0, "ms": 0.0, "alg_bytes": 0})
-                for key in a:
-                    a[key] += c[key]
-            agg.setdefault("_total_launches", {"n": 0})["n"] += st["total_launches"]
-        for k in ks:
-            counts.append(g.kclique(k))
-            if collect:
-                st = ctx.stats()
-                for name, c in st["classes"].items():
-                    a = agg.setdefault(name, {"launches": 0, "ms": 0.0, "alg_bytes": 0})
-                    for key in a:
-                        a[key] += c[key]
-                agg["_total_launches"]["n"] += st["total_launches"]
+    def step(src, dst, labels, coll):
+        g = ctx.load_edges(n, src, dst, labels)
+        if coll:
+            collect()
+        results = {}
+        if w["kind"] == "kcl":
+            for k in w["ks"]:
+                results[f"k{k}"] = g.kclique(k)
+                if coll:
+                    collect()
+            emb = sum(results.values())
+        elif w["kind"] == "sm":
+            for (q, lname, nv, e, plab) in sm_runs():
+                results[f"{q}/{lname}"] = g.match(nv, e, plab)[0]
+                if coll:
+                    collect()
+            emb = sum(results.values())
+        else:
+            pats = g.fpm(w["l"], w["minsup"])
+            st = collect() if coll else ctx.stats()
+            results = {f"frequent_l{l}": sum(1 for p in pats if p[0] == l) for l in range(1, w["l"] + 1)}
+            emb = st["level_entries"][w["l"]]
+            results["embeddings_l"] = emb
         info = g.info()
         g.free()
-        return counts, info
+        return emb, results, info
 
     def barrier():
         if world > 1:
             dist.barrier()
 
     for _ in range(args.warmup):
-        step(src_dev, dst_dev, False)
+        step(src_dev, dst_dev, lab_dev, False)
     torch.cuda.synchronize()
 
     clocks = ClockSampler(dev)
     clocks.start()
-    times, counts_seen = [], None
+    times, emb, results, info = [], 0, None, None
     for _ in range(args.steps):
         flush.fill_(1)
         barrier()
         torch.cuda.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
-        counts, info = step(src_dev, dst_dev, True)
+        emb, results, info = step(src_dev, dst_dev, lab_dev, True)
         e1.record(stream)
         torch.cuda.synchronize()
         barrier()
         times.append(e0.elapsed_time(e1))
-        counts_seen = counts
     clk = clocks.stop()
     total_ms = max_over_ranks(sum(times), world)
-    emb_per_step = sum(counts_seen)   # all-reduced global counts
-    value = emb_per_step * args.steps / (total_ms / 1000.0)
+    value = emb * args.steps / (total_ms / 1000.0)
 
-    # ---- e2e: same step through the public API from pinned host buffers ----
+    # ---- e2e: the same step through the public API from pinned host buffers ----
     e2e_times = []
     for _ in range(max(1, min(args.steps, 3))):
         flush.fill_(1)
@@ -279,12 +345,12 @@ def run_gamma(args):
         torch.cuda.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
-        c2, _ = step(src_pin, dst_pin, False)   # H2D inside gamma_load_edges; counts D2H per call
+        step(src_pin, dst_pin, lab_pin, False)   # H2D inside gamma_load_edges; results D2H per call
         e1.record(stream)
         torch.cuda.synchronize()
         barrier()
         e2e_times.append(e0.elapsed_time(e1))
-    e2e_value = emb_per_step * len(e2e_times) / (max_over_ranks(sum(e2e_times), world) / 1000.0)
+    e2e_value = emb * len(e2e_times) / (max_over_ranks(sum(e2e_times), world) / 1000.0)
 
     if rank != 0:
         if world > 1:
@@ -292,7 +358,7 @@ def run_gamma(args):
         return 0
 
     hbm, peak_src = peaks()
-    cand = {k: v for k, v in agg.items() if not k.startswith("_") and k in ("extend", "count", "fused")}
+    cand = {k: v for k, v in agg.items() if not k.startswith("_") and k in COMPUTE_CLASSES}
     dom = max(cand, key=lambda k: cand[k]["ms"]) if cand else None
     roof = None
     if dom and cand[dom]["ms"] > 0:
@@ -305,24 +371,25 @@ def run_gamma(args):
                 "share_of_step": cand[dom]["ms"] / total_ms}
     cpu = None
     if world == 1 and not args.no_cpu_baseline:
-        cpu = cpu_oracle_sample(n, s, d, ks, budget_s=args.cpu_seconds)
+        cpu = cpu_oracle_sample(n, s, d, lab, w, budget_s=args.cpu_seconds)
         cpu.pop("embeddings", None)
         cpu.pop("seconds", None)
+    h2d = 2 * 4 * m_raw + (0 if lab is None else 4 * n)
+    nres = len(w.get("ks", ())) or (len(sm_runs()) if w["kind"] == "sm" else 1)
     out = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": total_ms / args.steps, "higher_is_better": True,
         "scaling": "strong", "vs_baseline": None, "dtype": "u32 ids / u64 counts (integer)",
         "data": "synthetic",
-        "config": {"workload": desc, "k": list(ks), "n": n, "m_raw": int(m_raw), "m": int(info["m"]),
+        "config": {"workload": w["desc"], "n": n, "m_raw": int(m_raw), "m": int(info["m"]),
                    "max_degree": info["max_degree"], "max_out_degree": info["max_out_degree"],
-                   "counts": {str(k): c for k, c in zip(ks, counts_seen)},
+                   "results": results, "embeddings_per_step": emb,
                    "l2": "flushed between steps (256 MiB write)",
                    "parallelism": f"root-partition dp{world} (CSR replicated)"},
         "roofline": roof,
         "cpu_baseline": cpu,
-        "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(2 * 4 * m_raw),
-                "d2h_bytes_per_step": int(8 * len(ks))},
-        "gpu_launches": int(agg.get("_total_launches", {"n": 0})["n"]),
+        "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(8 * nres)},
+        "gpu_launches": int(agg["_total_launches"]["n"]),
         "clocks": clk,
         "kernels": {k: v for k, v in agg.items() if not k.startswith("_") and v["launches"]},
         "build_ms_per_step": info["build_ms"],

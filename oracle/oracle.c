@@ -316,6 +316,28 @@ int og_match(const og_graph *g, uint32_t nv, uint32_t ne, const uint32_t *edges,
   return OG_OK;
 }
 
+/* Mappings whose image of BFS-order vertex 0 (pattern vertex 0) is roots[i]; the sum
+ * over all vertices is the `mappings` of og_match.  For sampled timing / parity. */
+int og_match_roots(const og_graph *g, uint32_t nv, uint32_t ne, const uint32_t *edges,
+                   const uint32_t *plabels, uint64_t nroots, const uint32_t *roots, uint64_t *out,
+                   int threads) {
+  og_pat p;
+  int st = pat_init(&p, nv, ne, edges, plabels);
+  if (st) return st;
+  set_threads(threads);
+  uint32_t r = p.order[0];
+#pragma omp parallel for schedule(dynamic, 16)
+  for (int64_t i = 0; i < (int64_t)nroots; i++) {
+    uint32_t v = roots[i];
+    out[i] = 0;
+    if (v >= g->n || (p.labeled && g->lab[v] != p.plab[r])) continue;
+    uint32_t phi[OG_MAXV];
+    phi[r] = v;
+    out[i] = match_rec(g, &p, 1, phi);
+  }
+  return OG_OK;
+}
+
 /* ---------------------------------------------------------------------------
  * O-3: frequent pattern mining, edge-induced patterns of 1..l edges (l <= 3),
  * MNI support.

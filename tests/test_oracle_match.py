@@ -114,6 +114,18 @@ def test_brute_force_subsets(oracle_mod, seed, q):
     assert g.match(nv, e, plab)[1] == brute.mappings(n, E, nv, e, plab, lab)
 
 
+@pytest.mark.parametrize("q", ["c4", "house"])
+def test_match_roots_partition(oracle_mod, q):
+    nv, e = Q[q]
+    n = 64
+    s, d = gg.er(n, 300, 9)
+    lab = gg.labels(n, 2, 9)
+    g = oracle_mod.Graph(n, s, d, lab)
+    plab = [i % 2 for i in range(nv)]
+    per = g.match_roots(nv, e, np.arange(n, dtype=np.uint32), plab)
+    assert int(per.sum()) == g.match(nv, e, plab)[1]
+
+
 def test_disconnected_pattern_rejected(oracle_mod):
     g = G(oracle_mod, gg.complete(5))
     with pytest.raises(ValueError):
