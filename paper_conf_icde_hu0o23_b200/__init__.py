@@ -14,6 +14,8 @@ The C names are re-exported 1:1 (``gamma_ctx_create``, ``gamma_load_edges``,
 from __future__ import annotations
 
 import ctypes as C
+import sys
+import weakref
 from typing import Optional
 
 import numpy as np
@@ -123,6 +125,7 @@ class Context:
                  use_torch: bool = True, hbm_budget_bytes: int = 0, host_spill_bytes: int = 0,
                  time_kernels: bool = False, flags: int = 0, reduce: bool = True):
         self._keep = []
+        self._graphs = weakref.WeakSet()
         d = N.gamma_ctx_desc()
         d.device = device
         self._torch = None
@@ -173,11 +176,19 @@ class Context:
         return self._h
 
     def close(self):
+        """Free every live graph of this context, then the context itself (a graph
+        must never outlive its context, whatever order the garbage collector picks)."""
         if getattr(self, "_h", None):
+            for g in list(getattr(self, "_graphs", ())):
+                g.free()
             _lib.gamma_ctx_destroy(self._h)
             self._h = None
 
     def __del__(self):
+        # at interpreter shutdown the allocator callbacks (into torch) may already be
+        # gone: leak instead of calling back into a half-finalised interpreter
+        if sys.is_finalizing():
+            return
         try:
             self.close()
         except Exception:   # noqa: BLE001
@@ -220,13 +231,17 @@ class Graph:
     def __init__(self, ctx: Context, h):
         self.ctx = ctx
         self._h = h
+        ctx._graphs.add(self)
 
     def free(self):
         if getattr(self, "_h", None):
-            _lib.gamma_graph_free(self._h)
+            if getattr(self.ctx, "_h", None):   # the context still exists
+                _lib.gamma_graph_free(self._h)
             self._h = None
 
     def __del__(self):
+        if sys.is_finalizing():
+            return
         try:
             self.free()
         except Exception:   # noqa: BLE001

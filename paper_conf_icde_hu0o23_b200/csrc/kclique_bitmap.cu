@@ -194,24 +194,36 @@ __global__ void __launch_bounds__(256) kcl_bitmap_kernel(BmArgs a) {
         beg = (uint32_t)cb;
       }
       elems += dl;
+      // compact the children with non-empty lists to lanes 0..nnz-1 (so that every
+      // list has a distinct start offset), then exclusive-scan their lengths
+      const uint32_t nz = __ballot_sync(0xffffffffu, dl > 0);
+      const uint32_t nnz = __popc(nz);
+      const uint32_t src = lane < (int)nnz ? __fns(nz, 0, lane + 1) : 0;
+      const uint32_t cbeg = __shfl_sync(0xffffffffu, beg, src);
+      const uint32_t sdl = __shfl_sync(0xffffffffu, dl, src);
+      const uint32_t cdl = lane < (int)nnz ? sdl : 0u;
+      const uint32_t crow = w0 + src;
       uint32_t T;
-      const uint32_t o = excl_scan32(dl, lane, T);
+      const uint32_t o = excl_scan32(cdl, lane, T);
+      const uint32_t upto = lane == 31 ? 0xffffffffu : ((2u << lane) - 1u);
+      uint32_t nb = 0;   // lists that started before this tile
       for (uint32_t t0 = 0; t0 < T; t0 += 32) {
         const uint32_t t = t0 + lane;
-        int j = 0;
-#pragma unroll
-        for (int step = 16; step > 0; step >>= 1) {
-          const uint32_t oc = __shfl_sync(0xffffffffu, o, (j + step) & 31);
-          if (j + step < 32 && oc <= t) j += step;
-        }
-        const uint32_t bj = __shfl_sync(0xffffffffu, beg, j);
-        const uint32_t oj = __shfl_sync(0xffffffffu, o, j);
+        // lane t's list = the last list starting at or before t: one OR-reduction of
+        // the start offsets that fall in this tile
+        const uint32_t mine = (lane < (int)nnz && o >= t0 && o < t0 + 32) ? (1u << (o - t0)) : 0u;
+        const uint32_t S = __reduce_or_sync(0xffffffffu, mine);
+        const int j = (int)(nb + __popc(S & upto)) - 1;
+        nb += __popc(S);
+        const uint32_t bj = __shfl_sync(0xffffffffu, cbeg, j & 31);
+        const uint32_t oj = __shfl_sync(0xffffffffu, o, j & 31);
+        const uint32_t rj = __shfl_sync(0xffffffffu, crow, j & 31);
         int p = -1;
         if (t < T) {
           const uint32_t y = __ldg(a.dag_col + bj + (t - oj));
           if (y >= rmin && y <= rmax) p = find_pos(R, L, y);
         }
-        if (p >= 0) atomicOr(&B[(w0 + j) * W + (p >> 5)], 1u << (p & 31));
+        if (p >= 0) atomicOr(&B[rj * W + (p >> 5)], 1u << (p & 31));
         hits += __popc(__ballot_sync(0xffffffffu, p >= 0)) * (lane == 0);
       }
     }

@@ -1,0 +1,53 @@
+#!/usr/bin/env python3
+"""Ad-hoc timing probes run on the GPU box (one case per process, under `timeout`).
+
+    python tools/diag.py fpm_gpu|fpm_oracle|sm <index>
+"""
+import os
+import sys
+import time
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import gamma_gen as gg  # noqa: E402
+
+PATS = [(3, [(0, 1), (1, 2), (0, 2)]), (3, [(0, 1), (1, 2)]), (4, [(0, 1), (0, 2), (0, 3)]),
+        (4, [(0, 1), (0, 2), (0, 3), (1, 2), (1, 3), (2, 3)]), (5, [(0, 1), (1, 2), (2, 3), (3, 4), (4, 0)]),
+        (6, [(0, 1), (1, 2), (2, 0), (2, 3), (3, 4), (4, 5), (5, 3)]), (2, [(0, 1)])]
+
+
+def main():
+    what = sys.argv[1]
+    if what.startswith("fpm"):
+        scale = int(sys.argv[2]) if len(sys.argv) > 2 else 13
+        n, s, d, lab = gg.config_graph("c4", seed=1, scale=scale)
+        t = time.time()
+        if what == "fpm_gpu":
+            import paper_conf_icde_hu0o23_b200 as G
+            c = G.Context(time_kernels=True)
+            g = c.load_edges(n, s, d, lab)
+            r = g.fpm(3, 3)
+            print("gpu", len(r), time.time() - t, c.stats()["level_entries"][:4], c.stats()["retries"], flush=True)
+        else:
+            import oracle
+            o = oracle.Graph(n, s, d, lab)
+            r = o.fpm(3, 3, pattern_cap=1 << 20)
+            print("oracle", len(r), time.time() - t, flush=True)
+    elif what == "sm":
+        i = int(sys.argv[2])
+        nv, e = PATS[i]
+        n, s, d, _ = gg.config_graph("c1", seed=2, scale=10)
+        lab = gg.labels(n, 3, 2)
+        import paper_conf_icde_hu0o23_b200 as G
+        import oracle
+        c = G.Context()
+        g = c.load_edges(n, s, d, lab)
+        for plab in (None, [(j * 7) % 3 for j in range(nv)]):
+            t = time.time()
+            got = g.match(nv, e, plab)
+            t1 = time.time()
+            want = oracle.Graph(n, s, d, lab).match(nv, e, plab)
+            print("sm", i, plab, got, want[:2], f"gpu {t1 - t:.2f}s oracle {time.time() - t1:.2f}s", flush=True)
+
+
+if __name__ == "__main__":
+    main()
