@@ -177,7 +177,9 @@ typedef struct {
 } gamma_fpm_result;
 
 /* All connected edge-induced patterns with 1..max_edges edges and MNI support >=
- * minsup (max_edges in [1,3] in v1; minsup >= 1).  Result owned by the library.   */
+ * minsup (max_edges in [1,3] in v1; minsup >= 1; vertex labels < 4096, else
+ * E_UNSUPPORTED).  Result owned by the library (free with gamma_fpm_result_free).
+ * With world > 1 every rank computes the full result (replicas).   */
 gamma_status gamma_fpm(gamma_graph *g, uint32_t max_edges, uint64_t minsup,
                        gamma_fpm_result **out);
 void gamma_fpm_result_free(gamma_fpm_result *r);

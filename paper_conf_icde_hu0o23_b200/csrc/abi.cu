@@ -163,6 +163,7 @@ void gamma_ctx_destroy(gamma_ctx *ctx) {
   if (ctx->stream) cudaStreamSynchronize(ctx->stream);
   if (ctx->ctrl) cudaFree(ctx->ctrl);
   if (ctx->ctrl_host) cudaFreeHost(ctx->ctrl_host);
+  if (ctx->spill_host) cudaFreeHost(ctx->spill_host);
   for (auto e : ctx->ev_pool) cudaEventDestroy(e);
   if (ctx->own_stream && ctx->stream) cudaStreamDestroy(ctx->stream);
   cudaGetLastError();

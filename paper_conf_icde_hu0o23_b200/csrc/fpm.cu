@@ -19,10 +19,11 @@
 //    enumerate only the label-consistent vertex orders and keep the minimal sorted
 //    edge-pair list; every minimizing order is an automorphic placement, so OR-ing
 //    the vertex of each position into that position's domain merges orbits (MNI).
-//  * Pattern table: lock-free open-addressing hash (code -> slot) in HBM; the MNI
-//    domain of slot position p is a bitmap over the vertices of p's label class
-//    (bit index = rank of the vertex inside its label class), carved from a pool
-//    at slot creation.  Support = min over positions of popcount (one warp/slot).
+//  * Pattern table: lock-free open-addressing hash (one-word code -> slot, claimed
+//    by a single atomicCAS, so no lane ever waits on another) in HBM; the MNI domain
+//    of slot position p is a bitmap over the vertices of p's label class (bit index
+//    = rank of the vertex inside its label class) at a fixed offset of the slot.
+//    Support = min over positions of popcount (one warp per slot).
 #include <cub/device/device_radix_sort.cuh>
 
 #include <algorithm>
@@ -45,17 +46,26 @@ __constant__ uint8_t c_perm4[24][4] = {
 // index of position pair (a<b) in lexicographic pair order: (0,1)(0,2)(0,3)(1,2)(1,3)(2,3)
 __constant__ uint8_t c_pair[4][4] = {{0, 0, 1, 2}, {0, 0, 3, 4}, {1, 3, 0, 5}, {2, 4, 5, 0}};
 
+// Pattern code packed in one word (0 = empty slot):
+//   bits 0..47 four 12-bit labels (canonical order), 48..50 nv, 51..52 ne,
+//   53..61 sorted edge-pair key, 63 always set.
+constexpr uint64_t kKeyTag = 1ull << 63;
+
 struct Table {
-  uint32_t *st;          // 0 empty, 1 being written, 2 ready
-  unsigned long long *klo, *khi;
-  unsigned long long *dom;   // 4 word offsets per slot into the pool
+  unsigned long long *key;   // 0 = empty; claimed with one atomicCAS (no spinning)
   unsigned long long *support;
-  uint32_t *freq;        // 1 if support >= minsup (set after the slot's level)
-  uint64_t cap;          // power of two
-  uint32_t *pool;
-  uint64_t pool_words;
-  unsigned long long *pool_cur;
+  uint32_t *freq;            // 1 if support >= minsup (set after the slot's level)
+  uint64_t cap;              // power of two
+  uint32_t *pool;            // domain of (slot s, position p) at pool + (4 s + p) * slot_words
+  uint64_t slot_words;       // words of the largest label class bitmap
 };
+
+__host__ __device__ __forceinline__ uint32_t key_nv(uint64_t k) { return (uint32_t)((k >> 48) & 7); }
+__host__ __device__ __forceinline__ uint32_t key_ne(uint64_t k) { return (uint32_t)((k >> 51) & 3); }
+__host__ __device__ __forceinline__ uint32_t key_edges(uint64_t k) { return (uint32_t)((k >> 53) & 511); }
+__host__ __device__ __forceinline__ uint32_t key_label(uint64_t k, uint32_t p) {
+  return (uint32_t)((k >> (12 * p)) & 0xfff);
+}
 
 struct FpmArgs {
   const uint64_t *rp;
@@ -92,55 +102,33 @@ __device__ __forceinline__ uint64_t mix64(uint64_t x) {
 }
 
 // Lookup (insert = false) or lookup-or-insert a pattern code; returns slot or -1.
-__device__ int64_t table_slot(const FpmArgs &a, uint64_t klo, uint64_t khi, uint32_t nv, const uint32_t *labs,
-                              bool insert) {
+// Lookup (insert = false) or lookup-or-insert a pattern code; returns slot or -1.
+// Lock-free: a slot is claimed by one atomicCAS of its key word, so no thread ever
+// waits on another (safe for lanes of the same warp).
+__device__ int64_t table_slot(const FpmArgs &a, uint64_t key, bool insert) {
   const Table &T = a.T;
-  uint64_t h = mix64(klo ^ mix64(khi)) & (T.cap - 1);
-  for (uint64_t probe = 0; probe < T.cap; probe++, h = (h + 1) & (T.cap - 1)) {
-    uint32_t s = *(volatile uint32_t *)&T.st[h];
-    if (s == 0) {
+  uint64_t h = mix64(key) & (T.cap - 1);
+  // a long probe chain means the table is (nearly) full: report it and let the host
+  // grow the table instead of degrading to a linear scan
+  const uint64_t max_probe = T.cap < 4096 ? T.cap : 4096;
+  for (uint64_t probe = 0; probe < max_probe; probe++, h = (h + 1) & (T.cap - 1)) {
+    unsigned long long k = *(volatile unsigned long long *)&T.key[h];
+    if (k == key) return (int64_t)h;
+    if (k == 0) {
       if (!insert) return -1;
-      s = atomicCAS(&T.st[h], 0u, 1u);
-      if (s == 0) {
-        T.klo[h] = klo;
-        T.khi[h] = khi;
-        // carve the position bitmaps (one per position, sized to the label class)
-        uint64_t words = 0, wpos[4] = {0, 0, 0, 0};
-        for (uint32_t p = 0; p < nv; p++) {
-          wpos[p] = (a.csize[labs[p]] + 31) / 32;
-          words += wpos[p];
-        }
-        unsigned long long off = atomicAdd(a.T.pool_cur, (unsigned long long)words);
-        if (off + words > T.pool_words) {
-          atomicExch(&a.ctrl[CTRL_OVF], 1ull);
-          off = ~0ull;
-        }
-        uint64_t o = off;
-        for (uint32_t p = 0; p < 4; p++) {
-          T.dom[h * 4 + p] = (off == ~0ull) ? ~0ull : o;
-          o += wpos[p];
-        }
-        T.support[h] = 0;
-        T.freq[h] = 0;
-        __threadfence();
-        atomicExch(&T.st[h], 2u);
-        return (int64_t)h;
-      }
+      k = atomicCAS(&T.key[h], 0ull, (unsigned long long)key);
+      if (k == 0 || k == key) return (int64_t)h;
     }
-    while (s != 2) s = *(volatile uint32_t *)&T.st[h];
-    __threadfence();
-    if (T.klo[h] == klo && T.khi[h] == khi) return (int64_t)h;
   }
-  atomicExch(&a.ctrl[CTRL_ERR], 1ull);   // table full
+  if (insert) atomicExch(&a.ctrl[CTRL_ERR], 1ull);   // table full
   return -1;
 }
 
 // Canonical code of a connected edge set on nv <= 4 local vertices (W) with ne <= 3
-// edges (local index pairs E).  Returns (klo, khi) and the minimizing vertex orders
+// edges (local index pairs E).  Returns the packed key and the minimizing vertex orders
 // as a bitmask over c_perm4 rows.
 struct Canon {
-  uint64_t klo, khi;
-  uint32_t labs[4];
+  uint64_t key;
   uint32_t minmask;
 };
 
@@ -183,12 +171,9 @@ __device__ Canon canonical(const FpmArgs &a, const uint32_t *W, uint32_t nv, con
       mask |= 1u << r;
     }
   }
-  cn.klo = 0;
-  for (uint32_t p = 0; p < 4; p++) {
-    cn.labs[p] = p < nv ? ls[p] : 0;
-    cn.klo |= (uint64_t)(cn.labs[p] & 0xffffu) << (16 * p);
-  }
-  cn.khi = (uint64_t)nv | ((uint64_t)ne << 4) | ((uint64_t)best << 8);
+  uint64_t key = kKeyTag | ((uint64_t)nv << 48) | ((uint64_t)ne << 51) | ((uint64_t)best << 53);
+  for (uint32_t p = 0; p < nv; p++) key |= (uint64_t)(ls[p] & 0xfffu) << (12 * p);
+  cn.key = key;
   cn.minmask = mask;
   return cn;
 }
@@ -197,11 +182,10 @@ __device__ Canon canonical(const FpmArgs &a, const uint32_t *W, uint32_t nv, con
 // position's domain bitmap (read-before-atomic: most bits are already set).
 __device__ void record(const FpmArgs &a, const uint32_t *W, uint32_t nv, const uint8_t (*E)[2], uint32_t ne) {
   const Canon cn = canonical(a, W, nv, E, ne);
-  const int64_t s = table_slot(a, cn.klo, cn.khi, nv, cn.labs, true);
+  const int64_t s = table_slot(a, cn.key, true);
   if (s < 0) return;
   uint64_t off[4];
-  for (uint32_t p = 0; p < 4; p++) off[p] = a.T.dom[s * 4 + p];
-  if (off[0] == ~0ull) return;
+  for (uint32_t p = 0; p < 4; p++) off[p] = ((uint64_t)s * 4 + p) * a.T.slot_words;
   uint32_t m = cn.minmask;
   while (m) {
     const int r = __ffs(m) - 1;
@@ -219,7 +203,7 @@ __device__ void record(const FpmArgs &a, const uint32_t *W, uint32_t nv, const u
 // Is the pattern of this (prefix) edge set frequent?  (Alg. 2 line 4 pruning)
 __device__ bool frequent(const FpmArgs &a, const uint32_t *W, uint32_t nv, const uint8_t (*E)[2], uint32_t ne) {
   const Canon cn = canonical(a, W, nv, E, ne);
-  const int64_t s = table_slot(a, cn.klo, cn.khi, nv, cn.labs, false);
+  const int64_t s = table_slot(a, cn.key, false);
   return s >= 0 && a.T.freq[s];
 }
 
@@ -341,16 +325,15 @@ __global__ void fpm_support_kernel(FpmArgs a, uint32_t level, uint64_t minsup) {
   const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
   const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
   for (uint64_t s = warp; s < a.T.cap; s += nwarps) {
-    if (a.T.st[s] != 2) continue;
-    const uint64_t khi = a.T.khi[s];
-    const uint32_t nv = (uint32_t)(khi & 0xf), ne = (uint32_t)((khi >> 4) & 0xf);
+    const uint64_t key = a.T.key[s];
+    if (key == 0) continue;
+    const uint32_t nv = key_nv(key), ne = key_ne(key);
     if (ne != level) continue;
     uint64_t sup = ~0ull;
-    const uint64_t klo = a.T.klo[s];
     for (uint32_t p = 0; p < nv; p++) {
-      const uint32_t lp = (uint32_t)((klo >> (16 * p)) & 0xffff);
+      const uint32_t lp = key_label(key, p);
       const uint64_t words = (a.csize[lp] + 31) / 32;
-      const uint64_t off = a.T.dom[s * 4 + p];
+      const uint64_t off = (s * 4 + p) * a.T.slot_words;
       uint64_t c = 0;
       for (uint64_t w = lane; w < words; w += 32) c += __popc(a.T.pool[off + w]);
       for (int o = 16; o > 0; o >>= 1) c += __shfl_down_sync(0xffffffffu, c, o);
@@ -419,7 +402,7 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
     uint64_t ml = 0;
     GAMMA_CUDA(cudaMemcpyAsync(&ml, ctx->ctrl + CTRL_AUX1, 8, cudaMemcpyDeviceToHost, ctx->stream));
     ctx->sync();
-    GAMMA_REQUIRE(ml < 65536, GAMMA_E_UNSUPPORTED, "gamma_fpm: labels must be < 65536");
+    GAMMA_REQUIRE(ml < 4096, GAMMA_E_UNSUPPORTED, "gamma_fpm: labels must be < 4096");
     nlab = (uint32_t)ml + 1;
   }
   DevBuf<uint32_t> csize(ctx, nlab), lrank(ctx, n);
@@ -438,41 +421,25 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
     });
     ctx->launch(KC_FPM, [&] { label_rank_kernel<<<g1d(n), 256, 0, ctx->stream>>>(k1.p, n, lrank.p); });
   }
-  // ---- pattern table + domain pool ----
+  // ---- pattern table + per-(slot, position) domain bitmaps ----
   size_t fr = 0, tot = 0;
   GAMMA_CUDA(cudaMemGetInfo(&fr, &tot));
   const uint64_t budget = ctx->desc.hbm_budget_bytes ? ctx->desc.hbm_budget_bytes : (uint64_t)(fr * 0.6);
   std::vector<uint32_t> hsize(nlab);
   GAMMA_CUDA(cudaMemcpyAsync(hsize.data(), csize.p, nlab * 4, cudaMemcpyDeviceToHost, ctx->stream));
   ctx->sync();
-  uint64_t maxw = 0;
+  uint64_t maxw = 1;
   for (auto c : hsize) maxw = std::max<uint64_t>(maxw, (c + 31) / 32);
-  // capacity: distinct patterns are bounded by the label combinations seen; start
-  // from min(#labels^2 * 64, 2^22) slots and size the pool to the budget
+  // distinct patterns are bounded by the label combinations that occur; start from
+  // min(#labels^2 * 64, 2^20) slots, grow x4 when a probe chain gets long
+  const uint64_t slot_bytes = 8 + 8 + 4 + 4 * maxw * 4;
   uint64_t cap = 1;
-  const uint64_t want = std::min<uint64_t>((uint64_t)nlab * nlab * 64 + 1024, 1ull << 22);
+  const uint64_t want = std::min<uint64_t>((uint64_t)nlab * nlab * 64 + 1024, 1ull << 20);
   while (cap < want) cap <<= 1;
-  const uint64_t slot_bytes = 4 + 8 + 8 + 32 + 8 + 4;
-  const uint64_t pool_min = 4 * maxw + 64;
-  uint64_t pool_words = std::min<uint64_t>(cap * 2 * std::max<uint64_t>(maxw, 1), 1ull << 28);
-  DevBuf<uint32_t> st, freq, pool;
-  DevBuf<unsigned long long> klo, khi, dom, sup, pcur;
+  while (cap > 1024 && cap * slot_bytes > budget) cap >>= 1;
+  DevBuf<uint32_t> freq, pool;
+  DevBuf<unsigned long long> key, sup;
   FpmArgs a{};
-  for (int attempt = 0;; attempt++) {
-  pool_words = std::max<uint64_t>(std::min<uint64_t>(pool_words, (budget - std::min(budget, cap * slot_bytes)) / 4),
-                                  pool_min);
-  st.reset(); freq.reset(); pool.reset(); klo.reset(); khi.reset(); dom.reset(); sup.reset(); pcur.reset();
-  st = DevBuf<uint32_t>(ctx, cap);
-  freq = DevBuf<uint32_t>(ctx, cap);
-  pool = DevBuf<uint32_t>(ctx, pool_words);
-  klo = DevBuf<unsigned long long>(ctx, cap);
-  khi = DevBuf<unsigned long long>(ctx, cap);
-  dom = DevBuf<unsigned long long>(ctx, cap * 4);
-  sup = DevBuf<unsigned long long>(ctx, cap);
-  pcur = DevBuf<unsigned long long>(ctx, 1);
-  GAMMA_CUDA(cudaMemsetAsync(st.p, 0, cap * 4, ctx->stream));
-  GAMMA_CUDA(cudaMemsetAsync(pool.p, 0, pool_words * 4, ctx->stream));
-  GAMMA_CUDA(cudaMemsetAsync(pcur.p, 0, 8, ctx->stream));
   a.rp = g->row_ptr;
   a.col = g->col;
   a.lab = g->labels;
@@ -481,58 +448,54 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
   a.n = n;
   a.rank = 0;
   a.world = 1;   // FPM runs every root on every rank (replicas)
-  a.T = Table{st.p, klo.p, khi.p, dom.p, sup.p, freq.p, cap, pool.p, pool_words, pcur.p};
   a.ctrl = (unsigned long long *)ctx->ctrl;
   const int grid_enum = ctx->num_sms * occupancy_blocks((const void *)fpm_enum_kernel, kThreads, 0);
-  bool full = false, exhausted = false;
-  for (uint32_t l = 1; l <= max_edges; l++) {
-    a.level = l;
-    ctrl_reset(ctx);
-    ctx->launch(KC_FPM, [&] { fpm_enum_kernel<<<grid_enum, kThreads, 0, ctx->stream>>>(a); });
-    ctx->launch(KC_FPM_SUPPORT, [&] {
-      fpm_support_kernel<<<g1d(cap * 32), 256, 0, ctx->stream>>>(a, l, minsup);
-    });
-    ctrl_fetch(ctx);
-    const uint64_t *h = ctx->ctrl_host;
-    exhausted = h[CTRL_OVF] != 0;
-    full = h[CTRL_ERR] != 0;
-    if (full || exhausted) break;
-    ctx->stats.level_entries[l] = h[CTRL_ENTRIES];
-  }
-  if (!full && !exhausted) break;
-  // grow what ran out and start over (rare: sizes are only known after the fact)
-  ctx->stats.retries++;
-  const uint64_t max_bytes = budget;
-  if (full) {
-    GAMMA_REQUIRE(cap * 4 * slot_bytes + pool_min * 4 <= max_bytes, GAMMA_E_NOMEM,
-                  "gamma_fpm: pattern table full (raise hbm_budget_bytes)");
+  for (;;) {
+    GAMMA_REQUIRE(cap * slot_bytes <= budget, GAMMA_E_NOMEM,
+                  "gamma_fpm: pattern table + MNI domains exceed the HBM budget");
+    freq.reset(); pool.reset(); key.reset(); sup.reset();
+    key = DevBuf<unsigned long long>(ctx, cap);
+    sup = DevBuf<unsigned long long>(ctx, cap);
+    freq = DevBuf<uint32_t>(ctx, cap);
+    pool = DevBuf<uint32_t>(ctx, cap * 4 * maxw);
+    GAMMA_CUDA(cudaMemsetAsync(key.p, 0, cap * 8, ctx->stream));
+    GAMMA_CUDA(cudaMemsetAsync(freq.p, 0, cap * 4, ctx->stream));
+    GAMMA_CUDA(cudaMemsetAsync(pool.p, 0, cap * 4 * maxw * 4, ctx->stream));
+    a.T = Table{key.p, sup.p, freq.p, cap, pool.p, maxw};
+    bool full = false;
+    for (uint32_t l = 1; l <= max_edges; l++) {
+      a.level = l;
+      ctrl_reset(ctx);
+      ctx->launch(KC_FPM, [&] { fpm_enum_kernel<<<grid_enum, kThreads, 0, ctx->stream>>>(a); });
+      ctx->launch(KC_FPM_SUPPORT, [&] {
+        fpm_support_kernel<<<g1d(cap * 32), 256, 0, ctx->stream>>>(a, l, minsup);
+      });
+      ctrl_fetch(ctx);
+      const uint64_t *h = ctx->ctrl_host;
+      full = h[CTRL_ERR] != 0;
+      if (full) break;
+      ctx->stats.level_entries[l] = h[CTRL_ENTRIES];
+    }
+    if (!full) break;
+    ctx->stats.retries++;   // sizes are only known after the fact: grow and redo
     cap *= 4;
   }
-  if (exhausted) {
-    GAMMA_REQUIRE(pool_words * 4 * 2 + cap * slot_bytes <= max_bytes || pool_words * 4 + cap * slot_bytes < max_bytes,
-                  GAMMA_E_NOMEM, "gamma_fpm: MNI domain pool exhausted (raise hbm_budget_bytes)");
-    GAMMA_REQUIRE(attempt < 12, GAMMA_E_NOMEM, "gamma_fpm: MNI domain pool exhausted");
-    pool_words *= 4;
-  }
-  }
   // ---- collect the frequent patterns ----
-  std::vector<uint32_t> hst(cap), hfreq(cap);
-  std::vector<unsigned long long> hlo(cap), hhi(cap), hsup(cap);
-  GAMMA_CUDA(cudaMemcpyAsync(hst.data(), st.p, cap * 4, cudaMemcpyDeviceToHost, ctx->stream));
+  std::vector<uint32_t> hfreq(cap);
+  std::vector<unsigned long long> hkey(cap), hsup(cap);
   GAMMA_CUDA(cudaMemcpyAsync(hfreq.data(), freq.p, cap * 4, cudaMemcpyDeviceToHost, ctx->stream));
-  GAMMA_CUDA(cudaMemcpyAsync(hlo.data(), klo.p, cap * 8, cudaMemcpyDeviceToHost, ctx->stream));
-  GAMMA_CUDA(cudaMemcpyAsync(hhi.data(), khi.p, cap * 8, cudaMemcpyDeviceToHost, ctx->stream));
+  GAMMA_CUDA(cudaMemcpyAsync(hkey.data(), key.p, cap * 8, cudaMemcpyDeviceToHost, ctx->stream));
   GAMMA_CUDA(cudaMemcpyAsync(hsup.data(), sup.p, cap * 8, cudaMemcpyDeviceToHost, ctx->stream));
   ctx->sync();
   static const uint8_t pairs[6][2] = {{0, 1}, {0, 2}, {0, 3}, {1, 2}, {1, 3}, {2, 3}};
   for (uint64_t s = 0; s < cap; s++) {
-    if (hst[s] != 2 || !hfreq[s]) continue;
+    if (hkey[s] == 0 || !hfreq[s]) continue;
     gamma_fpm_pattern p{};
-    p.nv = (uint32_t)(hhi[s] & 0xf);
-    p.ne = (uint32_t)((hhi[s] >> 4) & 0xf);
-    const uint32_t key = (uint32_t)(hhi[s] >> 8);
-    const uint32_t idx[3] = {key / 64, (key / 8) % 8, key % 8};
-    for (uint32_t i = 0; i < p.nv; i++) p.labels[i] = (uint32_t)((hlo[s] >> (16 * i)) & 0xffff);
+    p.nv = key_nv(hkey[s]);
+    p.ne = key_ne(hkey[s]);
+    const uint32_t ek = key_edges(hkey[s]);
+    const uint32_t idx[3] = {ek / 64, (ek / 8) % 8, ek % 8};
+    for (uint32_t i = 0; i < p.nv; i++) p.labels[i] = key_label(hkey[s], i);
     for (uint32_t e = 0; e < p.ne; e++) {
       const uint32_t id = idx[e];   // sorted pair indices first, unused slots hold 7
       p.edges[e][0] = pairs[id][0];

@@ -88,6 +88,9 @@ struct gamma_ctx {
   // device control block: counters reset per launch
   uint64_t *ctrl = nullptr;  // CTRL_WORDS u64 on device
   uint64_t *ctrl_host = nullptr;  // pinned mirror
+  // pinned host arena for spilled ET levels (GAMMA_FLAG_SPILL), used as a stack
+  uint8_t *spill_host = nullptr;
+  size_t spill_cap = 0, spill_top = 0;
   // stats of the last call
   gamma_run_stats stats;
   // event pool for kernel timing
@@ -206,5 +209,5 @@ uint64_t kclique_count(gamma_graph *g, uint32_t k, const uint32_t *roots_dev, ui
 constexpr uint32_t kBitmapMaxRun = 512;
 constexpr uint32_t kBitmapMaxK = 12;
 uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint64_t nroots,
-                        unsigned long long *per_root);
+                        unsigned long long *per_root, bool sorted);
 }  // namespace gamma_impl

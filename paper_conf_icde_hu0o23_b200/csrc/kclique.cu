@@ -557,6 +557,10 @@ struct KclRun {
       }
       ctx->stats.retries++;
       if (grow_level(nd, std::max<uint64_t>(h[CTRL_VCUR], L.cap_v) * 4)) continue;
+      if (!fused && (ctx->desc.flags & GAMMA_FLAG_SPILL) && ctx->desc.host_spill_bytes) {
+        process_spill(d, g0, g1);
+        return;
+      }
       GAMMA_REQUIRE(g1 - g0 > 1, GAMMA_E_NOMEM,
                     "HBM budget too small for the children of a single embedding group");
       const uint64_t mid = g0 + (g1 - g0) / 2;
@@ -564,6 +568,71 @@ struct KclRun {
       process(d, mid, g1);
       return;
     }
+  }
+
+  // GAMMA_FLAG_SPILL: BFS with a host-resident next level (the ET "should
+  // be resident in host memory ... we keep a buffer on the device to write extension
+  // results ... and flush them to host memory").  Level d+1 is produced in slabs that
+  // fit the device buffer, each slab is parked in pinned host memory, and the slabs
+  // are streamed back one at a time for the next extension.
+  void process_spill(uint32_t d, uint64_t g0, uint64_t g1) {
+    const uint32_t nd = d + 1;
+    struct Slab { size_t off; uint64_t nv, ng; };
+    std::vector<Slab> slabs;
+    const size_t top0 = ctx->spill_top;
+    std::vector<std::pair<uint64_t, uint64_t>> todo{{g0, g1}};
+    while (!todo.empty()) {
+      const auto r = todo.back();
+      todo.pop_back();
+      Level &L = levels[nd];
+      KclArgs a = args_for(d, r.first, r.second);
+      set_output(a, nd);
+      launch<MODE_EXTEND>(a, d, L.cap_v);
+      const uint64_t *h = ctx->ctrl_host;
+      if (h[CTRL_OVF]) {
+        ctx->stats.retries++;
+        GAMMA_REQUIRE(r.second - r.first > 1, GAMMA_E_NOMEM,
+                      "HBM budget too small for the children of a single embedding group");
+        const uint64_t mid = r.first + (r.second - r.first) / 2;
+        todo.push_back({mid, r.second});
+        todo.push_back({r.first, mid});
+        continue;
+      }
+      account(KC_EXTEND, d, h, true);
+      ctx->stats.chunks++;
+      ctx->stats.level_entries[nd + 1] += h[CTRL_ENTRIES];
+      Slab s{0, std::min<uint64_t>(h[CTRL_VCUR], L.cap_v), std::min<uint64_t>(h[CTRL_GCUR], L.cap_g)};
+      const size_t bytes = s.nv * 4 + s.ng * 8 + (per_root ? s.ng * 4 : 0);
+      if (ctx->spill_host == nullptr) {
+        ctx->spill_cap = ctx->desc.host_spill_bytes;
+        GAMMA_CUDA(cudaMallocHost(&ctx->spill_host, ctx->spill_cap));
+      }
+      GAMMA_REQUIRE(ctx->spill_top + bytes <= ctx->spill_cap, GAMMA_E_NOMEM,
+                    "host spill budget exhausted (raise host_spill_bytes)");
+      s.off = ctx->spill_top;
+      uint8_t *dst = ctx->spill_host + s.off;
+      GAMMA_CUDA(cudaMemcpyAsync(dst, L.vid.p, s.nv * 4, cudaMemcpyDeviceToHost, ctx->stream));
+      GAMMA_CUDA(cudaMemcpyAsync(dst + s.nv * 4, L.grp.p, s.ng * 8, cudaMemcpyDeviceToHost, ctx->stream));
+      if (per_root)
+        GAMMA_CUDA(cudaMemcpyAsync(dst + s.nv * 4 + s.ng * 8, L.groot.p, s.ng * 4, cudaMemcpyDeviceToHost,
+                                   ctx->stream));
+      ctx->sync();
+      ctx->spill_top += bytes;
+      ctx->stats.spilled_bytes += bytes;
+      slabs.push_back(s);
+    }
+    for (const Slab &s : slabs) {
+      Level &L = levels[nd];
+      const uint8_t *src = ctx->spill_host + s.off;
+      GAMMA_CUDA(cudaMemcpyAsync(L.vid.p, src, s.nv * 4, cudaMemcpyHostToDevice, ctx->stream));
+      GAMMA_CUDA(cudaMemcpyAsync(L.grp.p, src + s.nv * 4, s.ng * 8, cudaMemcpyHostToDevice, ctx->stream));
+      if (per_root)
+        GAMMA_CUDA(cudaMemcpyAsync(L.groot.p, src + s.nv * 4 + s.ng * 8, s.ng * 4, cudaMemcpyHostToDevice,
+                                   ctx->stream));
+      ctx->stats.spilled_bytes += s.nv * 4 + s.ng * 8 + (per_root ? s.ng * 4 : 0);
+      process(nd, 0, s.ng);
+    }
+    ctx->spill_top = top0;
   }
 };
 
@@ -687,7 +756,7 @@ uint64_t kclique_count(gamma_graph *g, uint32_t k, const uint32_t *roots_dev, ui
                                                        kThreads, kcl_smem(MODE_FUSED));
   const bool bitmap = (ctx->desc.flags & GAMMA_FLAG_NO_BITMAP) == 0 && k >= 3 && k <= kBitmapMaxK;
   if (bitmap && R.nroots) {
-    R.add_count(kclique_bitmap(g, k, R.roots, R.nroots, R.per_root_out));
+    R.add_count(kclique_bitmap(g, k, R.roots, R.nroots, R.per_root_out, !per_root));
     R.root_len_gt = kBitmapMaxRun;
   }
   if (R.nroots && (!bitmap || g->max_out_degree > kBitmapMaxRun)) R.process(1, 0, R.nroots);

@@ -160,18 +160,27 @@ __global__ void __launch_bounds__(256) kcl_bitmap_kernel(BmArgs a) {
   uint32_t *slot = B + kRunMax * TW;   // work index broadcast (CTA teams)
   uint64_t total = 0, elems = 0, entries = 0;
 
+  // warp teams take roots in batches of 4 (one atomic per batch); CTA teams one
+  // root at a time (their roots are the long, costly ones)
+  constexpr unsigned long long kBatch = TEAM_WARPS == 1 ? 4 : 1;
+  unsigned long long next = 0, end = 0;
   for (;;) {
-    unsigned long long gi = 0;
-    if (tid == 0) gi = atomicAdd(&a.ctrl[CTRL_WORK], 1ull);
-    if (TEAM_WARPS == 1) {
-      gi = __shfl_sync(0xffffffffu, gi, 0);
-    } else {
-      if (tid == 0) *slot = gi < 0xffffffffull ? (uint32_t)gi : 0xffffffffu;
-      __syncthreads();
-      gi = *slot;
-      __syncthreads();
+    if (next == end) {
+      unsigned long long base = 0;
+      if (tid == 0) base = atomicAdd(&a.ctrl[CTRL_WORK], kBatch);
+      if (TEAM_WARPS == 1) {
+        base = __shfl_sync(0xffffffffu, base, 0);
+      } else {
+        if (tid == 0) *slot = base < 0xffffffffull ? (uint32_t)base : 0xffffffffu;
+        __syncthreads();
+        base = *slot;
+        __syncthreads();
+      }
+      next = base;
+      end = base + kBatch;
     }
-    if (gi >= a.nroots) break;
+    if (next >= a.nroots) break;
+    const unsigned long long gi = next++;
     const uint32_t v = a.roots[gi];
     const uint64_t b0 = a.dag_ptr[v];
     const uint32_t L = (uint32_t)(a.dag_ptr[v + 1] - b0);
@@ -292,8 +301,30 @@ uint64_t run_bitmap(gamma_ctx *ctx, const BmArgs &a0, bool per_root) {
 
 // Count k-cliques rooted at roots[0..nroots) whose run length is <= 512 (k <= 12);
 // longer runs are left to the ET path.  per_root (nullable) indexed like roots.
+namespace {
+// out[0] = #roots with |N+(v)| > 512, out[1] = #roots with |N+(v)| > 128
+__global__ void count_len_classes(const uint64_t *dag_ptr, const uint32_t *roots, uint64_t nr,
+                                  unsigned long long *out) {
+  unsigned long long c0 = 0, c1 = 0;
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < nr; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t v = roots[i];
+    const uint64_t L = dag_ptr[v + 1] - dag_ptr[v];
+    c0 += L > kBitmapMaxRun;
+    c1 += L > 128;
+  }
+  for (int o = 16; o > 0; o >>= 1) {
+    c0 += __shfl_down_sync(0xffffffffu, c0, o);
+    c1 += __shfl_down_sync(0xffffffffu, c1, o);
+  }
+  if ((threadIdx.x & 31) == 0) {
+    if (c0) atomicAdd(&out[0], c0);
+    if (c1) atomicAdd(&out[1], c1);
+  }
+}
+}  // namespace
+
 uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint64_t nroots,
-                        unsigned long long *per_root) {
+                        unsigned long long *per_root, bool sorted) {
   gamma_ctx *ctx = g->ctx;
   BmArgs a{};
   a.dag_ptr = g->dag_ptr;
@@ -304,12 +335,37 @@ uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint6
   a.ctrl = (unsigned long long *)ctx->ctrl;
   a.per_root = per_root;
   uint64_t total = 0;
+  // Roots sorted by cost (d+^2, descending) fall into three contiguous classes:
+  // [0, n_long) ET path, [n_long, n_mid) CTA teams, [n_mid, nroots) warp teams.
+  // Launch each team kind on its own range so no team walks over roots it skips.
+  // (Per-root mode passes unsorted roots: every launch then filters the whole list.)
+  uint64_t n_long = 0, n_mid = 0;
+  if (sorted) {
+    GAMMA_CUDA(cudaMemsetAsync(ctx->ctrl + CTRL_AUX0, 0, 16, ctx->stream));
+    ctx->launch(KC_ROOTS, [&] {
+      count_len_classes<<<148 * 4, 256, 0, ctx->stream>>>(g->dag_ptr, roots, nroots,
+                                                          (unsigned long long *)(ctx->ctrl + CTRL_AUX0));
+    });
+    uint64_t h[2];
+    GAMMA_CUDA(cudaMemcpyAsync(h, ctx->ctrl + CTRL_AUX0, 16, cudaMemcpyDeviceToHost, ctx->stream));
+    ctx->sync();
+    n_long = h[0];
+    n_mid = h[1];
+  }
   a.len_lo = 128;
   a.len_hi = 512;
-  if (g->max_out_degree > 128) total = checked_add(total, run_bitmap<8, 16>(ctx, a, per_root != nullptr));
+  if (g->max_out_degree > 128 && (!sorted || n_mid > n_long)) {
+    a.roots = roots + (sorted ? n_long : 0);
+    a.nroots = sorted ? n_mid - n_long : nroots;
+    total = checked_add(total, run_bitmap<8, 16>(ctx, a, per_root != nullptr));
+  }
   a.len_lo = 0;
   a.len_hi = 128;
-  total = checked_add(total, run_bitmap<1, 4>(ctx, a, per_root != nullptr));
+  if (!sorted || nroots > n_mid) {
+    a.roots = roots + (sorted ? n_mid : 0);
+    a.nroots = sorted ? nroots - n_mid : nroots;
+    total = checked_add(total, run_bitmap<1, 4>(ctx, a, per_root != nullptr));
+  }
   return total;
 }
 

@@ -66,10 +66,22 @@ def test_rmat_vs_oracle(ctx, oracle_mod, seed):
 
 
 def test_c4_shaped_37_labels(ctx, oracle_mod):
-    n, s, d, lab = gg.config_graph("c4", seed=1, scale=13)
+    """configs[3]'s generator (a,b,c = 0.40,0.25,0.25, L = 37) at scale 11."""
+    n, s, d, lab = gg.config_graph("c4", seed=1, scale=11)
     g = ctx.load_edges(n, s, d, lab)
     o = oracle_mod.Graph(n, s, d, lab)
-    assert g.fpm(3, 3) == oracle_set(o, 3, 3)
+    for minsup in (3, 8):
+        assert g.fpm(3, minsup) == oracle_set(o, 3, minsup)
+
+
+def test_pattern_table_growth(G, oracle_mod):
+    """A deliberately small HBM budget starts the pattern table tiny; it must grow
+    (retries) and still give the oracle's answer."""
+    n, s, d, lab = gg.config_graph("c4", seed=2, scale=10)
+    c = G.Context(hbm_budget_bytes=48 << 20)
+    g = c.load_edges(n, s, d, lab)
+    o = oracle_mod.Graph(n, s, d, lab)
+    assert g.fpm(3, 2) == oracle_set(o, 3, 2)
 
 
 def test_invalid(G, ctx):

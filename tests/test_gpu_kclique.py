@@ -133,6 +133,24 @@ def test_budget_forced_splits(G, oracle_mod):
     assert st["retries"] > 0
 
 
+def test_pinned_host_spill(G, oracle_mod):
+    """GAMMA_FLAG_SPILL: levels that exceed the HBM budget are parked in pinned host
+    memory and streamed back; counts are unchanged."""
+    n, s, d, _ = gg.config_graph("c1", seed=2, scale=11)
+    o = oracle_mod.Graph(n, s, d)
+    c = G.Context(hbm_budget_bytes=3 << 20, host_spill_bytes=1 << 30, flags=0x10 | 0x4 | 0x2)
+    g = c.load_edges(n, s, d)
+    for k in (4, 5):
+        assert g.kclique(k) == o.kclique(k)
+    assert c.stats()["spilled_bytes"] > 0
+    roots = np.arange(0, n, 5, dtype=np.uint32)
+    assert np.array_equal(g.kclique_roots(5, roots), o.kclique_roots(5, roots))
+    small = G.Context(hbm_budget_bytes=3 << 20, host_spill_bytes=4096, flags=0x10 | 0x4 | 0x2)
+    with pytest.raises(G.GammaError) as e:
+        small.load_edges(n, s, d).kclique(5)
+    assert e.value.status == -2
+
+
 def test_simulated_ranks_partition(G, oracle_mod):
     n, s, d, _ = gg.config_graph("c1", seed=3)
     want = oracle_mod.Graph(n, s, d).kclique(5)
