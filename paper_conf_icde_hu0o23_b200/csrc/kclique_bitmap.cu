@@ -47,17 +47,6 @@ __device__ __forceinline__ uint32_t excl_scan32(uint32_t x, int lane, uint32_t &
   return s - x;
 }
 
-// Position of y in sorted s[0..len) or -1.
-__device__ __forceinline__ int find_pos(const uint32_t *s, uint32_t len, uint32_t y) {
-  uint32_t base = 0, n = len;
-  while (n > 1) {
-    const uint32_t half = n >> 1;
-    base = (s[base + half] <= y) ? base + half : base;
-    n -= half;
-  }
-  return s[base] == y ? (int)base : -1;
-}
-
 template <int TW>
 __device__ __forceinline__ int next_bit(const uint32_t (&bm)[TW], uint32_t pos, uint32_t W) {
 #pragma unroll
@@ -146,6 +135,13 @@ __device__ __forceinline__ void team_sync() {
   else __syncthreads();
 }
 
+// Shared words per team: run R (32 TW), bitmap rows B (32 TW x TW), position hash
+// H (4 x 32 TW u16 = 64 TW words), work slot.
+template <int TW>
+constexpr int team_words() {
+  return TW * 32 + TW * 32 * TW + 2 * TW * 32 + 1;
+}
+
 template <int TEAM_WARPS, int TW, bool PER_ROOT>
 __global__ void __launch_bounds__(256) kcl_bitmap_kernel(BmArgs a) {
   extern __shared__ uint32_t smem[];
@@ -155,9 +151,10 @@ __global__ void __launch_bounds__(256) kcl_bitmap_kernel(BmArgs a) {
   const int team = threadIdx.x / kTeamThreads;
   const int tid = threadIdx.x % kTeamThreads;
   const int wit = tid >> 5;   // warp index inside the team
-  uint32_t *R = smem + team * (kRunMax + kRunMax * TW + 1);
+  uint32_t *R = smem + team * team_words<TW>();
   uint32_t *B = R + kRunMax;
-  uint32_t *slot = B + kRunMax * TW;   // work index broadcast (CTA teams)
+  unsigned short *H = reinterpret_cast<unsigned short *>(B + kRunMax * TW);   // 4 kRunMax entries
+  uint32_t *slot = B + kRunMax * TW + 2 * kRunMax;   // work index broadcast (CTA teams)
   uint64_t total = 0, elems = 0, entries = 0;
 
   // warp teams take roots in batches of 4 (one atomic per batch); CTA teams one
@@ -186,13 +183,23 @@ __global__ void __launch_bounds__(256) kcl_bitmap_kernel(BmArgs a) {
     const uint32_t L = (uint32_t)(a.dag_ptr[v + 1] - b0);
     if (L <= a.len_lo || L > a.len_hi || L < a.k - 1) continue;   // uniform across the team
     const uint32_t W = (L + 31) >> 5;
+    // open-addressing position table for R: H[h] = 1 + position (0 = empty), size a
+    // power of two >= 4 |R| (load <= 1/4: ~1.2 probes per lookup)
+    uint32_t hbits = 2;
+    while ((1u << hbits) < 4 * L) hbits++;
+    const uint32_t hmask = (1u << hbits) - 1u;
     for (uint32_t i = tid; i < L; i += kTeamThreads) R[i] = a.dag_col[b0 + i];
     for (uint32_t i = tid; i < L * W; i += kTeamThreads) B[i] = 0u;
+    for (uint32_t i = tid; i <= hmask / 2; i += kTeamThreads) reinterpret_cast<uint32_t *>(H)[i] = 0u;
     if (tid == 0) entries += L;
+    team_sync<TEAM_WARPS>();
+    for (uint32_t i = tid; i < L; i += kTeamThreads) {
+      uint32_t h = (R[i] * 0x9E3779B1u) >> (32 - hbits);
+      while (atomicCAS(&H[h], (unsigned short)0, (unsigned short)(i + 1)) != 0) h = (h + 1) & hmask;
+    }
     team_sync<TEAM_WARPS>();
     const uint32_t rmin = R[0], rmax = R[L - 1];
     // ---- depth-2 extension: row i = positions of R ∩ N+(R[i]) (flattened windows) ----
-    uint64_t hits = 0;
     for (uint32_t w0 = wit * 32; w0 < L; w0 += TEAM_WARPS * 32) {
       const uint32_t i = w0 + lane;
       uint32_t beg = 0, dl = 0;
@@ -230,20 +237,27 @@ __global__ void __launch_bounds__(256) kcl_bitmap_kernel(BmArgs a) {
         int p = -1;
         if (t < T) {
           const uint32_t y = __ldg(a.dag_col + bj + (t - oj));
-          if (y >= rmin && y <= rmax) p = find_pos(R, L, y);
+          if (y >= rmin && y <= rmax) {
+            uint32_t h = (y * 0x9E3779B1u) >> (32 - hbits);
+            for (;;) {
+              const uint32_t e = H[h];
+              if (e == 0) break;
+              if (R[e - 1] == y) {
+                p = (int)e - 1;
+                break;
+              }
+              h = (h + 1) & hmask;
+            }
+          }
         }
         if (p >= 0) atomicOr(&B[rj * W + (p >> 5)], 1u << (p & 31));
-        hits += __popc(__ballot_sync(0xffffffffu, p >= 0)) * (lane == 0);
       }
     }
     team_sync<TEAM_WARPS>();
-    // ---- deeper extensions: bitmap DFS, one first-level child per thread ----
+    // ---- deeper extensions: bitmap DFS, one first-level child per thread (k = 3:
+    // the popcount of each row) ----
     uint64_t cnt = 0;
-    if (a.k == 3) {
-      cnt = hits;
-    } else {
-      for (uint32_t j1 = tid; j1 < L; j1 += kTeamThreads) cnt += dfs_from<TW>(B, W, j1, a.k);
-    }
+    for (uint32_t j1 = tid; j1 < L; j1 += kTeamThreads) cnt += dfs_from<TW>(B, W, j1, a.k);
     total += cnt;
     if (PER_ROOT) {
 #pragma unroll
@@ -267,7 +281,7 @@ __global__ void __launch_bounds__(256) kcl_bitmap_kernel(BmArgs a) {
 
 template <int TEAM_WARPS, int TW>
 constexpr size_t bm_smem() {
-  return (size_t)(256 / (TEAM_WARPS * 32)) * (TW * 32 + TW * 32 * TW + 1) * sizeof(uint32_t);
+  return (size_t)(256 / (TEAM_WARPS * 32)) * team_words<TW>() * sizeof(uint32_t);
 }
 
 template <int TEAM_WARPS, int TW>
