@@ -72,21 +72,18 @@ __device__ __forceinline__ uint32_t popc_and(const uint32_t (&x)[TW], const uint
   return c;
 }
 
-// Count the k-cliques whose two lowest vertices are (v, R[j1]): DFS over the bitmap
-// rows B (stride W words), starting from cur = B[j1].
+// Count the k-cliques that extend a clique of `chosen` vertices whose common
+// candidates (a subset of R) are the bitmap `cur`: DFS over the rows B (stride W).
 template <int TW>
-__device__ uint64_t dfs_from(const uint32_t *B, uint32_t W, uint32_t j1, uint32_t k) {
-  uint32_t cur[TW];
+__device__ uint64_t dfs_count(const uint32_t *B, uint32_t W, const uint32_t (&cur)[TW], uint32_t chosen,
+                              uint32_t k) {
   uint32_t c0 = 0;
 #pragma unroll
-  for (int w = 0; w < TW; w++) {
-    cur[w] = (w < (int)W) ? B[j1 * W + w] : 0u;
-    c0 += __popc(cur[w]);
-  }
-  if (k == 3) return c0;
-  if (c0 < k - 2) return 0;
+  for (int w = 0; w < TW; w++) c0 += __popc(cur[w]);
+  if (chosen + 1 == k) return c0;   // each candidate completes one k-clique
+  if (c0 < k - chosen) return 0;
   uint64_t cnt = 0;
-  if (k == 4) {   // sum over j in cur of |cur ∩ B_j|
+  if (chosen + 2 == k) {   // sum over j in cur of |cur ∩ B_j|
     uint32_t pos = 0;
     for (;;) {
       const int j = next_bit<TW>(cur, pos, W);
@@ -113,7 +110,7 @@ __device__ uint64_t dfs_from(const uint32_t *B, uint32_t W, uint32_t j1, uint32_
       continue;
     }
     pos[s] = j + 1;
-    const uint32_t t = s + 3;            // vertices chosen after taking j
+    const uint32_t t = s + chosen + 1;   // vertices chosen after taking j
     uint32_t nx[TW];
     const uint32_t c = popc_and<TW>(top, B + j * W, W, nx);
     if (t == k - 1) {
@@ -136,10 +133,10 @@ __device__ __forceinline__ void team_sync() {
 }
 
 // Shared words per team: run R (32 TW), bitmap rows B (32 TW x TW), position hash
-// H (4 x 32 TW u16 = 64 TW words), work slot.
+// H (4 x 32 TW u16 = 64 TW words), row offsets P (32 TW + 1), work slot.
 template <int TW>
 constexpr int team_words() {
-  return TW * 32 + TW * 32 * TW + 2 * TW * 32 + 1;
+  return TW * 32 + TW * 32 * TW + 2 * TW * 32 + TW * 32 + 1 + 1;
 }
 
 template <int TEAM_WARPS, int TW, bool PER_ROOT>
@@ -154,7 +151,8 @@ __global__ void __launch_bounds__(256) kcl_bitmap_kernel(BmArgs a) {
   uint32_t *R = smem + team * team_words<TW>();
   uint32_t *B = R + kRunMax;
   unsigned short *H = reinterpret_cast<unsigned short *>(B + kRunMax * TW);   // 4 kRunMax entries
-  uint32_t *slot = B + kRunMax * TW + 2 * kRunMax;   // work index broadcast (CTA teams)
+  uint32_t *P = B + kRunMax * TW + 2 * kRunMax;       // exclusive scan of row popcounts
+  uint32_t *slot = P + kRunMax + 1;                    // work index broadcast (CTA teams)
   uint64_t total = 0, elems = 0, entries = 0;
 
   // warp teams take roots in batches of 4 (one atomic per batch); CTA teams one
@@ -254,10 +252,58 @@ __global__ void __launch_bounds__(256) kcl_bitmap_kernel(BmArgs a) {
       }
     }
     team_sync<TEAM_WARPS>();
-    // ---- deeper extensions: bitmap DFS, one first-level child per thread (k = 3:
-    // the popcount of each row) ----
+    // ---- deeper extensions: bitmap DFS.  k = 3: one row per thread (its popcount).
+    // k >= 4: the work items are the triangles (v, R[j1], R[j2]), j2 in row j1 --
+    // fine-grained enough to balance the team; item q -> (j1, j2) through the
+    // exclusive scan P of the row popcounts ----
     uint64_t cnt = 0;
-    for (uint32_t j1 = tid; j1 < L; j1 += kTeamThreads) cnt += dfs_from<TW>(B, W, j1, a.k);
+    if (a.k == 3) {
+      for (uint32_t j1 = tid; j1 < L; j1 += kTeamThreads) {
+        uint32_t c = 0;
+        for (uint32_t w = 0; w < W; w++) c += __popc(B[j1 * W + w]);
+        cnt += c;
+      }
+    } else {
+      if (wit == 0) {   // warp 0 of the team scans the row popcounts
+        uint32_t carry = 0;
+        for (uint32_t r0 = 0; r0 < L; r0 += 32) {
+          const uint32_t r = r0 + lane;
+          uint32_t c = 0;
+          if (r < L)
+            for (uint32_t w = 0; w < W; w++) c += __popc(B[r * W + w]);
+          uint32_t tot;
+          const uint32_t ex = excl_scan32(c, lane, tot);
+          if (r < L) P[r] = carry + ex;
+          carry += tot;
+        }
+        if (lane == 0) P[L] = carry;
+      }
+      team_sync<TEAM_WARPS>();
+      const uint32_t items = P[L];
+      for (uint32_t q = tid; q < items; q += kTeamThreads) {
+        uint32_t lo = 0, hi = L;   // j1 = last row with P[j1] <= q
+        while (hi - lo > 1) {
+          const uint32_t mid = (lo + hi) >> 1;
+          if (P[mid] <= q) lo = mid; else hi = mid;
+        }
+        const uint32_t j1 = lo;
+        uint32_t r = q - P[j1], j2 = 0;
+        for (uint32_t w = 0; w < W; w++) {
+          const uint32_t word = B[j1 * W + w];
+          const uint32_t pc = __popc(word);
+          if (r < pc) {
+            j2 = w * 32 + __fns(word, 0, r + 1);
+            break;
+          }
+          r -= pc;
+        }
+        uint32_t cur[TW];
+#pragma unroll
+        for (int w = 0; w < TW; w++)
+          cur[w] = (w < (int)W) ? (B[j1 * W + w] & B[j2 * W + w]) : 0u;
+        cnt += dfs_count<TW>(B, W, cur, 3, a.k);
+      }
+    }
     total += cnt;
     if (PER_ROOT) {
 #pragma unroll
