@@ -83,6 +83,8 @@ typedef struct {
                                           (exercises the hub / long-run code path)   */
 #define GAMMA_FLAG_NO_BITMAP    0x10u  /* kCL: use the ET-level path for every root
                                           (no local-bitmap DFS; ablation / testing)  */
+#define GAMMA_FLAG_NO_SPLIT     0x20u  /* kCL bitmap path: never split heavy roots    */
+#define GAMMA_FLAG_DEBUG_SPLIT_ALL 0x40u /* test hook: split every root (k >= 6)      */
 
 /* Create / destroy a context.  Errors: E_INVAL (NULL args), E_CUDA (no device). */
 gamma_status gamma_ctx_create(const gamma_ctx_desc *desc, gamma_ctx **out);

@@ -22,6 +22,9 @@ GAMMA_FLAG_TIME_KERNELS = 0x1
 GAMMA_FLAG_NO_FUSE = 0x2
 GAMMA_FLAG_SPILL = 0x4
 GAMMA_FLAG_DEBUG_NOSTAGE = 0x8
+GAMMA_FLAG_NO_BITMAP = 0x10
+GAMMA_FLAG_NO_SPLIT = 0x20
+GAMMA_FLAG_DEBUG_SPLIT_ALL = 0x40
 
 ALLOC_FN = C.CFUNCTYPE(C.c_void_p, C.c_size_t, C.c_void_p, C.c_void_p)
 FREE_FN = C.CFUNCTYPE(None, C.c_void_p, C.c_void_p)

@@ -9,11 +9,15 @@
 // positions; every deeper extension is then a W-word AND of rows, and the last one
 // is a popcount (the last extension is counted, not stored).  The
 // embedding table below the root is held as these bitmaps, in shared memory, and
-// walked depth-first per thread (BFS across roots, DFS inside a root).
+// walked depth-first (BFS across roots, DFS inside a root).
 //
 // Teams: one warp per root for |R| <= 128 (rows of <= 4 words), one CTA per root for
-// 128 < |R| <= 512 (<= 16 words).  Longer runs (and k > 12) use the ET-level path
-// in kclique.cu.
+// 128 < |R| <= 512 (<= 16 words).  Work inside a root is split into the root's
+// triangles (v, R[j1], R[j2]) so the team stays balanced.  Roots whose 4-clique
+// count exceeds a cut (k >= 6 only, where the DFS below a triangle is deep) are not
+// expanded by their team: they are cut into parts that separate CTAs take from a
+// work list in a second launch (hub splitting, SURVEY.md §7 "skew").  Longer runs
+// (and k > 12) use the ET-level path in kclique.cu.
 #include <algorithm>
 
 #include "device_common.cuh"
@@ -23,7 +27,9 @@ namespace gamma_impl {
 
 namespace {
 
-constexpr int kMaxStack = 10;   // DFS levels below the first child: k <= 12
+constexpr int kMaxStack = 10;        // DFS levels below the first child: k <= 12
+constexpr uint32_t kPartCost = 4096; // 4-cliques per heavy-root part
+constexpr uint32_t kMaxParts = 4096;
 
 struct BmArgs {
   const uint64_t *dag_ptr;
@@ -34,6 +40,10 @@ struct BmArgs {
   uint32_t len_lo, len_hi;    // this launch handles roots with len_lo < |R| <= len_hi
   unsigned long long *ctrl;
   unsigned long long *per_root;
+  // hub splitting (k >= 6): roots with more than heavy_cut 4-cliques are deferred
+  uint64_t heavy_cut;         // 0: never defer
+  uint2 *parts;               // (root index, part | nparts << 16)
+  uint32_t parts_cap;
 };
 
 __device__ __forceinline__ uint32_t excl_scan32(uint32_t x, int lane, uint32_t &total) {
@@ -133,26 +143,172 @@ __device__ __forceinline__ void team_sync() {
 }
 
 // Shared words per team: run R (32 TW), bitmap rows B (32 TW x TW), position hash
-// H (4 x 32 TW u16 = 64 TW words), row offsets P (32 TW + 1), work slot.
+// H (4 x 32 TW u16 = 64 TW words), row offsets P (32 TW + 1, padded to +2), two
+// broadcast slots (8-byte aligned: every region starts at an even word).
 template <int TW>
 constexpr int team_words() {
-  return TW * 32 + TW * 32 * TW + 2 * TW * 32 + TW * 32 + 1 + 1;
+  return TW * 32 + TW * 32 * TW + 2 * TW * 32 + TW * 32 + 2 + 2;
+}
+
+template <int TW>
+struct TeamMem {
+  uint32_t *R, *B, *P, *slot;
+  unsigned short *H;
+  __device__ TeamMem(uint32_t *base) {
+    R = base;
+    B = R + TW * 32;
+    H = reinterpret_cast<unsigned short *>(B + TW * 32 * TW);
+    P = B + TW * 32 * TW + 2 * TW * 32;
+    slot = P + TW * 32 + 2;
+  }
+};
+
+// Depth-2 extension of root v: R = N+(v), rows B[i] = positions of R ∩ N+(R[i]).
+// Flattened windows of 32 children; each list element is located in R through a
+// shared-memory open-addressing position table.  Returns Σ|N+(c)| (for the bytes).
+template <int TEAM_WARPS, int TW>
+__device__ uint64_t build_rows(const BmArgs &a, const TeamMem<TW> &m, uint64_t b0, uint32_t L, int tid, int lane) {
+  constexpr int kTeamThreads = TEAM_WARPS * 32;
+  const int wit = tid >> 5;
+  const uint32_t W = (L + 31) >> 5;
+  uint32_t hbits = 2;
+  while ((1u << hbits) < 4 * L) hbits++;
+  const uint32_t hmask = (1u << hbits) - 1u;
+  for (uint32_t i = tid; i < L; i += kTeamThreads) m.R[i] = a.dag_col[b0 + i];
+  for (uint32_t i = tid; i < L * W; i += kTeamThreads) m.B[i] = 0u;
+  for (uint32_t i = tid; i <= hmask / 2; i += kTeamThreads) reinterpret_cast<uint32_t *>(m.H)[i] = 0u;
+  team_sync<TEAM_WARPS>();
+  for (uint32_t i = tid; i < L; i += kTeamThreads) {
+    uint32_t h = (m.R[i] * 0x9E3779B1u) >> (32 - hbits);
+    while (atomicCAS(&m.H[h], (unsigned short)0, (unsigned short)(i + 1)) != 0) h = (h + 1) & hmask;
+  }
+  team_sync<TEAM_WARPS>();
+  const uint32_t rmin = m.R[0], rmax = m.R[L - 1];
+  uint64_t elems = 0;
+  for (uint32_t w0 = wit * 32; w0 < L; w0 += TEAM_WARPS * 32) {
+    const uint32_t i = w0 + lane;
+    uint32_t beg = 0, dl = 0;
+    if (i < L) {
+      const uint32_t c = m.R[i];
+      const uint64_t cb = a.dag_ptr[c];
+      dl = (uint32_t)(a.dag_ptr[c + 1] - cb);
+      beg = (uint32_t)cb;
+    }
+    elems += dl;
+    // compact the children with non-empty lists to lanes 0..nnz-1 (every list then
+    // has a distinct start offset) and exclusive-scan their lengths
+    const uint32_t nz = __ballot_sync(0xffffffffu, dl > 0);
+    const uint32_t nnz = __popc(nz);
+    const uint32_t src = lane < (int)nnz ? __fns(nz, 0, lane + 1) : 0;
+    const uint32_t cbeg = __shfl_sync(0xffffffffu, beg, src);
+    const uint32_t sdl = __shfl_sync(0xffffffffu, dl, src);
+    const uint32_t cdl = lane < (int)nnz ? sdl : 0u;
+    const uint32_t crow = w0 + src;
+    uint32_t T;
+    const uint32_t o = excl_scan32(cdl, lane, T);
+    const uint32_t upto = lane == 31 ? 0xffffffffu : ((2u << lane) - 1u);
+    uint32_t nb = 0;   // lists that started before this tile
+    for (uint32_t t0 = 0; t0 < T; t0 += 32) {
+      const uint32_t t = t0 + lane;
+      // lane t's list = the last list starting at or before t: one OR-reduction of the
+      // start offsets that fall in this tile
+      const uint32_t mine = (lane < (int)nnz && o >= t0 && o < t0 + 32) ? (1u << (o - t0)) : 0u;
+      const uint32_t S = __reduce_or_sync(0xffffffffu, mine);
+      const int j = (int)(nb + __popc(S & upto)) - 1;
+      nb += __popc(S);
+      const uint32_t bj = __shfl_sync(0xffffffffu, cbeg, j & 31);
+      const uint32_t oj = __shfl_sync(0xffffffffu, o, j & 31);
+      const uint32_t rj = __shfl_sync(0xffffffffu, crow, j & 31);
+      if (t < T) {
+        const uint32_t y = __ldg(a.dag_col + bj + (t - oj));
+        if (y >= rmin && y <= rmax) {
+          uint32_t h = (y * 0x9E3779B1u) >> (32 - hbits);
+          for (;;) {
+            const uint32_t e = m.H[h];
+            if (e == 0) break;
+            if (m.R[e - 1] == y) {
+              atomicOr(&m.B[rj * W + ((e - 1) >> 5)], 1u << ((e - 1) & 31));
+              break;
+            }
+            h = (h + 1) & hmask;
+          }
+        }
+      }
+    }
+  }
+  team_sync<TEAM_WARPS>();
+  return elems;
+}
+
+// P[r] = exclusive scan of the row popcounts (the triangle items), P[L] = total.
+template <int TEAM_WARPS, int TW>
+__device__ void scan_rows(const TeamMem<TW> &m, uint32_t L, int tid, int lane) {
+  const uint32_t W = (L + 31) >> 5;
+  if ((tid >> 5) == 0) {
+    uint32_t carry = 0;
+    for (uint32_t r0 = 0; r0 < L; r0 += 32) {
+      const uint32_t r = r0 + lane;
+      uint32_t c = 0;
+      if (r < L)
+        for (uint32_t w = 0; w < W; w++) c += __popc(m.B[r * W + w]);
+      uint32_t tot;
+      const uint32_t ex = excl_scan32(c, lane, tot);
+      if (r < L) m.P[r] = carry + ex;
+      carry += tot;
+    }
+    if (lane == 0) m.P[L] = carry;
+  }
+  team_sync<TEAM_WARPS>();
+}
+
+// Item q -> candidates of the triangle (v, R[j1], R[j2]).
+template <int TW>
+__device__ __forceinline__ void item_cur(const TeamMem<TW> &m, uint32_t L, uint32_t W, uint32_t q,
+                                         uint32_t (&cur)[TW]) {
+  uint32_t lo = 0, hi = L;   // j1 = last row with P[j1] <= q
+  while (hi - lo > 1) {
+    const uint32_t mid = (lo + hi) >> 1;
+    if (m.P[mid] <= q) lo = mid; else hi = mid;
+  }
+  const uint32_t j1 = lo;
+  uint32_t r = q - m.P[j1], j2 = 0;
+  for (uint32_t w = 0; w < W; w++) {
+    const uint32_t word = m.B[j1 * W + w];
+    const uint32_t pc = __popc(word);
+    if (r < pc) {
+      j2 = w * 32 + __fns(word, 0, r + 1);
+      break;
+    }
+    r -= pc;
+  }
+#pragma unroll
+  for (int w = 0; w < TW; w++) cur[w] = (w < (int)W) ? (m.B[j1 * W + w] & m.B[j2 * W + w]) : 0u;
+}
+
+template <int TEAM_WARPS>
+__device__ __forceinline__ uint64_t team_sum(uint64_t x, int lane, uint32_t *slot) {
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) x += __shfl_down_sync(0xffffffffu, x, off);
+  x = __shfl_sync(0xffffffffu, x, 0);
+  if (TEAM_WARPS == 1) return x;
+  unsigned long long *s64 = reinterpret_cast<unsigned long long *>(slot);   // 8-byte aligned slot pair
+  if (threadIdx.x == 0) *s64 = 0;
+  __syncthreads();
+  if (lane == 0) atomicAdd(s64, (unsigned long long)x);
+  __syncthreads();
+  const uint64_t r = *s64;
+  __syncthreads();
+  return r;
 }
 
 template <int TEAM_WARPS, int TW, bool PER_ROOT>
 __global__ void __launch_bounds__(256) kcl_bitmap_kernel(BmArgs a) {
   extern __shared__ uint32_t smem[];
   constexpr int kTeamThreads = TEAM_WARPS * 32;
-  constexpr int kRunMax = TW * 32;
   const int lane = threadIdx.x & 31;
   const int team = threadIdx.x / kTeamThreads;
   const int tid = threadIdx.x % kTeamThreads;
-  const int wit = tid >> 5;   // warp index inside the team
-  uint32_t *R = smem + team * team_words<TW>();
-  uint32_t *B = R + kRunMax;
-  unsigned short *H = reinterpret_cast<unsigned short *>(B + kRunMax * TW);   // 4 kRunMax entries
-  uint32_t *P = B + kRunMax * TW + 2 * kRunMax;       // exclusive scan of row popcounts
-  uint32_t *slot = P + kRunMax + 1;                    // work index broadcast (CTA teams)
+  const TeamMem<TW> m(smem + team * team_words<TW>());
   uint64_t total = 0, elems = 0, entries = 0;
 
   // warp teams take roots in batches of 4 (one atomic per batch); CTA teams one
@@ -166,9 +322,9 @@ __global__ void __launch_bounds__(256) kcl_bitmap_kernel(BmArgs a) {
       if (TEAM_WARPS == 1) {
         base = __shfl_sync(0xffffffffu, base, 0);
       } else {
-        if (tid == 0) *slot = base < 0xffffffffull ? (uint32_t)base : 0xffffffffu;
+        if (tid == 0) m.slot[0] = base < 0xffffffffull ? (uint32_t)base : 0xffffffffu;
         __syncthreads();
-        base = *slot;
+        base = m.slot[0];
         __syncthreads();
       }
       next = base;
@@ -181,128 +337,55 @@ __global__ void __launch_bounds__(256) kcl_bitmap_kernel(BmArgs a) {
     const uint32_t L = (uint32_t)(a.dag_ptr[v + 1] - b0);
     if (L <= a.len_lo || L > a.len_hi || L < a.k - 1) continue;   // uniform across the team
     const uint32_t W = (L + 31) >> 5;
-    // open-addressing position table for R: H[h] = 1 + position (0 = empty), size a
-    // power of two >= 4 |R| (load <= 1/4: ~1.2 probes per lookup)
-    uint32_t hbits = 2;
-    while ((1u << hbits) < 4 * L) hbits++;
-    const uint32_t hmask = (1u << hbits) - 1u;
-    for (uint32_t i = tid; i < L; i += kTeamThreads) R[i] = a.dag_col[b0 + i];
-    for (uint32_t i = tid; i < L * W; i += kTeamThreads) B[i] = 0u;
-    for (uint32_t i = tid; i <= hmask / 2; i += kTeamThreads) reinterpret_cast<uint32_t *>(H)[i] = 0u;
     if (tid == 0) entries += L;
-    team_sync<TEAM_WARPS>();
-    for (uint32_t i = tid; i < L; i += kTeamThreads) {
-      uint32_t h = (R[i] * 0x9E3779B1u) >> (32 - hbits);
-      while (atomicCAS(&H[h], (unsigned short)0, (unsigned short)(i + 1)) != 0) h = (h + 1) & hmask;
-    }
-    team_sync<TEAM_WARPS>();
-    const uint32_t rmin = R[0], rmax = R[L - 1];
-    // ---- depth-2 extension: row i = positions of R ∩ N+(R[i]) (flattened windows) ----
-    for (uint32_t w0 = wit * 32; w0 < L; w0 += TEAM_WARPS * 32) {
-      const uint32_t i = w0 + lane;
-      uint32_t beg = 0, dl = 0;
-      if (i < L) {
-        const uint32_t c = R[i];
-        const uint64_t cb = a.dag_ptr[c];
-        dl = (uint32_t)(a.dag_ptr[c + 1] - cb);
-        beg = (uint32_t)cb;
-      }
-      elems += dl;
-      // compact the children with non-empty lists to lanes 0..nnz-1 (so that every
-      // list has a distinct start offset), then exclusive-scan their lengths
-      const uint32_t nz = __ballot_sync(0xffffffffu, dl > 0);
-      const uint32_t nnz = __popc(nz);
-      const uint32_t src = lane < (int)nnz ? __fns(nz, 0, lane + 1) : 0;
-      const uint32_t cbeg = __shfl_sync(0xffffffffu, beg, src);
-      const uint32_t sdl = __shfl_sync(0xffffffffu, dl, src);
-      const uint32_t cdl = lane < (int)nnz ? sdl : 0u;
-      const uint32_t crow = w0 + src;
-      uint32_t T;
-      const uint32_t o = excl_scan32(cdl, lane, T);
-      const uint32_t upto = lane == 31 ? 0xffffffffu : ((2u << lane) - 1u);
-      uint32_t nb = 0;   // lists that started before this tile
-      for (uint32_t t0 = 0; t0 < T; t0 += 32) {
-        const uint32_t t = t0 + lane;
-        // lane t's list = the last list starting at or before t: one OR-reduction of
-        // the start offsets that fall in this tile
-        const uint32_t mine = (lane < (int)nnz && o >= t0 && o < t0 + 32) ? (1u << (o - t0)) : 0u;
-        const uint32_t S = __reduce_or_sync(0xffffffffu, mine);
-        const int j = (int)(nb + __popc(S & upto)) - 1;
-        nb += __popc(S);
-        const uint32_t bj = __shfl_sync(0xffffffffu, cbeg, j & 31);
-        const uint32_t oj = __shfl_sync(0xffffffffu, o, j & 31);
-        const uint32_t rj = __shfl_sync(0xffffffffu, crow, j & 31);
-        int p = -1;
-        if (t < T) {
-          const uint32_t y = __ldg(a.dag_col + bj + (t - oj));
-          if (y >= rmin && y <= rmax) {
-            uint32_t h = (y * 0x9E3779B1u) >> (32 - hbits);
-            for (;;) {
-              const uint32_t e = H[h];
-              if (e == 0) break;
-              if (R[e - 1] == y) {
-                p = (int)e - 1;
-                break;
-              }
-              h = (h + 1) & hmask;
-            }
-          }
-        }
-        if (p >= 0) atomicOr(&B[rj * W + (p >> 5)], 1u << (p & 31));
-      }
-    }
-    team_sync<TEAM_WARPS>();
+    elems += build_rows<TEAM_WARPS, TW>(a, m, b0, L, tid, lane);
     // ---- deeper extensions: bitmap DFS.  k = 3: one row per thread (its popcount).
-    // k >= 4: the work items are the triangles (v, R[j1], R[j2]), j2 in row j1 --
-    // fine-grained enough to balance the team; item q -> (j1, j2) through the
-    // exclusive scan P of the row popcounts ----
+    // k >= 4: the work items are the triangles (v, R[j1], R[j2]), j2 in row j1 ----
     uint64_t cnt = 0;
     if (a.k == 3) {
       for (uint32_t j1 = tid; j1 < L; j1 += kTeamThreads) {
         uint32_t c = 0;
-        for (uint32_t w = 0; w < W; w++) c += __popc(B[j1 * W + w]);
+        for (uint32_t w = 0; w < W; w++) c += __popc(m.B[j1 * W + w]);
         cnt += c;
       }
     } else {
-      if (wit == 0) {   // warp 0 of the team scans the row popcounts
-        uint32_t carry = 0;
-        for (uint32_t r0 = 0; r0 < L; r0 += 32) {
-          const uint32_t r = r0 + lane;
+      scan_rows<TEAM_WARPS, TW>(m, L, tid, lane);
+      const uint32_t items = m.P[L];
+      bool deferred = false;
+      if (a.heavy_cut) {   // hub splitting: estimate the DFS by the 4-clique count
+        uint64_t est = 0;
+        for (uint32_t q = tid; q < items; q += kTeamThreads) {
+          uint32_t cur[TW];
+          item_cur<TW>(m, L, W, q, cur);
           uint32_t c = 0;
-          if (r < L)
-            for (uint32_t w = 0; w < W; w++) c += __popc(B[r * W + w]);
-          uint32_t tot;
-          const uint32_t ex = excl_scan32(c, lane, tot);
-          if (r < L) P[r] = carry + ex;
-          carry += tot;
-        }
-        if (lane == 0) P[L] = carry;
-      }
-      team_sync<TEAM_WARPS>();
-      const uint32_t items = P[L];
-      for (uint32_t q = tid; q < items; q += kTeamThreads) {
-        uint32_t lo = 0, hi = L;   // j1 = last row with P[j1] <= q
-        while (hi - lo > 1) {
-          const uint32_t mid = (lo + hi) >> 1;
-          if (P[mid] <= q) lo = mid; else hi = mid;
-        }
-        const uint32_t j1 = lo;
-        uint32_t r = q - P[j1], j2 = 0;
-        for (uint32_t w = 0; w < W; w++) {
-          const uint32_t word = B[j1 * W + w];
-          const uint32_t pc = __popc(word);
-          if (r < pc) {
-            j2 = w * 32 + __fns(word, 0, r + 1);
-            break;
-          }
-          r -= pc;
-        }
-        uint32_t cur[TW];
 #pragma unroll
-        for (int w = 0; w < TW; w++)
-          cur[w] = (w < (int)W) ? (B[j1 * W + w] & B[j2 * W + w]) : 0u;
-        cnt += dfs_count<TW>(B, W, cur, 3, a.k);
+          for (int w = 0; w < TW; w++) c += __popc(cur[w]);
+          est += c;
+        }
+        est = team_sum<TEAM_WARPS>(est, lane, m.slot);
+        if (est > a.heavy_cut) {
+          const uint64_t want = est / kPartCost + 1;
+          const uint32_t nparts = want < kMaxParts ? (uint32_t)want : kMaxParts;
+          if (tid == 0) {
+            const unsigned long long at = atomicAdd(&a.ctrl[CTRL_AUX1], (unsigned long long)nparts);
+            if (at + nparts <= a.parts_cap) {
+              for (uint32_t p = 0; p < nparts; p++) a.parts[at + p] = make_uint2((uint32_t)gi, p | (nparts << 16));
+              m.slot[0] = 1;
+            } else {
+              m.slot[0] = 0;   // list full: expand here
+            }
+          }
+          team_sync<TEAM_WARPS>();
+          deferred = m.slot[0] == 1;
+          team_sync<TEAM_WARPS>();
+        }
       }
+      if (!deferred)
+        for (uint32_t q = tid; q < items; q += kTeamThreads) {
+          uint32_t cur[TW];
+          item_cur<TW>(m, L, W, q, cur);
+          cnt += dfs_count<TW>(m.B, W, cur, 3, a.k);
+        }
     }
     total += cnt;
     if (PER_ROOT) {
@@ -323,6 +406,53 @@ __global__ void __launch_bounds__(256) kcl_bitmap_kernel(BmArgs a) {
     atomicAdd(&a.ctrl[CTRL_ELEMS], (unsigned long long)elems);
     atomicAdd(&a.ctrl[CTRL_AUX0], (unsigned long long)entries);
   }
+}
+
+// Second launch for the deferred heavy roots: one CTA per (root, part); the part
+// rebuilds the root's rows (cheap next to the DFS) and takes every nparts-th item.
+template <bool PER_ROOT>
+__global__ void __launch_bounds__(256) kcl_bitmap_parts_kernel(BmArgs a, uint64_t nparts_total) {
+  extern __shared__ uint32_t smem[];
+  constexpr int TW = 16;
+  const int lane = threadIdx.x & 31;
+  const int tid = threadIdx.x;
+  const TeamMem<TW> m(smem);
+  uint64_t total = 0;
+  for (;;) {
+    if (tid == 0) {
+      const unsigned long long w = atomicAdd(&a.ctrl[CTRL_WORK], 1ull);
+      m.slot[0] = w < nparts_total ? (uint32_t)w : 0xffffffffu;
+    }
+    __syncthreads();
+    const uint32_t wi = m.slot[0];
+    __syncthreads();
+    if (wi == 0xffffffffu) break;
+    const uint2 pt = a.parts[wi];
+    const uint32_t gi = pt.x, part = pt.y & 0xffff, nparts = pt.y >> 16;
+    const uint32_t v = a.roots[gi];
+    const uint64_t b0 = a.dag_ptr[v];
+    const uint32_t L = (uint32_t)(a.dag_ptr[v + 1] - b0);
+    const uint32_t W = (L + 31) >> 5;
+    build_rows<8, TW>(a, m, b0, L, tid, lane);
+    scan_rows<8, TW>(m, L, tid, lane);
+    const uint32_t items = m.P[L];
+    uint64_t cnt = 0;
+    for (uint32_t q = part + tid * nparts; q < items; q += 256 * nparts) {
+      uint32_t cur[TW];
+      item_cur<TW>(m, L, W, q, cur);
+      cnt += dfs_count<TW>(m.B, W, cur, 3, a.k);
+    }
+    total += cnt;
+    if (PER_ROOT) {
+#pragma unroll
+      for (int off = 16; off > 0; off >>= 1) cnt += __shfl_down_sync(0xffffffffu, cnt, off);
+      if (lane == 0 && cnt) atomicAdd(&a.per_root[gi], (unsigned long long)cnt);
+    }
+    __syncthreads();
+  }
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) total += __shfl_down_sync(0xffffffffu, total, off);
+  if (lane == 0 && total) atomicAdd(&a.ctrl[CTRL_COUNT], (unsigned long long)total);
 }
 
 template <int TEAM_WARPS, int TW>
@@ -354,14 +484,33 @@ uint64_t run_bitmap(gamma_ctx *ctx, const BmArgs &a0, bool per_root) {
   ctx->stats.list_elems += h[CTRL_ELEMS];
   ctx->stats.level_entries[2] += h[CTRL_AUX0];
   ctx->stats.alg_bytes[KC_BITMAP] += 4 * h[CTRL_AUX0] + 4 * h[CTRL_ELEMS];
-  return h[CTRL_COUNT];
+  uint64_t count = h[CTRL_COUNT];
+  const uint64_t nparts = std::min<uint64_t>(h[CTRL_AUX1], a0.parts_cap);
+  if (nparts) {   // the deferred heavy roots, one CTA per part
+    static bool pattr = false;
+    if (!pattr) {
+      GAMMA_CUDA(cudaFuncSetAttribute(kcl_bitmap_parts_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                      (int)bm_smem<8, 16>()));
+      GAMMA_CUDA(cudaFuncSetAttribute(kcl_bitmap_parts_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                      (int)bm_smem<8, 16>()));
+      pattr = true;
+    }
+    const int pgrid = ctx->num_sms * occupancy_blocks((const void *)kcl_bitmap_parts_kernel<false>, 256,
+                                                      bm_smem<8, 16>());
+    ctrl_reset(ctx);
+    ctx->launch(KC_BITMAP, [&] {
+      if (per_root)
+        kcl_bitmap_parts_kernel<true><<<pgrid, 256, bm_smem<8, 16>(), ctx->stream>>>(a0, nparts);
+      else
+        kcl_bitmap_parts_kernel<false><<<pgrid, 256, bm_smem<8, 16>(), ctx->stream>>>(a0, nparts);
+    });
+    ctrl_fetch(ctx);
+    count = checked_add(count, ctx->ctrl_host[CTRL_COUNT]);
+    ctx->stats.chunks += nparts;
+  }
+  return count;
 }
 
-}  // namespace
-
-// Count k-cliques rooted at roots[0..nroots) whose run length is <= 512 (k <= 12);
-// longer runs are left to the ET path.  per_root (nullable) indexed like roots.
-namespace {
 // out[0] = #roots with |N+(v)| > 512, out[1] = #roots with |N+(v)| > 128
 __global__ void count_len_classes(const uint64_t *dag_ptr, const uint32_t *roots, uint64_t nr,
                                   unsigned long long *out) {
@@ -381,8 +530,11 @@ __global__ void count_len_classes(const uint64_t *dag_ptr, const uint32_t *roots
     if (c1) atomicAdd(&out[1], c1);
   }
 }
+
 }  // namespace
 
+// Count k-cliques rooted at roots[0..nroots) whose run length is <= 512 (k <= 12);
+// longer runs are left to the ET path.  per_root (nullable) indexed like roots.
 uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint64_t nroots,
                         unsigned long long *per_root, bool sorted) {
   gamma_ctx *ctx = g->ctx;
@@ -394,6 +546,14 @@ uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint6
   a.k = k;
   a.ctrl = (unsigned long long *)ctx->ctrl;
   a.per_root = per_root;
+  // hub splitting only pays when the DFS below a triangle is deep (k >= 6)
+  DevBuf<uint2> parts;
+  if (k >= 6 && (ctx->desc.flags & GAMMA_FLAG_NO_SPLIT) == 0) {
+    a.parts_cap = 1u << 20;
+    parts = DevBuf<uint2>(ctx, a.parts_cap);
+    a.parts = parts.p;
+    a.heavy_cut = (ctx->desc.flags & GAMMA_FLAG_DEBUG_SPLIT_ALL) ? 1 : 4ull * kPartCost;
+  }
   uint64_t total = 0;
   // Roots sorted by cost (d+^2, descending) fall into three contiguous classes:
   // [0, n_long) ET path, [n_long, n_mid) CTA teams, [n_mid, nroots) warp teams.
@@ -417,6 +577,7 @@ uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint6
   if (g->max_out_degree > 128 && (!sorted || n_mid > n_long)) {
     a.roots = roots + (sorted ? n_long : 0);
     a.nroots = sorted ? n_mid - n_long : nroots;
+    a.per_root = per_root;
     total = checked_add(total, run_bitmap<8, 16>(ctx, a, per_root != nullptr));
   }
   a.len_lo = 0;

@@ -230,10 +230,12 @@ def test_hub_out_list_longer_than_staging(ctx, oracle_mod, a):
         assert np.array_equal(g.kclique_roots(k, roots), o.kclique_roots(k, roots))
 
 
-@pytest.mark.parametrize("flags", [0, 0x10, 0x2 | 0x10])
+@pytest.mark.parametrize("flags", [0, 0x10, 0x2 | 0x10, 0x20, 0x40])
 def test_paths_agree(G, oracle_mod, flags):
-    """Bitmap DFS (default), ET levels with the fused tail (NO_BITMAP), and ET levels
-    with every level materialised (NO_FUSE | NO_BITMAP) all equal the oracle."""
+    """Bitmap DFS (default), ET levels with the fused tail (NO_BITMAP), ET levels
+    with every level materialised (NO_FUSE | NO_BITMAP), the bitmap path without hub
+    splitting (NO_SPLIT) and with every root split into parts (DEBUG_SPLIT_ALL) all
+    equal the oracle."""
     c = G.Context(flags=flags)
     n, s, d, _ = gg.config_graph("c1", seed=4)
     g = c.load_edges(n, s, d)

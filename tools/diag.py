@@ -32,6 +32,29 @@ def main():
             o = oracle.Graph(n, s, d, lab)
             r = o.fpm(3, 3, pattern_cap=1 << 20)
             print("oracle", len(r), time.time() - t, flush=True)
+    elif what == "kcl_phases":
+        import torch
+        import paper_conf_icde_hu0o23_b200 as G
+        n, s, d, _ = gg.config_graph(sys.argv[2] if len(sys.argv) > 2 else "c2", seed=1)
+        c = G.Context(time_kernels=True)
+        sd = torch.from_numpy(s.view("int32")).cuda()
+        dd = torch.from_numpy(d.view("int32")).cuda()
+        for it in range(3):
+            torch.cuda.synchronize()
+            t = time.perf_counter()
+            g = c.load_edges(n, sd, dd)
+            torch.cuda.synchronize()
+            line = [f"build {1e3 * (time.perf_counter() - t):.2f}ms"]
+            for k in (4, 5, 6):
+                t = time.perf_counter()
+                cnt = g.kclique(k)
+                torch.cuda.synchronize()
+                st = c.stats()
+                kms = sum(v["ms"] for v in st["classes"].values())
+                line.append(f"k{k} wall {1e3 * (time.perf_counter() - t):.2f}ms lib {st['wall_ms']:.2f} "
+                            f"kernels {kms:.2f} launches {st['total_launches']}")
+            g.free()
+            print(" | ".join(line), flush=True)
     elif what == "sm":
         i = int(sys.argv[2])
         nv, e = PATS[i]
