@@ -393,6 +393,8 @@ def run_gamma(args):
         "clocks": clk,
         "kernels": {k: v for k, v in agg.items() if not k.startswith("_") and v["launches"]},
         "build_ms_per_step": info["build_ms"],
+        "step_ms": [round(x, 3) for x in times],
+        "e2e_step_ms": [round(x, 3) for x in e2e_times],
     }
     print(json.dumps(out))
     if world > 1:

@@ -231,6 +231,52 @@ __global__ void __launch_bounds__(kThreads) sm_kernel(SmArgs a) {
       }
       if (staged && lm_len == 0) continue;   // no child can extend
       const uint32_t *run = a.vid_in + beg;
+      if (last && staged && !(child_in_b && lm_len > 32)) {
+        // Last level over a staged L_m: count without a per-child warp loop.  The
+        // filters that involve the child c = phi_d are an order window (lo_c, hi_c)
+        // and possibly x != c; the prefix filters are already applied to L_m.
+        const bool lt_d = (a.P.ltmask[q] >> d) & 1u, gt_d = (a.P.gtmask[q] >> d) & 1u;
+        const bool inj_d = (a.P.injmask[q] >> d) & 1u;
+        uint64_t part = 0;
+        if (!child_in_b) {
+          // cand(c) = L_m ∩ window minus c: two binary searches per child, lane per child
+          for (uint32_t i = lane; i < len; i += 32) {
+            const uint32_t c = run[i];
+            const int64_t lo = lt_d ? max(bs.lo, (int64_t)c) : bs.lo;
+            const uint32_t hi = gt_d ? min(bs.hi, c) : bs.hi;
+            const uint32_t a0 = lo < 0 ? 0u : upper_bound_idx(slm, lm_len, (uint32_t)lo);
+            const uint32_t a1 = hi == 0 ? 0u : upper_bound_idx(slm, lm_len, hi - 1);
+            uint32_t cnt = a1 > a0 ? a1 - a0 : 0u;
+            if (inj_d && (int64_t)c > lo && c < hi && cnt && sorted_contains(slm, lm_len, c)) cnt--;
+            part += cnt;
+          }
+        } else {
+          // cand(c) = L_m ∩ N(c) ∩ window: flatten (child, L_m element) pairs over the
+          // lanes; each pair is one binary search of x in N(c)
+          const uint64_t T = (uint64_t)len * lm_len;
+          for (uint64_t t0 = 0; t0 < T; t0 += 32) {
+            const uint64_t t = t0 + lane;
+            bool ok = false;
+            if (t < T) {
+              const uint32_t i = (uint32_t)(t / lm_len), j = (uint32_t)(t - (uint64_t)i * lm_len);
+              const uint32_t c = run[i], x = slm[j];
+              const int64_t lo = lt_d ? max(bs.lo, (int64_t)c) : bs.lo;
+              const uint32_t hi = gt_d ? min(bs.hi, c) : bs.hi;
+              ok = (int64_t)x > lo && x < hi && !(inj_d && x == c);
+              if (ok) {
+                const uint64_t s0 = a.rp[c];
+                const uint32_t dl = (uint32_t)(a.rp[c + 1] - s0);
+                ok = dl > 0 && sorted_contains(a.col + s0, dl, x);
+              }
+            }
+            part += __popc(__ballot_sync(0xffffffffu, ok)) * (lane == 0);
+          }
+        }
+#pragma unroll
+        for (int off = 16; off > 0; off >>= 1) part += __shfl_down_sync(0xffffffffu, part, off);
+        acc += (lane == 0) ? part : 0;   // only lane 0's acc is published
+        continue;
+      }
       for (uint32_t i = 0; i < len && !stop; i++) {
         const uint32_t c = run[i];
         phi[d] = c;
