@@ -320,7 +320,8 @@ def run_gamma(args):
     torch.cuda.synchronize()
 
     clocks = ClockSampler(dev)
-    clocks.start()
+    if not args.no_clocks:
+        clocks.start()
     times, emb, results, info = [], 0, None, None
     for _ in range(args.steps):
         flush.fill_(1)
@@ -411,6 +412,7 @@ def main():
     ap.add_argument("--workload", default="c2", choices=sorted(WORKLOADS))
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-clocks", action="store_true", help="diagnostics only: skip nvidia-smi sampling")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)

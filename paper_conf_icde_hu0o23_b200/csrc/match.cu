@@ -193,6 +193,7 @@ __global__ void __launch_bounds__(kThreads) sm_kernel(SmArgs a) {
   const BlockPool pg{&a.ctrl[CTRL_GCUR], &a.ctrl[CTRL_OVF], a.cap_g, kBlkG};
   WarpBlock wv, wg;
   uint64_t acc = 0, in_entries = 0, out_entries = 0;
+  uint64_t elems = 0;   // adjacency elements the method fetches (SURVEY §8(d) B_l), lane-partial
   const uint64_t ng = a.g_end - a.g_begin;
   bool stop = false;
   const uint32_t prefix_mask = (1u << d) - 1u;
@@ -229,6 +230,14 @@ __global__ void __launch_bounds__(kThreads) sm_kernel(SmArgs a) {
           lm_len = r;
         }
       }
+      if (staged && lane == 0) {   // Opt 2: the prefix lists are fetched once per group
+        uint32_t m = bshared;
+        while (m) {
+          const int j = __ffs(m) - 1;
+          m &= m - 1;
+          elems += gdeg(a, phi[j]);
+        }
+      }
       if (staged && lm_len == 0) continue;   // no child can extend
       const uint32_t *run = a.vid_in + beg;
       if (last && staged && !(child_in_b && lm_len > 32)) {
@@ -254,6 +263,7 @@ __global__ void __launch_bounds__(kThreads) sm_kernel(SmArgs a) {
           // cand(c) = L_m ∩ N(c) ∩ window: flatten (child, L_m element) pairs over the
           // lanes; each pair is one binary search of x in N(c)
           const uint64_t T = (uint64_t)len * lm_len;
+          for (uint32_t i = lane; i < len; i += 32) elems += gdeg(a, run[i]);   // each N(c) once
           for (uint64_t t0 = 0; t0 < T; t0 += 32) {
             const uint64_t t = t0 + lane;
             bool ok = false;
@@ -280,6 +290,14 @@ __global__ void __launch_bounds__(kThreads) sm_kernel(SmArgs a) {
       for (uint32_t i = 0; i < len && !stop; i++) {
         const uint32_t c = run[i];
         phi[d] = c;
+        if (lane == 0) {   // the lists this child's extension fetches
+          uint32_t m = staged ? (child_in_b ? (1u << d) : 0u) : bq;
+          while (m) {
+            const int j = __ffs(m) - 1;
+            m &= m - 1;
+            elems += gdeg(a, phi[j]);
+          }
+        }
         const Bounds bc = bounds_for(a, q, prefix_mask | (1u << d), phi);
         uint32_t found;
         uint64_t pos = 0;
@@ -358,6 +376,11 @@ __global__ void __launch_bounds__(kThreads) sm_kernel(SmArgs a) {
   if (lane == 0) {
     if (acc) atomicAdd(&a.ctrl[CTRL_COUNT], (unsigned long long)acc);
     atomicAdd(&a.ctrl[CTRL_AUX0], (unsigned long long)in_entries);
+  }
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) elems += __shfl_down_sync(0xffffffffu, elems, off);
+  if (lane == 0) {
+    atomicAdd(&a.ctrl[CTRL_ELEMS], (unsigned long long)elems);
     atomicAdd(&a.ctrl[CTRL_ENTRIES], (unsigned long long)out_entries);
   }
 }
@@ -577,9 +600,14 @@ struct SmRun {
       gr = (int)std::max<uint64_t>(1, std::min<uint64_t>(gr, warps_ok / kWarps));
     }
     ctrl_reset(ctx);
-    ctx->launch(last ? KC_SM_COUNT : KC_SM_EXTEND,
-                [&] { sm_kernel<<<gr, kThreads, sm_smem(), ctx->stream>>>(a); });
+    const int kc = last ? KC_SM_COUNT : KC_SM_EXTEND;
+    ctx->launch(kc, [&] { sm_kernel<<<gr, kThreads, sm_smem(), ctx->stream>>>(a); });
     ctrl_fetch(ctx);
+    const uint64_t *h = ctx->ctrl_host;
+    if (!h[CTRL_OVF]) {   // 12 B per input entry, 4 B per list element, 8 B per output
+      ctx->stats.list_elems += h[CTRL_ELEMS];
+      ctx->stats.alg_bytes[kc] += 12 * h[CTRL_AUX0] + 4 * h[CTRL_ELEMS] + (last ? 0 : 8 * h[CTRL_ENTRIES]);
+    }
   }
 
   void process(uint32_t d, uint64_t g0, uint64_t g1) {

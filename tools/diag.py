@@ -55,6 +55,25 @@ def main():
                             f"kernels {kms:.2f} launches {st['total_launches']}")
             g.free()
             print(" | ".join(line), flush=True)
+    elif what == "sm_phases":
+        import torch
+        import paper_conf_icde_hu0o23_b200 as G
+        import bench
+        n, s, d, lab = gg.config_graph("c3", seed=1)
+        c = G.Context(time_kernels=True)
+        g = c.load_edges(n, torch.from_numpy(s.view("int32")).cuda(), torch.from_numpy(d.view("int32")).cuda(),
+                         torch.from_numpy(lab.view("int32")).cuda())
+        print("graph", g.info(), flush=True)
+        for it in range(2):
+            for (q, lname, nv, e, plab) in bench.sm_runs():
+                torch.cuda.synchronize()
+                t = time.perf_counter()
+                cnt = g.match(nv, e, plab)
+                torch.cuda.synchronize()
+                st = c.stats()
+                cl = {k: (v["launches"], round(v["ms"], 2)) for k, v in st["classes"].items() if v["launches"]}
+                print(f"{q}/{lname} {cnt[0]} {1e3 * (time.perf_counter() - t):.1f}ms levels "
+                      f"{st['level_entries'][:nv + 1]} {cl}", flush=True)
     elif what == "sm":
         i = int(sys.argv[2])
         nv, e = PATS[i]
