@@ -257,8 +257,15 @@ def run_gamma(args):
     import torch.distributed as dist
     rank, world, local = dist_env()
     if world > 1:
+        # one rank per GPU over NCCL; GAMMA_DIST_BACKEND=gloo lets several ranks share
+        # one GPU to exercise the multi-rank path on a single-GPU box
+        backend = os.environ.get("GAMMA_DIST_BACKEND", "nccl")
+        local = local % torch.cuda.device_count()
         torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
     dev = torch.cuda.current_device()
     import paper_conf_icde_hu0o23_b200 as G
 

@@ -419,6 +419,7 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
     ctx->launch(KC_FPM, [&] {
       GAMMA_CUDA(cub::DeviceRadixSort::SortKeys(t.p, tmp, k0.p, k1.p, (uint64_t)n, 0, endbit, ctx->stream));
     });
+    ctx->cub_sort_launched(KC_FPM, n, endbit);
     ctx->launch(KC_FPM, [&] { label_rank_kernel<<<g1d(n), 256, 0, ctx->stream>>>(k1.p, n, lrank.p); });
   }
   // ---- pattern table + per-(slot, position) domain bitmaps ----

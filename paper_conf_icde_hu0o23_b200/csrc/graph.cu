@@ -153,9 +153,7 @@ void sort_keys(gamma_ctx *ctx, const uint64_t *in, uint64_t *out, uint64_t nkeys
   ctx->launch(KC_BUILD, [&] {
     GAMMA_CUDA(cub::DeviceRadixSort::SortKeys(t.p, tmp, in, out, nkeys, 0, end_bit, ctx->stream));
   });
-  // onesweep: histogram + one pass per 8 key bits (+ the launch counted above)
-  ctx->stats.launches[KC_BUILD] += (end_bit + 7) / 8;
-  ctx->stats.total_launches += (end_bit + 7) / 8;
+  ctx->cub_sort_launched(KC_BUILD, nkeys, end_bit);
 }
 
 // keys -> (row_ptr, col) on g for M keys.
@@ -220,6 +218,7 @@ void build_dag(gamma_graph *g, uint64_t *keys, uint64_t M) {
   ctx->launch(KC_BUILD, [&] {
     GAMMA_CUDA(cub::DeviceSelect::If(t.p, tmp, keys, dkeys.p, nsel.p, (int64_t)M, op, ctx->stream));
   });
+  ctx->cub_select_launched(KC_BUILD);
   uint64_t mdag = 0;
   GAMMA_CUDA(cudaMemcpyAsync(&mdag, nsel.p, sizeof(uint64_t), cudaMemcpyDeviceToHost, ctx->stream));
   ctx->sync();
@@ -272,6 +271,7 @@ void build_from_edges(gamma_graph *g, const uint32_t *src, const uint32_t *dst, 
       ctx->launch(KC_BUILD, [&] {
         GAMMA_CUDA(cub::DeviceSelect::Unique(t.p, tmp, sorted.p, uniq.p, nsel.p, (int64_t)nkeys, ctx->stream));
       });
+      ctx->cub_select_launched(KC_BUILD);
     }
     uint64_t h[2] = {0, 0};
     GAMMA_CUDA(cudaMemcpyAsync(&h[0], nsel.p, sizeof(uint64_t), cudaMemcpyDeviceToHost, ctx->stream));

@@ -120,6 +120,18 @@ struct gamma_ctx {
     stats.launches[kc]++;
     stats.total_launches++;
   }
+  // Library calls (CUB) that launch several kernels inside one ctx->launch(): add the
+  // kernels beyond the first so total_launches matches the launch list.
+  void extra_launches(int kc, uint64_t n) {
+    stats.launches[kc] += n;
+    stats.total_launches += n;
+  }
+  // CUB onesweep radix sort: histogram + exclusive-sum + one pass per 8 key bits
+  // (a single-tile kernel for tiny inputs); DeviceSelect: init + sweep.
+  void cub_sort_launched(int kc, uint64_t items, int bits) {
+    extra_launches(kc, items <= 4096 ? 0 : 1 + (uint64_t)((bits + 7) / 8));
+  }
+  void cub_select_launched(int kc) { extra_launches(kc, 1); }
   cudaEvent_t next_event();
   void collect_timings();  // after a stream sync
   void sync() { GAMMA_CUDA(cudaStreamSynchronize(stream)); }

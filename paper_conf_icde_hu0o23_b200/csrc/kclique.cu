@@ -687,6 +687,7 @@ uint64_t kclique_count(gamma_graph *g, uint32_t k, const uint32_t *roots_dev, ui
       ctx->launch(KC_ROOTS, [&] {
         GAMMA_CUDA(cub::DeviceSelect::If(t.p, tmp, all.p, sel.p, nsel.p, (int64_t)n, op, ctx->stream));
       });
+      ctx->cub_select_launched(KC_ROOTS);
     }
     uint64_t nr = 0;
     GAMMA_CUDA(cudaMemcpyAsync(&nr, nsel.p, sizeof(uint64_t), cudaMemcpyDeviceToHost, ctx->stream));
@@ -707,6 +708,7 @@ uint64_t kclique_count(gamma_graph *g, uint32_t k, const uint32_t *roots_dev, ui
         GAMMA_CUDA(cub::DeviceRadixSort::SortPairsDescending(t.p, tmp, cost.p, cost2.p, sel.p, root_buf.p,
                                                              nr, 0, endbit, ctx->stream));
       });
+      ctx->cub_sort_launched(KC_ROOTS, nr, endbit);
     }
     if (ctx->desc.world > 1 && nr) {
       DevBuf<uint8_t> flag(ctx, nr);
@@ -723,6 +725,7 @@ uint64_t kclique_count(gamma_graph *g, uint32_t k, const uint32_t *roots_dev, ui
           GAMMA_CUDA(cub::DeviceSelect::Flagged(t.p, tmp, root_buf.p, flag.p, mine.p, nsel.p, (int64_t)nr,
                                                 ctx->stream));
         });
+        ctx->cub_select_launched(KC_ROOTS);
       }
       GAMMA_CUDA(cudaMemcpyAsync(&nr, nsel.p, sizeof(uint64_t), cudaMemcpyDeviceToHost, ctx->stream));
       ctx->sync();

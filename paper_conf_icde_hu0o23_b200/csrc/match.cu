@@ -677,6 +677,7 @@ static uint64_t match_count(gamma_graph *g, const SmPlan &P) {
     ctx->launch(KC_ROOTS, [&] {
       GAMMA_CUDA(cub::DeviceSelect::If(t.p, tmp, all.p, sel.p, nsel.p, (int64_t)n, op, ctx->stream));
     });
+    ctx->cub_select_launched(KC_ROOTS);
   }
   uint64_t nr = 0;
   GAMMA_CUDA(cudaMemcpyAsync(&nr, nsel.p, sizeof(uint64_t), cudaMemcpyDeviceToHost, ctx->stream));
@@ -707,6 +708,7 @@ static uint64_t match_count(gamma_graph *g, const SmPlan &P) {
       GAMMA_CUDA(cub::DeviceRadixSort::SortPairsDescending(t.p, tmp, cost.p, cost2.p, sel.p, roots.p, nr, 0,
                                                            endbit, ctx->stream));
     });
+    ctx->cub_sort_launched(KC_ROOTS, nr, endbit);
   }
   if (ctx->desc.world > 1 && nr) {
     DevBuf<uint8_t> flag(ctx, nr);
@@ -721,6 +723,7 @@ static uint64_t match_count(gamma_graph *g, const SmPlan &P) {
       ctx->launch(KC_ROOTS, [&] {
         GAMMA_CUDA(cub::DeviceSelect::Flagged(t.p, tmp, roots.p, flag.p, mine.p, nsel.p, (int64_t)nr, ctx->stream));
       });
+      ctx->cub_select_launched(KC_ROOTS);
     }
     GAMMA_CUDA(cudaMemcpyAsync(&nr, nsel.p, sizeof(uint64_t), cudaMemcpyDeviceToHost, ctx->stream));
     ctx->sync();

@@ -36,6 +36,8 @@ UNIT_SCALE = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "KB": 1e3, "M
 
 
 def kclass(name: str) -> str:
+    if "kcl_bitmap_parts_kernel" in name:
+        return "bitmap_parts"
     if "kcl_bitmap_kernel" in name:
         return "bitmap"
     m = re.search(r"kcl_kernel<(\d)", name)
