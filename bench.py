@@ -167,6 +167,14 @@ def make_input(name, seed=1):
 # ------------------------------------------------------------------------------------
 # CPU baseline: the oracle, as it stands, on a bounded seeded sample of the workload.
 # ------------------------------------------------------------------------------------
+def _aut(nv, edges, plab):
+    """|Aut_L(P)| by brute force over the nv! vertex permutations (plain Python)."""
+    import itertools
+    E = {frozenset(e) for e in edges}
+    return sum(1 for p in itertools.permutations(range(nv))
+               if all(plab[p[i]] == plab[i] for i in range(nv)) and {frozenset((p[a], p[b])) for a, b in edges} == E)
+
+
 def cpu_oracle_sample(n, s, d, lab, w, budget_s=12.0, seed=7):
     import oracle
     t0 = time.perf_counter()
@@ -183,7 +191,7 @@ def cpu_oracle_sample(n, s, d, lab, w, budget_s=12.0, seed=7):
             ns, ss, ds, ls = gg.config_graph(w["cfg"], seed=seed, scale=scale)
             gs = oracle.Graph(ns, ss, ds, ls)
             t1 = time.perf_counter()
-            res = gs.fpm(w["l"], max(1, int(w["minsup"] * 2.0 ** (scale - 22))), pattern_cap=1 << 21)
+            res = gs.fpm(w["l"], max(1, int(w["minsup"] * 2.0 ** (scale - 22))), threads=cores, pattern_cap=1 << 21)
             dt = time.perf_counter() - t1
             emb_l = sum(r[5] for r in res if r[0] == w["l"])
             if t_count + dt > budget_s * 3 and t_count > 0:
@@ -199,23 +207,26 @@ def cpu_oracle_sample(n, s, d, lab, w, budget_s=12.0, seed=7):
                 "embeddings": emb, "seconds": t_count}
     perm = rng.permutation(n).astype(np.uint32)
     frac, emb, t_count, used = 0.0005, 0.0, 0.0, 0
+    threads = cores   # all host cores (torchrun sets OMP_NUM_THREADS=1 per rank)
     while True:
         cnt = min(max(1, int(n * frac)), n - used)
         roots = perm[used:used + cnt]
         t1 = time.perf_counter()
         if w["kind"] == "kcl":
             for k in w["ks"]:
-                emb += int(g.kclique_roots(k, roots).sum())
+                emb += int(g.kclique_roots(k, roots, threads=threads).sum())
         else:
             for (q, lname, nv, e, plab) in sm_runs():
-                mp = int(g.match_roots(nv, e, roots, plab).sum())
-                import paper_conf_icde_hu0o23_b200 as G   # |Aut_L| from the host planner (no GPU)
-                emb += mp / G.pattern_plan(nv, e, plab)["aut"]
-        t_count += time.perf_counter() - t1
+                mp = int(g.match_roots(nv, e, roots, plab, threads=threads).sum())
+                emb += mp / _aut(nv, e, plab)
+        dt = time.perf_counter() - t1
+        t_count += dt
         used += cnt
         if t_count >= budget_s or used >= n:
             break
-        frac *= 2
+        # next chunk: double, but stay within the budget at the rate just seen
+        rate = cnt / max(dt, 1e-6)
+        frac = min(2 * cnt, max(1, int(rate * (budget_s - t_count)))) / n
     what = (f"k-clique counts k={list(w['ks'])}" if w["kind"] == "kcl" else
             "SM mappings / |Aut_L| over the 8 (query, labeling) runs")
     return {"value": emb / t_count if t_count > 0 else None, "unit": UNIT, "cores": cores, "kind": "oracle",

@@ -239,6 +239,7 @@ void gamma_graph_free(gamma_graph *g) {
     c->free(g->dag_ptr);
     c->free(g->dag_col);
     c->free(g->labels);
+    c->free(g->root_order);
     cudaStreamSynchronize(c->stream);
   }
   cudaGetLastError();

@@ -165,6 +165,11 @@ struct gamma_graph {
   uint32_t max_degree = 0, max_out_degree = 0;
   uint64_t device_bytes = 0;
   double build_ms = 0;
+  // kCL root order cache (kclique.cu ensure_root_order): this rank's vertices sorted by
+  // d+ descending, and root_ge[t] = how many of them have d+ >= t
+  uint32_t *root_order = nullptr;
+  std::vector<uint64_t> root_ge;
+  int32_t root_rank = -1, root_world = -1;
 };
 
 // RAII device buffer through the ctx allocator.
@@ -221,5 +226,6 @@ uint64_t kclique_count(gamma_graph *g, uint32_t k, const uint32_t *roots_dev, ui
 constexpr uint32_t kBitmapMaxRun = 512;
 constexpr uint32_t kBitmapMaxK = 12;
 uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint64_t nroots,
-                        unsigned long long *per_root, bool sorted);
+                        unsigned long long *per_root, bool sorted, uint64_t n_long, uint64_t n_mid);
+void ensure_root_order(gamma_graph *g);
 }  // namespace gamma_impl

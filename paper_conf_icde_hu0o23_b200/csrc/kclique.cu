@@ -647,6 +647,87 @@ void configure_kernels() {
 
 }  // namespace
 
+namespace {
+__global__ void outdeg_key_kernel(const uint64_t *dag_ptr, uint32_t n, uint32_t *key, uint32_t *val) {
+  for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x) {
+    key[v] = (uint32_t)(dag_ptr[v + 1] - dag_ptr[v]);
+    val[v] = (uint32_t)v;
+  }
+}
+
+__global__ void outdeg_hist_kernel(const uint64_t *dag_ptr, const uint32_t *roots, uint64_t nr, uint32_t *hist) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < nr; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t v = roots[i];
+    atomicAdd(&hist[dag_ptr[v + 1] - dag_ptr[v]], 1u);
+  }
+}
+}  // namespace
+
+// A2: all vertices sorted by d+ descending (stable: ties by id), this rank's share of
+// them (snake over the sorted order), and ge[t] = #roots with
+// d+ >= t.  Cached on the graph for the (rank, world) of its context.
+void ensure_root_order(gamma_graph *g) {
+  gamma_ctx *ctx = g->ctx;
+  if (g->root_order && g->root_rank == ctx->desc.rank && g->root_world == ctx->desc.world) return;
+  if (g->root_order) {
+    ctx->free(g->root_order);
+    g->root_order = nullptr;
+  }
+  const uint32_t n = g->n;
+  DevBuf<uint32_t> key(ctx, n), key2(ctx, n), val(ctx, n), order(ctx, n);
+  ctx->launch(KC_ROOTS, [&] { outdeg_key_kernel<<<grid1d(n), 256, 0, ctx->stream>>>(g->dag_ptr, n, key.p, val.p); });
+  int endbit = 1;
+  while (endbit < 32 && (1ull << endbit) <= g->max_out_degree) endbit++;
+  size_t tmp = 0;
+  GAMMA_CUDA(cub::DeviceRadixSort::SortPairsDescending(nullptr, tmp, key.p, key2.p, val.p, order.p, (uint64_t)n, 0,
+                                                       endbit, ctx->stream));
+  {
+    DevBuf<uint8_t> t(ctx, tmp);
+    ctx->launch(KC_ROOTS, [&] {
+      GAMMA_CUDA(cub::DeviceRadixSort::SortPairsDescending(t.p, tmp, key.p, key2.p, val.p, order.p, (uint64_t)n, 0,
+                                                           endbit, ctx->stream));
+    });
+    ctx->cub_sort_launched(KC_ROOTS, n, endbit);
+  }
+  uint64_t nr = n;
+  if (ctx->desc.world > 1) {
+    DevBuf<uint8_t> flag(ctx, n);
+    DevBuf<uint64_t> nsel(ctx, 1);
+    ctx->launch(KC_ROOTS, [&] {
+      rank_flag_kernel<<<grid1d(n), 256, 0, ctx->stream>>>(n, ctx->desc.rank, ctx->desc.world, flag.p);
+    });
+    DevBuf<uint32_t> mine(ctx, n);
+    tmp = 0;
+    GAMMA_CUDA(cub::DeviceSelect::Flagged(nullptr, tmp, order.p, flag.p, mine.p, nsel.p, (int64_t)n, ctx->stream));
+    {
+      DevBuf<uint8_t> t(ctx, tmp);
+      ctx->launch(KC_ROOTS, [&] {
+        GAMMA_CUDA(cub::DeviceSelect::Flagged(t.p, tmp, order.p, flag.p, mine.p, nsel.p, (int64_t)n, ctx->stream));
+      });
+      ctx->cub_select_launched(KC_ROOTS);
+    }
+    GAMMA_CUDA(cudaMemcpyAsync(&nr, nsel.p, sizeof(uint64_t), cudaMemcpyDeviceToHost, ctx->stream));
+    ctx->sync();
+    order = std::move(mine);
+  }
+  const uint32_t nb = g->max_out_degree + 2;
+  DevBuf<uint32_t> hist(ctx, nb);
+  GAMMA_CUDA(cudaMemsetAsync(hist.p, 0, nb * 4, ctx->stream));
+  if (nr)
+    ctx->launch(KC_ROOTS, [&] {
+      outdeg_hist_kernel<<<grid1d(nr), 256, 0, ctx->stream>>>(g->dag_ptr, order.p, nr, hist.p);
+    });
+  std::vector<uint32_t> h(nb);
+  GAMMA_CUDA(cudaMemcpyAsync(h.data(), hist.p, nb * 4, cudaMemcpyDeviceToHost, ctx->stream));
+  ctx->sync();
+  g->root_ge.assign(nb + 1, 0);
+  for (int64_t t = (int64_t)nb - 1; t >= 0; t--) g->root_ge[t] = g->root_ge[t + 1] + h[t];
+  g->root_order = order.release();
+  g->root_rank = ctx->desc.rank;
+  g->root_world = ctx->desc.world;
+  g->device_bytes += (uint64_t)n * 4;
+}
+
 uint64_t kclique_count(gamma_graph *g, uint32_t k, const uint32_t *roots_dev, uint64_t nroots,
                        uint64_t *per_root_dev) {
   gamma_ctx *ctx = g->ctx;
@@ -661,78 +742,17 @@ uint64_t kclique_count(gamma_graph *g, uint32_t k, const uint32_t *roots_dev, ui
   R.fuse = (ctx->desc.flags & GAMMA_FLAG_NO_FUSE) == 0;
   R.per_root_out = (unsigned long long *)per_root_dev;
   R.levels.resize(k + 1);
-  {
-    size_t fr = 0, tot = 0;
-    GAMMA_CUDA(cudaMemGetInfo(&fr, &tot));
-    const uint64_t budget = ctx->desc.hbm_budget_bytes ? ctx->desc.hbm_budget_bytes : (uint64_t)(fr * 0.8);
-    const uint64_t stored = k >= 4 ? k - 3 : 1;   // level tables at depths 2 .. k-2
-    R.level_share = budget / stored;
-  }
   // ---- A2: root list ----
   DevBuf<uint32_t> root_buf;
   if (per_root) {
     R.roots = roots_dev;
     R.nroots = nroots;
   } else {
-    const uint32_t n = g->n;
-    DevBuf<uint32_t> all(ctx, n);
-    ctx->launch(KC_ROOTS, [&] { iota_kernel<<<grid1d(n), 256, 0, ctx->stream>>>(all.p, n); });
-    DevBuf<uint32_t> sel(ctx, n);
-    DevBuf<uint64_t> nsel(ctx, 1);
-    RootNeed op{g->dag_ptr, k - 1};
-    size_t tmp = 0;
-    GAMMA_CUDA(cub::DeviceSelect::If(nullptr, tmp, all.p, sel.p, nsel.p, (int64_t)n, op, ctx->stream));
-    {
-      DevBuf<uint8_t> t(ctx, tmp);
-      ctx->launch(KC_ROOTS, [&] {
-        GAMMA_CUDA(cub::DeviceSelect::If(t.p, tmp, all.p, sel.p, nsel.p, (int64_t)n, op, ctx->stream));
-      });
-      ctx->cub_select_launched(KC_ROOTS);
-    }
-    uint64_t nr = 0;
-    GAMMA_CUDA(cudaMemcpyAsync(&nr, nsel.p, sizeof(uint64_t), cudaMemcpyDeviceToHost, ctx->stream));
-    ctx->sync();
-    DevBuf<uint64_t> cost(ctx, nr ? nr : 1), cost2(ctx, nr ? nr : 1);
-    root_buf = DevBuf<uint32_t>(ctx, nr ? nr : 1);
-    if (nr) {   // heavy first: sort by cost descending
-      ctx->launch(KC_ROOTS, [&] {
-        root_cost_kernel<<<grid1d(nr), 256, 0, ctx->stream>>>(g->dag_ptr, sel.p, nr, cost.p);
-      });
-      int endbit = 1;
-      while (endbit < 64 && (1ull << endbit) <= (uint64_t)g->max_out_degree * g->max_out_degree) endbit++;
-      tmp = 0;
-      GAMMA_CUDA(cub::DeviceRadixSort::SortPairsDescending(nullptr, tmp, cost.p, cost2.p, sel.p, root_buf.p,
-                                                           nr, 0, endbit, ctx->stream));
-      DevBuf<uint8_t> t(ctx, tmp);
-      ctx->launch(KC_ROOTS, [&] {
-        GAMMA_CUDA(cub::DeviceRadixSort::SortPairsDescending(t.p, tmp, cost.p, cost2.p, sel.p, root_buf.p,
-                                                             nr, 0, endbit, ctx->stream));
-      });
-      ctx->cub_sort_launched(KC_ROOTS, nr, endbit);
-    }
-    if (ctx->desc.world > 1 && nr) {
-      DevBuf<uint8_t> flag(ctx, nr);
-      ctx->launch(KC_ROOTS, [&] {
-        rank_flag_kernel<<<grid1d(nr), 256, 0, ctx->stream>>>(nr, ctx->desc.rank, ctx->desc.world, flag.p);
-      });
-      DevBuf<uint32_t> mine(ctx, nr);
-      tmp = 0;
-      GAMMA_CUDA(cub::DeviceSelect::Flagged(nullptr, tmp, root_buf.p, flag.p, mine.p, nsel.p, (int64_t)nr,
-                                            ctx->stream));
-      {
-        DevBuf<uint8_t> t(ctx, tmp);
-        ctx->launch(KC_ROOTS, [&] {
-          GAMMA_CUDA(cub::DeviceSelect::Flagged(t.p, tmp, root_buf.p, flag.p, mine.p, nsel.p, (int64_t)nr,
-                                                ctx->stream));
-        });
-        ctx->cub_select_launched(KC_ROOTS);
-      }
-      GAMMA_CUDA(cudaMemcpyAsync(&nr, nsel.p, sizeof(uint64_t), cudaMemcpyDeviceToHost, ctx->stream));
-      ctx->sync();
-      root_buf = std::move(mine);
-    }
-    R.roots = root_buf.p;
-    R.nroots = nr;
+    // heavy-first root order of this rank, computed once per graph (k only decides
+    // the prefix: d+(v) >= k-1), so a call needs no select / sort / size round trip
+    ensure_root_order(g);
+    R.roots = g->root_order;
+    R.nroots = (k - 1 < g->root_ge.size()) ? g->root_ge[k - 1] : 0;
   }
   ctx->stats.level_entries[1] = R.nroots;
   if (k <= 2) {   // per-root or partitioned k = 1 / 2: each root contributes 1 / d+(v)
@@ -759,10 +779,22 @@ uint64_t kclique_count(gamma_graph *g, uint32_t k, const uint32_t *roots_dev, ui
                                                        kThreads, kcl_smem(MODE_FUSED));
   const bool bitmap = (ctx->desc.flags & GAMMA_FLAG_NO_BITMAP) == 0 && k >= 3 && k <= kBitmapMaxK;
   if (bitmap && R.nroots) {
-    R.add_count(kclique_bitmap(g, k, R.roots, R.nroots, R.per_root_out, !per_root));
+    uint64_t n_long = 0, n_mid = 0;
+    if (!per_root) {
+      n_long = kBitmapMaxRun + 1 < g->root_ge.size() ? g->root_ge[kBitmapMaxRun + 1] : 0;
+      n_mid = 129 < g->root_ge.size() ? g->root_ge[129] : 0;
+    }
+    R.add_count(kclique_bitmap(g, k, R.roots, R.nroots, R.per_root_out, !per_root, n_long, n_mid));
     R.root_len_gt = kBitmapMaxRun;
   }
-  if (R.nroots && (!bitmap || g->max_out_degree > kBitmapMaxRun)) R.process(1, 0, R.nroots);
+  if (R.nroots && (!bitmap || g->max_out_degree > kBitmapMaxRun)) {
+    size_t fr = 0, tot = 0;
+    GAMMA_CUDA(cudaMemGetInfo(&fr, &tot));
+    const uint64_t budget = ctx->desc.hbm_budget_bytes ? ctx->desc.hbm_budget_bytes : (uint64_t)(fr * 0.8);
+    const uint64_t stored = k >= 4 ? k - 3 : 1;   // level tables at depths 2 .. k-2
+    R.level_share = budget / stored;
+    R.process(1, 0, R.nroots);
+  }
   ctx->sync();
   ctx->collect_timings();
   return R.total;

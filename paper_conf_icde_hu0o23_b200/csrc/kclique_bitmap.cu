@@ -42,8 +42,9 @@ struct BmArgs {
   unsigned long long *per_root;
   // hub splitting (k >= 6): roots with more than heavy_cut 4-cliques are deferred
   uint64_t heavy_cut;         // 0: never defer
-  uint2 *parts;               // (root index, part | nparts << 16)
+  uint2 *parts;               // (absolute root index, part | nparts << 16)
   uint32_t parts_cap;
+  uint64_t root_base;         // index of roots[0] in the full root list (parts are absolute)
 };
 
 __device__ __forceinline__ uint32_t excl_scan32(uint32_t x, int lane, uint32_t &total) {
@@ -369,7 +370,8 @@ __global__ void __launch_bounds__(256) kcl_bitmap_kernel(BmArgs a) {
           if (tid == 0) {
             const unsigned long long at = atomicAdd(&a.ctrl[CTRL_AUX1], (unsigned long long)nparts);
             if (at + nparts <= a.parts_cap) {
-              for (uint32_t p = 0; p < nparts; p++) a.parts[at + p] = make_uint2((uint32_t)gi, p | (nparts << 16));
+              for (uint32_t p = 0; p < nparts; p++)
+                a.parts[at + p] = make_uint2((uint32_t)(a.root_base + gi), p | (nparts << 16));
               m.slot[0] = 1;
             } else {
               m.slot[0] = 0;   // list full: expand here
@@ -411,7 +413,7 @@ __global__ void __launch_bounds__(256) kcl_bitmap_kernel(BmArgs a) {
 // Second launch for the deferred heavy roots: one CTA per (root, part); the part
 // rebuilds the root's rows (cheap next to the DFS) and takes every nparts-th item.
 template <bool PER_ROOT>
-__global__ void __launch_bounds__(256) kcl_bitmap_parts_kernel(BmArgs a, uint64_t nparts_total) {
+__global__ void __launch_bounds__(256) kcl_bitmap_parts_kernel(BmArgs a) {
   extern __shared__ uint32_t smem[];
   constexpr int TW = 16;
   const int lane = threadIdx.x & 31;
@@ -420,6 +422,9 @@ __global__ void __launch_bounds__(256) kcl_bitmap_parts_kernel(BmArgs a, uint64_
   uint64_t total = 0;
   for (;;) {
     if (tid == 0) {
+      // the part list was filled by the previous launch; its length sits in ctrl
+      const unsigned long long np = *(volatile unsigned long long *)&a.ctrl[CTRL_AUX1];
+      const unsigned long long nparts_total = np < a.parts_cap ? np : a.parts_cap;
       const unsigned long long w = atomicAdd(&a.ctrl[CTRL_WORK], 1ull);
       m.slot[0] = w < nparts_total ? (uint32_t)w : 0xffffffffu;
     }
@@ -460,8 +465,10 @@ constexpr size_t bm_smem() {
   return (size_t)(256 / (TEAM_WARPS * 32)) * team_words<TW>() * sizeof(uint32_t);
 }
 
+// Enqueue one team kind over a root range (no host round trip: the work counter is
+// reset on the stream, the counts accumulate in ctrl and are read once at the end).
 template <int TEAM_WARPS, int TW>
-uint64_t run_bitmap(gamma_ctx *ctx, const BmArgs &a0, bool per_root) {
+void enqueue_bitmap(gamma_ctx *ctx, const BmArgs &a0, bool per_root) {
   static bool attr = false;
   if (!attr) {
     GAMMA_CUDA(cudaFuncSetAttribute(kcl_bitmap_kernel<TEAM_WARPS, TW, false>,
@@ -471,64 +478,37 @@ uint64_t run_bitmap(gamma_ctx *ctx, const BmArgs &a0, bool per_root) {
     attr = true;
   }
   const size_t smem = bm_smem<TEAM_WARPS, TW>();
-  const int grid = ctx->num_sms * occupancy_blocks((const void *)kcl_bitmap_kernel<TEAM_WARPS, TW, false>, 256, smem);
-  ctrl_reset(ctx);
+  static int grid = 0;
+  if (!grid)
+    grid = ctx->num_sms * occupancy_blocks((const void *)kcl_bitmap_kernel<TEAM_WARPS, TW, false>, 256, smem);
+  GAMMA_CUDA(cudaMemsetAsync(ctx->ctrl + CTRL_WORK, 0, sizeof(uint64_t), ctx->stream));
   ctx->launch(KC_BITMAP, [&] {
     if (per_root)
       kcl_bitmap_kernel<TEAM_WARPS, TW, true><<<grid, 256, smem, ctx->stream>>>(a0);
     else
       kcl_bitmap_kernel<TEAM_WARPS, TW, false><<<grid, 256, smem, ctx->stream>>>(a0);
   });
-  ctrl_fetch(ctx);
-  const uint64_t *h = ctx->ctrl_host;
-  ctx->stats.list_elems += h[CTRL_ELEMS];
-  ctx->stats.level_entries[2] += h[CTRL_AUX0];
-  ctx->stats.alg_bytes[KC_BITMAP] += 4 * h[CTRL_AUX0] + 4 * h[CTRL_ELEMS];
-  uint64_t count = h[CTRL_COUNT];
-  const uint64_t nparts = std::min<uint64_t>(h[CTRL_AUX1], a0.parts_cap);
-  if (nparts) {   // the deferred heavy roots, one CTA per part
-    static bool pattr = false;
-    if (!pattr) {
-      GAMMA_CUDA(cudaFuncSetAttribute(kcl_bitmap_parts_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                      (int)bm_smem<8, 16>()));
-      GAMMA_CUDA(cudaFuncSetAttribute(kcl_bitmap_parts_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                      (int)bm_smem<8, 16>()));
-      pattr = true;
-    }
-    const int pgrid = ctx->num_sms * occupancy_blocks((const void *)kcl_bitmap_parts_kernel<false>, 256,
-                                                      bm_smem<8, 16>());
-    ctrl_reset(ctx);
-    ctx->launch(KC_BITMAP, [&] {
-      if (per_root)
-        kcl_bitmap_parts_kernel<true><<<pgrid, 256, bm_smem<8, 16>(), ctx->stream>>>(a0, nparts);
-      else
-        kcl_bitmap_parts_kernel<false><<<pgrid, 256, bm_smem<8, 16>(), ctx->stream>>>(a0, nparts);
-    });
-    ctrl_fetch(ctx);
-    count = checked_add(count, ctx->ctrl_host[CTRL_COUNT]);
-    ctx->stats.chunks += nparts;
-  }
-  return count;
 }
 
-// out[0] = #roots with |N+(v)| > 512, out[1] = #roots with |N+(v)| > 128
-__global__ void count_len_classes(const uint64_t *dag_ptr, const uint32_t *roots, uint64_t nr,
-                                  unsigned long long *out) {
-  unsigned long long c0 = 0, c1 = 0;
-  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < nr; i += (uint64_t)gridDim.x * blockDim.x) {
-    const uint32_t v = roots[i];
-    const uint64_t L = dag_ptr[v + 1] - dag_ptr[v];
-    c0 += L > kBitmapMaxRun;
-    c1 += L > 128;
+void enqueue_parts(gamma_ctx *ctx, const BmArgs &a0, bool per_root) {
+  static bool attr = false;
+  if (!attr) {
+    GAMMA_CUDA(cudaFuncSetAttribute(kcl_bitmap_parts_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                    (int)bm_smem<8, 16>()));
+    GAMMA_CUDA(cudaFuncSetAttribute(kcl_bitmap_parts_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                    (int)bm_smem<8, 16>()));
+    attr = true;
   }
-  for (int o = 16; o > 0; o >>= 1) {
-    c0 += __shfl_down_sync(0xffffffffu, c0, o);
-    c1 += __shfl_down_sync(0xffffffffu, c1, o);
-  }
-  if ((threadIdx.x & 31) == 0) {
-    if (c0) atomicAdd(&out[0], c0);
-    if (c1) atomicAdd(&out[1], c1);
-  }
+  static int pgrid = 0;
+  if (!pgrid)
+    pgrid = ctx->num_sms * occupancy_blocks((const void *)kcl_bitmap_parts_kernel<false>, 256, bm_smem<8, 16>());
+  GAMMA_CUDA(cudaMemsetAsync(ctx->ctrl + CTRL_WORK, 0, sizeof(uint64_t), ctx->stream));
+  ctx->launch(KC_BITMAP, [&] {
+    if (per_root)
+      kcl_bitmap_parts_kernel<true><<<pgrid, 256, bm_smem<8, 16>(), ctx->stream>>>(a0);
+    else
+      kcl_bitmap_parts_kernel<false><<<pgrid, 256, bm_smem<8, 16>(), ctx->stream>>>(a0);
+  });
 }
 
 }  // namespace
@@ -536,7 +516,7 @@ __global__ void count_len_classes(const uint64_t *dag_ptr, const uint32_t *roots
 // Count k-cliques rooted at roots[0..nroots) whose run length is <= 512 (k <= 12);
 // longer runs are left to the ET path.  per_root (nullable) indexed like roots.
 uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint64_t nroots,
-                        unsigned long long *per_root, bool sorted) {
+                        unsigned long long *per_root, bool sorted, uint64_t n_long, uint64_t n_mid) {
   gamma_ctx *ctx = g->ctx;
   BmArgs a{};
   a.dag_ptr = g->dag_ptr;
@@ -547,47 +527,52 @@ uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint6
   a.ctrl = (unsigned long long *)ctx->ctrl;
   a.per_root = per_root;
   // hub splitting only pays when the DFS below a triangle is deep (k >= 6)
+  const bool split = k >= 6 && (ctx->desc.flags & GAMMA_FLAG_NO_SPLIT) == 0;
   DevBuf<uint2> parts;
-  if (k >= 6 && (ctx->desc.flags & GAMMA_FLAG_NO_SPLIT) == 0) {
+  if (split) {
     a.parts_cap = 1u << 20;
     parts = DevBuf<uint2>(ctx, a.parts_cap);
     a.parts = parts.p;
     a.heavy_cut = (ctx->desc.flags & GAMMA_FLAG_DEBUG_SPLIT_ALL) ? 1 : 4ull * kPartCost;
   }
-  uint64_t total = 0;
-  // Roots sorted by cost (d+^2, descending) fall into three contiguous classes:
-  // [0, n_long) ET path, [n_long, n_mid) CTA teams, [n_mid, nroots) warp teams.
-  // Launch each team kind on its own range so no team walks over roots it skips.
-  // (Per-root mode passes unsorted roots: every launch then filters the whole list.)
-  uint64_t n_long = 0, n_mid = 0;
+  // Roots sorted by d+ descending fall into three contiguous classes: [0, n_long) ET
+  // path, [n_long, n_mid) CTA teams, [n_mid, nroots) warp teams; each team kind runs
+  // on its own range.  Unsorted (per-root mode) roots: every launch filters the list.
   if (sorted) {
-    GAMMA_CUDA(cudaMemsetAsync(ctx->ctrl + CTRL_AUX0, 0, 16, ctx->stream));
-    ctx->launch(KC_ROOTS, [&] {
-      count_len_classes<<<148 * 4, 256, 0, ctx->stream>>>(g->dag_ptr, roots, nroots,
-                                                          (unsigned long long *)(ctx->ctrl + CTRL_AUX0));
-    });
-    uint64_t h[2];
-    GAMMA_CUDA(cudaMemcpyAsync(h, ctx->ctrl + CTRL_AUX0, 16, cudaMemcpyDeviceToHost, ctx->stream));
-    ctx->sync();
-    n_long = h[0];
-    n_mid = h[1];
+    n_long = std::min(n_long, nroots);
+    n_mid = std::min(n_mid, nroots);
   }
+  ctrl_reset(ctx);
   a.len_lo = 128;
   a.len_hi = 512;
   if (g->max_out_degree > 128 && (!sorted || n_mid > n_long)) {
     a.roots = roots + (sorted ? n_long : 0);
+    a.root_base = sorted ? n_long : 0;
     a.nroots = sorted ? n_mid - n_long : nroots;
-    a.per_root = per_root;
-    total = checked_add(total, run_bitmap<8, 16>(ctx, a, per_root != nullptr));
+    enqueue_bitmap<8, 16>(ctx, a, per_root != nullptr);
   }
   a.len_lo = 0;
   a.len_hi = 128;
   if (!sorted || nroots > n_mid) {
     a.roots = roots + (sorted ? n_mid : 0);
+    a.root_base = sorted ? n_mid : 0;
     a.nroots = sorted ? nroots - n_mid : nroots;
-    total = checked_add(total, run_bitmap<1, 4>(ctx, a, per_root != nullptr));
+    enqueue_bitmap<1, 4>(ctx, a, per_root != nullptr);
   }
-  return total;
+  if (split) {
+    // parts carry absolute indices into the full root list
+    a.roots = roots;
+    a.root_base = 0;
+    a.nroots = nroots;
+    enqueue_parts(ctx, a, per_root != nullptr);
+  }
+  ctrl_fetch(ctx);
+  const uint64_t *h = ctx->ctrl_host;
+  ctx->stats.list_elems += h[CTRL_ELEMS];
+  ctx->stats.level_entries[2] += h[CTRL_AUX0];
+  ctx->stats.alg_bytes[KC_BITMAP] += 4 * h[CTRL_AUX0] + 4 * h[CTRL_ELEMS];
+  if (split) ctx->stats.chunks += std::min<uint64_t>(h[CTRL_AUX1], a.parts_cap);
+  return h[CTRL_COUNT];
 }
 
 }  // namespace gamma_impl
