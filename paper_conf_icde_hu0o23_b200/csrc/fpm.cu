@@ -43,8 +43,6 @@ __constant__ uint8_t c_perm4[24][4] = {
     {1, 0, 2, 3}, {1, 0, 3, 2}, {1, 2, 0, 3}, {1, 2, 3, 0}, {1, 3, 0, 2}, {1, 3, 2, 0},
     {2, 0, 1, 3}, {2, 0, 3, 1}, {2, 1, 0, 3}, {2, 1, 3, 0}, {2, 3, 0, 1}, {2, 3, 1, 0},
     {3, 0, 1, 2}, {3, 0, 2, 1}, {3, 1, 0, 2}, {3, 1, 2, 0}, {3, 2, 0, 1}, {3, 2, 1, 0}};
-// index of position pair (a<b) in lexicographic pair order: (0,1)(0,2)(0,3)(1,2)(1,3)(2,3)
-__constant__ uint8_t c_pair[4][4] = {{0, 0, 1, 2}, {0, 0, 3, 4}, {1, 3, 0, 5}, {2, 4, 5, 0}};
 
 // Pattern code packed in one word (0 = empty slot):
 //   bits 0..47 four 12-bit labels (canonical order), 48..50 nv, 51..52 ne,
@@ -158,7 +156,13 @@ __device__ Canon canonical(const FpmArgs &a, const uint32_t *W, uint32_t nv, con
     uint32_t inv[4];
     for (uint32_t p = 0; p < 4; p++) inv[c_perm4[r][p]] = p;
     uint32_t idx[3] = {7, 7, 7};
-    for (uint32_t e = 0; e < ne; e++) idx[e] = c_pair[inv[E[e][0]]][inv[E[e][1]]];
+    for (uint32_t e = 0; e < ne; e++) {
+      // index of the position pair (p<q) in lexicographic order (0,1)(0,2)(0,3)(1,2)(1,3)(2,3),
+      // computed (a per-lane constant-table lookup would serialise across lanes)
+      const uint32_t x = inv[E[e][0]], y = inv[E[e][1]];
+      const uint32_t p = x < y ? x : y, q = x < y ? y : x;
+      idx[e] = p * 3 - (p * (p - 1)) / 2 + (q - p - 1);
+    }
     // sort ne <= 3 pair indices
     if (idx[0] > idx[1]) { const uint32_t t = idx[0]; idx[0] = idx[1]; idx[1] = t; }
     if (idx[1] > idx[2]) { const uint32_t t = idx[1]; idx[1] = idx[2]; idx[2] = t; }

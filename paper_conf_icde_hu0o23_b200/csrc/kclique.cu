@@ -655,11 +655,26 @@ __global__ void outdeg_key_kernel(const uint64_t *dag_ptr, uint32_t n, uint32_t 
   }
 }
 
-__global__ void outdeg_hist_kernel(const uint64_t *dag_ptr, const uint32_t *roots, uint64_t nr, uint32_t *hist) {
+// d+ histogram of a root list: block-private shared-memory bins (most roots fall in a
+// handful of small-degree bins, so global atomics would serialise), flushed once
+constexpr uint32_t kHistSmem = 4096;
+__global__ void outdeg_hist_kernel(const uint64_t *dag_ptr, const uint32_t *roots, uint64_t nr, uint32_t nb,
+                                   uint32_t *hist) {
+  __shared__ uint32_t sh[kHistSmem];
+  const bool local = nb <= kHistSmem;
+  if (local)
+    for (uint32_t b = threadIdx.x; b < nb; b += blockDim.x) sh[b] = 0;
+  __syncthreads();
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < nr; i += (uint64_t)gridDim.x * blockDim.x) {
     const uint32_t v = roots[i];
-    atomicAdd(&hist[dag_ptr[v + 1] - dag_ptr[v]], 1u);
+    const uint32_t d = (uint32_t)(dag_ptr[v + 1] - dag_ptr[v]);
+    if (local) atomicAdd(&sh[d], 1u);
+    else atomicAdd(&hist[d], 1u);
   }
+  __syncthreads();
+  if (local)
+    for (uint32_t b = threadIdx.x; b < nb; b += blockDim.x)
+      if (sh[b]) atomicAdd(&hist[b], sh[b]);
 }
 }  // namespace
 
@@ -715,7 +730,8 @@ void ensure_root_order(gamma_graph *g) {
   GAMMA_CUDA(cudaMemsetAsync(hist.p, 0, nb * 4, ctx->stream));
   if (nr)
     ctx->launch(KC_ROOTS, [&] {
-      outdeg_hist_kernel<<<grid1d(nr), 256, 0, ctx->stream>>>(g->dag_ptr, order.p, nr, hist.p);
+      outdeg_hist_kernel<<<std::min<unsigned>(grid1d(nr), 148u * 4u), 256, 0, ctx->stream>>>(g->dag_ptr, order.p,
+                                                                                           nr, nb, hist.p);
     });
   std::vector<uint32_t> h(nb);
   GAMMA_CUDA(cudaMemcpyAsync(h.data(), hist.p, nb * 4, cudaMemcpyDeviceToHost, ctx->stream));

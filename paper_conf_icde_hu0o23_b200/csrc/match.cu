@@ -42,7 +42,7 @@ constexpr int kMaxV = 8;
 constexpr int kWarps = 8;
 constexpr int kThreads = kWarps * 32;
 constexpr uint32_t kLmCap = 1024;    // staged L_m per warp (u32)
-constexpr uint32_t kOutCap = 1024;   // staged child run per warp (u32)
+constexpr uint32_t kOutCap = 512;    // staged child run per warp (u32); longer runs go direct
 constexpr uint32_t kBlkV = 4096;
 constexpr uint32_t kBlkG = 256;      // descriptors per warp block
 constexpr uint32_t kSlice = 64;      // children per group descriptor
@@ -240,7 +240,7 @@ __global__ void __launch_bounds__(kThreads) sm_kernel(SmArgs a) {
       }
       if (staged && lm_len == 0) continue;   // no child can extend
       const uint32_t *run = a.vid_in + beg;
-      if (last && staged && !(child_in_b && lm_len > 32)) {
+      if (last && staged) {
         // Last level over a staged L_m: count without a per-child warp loop.  The
         // filters that involve the child c = phi_d are an order window (lo_c, hi_c)
         // and possibly x != c; the prefix filters are already applied to L_m.
@@ -259,9 +259,62 @@ __global__ void __launch_bounds__(kThreads) sm_kernel(SmArgs a) {
             if (inj_d && (int64_t)c > lo && c < hi && cnt && sorted_contains(slm, lm_len, c)) cnt--;
             part += cnt;
           }
+        } else if (lm_len > 32) {
+          // cand(c) = L_m ∩ N(c) ∩ window with a long L_m: stream the children's lists
+          // N(c) in flattened windows of 32 children (one element per lane per step,
+          // child found by an OR-reduction of the window's start offsets) and probe L_m
+          // in shared memory
+          const uint32_t lmin = slm[0], lmax = slm[lm_len - 1];
+          const uint32_t upto = lane == 31 ? 0xffffffffu : ((2u << lane) - 1u);
+          for (uint32_t w0 = 0; w0 < len; w0 += 32) {
+            const uint32_t i = w0 + lane;
+            uint32_t c = 0, beg = 0, dl = 0;
+            if (i < len) {
+              c = run[i];
+              const uint64_t s0 = a.rp[c];
+              dl = (uint32_t)(a.rp[c + 1] - s0);
+              beg = (uint32_t)s0;
+            }
+            elems += dl;
+            const uint32_t nz = __ballot_sync(0xffffffffu, dl > 0);
+            const uint32_t nnz = __popc(nz);
+            const uint32_t src = lane < (int)nnz ? __fns(nz, 0, lane + 1) : 0;
+            const uint32_t cbeg = __shfl_sync(0xffffffffu, beg, src);
+            const uint32_t sdl = __shfl_sync(0xffffffffu, dl, src);
+            const uint32_t cc = __shfl_sync(0xffffffffu, c, src);
+            const uint32_t cdl = lane < (int)nnz ? sdl : 0u;
+            uint32_t s = cdl;   // exclusive scan of the compacted lengths
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+              const uint32_t y = __shfl_up_sync(0xffffffffu, s, o);
+              if (lane >= o) s += y;
+            }
+            const uint32_t T = __shfl_sync(0xffffffffu, s, 31);
+            const uint32_t ost = s - cdl;
+            uint32_t nb = 0;
+            for (uint32_t t0 = 0; t0 < T; t0 += 32) {
+              const uint32_t t = t0 + lane;
+              const uint32_t mine = (lane < (int)nnz && ost >= t0 && ost < t0 + 32) ? (1u << (ost - t0)) : 0u;
+              const uint32_t S = __reduce_or_sync(0xffffffffu, mine);
+              const int j = (int)(nb + __popc(S & upto)) - 1;
+              nb += __popc(S);
+              const uint32_t bj = __shfl_sync(0xffffffffu, cbeg, j & 31);
+              const uint32_t oj = __shfl_sync(0xffffffffu, ost, j & 31);
+              const uint32_t cj = __shfl_sync(0xffffffffu, cc, j & 31);
+              bool ok = false;
+              if (t < T) {
+                const uint32_t x = __ldg(a.col + bj + (t - oj));
+                const int64_t lo = lt_d ? max(bs.lo, (int64_t)cj) : bs.lo;
+                const uint32_t hi = gt_d ? min(bs.hi, cj) : bs.hi;
+                ok = x >= lmin && x <= lmax && (int64_t)x > lo && x < hi && !(inj_d && x == cj) &&
+                     sorted_contains(slm, lm_len, x);
+              }
+              part += __popc(__ballot_sync(0xffffffffu, ok)) * (lane == 0);
+            }
+          }
         } else {
-          // cand(c) = L_m ∩ N(c) ∩ window: flatten (child, L_m element) pairs over the
-          // lanes; each pair is one binary search of x in N(c)
+          // cand(c) = L_m ∩ N(c) ∩ window with a short L_m: flatten (child, L_m element)
+          // pairs over the lanes; each pair is one binary search of x in N(c)
           const uint64_t T = (uint64_t)len * lm_len;
           for (uint32_t i = lane; i < len; i += 32) elems += gdeg(a, run[i]);   // each N(c) once
           for (uint64_t t0 = 0; t0 < T; t0 += 32) {
