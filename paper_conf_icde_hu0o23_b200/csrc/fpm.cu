@@ -20,10 +20,11 @@
 //    edge-pair list; every minimizing order is an automorphic placement, so OR-ing
 //    the vertex of each position into that position's domain merges orbits (MNI).
 //  * Pattern table: lock-free open-addressing hash (one-word code -> slot, claimed
-//    by a single atomicCAS, so no lane ever waits on another) in HBM; the MNI domain
-//    of slot position p is a bitmap over the vertices of p's label class (bit index
-//    = rank of the vertex inside its label class) at a fixed offset of the slot.
-//    Support = min over positions of popcount (one warp per slot).
+//    by a single atomicCAS) in HBM, sized from the number of label combinations so
+//    probe chains stay short; the claimer carves the slot's MNI domains from a pool:
+//    one bitmap per position over the vertices of that position's label class (bit
+//    index = rank of the vertex inside its class), so memory follows the patterns
+//    that occur.  Support = min over positions of popcount (one warp per slot).
 #include <cub/device/device_radix_sort.cuh>
 
 #include <algorithm>
@@ -50,12 +51,14 @@ __constant__ uint8_t c_perm4[24][4] = {
 constexpr uint64_t kKeyTag = 1ull << 63;
 
 struct Table {
-  unsigned long long *key;   // 0 = empty; claimed with one atomicCAS (no spinning)
+  unsigned long long *key;   // 0 = empty; claimed with one atomicCAS
   unsigned long long *support;
   uint32_t *freq;            // 1 if support >= minsup (set after the slot's level)
+  unsigned long long *dom;   // 1 + pool offset of the slot's domains (0: being carved, ~0: no room)
   uint64_t cap;              // power of two
-  uint32_t *pool;            // domain of (slot s, position p) at pool + (4 s + p) * slot_words
-  uint64_t slot_words;       // words of the largest label class bitmap
+  uint32_t *pool;            // per-slot domains, one bitmap per position over its label class
+  uint64_t pool_words;
+  unsigned long long *pool_cur;
 };
 
 __host__ __device__ __forceinline__ uint32_t key_nv(uint64_t k) { return (uint32_t)((k >> 48) & 7); }
@@ -100,9 +103,8 @@ __device__ __forceinline__ uint64_t mix64(uint64_t x) {
 }
 
 // Lookup (insert = false) or lookup-or-insert a pattern code; returns slot or -1.
-// Lookup (insert = false) or lookup-or-insert a pattern code; returns slot or -1.
-// Lock-free: a slot is claimed by one atomicCAS of its key word, so no thread ever
-// waits on another (safe for lanes of the same warp).
+// Lock-free: a slot is claimed by one atomicCAS of its key word; the claimer then
+// carves the slot's domains from the pool (record() waits for that with nanosleep).
 __device__ int64_t table_slot(const FpmArgs &a, uint64_t key, bool insert) {
   const Table &T = a.T;
   uint64_t h = mix64(key) & (T.cap - 1);
@@ -115,7 +117,23 @@ __device__ int64_t table_slot(const FpmArgs &a, uint64_t key, bool insert) {
     if (k == 0) {
       if (!insert) return -1;
       k = atomicCAS(&T.key[h], 0ull, (unsigned long long)key);
-      if (k == 0 || k == key) return (int64_t)h;
+      if (k == 0) {
+        // the claimer carves the slot's domains: one bitmap per position, sized to the
+        // position's label class
+        const uint32_t nv = key_nv(key);
+        uint64_t words = 0;
+        for (uint32_t p = 0; p < nv; p++) words += (a.csize[key_label(key, p)] + 31) / 32;
+        const unsigned long long off = atomicAdd(T.pool_cur, (unsigned long long)words);
+        unsigned long long d = off + 1;
+        if (off + words > T.pool_words) {
+          atomicExch(&a.ctrl[CTRL_OVF], 1ull);
+          d = ~0ull;
+        }
+        __threadfence();
+        atomicExch(&T.dom[h], d);
+        return (int64_t)h;
+      }
+      if (k == key) return (int64_t)h;
     }
   }
   if (insert) atomicExch(&a.ctrl[CTRL_ERR], 1ull);   // table full
@@ -189,7 +207,20 @@ __device__ void record(const FpmArgs &a, const uint32_t *W, uint32_t nv, const u
   const int64_t s = table_slot(a, cn.key, true);
   if (s < 0) return;
   uint64_t off[4];
-  for (uint32_t p = 0; p < 4; p++) off[p] = ((uint64_t)s * 4 + p) * a.T.slot_words;
+  // the claimer may still be carving this slot's domains (a few instructions away);
+  // the wait yields with nanosleep so a claiming lane of the same warp progresses
+  unsigned long long d = *(volatile unsigned long long *)&a.T.dom[s];
+  while (d == 0) {
+    __nanosleep(32);
+    d = *(volatile unsigned long long *)&a.T.dom[s];
+  }
+  if (d == ~0ull) return;   // pool exhausted: the host grows it and reruns
+  __threadfence();
+  uint64_t o = d - 1;
+  for (uint32_t p = 0; p < 4; p++) {
+    off[p] = o;
+    if (p < nv) o += (a.csize[key_label(cn.key, p)] + 31) / 32;
+  }
   uint32_t m = cn.minmask;
   while (m) {
     const int r = __ffs(m) - 1;
@@ -283,37 +314,95 @@ __global__ void __launch_bounds__(kThreads) fpm_enum_kernel(FpmArgs a) {
       const uint64_t nu = ue - us, ncand = nu + (ve - vs);
       for (uint64_t c0 = 0; c0 < ncand; c0 += 32) {
         const uint64_t ci = c0 + lane;
-        if (ci >= ncand) continue;
-        const uint32_t x = ci < nu ? u : v;
-        const uint32_t y = ci < nu ? a.col[us + ci] : a.col[vs + (ci - nu)];
-        const uint64_t e2 = ekey(x, y);
-        if (e2 <= e1) continue;   // also drops e1 itself
+        // lane's second edge e2 (a candidate prefix {e1, e2})
+        bool valid = ci < ncand;
+        uint64_t e2 = 0;
         ESet s2{};
-        add_edge(s2, e1);
-        add_edge(s2, e2);
-        if (a.level == 2) {
-          record(a, s2.W, s2.nv, s2.E, s2.ne);
-          emb++;
-          continue;
+        if (valid) {
+          const uint32_t x = ci < nu ? u : v;
+          const uint32_t y = ci < nu ? a.col[us + ci] : a.col[vs + (ci - nu)];
+          e2 = ekey(x, y);
+          valid = e2 > e1;   // also drops e1 itself
         }
-        if (!frequent(a, s2.W, s2.nv, s2.E, s2.ne)) continue;
-        // third edges: incident to the 3 vertices of {e1, e2}; an edge joining two of
-        // them is seen from both ends -- keep it at its smaller end only
-        for (uint32_t wi = 0; wi < 3; wi++) {
-          const uint32_t w = s2.W[wi];
-          for (uint64_t j = a.rp[w]; j < a.rp[w + 1]; j++) {
-            const uint32_t z = a.col[j];
-            const bool inner = z == s2.W[0] || z == s2.W[1] || z == s2.W[2];
-            if (inner && z < w) continue;
-            const uint64_t e3 = ekey(w, z);
-            if (e3 == e1 || e3 == e2) continue;
-            const bool ok = (e3 > e2) || (e3 > e1 && shares(e3, e2) && !shares(e3, e1));
-            if (!ok) continue;
-            ESet s3 = s2;
-            add_edge(s3, e3);
-            record(a, s3.W, s3.nv, s3.E, s3.ne);
+        if (valid) {
+          add_edge(s2, e1);
+          add_edge(s2, e2);
+          if (a.level == 2) {
+            record(a, s2.W, s2.nv, s2.E, s2.ne);
             emb++;
+            valid = false;
+          } else {
+            valid = frequent(a, s2.W, s2.nv, s2.E, s2.ne);   // Alg. 2 line 4
           }
+        }
+        if (a.level == 2) continue;   // uniform
+        // third edges: incident to the 3 vertices of a frequent prefix.  The candidate
+        // lists of the valid prefixes are concatenated and streamed by all 32 lanes
+        // (flattened windows; prefix found by an OR-reduction of the start offsets),
+        // so a hub prefix does not serialise on one lane.
+        uint32_t w0 = 0, w1 = 0, w2 = 0, d0 = 0, d1 = 0, d2 = 0, b0 = 0, b1 = 0, b2 = 0;
+        if (valid) {
+          w0 = s2.W[0]; w1 = s2.W[1]; w2 = s2.W[2];
+          b0 = (uint32_t)a.rp[w0]; d0 = (uint32_t)(a.rp[w0 + 1] - b0);
+          b1 = (uint32_t)a.rp[w1]; d1 = (uint32_t)(a.rp[w1 + 1] - b1);
+          b2 = (uint32_t)a.rp[w2]; d2 = (uint32_t)(a.rp[w2 + 1] - b2);
+        }
+        const uint32_t tl = d0 + d1 + d2;   // 0 unless valid (every vertex has an edge)
+        const uint32_t nz = __ballot_sync(0xffffffffu, tl > 0);
+        const uint32_t nnz = __popc(nz);
+        const uint32_t src = lane < (int)nnz ? __fns(nz, 0, lane + 1) : 0;
+        // compacted prefix data (lane k = k-th valid prefix)
+        const uint64_t ce2 = __shfl_sync(0xffffffffu, e2, src);
+        const uint32_t cw0 = __shfl_sync(0xffffffffu, w0, src), cw1 = __shfl_sync(0xffffffffu, w1, src);
+        const uint32_t cw2 = __shfl_sync(0xffffffffu, w2, src);
+        const uint32_t cb0 = __shfl_sync(0xffffffffu, b0, src), cb1 = __shfl_sync(0xffffffffu, b1, src);
+        const uint32_t cb2 = __shfl_sync(0xffffffffu, b2, src);
+        const uint32_t cd0 = __shfl_sync(0xffffffffu, d0, src), cd1 = __shfl_sync(0xffffffffu, d1, src);
+        const uint32_t stl = __shfl_sync(0xffffffffu, tl, src);
+        const uint32_t ctl = lane < (int)nnz ? stl : 0u;
+        uint32_t sc = ctl;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const uint32_t yv = __shfl_up_sync(0xffffffffu, sc, o);
+          if (lane >= o) sc += yv;
+        }
+        const uint32_t T = __shfl_sync(0xffffffffu, sc, 31);
+        const uint32_t ost = sc - ctl;
+        const uint32_t upto = lane == 31 ? 0xffffffffu : ((2u << lane) - 1u);
+        uint32_t nb = 0;
+        for (uint32_t t0 = 0; t0 < T; t0 += 32) {
+          const uint32_t t = t0 + lane;
+          const uint32_t mine = (lane < (int)nnz && ost >= t0 && ost < t0 + 32) ? (1u << (ost - t0)) : 0u;
+          const uint32_t S = __reduce_or_sync(0xffffffffu, mine);
+          const int j = ((int)(nb + __popc(S & upto)) - 1) & 31;
+          nb += __popc(S);
+          const uint64_t pe2 = __shfl_sync(0xffffffffu, ce2, j);
+          const uint32_t p0 = __shfl_sync(0xffffffffu, cw0, j), p1 = __shfl_sync(0xffffffffu, cw1, j);
+          const uint32_t p2 = __shfl_sync(0xffffffffu, cw2, j);
+          const uint32_t q0 = __shfl_sync(0xffffffffu, cb0, j), q1 = __shfl_sync(0xffffffffu, cb1, j);
+          const uint32_t q2 = __shfl_sync(0xffffffffu, cb2, j);
+          const uint32_t r0 = __shfl_sync(0xffffffffu, cd0, j), r1 = __shfl_sync(0xffffffffu, cd1, j);
+          const uint32_t oj = __shfl_sync(0xffffffffu, ost, j);
+          if (t >= T) continue;
+          const uint32_t r = t - oj;
+          uint32_t w, zi;
+          if (r < r0) { w = p0; zi = q0 + r; }
+          else if (r < r0 + r1) { w = p1; zi = q1 + (r - r0); }
+          else { w = p2; zi = q2 + (r - r0 - r1); }
+          const uint32_t z = a.col[zi];
+          // an edge joining two prefix vertices is seen from both ends: keep the smaller
+          const bool inner = z == p0 || z == p1 || z == p2;
+          if (inner && z < w) continue;
+          const uint64_t e3 = ekey(w, z);
+          if (e3 == e1 || e3 == pe2) continue;
+          const bool ok = (e3 > pe2) || (e3 > e1 && shares(e3, pe2) && !shares(e3, e1));
+          if (!ok) continue;
+          ESet s3{};
+          add_edge(s3, e1);
+          add_edge(s3, pe2);
+          add_edge(s3, e3);
+          record(a, s3.W, s3.nv, s3.E, s3.ne);
+          emb++;
         }
       }
     }
@@ -337,7 +426,8 @@ __global__ void fpm_support_kernel(FpmArgs a, uint32_t level, uint64_t minsup) {
     for (uint32_t p = 0; p < nv; p++) {
       const uint32_t lp = key_label(key, p);
       const uint64_t words = (a.csize[lp] + 31) / 32;
-      const uint64_t off = (s * 4 + p) * a.T.slot_words;
+      uint64_t off = a.T.dom[s] - 1;
+      for (uint32_t i = 0; i < p; i++) off += (a.csize[key_label(key, i)] + 31) / 32;
       uint64_t c = 0;
       for (uint64_t w = lane; w < words; w += 32) c += __popc(a.T.pool[off + w]);
       for (int o = 16; o > 0; o >>= 1) c += __shfl_down_sync(0xffffffffu, c, o);
@@ -435,15 +525,20 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
   ctx->sync();
   uint64_t maxw = 1;
   for (auto c : hsize) maxw = std::max<uint64_t>(maxw, (c + 31) / 32);
-  // distinct patterns are bounded by the label combinations that occur; start from
-  // min(#labels^2 * 64, 2^20) slots, grow x4 when a probe chain gets long
-  const uint64_t slot_bytes = 8 + 8 + 4 + 4 * maxw * 4;
-  uint64_t cap = 1;
-  const uint64_t want = std::min<uint64_t>((uint64_t)nlab * nlab * 64 + 1024, 1ull << 20);
-  while (cap < want) cap <<= 1;
-  while (cap > 1024 && cap * slot_bytes > budget) cap >>= 1;
+  // Distinct patterns are bounded by the label combinations of each shape (edge,
+  // wedge, triangle, 3-star, 3-path); size the table at twice that bound (load <= 1/2,
+  // short probe chains) and grow x4 if a chain still gets long.  The domain pool is
+  // bounded by the budget and by 4 class bitmaps per slot.
+  const double L = nlab;
+  double bound = L * (L + 1) / 2;                                  // edges
+  if (max_edges >= 2) bound += L * L * (L + 1) / 2;                // wedges
+  if (max_edges >= 3) bound += (L + 2) * (L + 1) * L / 6 * (1 + L) + L * L * L * L;   // triangles, 3-stars, 3-paths
+  uint64_t cap = 1024;
+  while ((double)cap < 2 * bound && cap < (1ull << 24)) cap <<= 1;
+  const uint64_t slot_bytes = 8 + 8 + 4 + 8;
+  while (cap > 1024 && cap * slot_bytes * 4 > budget) cap >>= 1;
   DevBuf<uint32_t> freq, pool;
-  DevBuf<unsigned long long> key, sup;
+  DevBuf<unsigned long long> key, sup, dom, pcur;
   FpmArgs a{};
   a.rp = g->row_ptr;
   a.col = g->col;
@@ -455,19 +550,24 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
   a.world = 1;   // FPM runs every root on every rank (replicas)
   a.ctrl = (unsigned long long *)ctx->ctrl;
   const int grid_enum = ctx->num_sms * occupancy_blocks((const void *)fpm_enum_kernel, kThreads, 0);
-  for (;;) {
-    GAMMA_REQUIRE(cap * slot_bytes <= budget, GAMMA_E_NOMEM,
-                  "gamma_fpm: pattern table + MNI domains exceed the HBM budget");
-    freq.reset(); pool.reset(); key.reset(); sup.reset();
+  for (int attempt = 0;; attempt++) {
+    GAMMA_REQUIRE(cap * slot_bytes < budget, GAMMA_E_NOMEM, "gamma_fpm: pattern table exceeds the HBM budget");
+    const uint64_t pool_words =
+        std::max<uint64_t>(64, std::min<uint64_t>((budget - cap * slot_bytes) / 4, cap * 4 * maxw));
+    freq.reset(); pool.reset(); key.reset(); sup.reset(); dom.reset(); pcur.reset();
     key = DevBuf<unsigned long long>(ctx, cap);
     sup = DevBuf<unsigned long long>(ctx, cap);
+    dom = DevBuf<unsigned long long>(ctx, cap);
     freq = DevBuf<uint32_t>(ctx, cap);
-    pool = DevBuf<uint32_t>(ctx, cap * 4 * maxw);
+    pool = DevBuf<uint32_t>(ctx, pool_words);
+    pcur = DevBuf<unsigned long long>(ctx, 1);
     GAMMA_CUDA(cudaMemsetAsync(key.p, 0, cap * 8, ctx->stream));
+    GAMMA_CUDA(cudaMemsetAsync(dom.p, 0, cap * 8, ctx->stream));
     GAMMA_CUDA(cudaMemsetAsync(freq.p, 0, cap * 4, ctx->stream));
-    GAMMA_CUDA(cudaMemsetAsync(pool.p, 0, cap * 4 * maxw * 4, ctx->stream));
-    a.T = Table{key.p, sup.p, freq.p, cap, pool.p, maxw};
-    bool full = false;
+    GAMMA_CUDA(cudaMemsetAsync(pool.p, 0, pool_words * 4, ctx->stream));
+    GAMMA_CUDA(cudaMemsetAsync(pcur.p, 0, 8, ctx->stream));
+    a.T = Table{key.p, sup.p, freq.p, dom.p, cap, pool.p, pool_words, pcur.p};
+    bool full = false, exhausted = false;
     for (uint32_t l = 1; l <= max_edges; l++) {
       a.level = l;
       ctrl_reset(ctx);
@@ -478,10 +578,13 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
       ctrl_fetch(ctx);
       const uint64_t *h = ctx->ctrl_host;
       full = h[CTRL_ERR] != 0;
-      if (full) break;
+      exhausted = h[CTRL_OVF] != 0;
+      if (full || exhausted) break;
       ctx->stats.level_entries[l] = h[CTRL_ENTRIES];
     }
-    if (!full) break;
+    if (!full && !exhausted) break;
+    GAMMA_REQUIRE(!exhausted, GAMMA_E_NOMEM, "gamma_fpm: MNI domain pool exceeds the HBM budget");
+    GAMMA_REQUIRE(attempt < 6, GAMMA_E_NOMEM, "gamma_fpm: pattern table keeps overflowing");
     ctx->stats.retries++;   // sizes are only known after the fact: grow and redo
     cap *= 4;
   }

@@ -356,15 +356,19 @@ __global__ void __launch_bounds__(kThreads) sm_kernel(SmArgs a) {
         uint64_t pos = 0;
         bool big = false;
         if (staged && !child_in_b) {
-          // candidates = L_m minus position-d filters (all prefix filters applied)
+          // candidates = L_m minus position-d filters (all prefix filters applied); a
+          // run longer than the staging buffer is written straight to the level
           found = 0;
+          big = !last && lm_len > kOutCap;
+          if (big && !pool_reserve(pv, lm_len, lane, pos)) { stop = true; break; }
+          uint32_t *dst = big ? a.vid_out + pos : sout;
           for (uint32_t j0 = 0; j0 < lm_len; j0 += 32) {
             const uint32_t jj = j0 + lane;
             const uint32_t x = jj < lm_len ? slm[jj] : 0xffffffffu;
             const bool ok = jj < lm_len && (int64_t)x > bc.lo && x < bc.hi &&
                             !(((a.P.injmask[q] >> d) & 1u) && x == c);
             const uint32_t bal = __ballot_sync(0xffffffffu, ok);
-            if (!last && ok) sout[found + __popc(bal & lanemask_lt())] = x;
+            if (!last && ok) dst[found + __popc(bal & lanemask_lt())] = x;
             found += __popc(bal);
           }
         } else {

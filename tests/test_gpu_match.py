@@ -108,6 +108,22 @@ def test_more_patterns(ctx, oracle_mod):
     assert g.match(1, [], [1])[0] == int((lab == 1).sum())
 
 
+def test_hub_staged_prefix_list(ctx, oracle_mod):
+    """A hub whose neighbour list (~900) fits the shared-memory L_m but not the
+    512-entry child-run staging: long runs must go straight to the level."""
+    rng = np.random.default_rng(11)
+    n = 1200
+    hub = [(0, i) for i in range(1, 901)]
+    extra = [tuple(x) for x in rng.integers(1, n, size=(5000, 2))]
+    e = np.array(hub + extra, dtype=np.uint32)
+    s, d = e[:, 0].copy(), e[:, 1].copy()
+    g = ctx.load_edges(n, s, d)
+    o = oracle_mod.Graph(n, s, d)
+    for q in ("diamond", "house", "tailed_triangle", "c4"):
+        nv, pe = Q[q]
+        assert g.match(nv, pe)[0] == o.match(nv, pe)[0], q
+
+
 def test_simulated_ranks(G, oracle_mod):
     n, s, d, _ = gg.config_graph("c3", seed=2, scale=11)
     lab = gg.labels(n, 4, 2)

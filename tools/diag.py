@@ -59,7 +59,8 @@ def main():
         import torch
         import paper_conf_icde_hu0o23_b200 as G
         import bench
-        n, s, d, lab = gg.config_graph("c3", seed=1)
+        sc = int(sys.argv[2]) if len(sys.argv) > 2 else None
+        n, s, d, lab = gg.config_graph("c3", seed=1, scale=sc)
         c = G.Context(time_kernels=True)
         g = c.load_edges(n, torch.from_numpy(s.view("int32")).cuda(), torch.from_numpy(d.view("int32")).cuda(),
                          torch.from_numpy(lab.view("int32")).cuda())
