@@ -274,26 +274,32 @@ __device__ __forceinline__ void add_edge(ESet &s, uint64_t e) {
 __global__ void __launch_bounds__(kThreads) fpm_enum_kernel(FpmArgs a) {
   const int lane = threadIdx.x & 31;
   uint64_t emb = 0;
+  const uint64_t ndir = a.rp[a.n];   // directed edges: the roots are the (u, v > u) ones
+  constexpr uint64_t kBatch = 8;
   for (;;) {
-    unsigned long long u0 = 0;
-    if (lane == 0) u0 = atomicAdd(&a.ctrl[CTRL_WORK], 1ull);
-    u0 = __shfl_sync(0xffffffffu, u0, 0);
-    if (u0 >= a.n) break;
-    const uint32_t u = (uint32_t)u0;
-    if (a.world > 1 && (u % a.world) != a.rank) continue;
-    const uint64_t us = a.rp[u], ue = a.rp[u + 1];
-    // first neighbour > u
-    uint64_t first = us;
+    // work unit = a batch of root edges (not a root vertex: a hub's edges spread
+    // over many warps)
+    unsigned long long i0 = 0;
+    if (lane == 0) i0 = atomicAdd(&a.ctrl[CTRL_WORK], kBatch);
+    i0 = __shfl_sync(0xffffffffu, i0, 0);
+    if (i0 >= ndir) break;
+    // u = row of directed edge i0 (binary search of row_ptr)
+    uint32_t u;
     {
-      uint64_t lo = us, hi = ue;
-      while (lo < hi) {
-        const uint64_t mid = (lo + hi) >> 1;
-        if (a.col[mid] <= u) lo = mid + 1; else hi = mid;
+      uint32_t lo = 0, hi = a.n;
+      while (hi - lo > 1) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (a.rp[mid] <= i0) lo = mid; else hi = mid;
       }
-      first = lo;
+      u = lo;
     }
-    for (uint64_t i1 = first; i1 < ue; i1++) {
+    const uint64_t iend = i0 + kBatch < ndir ? i0 + kBatch : ndir;
+    for (uint64_t i1 = i0; i1 < iend; i1++) {
+      while (a.rp[u + 1] <= i1) u++;   // the batch may cross rows
       const uint32_t v = a.col[i1];
+      if (v < u) continue;             // each undirected edge once, from its smaller end
+      if (a.world > 1 && (u % a.world) != a.rank) continue;
+      const uint64_t us = a.rp[u], ue = a.rp[u + 1];
       const uint64_t e1 = ekey(u, v);
       if (a.level == 1) {
         if (lane == 0) {
