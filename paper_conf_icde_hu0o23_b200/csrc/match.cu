@@ -77,6 +77,8 @@ struct SmArgs {
   unsigned long long *ctrl;
   uint32_t batch;
   uint32_t stage;           // 0: never stage L_m (debug)
+  uint32_t *lm_scratch;     // per-warp global L_m slices for hub prefixes (nullable)
+  uint32_t lm_scratch_cap;  // entries per warp slice
 };
 
 __device__ __forceinline__ uint32_t gdeg(const SmArgs &a, uint32_t v) {
@@ -222,8 +224,22 @@ __global__ void __launch_bounds__(kThreads) sm_kernel(SmArgs a) {
       const Bounds bs = bounds_for(a, q, prefix_mask, phi);
       bool staged = false;
       uint32_t lm_len = 0;
+      // L_m lives in shared memory when its bound (the shortest prefix list) fits,
+      // else in this warp's slice of a global scratch buffer (hub prefixes)
+      uint32_t *lm = slm;
+      uint32_t lm_cap = kLmCap;
       if (bshared && a.stage) {
-        const uint32_t r = sm_intersect<true>(a, q, bshared, phi, bs, last, nullptr, 0, slm, kLmCap, lane);
+        uint32_t bound = 0xffffffffu, mm = bshared;
+        while (mm) {
+          const int j = __ffs(mm) - 1;
+          mm &= mm - 1;
+          bound = min(bound, gdeg(a, phi[j]));
+        }
+        if (bound > kLmCap && a.lm_scratch) {
+          lm = a.lm_scratch + (uint64_t)(blockIdx.x * kWarps + wid) * a.lm_scratch_cap;
+          lm_cap = a.lm_scratch_cap;
+        }
+        const uint32_t r = sm_intersect<true>(a, q, bshared, phi, bs, last, nullptr, 0, lm, lm_cap, lane);
         __syncwarp();
         if (r != 0xffffffffu) {
           staged = true;
@@ -253,10 +269,10 @@ __global__ void __launch_bounds__(kThreads) sm_kernel(SmArgs a) {
             const uint32_t c = run[i];
             const int64_t lo = lt_d ? max(bs.lo, (int64_t)c) : bs.lo;
             const uint32_t hi = gt_d ? min(bs.hi, c) : bs.hi;
-            const uint32_t a0 = lo < 0 ? 0u : upper_bound_idx(slm, lm_len, (uint32_t)lo);
-            const uint32_t a1 = hi == 0 ? 0u : upper_bound_idx(slm, lm_len, hi - 1);
+            const uint32_t a0 = lo < 0 ? 0u : upper_bound_idx(lm, lm_len, (uint32_t)lo);
+            const uint32_t a1 = hi == 0 ? 0u : upper_bound_idx(lm, lm_len, hi - 1);
             uint32_t cnt = a1 > a0 ? a1 - a0 : 0u;
-            if (inj_d && (int64_t)c > lo && c < hi && cnt && sorted_contains(slm, lm_len, c)) cnt--;
+            if (inj_d && (int64_t)c > lo && c < hi && cnt && sorted_contains(lm, lm_len, c)) cnt--;
             part += cnt;
           }
         } else if (lm_len > 32) {
@@ -264,7 +280,7 @@ __global__ void __launch_bounds__(kThreads) sm_kernel(SmArgs a) {
           // N(c) in flattened windows of 32 children (one element per lane per step,
           // child found by an OR-reduction of the window's start offsets) and probe L_m
           // in shared memory
-          const uint32_t lmin = slm[0], lmax = slm[lm_len - 1];
+          const uint32_t lmin = lm[0], lmax = lm[lm_len - 1];
           const uint32_t upto = lane == 31 ? 0xffffffffu : ((2u << lane) - 1u);
           for (uint32_t w0 = 0; w0 < len; w0 += 32) {
             const uint32_t i = w0 + lane;
@@ -307,7 +323,7 @@ __global__ void __launch_bounds__(kThreads) sm_kernel(SmArgs a) {
                 const int64_t lo = lt_d ? max(bs.lo, (int64_t)cj) : bs.lo;
                 const uint32_t hi = gt_d ? min(bs.hi, cj) : bs.hi;
                 ok = x >= lmin && x <= lmax && (int64_t)x > lo && x < hi && !(inj_d && x == cj) &&
-                     sorted_contains(slm, lm_len, x);
+                     sorted_contains(lm, lm_len, x);
               }
               part += __popc(__ballot_sync(0xffffffffu, ok)) * (lane == 0);
             }
@@ -322,7 +338,7 @@ __global__ void __launch_bounds__(kThreads) sm_kernel(SmArgs a) {
             bool ok = false;
             if (t < T) {
               const uint32_t i = (uint32_t)(t / lm_len), j = (uint32_t)(t - (uint64_t)i * lm_len);
-              const uint32_t c = run[i], x = slm[j];
+              const uint32_t c = run[i], x = lm[j];
               const int64_t lo = lt_d ? max(bs.lo, (int64_t)c) : bs.lo;
               const uint32_t hi = gt_d ? min(bs.hi, c) : bs.hi;
               ok = (int64_t)x > lo && x < hi && !(inj_d && x == c);
@@ -364,7 +380,7 @@ __global__ void __launch_bounds__(kThreads) sm_kernel(SmArgs a) {
           uint32_t *dst = big ? a.vid_out + pos : sout;
           for (uint32_t j0 = 0; j0 < lm_len; j0 += 32) {
             const uint32_t jj = j0 + lane;
-            const uint32_t x = jj < lm_len ? slm[jj] : 0xffffffffu;
+            const uint32_t x = jj < lm_len ? lm[jj] : 0xffffffffu;
             const bool ok = jj < lm_len && (int64_t)x > bc.lo && x < bc.hi &&
                             !(((a.P.injmask[q] >> d) & 1u) && x == c);
             const uint32_t bal = __ballot_sync(0xffffffffu, ok);
@@ -386,9 +402,9 @@ __global__ void __launch_bounds__(kThreads) sm_kernel(SmArgs a) {
             if (big && !pool_reserve(pv, ub, lane, pos)) { stop = true; break; }
           }
           if (last)
-            found = sm_intersect<false>(a, q, lists, phi, bc, last, staged ? slm : nullptr, lm_len, nullptr, 0, lane);
+            found = sm_intersect<false>(a, q, lists, phi, bc, last, staged ? lm : nullptr, lm_len, nullptr, 0, lane);
           else
-            found = sm_intersect<true>(a, q, lists, phi, bc, last, staged ? slm : nullptr, lm_len,
+            found = sm_intersect<true>(a, q, lists, phi, bc, last, staged ? lm : nullptr, lm_len,
                                        big ? a.vid_out + pos : sout, big ? 0xffffffffu : kOutCap, lane);
         }
         if (last) {
@@ -612,6 +628,8 @@ struct SmRun {
   uint64_t total = 0;
   int grid = 0;
   uint32_t stage = 1;
+  DevBuf<uint32_t> lm_scratch;       // per-warp global L_m slices (hub prefixes)
+  uint32_t lm_scratch_cap = 0;
 
   bool grow(uint32_t d, uint64_t want_v) {
     SmLevel &L = lv[d];
@@ -647,6 +665,8 @@ struct SmRun {
     a.ctrl = (unsigned long long *)ctx->ctrl;
     a.batch = d == 0 ? 1 : 4;
     a.stage = stage;
+    a.lm_scratch = lm_scratch.p;
+    a.lm_scratch_cap = lm_scratch_cap;
     return a;
   }
 
@@ -802,6 +822,10 @@ static uint64_t match_count(gamma_graph *g, const SmPlan &P) {
     attr = true;
   }
   R.grid = ctx->num_sms * occupancy_blocks((const void *)sm_kernel, kThreads, sm_smem());
+  if (g->max_degree > kLmCap) {   // room for a hub's L_m (bounded by its degree) per warp
+    R.lm_scratch_cap = std::min<uint32_t>(g->max_degree, 1u << 16);
+    R.lm_scratch = DevBuf<uint32_t>(ctx, (uint64_t)R.grid * kWarps * R.lm_scratch_cap);
+  }
   R.process(0, 0, ngr);
   ctx->sync();
   ctx->collect_timings();

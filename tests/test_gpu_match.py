@@ -108,12 +108,14 @@ def test_more_patterns(ctx, oracle_mod):
     assert g.match(1, [], [1])[0] == int((lab == 1).sum())
 
 
-def test_hub_staged_prefix_list(ctx, oracle_mod):
-    """A hub whose neighbour list (~900) fits the shared-memory L_m but not the
-    512-entry child-run staging: long runs must go straight to the level."""
+@pytest.mark.parametrize("deg", [900, 1500])
+def test_hub_staged_prefix_list(ctx, oracle_mod, deg):
+    """A hub whose neighbour list fits the shared-memory L_m but not the 512-entry
+    child-run staging (900: long runs go straight to the level), or exceeds the
+    shared L_m (1500: L_m goes to the warp's global scratch slice)."""
     rng = np.random.default_rng(11)
-    n = 1200
-    hub = [(0, i) for i in range(1, 901)]
+    n = 1800
+    hub = [(0, i) for i in range(1, deg + 1)]
     extra = [tuple(x) for x in rng.integers(1, n, size=(5000, 2))]
     e = np.array(hub + extra, dtype=np.uint32)
     s, d = e[:, 0].copy(), e[:, 1].copy()
