@@ -132,6 +132,15 @@ gamma_status gamma_graph_copy_csr(const gamma_graph *g, int which, uint64_t *row
  * collective (else partial).                                                       */
 gamma_status gamma_kclique(gamma_graph *g, uint32_t k, uint64_t *count);
 
+/* Several clique sizes in one call: counts[i] = number of ks[i]-cliques (host
+ * arrays, nk entries, each 1 <= ks[i] <= 32).  When every ks[i] <= 12 and the DAG's
+ * max out-degree is <= 512, all sizes 3..max(ks) come from ONE bitmap DFS pass over
+ * the roots (each visited node with t chosen vertices adds popc(candidates) to the
+ * (t+1)-clique count), so the cost is that of the largest k alone; otherwise each
+ * size runs as gamma_kclique.  Same rank/world and all-reduce rules as
+ * gamma_kclique (one collective for all nk counts).                               */
+gamma_status gamma_kclique_multi(gamma_graph *g, uint32_t nk, const uint32_t *ks, uint64_t *counts);
+
 /* Per-root counts: counts[i] = number of k-cliques whose lowest vertex under
  * (deg, id) order is roots[i] (roots/counts host or device, nroots entries).  Used
  * for sampled parity at full size; ignores rank/world.                            */

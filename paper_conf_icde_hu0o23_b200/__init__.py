@@ -267,6 +267,13 @@ class Graph:
         _check(_lib.gamma_kclique(self._h, int(k), C.byref(c)), "gamma_kclique")
         return int(c.value)
 
+    def kclique_multi(self, ks) -> list:
+        """Counts for several clique sizes from one call (one bitmap pass when possible)."""
+        ka = np.ascontiguousarray(ks, dtype=np.uint32)
+        out = np.zeros(len(ka), np.uint64)
+        _check(_lib.gamma_kclique_multi(self._h, len(ka), ka.ctypes.data, out.ctypes.data), "gamma_kclique_multi")
+        return [int(x) for x in out]
+
     def kclique_roots(self, k: int, roots) -> np.ndarray:
         pr, kr, nr = _ptr(roots, np.uint32)
         out = np.zeros(nr, np.uint64)

@@ -97,6 +97,7 @@ SIGNATURES = [
     ("gamma_graph_get_info", C.c_int32, [C.c_void_p, C.POINTER(gamma_graph_info)]),
     ("gamma_graph_copy_csr", C.c_int32, [C.c_void_p, C.c_int, C.c_void_p, C.c_void_p]),
     ("gamma_kclique", C.c_int32, [C.c_void_p, C.c_uint32, C.POINTER(C.c_uint64)]),
+    ("gamma_kclique_multi", C.c_int32, [C.c_void_p, C.c_uint32, C.c_void_p, C.c_void_p]),
     ("gamma_kclique_roots", C.c_int32, [C.c_void_p, C.c_uint32, C.c_uint64, C.c_void_p, C.c_void_p]),
     ("gamma_pattern_plan", C.c_int32, [C.POINTER(gamma_pattern), C.POINTER(gamma_plan_info)]),
     ("gamma_match", C.c_int32, [C.c_void_p, C.POINTER(gamma_pattern), C.POINTER(C.c_uint64),

@@ -3,6 +3,7 @@
 // in graph.cu (A1), kclique.cu (A2-A8 kCL), match.cu (SM) and fpm.cu (FPM).
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <chrono>
 #include <cstring>
 #include <new>
@@ -289,6 +290,34 @@ gamma_status gamma_kclique(gamma_graph *g, uint32_t k, uint64_t *count) {
     }
     c->stats.wall_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
     *count = r;
+  });
+}
+
+gamma_status gamma_kclique_multi(gamma_graph *g, uint32_t nk, const uint32_t *ks, uint64_t *counts) {
+  return guarded([&] {
+    GAMMA_REQUIRE(g && (nk == 0 || (ks && counts)), GAMMA_E_INVAL, "gamma_kclique_multi: NULL argument");
+    uint32_t kmax = 0;
+    for (uint32_t i = 0; i < nk; i++) {
+      GAMMA_REQUIRE(ks[i] >= 1, GAMMA_E_INVAL, "gamma_kclique_multi: k must be >= 1");
+      GAMMA_REQUIRE(ks[i] <= 32, GAMMA_E_UNSUPPORTED, "gamma_kclique_multi: k > 32 unsupported");
+      kmax = std::max(kmax, ks[i]);
+    }
+    gamma_ctx *c = g->ctx;
+    GAMMA_CUDA(cudaSetDevice(c->device));
+    c->reset_stats();
+    if (nk == 0) return;
+    auto t0 = std::chrono::steady_clock::now();
+    uint64_t bysize[33] = {};
+    const bool one_pass = kclique_multi(g, kmax, bysize);
+    std::vector<uint64_t> r(nk);
+    for (uint32_t i = 0; i < nk; i++)
+      r[i] = (one_pass && ks[i] >= 3) ? bysize[ks[i]] : kclique_count(g, ks[i], nullptr, 0, nullptr);
+    if (c->desc.world > 1 && c->desc.allreduce_sum_u64) {
+      gamma_status st = c->desc.allreduce_sum_u64(r.data(), nk, c->desc.coll_user);
+      GAMMA_REQUIRE(st == GAMMA_OK, st, "allreduce_sum_u64 callback failed");
+    }
+    c->stats.wall_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    for (uint32_t i = 0; i < nk; i++) counts[i] = r[i];
   });
 }
 

@@ -428,11 +428,15 @@ __global__ void fpm_support_kernel(FpmArgs a, uint32_t level, uint64_t minsup) {
     if (key == 0) continue;
     const uint32_t nv = key_nv(key), ne = key_ne(key);
     if (ne != level) continue;
+    // no domains in this pass (pool exhausted, or another chunk of a split level):
+    // a later pass computes this slot
+    const unsigned long long d = a.T.dom[s];
+    if (d == 0 || d == ~0ull) continue;
     uint64_t sup = ~0ull;
     for (uint32_t p = 0; p < nv; p++) {
       const uint32_t lp = key_label(key, p);
       const uint64_t words = (a.csize[lp] + 31) / 32;
-      uint64_t off = a.T.dom[s] - 1;
+      uint64_t off = d - 1;
       for (uint32_t i = 0; i < p; i++) off += (a.csize[key_label(key, i)] + 31) / 32;
       uint64_t c = 0;
       for (uint64_t w = lane; w < words; w += 32) c += __popc(a.T.pool[off + w]);
@@ -573,23 +577,74 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
     GAMMA_CUDA(cudaMemsetAsync(pool.p, 0, pool_words * 4, ctx->stream));
     GAMMA_CUDA(cudaMemsetAsync(pcur.p, 0, 8, ctx->stream));
     a.T = Table{key.p, sup.p, freq.p, dom.p, cap, pool.p, pool_words, pcur.p};
-    bool full = false, exhausted = false;
-    for (uint32_t l = 1; l <= max_edges; l++) {
+    bool full = false;
+    for (uint32_t l = 1; l <= max_edges && !full; l++) {
       a.level = l;
       ctrl_reset(ctx);
       ctx->launch(KC_FPM, [&] { fpm_enum_kernel<<<grid_enum, kThreads, 0, ctx->stream>>>(a); });
       ctx->launch(KC_FPM_SUPPORT, [&] {
         fpm_support_kernel<<<g1d(cap * 32), 256, 0, ctx->stream>>>(a, l, minsup);
       });
+      uint64_t carved = 0;
+      GAMMA_CUDA(cudaMemcpyAsync(&carved, pcur.p, 8, cudaMemcpyDeviceToHost, ctx->stream));
       ctrl_fetch(ctx);
-      const uint64_t *h = ctx->ctrl_host;
-      full = h[CTRL_ERR] != 0;
-      exhausted = h[CTRL_OVF] != 0;
-      if (full || exhausted) break;
-      ctx->stats.level_entries[l] = h[CTRL_ENTRIES];
+      full = ctx->ctrl_host[CTRL_ERR] != 0;
+      if (full) break;
+      ctx->stats.level_entries[l] = ctx->ctrl_host[CTRL_ENTRIES];
+      // a level's domains are dead once its supports are known (the next level reads
+      // only freq): clear what it used and carve the next level from offset 0
+      uint64_t dirty = std::min<uint64_t>(carved, pool_words);
+      const auto clear_pool = [&] {
+        if (dirty) GAMMA_CUDA(cudaMemsetAsync(pool.p, 0, dirty * 4, ctx->stream));
+        GAMMA_CUDA(cudaMemsetAsync(pcur.p, 0, 8, ctx->stream));
+        dirty = 0;
+      };
+      if (ctx->ctrl_host[CTRL_OVF] == 0) {
+        clear_pool();
+        continue;
+      }
+      // The domains of this level did not all fit the pool.  Every pattern of the
+      // level is in the table by now (a slot is claimed before its domains are
+      // carved), and the slots that got domains have their support: split the rest
+      // into chunks that fit the pool and redo the level's enumeration once per
+      // chunk, recording only into that chunk's slots (dom = ~0 elsewhere).
+      std::vector<unsigned long long> hkey(cap), hdom(cap);
+      GAMMA_CUDA(cudaMemcpyAsync(hkey.data(), key.p, cap * 8, cudaMemcpyDeviceToHost, ctx->stream));
+      GAMMA_CUDA(cudaMemcpyAsync(hdom.data(), dom.p, cap * 8, cudaMemcpyDeviceToHost, ctx->stream));
+      ctx->sync();
+      std::vector<uint64_t> pending;
+      for (uint64_t s = 0; s < cap; s++)
+        if (hkey[s] && key_ne(hkey[s]) == l && hdom[s] == ~0ull) pending.push_back(s);
+      size_t next = 0;
+      while (next < pending.size()) {
+        std::fill(hdom.begin(), hdom.end(), ~0ull);
+        uint64_t used = 0;
+        for (; next < pending.size(); next++) {
+          const uint64_t k = hkey[pending[next]];
+          uint64_t words = 0;
+          for (uint32_t p = 0; p < key_nv(k); p++) words += (hsize[key_label(k, p)] + 31) / 32;
+          GAMMA_REQUIRE(words <= pool_words, GAMMA_E_NOMEM, "gamma_fpm: one pattern's domains exceed the HBM budget");
+          if (used + words > pool_words) break;
+          hdom[pending[next]] = 1 + used;
+          used += words;
+        }
+        GAMMA_CUDA(cudaMemcpyAsync(dom.p, hdom.data(), cap * 8, cudaMemcpyHostToDevice, ctx->stream));
+        clear_pool();
+        dirty = used;
+        GAMMA_CUDA(cudaMemcpyAsync(pcur.p, &pool_words, 8, cudaMemcpyHostToDevice, ctx->stream));
+        ctrl_reset(ctx);
+        ctx->launch(KC_FPM, [&] { fpm_enum_kernel<<<grid_enum, kThreads, 0, ctx->stream>>>(a); });
+        ctx->launch(KC_FPM_SUPPORT, [&] {
+          fpm_support_kernel<<<g1d(cap * 32), 256, 0, ctx->stream>>>(a, l, minsup);
+        });
+        ctrl_fetch(ctx);
+        GAMMA_REQUIRE(ctx->ctrl_host[CTRL_ERR] == 0 && ctx->ctrl_host[CTRL_OVF] == 0, GAMMA_E_CUDA,
+                      "gamma_fpm: a chunk pass met an unclaimed pattern");
+        ctx->stats.chunks++;
+      }
+      clear_pool();
     }
-    if (!full && !exhausted) break;
-    GAMMA_REQUIRE(!exhausted, GAMMA_E_NOMEM, "gamma_fpm: MNI domain pool exceeds the HBM budget");
+    if (!full) break;
     GAMMA_REQUIRE(attempt < 6, GAMMA_E_NOMEM, "gamma_fpm: pattern table keeps overflowing");
     ctx->stats.retries++;   // sizes are only known after the fact: grow and redo
     cap *= 4;

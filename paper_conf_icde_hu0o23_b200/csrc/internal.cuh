@@ -149,7 +149,8 @@ enum {
   CTRL_ERR = 7,       // validation error flag
   CTRL_AUX0 = 8,
   CTRL_AUX1 = 9,
-  CTRL_WORDS = 16
+  CTRL_MULTI = 16,    // CTRL_MULTI + s: number of s-cliques (gamma_kclique_multi), s <= 32
+  CTRL_WORDS = 64
 };
 
 struct gamma_graph {
@@ -226,6 +227,10 @@ uint64_t kclique_count(gamma_graph *g, uint32_t k, const uint32_t *roots_dev, ui
 constexpr uint32_t kBitmapMaxRun = 512;
 constexpr uint32_t kBitmapMaxK = 12;
 uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint64_t nroots,
-                        unsigned long long *per_root, bool sorted, uint64_t n_long, uint64_t n_mid);
+                        unsigned long long *per_root, bool sorted, uint64_t n_long, uint64_t n_mid,
+                        uint64_t *multi_out = nullptr);
+// One bitmap pass counting every clique size 3..kmax (multi_out[s], s <= kmax); false
+// when the graph needs the ET path (max out-degree > kBitmapMaxRun or kmax too big).
+bool kclique_multi(gamma_graph *g, uint32_t kmax, uint64_t *multi_out);
 void ensure_root_order(gamma_graph *g);
 }  // namespace gamma_impl

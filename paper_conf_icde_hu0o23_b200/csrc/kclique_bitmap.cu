@@ -45,6 +45,7 @@ struct BmArgs {
   uint2 *parts;               // (absolute root index, part | nparts << 16)
   uint32_t parts_cap;
   uint64_t root_base;         // index of roots[0] in the full root list (parts are absolute)
+  uint32_t multi;             // count every clique size 3..k at once (gamma_kclique_multi)
 };
 
 __device__ __forceinline__ uint32_t excl_scan32(uint32_t x, int lane, uint32_t &total) {
@@ -135,6 +136,45 @@ __device__ uint64_t dfs_count(const uint32_t *B, uint32_t W, const uint32_t (&cu
     pos[s] = 0;
   }
   return cnt;
+}
+
+// Multi-size variant: every visited node with `chosen` vertices and candidates cur
+// contributes popc(cur) cliques of size chosen+1; the walk goes down to size kmax
+// (no size pruning: a branch that cannot reach kmax still holds smaller cliques).
+template <int TW>
+__device__ void dfs_multi(const uint32_t *B, uint32_t W, const uint32_t (&cur)[TW], uint32_t chosen, uint32_t kmax,
+                          uint64_t (&mc)[kMaxStack + 3]) {
+  uint32_t c0 = 0;
+#pragma unroll
+  for (int w = 0; w < TW; w++) c0 += __popc(cur[w]);
+  mc[chosen + 1] += c0;
+  if (chosen + 1 >= kmax || c0 == 0) return;
+  uint32_t stk[kMaxStack][TW];
+  uint32_t pos[kMaxStack];
+#pragma unroll
+  for (int w = 0; w < TW; w++) stk[0][w] = cur[w];
+  pos[0] = 0;
+  int s = 0;
+  while (s >= 0) {
+    uint32_t top[TW];
+#pragma unroll
+    for (int w = 0; w < TW; w++) top[w] = stk[s][w];
+    const int j = next_bit<TW>(top, pos[s], W);
+    if (j < 0) {
+      s--;
+      continue;
+    }
+    pos[s] = j + 1;
+    const uint32_t t = s + chosen + 1;   // vertices chosen after taking j
+    uint32_t nx[TW];
+    const uint32_t c = popc_and<TW>(top, B + j * W, W, nx);
+    mc[t + 1] += c;
+    if (t + 1 >= kmax || c == 0) continue;
+    s++;
+#pragma unroll
+    for (int w = 0; w < TW; w++) stk[s][w] = nx[w];
+    pos[s] = 0;
+  }
 }
 
 template <int TEAM_WARPS>
@@ -302,6 +342,15 @@ __device__ __forceinline__ uint64_t team_sum(uint64_t x, int lane, uint32_t *slo
   return r;
 }
 
+__device__ __forceinline__ void flush_multi(uint64_t (&mc)[kMaxStack + 3], const BmArgs &a, int lane) {
+  for (uint32_t sz = 3; sz <= a.k && sz < kMaxStack + 3; sz++) {
+    uint64_t x = mc[sz];
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) x += __shfl_down_sync(0xffffffffu, x, off);
+    if (lane == 0 && x) atomicAdd(&a.ctrl[CTRL_MULTI + sz], (unsigned long long)x);
+  }
+}
+
 template <int TEAM_WARPS, int TW, bool PER_ROOT>
 __global__ void __launch_bounds__(256) kcl_bitmap_kernel(BmArgs a) {
   extern __shared__ uint32_t smem[];
@@ -311,6 +360,7 @@ __global__ void __launch_bounds__(256) kcl_bitmap_kernel(BmArgs a) {
   const int tid = threadIdx.x % kTeamThreads;
   const TeamMem<TW> m(smem + team * team_words<TW>());
   uint64_t total = 0, elems = 0, entries = 0;
+  uint64_t mc[kMaxStack + 3] = {};   // multi mode: cliques per size
 
   // warp teams take roots in batches of 4 (one atomic per batch); CTA teams one
   // root at a time (their roots are the long, costly ones)
@@ -336,7 +386,7 @@ __global__ void __launch_bounds__(256) kcl_bitmap_kernel(BmArgs a) {
     const uint32_t v = a.roots[gi];
     const uint64_t b0 = a.dag_ptr[v];
     const uint32_t L = (uint32_t)(a.dag_ptr[v + 1] - b0);
-    if (L <= a.len_lo || L > a.len_hi || L < a.k - 1) continue;   // uniform across the team
+    if (L <= a.len_lo || L > a.len_hi || L < (a.multi ? 2u : a.k - 1)) continue;   // uniform across the team
     const uint32_t W = (L + 31) >> 5;
     if (tid == 0) entries += L;
     elems += build_rows<TEAM_WARPS, TW>(a, m, b0, L, tid, lane);
@@ -349,6 +399,7 @@ __global__ void __launch_bounds__(256) kcl_bitmap_kernel(BmArgs a) {
         for (uint32_t w = 0; w < W; w++) c += __popc(m.B[j1 * W + w]);
         cnt += c;
       }
+      if (a.multi) mc[3] += cnt;
     } else {
       scan_rows<TEAM_WARPS, TW>(m, L, tid, lane);
       const uint32_t items = m.P[L];
@@ -386,7 +437,12 @@ __global__ void __launch_bounds__(256) kcl_bitmap_kernel(BmArgs a) {
         for (uint32_t q = tid; q < items; q += kTeamThreads) {
           uint32_t cur[TW];
           item_cur<TW>(m, L, W, q, cur);
-          cnt += dfs_count<TW>(m.B, W, cur, 3, a.k);
+          if (a.multi) {
+            mc[3] += 1;   // the item is one triangle
+            dfs_multi<TW>(m.B, W, cur, 3, a.k, mc);
+          } else {
+            cnt += dfs_count<TW>(m.B, W, cur, 3, a.k);
+          }
         }
     }
     total += cnt;
@@ -408,6 +464,7 @@ __global__ void __launch_bounds__(256) kcl_bitmap_kernel(BmArgs a) {
     atomicAdd(&a.ctrl[CTRL_ELEMS], (unsigned long long)elems);
     atomicAdd(&a.ctrl[CTRL_AUX0], (unsigned long long)entries);
   }
+  if (a.multi) flush_multi(mc, a, lane);
 }
 
 // Second launch for the deferred heavy roots: one CTA per (root, part); the part
@@ -420,6 +477,7 @@ __global__ void __launch_bounds__(256) kcl_bitmap_parts_kernel(BmArgs a) {
   const int tid = threadIdx.x;
   const TeamMem<TW> m(smem);
   uint64_t total = 0;
+  uint64_t mc[kMaxStack + 3] = {};
   for (;;) {
     if (tid == 0) {
       // the part list was filled by the previous launch; its length sits in ctrl
@@ -445,7 +503,12 @@ __global__ void __launch_bounds__(256) kcl_bitmap_parts_kernel(BmArgs a) {
     for (uint32_t q = part + tid * nparts; q < items; q += 256 * nparts) {
       uint32_t cur[TW];
       item_cur<TW>(m, L, W, q, cur);
-      cnt += dfs_count<TW>(m.B, W, cur, 3, a.k);
+      if (a.multi) {
+        mc[3] += 1;
+        dfs_multi<TW>(m.B, W, cur, 3, a.k, mc);
+      } else {
+        cnt += dfs_count<TW>(m.B, W, cur, 3, a.k);
+      }
     }
     total += cnt;
     if (PER_ROOT) {
@@ -458,6 +521,7 @@ __global__ void __launch_bounds__(256) kcl_bitmap_parts_kernel(BmArgs a) {
 #pragma unroll
   for (int off = 16; off > 0; off >>= 1) total += __shfl_down_sync(0xffffffffu, total, off);
   if (lane == 0 && total) atomicAdd(&a.ctrl[CTRL_COUNT], (unsigned long long)total);
+  if (a.multi) flush_multi(mc, a, lane);
 }
 
 template <int TEAM_WARPS, int TW>
@@ -516,7 +580,8 @@ void enqueue_parts(gamma_ctx *ctx, const BmArgs &a0, bool per_root) {
 // Count k-cliques rooted at roots[0..nroots) whose run length is <= 512 (k <= 12);
 // longer runs are left to the ET path.  per_root (nullable) indexed like roots.
 uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint64_t nroots,
-                        unsigned long long *per_root, bool sorted, uint64_t n_long, uint64_t n_mid) {
+                        unsigned long long *per_root, bool sorted, uint64_t n_long, uint64_t n_mid,
+                        uint64_t *multi_out) {
   gamma_ctx *ctx = g->ctx;
   BmArgs a{};
   a.dag_ptr = g->dag_ptr;
@@ -526,6 +591,7 @@ uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint6
   a.k = k;
   a.ctrl = (unsigned long long *)ctx->ctrl;
   a.per_root = per_root;
+  a.multi = multi_out != nullptr;
   // hub splitting only pays when the DFS below a triangle is deep (k >= 6)
   const bool split = k >= 6 && (ctx->desc.flags & GAMMA_FLAG_NO_SPLIT) == 0;
   DevBuf<uint2> parts;
@@ -572,6 +638,8 @@ uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint6
   ctx->stats.level_entries[2] += h[CTRL_AUX0];
   ctx->stats.alg_bytes[KC_BITMAP] += 4 * h[CTRL_AUX0] + 4 * h[CTRL_ELEMS];
   if (split) ctx->stats.chunks += std::min<uint64_t>(h[CTRL_AUX1], a.parts_cap);
+  if (multi_out)
+    for (uint32_t sz = 0; sz <= k && sz < 32; sz++) multi_out[sz] = sz >= 3 ? h[CTRL_MULTI + sz] : 0;
   return h[CTRL_COUNT];
 }
 

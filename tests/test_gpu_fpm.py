@@ -84,6 +84,20 @@ def test_pattern_table_growth(G, oracle_mod):
     assert g.fpm(3, 2) == oracle_set(o, 3, 2)
 
 
+@pytest.mark.parametrize("budget_kb", [120, 160])
+def test_domain_pool_chunks(G, oracle_mod, budget_kb):
+    """A budget too small for one level's MNI domains: the level is redone in chunks
+    of patterns that fit the pool (and the table grows too at 160 KB)."""
+    n, s, d, lab = gg.config_graph("c4", seed=1, scale=11)
+    lab = gg.labels(n, 5, 1)
+    c = G.Context(hbm_budget_bytes=budget_kb << 10)
+    g = c.load_edges(n, s, d, lab)
+    o = oracle_mod.Graph(n, s, d, lab)
+    assert g.fpm(2, 5) == oracle_set(o, 2, 5)
+    assert g.fpm(3, 20) == oracle_set(o, 3, 20)
+    assert c.stats()["chunks"] > 0
+
+
 def test_invalid(G, ctx):
     n, (s, d) = gg.complete(4)
     g = ctx.load_edges(n, s, d)

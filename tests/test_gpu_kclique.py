@@ -89,6 +89,11 @@ def test_complete_large_k(ctx):
     g = load(ctx, n, s, d)
     for k in (5, 8, 12, 20, 24, 25, 32):
         assert g.kclique(k) == comb(24, k)
+    # one bitmap pass for sizes 3..12; sizes beyond 12 fall back to per-k calls
+    ks = list(range(1, 13))
+    assert g.kclique_multi(ks) == [comb(24, k) for k in ks]
+    assert g.kclique_multi([3, 16, 24]) == [comb(24, 3), comb(24, 16), 1]
+    assert g.kclique_multi([]) == []
 
 
 @pytest.mark.parametrize("seed", [1, 2, 3, 4, 5])
@@ -160,6 +165,14 @@ def test_simulated_ranks_partition(G, oracle_mod):
             c = G.Context(rank=r, world=world, reduce=False)
             tot += c.load_edges(n, s, d).kclique(5)
         assert tot == want
+    # multi-k over the same partition
+    o = oracle_mod.Graph(n, s, d)
+    want = [o.kclique(k) for k in (3, 4, 5, 6)]
+    tot = [0] * 4
+    for r in range(3):
+        part = G.Context(rank=r, world=3, reduce=False).load_edges(n, s, d).kclique_multi([3, 4, 5, 6])
+        tot = [x + y for x, y in zip(tot, part)]
+    assert tot == want
 
 
 def test_load_csr_roundtrip_and_validation(G, ctx, oracle_mod):
@@ -228,6 +241,8 @@ def test_hub_out_list_longer_than_staging(ctx, oracle_mod, a):
     roots = np.array([0], np.uint32)
     for k in (3, 4):
         assert np.array_equal(g.kclique_roots(k, roots), o.kclique_roots(k, roots))
+    # max out-degree > 512 sends multi-k to per-k calls (ET path for the hub)
+    assert g.kclique_multi([3, 4, 5]) == [o.kclique(k) for k in (3, 4, 5)]
 
 
 @pytest.mark.parametrize("flags", [0, 0x10, 0x2 | 0x10, 0x20, 0x40])
@@ -240,8 +255,12 @@ def test_paths_agree(G, oracle_mod, flags):
     n, s, d, _ = gg.config_graph("c1", seed=4)
     g = c.load_edges(n, s, d)
     o = oracle_mod.Graph(n, s, d)
+    want = [o.kclique(k) for k in range(1, 9)]
     for k in (3, 4, 5, 6, 7):
-        assert g.kclique(k) == o.kclique(k), (flags, k)
+        assert g.kclique(k) == want[k - 1], (flags, k)
+    # every size from one multi-k pass (per-k calls under NO_BITMAP)
+    assert g.kclique_multi(list(range(1, 9))) == want, flags
+    assert g.kclique_multi([6, 4]) == [want[5], want[3]], flags
     roots = np.arange(0, n, 3, dtype=np.uint32)
     assert np.array_equal(g.kclique_roots(5, roots), o.kclique_roots(5, roots))
 
