@@ -28,6 +28,7 @@
 #include <cub/device/device_radix_sort.cuh>
 
 #include <algorithm>
+#include <chrono>
 #include <vector>
 
 #include "device_common.cuh"
@@ -700,8 +701,10 @@ extern "C" gamma_status gamma_fpm(gamma_graph *g, uint32_t max_edges, uint64_t m
     gamma_ctx *c = g->ctx;
     GAMMA_CUDA(cudaSetDevice(c->device));
     c->reset_stats();
+    const auto t0 = std::chrono::steady_clock::now();
     std::vector<gamma_fpm_pattern> pats;
     fpm_run(g, max_edges, minsup, pats);
+    c->stats.wall_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
     auto *r = new gamma_fpm_result();
     r->n = pats.size();
     r->pats = new gamma_fpm_pattern[pats.size() ? pats.size() : 1];

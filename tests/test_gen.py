@@ -43,3 +43,15 @@ def test_config_graph_small():
     n, s, d, lab = gg.config_graph("c3", scale=10)
     assert n == 1024 and lab is not None and lab.max() < 8
     assert s.size == int(43_500_000 * 2.0 ** (10 - 23))
+
+
+def test_torch_twin_matches_numpy():
+    """gamma_gen.torch_gen (used to draw C5 in device memory) reproduces the numpy
+    recipe element by element, across block boundaries and scales up to 31 bits."""
+    from gamma_gen.torch_gen import rmat_torch
+    for sc, ns, (a, b, c), seed in [(12, 9000, (0.57, 0.19, 0.19), 1), (26, 50_000, (0.55, 0.2, 0.2), 3),
+                                    (7, 1000, (0.4, 0.25, 0.25), 2), (31, 5000, (0.5, 0.2, 0.2), 4)]:
+        s, d = gg.rmat(sc, ns, a, b, c, seed)
+        ts, td = rmat_torch(sc, ns, a, b, c, seed, device="cpu", block=4096)
+        assert np.array_equal(s, ts.numpy().view(np.uint32)), sc
+        assert np.array_equal(d, td.numpy().view(np.uint32)), sc

@@ -84,7 +84,7 @@ def test_pattern_table_growth(G, oracle_mod):
     assert g.fpm(3, 2) == oracle_set(o, 3, 2)
 
 
-@pytest.mark.parametrize("budget_kb", [120, 160])
+@pytest.mark.parametrize("budget_kb", [100, 120])
 def test_domain_pool_chunks(G, oracle_mod, budget_kb):
     """A budget too small for one level's MNI domains: the level is redone in chunks
     of patterns that fit the pool (and the table grows too at 160 KB)."""

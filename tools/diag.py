@@ -23,10 +23,17 @@ def main():
         t = time.time()
         if what == "fpm_gpu":
             import paper_conf_icde_hu0o23_b200 as G
+            minsup = int(sys.argv[3]) if len(sys.argv) > 3 else 3
             c = G.Context(time_kernels=True)
             g = c.load_edges(n, s, d, lab)
-            r = g.fpm(3, 3)
-            print("gpu", len(r), time.time() - t, c.stats()["level_entries"][:4], c.stats()["retries"], flush=True)
+            for it in range(2):
+                t = time.time()
+                r = g.fpm(3, minsup)
+                st = c.stats()
+                print("gpu", len(r), f"{time.time() - t:.2f}s", st["level_entries"][:4], "retries", st["retries"],
+                      "chunks", st["chunks"], "wall_ms", round(st["wall_ms"]),
+                      {k: (v["launches"], round(v["ms"])) for k, v in st["classes"].items() if v["launches"]},
+                      flush=True)
         else:
             import oracle
             o = oracle.Graph(n, s, d, lab)
