@@ -39,7 +39,7 @@
 extern "C" {
 #endif
 
-#define GAMMA_ABI_VERSION 1
+#define GAMMA_ABI_VERSION 2
 
 typedef int32_t gamma_status;
 enum {
@@ -73,6 +73,13 @@ typedef struct {
   uint64_t hbm_budget_bytes; /* cap on embedding-table bytes; 0: 80% of free HBM     */
   uint64_t host_spill_bytes; /* pinned-host spill capacity for ET levels; 0: none    */
   uint32_t flags;            /* GAMMA_FLAG_* below                                   */
+  /* Optional collective used by gamma_fpm when world > 1 (together with
+     allreduce_sum_u64): all-to-all of DEVICE buffers.  Rank r's
+     send[g*n_per_rank .. (g+1)*n_per_rank) arrives in rank g's
+     recv[r*n_per_rank .. (r+1)*n_per_rank).  The library has synchronised its stream
+     before the call; the callback returns once recv is complete.  NULL: gamma_fpm
+     computes the whole result on every rank (replicas).                             */
+  gamma_status (*alltoall_u32)(const uint32_t *send, uint32_t *recv, uint64_t n_per_rank, void *user);
 } gamma_ctx_desc;
 
 #define GAMMA_FLAG_TIME_KERNELS 0x1u   /* record per-launch CUDA-event times (stats) */
@@ -190,7 +197,12 @@ typedef struct {
 /* All connected edge-induced patterns with 1..max_edges edges and MNI support >=
  * minsup (max_edges in [1,3] in v1; minsup >= 1; vertex labels < 4096, else
  * E_UNSUPPORTED).  Result owned by the library (free with gamma_fpm_result_free).
- * With world > 1 every rank computes the full result (replicas).   */
+ * With world > 1 and both collectives (allreduce_sum_u64, alltoall_u32) levels
+ * 1..max_edges-1 run on every rank and the last level is split over the ranks by
+ * root-edge batch; its MNI domain bitmaps are OR-reduced by an all-to-all of word
+ * shards plus a SUM all-reduce of per-shard popcounts, and every rank
+ * returns the same full result.  Without the collectives every rank computes the
+ * full result alone (replicas).                                                  */
 gamma_status gamma_fpm(gamma_graph *g, uint32_t max_edges, uint64_t minsup,
                        gamma_fpm_result **out);
 void gamma_fpm_result_free(gamma_fpm_result *r);

@@ -90,27 +90,71 @@ def pattern_plan(nv: int, edges, labels=None, induced: bool = False) -> dict:
             "greater_mask": [info.greater_mask[i] for i in range(nv)], "aut": int(info.aut)}
 
 
-def make_allreduce_callback(device: int = 0):
-    """The ctx's ``allreduce_sum_u64`` callback: an in-place SUM of n uint64 values
-    held in host memory, over the default torch.distributed process group (a CUDA
-    int64 tensor for NCCL, a CPU one for gloo).  Returns the ctypes function."""
+def allreduce_sum_inplace(arr: np.ndarray) -> None:
+    """SUM all-reduce of a host uint64 array over the default process group (a CUDA
+    int64 tensor for NCCL, a CPU one for gloo); wrapping int64 sums equal uint64 sums."""
     import torch
     import torch.distributed as dist
-    backend = dist.get_backend()
+    t = torch.from_numpy(arr.view(np.int64).copy())
+    if dist.get_backend() == "nccl":
+        t = t.cuda()
+    dist.all_reduce(t, op=dist.ReduceOp.SUM)
+    arr[:] = t.cpu().numpy().view(np.uint64)
+
+
+def alltoall_tensors(send, recv) -> None:
+    """all_to_all_single over the default group; gloo goes through host copies."""
+    import torch.distributed as dist
+    if dist.get_backend() == "nccl" or not send.is_cuda:
+        dist.all_to_all_single(recv, send)
+    else:
+        rc = send.new_empty(send.shape, device="cpu")
+        dist.all_to_all_single(rc, send.cpu())
+        recv.copy_(rc)
+
+
+def make_allreduce_callback(device: int = 0):
+    """The ctx's ``allreduce_sum_u64`` callback: an in-place SUM of n uint64 values
+    held in host memory.  Returns the ctypes function."""
 
     def _allreduce(buf, n, user):
         try:
-            vals = [buf[i] for i in range(n)]
-            dev = torch.device("cuda", device) if backend == "nccl" else torch.device("cpu")
-            t = torch.tensor(vals, dtype=torch.int64, device=dev)
-            dist.all_reduce(t, op=dist.ReduceOp.SUM)
-            for i, v in enumerate(t.cpu().tolist()):
-                buf[i] = v
+            if n:
+                allreduce_sum_inplace(np.ctypeslib.as_array(buf, shape=(n,)))
             return 0
         except Exception:   # noqa: BLE001 -- reported as a gamma_status
             return N.GAMMA_E_CUDA
 
     return N.ALLREDUCE_FN(_allreduce)
+
+
+class _DeviceView:
+    """Zero-copy int32 view of a library-owned device buffer (CUDA array interface)."""
+
+    def __init__(self, ptr: int, n: int):
+        self.__cuda_array_interface__ = {"shape": (int(n),), "typestr": "<i4", "data": (int(ptr), False),
+                                         "version": 3, "strides": None}
+
+
+def make_alltoall_callback(device: int = 0):
+    """The ctx's ``alltoall_u32`` callback (gamma_fpm's domain-bitmap exchange): device
+    buffers of world * n_per_rank words, exchanged with all_to_all_single."""
+    import torch
+    import torch.distributed as dist
+
+    def _alltoall(send, recv, n, user):
+        try:
+            total = dist.get_world_size() * int(n)
+            if total:
+                s = torch.as_tensor(_DeviceView(send, total), device=torch.device("cuda", device))
+                r = torch.as_tensor(_DeviceView(recv, total), device=torch.device("cuda", device))
+                alltoall_tensors(s, r)
+                torch.cuda.synchronize(device)
+            return 0
+        except Exception:   # noqa: BLE001 -- reported as a gamma_status
+            return N.GAMMA_E_CUDA
+
+    return N.ALLTOALL_FN(_alltoall)
 
 
 class Context:
@@ -162,6 +206,10 @@ class Context:
             fr = make_allreduce_callback(device)
             d.allreduce_sum_u64 = fr
             self._keep.append(fr)
+            if self._torch is not None and self._torch.cuda.is_available():
+                fa2a = make_alltoall_callback(device)
+                d.alltoall_u32 = fa2a
+                self._keep.append(fa2a)
         d.hbm_budget_bytes = hbm_budget_bytes
         d.host_spill_bytes = host_spill_bytes
         d.flags = flags | (N.GAMMA_FLAG_TIME_KERNELS if time_kernels else 0)
@@ -289,6 +337,11 @@ class Graph:
 
     def fpm(self, max_edges: int, minsup: int):
         """Frequent patterns: sorted list of (ne, nv, labels, edges, support)."""
+        t = self.ctx._torch
+        if t is not None and t.cuda.is_available():
+            # the MNI domain pool is sized from free HBM: give the caching allocator's
+            # idle blocks (e.g. the previous call's pool) back first
+            t.cuda.empty_cache()
         r = C.POINTER(N.gamma_fpm_result)()
         _check(_lib.gamma_fpm(self._h, int(max_edges), int(minsup), C.byref(r)), "gamma_fpm")
         try:

@@ -29,6 +29,7 @@ GAMMA_FLAG_DEBUG_SPLIT_ALL = 0x40
 ALLOC_FN = C.CFUNCTYPE(C.c_void_p, C.c_size_t, C.c_void_p, C.c_void_p)
 FREE_FN = C.CFUNCTYPE(None, C.c_void_p, C.c_void_p)
 ALLREDUCE_FN = C.CFUNCTYPE(C.c_int32, C.POINTER(C.c_uint64), C.c_size_t, C.c_void_p)
+ALLTOALL_FN = C.CFUNCTYPE(C.c_int32, C.c_void_p, C.c_void_p, C.c_uint64, C.c_void_p)
 
 
 class gamma_ctx_desc(C.Structure):
@@ -39,6 +40,7 @@ class gamma_ctx_desc(C.Structure):
         ("allreduce_sum_u64", ALLREDUCE_FN), ("coll_user", C.c_void_p),
         ("hbm_budget_bytes", C.c_uint64), ("host_spill_bytes", C.c_uint64),
         ("flags", C.c_uint32),
+        ("alltoall_u32", ALLTOALL_FN),
     ]
 
 

@@ -26,9 +26,11 @@
 //    index = rank of the vertex inside its class), so memory follows the patterns
 //    that occur.  Support = min over positions of popcount (one warp per slot).
 #include <cub/device/device_radix_sort.cuh>
+#include <cub/device/device_select.cuh>
 
 #include <algorithm>
 #include <chrono>
+#include <unordered_map>
 #include <vector>
 
 #include "device_common.cuh"
@@ -77,7 +79,8 @@ struct FpmArgs {
   const uint32_t *csize;     // label class sizes
   uint32_t n;
   uint32_t level;            // edges per recorded embedding
-  uint32_t rank, world;      // root partition
+  uint32_t rank, world;      // root partition: this rank takes edge batches b = rank (mod world)
+  uint32_t claim_only;       // claim pattern slots without carving domains (distributed level)
   Table T;
   unsigned long long *ctrl;
 };
@@ -121,14 +124,17 @@ __device__ int64_t table_slot(const FpmArgs &a, uint64_t key, bool insert) {
       if (k == 0) {
         // the claimer carves the slot's domains: one bitmap per position, sized to the
         // position's label class
-        const uint32_t nv = key_nv(key);
-        uint64_t words = 0;
-        for (uint32_t p = 0; p < nv; p++) words += (a.csize[key_label(key, p)] + 31) / 32;
-        const unsigned long long off = atomicAdd(T.pool_cur, (unsigned long long)words);
-        unsigned long long d = off + 1;
-        if (off + words > T.pool_words) {
-          atomicExch(&a.ctrl[CTRL_OVF], 1ull);
-          d = ~0ull;
+        unsigned long long d = ~0ull;
+        if (!a.claim_only) {
+          const uint32_t nv = key_nv(key);
+          uint64_t words = 0;
+          for (uint32_t p = 0; p < nv; p++) words += (a.csize[key_label(key, p)] + 31) / 32;
+          const unsigned long long off = atomicAdd(T.pool_cur, (unsigned long long)words);
+          d = off + 1;
+          if (off + words > T.pool_words) {
+            atomicExch(&a.ctrl[CTRL_OVF], 1ull);
+            d = ~0ull;
+          }
         }
         __threadfence();
         atomicExch(&T.dom[h], d);
@@ -280,9 +286,10 @@ __global__ void __launch_bounds__(kThreads) fpm_enum_kernel(FpmArgs a) {
   for (;;) {
     // work unit = a batch of root edges (not a root vertex: a hub's edges spread
     // over many warps)
-    unsigned long long i0 = 0;
-    if (lane == 0) i0 = atomicAdd(&a.ctrl[CTRL_WORK], kBatch);
-    i0 = __shfl_sync(0xffffffffu, i0, 0);
+    unsigned long long b = 0;
+    if (lane == 0) b = atomicAdd(&a.ctrl[CTRL_WORK], 1ull);
+    b = __shfl_sync(0xffffffffu, b, 0);
+    const uint64_t i0 = (b * a.world + a.rank) * kBatch;   // this rank's share of the batches
     if (i0 >= ndir) break;
     // u = row of directed edge i0 (binary search of row_ptr)
     uint32_t u;
@@ -299,7 +306,6 @@ __global__ void __launch_bounds__(kThreads) fpm_enum_kernel(FpmArgs a) {
       while (a.rp[u + 1] <= i1) u++;   // the batch may cross rows
       const uint32_t v = a.col[i1];
       if (v < u) continue;             // each undirected edge once, from its smaller end
-      if (a.world > 1 && (u % a.world) != a.rank) continue;
       const uint64_t us = a.rp[u], ue = a.rp[u + 1];
       const uint64_t e1 = ekey(u, v);
       if (a.level == 1) {
@@ -487,12 +493,226 @@ __global__ void max_label_kernel(const uint32_t *lab, uint32_t n, unsigned long 
   if ((threadIdx.x & 31) == 0) atomicMax(out, m);
 }
 
+// ---- distributed last level (world > 1) ----
+// this rank's pattern codes of one level, in any order
+__global__ void level_keys_kernel(const unsigned long long *key, uint64_t cap, uint32_t level,
+                                  unsigned long long *out, unsigned long long *cursor) {
+  for (uint64_t s = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; s < cap; s += (uint64_t)gridDim.x * blockDim.x) {
+    const unsigned long long k = key[s];
+    if (k && key_ne(k) == level) out[atomicAdd(cursor, 1ull)] = k;
+  }
+}
+
+// after the all-to-all, recv holds G shards of this rank's word range: OR them into
+// the first one
+__global__ void or_shards_kernel(uint32_t *recv, uint32_t G, uint64_t shard) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < shard; i += (uint64_t)gridDim.x * blockDim.x) {
+    uint32_t x = recv[i];
+    for (uint32_t g = 1; g < G; g++) x |= recv[g * shard + i];
+    recv[i] = x;
+  }
+}
+
+// popcount of the part of each domain bitmap (global word range [off, off + w)) that
+// lies in this rank's range [lo, lo + shard); one warp per bitmap
+__global__ void seg_popc_kernel(const uint32_t *buf, uint64_t lo, uint64_t shard, const uint64_t *seg_off,
+                                const uint32_t *seg_w, uint64_t nseg, unsigned long long *cnt) {
+  const int lane = threadIdx.x & 31;
+  const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  for (uint64_t q = warp; q < nseg; q += nwarps) {
+    const uint64_t b = seg_off[q] > lo ? seg_off[q] : lo;
+    const uint64_t e0 = seg_off[q] + seg_w[q], e1 = lo + shard;
+    const uint64_t e = e0 < e1 ? e0 : e1;
+    unsigned long long c = 0;
+    for (uint64_t x = b + lane; x < e; x += 32) c += __popc(buf[x - lo]);
+    for (int o = 16; o > 0; o >>= 1) c += __shfl_down_sync(0xffffffffu, c, o);
+    if (lane == 0) cnt[q] = c;
+  }
+}
+
 inline unsigned g1d(uint64_t n) {
   const uint64_t b = (n + 255) / 256;
   return (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(b, 148u * 32u));
 }
 
 }  // namespace
+
+static gamma_fpm_pattern decode_pattern(uint64_t key, uint64_t support) {
+  static const uint8_t pairs[6][2] = {{0, 1}, {0, 2}, {0, 3}, {1, 2}, {1, 3}, {2, 3}};
+  gamma_fpm_pattern p{};
+  p.nv = key_nv(key);
+  p.ne = key_ne(key);
+  const uint32_t ek = key_edges(key);
+  const uint32_t idx[3] = {ek / 64, (ek / 8) % 8, ek % 8};
+  for (uint32_t i = 0; i < p.nv; i++) p.labels[i] = key_label(key, i);
+  for (uint32_t e = 0; e < p.ne; e++) {
+    const uint32_t id = idx[e];   // sorted pair indices first, unused slots hold 7
+    p.edges[e][0] = pairs[id][0];
+    p.edges[e][1] = pairs[id][1];
+  }
+  p.support = support;
+  return p;
+}
+
+static void coll_allreduce(gamma_ctx *ctx, uint64_t *v, size_t n) {
+  const gamma_status st = ctx->desc.allreduce_sum_u64(v, n, ctx->desc.coll_user);
+  GAMMA_REQUIRE(st == GAMMA_OK, st, "allreduce_sum_u64 callback failed");
+}
+
+static void coll_alltoall(gamma_ctx *ctx, const uint32_t *send, uint32_t *recv, uint64_t n_per_rank) {
+  ctx->sync();   // the callback may run on another stream
+  const gamma_status st = ctx->desc.alltoall_u32(send, recv, n_per_rank, ctx->desc.coll_user);
+  GAMMA_REQUIRE(st == GAMMA_OK, st, "alltoall_u32 callback failed");
+}
+
+// The last level of a multi-GPU FPM run: every rank enumerates only its
+// share of the root-edge batches, so a pattern's MNI domains are spread over the
+// ranks and must be OR-ed.  1. claim pass: the rank's level-l pattern codes enter its
+// table (no domains); 2. the codes are all-to-all exchanged, sorted and deduplicated
+// into the same global list U on every rank; 3. U is cut into chunks whose domains fit
+// half the pool, laid out identically on every rank; per chunk each rank re-runs its
+// share of the enumeration recording into that layout, the bitmaps are all-to-all
+// exchanged in G shards (NCCL has no bitwise-OR reduction), each rank ORs the shards
+// of its word range and popcounts the pieces of every domain in it, and one SUM
+// all-reduce of those pieces gives every rank the same |domain| per (pattern,
+// position), hence the same supports and output.  Returns false when some rank's
+// table overflowed (all ranks then grow it and retry together).
+static bool fpm_dist_level(gamma_ctx *ctx, FpmArgs &a, int grid_enum, uint32_t l, uint64_t minsup,
+                           const std::vector<uint32_t> &hsize, uint64_t cap, unsigned long long *key_d,
+                           unsigned long long *dom_d, uint32_t *pool_d, uint64_t pool_words,
+                           unsigned long long *pcur_d, std::vector<gamma_fpm_pattern> &found) {
+  const uint32_t G = (uint32_t)ctx->desc.world, R = (uint32_t)ctx->desc.rank;
+  a.level = l;
+  a.rank = R;
+  a.world = G;
+  // ---- 1. claim pass ----
+  a.claim_only = 1;
+  ctrl_reset(ctx);
+  ctx->launch(KC_FPM, [&] { fpm_enum_kernel<<<grid_enum, kThreads, 0, ctx->stream>>>(a); });
+  a.claim_only = 0;
+  DevBuf<unsigned long long> mine(ctx, cap);
+  ctx->launch(KC_MISC, [&] {
+    level_keys_kernel<<<g1d(cap), 256, 0, ctx->stream>>>(key_d, cap, l, mine.p,
+                                                         (unsigned long long *)ctx->ctrl + CTRL_AUX0);
+  });
+  ctrl_fetch(ctx);
+  // agree on: table overflow anywhere, every rank's code count, the smallest pool,
+  // and the level's embedding count
+  std::vector<uint64_t> v(2 * G + 2, 0);
+  v[R] = ctx->ctrl_host[CTRL_AUX0];
+  v[G + R] = pool_words;
+  v[2 * G] = ctx->ctrl_host[CTRL_ERR] != 0;
+  v[2 * G + 1] = ctx->ctrl_host[CTRL_ENTRIES];
+  coll_allreduce(ctx, v.data(), v.size());
+  if (v[2 * G]) return false;
+  ctx->stats.level_entries[l] = v[2 * G + 1];
+  uint64_t maxc = 1, half = ~0ull;
+  for (uint32_t r = 0; r < G; r++) {
+    maxc = std::max<uint64_t>(maxc, v[r]);
+    half = std::min<uint64_t>(half, v[G + r] / 2);
+  }
+  const uint64_t nmine = v[R];
+  // ---- 2. global code list U ----
+  uint64_t nU = 0;
+  std::vector<unsigned long long> U;
+  {
+    DevBuf<unsigned long long> send(ctx, G * maxc), recv(ctx, G * maxc), sorted(ctx, G * maxc);
+    GAMMA_CUDA(cudaMemsetAsync(send.p, 0, G * maxc * 8, ctx->stream));
+    for (uint32_t r = 0; r < G; r++)
+      if (nmine)
+        GAMMA_CUDA(cudaMemcpyAsync(send.p + r * maxc, mine.p, nmine * 8, cudaMemcpyDeviceToDevice, ctx->stream));
+    coll_alltoall(ctx, (const uint32_t *)send.p, (uint32_t *)recv.p, 2 * maxc);
+    const uint64_t tot = G * maxc;
+    size_t t1 = 0, t2 = 0;
+    GAMMA_CUDA(cub::DeviceRadixSort::SortKeys(nullptr, t1, recv.p, sorted.p, tot, 0, 64, ctx->stream));
+    GAMMA_CUDA(cub::DeviceSelect::Unique(nullptr, t2, sorted.p, send.p, (unsigned long long *)ctx->ctrl + CTRL_AUX1,
+                                         tot, ctx->stream));
+    DevBuf<uint8_t> tmp(ctx, std::max(t1, t2));
+    ctx->launch(KC_MISC, [&] {
+      GAMMA_CUDA(cub::DeviceRadixSort::SortKeys(tmp.p, t1, recv.p, sorted.p, tot, 0, 64, ctx->stream));
+    });
+    ctx->cub_sort_launched(KC_MISC, tot, 64);
+    ctx->launch(KC_MISC, [&] {
+      GAMMA_CUDA(cub::DeviceSelect::Unique(tmp.p, t2, sorted.p, send.p, (unsigned long long *)ctx->ctrl + CTRL_AUX1,
+                                           tot, ctx->stream));
+    });
+    ctx->cub_select_launched(KC_MISC);
+    ctrl_fetch(ctx);
+    nU = ctx->ctrl_host[CTRL_AUX1];
+    U.resize(nU);
+    if (nU) GAMMA_CUDA(cudaMemcpyAsync(U.data(), send.p, nU * 8, cudaMemcpyDeviceToHost, ctx->stream));
+    ctx->sync();
+    if (nU && U[0] == 0) U.erase(U.begin());   // padding
+  }
+  // ---- 3. chunks of U ----
+  std::vector<unsigned long long> hkey(cap), hdom(cap);
+  GAMMA_CUDA(cudaMemcpyAsync(hkey.data(), key_d, cap * 8, cudaMemcpyDeviceToHost, ctx->stream));
+  ctx->sync();
+  std::unordered_map<uint64_t, uint64_t> slot_of;
+  slot_of.reserve(nmine * 2 + 1);
+  for (uint64_t s = 0; s < cap; s++)
+    if (hkey[s] && key_ne(hkey[s]) == l) slot_of.emplace(hkey[s], s);
+  uint32_t *dom_buf = pool_d, *recv_buf = pool_d + half;
+  std::vector<uint64_t> seg_off;
+  std::vector<uint32_t> seg_w;
+  size_t next = 0;
+  while (next < U.size()) {
+    std::fill(hdom.begin(), hdom.end(), ~0ull);
+    seg_off.clear();
+    seg_w.clear();
+    uint64_t used = 0;
+    const size_t j0 = next;
+    for (; next < U.size(); next++) {
+      const uint64_t k = U[next];
+      uint64_t words = 0;
+      for (uint32_t p = 0; p < key_nv(k); p++) words += (hsize[key_label(k, p)] + 31) / 32;
+      GAMMA_REQUIRE(words + G <= half, GAMMA_E_NOMEM, "gamma_fpm: one pattern's domains exceed the HBM budget");
+      if (used + words + G > half) break;
+      auto it = slot_of.find(k);
+      if (it != slot_of.end()) hdom[it->second] = 1 + used;
+      for (uint32_t p = 0; p < key_nv(k); p++) {
+        const uint32_t w = (hsize[key_label(k, p)] + 31) / 32;
+        seg_off.push_back(used);
+        seg_w.push_back(w);
+        used += w;
+      }
+    }
+    const size_t j1 = next;
+    const uint64_t shard = (used + G - 1) / G;
+    GAMMA_CUDA(cudaMemcpyAsync(dom_d, hdom.data(), cap * 8, cudaMemcpyHostToDevice, ctx->stream));
+    GAMMA_CUDA(cudaMemsetAsync(dom_buf, 0, shard * G * 4, ctx->stream));
+    GAMMA_CUDA(cudaMemcpyAsync(pcur_d, &pool_words, 8, cudaMemcpyHostToDevice, ctx->stream));
+    ctrl_reset(ctx);
+    ctx->launch(KC_FPM, [&] { fpm_enum_kernel<<<grid_enum, kThreads, 0, ctx->stream>>>(a); });
+    ctrl_fetch(ctx);
+    GAMMA_REQUIRE(ctx->ctrl_host[CTRL_ERR] == 0 && ctx->ctrl_host[CTRL_OVF] == 0, GAMMA_E_CUDA,
+                  "gamma_fpm: a distributed chunk pass met an unclaimed pattern");
+    coll_alltoall(ctx, dom_buf, recv_buf, shard);
+    const uint64_t nseg = seg_off.size();
+    DevBuf<uint64_t> soff = to_device(ctx, seg_off.data(), nseg);
+    DevBuf<uint32_t> sw = to_device(ctx, seg_w.data(), nseg);
+    DevBuf<unsigned long long> cnt(ctx, nseg);
+    ctx->launch(KC_FPM_SUPPORT, [&] { or_shards_kernel<<<g1d(shard), 256, 0, ctx->stream>>>(recv_buf, G, shard); });
+    ctx->launch(KC_FPM_SUPPORT, [&] {
+      seg_popc_kernel<<<g1d(nseg * 32), 256, 0, ctx->stream>>>(recv_buf, R * shard, shard, soff.p, sw.p, nseg, cnt.p);
+    });
+    std::vector<uint64_t> hc(nseg);
+    GAMMA_CUDA(cudaMemcpyAsync(hc.data(), cnt.p, nseg * 8, cudaMemcpyDeviceToHost, ctx->stream));
+    ctx->sync();
+    coll_allreduce(ctx, hc.data(), nseg);
+    size_t q = 0;
+    for (size_t j = j0; j < j1; j++) {
+      uint64_t sup = ~0ull;
+      for (uint32_t p = 0; p < key_nv(U[j]); p++, q++) sup = std::min<uint64_t>(sup, hc[q]);
+      if (sup >= minsup) found.push_back(decode_pattern(U[j], sup));
+    }
+    ctx->stats.chunks++;
+  }
+  a.rank = 0;
+  a.world = 1;
+  return true;
+}
 
 static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::vector<gamma_fpm_pattern> &out) {
   gamma_ctx *ctx = g->ctx;
@@ -558,7 +778,11 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
   a.csize = csize.p;
   a.n = n;
   a.rank = 0;
-  a.world = 1;   // FPM runs every root on every rank (replicas)
+  a.world = 1;   // levels < l run on every rank; the last one is split when dist
+  // multi-GPU: the last level is partitioned over the ranks and its domains OR-reduced
+  // (fpm_dist_level); without the collectives every rank computes everything
+  const bool dist = ctx->desc.world > 1 && ctx->desc.allreduce_sum_u64 && ctx->desc.alltoall_u32;
+  std::vector<gamma_fpm_pattern> found_last;
   a.ctrl = (unsigned long long *)ctx->ctrl;
   const int grid_enum = ctx->num_sms * occupancy_blocks((const void *)fpm_enum_kernel, kThreads, 0);
   for (int attempt = 0;; attempt++) {
@@ -579,7 +803,13 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
     GAMMA_CUDA(cudaMemsetAsync(pcur.p, 0, 8, ctx->stream));
     a.T = Table{key.p, sup.p, freq.p, dom.p, cap, pool.p, pool_words, pcur.p};
     bool full = false;
+    found_last.clear();
     for (uint32_t l = 1; l <= max_edges && !full; l++) {
+      if (dist && l == max_edges) {
+        full = !fpm_dist_level(ctx, a, grid_enum, l, minsup, hsize, cap, key.p, dom.p, pool.p, pool_words, pcur.p,
+                               found_last);
+        break;
+      }
       a.level = l;
       ctrl_reset(ctx);
       ctx->launch(KC_FPM, [&] { fpm_enum_kernel<<<grid_enum, kThreads, 0, ctx->stream>>>(a); });
@@ -590,6 +820,11 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
       GAMMA_CUDA(cudaMemcpyAsync(&carved, pcur.p, 8, cudaMemcpyDeviceToHost, ctx->stream));
       ctrl_fetch(ctx);
       full = ctx->ctrl_host[CTRL_ERR] != 0;
+      if (dist) {   // the ranks must agree on growing the table
+        uint64_t f = full;
+        coll_allreduce(ctx, &f, 1);
+        full = f != 0;
+      }
       if (full) break;
       ctx->stats.level_entries[l] = ctx->ctrl_host[CTRL_ENTRIES];
       // a level's domains are dead once its supports are known (the next level reads
@@ -657,23 +892,12 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
   GAMMA_CUDA(cudaMemcpyAsync(hkey.data(), key.p, cap * 8, cudaMemcpyDeviceToHost, ctx->stream));
   GAMMA_CUDA(cudaMemcpyAsync(hsup.data(), sup.p, cap * 8, cudaMemcpyDeviceToHost, ctx->stream));
   ctx->sync();
-  static const uint8_t pairs[6][2] = {{0, 1}, {0, 2}, {0, 3}, {1, 2}, {1, 3}, {2, 3}};
   for (uint64_t s = 0; s < cap; s++) {
     if (hkey[s] == 0 || !hfreq[s]) continue;
-    gamma_fpm_pattern p{};
-    p.nv = key_nv(hkey[s]);
-    p.ne = key_ne(hkey[s]);
-    const uint32_t ek = key_edges(hkey[s]);
-    const uint32_t idx[3] = {ek / 64, (ek / 8) % 8, ek % 8};
-    for (uint32_t i = 0; i < p.nv; i++) p.labels[i] = key_label(hkey[s], i);
-    for (uint32_t e = 0; e < p.ne; e++) {
-      const uint32_t id = idx[e];   // sorted pair indices first, unused slots hold 7
-      p.edges[e][0] = pairs[id][0];
-      p.edges[e][1] = pairs[id][1];
-    }
-    p.support = hsup[s];
-    out.push_back(p);
+    if (dist && key_ne(hkey[s]) == max_edges) continue;   // from found_last
+    out.push_back(decode_pattern(hkey[s], hsup[s]));
   }
+  out.insert(out.end(), found_last.begin(), found_last.end());
   std::sort(out.begin(), out.end(), [](const gamma_fpm_pattern &x, const gamma_fpm_pattern &y) {
     if (x.ne != y.ne) return x.ne < y.ne;
     if (x.nv != y.nv) return x.nv < y.nv;

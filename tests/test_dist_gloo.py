@@ -1,5 +1,6 @@
 """Multi-process host logic on CPU (gloo, world_size 2): the count all-reduce
-callback the C library calls for world > 1, and bench.py's max-over-ranks timing."""
+callback the C library calls for world > 1, the all-to-all behind gamma_fpm's
+domain-bitmap exchange, and bench.py's max-over-ranks timing."""
 import ctypes as C
 import os
 import socket
@@ -27,9 +28,15 @@ def _worker(rank, world, port, q):
         cb = G.make_allreduce_callback(0)
         buf = (C.c_uint64 * 3)(rank + 1, 10 * (rank + 1), 2 ** 40 + rank)
         st = cb(buf, 3, None)
+        big = (C.c_uint64 * 1)(2 ** 63 + 5)     # uint64 sums wrap like the library's
+        st2 = cb(big, 1, None)
+        # all-to-all layout of the FPM exchange: rank r's block g lands in rank g's block r
+        send = torch.arange(6, dtype=torch.int32) + 100 * rank
+        recv = torch.empty(6, dtype=torch.int32)
+        G.alltoall_tensors(send, recv)
         import bench
         t = bench.max_over_ranks(1.5 + rank, world)
-        q.put((rank, st, list(buf), t))
+        q.put((rank, st + st2, list(buf) + [big[0]], recv.tolist(), t))
     finally:
         dist.destroy_process_group()
 
@@ -46,7 +53,8 @@ def test_allreduce_callback_and_max_timing():
     for p in procs:
         p.join(timeout=60)
         assert p.exitcode == 0
-    for rank, st, buf, t in res:
+    for rank, st, buf, recv, t in res:
         assert st == 0
-        assert buf == [3, 30, 2 * 2 ** 40 + 1]
+        assert buf == [3, 30, 2 * 2 ** 40 + 1, 10]
+        assert recv == [3 * rank, 3 * rank + 1, 3 * rank + 2, 100 + 3 * rank, 101 + 3 * rank, 102 + 3 * rank]
         assert t == 2.5
