@@ -58,41 +58,103 @@ static void set_threads(int threads) {
  * ------------------------------------------------------------------------- */
 og_graph *og_build(uint32_t n, uint64_t m_raw, const uint32_t *src, const uint32_t *dst,
                    const uint32_t *labels) {
+  /* The same steps as the plain definition -- one key (min, max) per sample without
+   * self-loops, sort, drop duplicates, count degrees, fill and sort the lists -- with
+   * the sort done per bucket of the smaller endpoint's high bits so that threads can
+   * share it (a key's duplicates all fall in its own bucket).  Needed for C5 (~2e9
+   * samples); the result does not depend on the bucketing. */
   og_graph *g = (og_graph *)calloc(1, sizeof(og_graph));
   if (!g) return NULL;
   g->n = n;
+  int bad = 0;
+#pragma omp parallel for reduction(| : bad)
+  for (int64_t i = 0; i < (int64_t)m_raw; i++) bad |= (src[i] >= n || dst[i] >= n);
+  if (bad) { free(g); return NULL; }
+  int sh = 0;
+  while (((uint64_t)n >> sh) > 65536) sh++;
+  const uint64_t nb = ((uint64_t)n >> sh) + 1;
+  const int T = omp_get_max_threads();
+  uint64_t *hist = (uint64_t *)calloc((size_t)T * nb + 1, sizeof(uint64_t));
   uint64_t *key = (uint64_t *)malloc((m_raw ? m_raw : 1) * sizeof(uint64_t));
-  uint64_t k = 0;
-  for (uint64_t i = 0; i < m_raw; i++) {
-    uint32_t u = src[i], v = dst[i];
-    if (u >= n || v >= n) { free(key); free(g); return NULL; }
-    if (u == v) continue;                       /* no self-loops */
-    uint32_t a = u < v ? u : v, b = u < v ? v : u;
-    key[k++] = ((uint64_t)a << 32) | b;         /* one key per undirected edge */
+  uint64_t *bstart = (uint64_t *)calloc(nb + 1, sizeof(uint64_t));
+  uint64_t *bkeep = (uint64_t *)calloc(nb + 1, sizeof(uint64_t));
+  /* pass 1: per-thread bucket histograms (static schedule: same ranges in pass 2) */
+#pragma omp parallel num_threads(T)
+  {
+    uint64_t *h = hist + (size_t)omp_get_thread_num() * nb;
+#pragma omp for schedule(static)
+    for (int64_t i = 0; i < (int64_t)m_raw; i++) {
+      uint32_t u = src[i], v = dst[i];
+      if (u == v) continue;                     /* no self-loops */
+      h[(u < v ? u : v) >> sh]++;
+    }
   }
-  qsort(key, k, sizeof(uint64_t), cmp_u64);
+  /* bucket-major, thread-minor offsets */
+  uint64_t run = 0;
+  for (uint64_t b = 0; b < nb; b++) {
+    bstart[b] = run;
+    for (int t = 0; t < T; t++) {
+      uint64_t c = hist[(size_t)t * nb + b];
+      hist[(size_t)t * nb + b] = run;
+      run += c;
+    }
+  }
+  bstart[nb] = run;
+  /* pass 2: scatter one key per undirected edge sample into its bucket */
+#pragma omp parallel num_threads(T)
+  {
+    uint64_t *h = hist + (size_t)omp_get_thread_num() * nb;
+#pragma omp for schedule(static)
+    for (int64_t i = 0; i < (int64_t)m_raw; i++) {
+      uint32_t u = src[i], v = dst[i];
+      if (u == v) continue;
+      uint32_t a = u < v ? u : v, b = u < v ? v : u;
+      key[h[a >> sh]++] = ((uint64_t)a << 32) | b;
+    }
+  }
+  free(hist);
+  /* sort each bucket and drop duplicates in place */
+#pragma omp parallel for schedule(dynamic, 16)
+  for (int64_t b = 0; b < (int64_t)nb; b++) {
+    uint64_t *kb = key + bstart[b];
+    uint64_t len = bstart[b + 1] - bstart[b], w = 0;
+    qsort(kb, len, sizeof(uint64_t), cmp_u64);
+    for (uint64_t i = 0; i < len; i++)
+      if (i == 0 || kb[i] != kb[i - 1]) kb[w++] = kb[i];
+    bkeep[b] = w;
+  }
   uint64_t m = 0;
-  for (uint64_t i = 0; i < k; i++)              /* drop duplicates */
-    if (i == 0 || key[i] != key[i - 1]) key[m++] = key[i];
+  for (uint64_t b = 0; b < nb; b++) m += bkeep[b];
   g->m = m;
+  /* degrees */
   uint64_t *deg = (uint64_t *)calloc((size_t)n + 1, sizeof(uint64_t));
-  for (uint64_t i = 0; i < m; i++) { deg[key[i] >> 32]++; deg[key[i] & 0xffffffffu]++; }
+#pragma omp parallel for schedule(dynamic, 16)
+  for (int64_t b = 0; b < (int64_t)nb; b++)
+    for (uint64_t i = bstart[b]; i < bstart[b] + bkeep[b]; i++) {
+      __atomic_fetch_add(&deg[key[i] >> 32], 1, __ATOMIC_RELAXED);
+      __atomic_fetch_add(&deg[key[i] & 0xffffffffu], 1, __ATOMIC_RELAXED);
+    }
   g->off = (uint64_t *)malloc(((size_t)n + 1) * sizeof(uint64_t));
   g->off[0] = 0;
   for (uint32_t v = 0; v < n; v++) g->off[v + 1] = g->off[v] + deg[v];
   g->adj = (uint32_t *)malloc((m > 0 ? 2 * m : 1) * sizeof(uint32_t));
   for (uint32_t v = 0; v < n; v++) deg[v] = g->off[v];   /* reuse as fill cursor */
-  for (uint64_t i = 0; i < m; i++) {
-    uint32_t a = (uint32_t)(key[i] >> 32), b = (uint32_t)(key[i] & 0xffffffffu);
-    g->adj[deg[a]++] = b;
-    g->adj[deg[b]++] = a;
-  }
-  for (uint32_t v = 0; v < n; v++)
+#pragma omp parallel for schedule(dynamic, 16)
+  for (int64_t b = 0; b < (int64_t)nb; b++)
+    for (uint64_t i = bstart[b]; i < bstart[b] + bkeep[b]; i++) {
+      uint32_t a = (uint32_t)(key[i] >> 32), c = (uint32_t)(key[i] & 0xffffffffu);
+      g->adj[__atomic_fetch_add(&deg[a], 1, __ATOMIC_RELAXED)] = c;
+      g->adj[__atomic_fetch_add(&deg[c], 1, __ATOMIC_RELAXED)] = a;
+    }
+#pragma omp parallel for schedule(dynamic, 1024)
+  for (int64_t v = 0; v < (int64_t)n; v++)
     qsort(g->adj + g->off[v], g->off[v + 1] - g->off[v], sizeof(uint32_t), cmp_u32);
   g->lab = (uint32_t *)malloc(((size_t)n ? n : 1) * sizeof(uint32_t));
   for (uint32_t v = 0; v < n; v++) g->lab[v] = labels ? labels[v] : 0;
   free(deg);
   free(key);
+  free(bstart);
+  free(bkeep);
   return g;
 }
 
