@@ -224,13 +224,14 @@ void build_dag(gamma_graph *g, uint64_t *sorted_keys_dev, uint64_t nkeys);
 uint64_t kclique_count(gamma_graph *g, uint32_t k, const uint32_t *roots_dev, uint64_t nroots,
                        uint64_t *per_root_dev);
 // kCL local-bitmap path for roots with |N+(v)| <= kBitmapMaxRun (kclique_bitmap.cu)
-constexpr uint32_t kBitmapMaxRun = 512;
+constexpr uint32_t kBitmapMaxRun = 512;     // shared-memory rows up to here
+constexpr uint32_t kWideMaxRun = 8192;      // global-scratch rows ("wide") up to here
 constexpr uint32_t kBitmapMaxK = 12;
 uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint64_t nroots,
-                        unsigned long long *per_root, bool sorted, uint64_t n_long, uint64_t n_mid,
+                        unsigned long long *per_root, bool sorted, uint64_t n_xl, uint64_t n_long, uint64_t n_mid,
                         uint64_t *multi_out = nullptr);
 // One bitmap pass counting every clique size 3..kmax (multi_out[s], s <= kmax); false
-// when the graph needs the ET path (max out-degree > kBitmapMaxRun or kmax too big).
+// when the graph needs the ET path (max out-degree > kWideMaxRun or kmax too big).
 bool kclique_multi(gamma_graph *g, uint32_t kmax, uint64_t *multi_out);
 void ensure_root_order(gamma_graph *g);
 }  // namespace gamma_impl

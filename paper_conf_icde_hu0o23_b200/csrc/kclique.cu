@@ -795,15 +795,16 @@ uint64_t kclique_count(gamma_graph *g, uint32_t k, const uint32_t *roots_dev, ui
                                                        kThreads, kcl_smem(MODE_FUSED));
   const bool bitmap = (ctx->desc.flags & GAMMA_FLAG_NO_BITMAP) == 0 && k >= 3 && k <= kBitmapMaxK;
   if (bitmap && R.nroots) {
-    uint64_t n_long = 0, n_mid = 0;
+    uint64_t n_xl = 0, n_long = 0, n_mid = 0;
     if (!per_root) {
+      n_xl = kWideMaxRun + 1 < g->root_ge.size() ? g->root_ge[kWideMaxRun + 1] : 0;
       n_long = kBitmapMaxRun + 1 < g->root_ge.size() ? g->root_ge[kBitmapMaxRun + 1] : 0;
       n_mid = 129 < g->root_ge.size() ? g->root_ge[129] : 0;
     }
-    R.add_count(kclique_bitmap(g, k, R.roots, R.nroots, R.per_root_out, !per_root, n_long, n_mid));
-    R.root_len_gt = kBitmapMaxRun;
+    R.add_count(kclique_bitmap(g, k, R.roots, R.nroots, R.per_root_out, !per_root, n_xl, n_long, n_mid));
+    R.root_len_gt = kWideMaxRun;
   }
-  if (R.nroots && (!bitmap || g->max_out_degree > kBitmapMaxRun)) {
+  if (R.nroots && (!bitmap || g->max_out_degree > kWideMaxRun)) {
     size_t fr = 0, tot = 0;
     GAMMA_CUDA(cudaMemGetInfo(&fr, &tot));
     const uint64_t budget = ctx->desc.hbm_budget_bytes ? ctx->desc.hbm_budget_bytes : (uint64_t)(fr * 0.8);
@@ -819,7 +820,7 @@ uint64_t kclique_count(gamma_graph *g, uint32_t k, const uint32_t *roots_dev, ui
 bool kclique_multi(gamma_graph *g, uint32_t kmax, uint64_t *multi_out) {
   gamma_ctx *ctx = g->ctx;
   if ((ctx->desc.flags & GAMMA_FLAG_NO_BITMAP) || kmax < 3 || kmax > kBitmapMaxK ||
-      g->max_out_degree > kBitmapMaxRun)
+      g->max_out_degree > kWideMaxRun)
     return false;
   GAMMA_REQUIRE(g->m < 0xFFFFFFFFull, GAMMA_E_UNSUPPORTED, "DAG with >= 2^32 edges");
   ensure_root_order(g);
@@ -829,7 +830,7 @@ bool kclique_multi(gamma_graph *g, uint32_t kmax, uint64_t *multi_out) {
   if (nroots) {
     const uint64_t n_long = kBitmapMaxRun + 1 < g->root_ge.size() ? g->root_ge[kBitmapMaxRun + 1] : 0;
     const uint64_t n_mid = 129 < g->root_ge.size() ? g->root_ge[129] : 0;
-    kclique_bitmap(g, kmax, g->root_order, nroots, nullptr, true, n_long, n_mid, multi_out);
+    kclique_bitmap(g, kmax, g->root_order, nroots, nullptr, true, 0, n_long, n_mid, multi_out);
   }
   ctx->sync();
   ctx->collect_timings();

@@ -46,6 +46,8 @@ struct BmArgs {
   uint32_t parts_cap;
   uint64_t root_base;         // index of roots[0] in the full root list (parts are absolute)
   uint32_t multi;             // count every clique size 3..k at once (gamma_kclique_multi)
+  uint32_t *wide_rows;        // wide runs: per-CTA global row scratch (wide_stride words each)
+  uint64_t wide_stride;
 };
 
 __device__ __forceinline__ uint32_t excl_scan32(uint32_t x, int lane, uint32_t &total) {
@@ -207,30 +209,33 @@ struct TeamMem {
 // Depth-2 extension of root v: R = N+(v), rows B[i] = positions of R ∩ N+(R[i]).
 // Flattened windows of 32 children; each list element is located in R through a
 // shared-memory open-addressing position table.  Returns Σ|N+(c)| (for the bytes).
-template <int TEAM_WARPS, int TW>
-__device__ uint64_t build_rows(const BmArgs &a, const TeamMem<TW> &m, uint64_t b0, uint32_t L, int tid, int lane) {
+// R and H live in shared memory; B in shared memory (<= 512-long runs) or in a
+// global scratch slice (wide runs).
+template <int TEAM_WARPS>
+__device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H, uint32_t *B, uint64_t b0,
+                                 uint32_t L, int tid, int lane) {
   constexpr int kTeamThreads = TEAM_WARPS * 32;
   const int wit = tid >> 5;
   const uint32_t W = (L + 31) >> 5;
   uint32_t hbits = 2;
   while ((1u << hbits) < 4 * L) hbits++;
   const uint32_t hmask = (1u << hbits) - 1u;
-  for (uint32_t i = tid; i < L; i += kTeamThreads) m.R[i] = a.dag_col[b0 + i];
-  for (uint32_t i = tid; i < L * W; i += kTeamThreads) m.B[i] = 0u;
-  for (uint32_t i = tid; i <= hmask / 2; i += kTeamThreads) reinterpret_cast<uint32_t *>(m.H)[i] = 0u;
+  for (uint32_t i = tid; i < L; i += kTeamThreads) R[i] = a.dag_col[b0 + i];
+  for (uint32_t i = tid; i < L * W; i += kTeamThreads) B[i] = 0u;
+  for (uint32_t i = tid; i <= hmask / 2; i += kTeamThreads) reinterpret_cast<uint32_t *>(H)[i] = 0u;
   team_sync<TEAM_WARPS>();
   for (uint32_t i = tid; i < L; i += kTeamThreads) {
-    uint32_t h = (m.R[i] * 0x9E3779B1u) >> (32 - hbits);
-    while (atomicCAS(&m.H[h], (unsigned short)0, (unsigned short)(i + 1)) != 0) h = (h + 1) & hmask;
+    uint32_t h = (R[i] * 0x9E3779B1u) >> (32 - hbits);
+    while (atomicCAS(&H[h], (unsigned short)0, (unsigned short)(i + 1)) != 0) h = (h + 1) & hmask;
   }
   team_sync<TEAM_WARPS>();
-  const uint32_t rmin = m.R[0], rmax = m.R[L - 1];
+  const uint32_t rmin = R[0], rmax = R[L - 1];
   uint64_t elems = 0;
   for (uint32_t w0 = wit * 32; w0 < L; w0 += TEAM_WARPS * 32) {
     const uint32_t i = w0 + lane;
     uint32_t beg = 0, dl = 0;
     if (i < L) {
-      const uint32_t c = m.R[i];
+      const uint32_t c = R[i];
       const uint64_t cb = a.dag_ptr[c];
       dl = (uint32_t)(a.dag_ptr[c + 1] - cb);
       beg = (uint32_t)cb;
@@ -265,10 +270,10 @@ __device__ uint64_t build_rows(const BmArgs &a, const TeamMem<TW> &m, uint64_t b
         if (y >= rmin && y <= rmax) {
           uint32_t h = (y * 0x9E3779B1u) >> (32 - hbits);
           for (;;) {
-            const uint32_t e = m.H[h];
+            const uint32_t e = H[h];
             if (e == 0) break;
-            if (m.R[e - 1] == y) {
-              atomicOr(&m.B[rj * W + ((e - 1) >> 5)], 1u << ((e - 1) & 31));
+            if (R[e - 1] == y) {
+              atomicOr(&B[rj * W + ((e - 1) >> 5)], 1u << ((e - 1) & 31));
               break;
             }
             h = (h + 1) & hmask;
@@ -277,8 +282,14 @@ __device__ uint64_t build_rows(const BmArgs &a, const TeamMem<TW> &m, uint64_t b
       }
     }
   }
-  team_sync<TEAM_WARPS>();
+  team_sync<TEAM_WARPS>();   // (a CTA barrier also orders the global-memory rows)
   return elems;
+}
+
+template <int TEAM_WARPS, int TW>
+__device__ __forceinline__ uint64_t build_rows(const BmArgs &a, const TeamMem<TW> &m, uint64_t b0, uint32_t L,
+                                               int tid, int lane) {
+  return build_rows_p<TEAM_WARPS>(a, m.R, m.H, m.B, b0, L, tid, lane);
 }
 
 // P[r] = exclusive scan of the row popcounts (the triangle items), P[L] = total.
@@ -524,6 +535,182 @@ __global__ void __launch_bounds__(256) kcl_bitmap_parts_kernel(BmArgs a) {
   if (a.multi) flush_multi(mc, a, lane);
 }
 
+// ---- wide runs (kBitmapMaxRun < |R| <= kWideMaxRun): one CTA per root ------------
+// The rows (|R| x W words, W <= 32 WL) do not fit shared memory: they go to the CTA's
+// slice of a global scratch (L2-resident for the run of one root), R and the position
+// hash stay in shared memory.  A warp takes one row i at a time (candidates of the
+// edge (v, R[i])) and walks the DFS below it with every candidate bitmap spread over
+// its lanes (lane l holds words l, l+32, ...): the next candidate is found with one
+// ballot per word slice, the AND with a row is a coalesced 128-byte load per slice,
+// and every lane accumulates the popcounts of its own words.
+constexpr int kWideThreads = 512;
+
+template <int WL>
+__device__ __forceinline__ int wide_pop_next(uint32_t (&rem)[WL], int lane) {
+#pragma unroll
+  for (int t = 0; t < WL; t++) {
+    const uint32_t bal = __ballot_sync(0xffffffffu, rem[t] != 0u);
+    if (bal) {
+      const int l = __ffs(bal) - 1;
+      const uint32_t w = __shfl_sync(0xffffffffu, rem[t], l);
+      if (lane == l) rem[t] &= rem[t] - 1u;
+      return (l + 32 * t) * 32 + __ffs(w) - 1;
+    }
+  }
+  return -1;
+}
+
+// DFS below the candidates `cur` of a clique of `chosen` vertices (lane-distributed);
+// returns this lane's share of the k-clique count (multi: adds to mc per size).
+template <int WL>
+__device__ uint64_t wide_dfs(const uint32_t *B, uint32_t W, const uint32_t (&cur0)[WL], uint32_t chosen,
+                             uint32_t k, bool multi, uint64_t (&mc)[kMaxStack + 3], int lane) {
+  uint32_t cur[kMaxStack][WL], rem[kMaxStack][WL];
+#pragma unroll
+  for (int t = 0; t < WL; t++) cur[0][t] = rem[0][t] = cur0[t];
+  uint64_t cnt = 0;
+  int s = 0;
+  while (s >= 0) {
+    uint32_t r[WL];
+#pragma unroll
+    for (int t = 0; t < WL; t++) r[t] = rem[s][t];
+    const int j = wide_pop_next<WL>(r, lane);
+#pragma unroll
+    for (int t = 0; t < WL; t++) rem[s][t] = r[t];
+    if (j < 0) {
+      s--;
+      continue;
+    }
+    const uint32_t tk = chosen + s + 1;   // vertices chosen after taking j
+    uint32_t nx[WL];
+    uint32_t c = 0;
+#pragma unroll
+    for (int t = 0; t < WL; t++) {
+      const uint32_t w = lane + 32 * t;
+      nx[t] = w < W ? (cur[s][t] & B[(uint64_t)j * W + w]) : 0u;
+      c += __popc(nx[t]);
+    }
+    if (multi) mc[tk + 1] += c;
+    if (tk + 1 >= k) {
+      cnt += c;
+      continue;
+    }
+    // prune: fewer candidates than vertices still missing (single-k only)
+    if (!multi && __reduce_add_sync(0xffffffffu, c) < k - tk - 1) continue;
+    if (multi && __reduce_add_sync(0xffffffffu, c) == 0) continue;
+    s++;
+#pragma unroll
+    for (int t = 0; t < WL; t++) cur[s][t] = rem[s][t] = nx[t];
+  }
+  return cnt;
+}
+
+template <int WL, bool PER_ROOT>
+__global__ void __launch_bounds__(kWideThreads) kcl_wide_kernel(BmArgs a) {
+  extern __shared__ uint32_t smem[];
+  constexpr int kMaxL = 1024 * WL;
+  uint32_t *R = smem;                                                   // kMaxL
+  unsigned short *H = reinterpret_cast<unsigned short *>(smem + kMaxL); // 4 kMaxL u16
+  uint32_t *slot = smem + kMaxL + 2 * kMaxL;                            // 4 words
+  uint32_t *B = a.wide_rows + (uint64_t)blockIdx.x * a.wide_stride;
+  const int tid = threadIdx.x, lane = tid & 31;
+  uint64_t total = 0, elems = 0, entries = 0;
+  uint64_t mc[kMaxStack + 3] = {};
+  for (;;) {
+    if (tid == 0) {
+      const unsigned long long w = atomicAdd(&a.ctrl[CTRL_WORK], 1ull);
+      slot[0] = w < a.nroots ? (uint32_t)w : 0xffffffffu;
+      slot[1] = 0;   // row cursor
+    }
+    __syncthreads();
+    const uint32_t gi = slot[0];
+    if (gi == 0xffffffffu) break;
+    const uint32_t v = a.roots[gi];
+    const uint64_t b0 = a.dag_ptr[v];
+    const uint32_t L = (uint32_t)(a.dag_ptr[v + 1] - b0);
+    if (L <= a.len_lo || L > a.len_hi || L < (a.multi ? 2u : a.k - 1)) {
+      __syncthreads();
+      continue;
+    }
+    const uint32_t W = (L + 31) >> 5;
+    if (tid == 0) entries += L;
+    elems += build_rows_p<kWideThreads / 32>(a, R, H, B, b0, L, tid, lane);
+    uint64_t cnt = 0;
+    for (;;) {
+      uint32_t i = 0;
+      if (lane == 0) i = atomicAdd(&slot[1], 1u);
+      i = __shfl_sync(0xffffffffu, i, 0);
+      if (i >= L) break;
+      uint32_t cur[WL];
+      uint32_t c = 0;
+#pragma unroll
+      for (int t = 0; t < WL; t++) {
+        const uint32_t w = lane + 32 * t;
+        cur[t] = w < W ? B[(uint64_t)i * W + w] : 0u;
+        c += __popc(cur[t]);
+      }
+      if (a.multi) mc[3] += c;
+      if (a.k == 3) {
+        cnt += c;
+        continue;
+      }
+      if (__reduce_add_sync(0xffffffffu, c) == 0) continue;
+      cnt += wide_dfs<WL>(B, W, cur, 2, a.k, a.multi != 0, mc, lane);
+    }
+    total += cnt;
+    if (PER_ROOT) {
+#pragma unroll
+      for (int off = 16; off > 0; off >>= 1) cnt += __shfl_down_sync(0xffffffffu, cnt, off);
+      if (lane == 0 && cnt) atomicAdd(&a.per_root[gi], (unsigned long long)cnt);
+    }
+    __syncthreads();   // R, H, B and the slots are rewritten by the next root
+  }
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) {
+    total += __shfl_down_sync(0xffffffffu, total, off);
+    elems += __shfl_down_sync(0xffffffffu, elems, off);
+    entries += __shfl_down_sync(0xffffffffu, entries, off);
+  }
+  if (lane == 0) {
+    if (total) atomicAdd(&a.ctrl[CTRL_COUNT], (unsigned long long)total);
+    atomicAdd(&a.ctrl[CTRL_ELEMS], (unsigned long long)elems);
+    atomicAdd(&a.ctrl[CTRL_AUX0], (unsigned long long)entries);
+  }
+  if (a.multi) flush_multi(mc, a, lane);
+}
+
+template <int WL>
+constexpr size_t wide_smem() {
+  return (size_t)(1024 * WL + 2 * 1024 * WL + 4) * sizeof(uint32_t);
+}
+
+// rows scratch: grid x (run length x words) for the longest run of the launch
+template <int WL>
+void enqueue_wide(gamma_ctx *ctx, BmArgs a, bool per_root, uint32_t max_len, DevBuf<uint32_t> &rows) {
+  static bool attr = false;
+  if (!attr) {
+    GAMMA_CUDA(cudaFuncSetAttribute(kcl_wide_kernel<WL, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                    (int)wide_smem<WL>()));
+    GAMMA_CUDA(cudaFuncSetAttribute(kcl_wide_kernel<WL, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                    (int)wide_smem<WL>()));
+    attr = true;
+  }
+  static int grid = 0;
+  if (!grid) grid = ctx->num_sms * occupancy_blocks((const void *)kcl_wide_kernel<WL, false>, kWideThreads, wide_smem<WL>());
+  const uint64_t L = std::min<uint64_t>(max_len, 1024u * WL);
+  a.wide_stride = L * ((L + 31) / 32);
+  const uint64_t g = std::min<uint64_t>(grid, a.nroots);
+  rows = DevBuf<uint32_t>(ctx, g * a.wide_stride);
+  a.wide_rows = rows.p;
+  GAMMA_CUDA(cudaMemsetAsync(ctx->ctrl + CTRL_WORK, 0, sizeof(uint64_t), ctx->stream));
+  ctx->launch(KC_BITMAP, [&] {
+    if (per_root)
+      kcl_wide_kernel<WL, true><<<(unsigned)g, kWideThreads, wide_smem<WL>(), ctx->stream>>>(a);
+    else
+      kcl_wide_kernel<WL, false><<<(unsigned)g, kWideThreads, wide_smem<WL>(), ctx->stream>>>(a);
+  });
+}
+
 template <int TEAM_WARPS, int TW>
 constexpr size_t bm_smem() {
   return (size_t)(256 / (TEAM_WARPS * 32)) * team_words<TW>() * sizeof(uint32_t);
@@ -577,10 +764,12 @@ void enqueue_parts(gamma_ctx *ctx, const BmArgs &a0, bool per_root) {
 
 }  // namespace
 
-// Count k-cliques rooted at roots[0..nroots) whose run length is <= 512 (k <= 12);
-// longer runs are left to the ET path.  per_root (nullable) indexed like roots.
+// Count k-cliques rooted at roots[0..nroots) whose run length is <= kWideMaxRun
+// (k <= 12); longer runs are left to the ET path.  per_root (nullable) indexed like
+// roots.  Sorted roots (d+ descending): [0, n_xl) ET path, [n_xl, n_long) wide CTA,
+// [n_long, n_mid) CTA teams, [n_mid, nroots) warp teams.
 uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint64_t nroots,
-                        unsigned long long *per_root, bool sorted, uint64_t n_long, uint64_t n_mid,
+                        unsigned long long *per_root, bool sorted, uint64_t n_xl, uint64_t n_long, uint64_t n_mid,
                         uint64_t *multi_out) {
   gamma_ctx *ctx = g->ctx;
   BmArgs a{};
@@ -605,10 +794,27 @@ uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint6
   // path, [n_long, n_mid) CTA teams, [n_mid, nroots) warp teams; each team kind runs
   // on its own range.  Unsorted (per-root mode) roots: every launch filters the list.
   if (sorted) {
+    n_xl = std::min(n_xl, nroots);
     n_long = std::min(n_long, nroots);
     n_mid = std::min(n_mid, nroots);
   }
   ctrl_reset(ctx);
+  // wide runs, [n_xl, n_long): 512 < |R| <= 2048 with 2 words per lane, longer with 8
+  DevBuf<uint32_t> rows_a, rows_b;
+  if (g->max_out_degree > kBitmapMaxRun && (!sorted || n_long > n_xl)) {
+    a.roots = roots + (sorted ? n_xl : 0);
+    a.nroots = sorted ? n_long - n_xl : nroots;
+    if (g->max_out_degree > 2048) {
+      a.len_lo = 2048;
+      a.len_hi = kWideMaxRun;
+      enqueue_wide<8>(ctx, a, per_root != nullptr, g->max_out_degree, rows_a);
+    }
+    a.len_lo = kBitmapMaxRun;
+    a.len_hi = 2048;
+    enqueue_wide<2>(ctx, a, per_root != nullptr, std::min<uint32_t>(g->max_out_degree, 2048), rows_b);
+    a.roots = roots;
+    a.nroots = nroots;
+  }
   a.len_lo = 128;
   a.len_hi = 512;
   if (g->max_out_degree > 128 && (!sorted || n_mid > n_long)) {

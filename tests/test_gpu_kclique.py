@@ -222,11 +222,12 @@ def test_unstaged_long_run_path(G, oracle_mod):
             assert g.kclique(k) == o.kclique(k)
 
 
-@pytest.mark.parametrize("a", [200, 1100])
-def test_hub_out_list_longer_than_staging(ctx, oracle_mod, a):
+@pytest.mark.parametrize("a", [200, 1100, 2500])
+def test_hub_out_list_longer_than_staging(G, ctx, oracle_mod, a):
     """A real vertex with a long DAG out-list: v joined to the a vertices of one side
     of K_{a,a+1} (those outrank v), plus a sprinkle of edges among them.  a=200
-    takes the CTA-team bitmap path, a=1100 the ET path with an unstaged run."""
+    takes the CTA-team bitmap path, a=1100 the wide path with 2 words per lane,
+    a=2500 the wide path with 8 words per lane."""
     b = a + 1
     U = np.arange(1, 1 + a)
     F = np.arange(1 + a, 1 + a + b)
@@ -239,10 +240,33 @@ def test_hub_out_list_longer_than_staging(ctx, oracle_mod, a):
     assert g.info()["max_out_degree"] >= a
     o = oracle_mod.Graph(n, e[:, 0].copy(), e[:, 1].copy())
     roots = np.array([0], np.uint32)
-    for k in (3, 4):
+    for k in (3, 4, 5):
         assert np.array_equal(g.kclique_roots(k, roots), o.kclique_roots(k, roots))
-    # max out-degree > 512 sends multi-k to per-k calls (ET path for the hub)
-    assert g.kclique_multi([3, 4, 5]) == [o.kclique(k) for k in (3, 4, 5)]
+    want = [o.kclique(k) for k in (3, 4, 5)]
+    assert [g.kclique(k) for k in (3, 4, 5)] == want
+    assert g.kclique_multi([3, 4, 5]) == want
+    # the same counts through the ET path
+    c = G.Context(flags=0x10)
+    assert [c.load_edges(n, e[:, 0].copy(), e[:, 1].copy()).kclique(k) for k in (3, 4)] == want[:2]
+
+
+def test_wide_runs_closed_forms(ctx):
+    """K_n puts a run of length n-1-i under root i: every path (warp, CTA, wide with 2
+    and 8 words per lane, and the ET path past 8192) against C(n, k)."""
+    def kn(n):
+        s, d = np.triu_indices(n, 1)
+        return n, (s.astype(np.uint32), d.astype(np.uint32))
+
+    n, (s, d) = kn(2600)
+    g = load(ctx, n, s, d)
+    assert g.info()["max_out_degree"] == 2599
+    assert g.kclique_multi([3, 4]) == [comb(2600, 3), comb(2600, 4)]
+    roots = np.array([0, 1, 100, 600, 1000, 2000, 2400, 2599], np.uint32)
+    assert list(g.kclique_roots(4, roots)) == [comb(2599 - int(i), 3) for i in roots]
+    assert list(g.kclique_roots(5, roots[3:])) == [comb(2599 - int(i), 4) for i in roots[3:]]
+    n, (s, d) = kn(8194)   # root 0 has d+ = 8193 > 8192: ET path
+    g = load(ctx, n, s, d)
+    assert g.kclique(3) == comb(8194, 3)
 
 
 @pytest.mark.parametrize("flags", [0, 0x10, 0x2 | 0x10, 0x20, 0x40])
