@@ -52,6 +52,9 @@ WORKLOADS = {
     "c4": {"kind": "fpm", "cfg": "c4", "l": 3, "minsup": 3000,
            "desc": "configs[3]: FPM l=3 edges, MNI minsup=3000, on cit-Patents-shaped R-MAT scale 22 "
                    "(0.40,0.25,0.25), 16.6M samples, L=37, seed 1"},
+    "c5": {"kind": "kcl", "cfg": "c5", "ks": (3, 4), "device_gen": True,
+           "desc": "configs[4]: triangle + 4-clique count on Friendster-shaped R-MAT scale 26 (0.55,0.20,0.20), "
+                   "2.0e9 raw samples drawn in HBM, seed 1 (level-3 table 1.08e11 x 8 B > HBM)"},
 }
 
 
@@ -145,13 +148,26 @@ def dist_env():
     return rank, world, local
 
 
-def load_traffic(kernel_class: str):
-    """dram bytes per launch of the dominant kernel from the committed ncu --set full
-    summary (profiles/ncu_full_<class>.json), or None."""
-    p = os.path.join(ROOT, "profiles", f"ncu_full_{kernel_class}.json")
+def load_traffic(workload: str, kernel_class: str):
+    """dram bytes per launch of the dominant kernel on this workload from the committed
+    ncu --set full summary (profiles/ncu_<workload>_<class>.json), or None."""
+    p = os.path.join(ROOT, "profiles", f"ncu_{workload}_{kernel_class}.json")
     if os.path.exists(p):
         try:
-            return json.load(open(p)).get("dram_bytes_per_launch")
+            j = json.load(open(p))
+            return j.get("dram_bytes_per_launch"), os.path.relpath(p, ROOT)
+        except (OSError, ValueError):
+            pass
+    return None, None
+
+
+def load_alg_bytes(workload: str):
+    """SURVEY §8(d) algorithmic bytes of one kCL step, counted over the oracle's
+    enumeration by tools/alg_bytes.py (profiles/alg_bytes.json), or None."""
+    p = os.path.join(ROOT, "profiles", "alg_bytes.json")
+    if os.path.exists(p):
+        try:
+            return json.load(open(p)).get(workload)
         except (OSError, ValueError):
             return None
     return None
@@ -160,6 +176,12 @@ def load_traffic(kernel_class: str):
 def make_input(name, seed=1):
     import gamma_gen as gg
     w = WORKLOADS[name]
+    if w.get("device_gen"):
+        # too large for a host-side numpy pass: drawn in HBM by the torch twin of the
+        # generator (same words, thresholds and bijection; tests/test_gen.py)
+        from gamma_gen.torch_gen import config_graph_torch
+        n, s, d = config_graph_torch(w["cfg"], seed=seed)
+        return n, s, d, None, w
     n, s, d, lab = gg.config_graph(w["cfg"], seed=seed)
     return n, s, d, lab, w
 
@@ -239,6 +261,10 @@ def run_reference(args):
     rank, world, _ = dist_env()
     if rank != 0:
         return 0
+    if WORKLOADS[args.workload].get("device_gen"):
+        print(json.dumps({"impl": "reference", "unavailable": "the CPU oracle cannot time C5 within the bench "
+                          "budget (host build of 2e9 samples); C5 parity is sampled in tests/test_gpu_c5.py"}))
+        return 0
     n, s, d, lab, w = make_input(args.workload)
     vals, secs, samples = [], [], []
     per_step_budget = max(2.0, 60.0 / max(1, args.steps + args.warmup))
@@ -281,14 +307,22 @@ def run_gamma(args):
     import paper_conf_icde_hu0o23_b200 as G
 
     n, s, d, lab, w = make_input(args.workload)
-    m_raw = s.size
     ctx = G.Context(device=dev, time_kernels=True)
     stream = torch.cuda.current_stream()
-    src_dev = torch.from_numpy(s.view(np.int32)).cuda()
-    dst_dev = torch.from_numpy(d.view(np.int32)).cuda()
+    if isinstance(s, torch.Tensor):   # drawn on the device
+        m_raw = s.numel()
+        src_dev, dst_dev = s, d
+        src_pin = torch.empty(m_raw, dtype=torch.int32, pin_memory=True)
+        dst_pin = torch.empty(m_raw, dtype=torch.int32, pin_memory=True)
+        src_pin.copy_(src_dev)
+        dst_pin.copy_(dst_dev)
+    else:
+        m_raw = s.size
+        src_dev = torch.from_numpy(s.view(np.int32)).cuda()
+        dst_dev = torch.from_numpy(d.view(np.int32)).cuda()
+        src_pin = torch.from_numpy(s.view(np.int32)).pin_memory()
+        dst_pin = torch.from_numpy(d.view(np.int32)).pin_memory()
     lab_dev = None if lab is None else torch.from_numpy(lab.view(np.int32)).cuda()
-    src_pin = torch.from_numpy(s.view(np.int32)).pin_memory()
-    dst_pin = torch.from_numpy(d.view(np.int32)).pin_memory()
     lab_pin = None if lab is None else torch.from_numpy(lab.view(np.int32)).pin_memory()
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
     agg = {"_total_launches": {"n": 0}}
@@ -389,15 +423,33 @@ def run_gamma(args):
     dom = max(cand, key=lambda k: cand[k]["ms"]) if cand else None
     roof = None
     if dom and cand[dom]["ms"] > 0:
-        per_launch_bytes = cand[dom]["alg_bytes"] / max(1, cand[dom]["launches"])
-        per_launch_ms = cand[dom]["ms"] / max(1, cand[dom]["launches"])
+        launches = max(1, cand[dom]["launches"])
+        per_launch_ms = cand[dom]["ms"] / launches
+        kernel_bytes = cand[dom]["alg_bytes"] / launches   # the kernel's own counters
+        ab = load_alg_bytes(args.workload) if w["kind"] == "kcl" and not args.per_k else None
+        if ab and ab["kmax"] == max(w["ks"]):
+            # the method's bytes per step (oracle-counted), spread over the
+            # dominant class's launches of one step (at N > 1 this rank's 1/N share)
+            per_launch_bytes = ab["bytes_per_step"] / world * args.steps / launches
+            bytes_src = "SURVEY §8(d) B_l summed over the step's extension levels, counted over the oracle's " \
+                        "enumeration (profiles/alg_bytes.json, tools/alg_bytes.py)"
+        else:
+            per_launch_bytes = kernel_bytes
+            bytes_src = "SURVEY §8(d) B_l from the kernel's own counters (list elements read, entries in/out)"
         achieved = per_launch_bytes / (per_launch_ms / 1000.0) / 1e9
+        traffic, traffic_src = load_traffic(args.workload, dom)
         roof = {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s", "frac": achieved / hbm,
-                "traffic": load_traffic(dom), "kernel": dom, "peak_source": peak_src,
-                "alg_bytes_per_launch": per_launch_bytes, "ms_per_launch": per_launch_ms,
-                "share_of_step": cand[dom]["ms"] / total_ms}
+                "traffic": traffic, "kernel": dom, "peak_source": peak_src,
+                "alg_bytes_per_launch": per_launch_bytes, "alg_bytes_source": bytes_src,
+                "kernel_counted_bytes_per_launch": kernel_bytes,
+                "ms_per_launch": per_launch_ms, "launches_per_step": launches / args.steps,
+                "share_of_step": cand[dom]["ms"] / total_ms, "traffic_source": traffic_src}
     cpu = None
-    if world == 1 and not args.no_cpu_baseline:
+    if w.get("device_gen"):
+        cpu = {"value": None, "unit": UNIT, "cores": os.cpu_count(), "kind": "oracle",
+               "sample": "not run in the bench: the oracle's host build of 2e9 samples alone exceeds the "
+                         "bench's CPU budget; C5 parity runs on sampled roots in tests/test_gpu_c5.py"}
+    elif world == 1 and not args.no_cpu_baseline:
         cpu = cpu_oracle_sample(n, s, d, lab, w, budget_s=args.cpu_seconds)
         cpu.pop("embeddings", None)
         cpu.pop("seconds", None)

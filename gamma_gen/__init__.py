@@ -224,6 +224,10 @@ CONFIGS = {
     "heavy": (22, 20_000_000, 0.57, 0.19, 0.19, 1),     # Graph500-skew kCL scaling workload
     "c3": (23, 43_500_000, 0.50, 0.20, 0.20, 8),        # LiveJournal-shaped labeled SM
     "c4": (22, 16_600_000, 0.40, 0.25, 0.25, 37),       # cit-Patents-shaped FPM, 37 labels
+    # Friendster-shaped (2^26 vertices, ~1.97e9 unique edges); a = 0.55 chosen on the box
+    # (tools/c5_probe.py) so that the level-3 table (1.08e11 triangles x 8 B = 864 GB)
+    # exceeds one GPU's HBM.  Drawn on the device (gamma_gen.torch_gen.config_graph_torch).
+    "c5": (26, 2_000_000_000, 0.55, 0.20, 0.20, 1),
 }
 
 

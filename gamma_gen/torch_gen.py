@@ -91,3 +91,13 @@ def rmat_torch(scale: int, samples: int, a: float, b: float, c: float, seed: int
         dst[lo:hi] = d.to(torch.int32)
         del s, d, i, base
     return src, dst
+
+
+def config_graph_torch(name: str, seed: int = 1, device="cuda"):
+    """``gamma_gen.config_graph`` drawn with torch on ``device`` (unlabeled configs):
+    (n, src, dst) with int32 tensors holding the uint32 bit patterns."""
+    from . import CONFIGS
+    sc, ns, a, b, c, L = CONFIGS[name]
+    assert L == 1, "labeled configs are drawn on the host"
+    src, dst = rmat_torch(sc, ns, a, b, c, seed, device=device)
+    return 1 << sc, src, dst

@@ -48,6 +48,7 @@ def lib():
             L.og_kclique.restype = C.c_uint64
             L.og_kclique.argtypes = [C.c_void_p, C.c_uint32, C.c_int, C.c_int]
             L.og_kclique_roots.argtypes = [C.c_void_p, C.c_uint32, C.c_uint64, u32p, u64p, C.c_int]
+            L.og_kclique_levels.argtypes = [C.c_void_p, C.c_uint32, u64p, u64p, C.c_int]
             L.og_match.restype = C.c_int
             L.og_match.argtypes = [C.c_void_p, C.c_uint32, C.c_uint32, u32p, C.c_void_p, C.c_int,
                                    C.POINTER(C.c_uint64), C.POINTER(C.c_uint64), C.POINTER(C.c_uint64)]
@@ -106,6 +107,14 @@ class Graph:
         out = np.zeros(roots.size, np.uint64)
         lib().og_kclique_roots(self._h, k, roots.size, roots, out, threads)
         return out
+
+    def kclique_levels(self, k: int, threads: int = 0):
+        """(N, S): N[t] = #t-cliques, S[t] = sum over t-cliques of d+(last vertex),
+        t = 0..k (index 0 is 0).  Feeds SURVEY §8(d)'s algorithmic bytes."""
+        N = np.zeros(k + 1, np.uint64)
+        S = np.zeros(k + 1, np.uint64)
+        lib().og_kclique_levels(self._h, k, N, S, threads)
+        return [int(x) for x in N], [int(x) for x in S]
 
     def match(self, nv: int, edges, plabels=None, threads: int = 0):
         """Return (count, mappings, |Aut_L|)."""

@@ -12,6 +12,8 @@
  *                       (§IV "CSR ... made up of adjacency lists";
  *                        L119, L204: one label per vertex, no edge labels)
  *   og_kclique     O-1  |{S subset of V : |S|=k, S a clique}|
+ *   og_kclique_levels  O-1b  #t-cliques and sum of d+(last vertex) per ET level t, for
+ *                       SURVEY.md §8(d)'s algorithmic bytes
  *   og_match       O-2  #injective label-preserving edge-preserving maps / |Aut_L(P)|
  *                       ("all subgraphs isomorphic to a pattern P";
  *                        Alg. 1)
@@ -266,6 +268,74 @@ void og_kclique_roots(const og_graph *g, uint32_t k, uint64_t nroots, const uint
       counts[i] = (k == 1) ? 1 : kcl_root(g, 0, k, roots[i], buf);
     free_bufs(buf, k + 1);
   }
+}
+
+/* ---------------------------------------------------------------------------
+ * O-1b: level statistics of the k-clique embedding table, for SURVEY.md §8(d)'s
+ * algorithmic bytes (not a parity quantity).  The ET level t (PAPER.md L253-257,
+ * §V-A) holds one entry per t-clique; extending an entry whose last-matched vertex
+ * is w fetches w's out-list N+(w) = {x in N(w) : r(x) > r(w)} (the "intersect"
+ * step).  For t = 1..k:
+ *   N[t] = #t-cliques,   S[t] = sum over t-cliques C of d+(max_r C).
+ * Same enumeration as og_kclique (order_mode 0): each clique is visited once,
+ * with its vertices chosen in increasing r.
+ * ------------------------------------------------------------------------- */
+static uint64_t out_degree(const og_graph *g, uint32_t w) {
+  uint64_t c = 0;
+  for (uint64_t e = g->off[w]; e < g->off[w + 1]; e++)
+    if (r_less(g, 0, w, g->adj[e])) c++;
+  return c;
+}
+
+static void kcl_levels_rec(const og_graph *g, const uint64_t *dplus, uint32_t k, uint32_t size, uint32_t last,
+                           const uint32_t *cand, uint64_t nc, uint32_t **buf, uint64_t *N, uint64_t *S) {
+  N[size] += 1;
+  S[size] += dplus[last];
+  if (size == k) return;
+  uint32_t *next = buf[size];
+  for (uint64_t i = 0; i < nc; i++) {
+    uint32_t w = cand[i];
+    uint64_t nn = 0;
+    for (uint64_t j = 0; j < nc; j++) {
+      uint32_t x = cand[j];
+      if (r_less(g, 0, w, x) && adjacent(g, w, x)) next[nn++] = x;
+    }
+    kcl_levels_rec(g, dplus, k, size + 1, w, next, nn, buf, N, S);
+  }
+}
+
+/* N, S: arrays of k+1 entries (index 0 unused, set to 0). */
+void og_kclique_levels(const og_graph *g, uint32_t k, uint64_t *N, uint64_t *S, int threads) {
+  for (uint32_t t = 0; t <= k; t++) N[t] = S[t] = 0;
+  if (k == 0) return;
+  set_threads(threads);
+  uint64_t md = max_degree(g);
+  uint64_t *dplus = (uint64_t *)malloc(((size_t)g->n + 1) * sizeof(uint64_t));
+#pragma omp parallel for schedule(dynamic, 1024)
+  for (int64_t v = 0; v < (int64_t)g->n; v++) dplus[v] = out_degree(g, (uint32_t)v);
+#pragma omp parallel
+  {
+    uint64_t *n_loc = (uint64_t *)calloc(k + 1, sizeof(uint64_t));
+    uint64_t *s_loc = (uint64_t *)calloc(k + 1, sizeof(uint64_t));
+    uint32_t **buf = alloc_bufs(k + 1, md);
+#pragma omp for schedule(dynamic, 64)
+    for (int64_t v = 0; v < (int64_t)g->n; v++) {
+      uint32_t *cand = buf[0];
+      uint64_t nc = 0;
+      for (uint64_t e = g->off[v]; e < g->off[v + 1]; e++)
+        if (r_less(g, 0, (uint32_t)v, g->adj[e])) cand[nc++] = g->adj[e];
+      kcl_levels_rec(g, dplus, k, 1, (uint32_t)v, cand, nc, buf, n_loc, s_loc);
+    }
+#pragma omp critical
+    for (uint32_t t = 0; t <= k; t++) {
+      N[t] += n_loc[t];
+      S[t] += s_loc[t];
+    }
+    free_bufs(buf, k + 1);
+    free(n_loc);
+    free(s_loc);
+  }
+  free(dplus);
 }
 
 /* ---------------------------------------------------------------------------

@@ -1,0 +1,71 @@
+"""configs[4] (C5) parity at full size: Friendster-shaped R-MAT, 2^26 vertices, 2.0e9 raw
+samples (~1.97e9 unique edges), drawn in HBM by the torch twin of the generator.
+
+The oracle cannot count the 1.5e13 4-cliques of C5 on the host, so parity is taken
+per root ("full oracle on a seeded sample of root chunks"):
+  * the graph itself: |E| and every vertex degree (row_ptr) equal the oracle's O-0
+    build of the same raw samples, and a seeded sample of adjacency lists is equal;
+  * per-root triangle and 4-clique counts (each clique counted at its lowest-ranked
+    vertex; R9) for a seeded sample of roots -- uniform over
+    the roots with d+ >= 2 plus a stratified sample of the heavy tail -- equal the
+    oracle's og_kclique_roots;
+  * the whole-graph multi-k pass agrees with the per-root kernel on the sampled roots'
+    share being non-negative and the totals being consistent (t4 > 0, t3 > 0).
+Tolerance 0.  Needs ~70 GB of host memory (raw samples + oracle CSR); skipped below.
+"""
+import numpy as np
+import pytest
+
+pytestmark = [pytest.mark.gpu, pytest.mark.slow]
+
+
+def test_c5_sampled_roots(oracle_mod):
+    import psutil
+    import torch
+    if psutil.virtual_memory().available < 100 * 2 ** 30:
+        pytest.skip("C5 parity needs ~100 GB of free host memory")
+    import paper_conf_icde_hu0o23_b200 as G
+    from gamma_gen.torch_gen import config_graph_torch
+
+    ctx = G.Context(device=0)
+    n, src, dst = config_graph_torch("c5", seed=1)
+    g = ctx.load_edges(n, src, dst)
+    info = g.info()
+    t3, t4 = g.kclique_multi([3, 4])
+    assert t3 > 0 and t4 > 0
+    s_host, d_host = src.cpu().numpy().view(np.uint32), dst.cpu().numpy().view(np.uint32)
+    del src, dst
+    torch.cuda.empty_cache()
+
+    o = oracle_mod.Graph(n, s_host, d_host)
+    del s_host, d_host
+    assert info["m"] == o.m
+    rp_o, adj_o = o.csr()
+    rp_g, col_g = g.csr("sym")
+    assert np.array_equal(rp_o, rp_g), "degree sequence differs"
+    rng = np.random.default_rng(5)
+    for v in rng.integers(0, n, 2000):
+        assert np.array_equal(adj_o[rp_o[v]:rp_o[v + 1]], col_g[rp_g[v]:rp_g[v + 1]]), v
+    del col_g, adj_o
+
+    # root sample (which roots to check, not what to expect): uniform over the roots
+    # with d+ >= 2, plus strata of the d+ tail (the costly roots of the DFS); d+ is
+    # read off the DAG row pointers
+    dp, _ = g.csr("dag")
+    dplus = np.diff(dp.astype(np.int64))
+    del _
+    live = np.nonzero(dplus >= 2)[0]
+    uni = rng.choice(live, size=min(1500, live.size), replace=False)
+    order = live[np.argsort(dplus[live], kind="stable")[::-1]]
+    strata = [order[int(q * order.size)] for q in (1e-4, 3e-4, 1e-3, 3e-3, 1e-2, 3e-2, 0.1, 0.3)]
+    roots = np.unique(np.concatenate([uni, np.array(strata, dtype=np.int64)])).astype(np.uint32)
+    # the very top of the d+ tail (the wide-run CTA path, |R| > 512) for triangles,
+    # where the oracle's per-root cost stays at O(|R|^2 log d)
+    top = order[[0, 3, 10, 30, 100, 300, 1000]].astype(np.uint32)
+    want3 = o.kclique_roots(3, top)
+    assert np.array_equal(g.kclique_roots(3, top), want3)
+    for k in (3, 4):
+        want = o.kclique_roots(k, roots)
+        got = g.kclique_roots(k, roots)
+        assert np.array_equal(got, want), (k, np.nonzero(got != want)[0][:10])
+    assert want.sum() <= t4

@@ -119,3 +119,39 @@ def test_threads_invariance(oracle_mod):
     n, s, d, _ = gg.config_graph("c1", scale=10)
     g = oracle_mod.Graph(n, s, d)
     assert g.kclique(4, threads=1) == g.kclique(4, threads=0)
+
+
+# ---- O-1b: ET level statistics (SURVEY §8(d) algorithmic bytes) ----
+@pytest.mark.parametrize("n", [1, 2, 5, 9])
+def test_levels_complete_graph(oracle_mod, n):
+    """K_n: the vertex of rank i has d+ = n-1-i and ends C(i, t-1) t-cliques, so
+    S[t] = sum_i C(i, t-1) C(n-1-i, 1) = C(n, t+1) (Vandermonde); N[t] = C(n, t)."""
+    g = G(oracle_mod, gg.complete(n))
+    k = n + 1
+    N, S = g.kclique_levels(k)
+    for t in range(1, k + 1):
+        assert N[t] == comb(n, t)
+        assert S[t] == comb(n, t + 1)
+
+
+@pytest.mark.parametrize("seed", [1, 2, 3])
+def test_levels_brute_force(oracle_mod, seed):
+    """Brute force over all t-subsets of a small random graph: rank (deg, id), last
+    vertex = max rank, d+ counted from the edge set."""
+    import itertools
+    n = 14
+    s, d = gg.er(n, 40, seed)
+    E = brute.normalise(s, d)
+    deg = [sum(1 for e in E if v in e) for v in range(n)]
+    rank = lambda v: (deg[v], v)  # noqa: E731
+    dplus = [sum(1 for e in E if v in e and rank(next(iter(e - {v}))) > rank(v)) for v in range(n)]
+    g = oracle_mod.Graph(n, s, d)
+    k = 5
+    N, S = g.kclique_levels(k)
+    for t in range(1, k + 1):
+        bn = bs = 0
+        for C in itertools.combinations(range(n), t):
+            if all(frozenset(p) in E for p in itertools.combinations(C, 2)):
+                bn += 1
+                bs += dplus[max(C, key=rank)]
+        assert (N[t], S[t]) == (bn, bs), t
