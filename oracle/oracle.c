@@ -292,6 +292,11 @@ static void kcl_levels_rec(const og_graph *g, const uint64_t *dplus, uint32_t k,
   N[size] += 1;
   S[size] += dplus[last];
   if (size == k) return;
+  if (size + 1 == k) {   /* every candidate ends one k-clique: no need to descend */
+    N[k] += nc;
+    for (uint64_t i = 0; i < nc; i++) S[k] += dplus[cand[i]];
+    return;
+  }
   uint32_t *next = buf[size];
   for (uint64_t i = 0; i < nc; i++) {
     uint32_t w = cand[i];

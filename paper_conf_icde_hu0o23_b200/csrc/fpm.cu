@@ -29,6 +29,7 @@
 #include <cub/device/device_select.cuh>
 
 #include <algorithm>
+#include <array>
 #include <chrono>
 #include <unordered_map>
 #include <vector>
@@ -42,24 +43,30 @@ namespace {
 
 constexpr int kThreads = 256;
 
-__constant__ uint8_t c_perm4[24][4] = {
-    {0, 1, 2, 3}, {0, 1, 3, 2}, {0, 2, 1, 3}, {0, 2, 3, 1}, {0, 3, 1, 2}, {0, 3, 2, 1},
-    {1, 0, 2, 3}, {1, 0, 3, 2}, {1, 2, 0, 3}, {1, 2, 3, 0}, {1, 3, 0, 2}, {1, 3, 2, 0},
-    {2, 0, 1, 3}, {2, 0, 3, 1}, {2, 1, 0, 3}, {2, 1, 3, 0}, {2, 3, 0, 1}, {2, 3, 1, 0},
-    {3, 0, 1, 2}, {3, 0, 2, 1}, {3, 1, 0, 2}, {3, 1, 2, 0}, {3, 2, 0, 1}, {3, 2, 1, 0}};
-
 // Pattern code packed in one word (0 = empty slot):
 //   bits 0..47 four 12-bit labels (canonical order), 48..50 nv, 51..52 ne,
 //   53..61 sorted edge-pair key, 63 always set.
 constexpr uint64_t kKeyTag = 1ull << 63;
 
+// Positions p < q of a <= 4-vertex pattern index its 6 vertex pairs as
+// (0,1)(0,2)(0,3)(1,2)(1,3)(2,3) -> 0..5; kPid holds that index (15 on the diagonal)
+// in 4-bit fields at 4(4p+q).  kPairA/kPairB: the endpoints of pair i, 2 bits each.
+constexpr uint64_t kPid = 0xf5425f3143f0210full;
+constexpr uint32_t kPairA = 0u | 0u << 2 | 0u << 4 | 1u << 6 | 1u << 8 | 2u << 10;
+constexpr uint32_t kPairB = 1u | 2u << 2 | 3u << 4 | 2u << 6 | 3u << 8 | 3u << 10;
+constexpr int kCanonEntries = 512;   // (sorted-position edge mask M: 6 bits) x (tie mask: 3 bits)
+
+__host__ __device__ __forceinline__ uint32_t pid(uint32_t p, uint32_t q) {
+  return (uint32_t)(kPid >> (4 * (4 * p + q))) & 15u;
+}
+
 struct Table {
-  unsigned long long *key;   // 0 = empty; claimed with one atomicCAS
+  unsigned long long *slots;  // 2 words per slot: key (0 = empty; claimed with one atomicCAS)
+                              // and dom = 1 + pool offset of its domains (0: being carved, ~0: no room)
   unsigned long long *support;
-  uint32_t *freq;            // 1 if support >= minsup (set after the slot's level)
-  unsigned long long *dom;   // 1 + pool offset of the slot's domains (0: being carved, ~0: no room)
-  uint64_t cap;              // power of two
-  uint32_t *pool;            // per-slot domains, one bitmap per position over its label class
+  uint32_t *freq;             // 1 if support >= minsup (set after the slot's level)
+  uint64_t cap;               // power of two
+  uint32_t *pool;             // per-slot domains, one bitmap per position over its label class
   uint64_t pool_words;
   unsigned long long *pool_cur;
 };
@@ -76,7 +83,9 @@ struct FpmArgs {
   const uint32_t *col;
   const uint32_t *lab;       // nullable
   const uint32_t *lrank;     // rank of v inside its label class
-  const uint32_t *csize;     // label class sizes
+  const uint32_t *cwords;    // words of one domain bitmap of each label class
+  const uint2 *canon_tab;    // kCanonEntries: {best edge key, minimizing sigma set}
+  const uint32_t *perm_tab;  // 24 rows: sigma[c] in bits 2c..2c+1 (c_perm order)
   uint32_t n;
   uint32_t level;            // edges per recorded embedding
   uint32_t rank, world;      // root partition: this rank takes edge batches b = rank (mod world)
@@ -85,7 +94,7 @@ struct FpmArgs {
   unsigned long long *ctrl;
 };
 
-__device__ __forceinline__ uint32_t labof(const FpmArgs &a, uint32_t v) { return a.lab ? a.lab[v] : 0u; }
+__device__ __forceinline__ uint32_t labof(const FpmArgs &a, uint32_t v) { return a.lab ? __ldg(a.lab + v) : 0u; }
 
 __device__ __forceinline__ uint64_t ekey(uint32_t x, uint32_t y) {
   const uint32_t lo = x < y ? x : y, hi = x < y ? y : x;
@@ -106,21 +115,25 @@ __device__ __forceinline__ uint64_t mix64(uint64_t x) {
   return x;
 }
 
-// Lookup (insert = false) or lookup-or-insert a pattern code; returns slot or -1.
-// Lock-free: a slot is claimed by one atomicCAS of its key word; the claimer then
-// carves the slot's domains from the pool (record() waits for that with nanosleep).
-__device__ int64_t table_slot(const FpmArgs &a, uint64_t key, bool insert) {
+// Lookup (insert = false) or lookup-or-insert a pattern code; returns the slot (or -1)
+// and its dom word.  Lock-free: a slot is claimed by one atomicCAS of its key word; the
+// claimer then carves the slot's domains from the pool (dom stays 0 until then).  Key
+// and dom share 16 bytes, read with one L1-bypassing vector load.
+__device__ int64_t table_slot(const FpmArgs &a, uint64_t key, bool insert, unsigned long long &dom) {
   const Table &T = a.T;
   uint64_t h = mix64(key) & (T.cap - 1);
   // a long probe chain means the table is (nearly) full: report it and let the host
   // grow the table instead of degrading to a linear scan
   const uint64_t max_probe = T.cap < 4096 ? T.cap : 4096;
   for (uint64_t probe = 0; probe < max_probe; probe++, h = (h + 1) & (T.cap - 1)) {
-    unsigned long long k = *(volatile unsigned long long *)&T.key[h];
-    if (k == key) return (int64_t)h;
-    if (k == 0) {
+    const ulonglong2 kd = __ldcg(reinterpret_cast<const ulonglong2 *>(T.slots) + h);
+    if (kd.x == key) {
+      dom = kd.y;
+      return (int64_t)h;
+    }
+    if (kd.x == 0) {
       if (!insert) return -1;
-      k = atomicCAS(&T.key[h], 0ull, (unsigned long long)key);
+      const unsigned long long k = atomicCAS(&T.slots[2 * h], 0ull, (unsigned long long)key);
       if (k == 0) {
         // the claimer carves the slot's domains: one bitmap per position, sized to the
         // position's label class
@@ -128,7 +141,7 @@ __device__ int64_t table_slot(const FpmArgs &a, uint64_t key, bool insert) {
         if (!a.claim_only) {
           const uint32_t nv = key_nv(key);
           uint64_t words = 0;
-          for (uint32_t p = 0; p < nv; p++) words += (a.csize[key_label(key, p)] + 31) / 32;
+          for (uint32_t p = 0; p < nv; p++) words += __ldg(a.cwords + key_label(key, p));
           const unsigned long long off = atomicAdd(T.pool_cur, (unsigned long long)words);
           d = off + 1;
           if (off + words > T.pool_words) {
@@ -137,150 +150,140 @@ __device__ int64_t table_slot(const FpmArgs &a, uint64_t key, bool insert) {
           }
         }
         __threadfence();
-        atomicExch(&T.dom[h], d);
+        atomicExch(&T.slots[2 * h + 1], d);
+        dom = d;
         return (int64_t)h;
       }
-      if (k == key) return (int64_t)h;
+      if (k == key) {
+        dom = __ldcg(&T.slots[2 * h + 1]);
+        return (int64_t)h;
+      }
     }
   }
   if (insert) atomicExch(&a.ctrl[CTRL_ERR], 1ull);   // table full
   return -1;
 }
 
-// Canonical code of a connected edge set on nv <= 4 local vertices (W) with ne <= 3
-// edges (local index pairs E).  Returns the packed key and the minimizing vertex orders
-// as a bitmask over c_perm4 rows.
+// Canonical code (reading R7: min over vertex orders of (labels in order, sorted
+// edge-pair list)) of a connected edge set on nv <= 4 local vertices with labels
+// l0..l3 and local edge mask em (bit pid(a, b) per edge).  The minimal label sequence
+// is the sorted labels, so the minimizing orders are (stable label sort) o sigma with
+// sigma permuting positions of equal labels only; which sigmas minimise the edge list
+// depends only on the edge mask in sorted positions and on which neighbouring sorted
+// labels are equal -- a 512-entry table (canon_tab, built on the host by enumerating
+// the 24 sigmas, fpm_canon_tables).  ordw: local index at sorted position s in bits 2s.
 struct Canon {
   uint64_t key;
-  uint32_t minmask;
+  uint32_t minmask;   // minimizing sigmas (rows of perm_tab)
+  uint32_t ordw;
 };
 
-__device__ Canon canonical(const FpmArgs &a, const uint32_t *W, uint32_t nv, const uint8_t (*E)[2], uint32_t ne) {
-  Canon cn;
-  uint32_t lw[4];
-  for (uint32_t i = 0; i < 4; i++) lw[i] = i < nv ? labof(a, W[i]) : 0xffffffffu;
-  // minimal label sequence = sorted labels
-  uint32_t ls[4] = {lw[0], lw[1], lw[2], lw[3]};
-  for (int i = 1; i < 4; i++)
-    for (int j = i; j > 0 && ls[j - 1] > ls[j]; j--) {
-      const uint32_t t = ls[j - 1];
-      ls[j - 1] = ls[j];
-      ls[j] = t;
-    }
-  uint32_t best = 0xffffffffu, mask = 0;
-  for (int r = 0; r < 24; r++) {
-    // row r places local vertex c_perm4[r][p] at position p; only rows that keep
-    // positions >= nv fixed are vertex orders of the first nv vertices
-    bool ok = true;
-    for (uint32_t p = 0; p < 4 && ok; p++) {
-      const uint32_t lv = c_perm4[r][p];
-      if (p >= nv) ok = lv == p;
-      else ok = lv < nv && lw[lv] == ls[p];
-    }
-    if (!ok) continue;
-    uint32_t inv[4];
-    for (uint32_t p = 0; p < 4; p++) inv[c_perm4[r][p]] = p;
-    uint32_t idx[3] = {7, 7, 7};
-    for (uint32_t e = 0; e < ne; e++) {
-      // index of the position pair (p<q) in lexicographic order (0,1)(0,2)(0,3)(1,2)(1,3)(2,3),
-      // computed (a per-lane constant-table lookup would serialise across lanes)
-      const uint32_t x = inv[E[e][0]], y = inv[E[e][1]];
-      const uint32_t p = x < y ? x : y, q = x < y ? y : x;
-      idx[e] = p * 3 - (p * (p - 1)) / 2 + (q - p - 1);
-    }
-    // sort ne <= 3 pair indices
-    if (idx[0] > idx[1]) { const uint32_t t = idx[0]; idx[0] = idx[1]; idx[1] = t; }
-    if (idx[1] > idx[2]) { const uint32_t t = idx[1]; idx[1] = idx[2]; idx[2] = t; }
-    if (idx[0] > idx[1]) { const uint32_t t = idx[0]; idx[0] = idx[1]; idx[1] = t; }
-    const uint32_t key = idx[0] * 64 + idx[1] * 8 + idx[2];
-    if (key < best) {
-      best = key;
-      mask = 1u << r;
-    } else if (key == best) {
-      mask |= 1u << r;
-    }
+__device__ __forceinline__ Canon canonical(const uint2 *tab, uint32_t l0, uint32_t l1, uint32_t l2, uint32_t l3,
+                                           uint32_t nv, uint32_t em) {
+  // composite (label, local index); the padding positions sort last, in local order
+  uint32_t c0 = l0 << 2, c1 = ((nv > 1 ? l1 : 4096u) << 2) | 1u;
+  uint32_t c2 = ((nv > 2 ? l2 : 4096u) << 2) | 2u, c3 = ((nv > 3 ? l3 : 4096u) << 2) | 3u;
+#define GAMMA_CX(x, y)                 \
+  {                                    \
+    const uint32_t t_ = min(x, y);     \
+    y = max(x, y);                     \
+    x = t_;                            \
   }
-  uint64_t key = kKeyTag | ((uint64_t)nv << 48) | ((uint64_t)ne << 51) | ((uint64_t)best << 53);
-  for (uint32_t p = 0; p < nv; p++) key |= (uint64_t)(ls[p] & 0xfffu) << (12 * p);
-  cn.key = key;
-  cn.minmask = mask;
-  return cn;
+  GAMMA_CX(c0, c1);
+  GAMMA_CX(c2, c3);
+  GAMMA_CX(c0, c2);
+  GAMMA_CX(c1, c3);
+  GAMMA_CX(c1, c2);
+#undef GAMMA_CX
+  const uint32_t ordw = (c0 & 3u) | (c1 & 3u) << 2 | (c2 & 3u) << 4 | (c3 & 3u) << 6;
+  const uint32_t posw = (1u << (2 * (c1 & 3u))) | (2u << (2 * (c2 & 3u))) | (3u << (2 * (c3 & 3u)));
+  uint32_t M = 0;
+#pragma unroll
+  for (uint32_t i = 0; i < 6; i++)
+    if ((em >> i) & 1u) {
+      const uint32_t pa = (posw >> (2 * ((kPairA >> (2 * i)) & 3u))) & 3u;
+      const uint32_t pb = (posw >> (2 * ((kPairB >> (2 * i)) & 3u))) & 3u;
+      M |= 1u << pid(pa, pb);
+    }
+  const uint32_t s0 = c0 >> 2, s1 = c1 >> 2, s2 = c2 >> 2, s3 = c3 >> 2;
+  const uint32_t tie = (uint32_t)(s0 == s1) | (uint32_t)(nv > 2 && s1 == s2) << 1 | (uint32_t)(nv > 3 && s2 == s3) << 2;
+  const uint2 e = tab[(M << 3) | tie];
+  uint64_t key = kKeyTag | ((uint64_t)nv << 48) | ((uint64_t)__popc(M) << 51) | ((uint64_t)e.x << 53);
+  key |= (uint64_t)(s0 & 0xfffu) | (uint64_t)(s1 & 0xfffu) << 12;
+  if (nv > 2) key |= (uint64_t)(s2 & 0xfffu) << 24;
+  if (nv > 3) key |= (uint64_t)(s3 & 0xfffu) << 36;
+  return Canon{key, e.y, ordw};
+}
+
+__device__ __forceinline__ uint32_t pick4(uint32_t i, uint32_t v0, uint32_t v1, uint32_t v2, uint32_t v3) {
+  return i == 0 ? v0 : i == 1 ? v1 : i == 2 ? v2 : v3;
 }
 
 // Aggregation: OR the vertex of every position of every minimizing order into the
 // position's domain bitmap (read-before-atomic: most bits are already set).
-__device__ void record(const FpmArgs &a, const uint32_t *W, uint32_t nv, const uint8_t (*E)[2], uint32_t ne) {
-  const Canon cn = canonical(a, W, nv, E, ne);
-  const int64_t s = table_slot(a, cn.key, true);
+__device__ void record(const FpmArgs &a, const uint2 *tab, const uint32_t *prm, uint32_t v0, uint32_t v1,
+                       uint32_t v2, uint32_t v3, uint32_t l0, uint32_t l1, uint32_t l2, uint32_t l3, uint32_t nv,
+                       uint32_t em) {
+  const Canon cn = canonical(tab, l0, l1, l2, l3, nv, em);
+  unsigned long long d = 0;
+  const int64_t s = table_slot(a, cn.key, true, d);
   if (s < 0) return;
-  uint64_t off[4];
   // the claimer may still be carving this slot's domains (a few instructions away);
   // the wait yields with nanosleep so a claiming lane of the same warp progresses
-  unsigned long long d = *(volatile unsigned long long *)&a.T.dom[s];
   while (d == 0) {
     __nanosleep(32);
-    d = *(volatile unsigned long long *)&a.T.dom[s];
+    d = __ldcg(&a.T.slots[2 * s + 1]);
   }
-  if (d == ~0ull) return;   // pool exhausted: the host grows it and reruns
+  if (d == ~0ull) return;   // no domains in this pass (pool exhausted / another chunk)
   __threadfence();
-  uint64_t o = d - 1;
-  for (uint32_t p = 0; p < 4; p++) {
-    off[p] = o;
-    if (p < nv) o += (a.csize[key_label(cn.key, p)] + 31) / 32;
-  }
+  uint64_t off[4];
+  off[0] = d - 1;
+  off[1] = off[0] + __ldg(a.cwords + key_label(cn.key, 0));
+  off[2] = off[1] + __ldg(a.cwords + key_label(cn.key, 1));
+  off[3] = off[2] + (nv > 2 ? __ldg(a.cwords + key_label(cn.key, 2)) : 0u);
   uint32_t m = cn.minmask;
   while (m) {
     const int r = __ffs(m) - 1;
     m &= m - 1;
-    for (uint32_t p = 0; p < nv; p++) {
-      const uint32_t v = W[c_perm4[r][p]];
-      const uint32_t bit = a.lrank[v];
-      uint32_t *w = a.T.pool + off[p] + (bit >> 5);
+    const uint32_t sg = prm[r];
+#pragma unroll
+    for (uint32_t c = 0; c < 4; c++) {
+      if (c >= nv) break;
+      const uint32_t sp = (sg >> (2 * c)) & 3u;            // sorted position placed at canonical c
+      const uint32_t v = pick4((cn.ordw >> (2 * sp)) & 3u, v0, v1, v2, v3);
+      const uint32_t bit = __ldg(a.lrank + v);
+      uint32_t *w = a.T.pool + off[c] + (bit >> 5);
       const uint32_t b = 1u << (bit & 31);
-      if (!(*(volatile uint32_t *)w & b)) atomicOr(w, b);
+      if (!(__ldcg(w) & b)) atomicOr(w, b);
     }
   }
 }
 
 // Is the pattern of this (prefix) edge set frequent?  (Alg. 2 line 4 pruning)
-__device__ bool frequent(const FpmArgs &a, const uint32_t *W, uint32_t nv, const uint8_t (*E)[2], uint32_t ne) {
-  const Canon cn = canonical(a, W, nv, E, ne);
-  const int64_t s = table_slot(a, cn.key, false);
+__device__ __forceinline__ bool frequent(const FpmArgs &a, const uint2 *tab, uint32_t l0, uint32_t l1, uint32_t l2,
+                                         uint32_t nv, uint32_t em) {
+  const Canon cn = canonical(tab, l0, l1, l2, 0u, nv, em);
+  unsigned long long d;
+  const int64_t s = table_slot(a, cn.key, false, d);
   return s >= 0 && a.T.freq[s];
 }
 
-// Local view of an edge set: distinct vertices W and local edge pairs E.
-struct ESet {
-  uint32_t W[4];
-  uint8_t E[3][2];
-  uint32_t nv, ne;
-};
-
-__device__ __forceinline__ uint32_t local_of(ESet &s, uint32_t x) {
-  for (uint32_t i = 0; i < s.nv; i++)
-    if (s.W[i] == x) return i;
-  s.W[s.nv] = x;
-  return s.nv++;
-}
-
-__device__ __forceinline__ void add_edge(ESet &s, uint64_t e) {
-  const uint32_t a = local_of(s, (uint32_t)(e >> 32));
-  const uint32_t b = local_of(s, (uint32_t)e);
-  s.E[s.ne][0] = (uint8_t)a;
-  s.E[s.ne][1] = (uint8_t)b;
-  s.ne++;
-}
-
-// One warp per root vertex u; roots e1 = (u, v), v > u.
+// One warp per batch of root edges e1 = (u, v), v > u.
 //   level 1: record e1.
 //   level 2: e2 > e1 adjacent to e1 (an edge at u or v), prefix {e1} frequent.
 //   level 3: from each frequent 2-edge prefix (a, b), a < b adjacent, add c with
 //            (c > b, c adjacent to a or b)  or  (a < c < b, c adjacent to b, not to a).
 //            Every connected {e1<e2<e3} arises exactly once: if e1~e2 from (e1,e2)+e3,
 //            else (e3 joins them) from (e1,e3)+e2.
+// Local vertices: 0 = u, 1 = v, 2 = the new end y of e2, 3 = the new end of e3.
 __global__ void __launch_bounds__(kThreads) fpm_enum_kernel(FpmArgs a) {
+  __shared__ uint2 s_tab[kCanonEntries];
+  __shared__ uint32_t s_prm[24];
+  for (int i = threadIdx.x; i < kCanonEntries; i += blockDim.x) s_tab[i] = a.canon_tab[i];
+  if (threadIdx.x < 24) s_prm[threadIdx.x] = a.perm_tab[threadIdx.x];
+  __syncthreads();
   const int lane = threadIdx.x & 31;
-  uint64_t emb = 0;
+  uint64_t emb = 0, elems = 0;       // embeddings recorded; adjacency elements streamed (lane 0)
   const uint64_t ndir = a.rp[a.n];   // directed edges: the roots are the (u, v > u) ones
   constexpr uint64_t kBatch = 8;
   for (;;) {
@@ -308,69 +311,63 @@ __global__ void __launch_bounds__(kThreads) fpm_enum_kernel(FpmArgs a) {
       if (v < u) continue;             // each undirected edge once, from its smaller end
       const uint64_t us = a.rp[u], ue = a.rp[u + 1];
       const uint64_t e1 = ekey(u, v);
+      const uint32_t lu = labof(a, u), lv = labof(a, v);
       if (a.level == 1) {
         if (lane == 0) {
-          ESet s{};
-          add_edge(s, e1);
-          record(a, s.W, s.nv, s.E, s.ne);
+          record(a, s_tab, s_prm, u, v, 0u, 0u, lu, lv, 0u, 0u, 2, 1u << pid(0, 1));
           emb++;
         }
         continue;
       }
-      {
-        ESet s{};
-        add_edge(s, e1);
-        if (!frequent(a, s.W, s.nv, s.E, s.ne)) continue;   // uniform: same e1 in all lanes
-      }
+      if (!frequent(a, s_tab, lu, lv, 0u, 2, 1u << pid(0, 1))) continue;   // uniform: same e1 in all lanes
       // candidate second edges: incident to u or v (lists of u then v), e2 > e1
       const uint64_t vs = a.rp[v], ve = a.rp[v + 1];
       const uint64_t nu = ue - us, ncand = nu + (ve - vs);
+      if (lane == 0) elems += ncand;
       for (uint64_t c0 = 0; c0 < ncand; c0 += 32) {
         const uint64_t ci = c0 + lane;
-        // lane's second edge e2 (a candidate prefix {e1, e2})
+        // lane's second edge e2 = (x, y), x in {u, v}: a candidate prefix {e1, e2}
         bool valid = ci < ncand;
         uint64_t e2 = 0;
-        ESet s2{};
+        uint32_t y = 0, ly = 0, em2 = 0;
         if (valid) {
-          const uint32_t x = ci < nu ? u : v;
-          const uint32_t y = ci < nu ? a.col[us + ci] : a.col[vs + (ci - nu)];
-          e2 = ekey(x, y);
-          valid = e2 > e1;   // also drops e1 itself
+          const bool at_u = ci < nu;
+          y = at_u ? a.col[us + ci] : a.col[vs + (ci - nu)];
+          e2 = ekey(at_u ? u : v, y);
+          valid = e2 > e1;   // also drops e1 itself (y is then u or v)
+          em2 = (1u << pid(0, 1)) | (1u << pid(at_u ? 0 : 1, 2));
         }
         if (valid) {
-          add_edge(s2, e1);
-          add_edge(s2, e2);
+          ly = labof(a, y);
           if (a.level == 2) {
-            record(a, s2.W, s2.nv, s2.E, s2.ne);
+            record(a, s_tab, s_prm, u, v, y, 0u, lu, lv, ly, 0u, 3, em2);
             emb++;
             valid = false;
           } else {
-            valid = frequent(a, s2.W, s2.nv, s2.E, s2.ne);   // Alg. 2 line 4
+            valid = frequent(a, s_tab, lu, lv, ly, 3, em2);   // Alg. 2 line 4
           }
         }
         if (a.level == 2) continue;   // uniform
-        // third edges: incident to the 3 vertices of a frequent prefix.  The candidate
-        // lists of the valid prefixes are concatenated and streamed by all 32 lanes
-        // (flattened windows; prefix found by an OR-reduction of the start offsets),
-        // so a hub prefix does not serialise on one lane.
-        uint32_t w0 = 0, w1 = 0, w2 = 0, d0 = 0, d1 = 0, d2 = 0, b0 = 0, b1 = 0, b2 = 0;
+        // third edges: incident to the 3 vertices u, v, y of a frequent prefix.  The
+        // candidate lists N(u) ++ N(v) ++ N(y) of the valid prefixes are concatenated
+        // and streamed by all 32 lanes (flattened windows; prefix found by an
+        // OR-reduction of the start offsets), so a hub prefix does not serialise on
+        // one lane.  N(u), N(v) are the same for every prefix of this e1.
+        const uint32_t du = (uint32_t)nu, dv = (uint32_t)(ve - vs);
+        uint32_t by = 0, dy = 0;
         if (valid) {
-          w0 = s2.W[0]; w1 = s2.W[1]; w2 = s2.W[2];
-          b0 = (uint32_t)a.rp[w0]; d0 = (uint32_t)(a.rp[w0 + 1] - b0);
-          b1 = (uint32_t)a.rp[w1]; d1 = (uint32_t)(a.rp[w1 + 1] - b1);
-          b2 = (uint32_t)a.rp[w2]; d2 = (uint32_t)(a.rp[w2 + 1] - b2);
+          by = (uint32_t)a.rp[y];
+          dy = (uint32_t)(a.rp[y + 1] - by);
         }
-        const uint32_t tl = d0 + d1 + d2;   // 0 unless valid (every vertex has an edge)
+        const uint32_t tl = valid ? du + dv + dy : 0u;
         const uint32_t nz = __ballot_sync(0xffffffffu, tl > 0);
         const uint32_t nnz = __popc(nz);
         const uint32_t src = lane < (int)nnz ? __fns(nz, 0, lane + 1) : 0;
-        // compacted prefix data (lane k = k-th valid prefix)
-        const uint64_t ce2 = __shfl_sync(0xffffffffu, e2, src);
-        const uint32_t cw0 = __shfl_sync(0xffffffffu, w0, src), cw1 = __shfl_sync(0xffffffffu, w1, src);
-        const uint32_t cw2 = __shfl_sync(0xffffffffu, w2, src);
-        const uint32_t cb0 = __shfl_sync(0xffffffffu, b0, src), cb1 = __shfl_sync(0xffffffffu, b1, src);
-        const uint32_t cb2 = __shfl_sync(0xffffffffu, b2, src);
-        const uint32_t cd0 = __shfl_sync(0xffffffffu, d0, src), cd1 = __shfl_sync(0xffffffffu, d1, src);
+        // compacted prefix data (lane k = k-th valid prefix); em2 travels in the top
+        // bits of the label word (labels < 4096)
+        const uint32_t cy = __shfl_sync(0xffffffffu, y, src);
+        const uint32_t cl = __shfl_sync(0xffffffffu, ly | (em2 << 16), src);
+        const uint32_t cby = __shfl_sync(0xffffffffu, by, src);
         const uint32_t stl = __shfl_sync(0xffffffffu, tl, src);
         const uint32_t ctl = lane < (int)nnz ? stl : 0u;
         uint32_t sc = ctl;
@@ -380,6 +377,7 @@ __global__ void __launch_bounds__(kThreads) fpm_enum_kernel(FpmArgs a) {
           if (lane >= o) sc += yv;
         }
         const uint32_t T = __shfl_sync(0xffffffffu, sc, 31);
+        if (lane == 0) elems += T;
         const uint32_t ost = sc - ctl;
         const uint32_t upto = lane == 31 ? 0xffffffffu : ((2u << lane) - 1u);
         uint32_t nb = 0;
@@ -389,32 +387,28 @@ __global__ void __launch_bounds__(kThreads) fpm_enum_kernel(FpmArgs a) {
           const uint32_t S = __reduce_or_sync(0xffffffffu, mine);
           const int j = ((int)(nb + __popc(S & upto)) - 1) & 31;
           nb += __popc(S);
-          const uint64_t pe2 = __shfl_sync(0xffffffffu, ce2, j);
-          const uint32_t p0 = __shfl_sync(0xffffffffu, cw0, j), p1 = __shfl_sync(0xffffffffu, cw1, j);
-          const uint32_t p2 = __shfl_sync(0xffffffffu, cw2, j);
-          const uint32_t q0 = __shfl_sync(0xffffffffu, cb0, j), q1 = __shfl_sync(0xffffffffu, cb1, j);
-          const uint32_t q2 = __shfl_sync(0xffffffffu, cb2, j);
-          const uint32_t r0 = __shfl_sync(0xffffffffu, cd0, j), r1 = __shfl_sync(0xffffffffu, cd1, j);
+          const uint32_t py = __shfl_sync(0xffffffffu, cy, j);
+          const uint32_t pl = __shfl_sync(0xffffffffu, cl, j);
+          const uint32_t pby = __shfl_sync(0xffffffffu, cby, j);
           const uint32_t oj = __shfl_sync(0xffffffffu, ost, j);
           if (t >= T) continue;
           const uint32_t r = t - oj;
-          uint32_t w, zi;
-          if (r < r0) { w = p0; zi = q0 + r; }
-          else if (r < r0 + r1) { w = p1; zi = q1 + (r - r0); }
-          else { w = p2; zi = q2 + (r - r0 - r1); }
+          uint32_t w, zi, lw;
+          if (r < du) { w = u; zi = (uint32_t)us + r; lw = 0; }
+          else if (r < du + dv) { w = v; zi = (uint32_t)vs + (r - du); lw = 1; }
+          else { w = py; zi = pby + (r - du - dv); lw = 2; }
           const uint32_t z = a.col[zi];
           // an edge joining two prefix vertices is seen from both ends: keep the smaller
-          const bool inner = z == p0 || z == p1 || z == p2;
-          if (inner && z < w) continue;
+          const uint32_t lz = z == u ? 0u : z == v ? 1u : z == py ? 2u : 3u;
+          if (lz < 3 && z < w) continue;
+          const uint64_t pe2 = ekey((pl >> 16) & (1u << pid(1, 2)) ? v : u, py);
           const uint64_t e3 = ekey(w, z);
           if (e3 == e1 || e3 == pe2) continue;
           const bool ok = (e3 > pe2) || (e3 > e1 && shares(e3, pe2) && !shares(e3, e1));
           if (!ok) continue;
-          ESet s3{};
-          add_edge(s3, e1);
-          add_edge(s3, pe2);
-          add_edge(s3, e3);
-          record(a, s3.W, s3.nv, s3.E, s3.ne);
+          const uint32_t em3 = (pl >> 16) | (1u << pid(lw, lz));
+          record(a, s_tab, s_prm, u, v, py, z, lu, lv, pl & 0xffffu, lz == 3 ? labof(a, z) : 0u, lz == 3 ? 4 : 3,
+                 em3);
           emb++;
         }
       }
@@ -422,6 +416,7 @@ __global__ void __launch_bounds__(kThreads) fpm_enum_kernel(FpmArgs a) {
   }
   for (int off = 16; off > 0; off >>= 1) emb += __shfl_down_sync(0xffffffffu, emb, off);
   if (lane == 0 && emb) atomicAdd(&a.ctrl[CTRL_ENTRIES], (unsigned long long)emb);
+  if (lane == 0 && elems) atomicAdd(&a.ctrl[CTRL_ELEMS], (unsigned long long)elems);
 }
 
 // Support of every slot of the given level: min over positions of popcount; one
@@ -431,20 +426,20 @@ __global__ void fpm_support_kernel(FpmArgs a, uint32_t level, uint64_t minsup) {
   const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
   const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
   for (uint64_t s = warp; s < a.T.cap; s += nwarps) {
-    const uint64_t key = a.T.key[s];
+    const uint64_t key = a.T.slots[2 * s];
     if (key == 0) continue;
     const uint32_t nv = key_nv(key), ne = key_ne(key);
     if (ne != level) continue;
     // no domains in this pass (pool exhausted, or another chunk of a split level):
     // a later pass computes this slot
-    const unsigned long long d = a.T.dom[s];
+    const unsigned long long d = a.T.slots[2 * s + 1];
     if (d == 0 || d == ~0ull) continue;
     uint64_t sup = ~0ull;
     for (uint32_t p = 0; p < nv; p++) {
       const uint32_t lp = key_label(key, p);
-      const uint64_t words = (a.csize[lp] + 31) / 32;
+      const uint64_t words = a.cwords[lp];
       uint64_t off = d - 1;
-      for (uint32_t i = 0; i < p; i++) off += (a.csize[key_label(key, i)] + 31) / 32;
+      for (uint32_t i = 0; i < p; i++) off += a.cwords[key_label(key, i)];
       uint64_t c = 0;
       for (uint64_t w = lane; w < words; w += 32) c += __popc(a.T.pool[off + w]);
       for (int o = 16; o > 0; o >>= 1) c += __shfl_down_sync(0xffffffffu, c, o);
@@ -498,7 +493,7 @@ __global__ void max_label_kernel(const uint32_t *lab, uint32_t n, unsigned long 
 __global__ void level_keys_kernel(const unsigned long long *key, uint64_t cap, uint32_t level,
                                   unsigned long long *out, unsigned long long *cursor) {
   for (uint64_t s = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; s < cap; s += (uint64_t)gridDim.x * blockDim.x) {
-    const unsigned long long k = key[s];
+    const unsigned long long k = key[2 * s];   // slots: (key, dom) pairs
     if (k && key_ne(k) == level) out[atomicAdd(cursor, 1ull)] = k;
   }
 }
@@ -538,6 +533,65 @@ inline unsigned g1d(uint64_t n) {
 
 }  // namespace
 
+// Canonical-code tables for the device (reading R7), by enumeration of the 24 vertex
+// orders sigma of the sorted positions: entry (M << 3 | tie) = {min over valid sigma of
+// the sorted edge-pair key of the edge mask M under sigma, set of sigmas reaching it}.
+// sigma is valid iff it only permutes positions of equal labels (tie bit i: sorted
+// labels i and i+1 equal).  perm rows in lexicographic order, sigma[c] in bits 2c.
+static void fpm_canon_tables(std::vector<uint2> &tab, std::vector<uint32_t> &prm) {
+  std::vector<std::array<uint32_t, 4>> perms;
+  std::array<uint32_t, 4> p{0, 1, 2, 3};
+  do perms.push_back(p);
+  while (std::next_permutation(p.begin(), p.end()));
+  prm.assign(24, 0);
+  for (int r = 0; r < 24; r++)
+    for (int c = 0; c < 4; c++) prm[r] |= perms[r][c] << (2 * c);
+  tab.assign(kCanonEntries, make_uint2(0, 0));
+  for (uint32_t M = 0; M < 64; M++)
+    for (uint32_t tie = 0; tie < 8; tie++) {
+      uint32_t grp[4] = {0, 0, 0, 0};
+      for (int i = 0; i < 3; i++) grp[i + 1] = grp[i] + (((tie >> i) & 1) ? 0 : 1);
+      uint32_t best = 0xffffffffu, mask = 0;
+      for (int r = 0; r < 24; r++) {
+        const auto &sg = perms[r];
+        bool ok = true;
+        for (int c = 0; c < 4; c++) ok = ok && grp[sg[c]] == grp[c];
+        if (!ok) continue;
+        uint32_t inv[4];
+        for (uint32_t c = 0; c < 4; c++) inv[sg[c]] = c;
+        uint32_t idx[3] = {7, 7, 7}, ne = 0;
+        for (uint32_t q = 0; q < 4; q++)
+          for (uint32_t pp = 0; pp < q; pp++)
+            if ((M >> pid(pp, q)) & 1u) {
+              const uint32_t x = inv[pp], y = inv[q];
+              if (ne < 3) idx[ne] = pid(std::min(x, y), std::max(x, y));
+              ne++;
+            }
+        if (ne > 3) continue;   // not a pattern of <= 3 edges
+        std::sort(idx, idx + 3);
+        const uint32_t key = idx[0] * 64 + idx[1] * 8 + idx[2];
+        if (key < best) {
+          best = key;
+          mask = 1u << r;
+        } else if (key == best) {
+          mask |= 1u << r;
+        }
+      }
+      tab[(M << 3) | tie] = make_uint2(best == 0xffffffffu ? 0u : best, mask);
+    }
+}
+
+// one column (0 = key, 1 = dom) of the (key, dom) slot pairs <-> a dense host array
+static void slots_get(gamma_ctx *ctx, std::vector<unsigned long long> &h, const unsigned long long *slots,
+                      uint64_t cap, int colm) {
+  h.resize(cap);
+  GAMMA_CUDA(cudaMemcpy2DAsync(h.data(), 8, slots + colm, 16, 8, cap, cudaMemcpyDeviceToHost, ctx->stream));
+}
+static void slots_put(gamma_ctx *ctx, unsigned long long *slots, const std::vector<unsigned long long> &h,
+                      uint64_t cap, int colm) {
+  GAMMA_CUDA(cudaMemcpy2DAsync(slots + colm, 16, h.data(), 8, 8, cap, cudaMemcpyHostToDevice, ctx->stream));
+}
+
 static gamma_fpm_pattern decode_pattern(uint64_t key, uint64_t support) {
   static const uint8_t pairs[6][2] = {{0, 1}, {0, 2}, {0, 3}, {1, 2}, {1, 3}, {2, 3}};
   gamma_fpm_pattern p{};
@@ -553,6 +607,13 @@ static gamma_fpm_pattern decode_pattern(uint64_t key, uint64_t support) {
   }
   p.support = support;
   return p;
+}
+
+// Algorithmic bytes of one enumeration pass (FPM): 4 B per adjacency
+// element streamed by the extension, 32 B per recorded embedding (its 16-byte
+// pattern-table slot + one 4-byte domain word per position, <= 4 positions).
+static void count_fpm_bytes(gamma_ctx *ctx) {
+  ctx->stats.alg_bytes[KC_FPM] += 4 * ctx->ctrl_host[CTRL_ELEMS] + 32 * ctx->ctrl_host[CTRL_ENTRIES];
 }
 
 static void coll_allreduce(gamma_ctx *ctx, uint64_t *v, size_t n) {
@@ -579,8 +640,8 @@ static void coll_alltoall(gamma_ctx *ctx, const uint32_t *send, uint32_t *recv, 
 // position), hence the same supports and output.  Returns false when some rank's
 // table overflowed (all ranks then grow it and retry together).
 static bool fpm_dist_level(gamma_ctx *ctx, FpmArgs &a, int grid_enum, uint32_t l, uint64_t minsup,
-                           const std::vector<uint32_t> &hsize, uint64_t cap, unsigned long long *key_d,
-                           unsigned long long *dom_d, uint32_t *pool_d, uint64_t pool_words,
+                           const std::vector<uint32_t> &hsize, uint64_t cap, unsigned long long *slots_d,
+                           uint32_t *pool_d, uint64_t pool_words,
                            unsigned long long *pcur_d, std::vector<gamma_fpm_pattern> &found) {
   const uint32_t G = (uint32_t)ctx->desc.world, R = (uint32_t)ctx->desc.rank;
   a.level = l;
@@ -593,7 +654,7 @@ static bool fpm_dist_level(gamma_ctx *ctx, FpmArgs &a, int grid_enum, uint32_t l
   a.claim_only = 0;
   DevBuf<unsigned long long> mine(ctx, cap);
   ctx->launch(KC_MISC, [&] {
-    level_keys_kernel<<<g1d(cap), 256, 0, ctx->stream>>>(key_d, cap, l, mine.p,
+    level_keys_kernel<<<g1d(cap), 256, 0, ctx->stream>>>(slots_d, cap, l, mine.p,
                                                          (unsigned long long *)ctx->ctrl + CTRL_AUX0);
   });
   ctrl_fetch(ctx);
@@ -646,8 +707,8 @@ static bool fpm_dist_level(gamma_ctx *ctx, FpmArgs &a, int grid_enum, uint32_t l
     if (nU && U[0] == 0) U.erase(U.begin());   // padding
   }
   // ---- 3. chunks of U ----
-  std::vector<unsigned long long> hkey(cap), hdom(cap);
-  GAMMA_CUDA(cudaMemcpyAsync(hkey.data(), key_d, cap * 8, cudaMemcpyDeviceToHost, ctx->stream));
+  std::vector<unsigned long long> hkey, hdom(cap);
+  slots_get(ctx, hkey, slots_d, cap, 0);
   ctx->sync();
   std::unordered_map<uint64_t, uint64_t> slot_of;
   slot_of.reserve(nmine * 2 + 1);
@@ -680,12 +741,13 @@ static bool fpm_dist_level(gamma_ctx *ctx, FpmArgs &a, int grid_enum, uint32_t l
     }
     const size_t j1 = next;
     const uint64_t shard = (used + G - 1) / G;
-    GAMMA_CUDA(cudaMemcpyAsync(dom_d, hdom.data(), cap * 8, cudaMemcpyHostToDevice, ctx->stream));
+    slots_put(ctx, slots_d, hdom, cap, 1);
     GAMMA_CUDA(cudaMemsetAsync(dom_buf, 0, shard * G * 4, ctx->stream));
     GAMMA_CUDA(cudaMemcpyAsync(pcur_d, &pool_words, 8, cudaMemcpyHostToDevice, ctx->stream));
     ctrl_reset(ctx);
     ctx->launch(KC_FPM, [&] { fpm_enum_kernel<<<grid_enum, kThreads, 0, ctx->stream>>>(a); });
     ctrl_fetch(ctx);
+    count_fpm_bytes(ctx);
     GAMMA_REQUIRE(ctx->ctrl_host[CTRL_ERR] == 0 && ctx->ctrl_host[CTRL_OVF] == 0, GAMMA_E_CUDA,
                   "gamma_fpm: a distributed chunk pass met an unclaimed pattern");
     coll_alltoall(ctx, dom_buf, recv_buf, shard);
@@ -750,12 +812,22 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
   // ---- pattern table + per-(slot, position) domain bitmaps ----
   size_t fr = 0, tot = 0;
   GAMMA_CUDA(cudaMemGetInfo(&fr, &tot));
-  const uint64_t budget = ctx->desc.hbm_budget_bytes ? ctx->desc.hbm_budget_bytes : (uint64_t)(fr * 0.6);
+  const uint64_t budget = ctx->desc.hbm_budget_bytes ? ctx->desc.hbm_budget_bytes : (uint64_t)(fr * 0.85);
   std::vector<uint32_t> hsize(nlab);
   GAMMA_CUDA(cudaMemcpyAsync(hsize.data(), csize.p, nlab * 4, cudaMemcpyDeviceToHost, ctx->stream));
   ctx->sync();
   uint64_t maxw = 1;
-  for (auto c : hsize) maxw = std::max<uint64_t>(maxw, (c + 31) / 32);
+  std::vector<uint32_t> hwords(nlab);
+  for (uint32_t l = 0; l < nlab; l++) {
+    hwords[l] = (hsize[l] + 31) / 32;
+    maxw = std::max<uint64_t>(maxw, hwords[l]);
+  }
+  DevBuf<uint32_t> cwords = to_device(ctx, hwords.data(), nlab);
+  std::vector<uint2> htab;
+  std::vector<uint32_t> hprm;
+  fpm_canon_tables(htab, hprm);
+  DevBuf<uint2> canon_tab = to_device(ctx, htab.data(), htab.size());
+  DevBuf<uint32_t> perm_tab = to_device(ctx, hprm.data(), hprm.size());
   // Distinct patterns are bounded by the label combinations of each shape (edge,
   // wedge, triangle, 3-star, 3-path); size the table at twice that bound (load <= 1/2,
   // short probe chains) and grow x4 if a chain still gets long.  The domain pool is
@@ -769,13 +841,15 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
   const uint64_t slot_bytes = 8 + 8 + 4 + 8;
   while (cap > 1024 && cap * slot_bytes * 4 > budget) cap >>= 1;
   DevBuf<uint32_t> freq, pool;
-  DevBuf<unsigned long long> key, sup, dom, pcur;
+  DevBuf<unsigned long long> slots, sup, pcur;
   FpmArgs a{};
   a.rp = g->row_ptr;
   a.col = g->col;
   a.lab = g->labels;
   a.lrank = lrank.p;
-  a.csize = csize.p;
+  a.cwords = cwords.p;
+  a.canon_tab = canon_tab.p;
+  a.perm_tab = perm_tab.p;
   a.n = n;
   a.rank = 0;
   a.world = 1;   // levels < l run on every rank; the last one is split when dist
@@ -789,24 +863,22 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
     GAMMA_REQUIRE(cap * slot_bytes < budget, GAMMA_E_NOMEM, "gamma_fpm: pattern table exceeds the HBM budget");
     const uint64_t pool_words =
         std::max<uint64_t>(64, std::min<uint64_t>((budget - cap * slot_bytes) / 4, cap * 4 * maxw));
-    freq.reset(); pool.reset(); key.reset(); sup.reset(); dom.reset(); pcur.reset();
-    key = DevBuf<unsigned long long>(ctx, cap);
+    freq.reset(); pool.reset(); slots.reset(); sup.reset(); pcur.reset();
+    slots = DevBuf<unsigned long long>(ctx, 2 * cap);
     sup = DevBuf<unsigned long long>(ctx, cap);
-    dom = DevBuf<unsigned long long>(ctx, cap);
     freq = DevBuf<uint32_t>(ctx, cap);
     pool = DevBuf<uint32_t>(ctx, pool_words);
     pcur = DevBuf<unsigned long long>(ctx, 1);
-    GAMMA_CUDA(cudaMemsetAsync(key.p, 0, cap * 8, ctx->stream));
-    GAMMA_CUDA(cudaMemsetAsync(dom.p, 0, cap * 8, ctx->stream));
+    GAMMA_CUDA(cudaMemsetAsync(slots.p, 0, cap * 16, ctx->stream));
     GAMMA_CUDA(cudaMemsetAsync(freq.p, 0, cap * 4, ctx->stream));
     GAMMA_CUDA(cudaMemsetAsync(pool.p, 0, pool_words * 4, ctx->stream));
     GAMMA_CUDA(cudaMemsetAsync(pcur.p, 0, 8, ctx->stream));
-    a.T = Table{key.p, sup.p, freq.p, dom.p, cap, pool.p, pool_words, pcur.p};
+    a.T = Table{slots.p, sup.p, freq.p, cap, pool.p, pool_words, pcur.p};
     bool full = false;
     found_last.clear();
     for (uint32_t l = 1; l <= max_edges && !full; l++) {
       if (dist && l == max_edges) {
-        full = !fpm_dist_level(ctx, a, grid_enum, l, minsup, hsize, cap, key.p, dom.p, pool.p, pool_words, pcur.p,
+        full = !fpm_dist_level(ctx, a, grid_enum, l, minsup, hsize, cap, slots.p, pool.p, pool_words, pcur.p,
                                found_last);
         break;
       }
@@ -819,6 +891,7 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
       uint64_t carved = 0;
       GAMMA_CUDA(cudaMemcpyAsync(&carved, pcur.p, 8, cudaMemcpyDeviceToHost, ctx->stream));
       ctrl_fetch(ctx);
+      count_fpm_bytes(ctx);
       full = ctx->ctrl_host[CTRL_ERR] != 0;
       if (dist) {   // the ranks must agree on growing the table
         uint64_t f = full;
@@ -844,9 +917,9 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
       // carved), and the slots that got domains have their support: split the rest
       // into chunks that fit the pool and redo the level's enumeration once per
       // chunk, recording only into that chunk's slots (dom = ~0 elsewhere).
-      std::vector<unsigned long long> hkey(cap), hdom(cap);
-      GAMMA_CUDA(cudaMemcpyAsync(hkey.data(), key.p, cap * 8, cudaMemcpyDeviceToHost, ctx->stream));
-      GAMMA_CUDA(cudaMemcpyAsync(hdom.data(), dom.p, cap * 8, cudaMemcpyDeviceToHost, ctx->stream));
+      std::vector<unsigned long long> hkey, hdom;
+      slots_get(ctx, hkey, slots.p, cap, 0);
+      slots_get(ctx, hdom, slots.p, cap, 1);
       ctx->sync();
       std::vector<uint64_t> pending;
       for (uint64_t s = 0; s < cap; s++)
@@ -864,7 +937,7 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
           hdom[pending[next]] = 1 + used;
           used += words;
         }
-        GAMMA_CUDA(cudaMemcpyAsync(dom.p, hdom.data(), cap * 8, cudaMemcpyHostToDevice, ctx->stream));
+        slots_put(ctx, slots.p, hdom, cap, 1);
         clear_pool();
         dirty = used;
         GAMMA_CUDA(cudaMemcpyAsync(pcur.p, &pool_words, 8, cudaMemcpyHostToDevice, ctx->stream));
@@ -874,6 +947,7 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
           fpm_support_kernel<<<g1d(cap * 32), 256, 0, ctx->stream>>>(a, l, minsup);
         });
         ctrl_fetch(ctx);
+        count_fpm_bytes(ctx);
         GAMMA_REQUIRE(ctx->ctrl_host[CTRL_ERR] == 0 && ctx->ctrl_host[CTRL_OVF] == 0, GAMMA_E_CUDA,
                       "gamma_fpm: a chunk pass met an unclaimed pattern");
         ctx->stats.chunks++;
@@ -887,9 +961,9 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
   }
   // ---- collect the frequent patterns ----
   std::vector<uint32_t> hfreq(cap);
-  std::vector<unsigned long long> hkey(cap), hsup(cap);
+  std::vector<unsigned long long> hkey, hsup(cap);
   GAMMA_CUDA(cudaMemcpyAsync(hfreq.data(), freq.p, cap * 4, cudaMemcpyDeviceToHost, ctx->stream));
-  GAMMA_CUDA(cudaMemcpyAsync(hkey.data(), key.p, cap * 8, cudaMemcpyDeviceToHost, ctx->stream));
+  slots_get(ctx, hkey, slots.p, cap, 0);
   GAMMA_CUDA(cudaMemcpyAsync(hsup.data(), sup.p, cap * 8, cudaMemcpyDeviceToHost, ctx->stream));
   ctx->sync();
   for (uint64_t s = 0; s < cap; s++) {

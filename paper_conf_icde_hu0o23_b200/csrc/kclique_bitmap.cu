@@ -179,6 +179,198 @@ __device__ void dfs_multi(const uint32_t *B, uint32_t W, const uint32_t (&cur)[T
   }
 }
 
+// ---- register-resident DFS (warp teams, rows of TW <= 4 words, stride TW) ----------
+// The DFS below a triangle item is unrolled into nested loops by template recursion
+// over the number S of chosen vertices (S < SM, a compile-time bound on k), so the
+// candidate bitmaps of every level, the set bits still to visit and the per-size
+// counters all live in registers (no local-memory stack); a row is one 16-byte
+// shared-memory load.
+template <int TW>
+__device__ __forceinline__ void load_row(const uint32_t *B, uint32_t j, uint32_t (&r)[TW]) {
+  if constexpr (TW == 4) {
+    const uint4 x = *reinterpret_cast<const uint4 *>(B + j * 4);
+    r[0] = x.x; r[1] = x.y; r[2] = x.z; r[3] = x.w;
+  } else {
+#pragma unroll
+    for (int w = 0; w < TW; w++) r[w] = B[j * TW + w];
+  }
+}
+
+// lowest set bit of rem (cleared), or -1
+template <int TW>
+__device__ __forceinline__ int pop_next(uint32_t (&rem)[TW]) {
+  int wi = -1;
+#pragma unroll
+  for (int w = TW - 1; w >= 0; w--)
+    if (rem[w]) wi = w;
+  if (wi < 0) return -1;
+  uint32_t word = 0;
+#pragma unroll
+  for (int w = 0; w < TW; w++)
+    if (w == wi) word = rem[w];
+#pragma unroll
+  for (int w = 0; w < TW; w++)
+    if (w == wi) rem[w] = word & (word - 1u);
+  return wi * 32 + __ffs(word) - 1;
+}
+
+template <int TW>
+__device__ __forceinline__ uint32_t popc_n(const uint32_t (&x)[TW]) {
+  uint32_t c = 0;
+#pragma unroll
+  for (int w = 0; w < TW; w++) c += __popc(x[w]);
+  return c;
+}
+
+// multi-size: node with S chosen vertices adds popc(cur) (S+1)-cliques; expands while
+// S + 1 < kmax
+template <int TW, int S, int SM, int N>
+__device__ __forceinline__ void rdfs_multi(const uint32_t *B, const uint32_t (&cur)[TW], uint32_t kmax,
+                                           uint64_t (&mc)[N]) {
+  static_assert(SM < N, "counter array too short");
+  const uint32_t c = popc_n<TW>(cur);
+  mc[S + 1] += c;
+  if constexpr (S + 1 < SM) {
+    if (S + 1 >= kmax || c == 0) return;
+    uint32_t rem[TW];
+#pragma unroll
+    for (int w = 0; w < TW; w++) rem[w] = cur[w];
+    for (;;) {
+      const int j = pop_next<TW>(rem);
+      if (j < 0) break;
+      uint32_t nx[TW];
+      load_row<TW>(B, (uint32_t)j, nx);
+#pragma unroll
+      for (int w = 0; w < TW; w++) nx[w] &= cur[w];
+      rdfs_multi<TW, S + 1, SM, N>(B, nx, kmax, mc);
+    }
+  }
+}
+
+// single k: k-cliques below a node with S chosen vertices (prunes nodes that cannot
+// reach k)
+template <int TW, int S, int SM>
+__device__ __forceinline__ uint64_t rdfs_count(const uint32_t *B, const uint32_t (&cur)[TW], uint32_t k) {
+  const uint32_t c = popc_n<TW>(cur);
+  if (S + 1 == k) return c;
+  uint64_t cnt = 0;
+  if constexpr (S + 1 < SM) {
+    if (c < k - S) return 0;
+    uint32_t rem[TW];
+#pragma unroll
+    for (int w = 0; w < TW; w++) rem[w] = cur[w];
+    for (;;) {
+      const int j = pop_next<TW>(rem);
+      if (j < 0) break;
+      uint32_t nx[TW];
+      load_row<TW>(B, (uint32_t)j, nx);
+#pragma unroll
+      for (int w = 0; w < TW; w++) nx[w] &= cur[w];
+      cnt += rdfs_count<TW, S + 1, SM>(B, nx, k);
+    }
+  }
+  return cnt;
+}
+
+// ---- lane-group DFS (CTA teams and heavy-root parts, rows of W <= 16 words) -------
+// A thread-per-item DFS over 16-word rows diverges badly (the subtree sizes of the
+// triangles of one hub differ by orders of magnitude; ncu: < 5 active threads per
+// warp instruction).  Here a group of kGroup = 16 aligned lanes walks one item, lane
+// gl holding word gl of every candidate bitmap: a node is one conflict-free row load,
+// an AND and a popcount per lane; the next child is one group ballot + shuffle.  The
+// counts stay per lane (summed by the final warp reduction).  Template recursion over
+// the number S of chosen vertices keeps every level in registers.
+constexpr int kGroup = 16;
+
+struct LaneGroup {
+  uint32_t mask;   // the group's lanes in the warp
+  int base;        // first lane of the group
+  int gl;          // this lane's index inside the group
+  int lane;
+};
+
+__device__ __forceinline__ LaneGroup lane_group(int lane) {
+  LaneGroup g;
+  g.base = lane & ~(kGroup - 1);
+  g.gl = lane - g.base;
+  g.mask = ((1u << kGroup) - 1u) << g.base;
+  g.lane = lane;
+  return g;
+}
+
+// next child of the group's remaining-bits word set (cleared), or -1
+__device__ __forceinline__ int group_next(const LaneGroup &g, uint32_t &rem) {
+  const uint32_t bal = __ballot_sync(g.mask, rem != 0u);
+  if (bal == 0) return -1;
+  const int src = __ffs(bal) - 1;
+  const uint32_t word = __shfl_sync(g.mask, rem, src);
+  if (g.lane == src) rem &= rem - 1u;
+  return (src - g.base) * 32 + __ffs(word) - 1;
+}
+
+template <int S, int SM, int N>
+__device__ __forceinline__ void gdfs_multi(const uint32_t *B, uint32_t W, uint32_t curw, uint32_t kmax,
+                                           uint64_t (&mc)[N], const LaneGroup &g) {
+  static_assert(SM < N, "counter array too short");
+  mc[S + 1] += __popc(curw);
+  if constexpr (S + 1 < SM) {
+    if (S + 1 >= kmax) return;
+    uint32_t rem = curw;
+    for (;;) {
+      const int j = group_next(g, rem);
+      if (j < 0) break;
+      const uint32_t row = g.gl < (int)W ? B[(uint32_t)j * W + g.gl] : 0u;
+      gdfs_multi<S + 1, SM, N>(B, W, curw & row, kmax, mc, g);
+    }
+  }
+}
+
+template <int S, int SM>
+__device__ __forceinline__ uint64_t gdfs_count(const uint32_t *B, uint32_t W, uint32_t curw, uint32_t k,
+                                               const LaneGroup &g) {
+  if (S + 1 == k) return __popc(curw);
+  uint64_t cnt = 0;
+  if constexpr (S + 1 < SM) {
+    const uint32_t c = __reduce_add_sync(g.mask, __popc(curw));
+    if (c < k - S) return 0;
+    uint32_t rem = curw;
+    for (;;) {
+      const int j = group_next(g, rem);
+      if (j < 0) break;
+      const uint32_t row = g.gl < (int)W ? B[(uint32_t)j * W + g.gl] : 0u;
+      cnt += gdfs_count<S + 1, SM>(B, W, curw & row, k, g);
+    }
+  }
+  return cnt;
+}
+
+// Item q -> this lane's word of the candidates of the triangle (v, R[j1], R[j2]).
+__device__ __forceinline__ uint32_t group_item_cur(const uint32_t *B, const uint32_t *P, uint32_t L, uint32_t W,
+                                                   uint32_t q, const LaneGroup &g) {
+  uint32_t lo = 0, hi = L;   // j1 = last row with P[j1] <= q
+  while (hi - lo > 1) {
+    const uint32_t mid = (lo + hi) >> 1;
+    if (P[mid] <= q) lo = mid; else hi = mid;
+  }
+  const uint32_t j1 = lo, r = q - P[j1];
+  const uint32_t w1 = g.gl < (int)W ? B[j1 * W + g.gl] : 0u;
+  // the r-th set bit of row j1: inclusive scan of the word popcounts over the group
+  const uint32_t pc = __popc(w1);
+  uint32_t inc = pc;
+#pragma unroll
+  for (int o = 1; o < kGroup; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(g.mask, inc, o);
+    if (g.gl >= o) inc += y;
+  }
+  const bool mine = r < inc && r >= inc - pc;
+  const uint32_t bal = __ballot_sync(g.mask, mine);
+  const int src = __ffs(bal) - 1;
+  const uint32_t j2b = mine ? (uint32_t)g.gl * 32 + __fns(w1, 0, r - (inc - pc) + 1) : 0u;
+  const uint32_t j2 = __shfl_sync(g.mask, j2b, src);
+  const uint32_t w2 = g.gl < (int)W ? B[j2 * W + g.gl] : 0u;
+  return w1 & w2;
+}
+
 template <int TEAM_WARPS>
 __device__ __forceinline__ void team_sync() {
   if (TEAM_WARPS == 1) __syncwarp();
@@ -213,10 +405,10 @@ struct TeamMem {
 // global scratch slice (wide runs).
 template <int TEAM_WARPS>
 __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H, uint32_t *B, uint64_t b0,
-                                 uint32_t L, int tid, int lane) {
+                                 uint32_t L, int tid, int lane, uint32_t stride) {
   constexpr int kTeamThreads = TEAM_WARPS * 32;
   const int wit = tid >> 5;
-  const uint32_t W = (L + 31) >> 5;
+  const uint32_t W = stride;   // row stride in words (>= the row's (L + 31) / 32 words)
   uint32_t hbits = 2;
   while ((1u << hbits) < 4 * L) hbits++;
   const uint32_t hmask = (1u << hbits) - 1u;
@@ -254,26 +446,36 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
     const uint32_t o = excl_scan32(cdl, lane, T);
     const uint32_t upto = lane == 31 ? 0xffffffffu : ((2u << lane) - 1u);
     uint32_t nb = 0;   // lists that started before this tile
-    for (uint32_t t0 = 0; t0 < T; t0 += 32) {
-      const uint32_t t = t0 + lane;
-      // lane t's list = the last list starting at or before t: one OR-reduction of the
-      // start offsets that fall in this tile
-      const uint32_t mine = (lane < (int)nnz && o >= t0 && o < t0 + 32) ? (1u << (o - t0)) : 0u;
-      const uint32_t S = __reduce_or_sync(0xffffffffu, mine);
-      const int j = (int)(nb + __popc(S & upto)) - 1;
-      nb += __popc(S);
-      const uint32_t bj = __shfl_sync(0xffffffffu, cbeg, j & 31);
-      const uint32_t oj = __shfl_sync(0xffffffffu, o, j & 31);
-      const uint32_t rj = __shfl_sync(0xffffffffu, crow, j & 31);
-      if (t < T) {
-        const uint32_t y = __ldg(a.dag_col + bj + (t - oj));
-        if (y >= rmin && y <= rmax) {
-          uint32_t h = (y * 0x9E3779B1u) >> (32 - hbits);
+    // kTiles tiles of 32 elements per step: their loads are issued back to back
+    // before any probe, so each lane keeps several L2 gathers in flight
+    constexpr int kTiles = 4;
+    for (uint32_t t0 = 0; t0 < T; t0 += 32 * kTiles) {
+      uint32_t y[kTiles], rj[kTiles];
+#pragma unroll
+      for (int u = 0; u < kTiles; u++) {
+        const uint32_t tb = t0 + 32 * u;
+        const uint32_t t = tb + lane;
+        // lane t's list = the last list starting at or before t: one OR-reduction of
+        // the start offsets that fall in this tile
+        const uint32_t mine = (lane < (int)nnz && o >= tb && o < tb + 32) ? (1u << (o - tb)) : 0u;
+        const uint32_t S = __reduce_or_sync(0xffffffffu, mine);
+        const int j = (int)(nb + __popc(S & upto)) - 1;
+        nb += __popc(S);
+        const uint32_t bj = __shfl_sync(0xffffffffu, cbeg, j & 31);
+        const uint32_t oj = __shfl_sync(0xffffffffu, o, j & 31);
+        rj[u] = __shfl_sync(0xffffffffu, crow, j & 31);
+        y[u] = t < T ? __ldg(a.dag_col + bj + (t - oj)) : 0xffffffffu;
+      }
+#pragma unroll
+      for (int u = 0; u < kTiles; u++) {
+        const uint32_t yy = y[u];
+        if (yy >= rmin && yy <= rmax) {   // (the padding 0xffffffff is above every rmax < n)
+          uint32_t h = (yy * 0x9E3779B1u) >> (32 - hbits);
           for (;;) {
             const uint32_t e = H[h];
             if (e == 0) break;
-            if (R[e - 1] == y) {
-              atomicOr(&B[rj * W + ((e - 1) >> 5)], 1u << ((e - 1) & 31));
+            if (R[e - 1] == yy) {
+              atomicOr(&B[rj[u] * W + ((e - 1) >> 5)], 1u << ((e - 1) & 31));
               break;
             }
             h = (h + 1) & hmask;
@@ -286,23 +488,30 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
   return elems;
 }
 
+// Row stride in shared memory: TW words for warp teams (16-byte rows, one vector
+// load each), the row's own W words for CTA teams.
+template <int TEAM_WARPS, int TW>
+__device__ __forceinline__ uint32_t row_stride(uint32_t L) {
+  return TEAM_WARPS == 1 ? (uint32_t)TW : (L + 31) >> 5;
+}
+
 template <int TEAM_WARPS, int TW>
 __device__ __forceinline__ uint64_t build_rows(const BmArgs &a, const TeamMem<TW> &m, uint64_t b0, uint32_t L,
                                                int tid, int lane) {
-  return build_rows_p<TEAM_WARPS>(a, m.R, m.H, m.B, b0, L, tid, lane);
+  return build_rows_p<TEAM_WARPS>(a, m.R, m.H, m.B, b0, L, tid, lane, row_stride<TEAM_WARPS, TW>(L));
 }
 
 // P[r] = exclusive scan of the row popcounts (the triangle items), P[L] = total.
 template <int TEAM_WARPS, int TW>
 __device__ void scan_rows(const TeamMem<TW> &m, uint32_t L, int tid, int lane) {
-  const uint32_t W = (L + 31) >> 5;
+  const uint32_t W = (L + 31) >> 5, BS = row_stride<TEAM_WARPS, TW>(L);
   if ((tid >> 5) == 0) {
     uint32_t carry = 0;
     for (uint32_t r0 = 0; r0 < L; r0 += 32) {
       const uint32_t r = r0 + lane;
       uint32_t c = 0;
       if (r < L)
-        for (uint32_t w = 0; w < W; w++) c += __popc(m.B[r * W + w]);
+        for (uint32_t w = 0; w < W; w++) c += __popc(m.B[r * BS + w]);
       uint32_t tot;
       const uint32_t ex = excl_scan32(c, lane, tot);
       if (r < L) m.P[r] = carry + ex;
@@ -315,7 +524,7 @@ __device__ void scan_rows(const TeamMem<TW> &m, uint32_t L, int tid, int lane) {
 
 // Item q -> candidates of the triangle (v, R[j1], R[j2]).
 template <int TW>
-__device__ __forceinline__ void item_cur(const TeamMem<TW> &m, uint32_t L, uint32_t W, uint32_t q,
+__device__ __forceinline__ void item_cur(const TeamMem<TW> &m, uint32_t L, uint32_t W, uint32_t BS, uint32_t q,
                                          uint32_t (&cur)[TW]) {
   uint32_t lo = 0, hi = L;   // j1 = last row with P[j1] <= q
   while (hi - lo > 1) {
@@ -325,7 +534,7 @@ __device__ __forceinline__ void item_cur(const TeamMem<TW> &m, uint32_t L, uint3
   const uint32_t j1 = lo;
   uint32_t r = q - m.P[j1], j2 = 0;
   for (uint32_t w = 0; w < W; w++) {
-    const uint32_t word = m.B[j1 * W + w];
+    const uint32_t word = m.B[j1 * BS + w];
     const uint32_t pc = __popc(word);
     if (r < pc) {
       j2 = w * 32 + __fns(word, 0, r + 1);
@@ -334,7 +543,7 @@ __device__ __forceinline__ void item_cur(const TeamMem<TW> &m, uint32_t L, uint3
     r -= pc;
   }
 #pragma unroll
-  for (int w = 0; w < TW; w++) cur[w] = (w < (int)W) ? (m.B[j1 * W + w] & m.B[j2 * W + w]) : 0u;
+  for (int w = 0; w < TW; w++) cur[w] = (w < (int)W) ? (m.B[j1 * BS + w] & m.B[j2 * BS + w]) : 0u;
 }
 
 template <int TEAM_WARPS>
@@ -354,7 +563,9 @@ __device__ __forceinline__ uint64_t team_sum(uint64_t x, int lane, uint32_t *slo
 }
 
 __device__ __forceinline__ void flush_multi(uint64_t (&mc)[kMaxStack + 3], const BmArgs &a, int lane) {
-  for (uint32_t sz = 3; sz <= a.k && sz < kMaxStack + 3; sz++) {
+#pragma unroll
+  for (uint32_t sz = 3; sz < kMaxStack + 3; sz++) {   // unrolled: mc stays in registers
+    if (sz > a.k) break;
     uint64_t x = mc[sz];
 #pragma unroll
     for (int off = 16; off > 0; off >>= 1) x += __shfl_down_sync(0xffffffffu, x, off);
@@ -362,7 +573,9 @@ __device__ __forceinline__ void flush_multi(uint64_t (&mc)[kMaxStack + 3], const
   }
 }
 
-template <int TEAM_WARPS, int TW, bool PER_ROOT>
+// KM: compile-time bound on k for the register-resident DFS of warp teams (6 or 12;
+// the deeper instantiation needs more registers, so k <= 6 gets its own kernel).
+template <int TEAM_WARPS, int TW, bool PER_ROOT, int KM>
 __global__ void __launch_bounds__(256) kcl_bitmap_kernel(BmArgs a) {
   extern __shared__ uint32_t smem[];
   constexpr int kTeamThreads = TEAM_WARPS * 32;
@@ -398,7 +611,7 @@ __global__ void __launch_bounds__(256) kcl_bitmap_kernel(BmArgs a) {
     const uint64_t b0 = a.dag_ptr[v];
     const uint32_t L = (uint32_t)(a.dag_ptr[v + 1] - b0);
     if (L <= a.len_lo || L > a.len_hi || L < (a.multi ? 2u : a.k - 1)) continue;   // uniform across the team
-    const uint32_t W = (L + 31) >> 5;
+    const uint32_t W = (L + 31) >> 5, BS = row_stride<TEAM_WARPS, TW>(L);
     if (tid == 0) entries += L;
     elems += build_rows<TEAM_WARPS, TW>(a, m, b0, L, tid, lane);
     // ---- deeper extensions: bitmap DFS.  k = 3: one row per thread (its popcount).
@@ -407,7 +620,7 @@ __global__ void __launch_bounds__(256) kcl_bitmap_kernel(BmArgs a) {
     if (a.k == 3) {
       for (uint32_t j1 = tid; j1 < L; j1 += kTeamThreads) {
         uint32_t c = 0;
-        for (uint32_t w = 0; w < W; w++) c += __popc(m.B[j1 * W + w]);
+        for (uint32_t w = 0; w < W; w++) c += __popc(m.B[j1 * BS + w]);
         cnt += c;
       }
       if (a.multi) mc[3] += cnt;
@@ -419,7 +632,7 @@ __global__ void __launch_bounds__(256) kcl_bitmap_kernel(BmArgs a) {
         uint64_t est = 0;
         for (uint32_t q = tid; q < items; q += kTeamThreads) {
           uint32_t cur[TW];
-          item_cur<TW>(m, L, W, q, cur);
+          item_cur<TW>(m, L, W, BS, q, cur);
           uint32_t c = 0;
 #pragma unroll
           for (int w = 0; w < TW; w++) c += __popc(cur[w]);
@@ -444,17 +657,34 @@ __global__ void __launch_bounds__(256) kcl_bitmap_kernel(BmArgs a) {
           team_sync<TEAM_WARPS>();
         }
       }
-      if (!deferred)
+      if (TEAM_WARPS == 1 && !deferred)
         for (uint32_t q = tid; q < items; q += kTeamThreads) {
           uint32_t cur[TW];
-          item_cur<TW>(m, L, W, q, cur);
-          if (a.multi) {
-            mc[3] += 1;   // the item is one triangle
-            dfs_multi<TW>(m.B, W, cur, 3, a.k, mc);
-          } else {
-            cnt += dfs_count<TW>(m.B, W, cur, 3, a.k);
+          item_cur<TW>(m, L, W, BS, q, cur);
+          if constexpr (TEAM_WARPS == 1) {   // register-resident nested loops
+            if (a.multi) {
+              mc[3] += 1;   // the item is one triangle
+              rdfs_multi<TW, 3, KM, kMaxStack + 3>(m.B, cur, a.k, mc);
+            } else {
+              cnt += rdfs_count<TW, 3, KM>(m.B, cur, a.k);
+            }
           }
         }
+      if constexpr (TEAM_WARPS > 1) {   // lane groups: one triangle item per 16-lane group
+        if (!deferred) {
+          const LaneGroup g = lane_group(lane);
+          constexpr uint32_t kGroups = kTeamThreads / kGroup;
+          for (uint32_t q = tid / kGroup; q < items; q += kGroups) {
+            const uint32_t curw = group_item_cur(m.B, m.P, L, W, q, g);
+            if (a.multi) {
+              if (g.gl == 0) mc[3] += 1;   // the item is one triangle
+              gdfs_multi<3, KM, kMaxStack + 3>(m.B, W, curw, a.k, mc, g);
+            } else {
+              cnt += gdfs_count<3, KM>(m.B, W, curw, a.k, g);
+            }
+          }
+        }
+      }
     }
     total += cnt;
     if (PER_ROOT) {
@@ -480,7 +710,7 @@ __global__ void __launch_bounds__(256) kcl_bitmap_kernel(BmArgs a) {
 
 // Second launch for the deferred heavy roots: one CTA per (root, part); the part
 // rebuilds the root's rows (cheap next to the DFS) and takes every nparts-th item.
-template <bool PER_ROOT>
+template <bool PER_ROOT, int KM>
 __global__ void __launch_bounds__(256) kcl_bitmap_parts_kernel(BmArgs a) {
   extern __shared__ uint32_t smem[];
   constexpr int TW = 16;
@@ -511,14 +741,15 @@ __global__ void __launch_bounds__(256) kcl_bitmap_parts_kernel(BmArgs a) {
     scan_rows<8, TW>(m, L, tid, lane);
     const uint32_t items = m.P[L];
     uint64_t cnt = 0;
-    for (uint32_t q = part + tid * nparts; q < items; q += 256 * nparts) {
-      uint32_t cur[TW];
-      item_cur<TW>(m, L, W, q, cur);
+    const LaneGroup g = lane_group(lane);
+    constexpr uint32_t kGroups = 256 / kGroup;
+    for (uint32_t q = part + (tid / kGroup) * nparts; q < items; q += kGroups * nparts) {
+      const uint32_t curw = group_item_cur(m.B, m.P, L, W, q, g);
       if (a.multi) {
-        mc[3] += 1;
-        dfs_multi<TW>(m.B, W, cur, 3, a.k, mc);
+        if (g.gl == 0) mc[3] += 1;
+        gdfs_multi<3, KM, kMaxStack + 3>(m.B, W, curw, a.k, mc, g);
       } else {
-        cnt += dfs_count<TW>(m.B, W, cur, 3, a.k);
+        cnt += gdfs_count<3, KM>(m.B, W, curw, a.k, g);
       }
     }
     total += cnt;
@@ -605,7 +836,65 @@ __device__ uint64_t wide_dfs(const uint32_t *B, uint32_t W, const uint32_t (&cur
   return cnt;
 }
 
-template <int WL, bool PER_ROOT>
+// Register-resident variants of wide_dfs (template recursion over the chosen-vertex
+// count S; SM = compile-time bound on k): the per-level candidate slices and the bits
+// still to visit stay in registers instead of a local-memory stack.
+template <int WL, int S, int SM, int N>
+__device__ __forceinline__ void wdfs_multi(const uint32_t *B, uint32_t W, const uint32_t (&cur)[WL], uint32_t kmax,
+                                           uint64_t (&mc)[N], int lane) {
+  static_assert(SM < N, "counter array too short");
+  uint32_t c = 0;
+#pragma unroll
+  for (int t = 0; t < WL; t++) c += __popc(cur[t]);
+  mc[S + 1] += c;
+  if constexpr (S + 1 < SM) {
+    if (S + 1 >= kmax) return;
+    uint32_t rem[WL];
+#pragma unroll
+    for (int t = 0; t < WL; t++) rem[t] = cur[t];
+    for (;;) {
+      const int j = wide_pop_next<WL>(rem, lane);
+      if (j < 0) break;
+      uint32_t nx[WL];
+#pragma unroll
+      for (int t = 0; t < WL; t++) {
+        const uint32_t w = lane + 32 * t;
+        nx[t] = w < W ? (cur[t] & B[(uint64_t)j * W + w]) : 0u;
+      }
+      wdfs_multi<WL, S + 1, SM, N>(B, W, nx, kmax, mc, lane);
+    }
+  }
+}
+
+template <int WL, int S, int SM>
+__device__ __forceinline__ uint64_t wdfs_count(const uint32_t *B, uint32_t W, const uint32_t (&cur)[WL], uint32_t k,
+                                               int lane) {
+  uint32_t c = 0;
+#pragma unroll
+  for (int t = 0; t < WL; t++) c += __popc(cur[t]);
+  if (S + 1 == k) return c;   // this lane's share
+  uint64_t cnt = 0;
+  if constexpr (S + 1 < SM) {
+    if (__reduce_add_sync(0xffffffffu, c) < k - S) return 0;
+    uint32_t rem[WL];
+#pragma unroll
+    for (int t = 0; t < WL; t++) rem[t] = cur[t];
+    for (;;) {
+      const int j = wide_pop_next<WL>(rem, lane);
+      if (j < 0) break;
+      uint32_t nx[WL];
+#pragma unroll
+      for (int t = 0; t < WL; t++) {
+        const uint32_t w = lane + 32 * t;
+        nx[t] = w < W ? (cur[t] & B[(uint64_t)j * W + w]) : 0u;
+      }
+      cnt += wdfs_count<WL, S + 1, SM>(B, W, nx, k, lane);
+    }
+  }
+  return cnt;
+}
+
+template <int WL, bool PER_ROOT, int KM>
 __global__ void __launch_bounds__(kWideThreads) kcl_wide_kernel(BmArgs a) {
   extern __shared__ uint32_t smem[];
   constexpr int kMaxL = 1024 * WL;
@@ -634,7 +923,7 @@ __global__ void __launch_bounds__(kWideThreads) kcl_wide_kernel(BmArgs a) {
     }
     const uint32_t W = (L + 31) >> 5;
     if (tid == 0) entries += L;
-    elems += build_rows_p<kWideThreads / 32>(a, R, H, B, b0, L, tid, lane);
+    elems += build_rows_p<kWideThreads / 32>(a, R, H, B, b0, L, tid, lane, W);
     uint64_t cnt = 0;
     for (;;) {
       uint32_t i = 0;
@@ -649,13 +938,15 @@ __global__ void __launch_bounds__(kWideThreads) kcl_wide_kernel(BmArgs a) {
         cur[t] = w < W ? B[(uint64_t)i * W + w] : 0u;
         c += __popc(cur[t]);
       }
-      if (a.multi) mc[3] += c;
       if (a.k == 3) {
+        if (a.multi) mc[3] += c;
         cnt += c;
         continue;
       }
-      if (__reduce_add_sync(0xffffffffu, c) == 0) continue;
-      cnt += wide_dfs<WL>(B, W, cur, 2, a.k, a.multi != 0, mc, lane);
+      if (a.multi)
+        wdfs_multi<WL, 2, KM, kMaxStack + 3>(B, W, cur, a.k, mc, lane);   // adds mc[3] += c itself
+      else
+        cnt += wdfs_count<WL, 2, KM>(B, W, cur, a.k, lane);
     }
     total += cnt;
     if (PER_ROOT) {
@@ -685,18 +976,19 @@ constexpr size_t wide_smem() {
 }
 
 // rows scratch: grid x (run length x words) for the longest run of the launch
-template <int WL>
-void enqueue_wide(gamma_ctx *ctx, BmArgs a, bool per_root, uint32_t max_len, DevBuf<uint32_t> &rows) {
+template <int WL, int KM>
+void enqueue_wide_km(gamma_ctx *ctx, BmArgs a, bool per_root, uint32_t max_len, DevBuf<uint32_t> &rows) {
   static bool attr = false;
   if (!attr) {
-    GAMMA_CUDA(cudaFuncSetAttribute(kcl_wide_kernel<WL, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    GAMMA_CUDA(cudaFuncSetAttribute(kcl_wide_kernel<WL, false, KM>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                     (int)wide_smem<WL>()));
-    GAMMA_CUDA(cudaFuncSetAttribute(kcl_wide_kernel<WL, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    GAMMA_CUDA(cudaFuncSetAttribute(kcl_wide_kernel<WL, true, KM>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                     (int)wide_smem<WL>()));
     attr = true;
   }
   static int grid = 0;
-  if (!grid) grid = ctx->num_sms * occupancy_blocks((const void *)kcl_wide_kernel<WL, false>, kWideThreads, wide_smem<WL>());
+  if (!grid)
+    grid = ctx->num_sms * occupancy_blocks((const void *)kcl_wide_kernel<WL, false, KM>, kWideThreads, wide_smem<WL>());
   const uint64_t L = std::min<uint64_t>(max_len, 1024u * WL);
   a.wide_stride = L * ((L + 31) / 32);
   const uint64_t g = std::min<uint64_t>(grid, a.nroots);
@@ -705,10 +997,18 @@ void enqueue_wide(gamma_ctx *ctx, BmArgs a, bool per_root, uint32_t max_len, Dev
   GAMMA_CUDA(cudaMemsetAsync(ctx->ctrl + CTRL_WORK, 0, sizeof(uint64_t), ctx->stream));
   ctx->launch(KC_BITMAP, [&] {
     if (per_root)
-      kcl_wide_kernel<WL, true><<<(unsigned)g, kWideThreads, wide_smem<WL>(), ctx->stream>>>(a);
+      kcl_wide_kernel<WL, true, KM><<<(unsigned)g, kWideThreads, wide_smem<WL>(), ctx->stream>>>(a);
     else
-      kcl_wide_kernel<WL, false><<<(unsigned)g, kWideThreads, wide_smem<WL>(), ctx->stream>>>(a);
+      kcl_wide_kernel<WL, false, KM><<<(unsigned)g, kWideThreads, wide_smem<WL>(), ctx->stream>>>(a);
   });
+}
+
+template <int WL>
+void enqueue_wide(gamma_ctx *ctx, BmArgs a, bool per_root, uint32_t max_len, DevBuf<uint32_t> &rows) {
+  if (a.k <= 6)
+    enqueue_wide_km<WL, 6>(ctx, a, per_root, max_len, rows);
+  else
+    enqueue_wide_km<WL, kBitmapMaxK>(ctx, a, per_root, max_len, rows);
 }
 
 template <int TEAM_WARPS, int TW>
@@ -718,48 +1018,64 @@ constexpr size_t bm_smem() {
 
 // Enqueue one team kind over a root range (no host round trip: the work counter is
 // reset on the stream, the counts accumulate in ctrl and are read once at the end).
-template <int TEAM_WARPS, int TW>
-void enqueue_bitmap(gamma_ctx *ctx, const BmArgs &a0, bool per_root) {
+template <int TEAM_WARPS, int TW, int KM>
+void enqueue_bitmap_km(gamma_ctx *ctx, const BmArgs &a0, bool per_root) {
   static bool attr = false;
   if (!attr) {
-    GAMMA_CUDA(cudaFuncSetAttribute(kcl_bitmap_kernel<TEAM_WARPS, TW, false>,
+    GAMMA_CUDA(cudaFuncSetAttribute(kcl_bitmap_kernel<TEAM_WARPS, TW, false, KM>,
                                     cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bm_smem<TEAM_WARPS, TW>()));
-    GAMMA_CUDA(cudaFuncSetAttribute(kcl_bitmap_kernel<TEAM_WARPS, TW, true>,
+    GAMMA_CUDA(cudaFuncSetAttribute(kcl_bitmap_kernel<TEAM_WARPS, TW, true, KM>,
                                     cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bm_smem<TEAM_WARPS, TW>()));
     attr = true;
   }
   const size_t smem = bm_smem<TEAM_WARPS, TW>();
   static int grid = 0;
   if (!grid)
-    grid = ctx->num_sms * occupancy_blocks((const void *)kcl_bitmap_kernel<TEAM_WARPS, TW, false>, 256, smem);
+    grid = ctx->num_sms * occupancy_blocks((const void *)kcl_bitmap_kernel<TEAM_WARPS, TW, false, KM>, 256, smem);
   GAMMA_CUDA(cudaMemsetAsync(ctx->ctrl + CTRL_WORK, 0, sizeof(uint64_t), ctx->stream));
   ctx->launch(KC_BITMAP, [&] {
     if (per_root)
-      kcl_bitmap_kernel<TEAM_WARPS, TW, true><<<grid, 256, smem, ctx->stream>>>(a0);
+      kcl_bitmap_kernel<TEAM_WARPS, TW, true, KM><<<grid, 256, smem, ctx->stream>>>(a0);
     else
-      kcl_bitmap_kernel<TEAM_WARPS, TW, false><<<grid, 256, smem, ctx->stream>>>(a0);
+      kcl_bitmap_kernel<TEAM_WARPS, TW, false, KM><<<grid, 256, smem, ctx->stream>>>(a0);
   });
 }
 
-void enqueue_parts(gamma_ctx *ctx, const BmArgs &a0, bool per_root) {
+template <int TEAM_WARPS, int TW>
+void enqueue_bitmap(gamma_ctx *ctx, const BmArgs &a0, bool per_root) {
+  if (a0.k <= 6)
+    enqueue_bitmap_km<TEAM_WARPS, TW, 6>(ctx, a0, per_root);
+  else
+    enqueue_bitmap_km<TEAM_WARPS, TW, kBitmapMaxK>(ctx, a0, per_root);
+}
+
+template <int KM>
+void enqueue_parts_km(gamma_ctx *ctx, const BmArgs &a0, bool per_root) {
   static bool attr = false;
   if (!attr) {
-    GAMMA_CUDA(cudaFuncSetAttribute(kcl_bitmap_parts_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    GAMMA_CUDA(cudaFuncSetAttribute(kcl_bitmap_parts_kernel<false, KM>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                     (int)bm_smem<8, 16>()));
-    GAMMA_CUDA(cudaFuncSetAttribute(kcl_bitmap_parts_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    GAMMA_CUDA(cudaFuncSetAttribute(kcl_bitmap_parts_kernel<true, KM>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                     (int)bm_smem<8, 16>()));
     attr = true;
   }
   static int pgrid = 0;
   if (!pgrid)
-    pgrid = ctx->num_sms * occupancy_blocks((const void *)kcl_bitmap_parts_kernel<false>, 256, bm_smem<8, 16>());
+    pgrid = ctx->num_sms * occupancy_blocks((const void *)kcl_bitmap_parts_kernel<false, KM>, 256, bm_smem<8, 16>());
   GAMMA_CUDA(cudaMemsetAsync(ctx->ctrl + CTRL_WORK, 0, sizeof(uint64_t), ctx->stream));
   ctx->launch(KC_BITMAP, [&] {
     if (per_root)
-      kcl_bitmap_parts_kernel<true><<<pgrid, 256, bm_smem<8, 16>(), ctx->stream>>>(a0);
+      kcl_bitmap_parts_kernel<true, KM><<<pgrid, 256, bm_smem<8, 16>(), ctx->stream>>>(a0);
     else
-      kcl_bitmap_parts_kernel<false><<<pgrid, 256, bm_smem<8, 16>(), ctx->stream>>>(a0);
+      kcl_bitmap_parts_kernel<false, KM><<<pgrid, 256, bm_smem<8, 16>(), ctx->stream>>>(a0);
   });
+}
+
+void enqueue_parts(gamma_ctx *ctx, const BmArgs &a0, bool per_root) {
+  if (a0.k <= 6)
+    enqueue_parts_km<6>(ctx, a0, per_root);
+  else
+    enqueue_parts_km<kBitmapMaxK>(ctx, a0, per_root);
 }
 
 }  // namespace

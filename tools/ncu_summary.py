@@ -2,7 +2,10 @@
 """Summarise an `ncu --set full` report into profiles/ncu_full_<class>.json (one file
 per kernel class, averaged over the captured launches) plus a markdown table.
 
-    python tools/ncu_summary.py gpurun_out/prof.ncu-rep profiles/ <round-tag>
+    python tools/ncu_summary.py gpurun_out/prof.ncu-rep profiles/ <round-tag> [<workload>]
+
+With a workload name the files are profiles/ncu_<workload>_<class>.json (read by
+bench.py's roofline "traffic" for that workload) and ncu_<workload>_<tag>.md.
 
 Kernel classes follow the library's stats names: kcl_kernel<0,..> extend,
 <1,..> count, <2,..> fused, kcl_bitmap_kernel bitmap, sm_kernel sm_extend,
@@ -26,6 +29,7 @@ METRICS = {
     "sm_throughput_pct": ("sm__throughput.avg.pct_of_peak_sustained_elapsed", 1.0),
     "dram_throughput_pct": ("gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed", 1.0),
     "issue_active_pct": ("sm__inst_issued.avg.pct_of_peak_sustained_active", 1.0),
+    "threads_per_warp_inst": ("smsp__thread_inst_executed_per_inst_executed.ratio", 1.0),
     "inst_executed": ("smsp__inst_executed.sum", 1.0),
     "registers": ("launch__registers_per_thread", 1.0),
     "grid": ("launch__grid_size", 1.0),
@@ -54,6 +58,7 @@ def kclass(name: str) -> str:
 
 def main():
     rep, outdir, tag = sys.argv[1], sys.argv[2], sys.argv[3] if len(sys.argv) > 3 else "r01"
+    prefix = f"ncu_{sys.argv[4]}_" if len(sys.argv) > 4 else "ncu_full_"
     raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
     rows = list(csv.reader(io.StringIO(raw)))
     hdr, units = rows[0], rows[1]
@@ -91,13 +96,14 @@ def main():
                    "sm_throughput_pct": avg("sm_throughput_pct"), "dram_throughput_pct": avg("dram_throughput_pct"),
                    "inst_executed_per_launch": avg("inst_executed"), "registers": avg("registers"),
                    "source": os.path.basename(rep), "launches": recs}
-        with open(os.path.join(outdir, f"ncu_full_{c}.json"), "w") as f:
+        summary["threads_per_warp_inst"] = avg("threads_per_warp_inst")
+        with open(os.path.join(outdir, f"{prefix}{c}.json"), "w") as f:
             json.dump(summary, f, indent=1)
         fmt = lambda x, p=1: "-" if x is None else f"{x:.{p}f}"   # noqa: E731
         lines.append(f"| {c} | {len(recs)} | {fmt(avg('duration_ms'), 3)} | {dram:.3e} | {fmt(avg('l2_hit_pct'))} | "
                      f"{fmt(avg('warps_active_pct'))} | {fmt(avg('issue_active_pct'))} | "
                      f"{fmt(avg('sm_throughput_pct'))} | {fmt(avg('dram_throughput_pct'))} | {fmt(avg('registers'), 0)} |")
-    with open(os.path.join(outdir, f"ncu_full_{tag}.md"), "w") as f:
+    with open(os.path.join(outdir, f"{prefix}{tag}.md"), "w") as f:
         f.write(f"ncu --set full summary of {os.path.basename(rep)} ({tag})\n\n" + "\n".join(lines) + "\n")
     print("\n".join(lines))
 
