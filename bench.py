@@ -367,6 +367,8 @@ def run_gamma(args):
             results = {f"frequent_l{l}": sum(1 for p in pats if p[0] == l) for l in range(1, w["l"] + 1)}
             emb = st["level_entries"][w["l"]]
             results["embeddings_l"] = emb
+            results["domain_chunk_passes"] = st.get("chunks")
+            results["table_retries"] = st.get("retries")
         info = g.info()
         g.free()
         return emb, results, info

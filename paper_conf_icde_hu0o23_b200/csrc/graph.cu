@@ -11,6 +11,8 @@
 // duplicates removed by a unique pass; row_ptr / col produced by one fused
 // boundary kernel.  Everything stays in HBM; the only host sync is to learn m.
 #include <cub/device/device_radix_sort.cuh>
+#include <cub/device/device_scan.cuh>
+#include <cub/device/device_segmented_sort.cuh>
 #include <cub/device/device_select.cuh>
 
 #include "internal.cuh"
@@ -140,6 +142,114 @@ __global__ void csr_symmetry_kernel(const uint64_t *__restrict__ rp, const uint3
   }
 }
 
+__global__ void narrow_u64_kernel(const uint64_t *__restrict__ in, uint64_t n, uint32_t *__restrict__ out) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+    out[i] = (uint32_t)in[i];
+}
+
+// ---- counting-sort builder (A1 when 2m' < 2^31): degree count -> scan -> scatter ->
+// segmented sort of each row -> per-row dedup, all row-local after the scatter ----
+__global__ void raw_degree_kernel(const uint32_t *__restrict__ src, const uint32_t *__restrict__ dst, uint64_t m,
+                                  uint32_t n, uint32_t *__restrict__ cnt, unsigned long long *err) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < m; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t u = src[i], v = dst[i];
+    if (u >= n || v >= n) {
+      atomicOr(err, 1ull);
+      continue;
+    }
+    if (u == v) continue;   // no self-loops
+    atomicAdd(&cnt[u], 1u);
+    atomicAdd(&cnt[v], 1u);
+  }
+}
+
+__global__ void raw_scatter_kernel(const uint32_t *__restrict__ src, const uint32_t *__restrict__ dst, uint64_t m,
+                                   uint32_t n, const uint32_t *__restrict__ off, uint32_t *__restrict__ cur,
+                                   uint32_t *__restrict__ col) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < m; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t u = src[i], v = dst[i];
+    if (u >= n || v >= n || u == v) continue;
+    col[off[u] + atomicAdd(&cur[u], 1u)] = v;
+    col[off[v] + atomicAdd(&cur[v], 1u)] = u;
+  }
+}
+
+// One warp per row of the sorted raw lists: number of distinct entries.
+__global__ void row_unique_count_kernel(const uint32_t *__restrict__ off, const uint32_t *__restrict__ col,
+                                        uint32_t n, uint64_t *__restrict__ deg) {
+  const int lane = threadIdx.x & 31;
+  for (uint64_t v = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5; v < n;
+       v += ((uint64_t)gridDim.x * blockDim.x) >> 5) {
+    const uint32_t s = off[v], e = off[v + 1];
+    uint32_t c = 0;
+    for (uint32_t i0 = s; i0 < e; i0 += 32) {
+      const uint32_t i = i0 + lane;
+      const bool keep = i < e && (i == s || col[i] != col[i - 1]);
+      c += __popc(__ballot_sync(0xffffffffu, keep));
+    }
+    if (lane == 0) deg[v] = c;
+  }
+}
+
+// One warp per row: write the distinct entries at row_ptr[v] (ballot compaction) and
+// count the DAG out-degree: keep v->x iff (deg v, v) < (deg x, x).
+__global__ void row_unique_write_kernel(const uint32_t *__restrict__ off, const uint32_t *__restrict__ col_in,
+                                        uint32_t n, const uint64_t *__restrict__ row_ptr,
+                                        uint32_t *__restrict__ col, uint64_t *__restrict__ dcnt) {
+  const int lane = threadIdx.x & 31;
+  const uint32_t below = (1u << lane) - 1u;
+  for (uint64_t v = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5; v < n;
+       v += ((uint64_t)gridDim.x * blockDim.x) >> 5) {
+    const uint32_t s = off[v], e = off[v + 1];
+    const uint64_t dv = row_ptr[v + 1] - row_ptr[v];
+    uint64_t w = row_ptr[v];
+    uint32_t dc = 0;
+    for (uint32_t i0 = s; i0 < e; i0 += 32) {
+      const uint32_t i = i0 + lane;
+      uint32_t x = 0;
+      bool keep = false;
+      if (i < e) {
+        x = col_in[i];
+        keep = i == s || x != col_in[i - 1];
+      }
+      const uint32_t bal = __ballot_sync(0xffffffffu, keep);
+      if (keep) {
+        col[w + __popc(bal & below)] = x;
+        const uint64_t dx = row_ptr[x + 1] - row_ptr[x];
+        dc += (dv < dx || (dv == dx && (uint32_t)v < x)) ? 1u : 0u;
+      }
+      w += __popc(bal);
+    }
+    for (int o = 16; o > 0; o >>= 1) dc += __shfl_down_sync(0xffffffffu, dc, o);
+    if (lane == 0) dcnt[v] = dc;
+  }
+}
+
+// One warp per row: the DAG list = the row filtered by the orientation (stays sorted).
+__global__ void dag_write_kernel(const uint64_t *__restrict__ row_ptr, const uint32_t *__restrict__ col, uint32_t n,
+                                 const uint64_t *__restrict__ dag_ptr, uint32_t *__restrict__ dag_col) {
+  const int lane = threadIdx.x & 31;
+  const uint32_t below = (1u << lane) - 1u;
+  for (uint64_t v = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5; v < n;
+       v += ((uint64_t)gridDim.x * blockDim.x) >> 5) {
+    const uint64_t s = row_ptr[v], e = row_ptr[v + 1], dv = e - s;
+    uint64_t w = dag_ptr[v];
+    for (uint64_t i0 = s; i0 < e; i0 += 32) {
+      const uint64_t i = i0 + lane;
+      uint32_t x = 0;
+      bool keep = false;
+      if (i < e) {
+        x = col[i];
+        const uint64_t dx = row_ptr[x + 1] - row_ptr[x];
+        keep = dv < dx || (dv == dx && (uint32_t)v < x);
+      }
+      const uint32_t bal = __ballot_sync(0xffffffffu, keep);
+      if (keep) dag_col[w + __popc(bal & below)] = x;
+      w += __popc(bal);
+    }
+  }
+}
+
 uint32_t bit_width(uint32_t n) {  // bits to represent n itself
   uint32_t b = 0;
   while (b < 32 && (uint64_t(1) << b) <= n) b++;
@@ -233,6 +343,106 @@ void build_dag(gamma_graph *g, uint64_t *keys, uint64_t M) {
   g->max_out_degree = max_degree(ctx, g->dag_ptr, g->n);
 }
 
+namespace {
+
+template <class T>
+void exclusive_sum(gamma_ctx *ctx, const T *in, uint64_t *out, uint64_t n) {
+  size_t tmp = 0;
+  GAMMA_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tmp, in, out, (int64_t)n, ctx->stream));
+  DevBuf<uint8_t> t(ctx, tmp);
+  ctx->launch(KC_BUILD, [&] { GAMMA_CUDA(cub::DeviceScan::ExclusiveSum(t.p, tmp, in, out, (int64_t)n, ctx->stream)); });
+  ctx->extra_launches(KC_BUILD, 1);   // init + scan
+}
+
+uint64_t read_u64(gamma_ctx *ctx, const uint64_t *p) {
+  uint64_t h = 0;
+  GAMMA_CUDA(cudaMemcpyAsync(&h, p, sizeof(uint64_t), cudaMemcpyDeviceToHost, ctx->stream));
+  ctx->sync();
+  return h;
+}
+
+// A1 without a global key sort (inputs with 2m' < 2^31): count each vertex's raw
+// degree, scatter every sample into its two rows, sort each row (CUB segmented sort),
+// then one warp per row drops duplicates, writes the symmetric list and counts the
+// DAG out-degree; a last warp-per-row pass writes the DAG lists (filtered rows stay
+// sorted).  Same result as the key-sort builder: symmetric, self-loop free,
+// duplicate free, ascending lists (O-0).
+void build_counting(gamma_graph *g, const uint32_t *src, const uint32_t *dst, uint64_t m) {
+  gamma_ctx *ctx = g->ctx;
+  const uint32_t n = g->n;
+  DevBuf<uint32_t> cnt(ctx, (size_t)n + 1);
+  GAMMA_CUDA(cudaMemsetAsync(cnt.p, 0, ((size_t)n + 1) * 4, ctx->stream));
+  GAMMA_CUDA(cudaMemsetAsync(ctx->ctrl + CTRL_ERR, 0, sizeof(uint64_t), ctx->stream));
+  ctx->launch(KC_BUILD, [&] {
+    raw_degree_kernel<<<grid_for(m), kThreads, 0, ctx->stream>>>(src, dst, m, n, cnt.p,
+                                                                  (unsigned long long *)(ctx->ctrl + CTRL_ERR));
+  });
+  DevBuf<uint64_t> off64(ctx, (size_t)n + 1);
+  exclusive_sum(ctx, cnt.p, off64.p, (uint64_t)n + 1);
+  uint64_t h[2] = {0, 0};
+  GAMMA_CUDA(cudaMemcpyAsync(&h[0], off64.p + n, sizeof(uint64_t), cudaMemcpyDeviceToHost, ctx->stream));
+  GAMMA_CUDA(cudaMemcpyAsync(&h[1], ctx->ctrl + CTRL_ERR, sizeof(uint64_t), cudaMemcpyDeviceToHost, ctx->stream));
+  ctx->sync();
+  GAMMA_REQUIRE(h[1] == 0, GAMMA_E_INVAL, "gamma_load_edges: vertex id >= n");
+  const uint64_t total = h[0];   // 2 x (samples without self-loops) < 2^31
+  // 32-bit row offsets for the segmented sort (total < 2^31)
+  DevBuf<uint32_t> off(ctx, (size_t)n + 1);
+  ctx->launch(KC_BUILD, [&] {
+    narrow_u64_kernel<<<grid_for((uint64_t)n + 1), kThreads, 0, ctx->stream>>>(off64.p, (uint64_t)n + 1, off.p);
+  });
+  off64.reset();
+  GAMMA_CUDA(cudaMemsetAsync(cnt.p, 0, ((size_t)n + 1) * 4, ctx->stream));
+  DevBuf<uint32_t> raw(ctx, total ? total : 1), sorted(ctx, total ? total : 1);
+  ctx->launch(KC_BUILD, [&] {
+    raw_scatter_kernel<<<grid_for(m), kThreads, 0, ctx->stream>>>(src, dst, m, n, off.p, cnt.p, raw.p);
+  });
+  cnt.reset();
+  if (total) {
+    size_t tmp = 0;
+    GAMMA_CUDA(cub::DeviceSegmentedSort::SortKeys(nullptr, tmp, raw.p, sorted.p, (int)total, (int)n, off.p,
+                                                  off.p + 1, ctx->stream));
+    DevBuf<uint8_t> t(ctx, tmp);
+    ctx->launch(KC_BUILD, [&] {
+      GAMMA_CUDA(cub::DeviceSegmentedSort::SortKeys(t.p, tmp, raw.p, sorted.p, (int)total, (int)n, off.p, off.p + 1,
+                                                    ctx->stream));
+    });
+    ctx->extra_launches(KC_BUILD, 2);   // partition + small/medium + large segment kernels
+  }
+  raw.reset();
+  const unsigned wgrid = grid_for((uint64_t)n * 32);
+  DevBuf<uint64_t> deg(ctx, (size_t)n + 1);
+  GAMMA_CUDA(cudaMemsetAsync(deg.p + n, 0, sizeof(uint64_t), ctx->stream));
+  ctx->launch(KC_BUILD, [&] { row_unique_count_kernel<<<wgrid, kThreads, 0, ctx->stream>>>(off.p, sorted.p, n, deg.p); });
+  DevBuf<uint64_t> rp(ctx, (size_t)n + 1);
+  exclusive_sum(ctx, deg.p, rp.p, (uint64_t)n + 1);
+  const uint64_t M = read_u64(ctx, rp.p + n);
+  GAMMA_REQUIRE(M % 2 == 0, GAMMA_E_CUDA, "asymmetric rows after dedup");
+  DevBuf<uint32_t> col(ctx, M ? M : 1);
+  GAMMA_CUDA(cudaMemsetAsync(deg.p + n, 0, sizeof(uint64_t), ctx->stream));   // deg reused as DAG counts
+  ctx->launch(KC_BUILD, [&] {
+    row_unique_write_kernel<<<wgrid, kThreads, 0, ctx->stream>>>(off.p, sorted.p, n, rp.p, col.p, deg.p);
+  });
+  sorted.reset();
+  off.reset();
+  DevBuf<uint64_t> dp(ctx, (size_t)n + 1);
+  exclusive_sum(ctx, deg.p, dp.p, (uint64_t)n + 1);
+  const uint64_t mdag = read_u64(ctx, dp.p + n);
+  GAMMA_REQUIRE(mdag == M / 2, GAMMA_E_CUDA, "DAG orientation kept " + std::to_string(mdag) + " of " +
+                                                 std::to_string(M / 2) + " edges");
+  DevBuf<uint32_t> dc(ctx, mdag ? mdag : 1);
+  ctx->launch(KC_BUILD, [&] { dag_write_kernel<<<wgrid, kThreads, 0, ctx->stream>>>(rp.p, col.p, n, dp.p, dc.p); });
+  g->m = M / 2;
+  g->row_ptr = rp.release();
+  g->col = col.release();
+  g->dag_ptr = dp.release();
+  g->dag_col = dc.release();
+  g->device_bytes += 2 * (((uint64_t)n + 1) * 8) + M * 4 + mdag * 4;
+  g->max_degree = max_degree(ctx, g->row_ptr, n);
+  g->max_out_degree = max_degree(ctx, g->dag_ptr, n);
+}
+
+}  // namespace
+
 void build_from_edges(gamma_graph *g, const uint32_t *src, const uint32_t *dst, uint64_t m,
                       bool on_device) {
   gamma_ctx *ctx = g->ctx;
@@ -246,6 +456,11 @@ void build_from_edges(gamma_graph *g, const uint32_t *src, const uint32_t *dst, 
     d_copy = to_device(ctx, dst, m);
     src = s_copy.p;
     dst = d_copy.p;
+  }
+  if (m && 2 * m < (1ull << 31) && (ctx->desc.flags & GAMMA_FLAG_KEY_SORT_BUILD) == 0) {
+    build_counting(g, src, dst, m);
+    g->build_ms = timer.stop();
+    return;
   }
   const uint64_t nkeys = 2 * m;
   uint64_t M = 0;

@@ -308,37 +308,63 @@ __device__ __forceinline__ int group_next(const LaneGroup &g, uint32_t &rem) {
   return (src - g.base) * 32 + __ffs(word) - 1;
 }
 
+// A node whose children are leaves only needs sum over children j of popc(cur & B[j])
+// (the edges inside cur): the group broadcasts cur to all its lanes and each lane
+// walks the children in its own word, reading whole rows (odd row stride: no bank
+// conflicts between lanes), so no per-child ballot/shuffle is needed.
+__device__ __forceinline__ uint32_t group_leaf_sum(const uint32_t *B, uint32_t BS, uint32_t W, uint32_t curw,
+                                                   const LaneGroup &g) {
+  uint32_t cur[kGroup];
+#pragma unroll
+  for (int w = 0; w < kGroup; w++) cur[w] = __shfl_sync(g.mask, curw, g.base + w);
+  uint32_t acc = 0, bits = curw;
+  while (bits) {
+    const uint32_t j = (uint32_t)g.gl * 32 + __ffs(bits) - 1;
+    bits &= bits - 1u;
+    const uint32_t *row = B + j * BS;
+#pragma unroll
+    for (int w = 0; w < kGroup; w++)
+      if (w < (int)W) acc += __popc(cur[w] & row[w]);
+  }
+  return acc;
+}
+
 template <int S, int SM, int N>
-__device__ __forceinline__ void gdfs_multi(const uint32_t *B, uint32_t W, uint32_t curw, uint32_t kmax,
+__device__ __forceinline__ void gdfs_multi(const uint32_t *B, uint32_t BS, uint32_t W, uint32_t curw, uint32_t kmax,
                                            uint64_t (&mc)[N], const LaneGroup &g) {
   static_assert(SM < N, "counter array too short");
   mc[S + 1] += __popc(curw);
   if constexpr (S + 1 < SM) {
     if (S + 1 >= kmax) return;
+    if (S + 2 == kmax) {   // children are leaves
+      mc[S + 2] += group_leaf_sum(B, BS, W, curw, g);
+      return;
+    }
     uint32_t rem = curw;
     for (;;) {
       const int j = group_next(g, rem);
       if (j < 0) break;
-      const uint32_t row = g.gl < (int)W ? B[(uint32_t)j * W + g.gl] : 0u;
-      gdfs_multi<S + 1, SM, N>(B, W, curw & row, kmax, mc, g);
+      const uint32_t row = g.gl < (int)W ? B[(uint32_t)j * BS + g.gl] : 0u;
+      gdfs_multi<S + 1, SM, N>(B, BS, W, curw & row, kmax, mc, g);
     }
   }
 }
 
 template <int S, int SM>
-__device__ __forceinline__ uint64_t gdfs_count(const uint32_t *B, uint32_t W, uint32_t curw, uint32_t k,
+__device__ __forceinline__ uint64_t gdfs_count(const uint32_t *B, uint32_t BS, uint32_t W, uint32_t curw, uint32_t k,
                                                const LaneGroup &g) {
   if (S + 1 == k) return __popc(curw);
   uint64_t cnt = 0;
   if constexpr (S + 1 < SM) {
+    if (S + 2 == k) return group_leaf_sum(B, BS, W, curw, g);
     const uint32_t c = __reduce_add_sync(g.mask, __popc(curw));
     if (c < k - S) return 0;
     uint32_t rem = curw;
     for (;;) {
       const int j = group_next(g, rem);
       if (j < 0) break;
-      const uint32_t row = g.gl < (int)W ? B[(uint32_t)j * W + g.gl] : 0u;
-      cnt += gdfs_count<S + 1, SM>(B, W, curw & row, k, g);
+      const uint32_t row = g.gl < (int)W ? B[(uint32_t)j * BS + g.gl] : 0u;
+      cnt += gdfs_count<S + 1, SM>(B, BS, W, curw & row, k, g);
     }
   }
   return cnt;
@@ -346,14 +372,14 @@ __device__ __forceinline__ uint64_t gdfs_count(const uint32_t *B, uint32_t W, ui
 
 // Item q -> this lane's word of the candidates of the triangle (v, R[j1], R[j2]).
 __device__ __forceinline__ uint32_t group_item_cur(const uint32_t *B, const uint32_t *P, uint32_t L, uint32_t W,
-                                                   uint32_t q, const LaneGroup &g) {
+                                                   uint32_t BS, uint32_t q, const LaneGroup &g) {
   uint32_t lo = 0, hi = L;   // j1 = last row with P[j1] <= q
   while (hi - lo > 1) {
     const uint32_t mid = (lo + hi) >> 1;
     if (P[mid] <= q) lo = mid; else hi = mid;
   }
   const uint32_t j1 = lo, r = q - P[j1];
-  const uint32_t w1 = g.gl < (int)W ? B[j1 * W + g.gl] : 0u;
+  const uint32_t w1 = g.gl < (int)W ? B[j1 * BS + g.gl] : 0u;
   // the r-th set bit of row j1: inclusive scan of the word popcounts over the group
   const uint32_t pc = __popc(w1);
   uint32_t inc = pc;
@@ -367,7 +393,7 @@ __device__ __forceinline__ uint32_t group_item_cur(const uint32_t *B, const uint
   const int src = __ffs(bal) - 1;
   const uint32_t j2b = mine ? (uint32_t)g.gl * 32 + __fns(w1, 0, r - (inc - pc) + 1) : 0u;
   const uint32_t j2 = __shfl_sync(g.mask, j2b, src);
-  const uint32_t w2 = g.gl < (int)W ? B[j2 * W + g.gl] : 0u;
+  const uint32_t w2 = g.gl < (int)W ? B[j2 * BS + g.gl] : 0u;
   return w1 & w2;
 }
 
@@ -377,23 +403,30 @@ __device__ __forceinline__ void team_sync() {
   else __syncthreads();
 }
 
-// Shared words per team: run R (32 TW), bitmap rows B (32 TW x TW), position hash
-// H (4 x 32 TW u16 = 64 TW words), row offsets P (32 TW + 1, padded to +2), two
-// broadcast slots (8-byte aligned: every region starts at an even word).
+// Shared words per team: run R (32 TW), bitmap rows B (32 TW x TW), position hash:
+// positions H (4 x 32 TW u16 = 64 TW words) and the vertex ids of the slots Hv
+// (4 x 32 TW words), row offsets P (32 TW + 1, padded to +2), two broadcast slots
+// (8-byte aligned: every region starts at an even word).
+template <int TW>
+constexpr int row_words_max() {   // largest row stride (see row_stride)
+  return TW == 4 ? 4 : TW + 1;
+}
+
 template <int TW>
 constexpr int team_words() {
-  return TW * 32 + TW * 32 * TW + 2 * TW * 32 + TW * 32 + 2 + 2;
+  return TW * 32 + TW * 32 * row_words_max<TW>() + 2 * TW * 32 + 4 * TW * 32 + TW * 32 + 2 + 2;
 }
 
 template <int TW>
 struct TeamMem {
-  uint32_t *R, *B, *P, *slot;
+  uint32_t *R, *B, *P, *slot, *Hv;
   unsigned short *H;
   __device__ TeamMem(uint32_t *base) {
     R = base;
     B = R + TW * 32;
-    H = reinterpret_cast<unsigned short *>(B + TW * 32 * TW);
-    P = B + TW * 32 * TW + 2 * TW * 32;
+    H = reinterpret_cast<unsigned short *>(B + TW * 32 * row_words_max<TW>());
+    Hv = B + TW * 32 * row_words_max<TW>() + 2 * TW * 32;
+    P = Hv + 4 * TW * 32;
     slot = P + TW * 32 + 2;
   }
 };
@@ -403,9 +436,15 @@ struct TeamMem {
 // shared-memory open-addressing position table.  Returns Σ|N+(c)| (for the bytes).
 // R and H live in shared memory; B in shared memory (<= 512-long runs) or in a
 // global scratch slice (wide runs).
+// With Hv (team kernels) the slot's vertex id is stored beside its position, so a
+// probe compares ids directly and checks two slots without branching; only when both
+// are taken by other ids (rare at load <= 1/4) does it walk the chain.  Without Hv
+// (wide runs, whose tables would not fit) the position table alone is probed.
+constexpr uint32_t kEmptyId = 0xffffffffu;   // vertex ids are < n <= 2^32 - 1
+
 template <int TEAM_WARPS>
 __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H, uint32_t *B, uint64_t b0,
-                                 uint32_t L, int tid, int lane, uint32_t stride) {
+                                 uint32_t L, int tid, int lane, uint32_t stride, uint32_t *Hv = nullptr) {
   constexpr int kTeamThreads = TEAM_WARPS * 32;
   const int wit = tid >> 5;
   const uint32_t W = stride;   // row stride in words (>= the row's (L + 31) / 32 words)
@@ -414,11 +453,21 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
   const uint32_t hmask = (1u << hbits) - 1u;
   for (uint32_t i = tid; i < L; i += kTeamThreads) R[i] = a.dag_col[b0 + i];
   for (uint32_t i = tid; i < L * W; i += kTeamThreads) B[i] = 0u;
-  for (uint32_t i = tid; i <= hmask / 2; i += kTeamThreads) reinterpret_cast<uint32_t *>(H)[i] = 0u;
+  if (Hv) {
+    for (uint32_t i = tid; i <= hmask; i += kTeamThreads) Hv[i] = kEmptyId;
+  } else {
+    for (uint32_t i = tid; i <= hmask / 2; i += kTeamThreads) reinterpret_cast<uint32_t *>(H)[i] = 0u;
+  }
   team_sync<TEAM_WARPS>();
   for (uint32_t i = tid; i < L; i += kTeamThreads) {
-    uint32_t h = (R[i] * 0x9E3779B1u) >> (32 - hbits);
-    while (atomicCAS(&H[h], (unsigned short)0, (unsigned short)(i + 1)) != 0) h = (h + 1) & hmask;
+    const uint32_t x = R[i];
+    uint32_t h = (x * 0x9E3779B1u) >> (32 - hbits);
+    if (Hv) {
+      while (atomicCAS(&Hv[h], kEmptyId, x) != kEmptyId) h = (h + 1) & hmask;
+      H[h] = (unsigned short)i;
+    } else {
+      while (atomicCAS(&H[h], (unsigned short)0, (unsigned short)(i + 1)) != 0) h = (h + 1) & hmask;
+    }
   }
   team_sync<TEAM_WARPS>();
   const uint32_t rmin = R[0], rmax = R[L - 1];
@@ -469,6 +518,28 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
 #pragma unroll
       for (int u = 0; u < kTiles; u++) {
         const uint32_t yy = y[u];
+        if (Hv) {
+          if (yy < rmin || yy > rmax) continue;   // (the padding 0xffffffff is above every rmax < n)
+          const uint32_t h0 = (yy * 0x9E3779B1u) >> (32 - hbits), h1 = (h0 + 1) & hmask;
+          const uint32_t v0 = Hv[h0], v1 = Hv[h1];
+          int e = -1;
+          if (v0 == yy) {
+            e = H[h0];
+          } else if (v1 == yy) {
+            e = H[h1];
+          } else if (v0 != kEmptyId && v1 != kEmptyId) {
+            for (uint32_t h = (h1 + 1) & hmask;; h = (h + 1) & hmask) {
+              const uint32_t vh = Hv[h];
+              if (vh == yy) {
+                e = H[h];
+                break;
+              }
+              if (vh == kEmptyId) break;
+            }
+          }
+          if (e >= 0) atomicOr(&B[rj[u] * W + ((uint32_t)e >> 5)], 1u << (e & 31));
+          continue;
+        }
         if (yy >= rmin && yy <= rmax) {   // (the padding 0xffffffff is above every rmax < n)
           uint32_t h = (yy * 0x9E3779B1u) >> (32 - hbits);
           for (;;) {
@@ -489,16 +560,18 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
 }
 
 // Row stride in shared memory: TW words for warp teams (16-byte rows, one vector
-// load each), the row's own W words for CTA teams.
+// load each); for CTA teams the row's own W words rounded up to an odd count, so that
+// lanes reading the same word of different rows hit different banks (the
+// lane-parallel leaf loop of the group DFS).
 template <int TEAM_WARPS, int TW>
 __device__ __forceinline__ uint32_t row_stride(uint32_t L) {
-  return TEAM_WARPS == 1 ? (uint32_t)TW : (L + 31) >> 5;
+  return TEAM_WARPS == 1 ? (uint32_t)TW : (((L + 31) >> 5) | 1u);
 }
 
 template <int TEAM_WARPS, int TW>
 __device__ __forceinline__ uint64_t build_rows(const BmArgs &a, const TeamMem<TW> &m, uint64_t b0, uint32_t L,
                                                int tid, int lane) {
-  return build_rows_p<TEAM_WARPS>(a, m.R, m.H, m.B, b0, L, tid, lane, row_stride<TEAM_WARPS, TW>(L));
+  return build_rows_p<TEAM_WARPS>(a, m.R, m.H, m.B, b0, L, tid, lane, row_stride<TEAM_WARPS, TW>(L), m.Hv);
 }
 
 // P[r] = exclusive scan of the row popcounts (the triangle items), P[L] = total.
@@ -675,12 +748,12 @@ __global__ void __launch_bounds__(256) kcl_bitmap_kernel(BmArgs a) {
           const LaneGroup g = lane_group(lane);
           constexpr uint32_t kGroups = kTeamThreads / kGroup;
           for (uint32_t q = tid / kGroup; q < items; q += kGroups) {
-            const uint32_t curw = group_item_cur(m.B, m.P, L, W, q, g);
+            const uint32_t curw = group_item_cur(m.B, m.P, L, W, BS, q, g);
             if (a.multi) {
               if (g.gl == 0) mc[3] += 1;   // the item is one triangle
-              gdfs_multi<3, KM, kMaxStack + 3>(m.B, W, curw, a.k, mc, g);
+              gdfs_multi<3, KM, kMaxStack + 3>(m.B, BS, W, curw, a.k, mc, g);
             } else {
-              cnt += gdfs_count<3, KM>(m.B, W, curw, a.k, g);
+              cnt += gdfs_count<3, KM>(m.B, BS, W, curw, a.k, g);
             }
           }
         }
@@ -736,7 +809,7 @@ __global__ void __launch_bounds__(256) kcl_bitmap_parts_kernel(BmArgs a) {
     const uint32_t v = a.roots[gi];
     const uint64_t b0 = a.dag_ptr[v];
     const uint32_t L = (uint32_t)(a.dag_ptr[v + 1] - b0);
-    const uint32_t W = (L + 31) >> 5;
+    const uint32_t W = (L + 31) >> 5, BS = row_stride<8, TW>(L);
     build_rows<8, TW>(a, m, b0, L, tid, lane);
     scan_rows<8, TW>(m, L, tid, lane);
     const uint32_t items = m.P[L];
@@ -744,12 +817,12 @@ __global__ void __launch_bounds__(256) kcl_bitmap_parts_kernel(BmArgs a) {
     const LaneGroup g = lane_group(lane);
     constexpr uint32_t kGroups = 256 / kGroup;
     for (uint32_t q = part + (tid / kGroup) * nparts; q < items; q += kGroups * nparts) {
-      const uint32_t curw = group_item_cur(m.B, m.P, L, W, q, g);
+      const uint32_t curw = group_item_cur(m.B, m.P, L, W, BS, q, g);
       if (a.multi) {
         if (g.gl == 0) mc[3] += 1;
-        gdfs_multi<3, KM, kMaxStack + 3>(m.B, W, curw, a.k, mc, g);
+        gdfs_multi<3, KM, kMaxStack + 3>(m.B, BS, W, curw, a.k, mc, g);
       } else {
-        cnt += gdfs_count<3, KM>(m.B, W, curw, a.k, g);
+        cnt += gdfs_count<3, KM>(m.B, BS, W, curw, a.k, g);
       }
     }
     total += cnt;

@@ -298,3 +298,44 @@ def test_c2_full_size(ctx, oracle_mod):
     assert g.info()["m"] == o.m
     for k in (4, 5, 6):
         assert g.kclique(k) == o.kclique(k), k
+
+
+@pytest.mark.parametrize("case", ["c1", "er", "dups", "selfloops", "one"])
+def test_builders_agree(G, ctx, oracle_mod, case):
+    """A1 has two builders -- counting sort + segmented row sort (default below 2^31
+    directed entries) and the global key sort (GAMMA_FLAG_KEY_SORT_BUILD, used above);
+    both must give the oracle's O-0 CSR and the same DAG."""
+    if case == "c1":
+        n, s, d, _ = gg.config_graph("c1", seed=2)
+    elif case == "er":
+        n = 5000
+        s, d = gg.er(n, 40000, 3)
+    elif case == "dups":
+        n = 64
+        s = np.array([1, 2, 1, 2, 3, 3, 5, 1] * 50, np.uint32)
+        d = np.array([2, 1, 2, 1, 4, 4, 1, 5] * 50, np.uint32)
+    elif case == "selfloops":
+        n = 10
+        s = np.arange(10, dtype=np.uint32)
+        d = s.copy()
+    else:
+        n = 2
+        s, d = np.array([0], np.uint32), np.array([1], np.uint32)
+    key = G.Context(device=0, flags=0x80)
+    g1, g2 = ctx.load_edges(n, s, d), key.load_edges(n, s, d)
+    o = oracle_mod.Graph(n, s, d)
+    orp, ocol = o.csr()
+    for g in (g1, g2):
+        rp, col = g.csr("sym")
+        assert np.array_equal(rp, orp) and np.array_equal(col, ocol)
+        assert g.info()["max_degree"] == (int(np.diff(orp.astype(np.int64)).max()) if n else 0)
+    d1, d2 = g1.csr("dag"), g2.csr("dag")
+    assert np.array_equal(d1[0], d2[0]) and np.array_equal(d1[1], d2[1])
+    assert g1.info()["max_out_degree"] == g2.info()["max_out_degree"]
+
+
+def test_builder_rejects_bad_ids(ctx):
+    s = np.array([0, 7], np.uint32)
+    d = np.array([1, 2], np.uint32)
+    with pytest.raises(Exception):
+        ctx.load_edges(4, s, d)
