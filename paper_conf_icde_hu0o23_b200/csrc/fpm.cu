@@ -15,12 +15,16 @@
 //  * The levels < l are regenerated per level rather than stored (DFS per root
 //    edge); Alg. 2's pruning is applied at every generated prefix by looking its
 //    pattern up in the pattern table (infrequent prefix => no extension).
-//  * Canonical code: sort the <= 4 vertex labels (the minimal label sequence), then
-//    enumerate only the label-consistent vertex orders and keep the minimal sorted
-//    edge-pair list; every minimizing order is an automorphic placement, so OR-ing
-//    the vertex of each position into that position's domain merges orbits (MNI).
+//  * Canonical code: a 5-comparator sorting network puts the <= 4 vertex labels in
+//    order (the minimal label sequence); the minimal sorted edge-pair list and the
+//    set of minimizing vertex orders then depend only on the edge mask in sorted
+//    positions and on which neighbouring sorted labels tie, read from a 512-entry
+//    shared-memory table built on the host by enumerating the 24 orders (no per-
+//    embedding permutation loop, all in registers).  Every minimizing order is an
+//    automorphic placement, so OR-ing the vertex of each position into that
+//    position's domain merges orbits (MNI).
 //  * Pattern table: lock-free open-addressing hash (one-word code -> slot, claimed
-//    by a single atomicCAS) in HBM, sized from the number of label combinations so
+//    by a single atomicCAS; key and domain offset share one 16-byte slot) in HBM, sized from the number of label combinations so
 //    probe chains stay short; the claimer carves the slot's MNI domains from a pool:
 //    one bitmap per position over the vertices of that position's label class (bit
 //    index = rank of the vertex inside its class), so memory follows the patterns
@@ -29,6 +33,8 @@
 #include <cub/device/device_select.cuh>
 
 #include <algorithm>
+#include <cstdio>
+#include <cstdlib>
 #include <array>
 #include <chrono>
 #include <unordered_map>
@@ -903,6 +909,10 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
       // a level's domains are dead once its supports are known (the next level reads
       // only freq): clear what it used and carve the next level from offset 0
       uint64_t dirty = std::min<uint64_t>(carved, pool_words);
+      if (getenv("GAMMA_DEBUG"))
+        fprintf(stderr, "[gamma_fpm] level %u: budget %.2f GB, table cap %llu, pool %.2f GB, carved %.2f GB, ovf %llu\n",
+                l, budget / 1e9, (unsigned long long)cap, pool_words * 4 / 1e9, carved * 4 / 1e9,
+                (unsigned long long)ctx->ctrl_host[CTRL_OVF]);
       const auto clear_pool = [&] {
         if (dirty) GAMMA_CUDA(cudaMemsetAsync(pool.p, 0, dirty * 4, ctx->stream));
         GAMMA_CUDA(cudaMemsetAsync(pcur.p, 0, 8, ctx->stream));

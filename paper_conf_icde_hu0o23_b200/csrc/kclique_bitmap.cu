@@ -312,21 +312,29 @@ __device__ __forceinline__ int group_next(const LaneGroup &g, uint32_t &rem) {
 // (the edges inside cur): the group broadcasts cur to all its lanes and each lane
 // walks the children in its own word, reading whole rows (odd row stride: no bank
 // conflicts between lanes), so no per-child ballot/shuffle is needed.
-__device__ __forceinline__ uint32_t group_leaf_sum(const uint32_t *B, uint32_t BS, uint32_t W, uint32_t curw,
-                                                   const LaneGroup &g) {
-  uint32_t cur[kGroup];
+template <int WW>   // compile-time word bound (>= W): predicated-off words still issue
+__device__ __forceinline__ uint32_t group_leaf_sum_w(const uint32_t *B, uint32_t BS, uint32_t W, uint32_t curw,
+                                                     const LaneGroup &g) {
+  uint32_t cur[WW];
 #pragma unroll
-  for (int w = 0; w < kGroup; w++) cur[w] = __shfl_sync(g.mask, curw, g.base + w);
+  for (int w = 0; w < WW; w++) cur[w] = __shfl_sync(g.mask, curw, g.base + w);
   uint32_t acc = 0, bits = curw;
   while (bits) {
     const uint32_t j = (uint32_t)g.gl * 32 + __ffs(bits) - 1;
     bits &= bits - 1u;
     const uint32_t *row = B + j * BS;
 #pragma unroll
-    for (int w = 0; w < kGroup; w++)
+    for (int w = 0; w < WW; w++)
       if (w < (int)W) acc += __popc(cur[w] & row[w]);
   }
   return acc;
+}
+
+__device__ __forceinline__ uint32_t group_leaf_sum(const uint32_t *B, uint32_t BS, uint32_t W, uint32_t curw,
+                                                   const LaneGroup &g) {
+  if (W <= 4) return group_leaf_sum_w<4>(B, BS, W, curw, g);
+  if (W <= 8) return group_leaf_sum_w<8>(B, BS, W, curw, g);
+  return group_leaf_sum_w<kGroup>(B, BS, W, curw, g);
 }
 
 template <int S, int SM, int N>
