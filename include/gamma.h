@@ -92,9 +92,10 @@ typedef struct {
                                           (no local-bitmap DFS; ablation / testing)  */
 #define GAMMA_FLAG_NO_SPLIT     0x20u  /* kCL bitmap path: never split heavy roots    */
 #define GAMMA_FLAG_DEBUG_SPLIT_ALL 0x40u /* test hook: split every root (k >= 6)      */
-#define GAMMA_FLAG_KEY_SORT_BUILD 0x80u /* gamma_load_edges: always use the global key-sort
-                                          builder (the counting-sort builder is the default
-                                          when 2m' < 2^31; both give the same CSR)          */
+#define GAMMA_FLAG_COUNT_SORT_BUILD 0x80u /* gamma_load_edges: counting sort + segmented row
+                                          sort instead of the global key sort (2m' < 2^31
+                                          only; same CSR; slower on hub-heavy graphs, where
+                                          the hub rows fall to CUB's large-segment kernel) */
 
 /* Create / destroy a context.  Errors: E_INVAL (NULL args), E_CUDA (no device). */
 gamma_status gamma_ctx_create(const gamma_ctx_desc *desc, gamma_ctx **out);

@@ -36,6 +36,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <array>
+#include <tuple>
 #include <chrono>
 #include <unordered_map>
 #include <vector>
@@ -96,6 +97,8 @@ struct FpmArgs {
   uint32_t level;            // edges per recorded embedding
   uint32_t rank, world;      // root partition: this rank takes edge batches b = rank (mod world)
   uint32_t claim_only;       // claim pattern slots without carving domains (distributed level)
+  uint32_t carve_below;      // carve domains only for patterns whose smallest label is below this
+  uint32_t walk_lo;          // last-level chunk pass: skip every embedding with a label < walk_lo
   Table T;
   unsigned long long *ctrl;
 };
@@ -144,7 +147,9 @@ __device__ int64_t table_slot(const FpmArgs &a, uint64_t key, bool insert, unsig
         // the claimer carves the slot's domains: one bitmap per position, sized to the
         // position's label class
         unsigned long long d = ~0ull;
-        if (!a.claim_only) {
+        if (!a.claim_only && key_label(key, 0) >= a.carve_below) {
+          atomicExch(&a.ctrl[CTRL_OVF], 1ull);   // left for a later, label-pruned pass
+        } else if (!a.claim_only) {
           const uint32_t nv = key_nv(key);
           uint64_t words = 0;
           for (uint32_t p = 0; p < nv; p++) words += __ldg(a.cwords + key_label(key, p));
@@ -318,6 +323,7 @@ __global__ void __launch_bounds__(kThreads) fpm_enum_kernel(FpmArgs a) {
       const uint64_t us = a.rp[u], ue = a.rp[u + 1];
       const uint64_t e1 = ekey(u, v);
       const uint32_t lu = labof(a, u), lv = labof(a, v);
+      if (lu < a.walk_lo || lv < a.walk_lo) continue;   // uniform; 0 except in chunk passes
       if (a.level == 1) {
         if (lane == 0) {
           record(a, s_tab, s_prm, u, v, 0u, 0u, lu, lv, 0u, 0u, 2, 1u << pid(0, 1));
@@ -345,6 +351,9 @@ __global__ void __launch_bounds__(kThreads) fpm_enum_kernel(FpmArgs a) {
         }
         if (valid) {
           ly = labof(a, y);
+          valid = ly >= a.walk_lo;
+        }
+        if (valid) {
           if (a.level == 2) {
             record(a, s_tab, s_prm, u, v, y, 0u, lu, lv, ly, 0u, 3, em2);
             emb++;
@@ -413,8 +422,9 @@ __global__ void __launch_bounds__(kThreads) fpm_enum_kernel(FpmArgs a) {
           const bool ok = (e3 > pe2) || (e3 > e1 && shares(e3, pe2) && !shares(e3, e1));
           if (!ok) continue;
           const uint32_t em3 = (pl >> 16) | (1u << pid(lw, lz));
-          record(a, s_tab, s_prm, u, v, py, z, lu, lv, pl & 0xffffu, lz == 3 ? labof(a, z) : 0u, lz == 3 ? 4 : 3,
-                 em3);
+          const uint32_t l3 = lz == 3 ? labof(a, z) : 0u;
+          if (lz == 3 && l3 < a.walk_lo) continue;
+          record(a, s_tab, s_prm, u, v, py, z, lu, lv, pl & 0xffffu, l3, lz == 3 ? 4 : 3, em3);
           emb++;
         }
       }
@@ -782,6 +792,41 @@ static bool fpm_dist_level(gamma_ctx *ctx, FpmArgs &a, int grid_enum, uint32_t l
   return true;
 }
 
+// Worst-case MNI domain words of the level-l patterns, by the pattern's smallest label
+// (every label combination of every shape occurring; shapes: edge; wedge; triangle,
+// 3-star, 3-path).  Used to pick the label threshold below which the first pass of a
+// level carves domains, so that the patterns left for the chunk passes all have large
+// smallest labels -- and a chunk pass with smallest label lo skips every root edge,
+// prefix and new vertex labelled below lo (few embeddings have only large labels).
+static std::vector<double> fpm_words_by_min_label(uint32_t l, const std::vector<uint32_t> &cw) {
+  const uint32_t L = (uint32_t)cw.size();
+  std::vector<double> W(L, 0.0);
+  if (l == 1) {
+    for (uint32_t a = 0; a < L; a++)
+      for (uint32_t b = a; b < L; b++) W[a] += cw[a] + cw[b];
+  } else if (l == 2) {
+    for (uint32_t c = 0; c < L; c++)
+      for (uint32_t x = 0; x < L; x++)
+        for (uint32_t y = x; y < L; y++) W[std::min(c, x)] += cw[c] + cw[x] + cw[y];
+  } else if (l == 3) {
+    for (uint32_t a = 0; a < L; a++)
+      for (uint32_t b = a; b < L; b++)
+        for (uint32_t c = b; c < L; c++) W[a] += cw[a] + cw[b] + cw[c];   // triangles
+    for (uint32_t c = 0; c < L; c++)                                         // 3-stars
+      for (uint32_t x = 0; x < L; x++)
+        for (uint32_t y = x; y < L; y++)
+          for (uint32_t z = y; z < L; z++) W[std::min(c, x)] += cw[c] + cw[x] + cw[y] + cw[z];
+    for (uint32_t a = 0; a < L; a++)                                         // 3-paths a-b-c-d
+      for (uint32_t b = 0; b < L; b++)
+        for (uint32_t c = 0; c < L; c++)
+          for (uint32_t d = 0; d < L; d++) {
+            if (std::make_tuple(a, b, c, d) > std::make_tuple(d, c, b, a)) continue;   // one per reversal
+            W[std::min(std::min(a, b), std::min(c, d))] += cw[a] + cw[b] + cw[c] + cw[d];
+          }
+  }
+  return W;
+}
+
 static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::vector<gamma_fpm_pattern> &out) {
   gamma_ctx *ctx = g->ctx;
   const uint32_t n = g->n;
@@ -859,6 +904,8 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
   a.n = n;
   a.rank = 0;
   a.world = 1;   // levels < l run on every rank; the last one is split when dist
+  a.carve_below = 0xffffffffu;
+  a.walk_lo = 0;
   // multi-GPU: the last level is partitioned over the ranks and its domains OR-reduced
   // (fpm_dist_level); without the collectives every rank computes everything
   const bool dist = ctx->desc.world > 1 && ctx->desc.allreduce_sum_u64 && ctx->desc.alltoall_u32;
@@ -889,11 +936,26 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
         break;
       }
       a.level = l;
+      // first pass of the level: carve domains only for patterns whose smallest label
+      // is below T, the largest threshold whose worst-case domains fit the pool (all
+      // labels when everything fits); the rest go to label-pruned chunk passes
+      a.carve_below = 0xffffffffu;
+      if (l >= 2 && nlab <= 64) {
+        const std::vector<double> W = fpm_words_by_min_label(l, hwords);
+        double acc = 0, total = 0;
+        for (double w : W) total += w;
+        if (total > (double)pool_words) {
+          uint32_t T = 0;
+          while (T < nlab && acc + W[T] <= (double)pool_words) acc += W[T++];
+          a.carve_below = std::max<uint32_t>(T, 1);
+        }
+      }
       ctrl_reset(ctx);
       ctx->launch(KC_FPM, [&] { fpm_enum_kernel<<<grid_enum, kThreads, 0, ctx->stream>>>(a); });
       ctx->launch(KC_FPM_SUPPORT, [&] {
         fpm_support_kernel<<<g1d(cap * 32), 256, 0, ctx->stream>>>(a, l, minsup);
       });
+      a.carve_below = 0xffffffffu;
       uint64_t carved = 0;
       GAMMA_CUDA(cudaMemcpyAsync(&carved, pcur.p, 8, cudaMemcpyDeviceToHost, ctx->stream));
       ctrl_fetch(ctx);
@@ -934,9 +996,13 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
       std::vector<uint64_t> pending;
       for (uint64_t s = 0; s < cap; s++)
         if (hkey[s] && key_ne(hkey[s]) == l && hdom[s] == ~0ull) pending.push_back(s);
+      // by smallest label: a chunk's pass skips every embedding with a smaller label
+      std::stable_sort(pending.begin(), pending.end(),
+                       [&](uint64_t x, uint64_t y) { return key_label(hkey[x], 0) < key_label(hkey[y], 0); });
       size_t next = 0;
       while (next < pending.size()) {
         std::fill(hdom.begin(), hdom.end(), ~0ull);
+        a.walk_lo = key_label(hkey[pending[next]], 0);
         uint64_t used = 0;
         for (; next < pending.size(); next++) {
           const uint64_t k = hkey[pending[next]];
@@ -962,6 +1028,7 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
                       "gamma_fpm: a chunk pass met an unclaimed pattern");
         ctx->stats.chunks++;
       }
+      a.walk_lo = 0;
       clear_pool();
     }
     if (!full) break;

@@ -84,12 +84,14 @@ def test_pattern_table_growth(G, oracle_mod):
     assert g.fpm(3, 2) == oracle_set(o, 3, 2)
 
 
-@pytest.mark.parametrize("budget_kb", [100, 120])
-def test_domain_pool_chunks(G, oracle_mod, budget_kb):
-    """A budget too small for one level's MNI domains: the level is redone in chunks
-    of patterns that fit the pool (and the table grows too at 160 KB)."""
+@pytest.mark.parametrize("budget_kb,nlab", [(100, 5), (120, 5), (2048, 12)])
+def test_domain_pool_chunks(G, oracle_mod, budget_kb, nlab):
+    """A budget too small for one level's MNI domains: the first pass carves domains
+    only for patterns whose smallest label is below a threshold, the rest are redone
+    in chunks (ascending smallest label) whose passes skip every embedding with a
+    smaller label; the table may have to grow too."""
     n, s, d, lab = gg.config_graph("c4", seed=1, scale=11)
-    lab = gg.labels(n, 5, 1)
+    lab = gg.labels(n, nlab, 1)
     c = G.Context(hbm_budget_bytes=budget_kb << 10)
     g = c.load_edges(n, s, d, lab)
     o = oracle_mod.Graph(n, s, d, lab)

@@ -302,9 +302,9 @@ def test_c2_full_size(ctx, oracle_mod):
 
 @pytest.mark.parametrize("case", ["c1", "er", "dups", "selfloops", "one"])
 def test_builders_agree(G, ctx, oracle_mod, case):
-    """A1 has two builders -- counting sort + segmented row sort (default below 2^31
-    directed entries) and the global key sort (GAMMA_FLAG_KEY_SORT_BUILD, used above);
-    both must give the oracle's O-0 CSR and the same DAG."""
+    """A1 has two builders -- the global key sort (default) and counting sort +
+    segmented row sort (GAMMA_FLAG_COUNT_SORT_BUILD); both must give the oracle's O-0
+    CSR and the same DAG."""
     if case == "c1":
         n, s, d, _ = gg.config_graph("c1", seed=2)
     elif case == "er":
@@ -321,8 +321,8 @@ def test_builders_agree(G, ctx, oracle_mod, case):
     else:
         n = 2
         s, d = np.array([0], np.uint32), np.array([1], np.uint32)
-    key = G.Context(device=0, flags=0x80)
-    g1, g2 = ctx.load_edges(n, s, d), key.load_edges(n, s, d)
+    counting = G.Context(device=0, flags=0x80)   # GAMMA_FLAG_COUNT_SORT_BUILD
+    g1, g2 = ctx.load_edges(n, s, d), counting.load_edges(n, s, d)
     o = oracle_mod.Graph(n, s, d)
     orp, ocol = o.csr()
     for g in (g1, g2):
