@@ -827,6 +827,28 @@ static std::vector<double> fpm_words_by_min_label(uint32_t l, const std::vector<
   return W;
 }
 
+// The MNI domain pool (most of free HBM) is taken with cudaMalloc and returned with
+// cudaFree, not through the context's allocator: a caching allocator (PyTorch's)
+// keeps a freed block reserved, and the next call would see a fraction of the HBM.
+struct PoolBuf {
+  uint32_t *p = nullptr;
+  void alloc(uint64_t words) {
+    reset();
+    const cudaError_t e = cudaMalloc(&p, words * sizeof(uint32_t));
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      p = nullptr;
+      throw Fail{GAMMA_E_NOMEM, "gamma_fpm: cudaMalloc of the domain pool failed: " +
+                                    std::string(cudaGetErrorString(e))};
+    }
+  }
+  void reset() {
+    if (p) cudaFree(p);
+    p = nullptr;
+  }
+  ~PoolBuf() { reset(); }
+};
+
 static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::vector<gamma_fpm_pattern> &out) {
   gamma_ctx *ctx = g->ctx;
   const uint32_t n = g->n;
@@ -891,7 +913,8 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
   while ((double)cap < 2 * bound && cap < (1ull << 24)) cap <<= 1;
   const uint64_t slot_bytes = 8 + 8 + 4 + 8;
   while (cap > 1024 && cap * slot_bytes * 4 > budget) cap >>= 1;
-  DevBuf<uint32_t> freq, pool;
+  DevBuf<uint32_t> freq;
+  PoolBuf pool;
   DevBuf<unsigned long long> slots, sup, pcur;
   FpmArgs a{};
   a.rp = g->row_ptr;
@@ -920,7 +943,7 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
     slots = DevBuf<unsigned long long>(ctx, 2 * cap);
     sup = DevBuf<unsigned long long>(ctx, cap);
     freq = DevBuf<uint32_t>(ctx, cap);
-    pool = DevBuf<uint32_t>(ctx, pool_words);
+    pool.alloc(pool_words);
     pcur = DevBuf<unsigned long long>(ctx, 1);
     GAMMA_CUDA(cudaMemsetAsync(slots.p, 0, cap * 16, ctx->stream));
     GAMMA_CUDA(cudaMemsetAsync(freq.p, 0, cap * 4, ctx->stream));

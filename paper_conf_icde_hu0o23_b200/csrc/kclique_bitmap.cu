@@ -471,6 +471,7 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
     const uint32_t x = R[i];
     uint32_t h = (x * 0x9E3779B1u) >> (32 - hbits);
     if (Hv) {
+      h &= ~1u;   // probing starts at an even slot: a lookup reads the slot pair in one load
       while (atomicCAS(&Hv[h], kEmptyId, x) != kEmptyId) h = (h + 1) & hmask;
       H[h] = (unsigned short)i;
     } else {
@@ -527,25 +528,29 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
       for (int u = 0; u < kTiles; u++) {
         const uint32_t yy = y[u];
         if (Hv) {
-          if (yy < rmin || yy > rmax) continue;   // (the padding 0xffffffff is above every rmax < n)
-          const uint32_t h0 = (yy * 0x9E3779B1u) >> (32 - hbits), h1 = (h0 + 1) & hmask;
-          const uint32_t v0 = Hv[h0], v1 = Hv[h1];
-          int e = -1;
-          if (v0 == yy) {
-            e = H[h0];
-          } else if (v1 == yy) {
-            e = H[h1];
-          } else if (v0 != kEmptyId && v1 != kEmptyId) {
-            for (uint32_t h = (h1 + 1) & hmask;; h = (h + 1) & hmask) {
+          // one 8-byte load of the even slot pair where y's probe sequence starts;
+          // both compares are predicated, and only a full pair without y (rare at
+          // load <= 1/4) continues the linear probe
+          const bool inr = yy >= rmin && yy <= rmax;   // (the padding 0xffffffff is above every rmax < n)
+          const uint32_t h0 = ((yy * 0x9E3779B1u) >> (32 - hbits)) & ~1u;
+          const uint2 vv = *reinterpret_cast<const uint2 *>(Hv + h0);
+          bool hit = inr && (vv.x == yy || vv.y == yy);
+          uint32_t hh = vv.x == yy ? h0 : h0 + 1;
+          if (inr && vv.x != yy && vv.y != yy && vv.x != kEmptyId && vv.y != kEmptyId) {
+            for (uint32_t h = (h0 + 2) & hmask;; h = (h + 1) & hmask) {
               const uint32_t vh = Hv[h];
               if (vh == yy) {
-                e = H[h];
+                hit = true;
+                hh = h;
                 break;
               }
               if (vh == kEmptyId) break;
             }
           }
-          if (e >= 0) atomicOr(&B[rj[u] * W + ((uint32_t)e >> 5)], 1u << (e & 31));
+          if (hit) {
+            const uint32_t e = H[hh];
+            atomicOr(&B[rj[u] * W + (e >> 5)], 1u << (e & 31));
+          }
           continue;
         }
         if (yy >= rmin && yy <= rmax) {   // (the padding 0xffffffff is above every rmax < n)

@@ -84,8 +84,8 @@ def test_pattern_table_growth(G, oracle_mod):
     assert g.fpm(3, 2) == oracle_set(o, 3, 2)
 
 
-@pytest.mark.parametrize("budget_kb,nlab", [(100, 5), (120, 5), (2048, 12)])
-def test_domain_pool_chunks(G, oracle_mod, budget_kb, nlab):
+@pytest.mark.parametrize("budget_kb,nlab,minsup3", [(100, 5, 20), (120, 5, 20), (1024, 12, 2)])
+def test_domain_pool_chunks(G, oracle_mod, budget_kb, nlab, minsup3):
     """A budget too small for one level's MNI domains: the first pass carves domains
     only for patterns whose smallest label is below a threshold, the rest are redone
     in chunks (ascending smallest label) whose passes skip every embedding with a
@@ -96,7 +96,7 @@ def test_domain_pool_chunks(G, oracle_mod, budget_kb, nlab):
     g = c.load_edges(n, s, d, lab)
     o = oracle_mod.Graph(n, s, d, lab)
     assert g.fpm(2, 5) == oracle_set(o, 2, 5)
-    assert g.fpm(3, 20) == oracle_set(o, 3, 20)
+    assert g.fpm(3, minsup3) == oracle_set(o, 3, minsup3)
     assert c.stats()["chunks"] > 0
 
 
