@@ -50,10 +50,10 @@ def lib():
             L.og_kclique_roots.argtypes = [C.c_void_p, C.c_uint32, C.c_uint64, u32p, u64p, C.c_int]
             L.og_kclique_levels.argtypes = [C.c_void_p, C.c_uint32, u64p, u64p, C.c_int]
             L.og_match.restype = C.c_int
-            L.og_match.argtypes = [C.c_void_p, C.c_uint32, C.c_uint32, u32p, C.c_void_p, C.c_int,
+            L.og_match.argtypes = [C.c_void_p, C.c_uint32, C.c_uint32, u32p, C.c_void_p, C.c_int, C.c_int,
                                    C.POINTER(C.c_uint64), C.POINTER(C.c_uint64), C.POINTER(C.c_uint64)]
             L.og_match_roots.restype = C.c_int
-            L.og_match_roots.argtypes = [C.c_void_p, C.c_uint32, C.c_uint32, u32p, C.c_void_p, C.c_uint64,
+            L.og_match_roots.argtypes = [C.c_void_p, C.c_uint32, C.c_uint32, u32p, C.c_void_p, C.c_int, C.c_uint64,
                                          u32p, u64p, C.c_int]
             L.og_fpm.restype = C.c_int64
             L.og_fpm.argtypes = [C.c_void_p, C.c_uint32, C.c_uint64, C.c_int, C.c_int, C.c_uint64,
@@ -116,25 +116,26 @@ class Graph:
         lib().og_kclique_levels(self._h, k, N, S, threads)
         return [int(x) for x in N], [int(x) for x in S]
 
-    def match(self, nv: int, edges, plabels=None, threads: int = 0):
-        """Return (count, mappings, |Aut_L|)."""
+    def match(self, nv: int, edges, plabels=None, threads: int = 0, induced: bool = False):
+        """Return (count, mappings, |Aut_L|); induced=True also maps non-edges to non-edges."""
         e = np.ascontiguousarray(np.asarray(edges, dtype=np.uint32).reshape(-1))
         pl = None if plabels is None else np.ascontiguousarray(plabels, dtype=np.uint32)
         c, mp, a = C.c_uint64(), C.c_uint64(), C.c_uint64()
         st = lib().og_match(self._h, nv, e.size // 2, e, None if pl is None else pl.ctypes.data,
-                            threads, C.byref(c), C.byref(mp), C.byref(a))
+                            int(bool(induced)), threads, C.byref(c), C.byref(mp), C.byref(a))
         if st != 0:
             raise ValueError(f"oracle og_match status {st}")
         return int(c.value), int(mp.value), int(a.value)
 
-    def match_roots(self, nv: int, edges, roots, plabels=None, threads: int = 0) -> np.ndarray:
+    def match_roots(self, nv: int, edges, roots, plabels=None, threads: int = 0,
+                    induced: bool = False) -> np.ndarray:
         """Mappings whose image of pattern vertex 0 is each given root."""
         e = np.ascontiguousarray(np.asarray(edges, dtype=np.uint32).reshape(-1))
         pl = None if plabels is None else np.ascontiguousarray(plabels, dtype=np.uint32)
         roots = np.ascontiguousarray(roots, dtype=np.uint32)
         out = np.zeros(roots.size, np.uint64)
         st = lib().og_match_roots(self._h, nv, e.size // 2, e, None if pl is None else pl.ctypes.data,
-                                  roots.size, roots, out, threads)
+                                  int(bool(induced)), roots.size, roots, out, threads)
         if st != 0:
             raise ValueError(f"oracle og_match_roots status {st}")
         return out

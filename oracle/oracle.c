@@ -16,7 +16,8 @@
  *                       SURVEY.md §8(d)'s algorithmic bytes
  *   og_match       O-2  #injective label-preserving edge-preserving maps / |Aut_L(P)|
  *                       ("all subgraphs isomorphic to a pattern P";
- *                        Alg. 1)
+ *                        Alg. 1); induced=1 also maps non-edges of P to
+ *                        non-edges of G
  *   og_fpm_*       O-3  edge-induced patterns with <= l edges and MNI support >= minsup
  *                       (Alg. 2; MNI per
  *                        DESIGN.md reading R1)
@@ -344,7 +345,11 @@ void og_kclique_levels(const og_graph *g, uint32_t k, uint64_t *N, uint64_t *S, 
 }
 
 /* ---------------------------------------------------------------------------
- * O-2: labeled, non-induced subgraph matching.  count = mappings / |Aut_L(P)|.
+ * O-2: labeled subgraph matching.  count = mappings / |Aut_L(P)|.
+ * Non-induced (reading R4): edges of P map to edges of G.  Induced
+ * ("anti-edge checks"): in addition, every
+ * non-edge of P maps to a non-edge of G.  Aut_L(P) is the same group for both
+ * (a permutation preserving E_P preserves its complement).
  * Matching order: BFS from pattern vertex 0 (deliberately not the GPU planner's
  * order).  Candidates of pattern vertex q = N(phi(bfs parent of q)); every other
  * backward edge checked by binary search; injectivity by linear scan.
@@ -355,6 +360,7 @@ typedef struct {
   uint32_t nv;
   int adjm[OG_MAXV][OG_MAXV];
   int labeled;
+  int induced;                 /* 1: also require non-edges of P to map to non-edges of G */
   uint32_t plab[OG_MAXV];
   uint32_t order[OG_MAXV];     /* BFS order */
   uint32_t parent[OG_MAXV];    /* BFS parent of order[i] (i>0) */
@@ -421,6 +427,7 @@ static uint64_t match_rec(const og_graph *g, const og_pat *p, uint32_t pos, uint
     for (uint32_t i = 0; i < pos && ok; i++) {
       uint32_t b = p->order[i];
       if (b != par && p->adjm[q][b] && !adjacent(g, phi[b], x)) ok = 0;           /* backward edges */
+      if (p->induced && !p->adjm[q][b] && adjacent(g, phi[b], x)) ok = 0;          /* backward non-edges */
     }
     if (!ok) continue;
     phi[q] = x;
@@ -430,11 +437,12 @@ static uint64_t match_rec(const og_graph *g, const og_pat *p, uint32_t pos, uint
 }
 
 int og_match(const og_graph *g, uint32_t nv, uint32_t ne, const uint32_t *edges,
-             const uint32_t *plabels, int threads, uint64_t *count, uint64_t *mappings,
+             const uint32_t *plabels, int induced, int threads, uint64_t *count, uint64_t *mappings,
              uint64_t *aut) {
   og_pat p;
   int st = pat_init(&p, nv, ne, edges, plabels);
   if (st) return st;
+  p.induced = induced != 0;
   set_threads(threads);
   uint64_t total = 0;
   uint32_t r = p.order[0];
@@ -456,11 +464,12 @@ int og_match(const og_graph *g, uint32_t nv, uint32_t ne, const uint32_t *edges,
 /* Mappings whose image of BFS-order vertex 0 (pattern vertex 0) is roots[i]; the sum
  * over all vertices is the `mappings` of og_match.  For sampled timing / parity. */
 int og_match_roots(const og_graph *g, uint32_t nv, uint32_t ne, const uint32_t *edges,
-                   const uint32_t *plabels, uint64_t nroots, const uint32_t *roots, uint64_t *out,
-                   int threads) {
+                   const uint32_t *plabels, int induced, uint64_t nroots, const uint32_t *roots,
+                   uint64_t *out, int threads) {
   og_pat p;
   int st = pat_init(&p, nv, ne, edges, plabels);
   if (st) return st;
+  p.induced = induced != 0;
   set_threads(threads);
   uint32_t r = p.order[0];
 #pragma omp parallel for schedule(dynamic, 16)

@@ -133,3 +133,21 @@ def connected_subset_counts(n, E):
     three = T + sum(comb(d, 3) for d in deg) + sum((deg[a] - 1) * (deg[b] - 1) for a, b in
                                                    (tuple(e) for e in E)) - 3 * T
     return two, three
+
+
+def induced_subgraphs(n, E, nv, pedges, plab=None, glab=None):
+    """Number of vertex subsets W (|W| = nv) whose induced subgraph G[W] is isomorphic
+    to P, labels respected (induced matching, counted by vertex subsets)."""
+    PE = _pattern_edges(pedges)
+    cnt = 0
+    for W in itertools.combinations(range(n), nv):
+        EW = {e for e in (frozenset(p) for p in itertools.combinations(W, 2)) if e in E}
+        if len(EW) != len(PE):
+            continue
+        for p in itertools.permutations(W):
+            if plab is not None and any(glab[p[i]] != plab[i] for i in range(nv)):
+                continue
+            if {frozenset((p[a], p[b])) for a, b in pedges} == EW:
+                cnt += 1
+                break
+    return cnt

@@ -130,3 +130,68 @@ def test_disconnected_pattern_rejected(oracle_mod):
     g = G(oracle_mod, gg.complete(5))
     with pytest.raises(ValueError):
         g.match(4, [(0, 1), (2, 3)])
+
+
+# ---- induced matching (anti-edge checks) ----------
+K4 = (4, [(0, 1), (0, 2), (0, 3), (1, 2), (1, 3), (2, 3)])
+
+
+def icount(g, name, plab=None):
+    nv, e = K4 if name == "k4" else Q[name]
+    return g.match(nv, e, plab, induced=True)[0]
+
+
+@pytest.mark.parametrize("n", [4, 5, 7])
+def test_induced_complete(oracle_mod, n):
+    g = G(oracle_mod, gg.complete(n))
+    for q in ("c4", "diamond", "tailed_triangle", "house"):
+        assert icount(g, q) == 0
+    assert icount(g, "k4") == comb(n, 4)
+
+
+@pytest.mark.parametrize("a,b", [(2, 2), (3, 4)])
+def test_induced_bipartite_grid(oracle_mod, a, b):
+    assert icount(G(oracle_mod, gg.complete_bipartite(a, b)), "c4") == comb(a, 2) * comb(b, 2)
+    assert icount(G(oracle_mod, gg.grid(a + 1, b + 1)), "c4") == a * b
+
+
+@pytest.mark.parametrize("n", [5, 6, 9])
+def test_induced_wheel(oracle_mod, n):
+    """W_n (n >= 5): every C4 has a chord through the hub; the diamonds hub,i-1,i,i+1
+    are induced (i-1, i+1 not adjacent for n >= 5); an induced tailed triangle is a
+    triangle hub,i,i+1 with the tail j hanging off the hub, j not in {i-1..i+2}:
+    n(n-4)."""
+    g = G(oracle_mod, gg.wheel(n))
+    assert icount(g, "c4") == 0
+    assert icount(g, "tailed_triangle") == n * (n - 4)
+    assert icount(g, "diamond") == n
+
+
+@pytest.mark.parametrize("seed", [1, 2, 3])
+def test_induced_supergraph_identities(oracle_mod, seed):
+    """Non-induced count = sum over the 4-vertex supergraphs H of P of
+    (#copies of P in H) x induced(H): C4 = iC4 + iDiamond + 3 iK4,
+    tailed triangle = iTT + 4 iDiamond + 12 iK4, diamond = iDiamond + 6 iK4."""
+    n = 64
+    s, d = gg.er(n, 700, seed)
+    g = oracle_mod.Graph(n, s, d)
+    ic4, idi, itt, ik4 = (icount(g, q) for q in ("c4", "diamond", "tailed_triangle", "k4"))
+    assert ik4 == g.kclique(4) and ik4 > 0 and idi > 0
+    assert count(g, "c4") == ic4 + idi + 3 * ik4
+    assert count(g, "tailed_triangle") == itt + 4 * idi + 12 * ik4
+    assert count(g, "diamond") == idi + 6 * ik4
+
+
+@pytest.mark.parametrize("seed", [1, 2])
+@pytest.mark.parametrize("q", ["c4", "diamond", "tailed_triangle", "house"])
+def test_induced_brute_force(oracle_mod, seed, q):
+    n = 11
+    s, d = gg.er(n, 30, seed)
+    E = brute.normalise(s, d)
+    lab = [int(x) for x in gg.labels(n, 2, seed)]
+    nv, e = Q[q]
+    g0 = oracle_mod.Graph(n, s, d)
+    g = oracle_mod.Graph(n, s, d, lab)
+    assert g0.match(nv, e, induced=True)[0] == brute.induced_subgraphs(n, E, nv, e)
+    plab = [i % 2 for i in range(nv)]
+    assert g.match(nv, e, plab, induced=True)[0] == brute.induced_subgraphs(n, E, nv, e, plab, lab)
