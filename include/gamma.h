@@ -7,8 +7,9 @@
  *                  common neighbours (L146) over a degree-ordered DAG.
  *   gamma_match    subgraph matching, "all subgraphs of G_d isomorphic to a pattern
  *                  P" (L112), by worst-case-optimal-join vertex extension + filtering
- *                  (Alg. 1).  Non-induced, labeled, counted as distinct
- *                  subgraphs (readings R4-R6).
+ *                  (Alg. 1).  Labeled, counted as distinct subgraphs
+ *                  (readings R4-R6); non-induced, or induced with
+ *                  anti-edge checks (R17).
  *   gamma_fpm      frequent pattern mining, "all patterns P whose support is at least a
  *                  given threshold" (L113, L144), by edge extension + aggregation +
  *                  filtering (Alg. 2), edge-induced, MNI support (R1-R3).
@@ -48,7 +49,7 @@ enum {
   GAMMA_E_NOMEM = -2,        /* device allocation failed or HBM/spill budget too small */
   GAMMA_E_CUDA = -3,         /* CUDA runtime / kernel error (incl. no device)        */
   GAMMA_E_OVERFLOW = -4,     /* uint64 count overflow                                */
-  GAMMA_E_UNSUPPORTED = -5   /* valid request outside this version (k>32, induced=1) */
+  GAMMA_E_UNSUPPORTED = -5   /* valid request outside this version (k>32, max_edges>3) */
 };
 
 typedef struct gamma_ctx gamma_ctx;
@@ -163,13 +164,14 @@ typedef struct {
   uint32_t nv, ne;           /* 1 <= nv <= 8, connected                              */
   const uint32_t *edges;     /* 2*ne vertex ids (host memory)                        */
   const uint32_t *labels;    /* nv labels or NULL (unlabeled: any vertex matches)    */
-  int32_t induced;           /* must be 0 in v1 (E_UNSUPPORTED otherwise)            */
+  int32_t induced;           /* 0: non-induced (edges of P -> edges of G); 1: induced
+                                (also non-edges of P -> non-edges of G); else E_INVAL  */
 } gamma_pattern;
 
 /* Host-only planning of a pattern (no device needed): the matching order delta_v
  * (Alg. 1 line 1; R10), |Aut_L(P)| and the symmetry-breaking
  * order constraints gamma_match applies.  Masks are over matching-order positions.
- * Errors: E_INVAL (nv out of [1,8], bad edge, disconnected), E_UNSUPPORTED (induced). */
+ * Errors: E_INVAL (nv out of [1,8], bad edge, disconnected, induced not 0/1).     */
 typedef struct {
   uint32_t nv;
   uint32_t order[8];         /* position -> pattern vertex                           */

@@ -1,6 +1,7 @@
 // match.cu -- subgraph matching, Alg. 1 (WOJ, query-vertex-at-a-time vertex
-// extension + filtering), non-induced, labeled, counting
-// distinct subgraphs (readings R4-R6, R10).
+// extension + filtering), labeled, counting distinct
+// subgraphs (readings R4-R6, R10); non-induced by default, induced on
+// request (the same extension with anti-edge checks, R17).
 //
 // Host planner:
 //  * matching order delta_v (PAPER.md L176 leaves it open; reading R10): the
@@ -57,6 +58,7 @@ struct SmPlan {
   uint32_t injmask[kMaxV];  // earlier non-neighbour positions (x != phi_j)
   uint32_t ltmask[kMaxV];   // earlier positions j with phi_j < x
   uint32_t gtmask[kMaxV];   // earlier positions j with x < phi_j
+  uint32_t antimask[kMaxV]; // induced: earlier non-neighbour positions j with x not in N(phi_j)
   uint64_t aut;
 };
 
@@ -89,6 +91,7 @@ struct Bounds {
   int64_t lo;     // x > lo
   uint32_t hi;    // x < hi (0xffffffff: none)
   uint32_t inj;   // positions to check x != phi_j
+  uint32_t anti;  // induced: positions to check x not in N(phi_j)
 };
 
 // Candidate filter for position q.
@@ -106,11 +109,22 @@ __device__ __forceinline__ bool sm_filter(const SmArgs &a, uint32_t q, uint32_t 
     if (phi[j] == x) return false;
   }
   if (!last && a.P.mindeg[q] > 1 && gdeg(a, x) < a.P.mindeg[q]) return false;
+  m = b.anti;   // induced: anti-edge checks, one binary search per non-neighbour
+  while (m) {
+    const int j = __ffs(m) - 1;
+    m &= m - 1;
+    const uint64_t s = a.rp[phi[j]];
+    const uint32_t l = (uint32_t)(a.rp[phi[j] + 1] - s);
+    if (l && sorted_contains(a.col + s, l, x)) return false;
+  }
   return true;
 }
 
-__device__ __forceinline__ Bounds bounds_for(const SmArgs &a, uint32_t q, uint32_t avail, const uint32_t *phi) {
-  Bounds b{-1, 0xffffffffu, a.P.injmask[q] & avail};
+// `anti_avail`: the placed positions whose anti-edge checks are still to be made
+// (a staged L_m has the prefix ones applied already).
+__device__ __forceinline__ Bounds bounds_for(const SmArgs &a, uint32_t q, uint32_t avail, const uint32_t *phi,
+                                             uint32_t anti_avail) {
+  Bounds b{-1, 0xffffffffu, a.P.injmask[q] & avail, a.P.antimask[q] & anti_avail};
   uint32_t m = a.P.ltmask[q] & avail;
   while (m) {
     const int j = __ffs(m) - 1;
@@ -202,6 +216,7 @@ __global__ void __launch_bounds__(kThreads) sm_kernel(SmArgs a) {
   const uint32_t bq = a.P.bmask[q];
   const uint32_t bshared = bq & prefix_mask;
   const bool child_in_b = (bq >> d) & 1u;
+  const bool anti_d = (a.P.antimask[q] >> d) & 1u;   // induced: x must not be adjacent to the child
 
   while (!stop) {
     unsigned long long base = 0;
@@ -221,7 +236,7 @@ __global__ void __launch_bounds__(kThreads) sm_kernel(SmArgs a) {
       for (int j = 0; j < kMaxV; j++) phi[j] = __shfl_sync(0xffffffffu, w, (2 + j) & 31);
       in_entries += (lane == 0) ? len : 0;
       // ---- Opt 2: L_m over the prefix-only backward lists, staged per group ----
-      const Bounds bs = bounds_for(a, q, prefix_mask, phi);
+      const Bounds bs = bounds_for(a, q, prefix_mask, phi, prefix_mask);
       bool staged = false;
       uint32_t lm_len = 0;
       // L_m lives in shared memory when its bound (the shortest prefix list) fits,
@@ -247,7 +262,7 @@ __global__ void __launch_bounds__(kThreads) sm_kernel(SmArgs a) {
         }
       }
       if (staged && lane == 0) {   // Opt 2: the prefix lists are fetched once per group
-        uint32_t m = bshared;
+        uint32_t m = bshared | (a.P.antimask[q] & prefix_mask);
         while (m) {
           const int j = __ffs(m) - 1;
           m &= m - 1;
@@ -256,7 +271,7 @@ __global__ void __launch_bounds__(kThreads) sm_kernel(SmArgs a) {
       }
       if (staged && lm_len == 0) continue;   // no child can extend
       const uint32_t *run = a.vid_in + beg;
-      if (last && staged) {
+      if (last && staged && !anti_d) {
         // Last level over a staged L_m: count without a per-child warp loop.  The
         // filters that involve the child c = phi_d are an order window (lo_c, hi_c)
         // and possibly x != c; the prefix filters are already applied to L_m.
@@ -360,14 +375,16 @@ __global__ void __launch_bounds__(kThreads) sm_kernel(SmArgs a) {
         const uint32_t c = run[i];
         phi[d] = c;
         if (lane == 0) {   // the lists this child's extension fetches
-          uint32_t m = staged ? (child_in_b ? (1u << d) : 0u) : bq;
+          uint32_t m = (staged ? (child_in_b ? (1u << d) : 0u) : (bq | (a.P.antimask[q] & prefix_mask))) |
+                       (anti_d ? (1u << d) : 0u);
           while (m) {
             const int j = __ffs(m) - 1;
             m &= m - 1;
             elems += gdeg(a, phi[j]);
           }
         }
-        const Bounds bc = bounds_for(a, q, prefix_mask | (1u << d), phi);
+        const Bounds bc = bounds_for(a, q, prefix_mask | (1u << d), phi,
+                                     staged ? (1u << d) : (prefix_mask | (1u << d)));
         uint32_t found;
         uint64_t pos = 0;
         bool big = false;
@@ -378,11 +395,14 @@ __global__ void __launch_bounds__(kThreads) sm_kernel(SmArgs a) {
           big = !last && lm_len > kOutCap;
           if (big && !pool_reserve(pv, lm_len, lane, pos)) { stop = true; break; }
           uint32_t *dst = big ? a.vid_out + pos : sout;
+          const uint64_t cs = a.rp[c];
+          const uint32_t cl = anti_d ? (uint32_t)(a.rp[c + 1] - cs) : 0u;
           for (uint32_t j0 = 0; j0 < lm_len; j0 += 32) {
             const uint32_t jj = j0 + lane;
             const uint32_t x = jj < lm_len ? lm[jj] : 0xffffffffu;
-            const bool ok = jj < lm_len && (int64_t)x > bc.lo && x < bc.hi &&
-                            !(((a.P.injmask[q] >> d) & 1u) && x == c);
+            bool ok = jj < lm_len && (int64_t)x > bc.lo && x < bc.hi &&
+                      !(((a.P.injmask[q] >> d) & 1u) && x == c);
+            if (ok && cl) ok = !sorted_contains(a.col + cs, cl, x);   // induced: x not adjacent to c
             const uint32_t bal = __ballot_sync(0xffffffffu, ok);
             if (!last && ok) dst[found + __popc(bal & lanemask_lt())] = x;
             found += __popc(bal);
@@ -510,7 +530,7 @@ constexpr size_t sm_smem() { return (size_t)kWarps * (kLmCap + kOutCap) * sizeof
 // ------------------------------------------------------------------------------------
 static void plan_pattern(const gamma_pattern *p, SmPlan &P) {
   GAMMA_REQUIRE(p->nv >= 1 && p->nv <= (uint32_t)kMaxV, GAMMA_E_INVAL, "pattern: nv must be in [1, 8]");
-  GAMMA_REQUIRE(p->induced == 0, GAMMA_E_UNSUPPORTED, "pattern: induced matching is not supported in v1");
+  GAMMA_REQUIRE(p->induced == 0 || p->induced == 1, GAMMA_E_INVAL, "pattern: induced must be 0 or 1");
   GAMMA_REQUIRE(p->ne == 0 || p->edges, GAMMA_E_INVAL, "pattern: NULL edges");
   const uint32_t nv = p->nv;
   int adj[kMaxV][kMaxV] = {};
@@ -589,6 +609,7 @@ static void plan_pattern(const gamma_pattern *p, SmPlan &P) {
     for (uint32_t t = 0; t < i; t++) {
       if (adj[u][order[t]]) P.bmask[i] |= 1u << t;
       else P.injmask[i] |= 1u << t;
+      if (!adj[u][order[t]] && p->induced) P.antimask[i] |= 1u << t;
     }
   }
   // stabilizer chain along the matching order

@@ -1,5 +1,5 @@
-"""GPU parity of gamma_match (Alg. 1, labeled non-induced SM) against the oracle
-(O-2), through the C ABI.  Tolerance 0."""
+"""GPU parity of gamma_match (Alg. 1, labeled SM, non-induced and induced) against
+the oracle (O-2), through the C ABI.  Tolerance 0."""
 from math import comb
 
 import numpy as np
@@ -144,8 +144,63 @@ def test_invalid_patterns(G, ctx):
     g = ctx.load_edges(n, s, d)
     with pytest.raises(G.GammaError):
         g.match(4, [(0, 1), (2, 3)])          # disconnected
-    with pytest.raises(G.GammaError) as e:
-        g.match(3, [(0, 1), (1, 2)], induced=True)
-    assert e.value.status == -5
+    assert g.match(3, [(0, 1), (1, 2)], induced=True)[0] == 0   # K5 has no induced path
     with pytest.raises(G.GammaError):
         g.match(9, [(i, i + 1) for i in range(8)])
+
+
+# ---- induced SM (R17) --------------------------------
+K4 = (4, [(0, 1), (0, 2), (0, 3), (1, 2), (1, 3), (2, 3)])
+IPATS = [Q["c4"], Q["diamond"], Q["tailed_triangle"], Q["house"], K4, (3, [(0, 1), (1, 2)]),
+         (4, [(0, 1), (1, 2), (2, 3)]), (4, [(0, 1), (0, 2), (0, 3)]),
+         (5, [(0, 1), (1, 2), (2, 3), (3, 4), (4, 0)])]
+
+
+def test_induced_closed_forms(ctx):
+    n, (s, d) = gg.complete(9)
+    g = ctx.load_edges(n, s, d)
+    assert [g.match(*Q[q], induced=True)[0] for q in ("c4", "diamond", "tailed_triangle", "house")] == [0] * 4
+    assert g.match(*K4, induced=True)[0] == comb(9, 4)
+    n, (s, d) = gg.wheel(11)
+    g = ctx.load_edges(n, s, d)
+    assert [g.match(*Q[q], induced=True)[0] for q in ("c4", "diamond", "tailed_triangle")] == [0, 11, 11 * 7]
+    n, (s, d) = gg.complete_bipartite(5, 7)
+    assert ctx.load_edges(n, s, d).match(*Q["c4"], induced=True)[0] == comb(5, 2) * comb(7, 2)
+
+
+@pytest.mark.parametrize("seed", [1, 2])
+def test_induced_rmat_vs_oracle(ctx, oracle_mod, seed):
+    n, s, d, _ = gg.config_graph("c3", seed=seed, scale=12)
+    lab = gg.labels(n, 8, seed)
+    g = ctx.load_edges(n, s, d, lab)
+    o = oracle_mod.Graph(n, s, d, lab)
+    for nv, e in IPATS[:5]:
+        for plab in ([0] * nv, [i % 2 for i in range(nv)], [i % 8 for i in range(nv)]):
+            got = g.match(nv, e, plab, induced=True)
+            want = o.match(nv, e, plab, induced=True)
+            assert got == (want[0], want[1]), (nv, e, plab)
+
+
+def test_induced_er_paths(G, ctx, oracle_mod):
+    """Unlabeled ER: every pattern above, default / unstaged (flag 0x8) / small budget."""
+    n = 700
+    s, d = gg.er(n, 4200, 8)
+    o = oracle_mod.Graph(n, s, d)
+    for c in (ctx, G.Context(flags=0x8), G.Context(hbm_budget_bytes=2 << 20)):
+        g = c.load_edges(n, s, d)
+        for nv, e in IPATS:
+            assert g.match(nv, e, induced=True)[0] == o.match(nv, e, induced=True)[0], (nv, e)
+
+
+@pytest.mark.parametrize("deg", [900, 1500])
+def test_induced_hub(ctx, oracle_mod, deg):
+    rng = np.random.default_rng(12)
+    n = 1800
+    hub = [(0, i) for i in range(1, deg + 1)]
+    extra = [tuple(x) for x in rng.integers(1, n, size=(5000, 2))]
+    e = np.array(hub + extra, dtype=np.uint32)
+    s, d = e[:, 0].copy(), e[:, 1].copy()
+    g = ctx.load_edges(n, s, d)
+    o = oracle_mod.Graph(n, s, d)
+    for nv, pe in IPATS[:5]:
+        assert g.match(nv, pe, induced=True)[0] == o.match(nv, pe, induced=True)[0], (nv, pe)
