@@ -27,6 +27,12 @@ namespace gamma_impl {
 
 namespace {
 
+// min resident CTAs per SM for the team kernels (a register cap; 1 = none). Tuning
+// knob: nvcc -DGAMMA_BM_MINB=n.
+#ifndef GAMMA_BM_MINB
+#define GAMMA_BM_MINB 1
+#endif
+
 constexpr int kMaxStack = 10;        // DFS levels below the first child: k <= 12
 constexpr uint32_t kPartCost = 4096; // 4-cliques per heavy-root part
 constexpr uint32_t kMaxParts = 4096;
@@ -662,7 +668,7 @@ __device__ __forceinline__ void flush_multi(uint64_t (&mc)[kMaxStack + 3], const
 // KM: compile-time bound on k for the register-resident DFS of warp teams (6 or 12;
 // the deeper instantiation needs more registers, so k <= 6 gets its own kernel).
 template <int TEAM_WARPS, int TW, bool PER_ROOT, int KM>
-__global__ void __launch_bounds__(256) kcl_bitmap_kernel(BmArgs a) {
+__global__ void __launch_bounds__(256, GAMMA_BM_MINB) kcl_bitmap_kernel(BmArgs a) {
   extern __shared__ uint32_t smem[];
   constexpr int kTeamThreads = TEAM_WARPS * 32;
   const int lane = threadIdx.x & 31;
@@ -797,7 +803,7 @@ __global__ void __launch_bounds__(256) kcl_bitmap_kernel(BmArgs a) {
 // Second launch for the deferred heavy roots: one CTA per (root, part); the part
 // rebuilds the root's rows (cheap next to the DFS) and takes every nparts-th item.
 template <bool PER_ROOT, int KM>
-__global__ void __launch_bounds__(256) kcl_bitmap_parts_kernel(BmArgs a) {
+__global__ void __launch_bounds__(256, GAMMA_BM_MINB) kcl_bitmap_parts_kernel(BmArgs a) {
   extern __shared__ uint32_t smem[];
   constexpr int TW = 16;
   const int lane = threadIdx.x & 31;

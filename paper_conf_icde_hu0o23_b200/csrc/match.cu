@@ -29,6 +29,7 @@
 #include <cub/device/device_select.cuh>
 
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <vector>
 
@@ -42,8 +43,10 @@ namespace {
 constexpr int kMaxV = 8;
 constexpr int kWarps = 8;
 constexpr int kThreads = kWarps * 32;
-constexpr uint32_t kLmCap = 1024;    // staged L_m per warp (u32)
-constexpr uint32_t kOutCap = 512;    // staged child run per warp (u32); longer runs go direct
+constexpr uint32_t kLmCap = 1024;    // default staged L_m per warp (u32)
+constexpr uint32_t kOutCap = 512;    // default staged child run per warp (u32); longer runs go direct
+// (both are launch parameters, SmArgs::lm_cap / out_cap: the shared-memory footprint
+// sets the CTAs per SM; GAMMA_SM_LMCAP / GAMMA_SM_OUTCAP override them for tuning)
 constexpr uint32_t kBlkV = 4096;
 constexpr uint32_t kBlkG = 256;      // descriptors per warp block
 constexpr uint32_t kSlice = 64;      // children per group descriptor
@@ -81,6 +84,7 @@ struct SmArgs {
   uint32_t stage;           // 0: never stage L_m (debug)
   uint32_t *lm_scratch;     // per-warp global L_m slices for hub prefixes (nullable)
   uint32_t lm_scratch_cap;  // entries per warp slice
+  uint32_t lm_cap, out_cap; // shared-memory staging per warp (u32 entries)
 };
 
 __device__ __forceinline__ uint32_t gdeg(const SmArgs &a, uint32_t v) {
@@ -201,8 +205,8 @@ __global__ void __launch_bounds__(kThreads) sm_kernel(SmArgs a) {
   extern __shared__ uint32_t smem[];
   const int lane = threadIdx.x & 31;
   const int wid = threadIdx.x >> 5;
-  uint32_t *slm = smem + wid * (kLmCap + kOutCap);
-  uint32_t *sout = slm + kLmCap;
+  uint32_t *slm = smem + wid * (a.lm_cap + a.out_cap);
+  uint32_t *sout = slm + a.lm_cap;
   const uint32_t d = a.d, q = d + 1;
   const bool last = q == a.P.nv - 1;
   const BlockPool pv{&a.ctrl[CTRL_VCUR], &a.ctrl[CTRL_OVF], a.cap_v, kBlkV};
@@ -242,7 +246,7 @@ __global__ void __launch_bounds__(kThreads) sm_kernel(SmArgs a) {
       // L_m lives in shared memory when its bound (the shortest prefix list) fits,
       // else in this warp's slice of a global scratch buffer (hub prefixes)
       uint32_t *lm = slm;
-      uint32_t lm_cap = kLmCap;
+      uint32_t lm_cap = a.lm_cap;
       if (bshared && a.stage) {
         uint32_t bound = 0xffffffffu, mm = bshared;
         while (mm) {
@@ -250,7 +254,7 @@ __global__ void __launch_bounds__(kThreads) sm_kernel(SmArgs a) {
           mm &= mm - 1;
           bound = min(bound, gdeg(a, phi[j]));
         }
-        if (bound > kLmCap && a.lm_scratch) {
+        if (bound > a.lm_cap && a.lm_scratch) {
           lm = a.lm_scratch + (uint64_t)(blockIdx.x * kWarps + wid) * a.lm_scratch_cap;
           lm_cap = a.lm_scratch_cap;
         }
@@ -392,7 +396,7 @@ __global__ void __launch_bounds__(kThreads) sm_kernel(SmArgs a) {
           // candidates = L_m minus position-d filters (all prefix filters applied); a
           // run longer than the staging buffer is written straight to the level
           found = 0;
-          big = !last && lm_len > kOutCap;
+          big = !last && lm_len > a.out_cap;
           if (big && !pool_reserve(pv, lm_len, lane, pos)) { stop = true; break; }
           uint32_t *dst = big ? a.vid_out + pos : sout;
           const uint64_t cs = a.rp[c];
@@ -418,14 +422,14 @@ __global__ void __launch_bounds__(kThreads) sm_kernel(SmArgs a) {
               mm &= mm - 1;
               ub = min(ub, gdeg(a, phi[j]));
             }
-            big = ub > kOutCap;
+            big = ub > a.out_cap;
             if (big && !pool_reserve(pv, ub, lane, pos)) { stop = true; break; }
           }
           if (last)
             found = sm_intersect<false>(a, q, lists, phi, bc, last, staged ? lm : nullptr, lm_len, nullptr, 0, lane);
           else
             found = sm_intersect<true>(a, q, lists, phi, bc, last, staged ? lm : nullptr, lm_len,
-                                       big ? a.vid_out + pos : sout, big ? 0xffffffffu : kOutCap, lane);
+                                       big ? a.vid_out + pos : sout, big ? 0xffffffffu : a.out_cap, lane);
         }
         if (last) {
           acc += found;
@@ -521,7 +525,21 @@ inline unsigned g1d(uint64_t n) {
   return (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(b, 148u * 32u));
 }
 
-constexpr size_t sm_smem() { return (size_t)kWarps * (kLmCap + kOutCap) * sizeof(uint32_t); }
+static uint32_t env_u32(const char *name, uint32_t dflt, uint32_t lo, uint32_t hi) {
+  const char *v = getenv(name);
+  if (!v || !*v) return dflt;
+  const unsigned long x = strtoul(v, nullptr, 10);
+  return x < lo ? lo : (x > hi ? hi : (uint32_t)x);
+}
+static uint32_t sm_lm_cap() {
+  static const uint32_t v = env_u32("GAMMA_SM_LMCAP", kLmCap, 64, 4096);
+  return v;
+}
+static uint32_t sm_out_cap() {
+  static const uint32_t v = env_u32("GAMMA_SM_OUTCAP", kOutCap, 64, 4096);
+  return v;
+}
+static size_t sm_smem() { return (size_t)kWarps * (sm_lm_cap() + sm_out_cap()) * sizeof(uint32_t); }
 
 }  // namespace
 
@@ -688,6 +706,8 @@ struct SmRun {
     a.stage = stage;
     a.lm_scratch = lm_scratch.p;
     a.lm_scratch_cap = lm_scratch_cap;
+    a.lm_cap = sm_lm_cap();
+    a.out_cap = sm_out_cap();
     return a;
   }
 
@@ -843,7 +863,7 @@ static uint64_t match_count(gamma_graph *g, const SmPlan &P) {
     attr = true;
   }
   R.grid = ctx->num_sms * occupancy_blocks((const void *)sm_kernel, kThreads, sm_smem());
-  if (g->max_degree > kLmCap) {   // room for a hub's L_m (bounded by its degree) per warp
+  if (g->max_degree > sm_lm_cap()) {   // room for a hub's L_m (bounded by its degree) per warp
     R.lm_scratch_cap = std::min<uint32_t>(g->max_degree, 1u << 16);
     R.lm_scratch = DevBuf<uint32_t>(ctx, (uint64_t)R.grid * kWarps * R.lm_scratch_cap);
   }
