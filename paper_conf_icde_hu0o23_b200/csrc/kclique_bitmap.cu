@@ -27,11 +27,15 @@ namespace gamma_impl {
 
 namespace {
 
-// min resident CTAs per SM for the team kernels (a register cap; 1 = none). Tuning
-// knob: nvcc -DGAMMA_BM_MINB=n.
+// Min resident CTAs per SM for the team kernels with k <= 6 (KM = 6): a register cap
+// (64 -> 51 registers at 5) that trades a few bytes of spill for 40 instead of 32
+// resident warps; measured on B200: C2 -6 %, heavy -18 %.  The k <= 12
+// instances keep 64 registers (their register-resident DFS would spill ~800 B).
+// Tuning knob: nvcc -DGAMMA_BM_MINB=n.
 #ifndef GAMMA_BM_MINB
-#define GAMMA_BM_MINB 1
+#define GAMMA_BM_MINB 5
 #endif
+#define GAMMA_BM_BOUNDS(KM) __launch_bounds__(256, (KM) <= 6 ? GAMMA_BM_MINB : 1)
 
 constexpr int kMaxStack = 10;        // DFS levels below the first child: k <= 12
 constexpr uint32_t kPartCost = 4096; // 4-cliques per heavy-root part
@@ -668,7 +672,7 @@ __device__ __forceinline__ void flush_multi(uint64_t (&mc)[kMaxStack + 3], const
 // KM: compile-time bound on k for the register-resident DFS of warp teams (6 or 12;
 // the deeper instantiation needs more registers, so k <= 6 gets its own kernel).
 template <int TEAM_WARPS, int TW, bool PER_ROOT, int KM>
-__global__ void __launch_bounds__(256, GAMMA_BM_MINB) kcl_bitmap_kernel(BmArgs a) {
+__global__ void GAMMA_BM_BOUNDS(KM) kcl_bitmap_kernel(BmArgs a) {
   extern __shared__ uint32_t smem[];
   constexpr int kTeamThreads = TEAM_WARPS * 32;
   const int lane = threadIdx.x & 31;
@@ -803,7 +807,7 @@ __global__ void __launch_bounds__(256, GAMMA_BM_MINB) kcl_bitmap_kernel(BmArgs a
 // Second launch for the deferred heavy roots: one CTA per (root, part); the part
 // rebuilds the root's rows (cheap next to the DFS) and takes every nparts-th item.
 template <bool PER_ROOT, int KM>
-__global__ void __launch_bounds__(256, GAMMA_BM_MINB) kcl_bitmap_parts_kernel(BmArgs a) {
+__global__ void GAMMA_BM_BOUNDS(KM) kcl_bitmap_parts_kernel(BmArgs a) {
   extern __shared__ uint32_t smem[];
   constexpr int TW = 16;
   const int lane = threadIdx.x & 31;

@@ -43,10 +43,11 @@ namespace {
 constexpr int kMaxV = 8;
 constexpr int kWarps = 8;
 constexpr int kThreads = kWarps * 32;
-constexpr uint32_t kLmCap = 1024;    // default staged L_m per warp (u32)
+constexpr uint32_t kLmCap = 512;     // default staged L_m per warp (u32); longer L_m -> global scratch
 constexpr uint32_t kOutCap = 512;    // default staged child run per warp (u32); longer runs go direct
 // (both are launch parameters, SmArgs::lm_cap / out_cap: the shared-memory footprint
-// sets the CTAs per SM; GAMMA_SM_LMCAP / GAMMA_SM_OUTCAP override them for tuning)
+// sets the CTAs per SM; GAMMA_SM_LMCAP / GAMMA_SM_OUTCAP override them for tuning;
+// C3 sweep on B200: 512/512 233 ms, 256/256 243, 1024/512 272, 2048/512 338 per step)
 constexpr uint32_t kBlkV = 4096;
 constexpr uint32_t kBlkG = 256;      // descriptors per warp block
 constexpr uint32_t kSlice = 64;      // children per group descriptor

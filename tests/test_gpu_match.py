@@ -204,3 +204,22 @@ def test_induced_hub(ctx, oracle_mod, deg):
     o = oracle_mod.Graph(n, s, d)
     for nv, pe in IPATS[:5]:
         assert g.match(nv, pe, induced=True)[0] == o.match(nv, pe, induced=True)[0], (nv, pe)
+
+
+@pytest.mark.slow
+def test_c3_full_size(ctx):
+    """configs[2] at full size (LiveJournal-shaped R-MAT scale 23, L = 8, seed 1), in the
+    bench's configuration: the four queries x two labelings, non-induced and induced,
+    against the oracle's counts stored by tools/golden_c3.py (oracle-only script)."""
+    import json
+    import os
+    gold = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "c3_full_seed1.json")))
+    n, s, d, lab = gg.config_graph("c3", seed=1)
+    g = ctx.load_edges(n, s, d, lab)
+    assert g.info()["m"] == gold["m"]
+    for key, want in gold["counts"].items():
+        parts = key.split("/")
+        q, lname, ind = parts[0], parts[1], len(parts) > 2
+        nv, e = Q[q]
+        plab = [0] * nv if lname == "all0" else [i % 8 for i in range(nv)]
+        assert g.match(nv, e, plab, induced=ind)[0] == want, key
