@@ -129,15 +129,15 @@ class ClockSampler:
                 "reasons": sorted(reasons), "samples": len(sm)}
 
 
-def max_over_ranks(value: float, world: int) -> float:
-    """Max of a per-rank number over the default process group (identity at world 1)."""
+def max_over_ranks(value: float, world: int, op: str = "max") -> float:
+    """Max (or sum) of a per-rank number over the default process group (identity at world 1)."""
     if world <= 1:
         return float(value)
     import torch
     import torch.distributed as dist
     dev = torch.device("cuda", torch.cuda.current_device()) if dist.get_backend() == "nccl" else torch.device("cpu")
     t = torch.tensor([float(value)], dtype=torch.float64, device=dev)
-    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX if op == "max" else dist.ReduceOp.SUM)
     return float(t.item())
 
 
@@ -398,6 +398,8 @@ def run_gamma(args):
         times.append(e0.elapsed_time(e1))
     clk = clocks.stop()
     total_ms = max_over_ranks(sum(times), world)
+    # load imbalance of the root partition = max / mean of the ranks' times
+    imbalance = total_ms / (max_over_ranks(sum(times), world, "sum") / world) if world > 1 else 1.0
     value = emb * args.steps / (total_ms / 1000.0)
 
     # ---- e2e: the same step through the public API from pinned host buffers ----
@@ -477,6 +479,7 @@ def run_gamma(args):
         "kernels": {k: v for k, v in agg.items() if not k.startswith("_") and v["launches"]},
         "build_ms_per_step": info["build_ms"],
         "step_ms": [round(x, 3) for x in times],
+        "rank_time_max_over_mean": imbalance,
         "e2e_step_ms": [round(x, 3) for x in e2e_times],
     }
     print(json.dumps(out))

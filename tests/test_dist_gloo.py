@@ -36,7 +36,8 @@ def _worker(rank, world, port, q):
         G.alltoall_tensors(send, recv)
         import bench
         t = bench.max_over_ranks(1.5 + rank, world)
-        q.put((rank, st + st2, list(buf) + [big[0]], recv.tolist(), t))
+        tsum = bench.max_over_ranks(1.5 + rank, world, "sum")
+        q.put((rank, st + st2, list(buf) + [big[0]], recv.tolist(), (t, tsum)))
     finally:
         dist.destroy_process_group()
 
@@ -57,4 +58,4 @@ def test_allreduce_callback_and_max_timing():
         assert st == 0
         assert buf == [3, 30, 2 * 2 ** 40 + 1, 10]
         assert recv == [3 * rank, 3 * rank + 1, 3 * rank + 2, 100 + 3 * rank, 101 + 3 * rank, 102 + 3 * rank]
-        assert t == 2.5
+        assert t == (2.5, 4.0)   # max and sum over ranks (imbalance = max / (sum / world))
