@@ -35,6 +35,16 @@ def library_path() -> str:
     return N.LIB_PATH
 
 
+# The connected graphs on 3 and 4 vertices (up to isomorphism), for Graph.motifs.
+MOTIFS = {
+    3: {"wedge": [(0, 1), (1, 2)], "triangle": [(0, 1), (1, 2), (0, 2)]},
+    4: {"path": [(0, 1), (1, 2), (2, 3)], "star": [(0, 1), (0, 2), (0, 3)],
+        "c4": [(0, 1), (1, 2), (2, 3), (3, 0)], "tailed_triangle": [(0, 1), (0, 2), (1, 2), (2, 3)],
+        "diamond": [(0, 1), (0, 2), (1, 2), (1, 3), (2, 3)],
+        "k4": [(0, 1), (0, 2), (0, 3), (1, 2), (1, 3), (2, 3)]},
+}
+
+
 class GammaError(RuntimeError):
     def __init__(self, status: int, where: str):
         msg = (_lib.gamma_last_error() or b"").decode(errors="replace")
@@ -334,6 +344,13 @@ class Graph:
         c, mp = C.c_uint64(), C.c_uint64()
         _check(_lib.gamma_match(self._h, C.byref(p), C.byref(c), C.byref(mp)), "gamma_match")
         return int(c.value), int(mp.value)
+
+    def motifs(self, k: int) -> dict:
+        """Motif counts: induced counts of every connected unlabeled k-vertex pattern
+        (k = 3, 4), one gamma_match(induced=1) call each."""
+        if k not in MOTIFS:
+            raise ValueError("motifs: k must be 3 or 4")
+        return {name: self.match(k, e, induced=True)[0] for name, e in MOTIFS[k].items()}
 
     def fpm(self, max_edges: int, minsup: int):
         """Frequent patterns: sorted list of (ne, nv, labels, edges, support)."""

@@ -223,3 +223,25 @@ def test_c3_full_size(ctx):
         nv, e = Q[q]
         plab = [0] * nv if lname == "all0" else [i % 8 for i in range(nv)]
         assert g.match(nv, e, plab, induced=ind)[0] == want, key
+
+
+def test_motifs(ctx, oracle_mod):
+    """Motif counts (induced, every connected 3-/4-vertex graph) against the oracle, plus
+    the identities sum_v C(d_v, 2) = iWedge + 3 T and sum over 4-motifs of
+    (#spanning-subgraph copies) = the non-induced counts of path / star."""
+    import paper_conf_icde_hu0o23_b200 as G
+    n, s, d, _ = gg.config_graph("c3", seed=3, scale=11)
+    g = ctx.load_edges(n, s, d)
+    o = oracle_mod.Graph(n, s, d)
+    for k in (3, 4):
+        got = g.motifs(k)
+        for name, e in G.MOTIFS[k].items():
+            assert got[name] == o.match(k, e, induced=True)[0], (k, name)
+    m3 = g.motifs(3)
+    rp, _ = g.csr()
+    deg = np.diff(np.asarray(rp, dtype=np.int64))
+    assert m3["wedge"] + 3 * m3["triangle"] == int((deg * (deg - 1) // 2).sum())
+    m4 = g.motifs(4)
+    # non-induced 3-stars: each induced star 1, tailed triangle 1, diamond 2, K4 4
+    assert m4["star"] + m4["tailed_triangle"] + 2 * m4["diamond"] + 4 * m4["k4"] == \
+        int((deg * (deg - 1) * (deg - 2) // 6).sum())

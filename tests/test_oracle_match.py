@@ -195,3 +195,23 @@ def test_induced_brute_force(oracle_mod, seed, q):
     assert g0.match(nv, e, induced=True)[0] == brute.induced_subgraphs(n, E, nv, e)
     plab = [i % 2 for i in range(nv)]
     assert g.match(nv, e, plab, induced=True)[0] == brute.induced_subgraphs(n, E, nv, e, plab, lab)
+
+
+@pytest.mark.parametrize("seed", [4, 5])
+def test_induced_degree_identities(oracle_mod, seed):
+    """sum_v C(d,2) = iWedge + 3T; sum_v C(d,3) = iStar + iTT + 2 iDiamond + 4 iK4
+    (the 3-stars inside each connected 4-vertex graph)."""
+    n = 80
+    s, d = gg.er(n, 600, seed)
+    E = brute.normalise(s, d)
+    deg = [0] * n
+    for e in E:
+        for x in e:
+            deg[x] += 1
+    g = oracle_mod.Graph(n, s, d)
+    iw = g.match(3, [(0, 1), (1, 2)], induced=True)[0]
+    t = g.kclique(3)
+    assert iw + 3 * t == sum(comb(x, 2) for x in deg)
+    ist = g.match(4, [(0, 1), (0, 2), (0, 3)], induced=True)[0]
+    assert ist + icount(g, "tailed_triangle") + 2 * icount(g, "diamond") + 4 * icount(g, "k4") == \
+        sum(comb(x, 3) for x in deg)
