@@ -14,6 +14,7 @@ The C names are re-exported 1:1 (``gamma_ctx_create``, ``gamma_load_edges``,
 from __future__ import annotations
 
 import ctypes as C
+import os
 import sys
 import weakref
 from typing import Optional
@@ -177,8 +178,11 @@ class Context:
 
     def __init__(self, device: int = 0, rank: Optional[int] = None, world: Optional[int] = None,
                  use_torch: bool = True, hbm_budget_bytes: int = 0, host_spill_bytes: int = 0,
-                 time_kernels: bool = False, flags: int = 0, reduce: bool = True):
+                 time_kernels: bool = False, flags: int = 0, reduce: bool = True,
+                 torch_alloc: Optional[bool] = None):
         self._keep = []
+        if torch_alloc is None:   # GAMMA_ALLOC=native: the library's stream-ordered pool
+            torch_alloc = os.environ.get("GAMMA_ALLOC", "torch") != "native"
         self._graphs = weakref.WeakSet()
         d = N.gamma_ctx_desc()
         d.device = device
@@ -198,6 +202,8 @@ class Context:
             torch = self._torch
             stream = torch.cuda.current_stream(device)
             d.stream = C.c_void_p(stream.cuda_stream)
+        if self._torch is not None and self._torch.cuda.is_available() and torch_alloc:
+            torch = self._torch
             dev = device
 
             def _alloc(size, strm, user):

@@ -147,6 +147,12 @@ gamma_status gamma_ctx_create(const gamma_ctx_desc *desc, gamma_ctx **out) {
         GAMMA_CUDA(cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking));
         c->own_stream = true;
       }
+      if (!desc->dev_alloc) {   // native allocation: keep freed blocks in the stream-ordered
+        cudaMemPool_t pool;     // pool across synchronisations (default threshold 0 trims them)
+        GAMMA_CUDA(cudaDeviceGetDefaultMemPool(&pool, c->device));
+        uint64_t keep = ~0ull;
+        GAMMA_CUDA(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep));
+      }
       GAMMA_CUDA(cudaMalloc(&c->ctrl, CTRL_WORDS * sizeof(uint64_t)));
       GAMMA_CUDA(cudaMallocHost(&c->ctrl_host, CTRL_WORDS * sizeof(uint64_t)));
       c->reset_stats();

@@ -884,6 +884,12 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
   }
   // ---- pattern table + per-(slot, position) domain bitmaps ----
   size_t fr = 0, tot = 0;
+  if (!ctx->desc.dev_alloc) {   // native pool: hand its idle blocks back before sizing from free HBM
+    cudaMemPool_t pool;
+    GAMMA_CUDA(cudaStreamSynchronize(ctx->stream));
+    GAMMA_CUDA(cudaDeviceGetDefaultMemPool(&pool, ctx->device));
+    GAMMA_CUDA(cudaMemPoolTrimTo(pool, 0));
+  }
   GAMMA_CUDA(cudaMemGetInfo(&fr, &tot));
   const uint64_t budget = ctx->desc.hbm_budget_bytes ? ctx->desc.hbm_budget_bytes : (uint64_t)(fr * 0.85);
   std::vector<uint32_t> hsize(nlab);

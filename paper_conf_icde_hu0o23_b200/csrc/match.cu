@@ -48,6 +48,7 @@ constexpr uint32_t kOutCap = 512;    // default staged child run per warp (u32);
 // (both are launch parameters, SmArgs::lm_cap / out_cap: the shared-memory footprint
 // sets the CTAs per SM; GAMMA_SM_LMCAP / GAMMA_SM_OUTCAP override them for tuning;
 // C3 sweep on B200: 512/512 233 ms, 256/256 243, 1024/512 272, 2048/512 338 per step)
+constexpr uint32_t kLongRatio = 1;   // see SmArgs::long_ratio (GAMMA_SM_LONGRATIO overrides; 0 = off)
 constexpr uint32_t kBlkV = 4096;
 constexpr uint32_t kBlkG = 256;      // descriptors per warp block
 constexpr uint32_t kSlice = 64;      // children per group descriptor
@@ -86,6 +87,7 @@ struct SmArgs {
   uint32_t *lm_scratch;     // per-warp global L_m slices for hub prefixes (nullable)
   uint32_t lm_scratch_cap;  // entries per warp slice
   uint32_t lm_cap, out_cap; // shared-memory staging per warp (u32 entries)
+  uint32_t long_ratio;      // last level: child lists > long_ratio * |L_m| are probed from L_m (0: off)
 };
 
 __device__ __forceinline__ uint32_t gdeg(const SmArgs &a, uint32_t v) {
@@ -202,7 +204,7 @@ __device__ uint32_t sm_intersect(const SmArgs &a, uint32_t q, uint32_t lists, co
   return found;
 }
 
-__global__ void __launch_bounds__(kThreads) sm_kernel(SmArgs a) {
+__global__ void __launch_bounds__(kThreads, 5) sm_kernel(SmArgs a) {
   extern __shared__ uint32_t smem[];
   const int lane = threadIdx.x & 31;
   const int wid = threadIdx.x >> 5;
@@ -302,6 +304,7 @@ __global__ void __launch_bounds__(kThreads) sm_kernel(SmArgs a) {
           // in shared memory
           const uint32_t lmin = lm[0], lmax = lm[lm_len - 1];
           const uint32_t upto = lane == 31 ? 0xffffffffu : ((2u << lane) - 1u);
+          const uint64_t long_at = a.long_ratio ? (uint64_t)a.long_ratio * lm_len : ~0ull;
           for (uint32_t w0 = 0; w0 < len; w0 += 32) {
             const uint32_t i = w0 + lane;
             uint32_t c = 0, beg = 0, dl = 0;
@@ -312,6 +315,32 @@ __global__ void __launch_bounds__(kThreads) sm_kernel(SmArgs a) {
               beg = (uint32_t)s0;
             }
             elems += dl;
+            // hub children (N(c) much longer than L_m): probe N(c) from L_m's side, one
+            // binary search per L_m element inside the child's order window, instead of
+            // streaming the whole list (the shorter side drives, as in sm_intersect)
+            const uint32_t dl0 = dl;
+            uint32_t lmask = __ballot_sync(0xffffffffu, (uint64_t)dl > long_at);
+            if (dl > long_at) dl = 0;
+            while (lmask) {
+              const int src = __ffs(lmask) - 1;
+              lmask &= lmask - 1;
+              const uint32_t cj = __shfl_sync(0xffffffffu, c, src);
+              const uint32_t bj = __shfl_sync(0xffffffffu, beg, src);
+              const uint32_t dj = __shfl_sync(0xffffffffu, dl0, src);
+              const int64_t lo = lt_d ? max(bs.lo, (int64_t)cj) : bs.lo;
+              const uint32_t hi = gt_d ? min(bs.hi, cj) : bs.hi;
+              const uint32_t a0 = lo < 0 ? 0u : upper_bound_idx(lm, lm_len, (uint32_t)lo);
+              const uint32_t a1 = hi == 0 ? 0u : upper_bound_idx(lm, lm_len, hi - 1);
+              for (uint32_t t0 = a0; t0 < a1; t0 += 32) {
+                const uint32_t t = t0 + lane;
+                bool ok = false;
+                if (t < a1) {
+                  const uint32_t x = lm[t];
+                  ok = !(inj_d && x == cj) && sorted_contains(a.col + bj, dj, x);
+                }
+                part += __popc(__ballot_sync(0xffffffffu, ok)) * (lane == 0);
+              }
+            }
             const uint32_t nz = __ballot_sync(0xffffffffu, dl > 0);
             const uint32_t nnz = __popc(nz);
             const uint32_t src = lane < (int)nnz ? __fns(nz, 0, lane + 1) : 0;
@@ -540,6 +569,10 @@ static uint32_t sm_out_cap() {
   static const uint32_t v = env_u32("GAMMA_SM_OUTCAP", kOutCap, 64, 4096);
   return v;
 }
+static uint32_t sm_long_ratio() {
+  static const uint32_t v = env_u32("GAMMA_SM_LONGRATIO", kLongRatio, 0, 1u << 20);
+  return v;
+}
 static size_t sm_smem() { return (size_t)kWarps * (sm_lm_cap() + sm_out_cap()) * sizeof(uint32_t); }
 
 }  // namespace
@@ -709,6 +742,7 @@ struct SmRun {
     a.lm_scratch_cap = lm_scratch_cap;
     a.lm_cap = sm_lm_cap();
     a.out_cap = sm_out_cap();
+    a.long_ratio = sm_long_ratio();
     return a;
   }
 

@@ -245,3 +245,44 @@ def test_motifs(ctx, oracle_mod):
     # non-induced 3-stars: each induced star 1, tailed triangle 1, diamond 2, K4 4
     assert m4["star"] + m4["tailed_triangle"] + 2 * m4["diamond"] + 4 * m4["k4"] == \
         int((deg * (deg - 1) * (deg - 2) // 6).sum())
+
+
+_SUB = r"""
+import json, sys
+sys.path.insert(0, sys.argv[1])
+import gamma_gen as gg
+import paper_conf_icde_hu0o23_b200 as G
+n, s, d, lab = gg.config_graph("c3", seed=2, scale=12)
+c = G.Context(device=0)
+g, g0 = c.load_edges(n, s, d, lab), c.load_edges(n, s, d)
+out = {}
+for q in ("c4", "diamond", "tailed_triangle", "house"):
+    nv, e = gg.QUERIES[q]
+    out[q + "/0"] = g0.match(nv, e)[0]
+    out[q + "/m"] = g.match(nv, e, [i % 8 for i in range(nv)])[0]
+print(json.dumps(out))
+"""
+
+
+@pytest.mark.parametrize("ratio", ["0", "1", "8"])
+def test_last_level_long_child_probe(oracle_mod, ratio):
+    """Last-level counting over a long staged L_m: hub children (|N(c)| > ratio * |L_m|)
+    are probed from L_m's side (binary search into N(c)) instead of streamed; ratio 0
+    turns the probe off, 1 sends nearly every child through it.  Same counts as the
+    oracle either way (each process reads GAMMA_SM_LONGRATIO once); unlabeled graph
+    (hub-heavy L_m and children) and 8 labels."""
+    import json
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, GAMMA_SM_LONGRATIO=ratio)
+    r = subprocess.run([sys.executable, "-c", _SUB, root], env=env, capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, r.stderr[-2000:]
+    got = json.loads(r.stdout.strip().splitlines()[-1])
+    n, s, d, lab = gg.config_graph("c3", seed=2, scale=12)
+    o, o0 = oracle_mod.Graph(n, s, d, lab), oracle_mod.Graph(n, s, d)
+    for q in ("c4", "diamond", "tailed_triangle", "house"):
+        nv, e = Q[q]
+        assert got[q + "/0"] == o0.match(nv, e)[0], (ratio, q, "unlabeled")
+        assert got[q + "/m"] == o.match(nv, e, [i % 8 for i in range(nv)])[0], (ratio, q, "imod8")

@@ -32,9 +32,13 @@ def main():
             torch.cuda.synchronize()
             ms = 1e3 * (time.perf_counter() - t)
             st = c.stats()
+            cur = (ms, cnt, {k: (v["launches"], round(v["ms"], 2)) for k, v in st["classes"].items()
+                             if v["launches"]}, st.get("level_entries"))
+            if os.environ.get("SMQ_ALL"):
+                print(f"  rep {q}/{tag}: {ms:.2f} ms kernels={cur[2]} retries={st['retries']} "
+                      f"chunks={st['chunks']}", flush=True)
             if best is None or ms < best[0]:
-                best = (ms, cnt, {k: (v["launches"], round(v["ms"], 2)) for k, v in st["classes"].items()
-                                  if v["launches"]}, st.get("level_entries"))
+                best = cur
         print(f"{q}/{tag}: {best[0]:.2f} ms count={best[1]} classes={best[2]} levels={best[3]}", flush=True)
 
 
