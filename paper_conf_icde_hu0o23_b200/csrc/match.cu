@@ -101,11 +101,13 @@ struct Bounds {
   uint32_t anti;  // induced: positions to check x not in N(phi_j)
 };
 
-// Candidate filter for position q.
+// Candidate filter for position q.  `staged`: x comes from (or was found in) a staged
+// L_m, whose entries already passed position q's label and degree filters, so only the
+// bounds, injectivity and anti-edge checks remain (no label / row-pointer gathers).
 __device__ __forceinline__ bool sm_filter(const SmArgs &a, uint32_t q, uint32_t x, const Bounds &b,
-                                          const uint32_t *phi, bool last) {
+                                          const uint32_t *phi, bool last, bool staged = false) {
   if ((int64_t)x <= b.lo || x >= b.hi) return false;
-  if (a.P.labeled) {
+  if (a.P.labeled && !staged) {
     const uint32_t lx = a.lab ? a.lab[x] : 0u;
     if (lx != a.P.label[q]) return false;
   }
@@ -115,7 +117,7 @@ __device__ __forceinline__ bool sm_filter(const SmArgs &a, uint32_t q, uint32_t 
     m &= m - 1;
     if (phi[j] == x) return false;
   }
-  if (!last && a.P.mindeg[q] > 1 && gdeg(a, x) < a.P.mindeg[q]) return false;
+  if (!last && !staged && a.P.mindeg[q] > 1 && gdeg(a, x) < a.P.mindeg[q]) return false;
   m = b.anti;   // induced: anti-edge checks, one binary search per non-neighbour
   while (m) {
     const int j = __ffs(m) - 1;
@@ -182,8 +184,10 @@ __device__ uint32_t sm_intersect(const SmArgs &a, uint32_t q, uint32_t lists, co
   for (uint32_t j0 = start; j0 < dlen; j0 += 32) {
     const uint32_t jj = j0 + lane;
     const uint32_t x = jj < dlen ? drv[jj] : 0xffffffffu;
-    bool ok = jj < dlen && sm_filter(a, q, x, bd, phi, last);
+    // membership in the staged L_m (shared memory) before the gathers of the full filter
+    bool ok = jj < dlen && (int64_t)x > bd.lo && x < bd.hi;
     if (ok && lm && !drive_lm) ok = sorted_contains(lm, lm_len, x);
+    ok = ok && sm_filter(a, q, x, bd, phi, last, lm != nullptr);
     uint32_t pm = probes;
     while (ok && pm) {
       const int j = __ffs(pm) - 1;
@@ -573,6 +577,10 @@ static uint32_t sm_long_ratio() {
   static const uint32_t v = env_u32("GAMMA_SM_LONGRATIO", kLongRatio, 0, 1u << 20);
   return v;
 }
+static uint32_t sm_batch() {   // groups per work-queue atomic below the roots
+  static const uint32_t v = env_u32("GAMMA_SM_BATCH", 4, 1, 256);
+  return v;
+}
 static size_t sm_smem() { return (size_t)kWarps * (sm_lm_cap() + sm_out_cap()) * sizeof(uint32_t); }
 
 }  // namespace
@@ -736,7 +744,7 @@ struct SmRun {
     a.g_begin = g0;
     a.g_end = g1;
     a.ctrl = (unsigned long long *)ctx->ctrl;
-    a.batch = d == 0 ? 1 : 4;
+    a.batch = d == 0 ? 1 : sm_batch();
     a.stage = stage;
     a.lm_scratch = lm_scratch.p;
     a.lm_scratch_cap = lm_scratch_cap;
