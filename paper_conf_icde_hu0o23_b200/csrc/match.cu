@@ -51,7 +51,11 @@ constexpr uint32_t kOutCap = 512;    // default staged child run per warp (u32);
 constexpr uint32_t kLongRatio = 1;   // see SmArgs::long_ratio (GAMMA_SM_LONGRATIO overrides; 0 = off)
 constexpr uint32_t kBlkV = 4096;
 constexpr uint32_t kBlkG = 256;      // descriptors per warp block
-constexpr uint32_t kSlice = 64;      // children per group descriptor
+constexpr uint32_t kSlice = 64;      // children per group descriptor when the count level consumes them
+constexpr uint32_t kSliceExt = 16;   // ... when an extension level does (SmArgs::slice; GAMMA_SM_SLICE /
+                                     // GAMMA_SM_SLICE_EXT; C3 sweep in profiles/sm_r01: finer groups
+                                     // balance the extension levels, the count level prefers fewer
+                                     // L_m rebuilds)
 constexpr uint32_t kRootChunk = 16;  // roots per depth-0 group
 
 struct SmPlan {
@@ -87,6 +91,7 @@ struct SmArgs {
   uint32_t *lm_scratch;     // per-warp global L_m slices for hub prefixes (nullable)
   uint32_t lm_scratch_cap;  // entries per warp slice
   uint32_t lm_cap, out_cap; // shared-memory staging per warp (u32 entries)
+  uint32_t slice;           // children per group descriptor of the next level
   uint32_t long_ratio;      // last level: child lists > long_ratio * |L_m| are probed from L_m (0: off)
 };
 
@@ -476,7 +481,8 @@ __global__ void __launch_bounds__(kThreads, 5) sm_kernel(SmArgs a) {
           for (uint32_t t = lane; t < found; t += 32) a.vid_out[pos + t] = sout[t];
         }
         // descriptors: slices of kSlice children, each carrying the prefix + c
-        const uint32_t ns = (found + kSlice - 1) / kSlice;
+        const uint32_t slice = a.slice;
+        const uint32_t ns = (found + slice - 1) / slice;
         uint64_t gpos;
         if (ns <= kBlkG)
           wb_retire_tail(wg, ns, lane, [&](uint64_t s) { a.desc_out[s * a.dw_out + 1] = 0u; });
@@ -486,8 +492,8 @@ __global__ void __launch_bounds__(kThreads, 5) sm_kernel(SmArgs a) {
           uint32_t *o = a.desc_out + (gpos + s) * a.dw_out;
           if (lane < (int)a.dw_out) {
             uint32_t val;
-            if (lane == 0) val = (uint32_t)(pos + s * kSlice);
-            else if (lane == 1) val = min(kSlice, found - s * kSlice);
+            if (lane == 0) val = (uint32_t)(pos + s * slice);
+            else if (lane == 1) val = min(slice, found - s * slice);
             else val = phi[0];
 #pragma unroll
             for (int j = 0; j < kMaxV; j++)
@@ -578,8 +584,13 @@ static uint32_t sm_long_ratio() {
   return v;
 }
 static uint32_t sm_batch() {   // groups per work-queue atomic below the roots
-  static const uint32_t v = env_u32("GAMMA_SM_BATCH", 4, 1, 256);
+  static const uint32_t v = env_u32("GAMMA_SM_BATCH", 2, 1, 256);   // C3: 1 164, 2 156, 4 171, 8 213 ms
   return v;
+}
+static uint32_t sm_slice(bool consumer_last) {
+  static const uint32_t v = env_u32("GAMMA_SM_SLICE", kSlice, 8, 1024);
+  static const uint32_t e = env_u32("GAMMA_SM_SLICE_EXT", kSliceExt, 8, 1024);
+  return consumer_last ? v : e;
 }
 static size_t sm_smem() { return (size_t)kWarps * (sm_lm_cap() + sm_out_cap()) * sizeof(uint32_t); }
 
@@ -751,6 +762,7 @@ struct SmRun {
     a.lm_cap = sm_lm_cap();
     a.out_cap = sm_out_cap();
     a.long_ratio = sm_long_ratio();
+    a.slice = sm_slice(d + 2 >= P.nv - 1);   // the groups written here are consumed at depth d+1
     return a;
   }
 
