@@ -380,6 +380,11 @@ def run_gamma(args):
     for _ in range(args.warmup):
         step(src_dev, dst_dev, lab_dev, False)
     torch.cuda.synchronize()
+    if os.environ.get("GAMMA_BENCH_GC", "1") == "0":   # diagnostics: no cyclic GC in the timed region
+        import gc
+        gc.collect()
+        gc.freeze()
+        gc.disable()
 
     clocks = ClockSampler(dev)
     if not args.no_clocks:

@@ -73,6 +73,29 @@ void *gamma_ctx::alloc(size_t bytes) {
   return p;
 }
 
+void *gamma_ctx::keep_take(size_t bytes, size_t &got) {
+  size_t best = kept.size();
+  for (size_t i = 0; i < kept.size(); i++)
+    if (kept[i].second >= bytes && (best == kept.size() || kept[i].second < kept[best].second)) best = i;
+  if (best < kept.size()) {
+    void *p = kept[best].first;
+    got = kept[best].second;
+    kept.erase(kept.begin() + best);
+    return p;
+  }
+  got = bytes;
+  return alloc(bytes);
+}
+
+void gamma_ctx::keep_give(void *p, size_t bytes) {
+  if (p) kept.emplace_back(p, bytes);
+}
+
+void gamma_ctx::keep_release() {
+  for (auto &b : kept) free(b.first);
+  kept.clear();
+}
+
 void gamma_ctx::free(void *p) {
   if (!p) return;
   if (desc.dev_free) desc.dev_free(p, desc.alloc_user);
@@ -168,6 +191,10 @@ void gamma_ctx_destroy(gamma_ctx *ctx) {
   if (!ctx) return;
   cudaSetDevice(ctx->device);
   if (ctx->stream) cudaStreamSynchronize(ctx->stream);
+  try {
+    ctx->keep_release();
+  } catch (...) {
+  }
   if (ctx->ctrl) cudaFree(ctx->ctrl);
   if (ctx->ctrl_host) cudaFreeHost(ctx->ctrl_host);
   if (ctx->spill_host) cudaFreeHost(ctx->spill_host);
@@ -288,6 +315,7 @@ gamma_status gamma_kclique(gamma_graph *g, uint32_t k, uint64_t *count) {
     gamma_ctx *c = g->ctx;
     GAMMA_CUDA(cudaSetDevice(c->device));
     c->reset_stats();
+    c->keep_release();   // kCL sizes its levels from free HBM
     auto t0 = std::chrono::steady_clock::now();
     uint64_t r = kclique_count(g, k, nullptr, 0, nullptr);
     if (c->desc.world > 1 && c->desc.allreduce_sum_u64) {
@@ -311,6 +339,7 @@ gamma_status gamma_kclique_multi(gamma_graph *g, uint32_t nk, const uint32_t *ks
     gamma_ctx *c = g->ctx;
     GAMMA_CUDA(cudaSetDevice(c->device));
     c->reset_stats();
+    c->keep_release();   // kCL sizes its levels from free HBM
     if (nk == 0) return;
     auto t0 = std::chrono::steady_clock::now();
     uint64_t bysize[33] = {};
@@ -336,6 +365,7 @@ gamma_status gamma_kclique_roots(gamma_graph *g, uint32_t k, uint64_t nroots, co
     gamma_ctx *c = g->ctx;
     GAMMA_CUDA(cudaSetDevice(c->device));
     c->reset_stats();
+    c->keep_release();   // kCL sizes its levels from free HBM
     if (nroots == 0) return;
     DevBuf<uint32_t> r = to_device(c, roots, nroots);
     DevBuf<uint64_t> out(c, nroots);

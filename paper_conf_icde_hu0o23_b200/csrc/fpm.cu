@@ -1105,6 +1105,7 @@ extern "C" gamma_status gamma_fpm(gamma_graph *g, uint32_t max_edges, uint64_t m
     gamma_ctx *c = g->ctx;
     GAMMA_CUDA(cudaSetDevice(c->device));
     c->reset_stats();
+    c->keep_release();   // FPM sizes its pattern table and domain pool from free HBM
     const auto t0 = std::chrono::steady_clock::now();
     std::vector<gamma_fpm_pattern> pats;
     fpm_run(g, max_edges, minsup, pats);

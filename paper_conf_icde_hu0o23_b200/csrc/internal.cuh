@@ -100,6 +100,12 @@ struct gamma_ctx {
 
   void *alloc(size_t bytes);
   void free(void *p);
+  // Idle device buffers kept across calls (SM level tables and L_m scratch): sizing them
+  // from free HBM per call made consecutive calls ask the allocator for different sizes.
+  std::vector<std::pair<void *, size_t>> kept;
+  void *keep_take(size_t bytes, size_t &got);   // smallest kept buffer >= bytes, else alloc
+  void keep_give(void *p, size_t bytes);
+  void keep_release();                          // free every kept buffer
   void reset_stats();
   // Launch helper: brackets the launch with events when timing is on.
   template <class F>
@@ -179,21 +185,32 @@ struct DevBuf {
   gamma_ctx *ctx = nullptr;
   T *p = nullptr;
   size_t n = 0;
+  size_t bytes = 0;   // kept buffers: the size actually held
+  bool kept = false;  // taken from / returned to the context's kept-buffer list
   DevBuf() = default;
   DevBuf(gamma_ctx *c, size_t count) : ctx(c), n(count) {
     p = static_cast<T *>(c->alloc(count * sizeof(T) ? count * sizeof(T) : 16));
   }
+  // kept = true: reuse an idle buffer of >= count elements kept by the context from an
+  // earlier call (no allocator round trip), and keep this one when it is released
+  DevBuf(gamma_ctx *c, size_t count, bool keep) : ctx(c), n(count), kept(keep) {
+    const size_t want = count * sizeof(T) ? count * sizeof(T) : 16;
+    p = static_cast<T *>(keep ? c->keep_take(want, bytes) : c->alloc(want));
+  }
   DevBuf(const DevBuf &) = delete;
   DevBuf &operator=(const DevBuf &) = delete;
-  DevBuf(DevBuf &&o) noexcept : ctx(o.ctx), p(o.p), n(o.n) { o.p = nullptr; }
+  DevBuf(DevBuf &&o) noexcept : ctx(o.ctx), p(o.p), n(o.n), bytes(o.bytes), kept(o.kept) { o.p = nullptr; }
   DevBuf &operator=(DevBuf &&o) noexcept {
     reset();
-    ctx = o.ctx; p = o.p; n = o.n; o.p = nullptr;
+    ctx = o.ctx; p = o.p; n = o.n; bytes = o.bytes; kept = o.kept; o.p = nullptr;
     return *this;
   }
   ~DevBuf() { reset(); }
   void reset() {
-    if (p && ctx) ctx->free(p);
+    if (p && ctx) {
+      if (kept) ctx->keep_give(p, bytes);
+      else ctx->free(p);
+    }
     p = nullptr;
   }
   T *release() { T *q = p; p = nullptr; return q; }

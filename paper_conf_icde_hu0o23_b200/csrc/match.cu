@@ -734,8 +734,8 @@ struct SmRun {
     const uint64_t cg = cv / 8 + 2 * kBlkG;
     L.vid.reset();
     L.desc.reset();
-    L.vid = DevBuf<uint32_t>(ctx, cv);
-    L.desc = DevBuf<uint32_t>(ctx, cg * dw);
+    L.vid = DevBuf<uint32_t>(ctx, cv, true);
+    L.desc = DevBuf<uint32_t>(ctx, cg * dw, true);
     L.cap_v = cv;
     L.cap_g = cg;
     L.dw = dw;
@@ -920,7 +920,7 @@ static uint64_t match_count(gamma_graph *g, const SmPlan &P) {
   R.grid = ctx->num_sms * occupancy_blocks((const void *)sm_kernel, kThreads, sm_smem());
   if (g->max_degree > sm_lm_cap()) {   // room for a hub's L_m (bounded by its degree) per warp
     R.lm_scratch_cap = std::min<uint32_t>(g->max_degree, 1u << 16);
-    R.lm_scratch = DevBuf<uint32_t>(ctx, (uint64_t)R.grid * kWarps * R.lm_scratch_cap);
+    R.lm_scratch = DevBuf<uint32_t>(ctx, (uint64_t)R.grid * kWarps * R.lm_scratch_cap, true);
   }
   R.process(0, 0, ngr);
   ctx->sync();
