@@ -40,7 +40,7 @@
 extern "C" {
 #endif
 
-#define GAMMA_ABI_VERSION 2
+#define GAMMA_ABI_VERSION 3
 
 typedef int32_t gamma_status;
 enum {
@@ -97,12 +97,21 @@ typedef struct {
                                           sort instead of the global key sort (2m' < 2^31
                                           only; same CSR; slower on hub-heavy graphs, where
                                           the hub rows fall to CUB's large-segment kernel) */
+#define GAMMA_FLAG_FPM_INSTANCES 0x100u /* gamma_fpm: also count each pattern's instances
+                                          (connected edge sets mapped to it; one atomic
+                                          per embedding -- a parity check, not for timing) */
 
 /* Create / destroy a context.  Errors: E_INVAL (NULL args), E_CUDA (no device). */
 gamma_status gamma_ctx_create(const gamma_ctx_desc *desc, gamma_ctx **out);
 void gamma_ctx_destroy(gamma_ctx *ctx);
 const char *gamma_last_error(void);
 int32_t gamma_abi_version(void);
+/* Give every idle device buffer the context keeps across calls (SM level tables and
+ * L_m scratch, capped at 8 GiB) back to the allocator, then synchronise the stream.
+ * Call before trimming an external caching allocator (the Python binding does so
+ * before gamma_fpm, which sizes its pattern table and MNI domain pool from free HBM).
+ * Errors: E_INVAL (NULL), E_CUDA. */
+gamma_status gamma_ctx_trim(gamma_ctx *ctx);
 
 /* ---- Graph data G_d (A1) ------------------------------------------------------
  * gamma_load_edges: build the graph from m raw samples (src[i], dst[i]) over n
@@ -193,6 +202,8 @@ typedef struct {
   uint32_t labels[8];        /* labels in canonical vertex order                     */
   uint8_t edges[8][2];       /* sorted (a<b) pairs in canonical positions            */
   uint64_t support;          /* MNI support                                          */
+  uint64_t instances;        /* edge sets mapped to the pattern (GAMMA_FLAG_FPM_INSTANCES;
+                                0 otherwise)                                         */
 } gamma_fpm_pattern;
 
 typedef struct {

@@ -358,12 +358,16 @@ class Graph:
             raise ValueError("motifs: k must be 3 or 4")
         return {name: self.match(k, e, induced=True)[0] for name, e in MOTIFS[k].items()}
 
-    def fpm(self, max_edges: int, minsup: int):
-        """Frequent patterns: sorted list of (ne, nv, labels, edges, support)."""
+    def fpm(self, max_edges: int, minsup: int, instances: bool = False):
+        """Frequent patterns: sorted list of (ne, nv, labels, edges, support); with
+        ``instances`` (needs a Context created with GAMMA_FLAG_FPM_INSTANCES) each
+        tuple also carries the pattern's instance count (connected edge sets)."""
         t = self.ctx._torch
         if t is not None and t.cuda.is_available():
-            # the MNI domain pool is sized from free HBM: give the caching allocator's
-            # idle blocks (e.g. the previous call's pool) back first
+            # the MNI domain pool is sized from free HBM: return the context's kept
+            # buffers to the caching allocator, then its idle blocks (e.g. the previous
+            # call's pool) to the device
+            _check(_lib.gamma_ctx_trim(self.ctx._h), "gamma_ctx_trim")
             t.cuda.empty_cache()
         r = C.POINTER(N.gamma_fpm_result)()
         _check(_lib.gamma_fpm(self._h, int(max_edges), int(minsup), C.byref(r)), "gamma_fpm")
@@ -374,7 +378,7 @@ class Graph:
                 pt = res.pats[i]
                 out.append((int(pt.ne), int(pt.nv), tuple(int(pt.labels[j]) for j in range(pt.nv)),
                             tuple((int(pt.edges[e][0]), int(pt.edges[e][1])) for e in range(pt.ne)),
-                            int(pt.support)))
+                            int(pt.support)) + ((int(pt.instances),) if instances else ()))
             return out
         finally:
             _lib.gamma_fpm_result_free(r)

@@ -26,6 +26,7 @@ GAMMA_FLAG_NO_BITMAP = 0x10
 GAMMA_FLAG_NO_SPLIT = 0x20
 GAMMA_FLAG_DEBUG_SPLIT_ALL = 0x40
 GAMMA_FLAG_COUNT_SORT_BUILD = 0x80
+GAMMA_FLAG_FPM_INSTANCES = 0x100
 
 ALLOC_FN = C.CFUNCTYPE(C.c_void_p, C.c_size_t, C.c_void_p, C.c_void_p)
 FREE_FN = C.CFUNCTYPE(None, C.c_void_p, C.c_void_p)
@@ -62,7 +63,8 @@ class gamma_plan_info(C.Structure):
 
 class gamma_fpm_pattern(C.Structure):
     _fields_ = [("nv", C.c_uint32), ("ne", C.c_uint32), ("labels", C.c_uint32 * 8),
-                ("edges", (C.c_uint8 * 2) * 8), ("support", C.c_uint64)]
+                ("edges", (C.c_uint8 * 2) * 8), ("support", C.c_uint64),
+                ("instances", C.c_uint64)]
 
 
 class gamma_fpm_result(C.Structure):
@@ -92,6 +94,7 @@ SIGNATURES = [
     ("gamma_last_error", C.c_char_p, []),
     ("gamma_ctx_create", C.c_int32, [C.POINTER(gamma_ctx_desc), C.POINTER(C.c_void_p)]),
     ("gamma_ctx_destroy", None, [C.c_void_p]),
+    ("gamma_ctx_trim", C.c_int32, [C.c_void_p]),
     ("gamma_load_edges", C.c_int32, [C.c_void_p, C.c_uint32, C.c_void_p, C.c_void_p, C.c_uint64,
                                      C.c_void_p, C.POINTER(C.c_void_p)]),
     ("gamma_load_csr", C.c_int32, [C.c_void_p, C.c_uint32, C.c_void_p, C.c_void_p, C.c_void_p,

@@ -87,8 +87,18 @@ void *gamma_ctx::keep_take(size_t bytes, size_t &got) {
   return alloc(bytes);
 }
 
+// Kept bytes are capped (kKeepCap): beyond it a returned buffer is freed instead.
+static constexpr size_t kKeepCap = 8ull << 30;
+
 void gamma_ctx::keep_give(void *p, size_t bytes) {
-  if (p) kept.emplace_back(p, bytes);
+  if (!p) return;
+  size_t held = 0;
+  for (auto &b : kept) held += b.second;
+  if (held + bytes > kKeepCap) {
+    free(p);
+    return;
+  }
+  kept.emplace_back(p, bytes);
 }
 
 void gamma_ctx::keep_release() {
@@ -204,6 +214,15 @@ void gamma_ctx_destroy(gamma_ctx *ctx) {
   delete ctx;
 }
 
+gamma_status gamma_ctx_trim(gamma_ctx *ctx) {
+  return guarded([&] {
+    GAMMA_REQUIRE(ctx, GAMMA_E_INVAL, "gamma_ctx_trim: NULL argument");
+    GAMMA_CUDA(cudaSetDevice(ctx->device));
+    ctx->keep_release();
+    GAMMA_CUDA(cudaStreamSynchronize(ctx->stream));
+  });
+}
+
 gamma_status gamma_get_stats(const gamma_ctx *ctx, gamma_run_stats *out) {
   return guarded([&] {
     GAMMA_REQUIRE(ctx && out, GAMMA_E_INVAL, "gamma_get_stats: NULL argument");
@@ -220,6 +239,7 @@ gamma_status gamma_load_edges(gamma_ctx *ctx, uint32_t n, const uint32_t *src, c
     GAMMA_REQUIRE(n < 0xFFFFFFFFu, GAMMA_E_INVAL, "gamma_load_edges: n too large");
     GAMMA_CUDA(cudaSetDevice(ctx->device));
     ctx->reset_stats();
+    ctx->keep_release();   // the build's scratch is sized from the input, not from kept buffers
     auto *g = new gamma_graph();
     g->ctx = ctx;
     g->n = n;
@@ -245,6 +265,7 @@ gamma_status gamma_load_csr(gamma_ctx *ctx, uint32_t n, const uint64_t *row_ptr,
     GAMMA_REQUIRE(n > 0 && n < 0xFFFFFFFFu, GAMMA_E_INVAL, "gamma_load_csr: bad n");
     GAMMA_CUDA(cudaSetDevice(ctx->device));
     ctx->reset_stats();
+    ctx->keep_release();
     auto *g = new gamma_graph();
     g->ctx = ctx;
     g->n = n;
@@ -274,6 +295,10 @@ void gamma_graph_free(gamma_graph *g) {
     c->free(g->dag_col);
     c->free(g->labels);
     c->free(g->root_order);
+    try {
+      c->keep_release();   // kept SM tables were sized for this graph
+    } catch (...) {
+    }
     cudaStreamSynchronize(c->stream);
   }
   cudaGetLastError();

@@ -76,6 +76,7 @@ struct Table {
   uint32_t *pool;             // per-slot domains, one bitmap per position over its label class
   uint64_t pool_words;
   unsigned long long *pool_cur;
+  unsigned long long *inst;   // per-slot instance counts (GAMMA_FLAG_FPM_INSTANCES), nullable
 };
 
 __host__ __device__ __forceinline__ uint32_t key_nv(uint64_t k) { return (uint32_t)((k >> 48) & 7); }
@@ -246,6 +247,8 @@ __device__ void record(const FpmArgs &a, const uint2 *tab, const uint32_t *prm, 
     d = __ldcg(&a.T.slots[2 * s + 1]);
   }
   if (d == ~0ull) return;   // no domains in this pass (pool exhausted / another chunk)
+  // instances: counted in the one pass that carves the slot's domains
+  if (a.T.inst) atomicAdd(&a.T.inst[s], 1ull);
   __threadfence();
   uint64_t off[4];
   off[0] = d - 1;
@@ -608,7 +611,7 @@ static void slots_put(gamma_ctx *ctx, unsigned long long *slots, const std::vect
   GAMMA_CUDA(cudaMemcpy2DAsync(slots + colm, 16, h.data(), 8, 8, cap, cudaMemcpyHostToDevice, ctx->stream));
 }
 
-static gamma_fpm_pattern decode_pattern(uint64_t key, uint64_t support) {
+static gamma_fpm_pattern decode_pattern(uint64_t key, uint64_t support, uint64_t instances = 0) {
   static const uint8_t pairs[6][2] = {{0, 1}, {0, 2}, {0, 3}, {1, 2}, {1, 3}, {2, 3}};
   gamma_fpm_pattern p{};
   p.nv = key_nv(key);
@@ -622,6 +625,7 @@ static gamma_fpm_pattern decode_pattern(uint64_t key, uint64_t support) {
     p.edges[e][1] = pairs[id][1];
   }
   p.support = support;
+  p.instances = instances;
   return p;
 }
 
@@ -775,16 +779,28 @@ static bool fpm_dist_level(gamma_ctx *ctx, FpmArgs &a, int grid_enum, uint32_t l
     ctx->launch(KC_FPM_SUPPORT, [&] {
       seg_popc_kernel<<<g1d(nseg * 32), 256, 0, ctx->stream>>>(recv_buf, R * shard, shard, soff.p, sw.p, nseg, cnt.p);
     });
-    std::vector<uint64_t> hc(nseg);
+    // per-segment popcounts, then (instance counting) each chunk pattern's instances
+    std::vector<uint64_t> hc(nseg + (a.T.inst ? j1 - j0 : 0), 0);
     GAMMA_CUDA(cudaMemcpyAsync(hc.data(), cnt.p, nseg * 8, cudaMemcpyDeviceToHost, ctx->stream));
+    std::vector<unsigned long long> hinst;
+    if (a.T.inst) {
+      hinst.resize(cap);
+      GAMMA_CUDA(cudaMemcpyAsync(hinst.data(), a.T.inst, cap * 8, cudaMemcpyDeviceToHost, ctx->stream));
+    }
     ctx->sync();
-    coll_allreduce(ctx, hc.data(), nseg);
+    if (a.T.inst)
+      for (size_t j = j0; j < j1; j++) {
+        auto it = slot_of.find(U[j]);
+        if (it != slot_of.end()) hc[nseg + (j - j0)] = hinst[it->second];
+      }
+    coll_allreduce(ctx, hc.data(), hc.size());
     size_t q = 0;
     for (size_t j = j0; j < j1; j++) {
       uint64_t sup = ~0ull;
       for (uint32_t p = 0; p < key_nv(U[j]); p++, q++) sup = std::min<uint64_t>(sup, hc[q]);
-      if (sup >= minsup) found.push_back(decode_pattern(U[j], sup));
+      if (sup >= minsup) found.push_back(decode_pattern(U[j], sup, a.T.inst ? hc[nseg + (j - j0)] : 0));
     }
+    if (a.T.inst) GAMMA_CUDA(cudaMemsetAsync(a.T.inst, 0, cap * 8, ctx->stream));
     ctx->stats.chunks++;
   }
   a.rank = 0;
@@ -921,7 +937,8 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
   while (cap > 1024 && cap * slot_bytes * 4 > budget) cap >>= 1;
   DevBuf<uint32_t> freq;
   PoolBuf pool;
-  DevBuf<unsigned long long> slots, sup, pcur;
+  DevBuf<unsigned long long> slots, sup, pcur, inst;
+  const bool want_inst = (ctx->desc.flags & GAMMA_FLAG_FPM_INSTANCES) != 0;
   FpmArgs a{};
   a.rp = g->row_ptr;
   a.col = g->col;
@@ -945,7 +962,7 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
     GAMMA_REQUIRE(cap * slot_bytes < budget, GAMMA_E_NOMEM, "gamma_fpm: pattern table exceeds the HBM budget");
     const uint64_t pool_words =
         std::max<uint64_t>(64, std::min<uint64_t>((budget - cap * slot_bytes) / 4, cap * 4 * maxw));
-    freq.reset(); pool.reset(); slots.reset(); sup.reset(); pcur.reset();
+    freq.reset(); pool.reset(); slots.reset(); sup.reset(); pcur.reset(); inst.reset();
     slots = DevBuf<unsigned long long>(ctx, 2 * cap);
     sup = DevBuf<unsigned long long>(ctx, cap);
     freq = DevBuf<uint32_t>(ctx, cap);
@@ -955,7 +972,11 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
     GAMMA_CUDA(cudaMemsetAsync(freq.p, 0, cap * 4, ctx->stream));
     GAMMA_CUDA(cudaMemsetAsync(pool.p, 0, pool_words * 4, ctx->stream));
     GAMMA_CUDA(cudaMemsetAsync(pcur.p, 0, 8, ctx->stream));
-    a.T = Table{slots.p, sup.p, freq.p, cap, pool.p, pool_words, pcur.p};
+    if (want_inst) {
+      inst = DevBuf<unsigned long long>(ctx, cap);
+      GAMMA_CUDA(cudaMemsetAsync(inst.p, 0, cap * 8, ctx->stream));
+    }
+    a.T = Table{slots.p, sup.p, freq.p, cap, pool.p, pool_words, pcur.p, want_inst ? inst.p : nullptr};
     bool full = false;
     found_last.clear();
     for (uint32_t l = 1; l <= max_edges && !full; l++) {
@@ -1067,15 +1088,16 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
   }
   // ---- collect the frequent patterns ----
   std::vector<uint32_t> hfreq(cap);
-  std::vector<unsigned long long> hkey, hsup(cap);
+  std::vector<unsigned long long> hkey, hsup(cap), hinst(want_inst ? cap : 0);
   GAMMA_CUDA(cudaMemcpyAsync(hfreq.data(), freq.p, cap * 4, cudaMemcpyDeviceToHost, ctx->stream));
+  if (want_inst) GAMMA_CUDA(cudaMemcpyAsync(hinst.data(), inst.p, cap * 8, cudaMemcpyDeviceToHost, ctx->stream));
   slots_get(ctx, hkey, slots.p, cap, 0);
   GAMMA_CUDA(cudaMemcpyAsync(hsup.data(), sup.p, cap * 8, cudaMemcpyDeviceToHost, ctx->stream));
   ctx->sync();
   for (uint64_t s = 0; s < cap; s++) {
     if (hkey[s] == 0 || !hfreq[s]) continue;
     if (dist && key_ne(hkey[s]) == max_edges) continue;   // from found_last
-    out.push_back(decode_pattern(hkey[s], hsup[s]));
+    out.push_back(decode_pattern(hkey[s], hsup[s], want_inst ? hinst[s] : 0));
   }
   out.insert(out.end(), found_last.begin(), found_last.end());
   std::sort(out.begin(), out.end(), [](const gamma_fpm_pattern &x, const gamma_fpm_pattern &y) {
@@ -1102,6 +1124,8 @@ extern "C" gamma_status gamma_fpm(gamma_graph *g, uint32_t max_edges, uint64_t m
     GAMMA_REQUIRE(minsup >= 1, GAMMA_E_INVAL, "gamma_fpm: minsup must be >= 1");
     GAMMA_REQUIRE(max_edges >= 1, GAMMA_E_INVAL, "gamma_fpm: max_edges must be >= 1");
     GAMMA_REQUIRE(max_edges <= 3, GAMMA_E_UNSUPPORTED, "gamma_fpm: max_edges > 3 not supported in v1");
+    // the enumeration carries symmetric-CSR offsets (< 2m) as u32
+    GAMMA_REQUIRE(2 * g->m < (1ull << 32), GAMMA_E_UNSUPPORTED, "gamma_fpm: graphs with 2m >= 2^32 unsupported");
     gamma_ctx *c = g->ctx;
     GAMMA_CUDA(cudaSetDevice(c->device));
     c->reset_stats();

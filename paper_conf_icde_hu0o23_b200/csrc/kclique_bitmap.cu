@@ -19,6 +19,7 @@
 // work list in a second launch (hub splitting, SURVEY.md §7 "skew").  Longer runs
 // (and k > 12) use the ET-level path in kclique.cu.
 #include <algorithm>
+#include <cstdlib>
 
 #include "device_common.cuh"
 #include "internal.cuh"
@@ -739,8 +740,20 @@ __global__ void GAMMA_BM_BOUNDS(KM) kcl_bitmap_kernel(BmArgs a) {
           const uint64_t want = est / kPartCost + 1;
           const uint32_t nparts = want < kMaxParts ? (uint32_t)want : kMaxParts;
           if (tid == 0) {
-            const unsigned long long at = atomicAdd(&a.ctrl[CTRL_AUX1], (unsigned long long)nparts);
-            if (at + nparts <= a.parts_cap) {
+            // reserve [at, at + nparts) only if it fits: the cursor never passes
+            // parts_cap, so every slot below it has been written by its reserver
+            // (the parts kernel reads exactly [0, cursor))
+            unsigned long long at = *(volatile unsigned long long *)&a.ctrl[CTRL_AUX1];
+            bool ok = false;
+            while (at + nparts <= a.parts_cap) {
+              const unsigned long long seen = atomicCAS(&a.ctrl[CTRL_AUX1], at, at + nparts);
+              if (seen == at) {
+                ok = true;
+                break;
+              }
+              at = seen;
+            }
+            if (ok) {
               for (uint32_t p = 0; p < nparts; p++)
                 a.parts[at + p] = make_uint2((uint32_t)(a.root_base + gi), p | (nparts << 16));
               m.slot[0] = 1;
@@ -817,9 +830,9 @@ __global__ void GAMMA_BM_BOUNDS(KM) kcl_bitmap_parts_kernel(BmArgs a) {
   uint64_t mc[kMaxStack + 3] = {};
   for (;;) {
     if (tid == 0) {
-      // the part list was filled by the previous launch; its length sits in ctrl
-      const unsigned long long np = *(volatile unsigned long long *)&a.ctrl[CTRL_AUX1];
-      const unsigned long long nparts_total = np < a.parts_cap ? np : a.parts_cap;
+      // the part list was filled by the previous launch; its length (<= parts_cap,
+      // every slot below it written) sits in ctrl
+      const unsigned long long nparts_total = *(volatile unsigned long long *)&a.ctrl[CTRL_AUX1];
       const unsigned long long w = atomicAdd(&a.ctrl[CTRL_WORK], 1ull);
       m.slot[0] = w < nparts_total ? (uint32_t)w : 0xffffffffu;
     }
@@ -1197,7 +1210,11 @@ uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint6
   const bool split = k >= 6 && (ctx->desc.flags & GAMMA_FLAG_NO_SPLIT) == 0;
   DevBuf<uint2> parts;
   if (split) {
-    a.parts_cap = 1u << 20;
+    // GAMMA_KCL_PARTS_CAP (tests): a small part list forces the "list full, expand
+    // here" fallback
+    const char *cap_env = getenv("GAMMA_KCL_PARTS_CAP");
+    a.parts_cap = cap_env && *cap_env ? (uint32_t)std::max(1ul, std::min(strtoul(cap_env, nullptr, 10), 1ul << 24))
+                                      : 1u << 20;
     parts = DevBuf<uint2>(ctx, a.parts_cap);
     a.parts = parts.p;
     a.heavy_cut = (ctx->desc.flags & GAMMA_FLAG_DEBUG_SPLIT_ALL) ? 1 : 4ull * kPartCost;

@@ -732,6 +732,10 @@ struct SmRun {
     cv = std::min<uint64_t>(cv, 0xFFFFFFFFull - kBlkV);
     if (cv <= L.cap_v) return false;
     const uint64_t cg = cv / 8 + 2 * kBlkG;
+    // the superseded (smaller) tables are freed, not kept: keeping them would hold
+    // ~1/3 more than level_share per level and shrink later budgets
+    L.vid.kept = false;
+    L.desc.kept = false;
     L.vid.reset();
     L.desc.reset();
     L.vid = DevBuf<uint32_t>(ctx, cv, true);
@@ -953,6 +957,8 @@ extern "C" gamma_status gamma_match(gamma_graph *g, const gamma_pattern *p, uint
                                     uint64_t *mappings) {
   return guarded([&] {
     GAMMA_REQUIRE(g && p && count, GAMMA_E_INVAL, "gamma_match: NULL argument");
+    // the extension kernels carry symmetric-CSR offsets (< 2m) as u32
+    GAMMA_REQUIRE(2 * g->m < (1ull << 32), GAMMA_E_UNSUPPORTED, "gamma_match: graphs with 2m >= 2^32 unsupported");
     SmPlan P;
     plan_pattern(p, P);
     gamma_ctx *c = g->ctx;

@@ -48,7 +48,7 @@ def test_binding_covers_every_symbol():
 
 def test_abi_version(lib):
     lib.gamma_abi_version.restype = C.c_int32
-    assert lib.gamma_abi_version() == 2
+    assert lib.gamma_abi_version() == 3
 
 
 def test_no_cpu_fallback():

@@ -9,8 +9,9 @@ per root ("full oracle on a seeded sample of root chunk
     vertex; R9) for a seeded sample of roots -- uniform over
     the roots with d+ >= 2 plus a stratified sample of the heavy tail -- equal the
     oracle's og_kclique_roots;
-  * the whole-graph multi-k pass agrees with the per-root kernel on the sampled roots'
-    share being non-negative and the totals being consistent (t4 > 0, t3 > 0).
+  * the whole-graph multi-k pass the bench times (gamma_kclique_multi) equals the
+    per-root path summed over ALL roots (a different launch configuration: unsorted
+    roots, every team kind filtering the full list, per-root atomics).
 Tolerance 0.  Needs ~70 GB of host memory (raw samples + oracle CSR); skipped below.
 """
 import numpy as np
@@ -33,6 +34,10 @@ def test_c5_sampled_roots(oracle_mod):
     info = g.info()
     t3, t4 = g.kclique_multi([3, 4])
     assert t3 > 0 and t4 > 0
+    every = np.arange(n, dtype=np.uint32)
+    assert int(g.kclique_roots(3, every).sum()) == t3
+    assert int(g.kclique_roots(4, every).sum()) == t4
+    del every
     s_host, d_host = src.cpu().numpy().view(np.uint32), dst.cpu().numpy().view(np.uint32)
     del src, dst
     torch.cuda.empty_cache()

@@ -109,3 +109,132 @@ def test_invalid(G, ctx):
     with pytest.raises(G.GammaError):
         g.fpm(2, 0)
     assert g.fpm(3, 100) == []
+
+
+def _closed_form_levels(o):
+    """Connected edge sets per size (SURVEY §8(c) O-3 pins): m, sum C(d,2),
+    T + sum C(d,3) + sum_{(u,v)} (d_u - 1)(d_v - 1) - 3T."""
+    off, adj = o.csr()
+    deg = np.diff(off.astype(np.int64))
+    src = np.repeat(np.arange(o.n), deg)
+    und = src < adj
+    du, dv = deg[src[und]], deg[adj[und].astype(np.int64)]
+    T = o.kclique(3)
+    return [int(und.sum()), int((deg * (deg - 1) // 2).sum()),
+            int(T + (deg * (deg - 1) * (deg - 2) // 6).sum() + ((du - 1) * (dv - 1)).sum() - 3 * T)]
+
+
+@pytest.mark.parametrize("case", ["er", "c4_11", "c4_12_l5"])
+def test_embedding_counts(G, oracle_mod, case):
+    """MNI hides duplicate or extra enumeration (an OR of bitmaps), so the embeddings
+    themselves are checked: at minsup = 1 every connected edge
+    set is enumerated once, so the GPU's per-level embedding counts equal the closed
+    forms and the oracle's summed per-pattern instance counts; at every minsup each
+    reported pattern's GPU instance count equals the oracle's."""
+    if case == "er":
+        n = 300
+        s, d = gg.er(n, 1500, 7)
+        lab = gg.labels(n, 3, 7)
+    elif case == "c4_11":
+        n, s, d, lab = gg.config_graph("c4", seed=1, scale=11)
+    else:
+        n, s, d, lab = gg.config_graph("c4", seed=2, scale=12)
+        lab = gg.labels(n, 5, 2)
+    c = G.Context(flags=G._native.GAMMA_FLAG_FPM_INSTANCES)
+    g = c.load_edges(n, s, d, lab)
+    o = oracle_mod.Graph(n, s, d, lab)
+    want_levels = _closed_form_levels(o)
+    got = g.fpm(3, 1, instances=True)
+    entries = c.stats()["level_entries"]
+    assert [entries[l] for l in (1, 2, 3)] == want_levels
+    ores = o.fpm(3, 1, pattern_cap=1 << 20)
+    assert [sum(r[5] for r in ores if r[0] == l) for l in (1, 2, 3)] == want_levels
+    assert got == [r[:6] for r in ores]
+    for minsup in (2, 5, 20):
+        assert g.fpm(3, minsup, instances=True) == [r[:6] for r in o.fpm(3, minsup, pattern_cap=1 << 20)], minsup
+
+
+def _canon(nv, labels, edges):
+    """Reading R7 written out for the test: min over vertex orders of (labels in
+    order, sorted edge-pair list), as the tuple layout gamma_fpm returns."""
+    import itertools
+    best = None
+    for p in itertools.permutations(range(nv)):   # p[i] = new position of vertex i
+        lab = [0] * nv
+        for i in range(nv):
+            lab[p[i]] = labels[i]
+        ed = tuple(sorted(tuple(sorted((p[a], p[b]))) for a, b in edges))
+        c = (tuple(lab), ed)
+        if best is None or c < best:
+            best = c
+    return (len(edges), nv) + best
+
+
+@pytest.mark.slow
+def test_c4_full_size_sampled(ctx, oracle_mod):
+    """configs[3] at full size (scale 22, L = 37, the bench's minsup = 3000), sampled
+    (no oracle can hold 10^6 patterns x 4 MNI bitmaps over 4M vertices): (a) the
+    support of >= 200 reported level-3 patterns, stratified by shape and including the
+    ones closest to minsup, equals the oracle's matching-based MNI (og_pattern_mni);
+    (b) >= 100 unreported 3-edge candidates grown from reported 2-edge patterns are
+    below minsup in the oracle; (c) every reported 1- and 2-edge pattern's support
+    equals the oracle's."""
+    import random
+    minsup = 3000
+    n, s, d, lab = gg.config_graph("c4", seed=1)
+    g = ctx.load_edges(n, s, d, lab)
+    o = oracle_mod.Graph(n, s, d, lab)
+    res = g.fpm(3, minsup)
+    got = {r[:4]: r[4] for r in res}
+    lv = {l: [r for r in res if r[0] == l] for l in (1, 2, 3)}
+    assert all(len(lv[l]) > 0 for l in (1, 2, 3))
+    rng = random.Random(5)
+
+    def mni(r):
+        return o.pattern_mni(r[1], list(r[3]), list(r[2]))
+
+    # (c) levels 1-2: a sample of 150 (or all) plus the 20 closest to minsup
+    for l in (1, 2):
+        pick = sorted(lv[l], key=lambda r: r[4])[:20] + rng.sample(lv[l], min(150, len(lv[l])))
+        for r in pick:
+            assert mni(r) == r[4], r
+    # (a) level 3 by shape (edge structure), near-minsup first
+    shapes = {}
+    for r in lv[3]:
+        shapes.setdefault(r[3], []).append(r)
+    checked = 0
+    for es, rs in shapes.items():
+        pick = sorted(rs, key=lambda r: r[4])[:10] + rng.sample(rs, min(50, len(rs)))
+        for r in pick:
+            assert mni(r) == r[4], r
+            checked += 1
+    assert checked >= 200
+    # (b) unreported candidates: a reported wedge (labels c; x, y) plus one edge
+    wedges = [r for r in lv[2] if r[1] == 3]
+    cands, tried = 0, 0
+    while cands < 100 and tried < 5000:
+        tried += 1
+        w = rng.choice(wedges)
+        (l0, l1, l2), es = w[2], w[3]
+        z = rng.randrange(37)
+        nv, e = 3, list(es)
+        kind = rng.randrange(3)
+        if kind == 0:
+            e.append([q for q in ((0, 1), (0, 2), (1, 2)) if q not in es][0])   # close the triangle
+            labels = [l0, l1, l2]
+        else:
+            anchor = rng.randrange(3)
+            e.append((anchor, 3))
+            nv, labels = 4, [l0, l1, l2, z]
+        if len(set(map(tuple, map(sorted, e)))) != 3:
+            continue
+        key = _canon(nv, labels, e)
+        if key[:2] != (3, nv):
+            continue
+        pat = (3, nv, key[2], key[3])
+        if pat in got:
+            continue
+        sup = o.pattern_mni(nv, e, labels)
+        assert sup < minsup, (pat, sup)
+        cands += 1
+    assert cands >= 100

@@ -289,15 +289,33 @@ def test_paths_agree(G, oracle_mod, flags):
     assert np.array_equal(g.kclique_roots(5, roots), o.kclique_roots(5, roots))
 
 
+@pytest.mark.parametrize("cap", [1, 3, 64])
+def test_parts_list_overflow(G, oracle_mod, monkeypatch, cap):
+    """Hub splitting with a part list too short for every deferred root:
+    a root whose parts do not fit is expanded by its own team, the parts kernel reads
+    only reserved slots, and every count still equals the oracle."""
+    monkeypatch.setenv("GAMMA_KCL_PARTS_CAP", str(cap))
+    c = G.Context(flags=0x40)   # GAMMA_FLAG_DEBUG_SPLIT_ALL: every k >= 6 root is deferred
+    n, s, d, _ = gg.config_graph("c1", seed=4)
+    g = c.load_edges(n, s, d)
+    o = oracle_mod.Graph(n, s, d)
+    assert g.kclique(6) == o.kclique(6)
+    assert g.kclique_multi([4, 5, 6, 7]) == [o.kclique(k) for k in (4, 5, 6, 7)]
+    roots = np.arange(0, n, 2, dtype=np.uint32)
+    assert np.array_equal(g.kclique_roots(6, roots), o.kclique_roots(6, roots))
+
+
 @pytest.mark.slow
 def test_c2_full_size(ctx, oracle_mod):
-    """configs[1] at full size: cit-Patents-shaped R-MAT scale 22, k = 4, 5, 6."""
+    """configs[1] at full size: cit-Patents-shaped R-MAT scale 22, k = 4, 5, 6, both
+    per k and through the one multi-k pass bench.py times (gamma_kclique_multi)."""
     n, s, d, _ = gg.config_graph("c2", seed=1)
     g = load(ctx, n, s, d)
     o = oracle_mod.Graph(n, s, d)
     assert g.info()["m"] == o.m
-    for k in (4, 5, 6):
-        assert g.kclique(k) == o.kclique(k), k
+    want = [o.kclique(k) for k in (4, 5, 6)]
+    assert [g.kclique(k) for k in (4, 5, 6)] == want
+    assert g.kclique_multi([4, 5, 6]) == want
 
 
 @pytest.mark.parametrize("case", ["c1", "er", "dups", "selfloops", "one"])
@@ -339,3 +357,20 @@ def test_builder_rejects_bad_ids(ctx):
     d = np.array([1, 2], np.uint32)
     with pytest.raises(Exception):
         ctx.load_edges(4, s, d)
+
+
+@pytest.mark.slow
+def test_heavy_full_size(ctx):
+    """The heavy kCL workload (Graph500-skew R-MAT scale 22, 20M samples, seed 1) at full
+    size, in the bench's configuration (one multi-k pass) and per k, against the
+    oracle's counts stored by tools/golden_heavy.py (oracle-only script)."""
+    import json
+    import os
+    gold = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "heavy_seed1.json")))
+    n, s, d, _ = gg.config_graph("heavy", seed=1)
+    g = load(ctx, n, s, d)
+    assert g.info()["m"] == gold["m"]
+    want = [gold["counts"][str(k)] for k in (3, 4, 5)]
+    assert g.kclique_multi([3, 4, 5]) == want
+    assert g.kclique_multi([4, 5]) == want[1:]
+    assert [g.kclique(k) for k in (4, 5)] == want[1:]

@@ -39,6 +39,35 @@ def test_normalisation_matches_set_definition(oracle_mod):
             assert v in adj[off[u]:off[u + 1]]
 
 
+@pytest.mark.parametrize("n,m", [(1 << 18, 2_000_000), ((1 << 18) + 77, 600_000)])
+def test_normalisation_bucketed_path(oracle_mod, n, m):
+    """O-0 at n > 65,536, where og_build sorts per bucket of the smaller endpoint across
+    threads: the CSR equals the set definition computed by numpy
+    (symmetrise, drop self-loops, dedup, ascending lists) on raw samples with planted
+    duplicates (both directions), self-loops and a hub."""
+    rng = np.random.default_rng(n)
+    s = rng.integers(0, n, m, dtype=np.uint32)
+    d = rng.integers(0, n, m, dtype=np.uint32)
+    k = m // 10
+    s[:k], d[:k] = d[k:2 * k], s[k:2 * k]          # reversed duplicates
+    d[2 * k:2 * k + 1000] = s[2 * k:2 * k + 1000]   # self-loops
+    s[3 * k:3 * k + 50_000] = 12345                 # a hub
+    g = oracle_mod.Graph(n, s, d)
+    lo, hi = np.minimum(s, d).astype(np.uint64), np.maximum(s, d).astype(np.uint64)
+    keep = lo != hi
+    und = np.unique((lo[keep] << np.uint64(32)) | hi[keep])
+    a, b = (und >> np.uint64(32)).astype(np.int64), (und & np.uint64(0xFFFFFFFF)).astype(np.int64)
+    assert g.m == und.size
+    src = np.concatenate([a, b])
+    dst = np.concatenate([b, a])
+    order = np.lexsort((dst, src))
+    want_off = np.zeros(n + 1, np.uint64)
+    np.cumsum(np.bincount(src, minlength=n), out=want_off[1:])
+    off, adj = g.csr()
+    assert np.array_equal(off, want_off)
+    assert np.array_equal(adj.astype(np.int64), dst[order])
+
+
 @pytest.mark.parametrize("n", range(1, 11))
 def test_complete_graph(oracle_mod, n):
     g = G(oracle_mod, gg.complete(n))
