@@ -3,10 +3,14 @@
 
 Default workload (N=1): configs[1], k-clique counting k = 4, 5, 6 on the
 cit-Patents-shaped R-MAT (scale 22, a,b,c = 0.53,0.20,0.20, 16.6M raw samples,
-seed 1).  One step = the whole hot path on one synthetic batch: A1 CSR + DAG build
-from the raw edge samples resident in HBM, then the k-clique counts for every k
-(A2-A8) from one gamma_kclique_multi pass (--per-k: one gamma_kclique per k).  value = matched embeddings (sum of the k-clique counts) / device time
-of the step (CUDA events, max over ranks), L2 flushed (256 MiB write) between steps.
+seed 1).  One step = the hot path from "CSR resident" to "global result on host" (SURVEY.md
+§8(d)): the k-clique counts for every k (A2-A8) from one gamma_kclique_multi pass
+(--per-k: one gamma_kclique per k).  Before each step the A1 CSR + DAG build runs
+from the raw edge samples resident in HBM (untimed, reported as build_ms_per_step;
+a fresh graph per step, so no per-graph cache outlives a step), then L2 is flushed
+(256 MiB write).  value = matched embeddings (sum of the k-clique counts) / device
+time of the steps (CUDA events, max over ranks).  e2e = the whole step through the
+public API from pinned host buffers: H2D of the raw samples + build + hot path.
 
 Other workloads (not the default line): c1 (configs[0]), heavy (kCL scaling
 workload), c3 (labeled SM, 4 queries x 2 labelings), c4 (FPM, l=3, MNI).
@@ -159,6 +163,30 @@ def load_traffic(workload: str, kernel_class: str):
         except (OSError, ValueError):
             pass
     return None, None
+
+
+def issue_roofline(workload: str, kernel_class: str, ms_per_launch: float, clk: dict):
+    """The ceiling that binds an L2-resident, integer path: instruction issue.  Warp
+    instructions per launch (committed ncu --set full summary of this workload's
+    dominant class, profiles/ncu_<workload>_<class>.json: smsp__inst_executed.sum over
+    the class's launches of one step, averaged) / (148 SMs x 4 schedulers x SM clock x
+    the live event-timed ms per launch).  1.0 = every scheduler issues every cycle."""
+    p = os.path.join(ROOT, "profiles", f"ncu_{workload}_{kernel_class}.json")
+    if not os.path.exists(p):
+        return None
+    try:
+        j = json.load(open(p))
+    except (OSError, ValueError):
+        return None
+    inst = j.get("inst_executed_per_launch")
+    if not inst:
+        return None
+    mhz = (clk or {}).get("sm_mhz") or (clk or {}).get("sm_max_mhz") or 1965.0
+    peak = 148 * 4 * mhz * 1e6                     # warp instructions / s
+    achieved = inst / (ms_per_launch / 1000.0)
+    return {"bound": "issue", "achieved": achieved, "peak": peak, "unit": "warp-inst/s", "frac": achieved / peak,
+            "inst_per_launch": inst, "sm_mhz": mhz, "threads_per_inst": j.get("threads_per_warp_inst"),
+            "source": os.path.relpath(p, ROOT)}
 
 
 def load_alg_bytes(workload: str):
@@ -336,10 +364,16 @@ def run_gamma(args):
         agg["_total_launches"]["n"] += st["total_launches"]
         return st
 
-    def step(src, dst, labels, coll):
-        g = ctx.load_edges(n, src, dst, labels)
+    def build(src, dst, labels, coll):
+        g = ctx.load_edges(n, src, dst, labels)   # A1 (reported as t_build)
         if coll:
             collect()
+        return g
+
+    def work(g, coll):
+        """One step of the hot path from "CSR resident" to "global result on host"
+        (SURVEY §8(d)): A2 root selection / partition, every extension level, the
+        aggregate and (N > 1) the collectives."""
         results = {}
         if w["kind"] == "kcl":
             if args.per_k:
@@ -366,19 +400,28 @@ def run_gamma(args):
             st = collect() if coll else ctx.stats()
             results = {f"frequent_l{l}": sum(1 for p in pats if p[0] == l) for l in range(1, w["l"] + 1)}
             emb = st["level_entries"][w["l"]]
+            results["embeddings_per_level"] = st["level_entries"][1:w["l"] + 1]
             results["embeddings_l"] = emb
             results["domain_chunk_passes"] = st.get("chunks")
             results["table_retries"] = st.get("retries")
-        info = g.info()
-        g.free()
-        return emb, results, info
+        return emb, results
 
     def barrier():
         if world > 1:
             dist.barrier()
 
+    def fresh_graph(coll):
+        """The graph of the next step: built from the raw samples in HBM (untimed, a
+        fresh handle so no per-graph cache such as the root order outlives a step), then
+        L2 flushed so the timed step starts cold."""
+        g = build(src_dev, dst_dev, lab_dev, coll)
+        flush.fill_(1)
+        return g
+
     for _ in range(args.warmup):
-        step(src_dev, dst_dev, lab_dev, False)
+        g = fresh_graph(False)
+        work(g, False)
+        g.free()
     torch.cuda.synchronize()
     if os.environ.get("GAMMA_BENCH_GC", "1") == "0":   # diagnostics: no cyclic GC in the timed region
         import gc
@@ -389,25 +432,29 @@ def run_gamma(args):
     clocks = ClockSampler(dev)
     if not args.no_clocks:
         clocks.start()
-    times, emb, results, info = [], 0, None, None
+    times, builds, emb, results, info = [], [], 0, None, None
     for _ in range(args.steps):
-        flush.fill_(1)
+        g = fresh_graph(True)
+        info = g.info()
+        builds.append(info["build_ms"])
         barrier()
         torch.cuda.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
-        emb, results, info = step(src_dev, dst_dev, lab_dev, True)
+        emb, results = work(g, True)
         e1.record(stream)
         torch.cuda.synchronize()
         barrier()
         times.append(e0.elapsed_time(e1))
+        g.free()
     clk = clocks.stop()
     total_ms = max_over_ranks(sum(times), world)
     # load imbalance of the root partition = max / mean of the ranks' times
     imbalance = total_ms / (max_over_ranks(sum(times), world, "sum") / world) if world > 1 else 1.0
     value = emb * args.steps / (total_ms / 1000.0)
 
-    # ---- e2e: the same step through the public API from pinned host buffers ----
+    # ---- e2e: the whole step through the public API from pinned host buffers: H2D of
+    # the raw samples, A1 build, the hot path, results D2H ----
     e2e_times = []
     for _ in range(max(1, min(args.steps, 3))):
         flush.fill_(1)
@@ -415,11 +462,13 @@ def run_gamma(args):
         torch.cuda.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
-        step(src_pin, dst_pin, lab_pin, False)   # H2D inside gamma_load_edges; results D2H per call
+        g = build(src_pin, dst_pin, lab_pin, False)   # H2D inside gamma_load_edges
+        work(g, False)                                  # results D2H per call
         e1.record(stream)
         torch.cuda.synchronize()
         barrier()
         e2e_times.append(e0.elapsed_time(e1))
+        g.free()
     e2e_value = emb * len(e2e_times) / (max_over_ranks(sum(e2e_times), world) / 1000.0)
 
     if rank != 0:
@@ -452,7 +501,8 @@ def run_gamma(args):
                 "alg_bytes_per_launch": per_launch_bytes, "alg_bytes_source": bytes_src,
                 "kernel_counted_bytes_per_launch": kernel_bytes,
                 "ms_per_launch": per_launch_ms, "launches_per_step": launches / args.steps,
-                "share_of_step": cand[dom]["ms"] / total_ms, "traffic_source": traffic_src}
+                "share_of_step": cand[dom]["ms"] / total_ms, "traffic_source": traffic_src,
+                "issue": issue_roofline(args.workload, dom, per_launch_ms, clk)}
     cpu = None
     if w.get("device_gen"):
         cpu = {"value": None, "unit": UNIT, "cores": os.cpu_count(), "kind": "oracle",
@@ -482,7 +532,10 @@ def run_gamma(args):
         "gpu_launches": int(agg["_total_launches"]["n"]),
         "clocks": clk,
         "kernels": {k: v for k, v in agg.items() if not k.startswith("_") and v["launches"]},
-        "build_ms_per_step": info["build_ms"],
+        "build_ms_per_step": statistics.median(builds),
+        "timed_region": "CSR resident -> global result on host (SURVEY §8(d)); the A1 build from the raw "
+                        "samples in HBM runs before each step, untimed (build_ms_per_step), then L2 is flushed; "
+                        "e2e includes H2D + build",
         "step_ms": [round(x, 3) for x in times],
         "rank_time_max_over_mean": imbalance,
         "e2e_step_ms": [round(x, 3) for x in e2e_times],

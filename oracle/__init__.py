@@ -55,6 +55,9 @@ def lib():
             L.og_match_roots.restype = C.c_int
             L.og_match_roots.argtypes = [C.c_void_p, C.c_uint32, C.c_uint32, u32p, C.c_void_p, C.c_int, C.c_uint64,
                                          u32p, u64p, C.c_int]
+            L.og_match_levels.restype = C.c_int
+            L.og_match_levels.argtypes = [C.c_void_p, C.c_uint32, C.c_uint32, u32p, C.c_void_p, u32p, u32p, u32p,
+                                          C.c_int, u64p, u64p, u64p]
             L.og_fpm.restype = C.c_int64
             L.og_fpm.argtypes = [C.c_void_p, C.c_uint32, C.c_uint64, C.c_int, C.c_int, C.c_uint64,
                                  u64p, C.c_uint64]
@@ -140,6 +143,24 @@ class Graph:
             raise ValueError(f"oracle og_match_roots status {st}")
         return out
 
+    def match_levels(self, nv: int, edges, plabels=None, plan=None, threads: int = 0):
+        """Per-level SM statistics (O-2b) in the matching order and with the order
+        constraints of ``plan`` (default: this oracle's own R10/R16 planner,
+        plan_r10_r16): (N, G, C) lists indexed by the number t of placed positions,
+        N[nv] = the match count.  Feeds SURVEY §8(d)'s algorithmic bytes of SM."""
+        order, lt, gt = plan if plan is not None else plan_r10_r16(nv, edges, plabels)
+        e = np.ascontiguousarray(np.asarray(edges, dtype=np.uint32).reshape(-1))
+        pl = None if plabels is None else np.ascontiguousarray(plabels, dtype=np.uint32)
+        N = np.zeros(nv + 1, np.uint64)
+        G = np.zeros(nv + 1, np.uint64)
+        Cc = np.zeros(nv + 1, np.uint64)
+        st = lib().og_match_levels(self._h, nv, e.size // 2, e, None if pl is None else pl.ctypes.data,
+                                   np.asarray(order, np.uint32), np.asarray(lt, np.uint32),
+                                   np.asarray(gt, np.uint32), threads, N, G, Cc)
+        if st != 0:
+            raise ValueError(f"oracle og_match_levels status {st}")
+        return [int(x) for x in N], [int(x) for x in G], [int(x) for x in Cc]
+
     def fpm(self, l: int, minsup: int, method: str = "shapes", threads: int = 0,
             pattern_cap: int = 1 << 16):
         """Frequent patterns as a sorted list of (ne, nv, labels, edges, support, instances).
@@ -173,3 +194,53 @@ class Graph:
         if st != 0:
             raise ValueError(f"oracle og_pattern_mni status {st}")
         return int(s.value)
+
+
+def automorphisms(nv: int, edges, plabels=None):
+    """Aut_L(P): every label- and edge-preserving permutation (brute force over nv!)."""
+    import itertools
+    E = {frozenset(e) for e in edges}
+    lab = list(plabels) if plabels is not None else [0] * nv
+    return [p for p in itertools.permutations(range(nv))
+            if all(lab[p[i]] == lab[i] for i in range(nv)) and {frozenset((p[a], p[b])) for a, b in edges} == E]
+
+
+def plan_r10_r16(nv: int, edges, plabels=None):
+    """The oracle's own statement of the method's matching order and symmetry breaking
+    (readings R10, R16; PAPER.md L176 leaves the order open):
+      order: the max-degree pattern vertex first (ties: lower id), then repeatedly the
+             unplaced vertex with the most placed neighbours (ties: higher degree, then
+             lower id), among those with at least one placed neighbour;
+      constraints: stabilizer chain of Aut_L(P) along the order -- for the vertex v at
+             position t, every other u in v's orbit under the automorphisms fixing the
+             vertices of positions < t must satisfy phi(v) < phi(u).
+    Returns (order, lt, gt): lt[t] / gt[t] = bitmask of earlier positions j with
+    phi(j) < phi(t) / phi(t) < phi(j)."""
+    deg = [0] * nv
+    adj = [set() for _ in range(nv)]
+    for a, b in edges:
+        adj[a].add(b)
+        adj[b].add(a)
+    for v in range(nv):
+        deg[v] = len(adj[v])
+    order = [max(range(nv), key=lambda v: (deg[v], -v))]
+    while len(order) < nv:
+        placed = set(order)
+        cand = [v for v in range(nv) if v not in placed and adj[v] & placed]
+        order.append(max(cand, key=lambda v: (len(adj[v] & placed), deg[v], -v)))
+    pos = {v: t for t, v in enumerate(order)}
+    auts = automorphisms(nv, edges, plabels)
+    lt, gt = [0] * nv, [0] * nv
+    fixed = []
+    group = auts
+    for t, v in enumerate(order):
+        group = [p for p in group if all(p[x] == x for x in fixed)]
+        orbit = {p[v] for p in group}
+        for u in orbit - {v}:
+            # phi(v) < phi(u): recorded at the later of the two positions
+            if pos[u] > t:
+                lt[pos[u]] |= 1 << t
+            else:
+                gt[t] |= 1 << pos[u]
+        fixed.append(v)
+    return order, lt, gt

@@ -485,6 +485,115 @@ int og_match_roots(const og_graph *g, uint32_t nv, uint32_t ne, const uint32_t *
 }
 
 /* ---------------------------------------------------------------------------
+ * O-2b: per-level statistics of SM in a GIVEN matching order with GIVEN order
+ * constraints (SURVEY.md §8(d) algorithmic bytes of the SM path; the order and the
+ * constraints are the method's choices -- DESIGN.md readings R10 and R16 -- computed
+ * by this oracle's own planner, oracle/__init__.py plan_r10_r16).  Position t holds
+ * pattern vertex order[t]; a partial match of t positions is an injective map of
+ * order[0..t-1] that respects labels, the pattern edges among them, the constraints
+ * phi(t) > phi(j) for j in lt[t] and phi(t) < phi(j) for j in gt[t], and (positions
+ * t < nv-1 only: a pruning that never removes a full match) deg(phi(t)) >=
+ * deg_P(order[t]) ("pruning ... at run-time").
+ *   N[t]  = number of partial matches with t positions (N[nv] = the match count);
+ *   G[t]  = sum over partial matches with t-1 positions of the degrees of the images
+ *           of the backward neighbours of position t that lie in positions < t-1
+ *           (Opt 2: the group's prefix lists, fetched once per group);
+ *   C[t]  = sum over partial matches with t positions of deg(phi(t-1)) if position
+ *           t-1 is a backward neighbour of position t (each child's own list).
+ * Step t -> t+1 of the ET then reads 12 N[t] + 4 (G[t] + C[t]) + 8 N[t+1] [t+1 < nv]
+ * bytes.  Candidates are enumerated by a check-based scan of N(phi(first backward
+ * neighbour)), as in og_match.
+ * ------------------------------------------------------------------------- */
+typedef struct {
+  uint32_t nv, order[OG_MAXV], lab[OG_MAXV], pdeg[OG_MAXV], labeled;
+  uint32_t back[OG_MAXV], lt[OG_MAXV], gt[OG_MAXV];   /* position bitmasks */
+} og_lplan;
+
+static uint64_t gdegree(const og_graph *g, uint32_t v) { return g->off[v + 1] - g->off[v]; }
+
+static void levels_rec(const og_graph *g, const og_lplan *P, uint32_t t, uint32_t *phi, uint64_t *N, uint64_t *G,
+                       uint64_t *C) {
+  /* a partial match of t positions */
+  N[t] += 1;
+  if (t >= 1 && t < P->nv && ((P->back[t] >> (t - 1)) & 1u)) C[t] += gdegree(g, phi[t - 1]);
+  if (t + 1 < P->nv) {   /* as the group (prefix) of the children at position t */
+    uint32_t m = P->back[t + 1] & ((1u << t) - 1u);
+    for (uint32_t j = 0; j < t; j++) if ((m >> j) & 1u) G[t + 1] += gdegree(g, phi[j]);
+  }
+  if (t == P->nv) return;
+  uint32_t b0 = (uint32_t)__builtin_ctz(P->back[t]);   /* first backward neighbour */
+  uint32_t base = phi[b0];
+  for (uint64_t e = g->off[base]; e < g->off[base + 1]; e++) {
+    uint32_t x = g->adj[e];
+    if (P->labeled && g->lab[x] != P->lab[t]) continue;
+    if (t + 1 < P->nv && gdegree(g, x) < P->pdeg[t]) continue;
+    int ok = 1;
+    for (uint32_t j = 0; j < t && ok; j++) {
+      if (phi[j] == x) ok = 0;
+      else if (((P->lt[t] >> j) & 1u) && !(x > phi[j])) ok = 0;
+      else if (((P->gt[t] >> j) & 1u) && !(x < phi[j])) ok = 0;
+      else if (j != b0 && ((P->back[t] >> j) & 1u) && !adjacent(g, phi[j], x)) ok = 0;
+    }
+    if (!ok) continue;
+    phi[t] = x;
+    levels_rec(g, P, t + 1, phi, N, G, C);
+  }
+}
+
+int og_match_levels(const og_graph *g, uint32_t nv, uint32_t ne, const uint32_t *edges, const uint32_t *plabels,
+                    const uint32_t *order, const uint32_t *lt, const uint32_t *gt, int threads, uint64_t *N,
+                    uint64_t *G, uint64_t *C) {
+  if (nv < 1 || nv > OG_MAXV) return OG_EINVAL;
+  og_lplan P;
+  memset(&P, 0, sizeof(P));
+  P.nv = nv;
+  P.labeled = plabels != NULL;
+  uint32_t adjm[OG_MAXV][OG_MAXV];
+  memset(adjm, 0, sizeof(adjm));
+  for (uint32_t e = 0; e < ne; e++) {
+    uint32_t a = edges[2 * e], b = edges[2 * e + 1];
+    if (a >= nv || b >= nv || a == b) return OG_EINVAL;
+    adjm[a][b] = adjm[b][a] = 1;
+  }
+  uint32_t pos_of[OG_MAXV], seen = 0;
+  for (uint32_t t = 0; t < nv; t++) {
+    if (order[t] >= nv || ((seen >> order[t]) & 1u)) return OG_EINVAL;
+    seen |= 1u << order[t];
+    pos_of[order[t]] = t;
+  }
+  for (uint32_t t = 0; t < nv; t++) {
+    uint32_t v = order[t];
+    P.order[t] = v;
+    P.lab[t] = plabels ? plabels[v] : 0;
+    P.lt[t] = lt[t] & ((1u << t) - 1u);
+    P.gt[t] = gt[t] & ((1u << t) - 1u);
+    for (uint32_t u = 0; u < nv; u++) {
+      if (!adjm[v][u]) continue;
+      P.pdeg[t]++;
+      if (pos_of[u] < t) P.back[t] |= 1u << pos_of[u];
+    }
+    if (t > 0 && P.back[t] == 0) return OG_EINVAL;   /* the order must stay connected */
+  }
+  for (uint32_t t = 0; t <= nv; t++) N[t] = G[t] = C[t] = 0;
+  set_threads(threads);
+#pragma omp parallel
+  {
+    uint64_t n_loc[OG_MAXV + 1] = {0}, g_loc[OG_MAXV + 1] = {0}, c_loc[OG_MAXV + 1] = {0};
+#pragma omp for schedule(dynamic, 64)
+    for (int64_t v = 0; v < (int64_t)g->n; v++) {
+      if (P.labeled && g->lab[v] != P.lab[0]) continue;
+      if (nv > 1 && gdegree(g, (uint32_t)v) < P.pdeg[0]) continue;
+      uint32_t phi[OG_MAXV];
+      phi[0] = (uint32_t)v;
+      levels_rec(g, &P, 1, phi, n_loc, g_loc, c_loc);
+    }
+#pragma omp critical
+    for (uint32_t t = 0; t <= nv; t++) { N[t] += n_loc[t]; G[t] += g_loc[t]; C[t] += c_loc[t]; }
+  }
+  return OG_OK;
+}
+
+/* ---------------------------------------------------------------------------
  * O-3: frequent pattern mining, edge-induced patterns of 1..l edges (l <= 3),
  * MNI support.
  *

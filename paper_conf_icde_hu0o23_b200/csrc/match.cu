@@ -85,7 +85,11 @@ struct SmArgs {
   uint32_t *desc_out;
   uint32_t dw_out;
   uint64_t cap_v, cap_g;
-  unsigned long long *ctrl;
+  unsigned long long *ctrl;  // this launch's control block (CTRL_* offsets)
+  unsigned long long *ovf;   // overflow word (shared by a launch chain: any level's overflow
+                             // stops every later level)
+  const unsigned long long *gcur_in;   // nullable: groups in = min(*gcur_in, cap_g_in) - g_begin,
+  uint64_t cap_g_in;                   // read on the device (chained launch), instead of g_end
   uint32_t batch;
   uint32_t stage;           // 0: never stage L_m (debug)
   uint32_t *lm_scratch;     // per-warp global L_m slices for hub prefixes (nullable)
@@ -221,12 +225,18 @@ __global__ void __launch_bounds__(kThreads, 5) sm_kernel(SmArgs a) {
   uint32_t *sout = slm + a.lm_cap;
   const uint32_t d = a.d, q = d + 1;
   const bool last = q == a.P.nv - 1;
-  const BlockPool pv{&a.ctrl[CTRL_VCUR], &a.ctrl[CTRL_OVF], a.cap_v, kBlkV};
-  const BlockPool pg{&a.ctrl[CTRL_GCUR], &a.ctrl[CTRL_OVF], a.cap_g, kBlkG};
+  const BlockPool pv{&a.ctrl[CTRL_VCUR], a.ovf, a.cap_v, kBlkV};
+  const BlockPool pg{&a.ctrl[CTRL_GCUR], a.ovf, a.cap_g, kBlkG};
   WarpBlock wv, wg;
   uint64_t acc = 0, in_entries = 0, out_entries = 0;
   uint64_t elems = 0;   // adjacency elements the method fetches (SURVEY §8(d) B_l), lane-partial
-  const uint64_t ng = a.g_end - a.g_begin;
+  uint64_t g_end = a.g_end;
+  if (a.gcur_in) {   // chained launch: the previous level's group cursor, read here
+    if (*(volatile unsigned long long *)a.ovf) return;   // an earlier level overflowed
+    const uint64_t gc = *(volatile const unsigned long long *)a.gcur_in;
+    g_end = gc < a.cap_g_in ? gc : a.cap_g_in;
+  }
+  const uint64_t ng = g_end > a.g_begin ? g_end - a.g_begin : 0;
   bool stop = false;
   const uint32_t prefix_mask = (1u << d) - 1u;
   const uint32_t bq = a.P.bmask[q];
@@ -239,7 +249,7 @@ __global__ void __launch_bounds__(kThreads, 5) sm_kernel(SmArgs a) {
     if (lane == 0) base = atomicAdd(&a.ctrl[CTRL_WORK], (unsigned long long)a.batch);
     base = __shfl_sync(0xffffffffu, base, 0);
     if (base >= ng) break;
-    if (!last && *(volatile unsigned long long *)&a.ctrl[CTRL_OVF]) break;
+    if (!last && *(volatile unsigned long long *)a.ovf) break;
     const uint64_t bend = min((uint64_t)base + a.batch, ng);
     for (uint64_t gi = a.g_begin + base; gi < a.g_begin + bend && !stop; gi++) {
       const uint32_t *dsc = a.desc_in + gi * a.dw_in;
@@ -759,6 +769,8 @@ struct SmRun {
     a.g_begin = g0;
     a.g_end = g1;
     a.ctrl = (unsigned long long *)ctx->ctrl;
+    a.ovf = a.ctrl + CTRL_OVF;
+    a.gcur_in = nullptr;
     a.batch = d == 0 ? 1 : sm_batch();
     a.stage = stage;
     a.lm_scratch = lm_scratch.p;
@@ -770,12 +782,17 @@ struct SmRun {
     return a;
   }
 
-  void run_kernel(const SmArgs &a, bool last, uint64_t cap_v) {
+  int grid_for(bool last, uint64_t cap_v) const {
     int gr = grid;
     if (!last) {
       const uint64_t warps_ok = std::max<uint64_t>(1, cap_v / (2ull * kBlkV));
       gr = (int)std::max<uint64_t>(1, std::min<uint64_t>(gr, warps_ok / kWarps));
     }
+    return gr;
+  }
+
+  void run_kernel(const SmArgs &a, bool last, uint64_t cap_v) {
+    const int gr = grid_for(last, cap_v);
     ctrl_reset(ctx);
     const int kc = last ? KC_SM_COUNT : KC_SM_EXTEND;
     ctx->launch(kc, [&] { sm_kernel<<<gr, kThreads, sm_smem(), ctx->stream>>>(a); });
@@ -785,6 +802,66 @@ struct SmRun {
       ctx->stats.list_elems += h[CTRL_ELEMS];
       ctx->stats.alg_bytes[kc] += 12 * h[CTRL_AUX0] + 4 * h[CTRL_ELEMS] + (last ? 0 : 8 * h[CTRL_ENTRIES]);
     }
+  }
+
+  // The whole level chain of a query enqueued back to back with one read-back at the
+  // end: level d's launch reads its group count from level d-1's cursor on the device
+  // (SmArgs::gcur_in), each level has its own control block (CTRL_LEVELS), and one
+  // shared overflow word makes every later level exit at once.  Returns false (nothing
+  // recorded) when some level overflowed its table; the caller then runs the careful
+  // per-level path (process), which grows tables and halves group ranges.
+  bool chain(uint64_t ngroups) {
+    const uint32_t nl = P.nv - 1;   // launches: d = 0 .. nv-2
+    for (uint32_t q = 1; q < nl; q++)
+      if (lv[q].cap_v == 0) grow(q, std::max<uint64_t>(1ull << 24, 4ull * kBlkV * kWarps * (uint64_t)grid));
+    unsigned long long *ctrl = (unsigned long long *)ctx->ctrl;
+    ctrl_reset(ctx);
+    for (uint32_t d = 0; d < nl; d++) {
+      const uint32_t q = d + 1;
+      const bool last = q == P.nv - 1;
+      SmArgs a = args(d, 0, ngroups);
+      a.ctrl = ctrl + CTRL_LEVELS + CTRL_LSTRIDE * d;
+      a.ovf = ctrl + CTRL_OVF;
+      if (d > 0) {
+        a.gcur_in = ctrl + CTRL_LEVELS + CTRL_LSTRIDE * (d - 1) + CTRL_GCUR;
+        a.cap_g_in = lv[d].cap_g;
+      }
+      if (!last) {
+        a.vid_out = lv[q].vid.p;
+        a.desc_out = lv[q].desc.p;
+        a.dw_out = 2 + q;
+        a.cap_v = lv[q].cap_v;
+        a.cap_g = lv[q].cap_g;
+      }
+      const int gr = grid_for(last, last ? 0 : lv[q].cap_v);
+      const int kc = last ? KC_SM_COUNT : KC_SM_EXTEND;
+      ctx->launch(kc, [&] { sm_kernel<<<gr, kThreads, sm_smem(), ctx->stream>>>(a); });
+    }
+    ctrl_fetch(ctx);
+    const uint64_t *h = ctx->ctrl_host;
+    if (h[CTRL_OVF]) {
+      // hint for the careful path: grow the tables that ran out
+      for (uint32_t d = 0; d + 1 < nl; d++) {
+        const uint64_t *b = h + CTRL_LEVELS + CTRL_LSTRIDE * d;
+        if (b[CTRL_VCUR] > lv[d + 1].cap_v) grow(d + 1, b[CTRL_VCUR]);
+      }
+      return false;
+    }
+    for (uint32_t d = 0; d < nl; d++) {
+      const uint64_t *b = h + CTRL_LEVELS + CTRL_LSTRIDE * d;
+      const bool last = d + 2 == P.nv;
+      const int kc = last ? KC_SM_COUNT : KC_SM_EXTEND;
+      ctx->stats.list_elems += b[CTRL_ELEMS];
+      ctx->stats.alg_bytes[kc] += 12 * b[CTRL_AUX0] + 4 * b[CTRL_ELEMS] + (last ? 0 : 8 * b[CTRL_ENTRIES]);
+      if (last) {
+        total = checked_add(total, b[CTRL_COUNT]);
+        ctx->stats.level_entries[P.nv] = checked_add(ctx->stats.level_entries[P.nv], b[CTRL_COUNT]);
+      } else {
+        ctx->stats.level_entries[d + 2] += b[CTRL_ENTRIES];
+        ctx->stats.chunks++;
+      }
+    }
+    return true;
   }
 
   void process(uint32_t d, uint64_t g0, uint64_t g1) {
@@ -926,7 +1003,14 @@ static uint64_t match_count(gamma_graph *g, const SmPlan &P) {
     R.lm_scratch_cap = std::min<uint32_t>(g->max_degree, 1u << 16);
     R.lm_scratch = DevBuf<uint32_t>(ctx, (uint64_t)R.grid * kWarps * R.lm_scratch_cap, true);
   }
-  R.process(0, 0, ngr);
+  // fast path: the whole level chain with one read-back; on a table overflow, the
+  // careful per-level path (DFS over group ranges with table growth and halving)
+  const bool fast = (ctx->desc.flags & GAMMA_FLAG_SPILL) == 0 && P.nv >= 2 && P.nv - 1 <= 12 &&
+                    getenv("GAMMA_SM_NO_CHAIN") == nullptr;
+  if (!fast || !R.chain(ngr)) {
+    if (fast) ctx->stats.retries++;
+    R.process(0, 0, ngr);
+  }
   ctx->sync();
   ctx->collect_timings();
   return R.total;

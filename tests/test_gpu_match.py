@@ -286,3 +286,19 @@ def test_last_level_long_child_probe(oracle_mod, ratio):
         nv, e = Q[q]
         assert got[q + "/0"] == o0.match(nv, e)[0], (ratio, q, "unlabeled")
         assert got[q + "/m"] == o.match(nv, e, [i % 8 for i in range(nv)])[0], (ratio, q, "imod8")
+
+
+@pytest.mark.parametrize("q", ["c4", "diamond", "tailed_triangle", "house"])
+def test_level_sizes_vs_oracle(ctx, oracle_mod, q):
+    """Every ET level the GPU builds, not only the final count: the number of partial
+    matches at each depth (stats level_entries) equals the oracle's O-2b level counts in
+    the same matching order and constraints (oracle planner plan_r10_r16, pinned in
+    tests/test_oracle_match_levels.py)."""
+    nv, e = Q[q]
+    n, s, d, lab = gg.config_graph("c3", seed=3, scale=12)
+    g = ctx.load_edges(n, s, d, lab)
+    o = oracle_mod.Graph(n, s, d, lab)
+    for plab in ([0] * nv, [i % 8 for i in range(nv)], [i % 2 for i in range(nv)]):
+        N, _, _ = o.match_levels(nv, e, plab)
+        assert g.match(nv, e, plab)[0] == N[nv]
+        assert ctx.stats()["level_entries"][1:nv + 1] == N[1:], plab
