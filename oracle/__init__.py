@@ -19,7 +19,7 @@ _LIB = os.path.join(_HERE, "liboracle.so")
 _lock = threading.Lock()
 _lib = None
 
-REC = 14  # uint64 words per FPM result record (see oracle.c)
+REC = 17  # uint64 words per FPM result record (see oracle.c)
 
 
 def build(force: bool = False) -> str:
@@ -181,8 +181,8 @@ class Graph:
             r = out[i * REC:(i + 1) * REC]
             ne, nv = int(r[0]), int(r[1])
             res.append((ne, nv, tuple(int(x) for x in r[2:2 + nv]),
-                        tuple((int(r[6 + 2 * e]), int(r[7 + 2 * e])) for e in range(ne)), int(r[12]),
-                        int(r[13])))
+                        tuple((int(r[7 + 2 * e]), int(r[8 + 2 * e])) for e in range(ne)), int(r[15]),
+                        int(r[16])))
         return res
 
     def pattern_mni(self, nv: int, edges, plabels=None, threads: int = 0) -> int:

@@ -594,18 +594,19 @@ int og_match_levels(const og_graph *g, uint32_t nv, uint32_t ne, const uint32_t 
 }
 
 /* ---------------------------------------------------------------------------
- * O-3: frequent pattern mining, edge-induced patterns of 1..l edges (l <= 3),
+ * O-3: frequent pattern mining, edge-induced patterns of 1..l edges (l <= 4),
  * MNI support.
  *
- * Canonical code of a connected edge set S with vertex set W (|W| = nv <= 4):
+ * Canonical code of a connected edge set S with vertex set W (|W| = nv <= 5):
  *   min over bijections pi : {0..nv-1} -> W  of
  *     ( lab(pi(0)), ..., lab(pi(nv-1)),  sorted list of pairs (i<j) with {pi(i),pi(j)} in S )
  *   compared lexicographically (labels first, then the sorted edge-pair list).
  * Domain of canonical position i: union over every minimizing pi of {pi(i)}.
  * sup(P) = min_i |domain(P, i)|  (MNI).  Output: every P with sup >= minsup.
  * ------------------------------------------------------------------------- */
-#define FPM_MAXNV 4
-#define FPM_MAXE 3
+#define FPM_MAXNV 5
+#define FPM_MAXE 4
+#define FPM_NPERM 120   /* 5! */
 
 typedef struct {
   uint32_t nv, ne;
@@ -669,18 +670,39 @@ static int64_t ptab_get(og_ptab *t, const og_code *c) {
 
 /* Canonicalise the edge set {ed[0..ne-1]} on vertex set W (nv vertices) and
  * OR every minimizing assignment into the pattern's domains. */
+/* All 120 orders of 5 symbols, lexicographic (filled once). */
+static uint8_t g_perms5[FPM_NPERM][FPM_MAXNV];
+static int g_perms5_ready = 0;
+static void perms5_init(void) {
+  if (__atomic_load_n(&g_perms5_ready, __ATOMIC_ACQUIRE)) return;
+#pragma omp critical(og_perms5)
+  if (!g_perms5_ready) {
+    uint8_t p[FPM_MAXNV] = {0, 1, 2, 3, 4};
+    for (int r = 0; r < FPM_NPERM; r++) {
+      memcpy(g_perms5[r], p, FPM_MAXNV);
+      /* next permutation */
+      int i = FPM_MAXNV - 2;
+      while (i >= 0 && p[i] > p[i + 1]) i--;
+      if (i < 0) break;
+      int j = FPM_MAXNV - 1;
+      while (p[j] < p[i]) j--;
+      uint8_t x = p[i]; p[i] = p[j]; p[j] = x;
+      for (int a = i + 1, b = FPM_MAXNV - 1; a < b; a++, b--) { x = p[a]; p[a] = p[b]; p[b] = x; }
+    }
+    __atomic_store_n(&g_perms5_ready, 1, __ATOMIC_RELEASE);
+  }
+}
+
 static void fpm_record(const og_graph *g, og_ptab *t, uint32_t nv, const uint32_t *W, uint32_t ne,
                        const uint32_t (*ed)[2]) {
-  static const uint8_t perms4[24][4] = {
-      {0,1,2,3},{0,1,3,2},{0,2,1,3},{0,2,3,1},{0,3,1,2},{0,3,2,1},{1,0,2,3},{1,0,3,2},
-      {1,2,0,3},{1,2,3,0},{1,3,0,2},{1,3,2,0},{2,0,1,3},{2,0,3,1},{2,1,0,3},{2,1,3,0},
-      {2,3,0,1},{2,3,1,0},{3,0,1,2},{3,0,2,1},{3,1,0,2},{3,1,2,0},{3,2,0,1},{3,2,1,0}};
+  perms5_init();
   og_code best; int have = 0;
-  uint32_t bestpi[24][FPM_MAXNV]; int nbest = 0;
-  for (int pi = 0; pi < 24; pi++) {
-    const uint8_t *P = perms4[pi];
-    int valid = 1;   /* permutation of the first nv symbols only */
+  uint32_t bestpi[FPM_NPERM][FPM_MAXNV]; int nbest = 0;
+  for (int pi = 0; pi < FPM_NPERM; pi++) {
+    const uint8_t *P = g_perms5[pi];
+    int valid = 1;   /* permutation of the first nv symbols only (the rest fixed) */
     for (uint32_t i = 0; i < nv; i++) if (P[i] >= nv) valid = 0;
+    for (uint32_t i = nv; i < FPM_MAXNV; i++) if (P[i] != i) valid = 0;
     if (!valid) continue;
     /* position i holds data vertex W[P[i]] */
     og_code c; memset(&c, 0, sizeof(c));
@@ -692,7 +714,7 @@ static void fpm_record(const og_graph *g, og_ptab *t, uint32_t nv, const uint32_
       for (uint32_t w = 0; w < nv; w++) { if (W[w] == ed[e][0]) a = pos_of[w]; if (W[w] == ed[e][1]) b = pos_of[w]; }
       c.e[e][0] = a < b ? a : b; c.e[e][1] = a < b ? b : a;
     }
-    /* sort the edge pairs (insertion sort, ne <= 3) */
+    /* sort the edge pairs (insertion sort, ne <= 4) */
     for (uint32_t i = 1; i < ne; i++)
       for (uint32_t j = i; j > 0; j--) {
         uint32_t *x = c.e[j - 1], *y = c.e[j];
@@ -724,7 +746,16 @@ static void fpm_record(const og_graph *g, og_ptab *t, uint32_t nv, const uint32_
  *   2 edges:  wedge, centre c with an unordered neighbour pair {a,b}
  *   3 edges:  triangle u<v<w; 3-star, centre c with a neighbour triple a<b<d;
  *             3-path a-b-c-d keyed by its middle edge {b,c} (b<c), a in N(b)-{c},
- *             d in N(c)-{b}, a != d. */
+ *             d in N(c)-{b}, a != d.
+ *   4 edges:  4-star, centre c with a neighbour quadruple;
+ *             4-cycle a-b-c-d-a keyed by its smallest vertex a and a's two cycle
+ *             neighbours b < d, c in N(b) & N(d), c != a (c > a);
+ *             paw (triangle + pendant edge): each triangle u<v<w once, the pendant at
+ *             x in {u,v,w} to y in N(x) outside the triangle;
+ *             4-path a-b-c-d-e keyed by its middle vertex c and its two legs c-b-a,
+ *             c-d-e taken unordered ((b,a) < (d,e)), five distinct vertices;
+ *             fork (spider with legs 2,1,1): centre c of degree 3, long leg c-x-w,
+ *             short legs y < z, all in N(c) (x, y, z distinct), w in N(x) - {c,y,z}. */
 static void fpm_enum_shapes(const og_graph *g, og_ptab *t, uint32_t l) {
 #pragma omp parallel for schedule(dynamic, 64)
   for (int64_t vv = 0; vv < (int64_t)g->n; vv++) {
@@ -775,6 +806,87 @@ static void fpm_enum_shapes(const og_graph *g, og_ptab *t, uint32_t l) {
         }
       }
     }
+    if (l >= 4) {
+      /* 4-star */
+      for (uint64_t i = s; i < e; i++)
+        for (uint64_t j = i + 1; j < e; j++)
+          for (uint64_t q = j + 1; q < e; q++)
+            for (uint64_t r = q + 1; r < e; r++) {
+              uint32_t a = g->adj[i], b = g->adj[j], c = g->adj[q], d = g->adj[r];
+              uint32_t W[5] = {v, a, b, c, d}; uint32_t ed[4][2] = {{v, a}, {v, b}, {v, c}, {v, d}};
+              fpm_record(g, t, 5, W, 4, ed);
+            }
+      /* 4-cycle v-b-c-d-v with v the smallest vertex, b < d */
+      for (uint64_t i = s; i < e; i++) {
+        uint32_t b = g->adj[i];
+        if (b <= v) continue;
+        for (uint64_t j = i + 1; j < e; j++) {
+          uint32_t d = g->adj[j];
+          for (uint64_t x = g->off[b]; x < g->off[b + 1]; x++) {
+            uint32_t c = g->adj[x];
+            if (c <= v || c == d || !adjacent(g, d, c)) continue;
+            uint32_t W[4] = {v, b, c, d}; uint32_t ed[4][2] = {{v, b}, {b, c}, {c, d}, {d, v}};
+            fpm_record(g, t, 4, W, 4, ed);
+          }
+        }
+      }
+      /* paw: triangle v<u<w + pendant */
+      for (uint64_t i = s; i < e; i++) {
+        uint32_t u = g->adj[i];
+        if (u <= v) continue;
+        for (uint64_t j = i + 1; j < e; j++) {
+          uint32_t w = g->adj[j];
+          if (!adjacent(g, u, w)) continue;
+          uint32_t tri[3] = {v, u, w};
+          for (int xi = 0; xi < 3; xi++) {
+            uint32_t x = tri[xi];
+            for (uint64_t y = g->off[x]; y < g->off[x + 1]; y++) {
+              uint32_t z = g->adj[y];
+              if (z == v || z == u || z == w) continue;
+              uint32_t W[4] = {v, u, w, z}; uint32_t ed[4][2] = {{v, u}, {v, w}, {u, w}, {x, z}};
+              fpm_record(g, t, 4, W, 4, ed);
+            }
+          }
+        }
+      }
+      /* 4-path a-b-v-d-c2 with middle vertex v, legs (b,a) < (d,c2) */
+      for (uint64_t i = s; i < e; i++) {
+        uint32_t b = g->adj[i];
+        for (uint64_t j = s; j < e; j++) {
+          uint32_t d = g->adj[j];
+          if (d == b) continue;
+          for (uint64_t x = g->off[b]; x < g->off[b + 1]; x++) {
+            uint32_t a = g->adj[x];
+            if (a == v || a == d) continue;
+            for (uint64_t y = g->off[d]; y < g->off[d + 1]; y++) {
+              uint32_t c2 = g->adj[y];
+              if (c2 == v || c2 == b || c2 == a) continue;
+              if (!(b < d || (b == d && a < c2))) continue;   /* unordered legs, once */
+              uint32_t W[5] = {a, b, v, d, c2}; uint32_t ed[4][2] = {{a, b}, {b, v}, {v, d}, {d, c2}};
+              fpm_record(g, t, 5, W, 4, ed);
+            }
+          }
+        }
+      }
+      /* fork: centre v, long leg v-x-w, short legs y < z */
+      for (uint64_t i = s; i < e; i++) {
+        uint32_t x = g->adj[i];
+        for (uint64_t q = g->off[x]; q < g->off[x + 1]; q++) {
+          uint32_t w = g->adj[q];
+          if (w == v) continue;
+          for (uint64_t j = s; j < e; j++) {
+            uint32_t y = g->adj[j];
+            if (y == x || y == w) continue;
+            for (uint64_t r = j + 1; r < e; r++) {
+              uint32_t z = g->adj[r];
+              if (z == x || z == w) continue;
+              uint32_t W[5] = {v, x, w, y, z}; uint32_t ed[4][2] = {{v, x}, {x, w}, {v, y}, {v, z}};
+              fpm_record(g, t, 5, W, 4, ed);
+            }
+          }
+        }
+      }
+    }
   }
 }
 
@@ -783,7 +895,7 @@ static void fpm_enum_shapes(const og_graph *g, og_ptab *t, uint32_t l) {
  * are ids into the list of undirected edges (u<v) in CSR order. */
 static int edges_connected(uint32_t ne, const uint32_t (*ed)[2]) {
   uint32_t comp[FPM_MAXE]; for (uint32_t i = 0; i < ne; i++) comp[i] = i;
-  for (int it = 0; it < 3; it++)
+  for (int it = 0; it < FPM_MAXE; it++)
     for (uint32_t i = 0; i < ne; i++)
       for (uint32_t j = 0; j < ne; j++)
         if (ed[i][0] == ed[j][0] || ed[i][0] == ed[j][1] || ed[i][1] == ed[j][0] || ed[i][1] == ed[j][1]) {
@@ -799,37 +911,44 @@ static void fpm_enum_brute(const og_graph *g, og_ptab *t, uint32_t l) {
   for (uint32_t v = 0; v < g->n; v++)
     for (uint64_t i = g->off[v]; i < g->off[v + 1]; i++)
       if (g->adj[i] > v) { E[k][0] = v; E[k][1] = g->adj[i]; k++; }
+  /* every set of ne = 1..l distinct edge ids i0 < i1 < ... (lexicographic odometer
+   * over the first edge in parallel) */
 #pragma omp parallel for schedule(dynamic, 1)
   for (int64_t a = 0; a < (int64_t)m; a++) {
-    for (uint64_t b = (uint64_t)a; b < (l >= 2 ? m : (uint64_t)a + 1); b++) {
-      for (uint64_t c = b; c < (l >= 3 ? m : b + 1); c++) {
-        uint64_t ids[3] = {(uint64_t)a, b, c};
-        uint32_t ne = 1 + (b > (uint64_t)a) + (c > b);
-        if ((b == (uint64_t)a && c != b)) continue;   /* only a<b<c or prefixes */
-        uint32_t ed[3][2]; uint32_t q = 0;
-        ed[q][0] = E[ids[0]][0]; ed[q][1] = E[ids[0]][1]; q++;
-        if (b > (uint64_t)a) { ed[q][0] = E[b][0]; ed[q][1] = E[b][1]; q++; }
-        if (c > b) { ed[q][0] = E[c][0]; ed[q][1] = E[c][1]; q++; }
-        if (!edges_connected(ne, (const uint32_t (*)[2])ed)) continue;
-        uint32_t W[4], nv = 0;
-        for (uint32_t e = 0; e < ne; e++)
-          for (int s = 0; s < 2; s++) {
-            uint32_t x = ed[e][s]; int f = 0;
-            for (uint32_t w = 0; w < nv; w++) if (W[w] == x) f = 1;
-            if (!f) W[nv++] = x;
-          }
-        if (nv > FPM_MAXNV) continue;
-        fpm_record(g, t, nv, W, ne, (const uint32_t (*)[2])ed);
+    for (uint32_t ne = 1; ne <= l; ne++) {
+      uint64_t ids[FPM_MAXE];
+      ids[0] = (uint64_t)a;
+      for (uint32_t i = 1; i < ne; i++) ids[i] = ids[i - 1] + 1;
+      if (ne > 1 && ids[ne - 1] >= m) continue;
+      for (;;) {
+        uint32_t ed[FPM_MAXE][2];
+        for (uint32_t i = 0; i < ne; i++) { ed[i][0] = E[ids[i]][0]; ed[i][1] = E[ids[i]][1]; }
+        if (edges_connected(ne, (const uint32_t (*)[2])ed)) {
+          uint32_t W[2 * FPM_MAXE], nv = 0;
+          for (uint32_t e = 0; e < ne; e++)
+            for (int s2 = 0; s2 < 2; s2++) {
+              uint32_t x = ed[e][s2]; int f = 0;
+              for (uint32_t w = 0; w < nv; w++) if (W[w] == x) f = 1;
+              if (!f) W[nv++] = x;
+            }
+          if (nv <= FPM_MAXNV) fpm_record(g, t, nv, W, ne, (const uint32_t (*)[2])ed);
+        }
+        /* next combination with ids[0] fixed */
+        int i = (int)ne - 1;
+        while (i >= 1 && ids[i] == m - ne + (uint64_t)i) i--;
+        if (i < 1) break;
+        ids[i]++;
+        for (uint32_t j = (uint32_t)i + 1; j < ne; j++) ids[j] = ids[j - 1] + 1;
       }
     }
   }
   free(E);
 }
 
-/* Result record layout (uint64 x 14):
- *   [0]=ne [1]=nv [2..5]=labels [6..11]=edge pairs (a0,b0,a1,b1,a2,b2) [12]=support
- *   [13]=number of edge sets (instances) mapped to the pattern. */
-#define OG_REC 14
+/* Result record layout (uint64 x 17):
+ *   [0]=ne [1]=nv [2..6]=labels [7..14]=edge pairs (a0,b0,...,a3,b3) [15]=support
+ *   [16]=number of edge sets (instances) mapped to the pattern. */
+#define OG_REC 17
 
 typedef struct { og_code c; uint64_t sup; uint64_t inst; } og_fres;
 
@@ -877,9 +996,9 @@ int64_t og_fpm(const og_graph *g, uint32_t l, uint64_t minsup, int method, int t
     memset(o, 0, OG_REC * sizeof(uint64_t));
     o[0] = res[i].c.ne; o[1] = res[i].c.nv;
     for (int j = 0; j < FPM_MAXNV; j++) o[2 + j] = j < (int)res[i].c.nv ? res[i].c.lab[j] : 0;
-    for (uint32_t e = 0; e < res[i].c.ne; e++) { o[6 + 2 * e] = res[i].c.e[e][0]; o[7 + 2 * e] = res[i].c.e[e][1]; }
-    o[12] = res[i].sup;
-    o[13] = res[i].inst;
+    for (uint32_t e = 0; e < res[i].c.ne; e++) { o[7 + 2 * e] = res[i].c.e[e][0]; o[8 + 2 * e] = res[i].c.e[e][1]; }
+    o[15] = res[i].sup;
+    o[16] = res[i].inst;
   }
   int ovf = t.overflow;
   free(res); free(t.key); free(t.used); free(t.dom); free(t.inst);

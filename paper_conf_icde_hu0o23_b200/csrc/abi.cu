@@ -355,11 +355,12 @@ gamma_status gamma_kclique(gamma_graph *g, uint32_t k, uint64_t *count) {
 gamma_status gamma_kclique_multi(gamma_graph *g, uint32_t nk, const uint32_t *ks, uint64_t *counts) {
   return guarded([&] {
     GAMMA_REQUIRE(g && (nk == 0 || (ks && counts)), GAMMA_E_INVAL, "gamma_kclique_multi: NULL argument");
-    uint32_t kmax = 0;
+    uint32_t kmax = 0, kmin = 0xffffffffu;
     for (uint32_t i = 0; i < nk; i++) {
       GAMMA_REQUIRE(ks[i] >= 1, GAMMA_E_INVAL, "gamma_kclique_multi: k must be >= 1");
       GAMMA_REQUIRE(ks[i] <= 32, GAMMA_E_UNSUPPORTED, "gamma_kclique_multi: k > 32 unsupported");
       kmax = std::max(kmax, ks[i]);
+      if (ks[i] >= 3) kmin = std::min(kmin, ks[i]);
     }
     gamma_ctx *c = g->ctx;
     GAMMA_CUDA(cudaSetDevice(c->device));
@@ -368,7 +369,7 @@ gamma_status gamma_kclique_multi(gamma_graph *g, uint32_t nk, const uint32_t *ks
     if (nk == 0) return;
     auto t0 = std::chrono::steady_clock::now();
     uint64_t bysize[33] = {};
-    const bool one_pass = kclique_multi(g, kmax, bysize);
+    const bool one_pass = kmax >= 3 && kclique_multi(g, kmin, kmax, bysize);
     std::vector<uint64_t> r(nk);
     for (uint32_t i = 0; i < nk; i++)
       r[i] = (one_pass && ks[i] >= 3) ? bysize[ks[i]] : kclique_count(g, ks[i], nullptr, 0, nullptr);

@@ -248,9 +248,10 @@ constexpr uint32_t kWideMaxRun = 8192;      // global-scratch rows ("wide") up t
 constexpr uint32_t kBitmapMaxK = 12;
 uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint64_t nroots,
                         unsigned long long *per_root, bool sorted, uint64_t n_xl, uint64_t n_long, uint64_t n_mid,
-                        uint64_t *multi_out = nullptr);
-// One bitmap pass counting every clique size 3..kmax (multi_out[s], s <= kmax); false
+                        uint64_t *multi_out = nullptr, uint32_t kmin = 3);
+// One bitmap pass counting every clique size kmin..kmax (multi_out[s], kmin <= s <= kmax;
+// kmin >= 3: roots with d+ < kmin - 1 hold no such clique and are skipped); false
 // when the graph needs the ET path (max out-degree > kWideMaxRun or kmax too big).
-bool kclique_multi(gamma_graph *g, uint32_t kmax, uint64_t *multi_out);
+bool kclique_multi(gamma_graph *g, uint32_t kmin, uint32_t kmax, uint64_t *multi_out);
 void ensure_root_order(gamma_graph *g);
 }  // namespace gamma_impl

@@ -817,20 +817,21 @@ uint64_t kclique_count(gamma_graph *g, uint32_t k, const uint32_t *roots_dev, ui
   return R.total;
 }
 
-bool kclique_multi(gamma_graph *g, uint32_t kmax, uint64_t *multi_out) {
+bool kclique_multi(gamma_graph *g, uint32_t kmin, uint32_t kmax, uint64_t *multi_out) {
   gamma_ctx *ctx = g->ctx;
   if ((ctx->desc.flags & GAMMA_FLAG_NO_BITMAP) || kmax < 3 || kmax > kBitmapMaxK ||
       g->max_out_degree > kWideMaxRun)
     return false;
   GAMMA_REQUIRE(g->m < 0xFFFFFFFFull, GAMMA_E_UNSUPPORTED, "DAG with >= 2^32 edges");
   ensure_root_order(g);
-  const uint64_t nroots = 2 < g->root_ge.size() ? g->root_ge[2] : 0;   // d+ >= 2
+  kmin = std::max<uint32_t>(3, std::min(kmin, kmax));
+  const uint64_t nroots = kmin - 1 < g->root_ge.size() ? g->root_ge[kmin - 1] : 0;   // d+ >= kmin - 1
   ctx->stats.level_entries[1] = nroots;
   for (uint32_t s = 0; s <= kmax; s++) multi_out[s] = 0;
   if (nroots) {
     const uint64_t n_long = kBitmapMaxRun + 1 < g->root_ge.size() ? g->root_ge[kBitmapMaxRun + 1] : 0;
     const uint64_t n_mid = 129 < g->root_ge.size() ? g->root_ge[129] : 0;
-    kclique_bitmap(g, kmax, g->root_order, nroots, nullptr, true, 0, n_long, n_mid, multi_out);
+    kclique_bitmap(g, kmax, g->root_order, nroots, nullptr, true, 0, n_long, n_mid, multi_out, kmin);
   }
   ctx->sync();
   ctx->collect_timings();

@@ -56,7 +56,8 @@ struct BmArgs {
   uint2 *parts;               // (absolute root index, part | nparts << 16)
   uint32_t parts_cap;
   uint64_t root_base;         // index of roots[0] in the full root list (parts are absolute)
-  uint32_t multi;             // count every clique size 3..k at once (gamma_kclique_multi)
+  uint32_t multi;             // count every clique size kmin..k at once (gamma_kclique_multi)
+  uint32_t kmin;              // multi: smallest size asked for (>= 3); shorter runs are skipped
   uint32_t *wide_rows;        // wide runs: per-CTA global row scratch (wide_stride words each)
   uint64_t wide_stride;
 };
@@ -707,7 +708,7 @@ __global__ void GAMMA_BM_BOUNDS(KM) kcl_bitmap_kernel(BmArgs a) {
     const uint32_t v = a.roots[gi];
     const uint64_t b0 = a.dag_ptr[v];
     const uint32_t L = (uint32_t)(a.dag_ptr[v + 1] - b0);
-    if (L <= a.len_lo || L > a.len_hi || L < (a.multi ? 2u : a.k - 1)) continue;   // uniform across the team
+    if (L <= a.len_lo || L > a.len_hi || L < (a.multi ? a.kmin - 1 : a.k - 1)) continue;   // uniform across the team
     const uint32_t W = (L + 31) >> 5, BS = row_stride<TEAM_WARPS, TW>(L);
     if (tid == 0) entries += L;
     elems += build_rows<TEAM_WARPS, TW>(a, m, b0, L, tid, lane);
@@ -1026,7 +1027,7 @@ __global__ void __launch_bounds__(kWideThreads) kcl_wide_kernel(BmArgs a) {
     const uint32_t v = a.roots[gi];
     const uint64_t b0 = a.dag_ptr[v];
     const uint32_t L = (uint32_t)(a.dag_ptr[v + 1] - b0);
-    if (L <= a.len_lo || L > a.len_hi || L < (a.multi ? 2u : a.k - 1)) {
+    if (L <= a.len_lo || L > a.len_hi || L < (a.multi ? a.kmin - 1 : a.k - 1)) {
       __syncthreads();
       continue;
     }
@@ -1195,7 +1196,7 @@ void enqueue_parts(gamma_ctx *ctx, const BmArgs &a0, bool per_root) {
 // [n_long, n_mid) CTA teams, [n_mid, nroots) warp teams.
 uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint64_t nroots,
                         unsigned long long *per_root, bool sorted, uint64_t n_xl, uint64_t n_long, uint64_t n_mid,
-                        uint64_t *multi_out) {
+                        uint64_t *multi_out, uint32_t kmin) {
   gamma_ctx *ctx = g->ctx;
   BmArgs a{};
   a.dag_ptr = g->dag_ptr;
@@ -1206,6 +1207,7 @@ uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint6
   a.ctrl = (unsigned long long *)ctx->ctrl;
   a.per_root = per_root;
   a.multi = multi_out != nullptr;
+  a.kmin = std::max<uint32_t>(3, std::min(kmin, k));
   // hub splitting only pays when the DFS below a triangle is deep (k >= 6)
   const bool split = k >= 6 && (ctx->desc.flags & GAMMA_FLAG_NO_SPLIT) == 0;
   DevBuf<uint2> parts;
@@ -1274,7 +1276,7 @@ uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint6
   ctx->stats.alg_bytes[KC_BITMAP] += 4 * h[CTRL_AUX0] + 4 * h[CTRL_ELEMS];
   if (split) ctx->stats.chunks += std::min<uint64_t>(h[CTRL_AUX1], a.parts_cap);
   if (multi_out)
-    for (uint32_t sz = 0; sz <= k && sz < 32; sz++) multi_out[sz] = sz >= 3 ? h[CTRL_MULTI + sz] : 0;
+    for (uint32_t sz = 0; sz <= k && sz < 32; sz++) multi_out[sz] = sz >= a.kmin ? h[CTRL_MULTI + sz] : 0;
   return h[CTRL_COUNT];
 }
 

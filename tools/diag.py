@@ -24,7 +24,8 @@ def main():
         if what == "fpm_gpu":
             import paper_conf_icde_hu0o23_b200 as G
             minsup = int(sys.argv[3]) if len(sys.argv) > 3 else 3
-            c = G.Context(time_kernels=True)
+            budget = int(float(sys.argv[4]) * 2 ** 30) if len(sys.argv) > 4 else 0   # GiB (ncu: small pool)
+            c = G.Context(time_kernels=True, hbm_budget_bytes=budget)
             g = c.load_edges(n, s, d, lab)
             for it in range(2):
                 t = time.time()
