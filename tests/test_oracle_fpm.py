@@ -128,3 +128,70 @@ def test_golden_fig2c(oracle_mod):
     res = {(r[2], r[3]): (r[4], r[5]) for r in g.fpm(2, 1)}
     key = (tuple(fx["expect"]["labels"]), tuple(tuple(e) for e in fx["expect"]["edges"]))
     assert res[key] == (fx["expect"]["support"], fx["expect"]["instances"])
+
+
+# ---- 4-edge patterns (FPM length 4) ----
+def _shape(nv, edges):
+    (labs, es), _ = brute.canon(nv, list(range(nv)), [tuple(e) for e in edges], [0] * nv)
+    return (4, nv, labs, es)
+
+
+C4 = _shape(4, [(0, 1), (1, 2), (2, 3), (3, 0)])
+PAW = _shape(4, [(0, 1), (0, 2), (1, 2), (2, 3)])
+STAR4 = _shape(5, [(0, 1), (0, 2), (0, 3), (0, 4)])
+PATH4 = _shape(5, [(0, 1), (1, 2), (2, 3), (3, 4)])
+FORK = _shape(5, [(0, 1), (1, 2), (0, 3), (0, 4)])
+
+
+@pytest.mark.parametrize("n", [5, 6, 7])
+def test_complete_l4(oracle_mod, n):
+    """K_n: the five connected 4-edge shapes, each with MNI n; instance counts
+    C4 3C(n,4), paw 3(n-3)C(n,3), 4-star n C(n-1,4), 4-path n!/(2(n-5)!),
+    fork n(n-1)(n-2)C(n-3,2)."""
+    from math import comb, factorial
+    res = {r[:4]: (r[4], r[5]) for r in G(oracle_mod, gg.complete(n)).fpm(4, 1) if r[0] == 4}
+    assert res == {C4: (n, 3 * comb(n, 4)), PAW: (n, 3 * (n - 3) * comb(n, 3)), STAR4: (n, n * comb(n - 1, 4)),
+                   PATH4: (n, factorial(n) // (2 * factorial(n - 5))), FORK: (n, n * (n - 1) * (n - 2) * comb(n - 3, 2))}
+
+
+@pytest.mark.parametrize("s", [4, 5, 7])
+def test_star_l4(oracle_mod, s):
+    from math import comb
+    res = {r[:4]: (r[4], r[5]) for r in G(oracle_mod, gg.star(s)).fpm(4, 1) if r[0] == 4}
+    assert res == {STAR4: (1, comb(s, 4))}
+
+
+@pytest.mark.parametrize("n", [4, 6, 9])
+def test_cycle_l4(oracle_mod, n):
+    res = {r[:4]: (r[4], r[5]) for r in G(oracle_mod, gg.cycle(n)).fpm(4, 1) if r[0] == 4}
+    assert res == ({C4: (4, 1)} if n == 4 else {PATH4: (n, n)})
+
+
+@pytest.mark.parametrize("seed", [1, 2, 3])
+def test_brute_force_python_l4(oracle_mod, seed):
+    n = 8
+    s, d = gg.er(n, 13, seed)
+    E = brute.normalise(s, d)
+    lab = gg.labels(n, 2, seed)
+    g = oracle_mod.Graph(n, s, d, lab)
+    assert g.fpm(4, 1) == brute.fpm(n, E, 4, 1, lab.tolist())
+
+
+@pytest.mark.parametrize("seed", [1, 2, 3])
+def test_two_enumerations_agree_l4(oracle_mod, seed):
+    n = 20
+    s, d = gg.er(n, 40, seed)
+    lab = gg.labels(n, 3, seed)
+    g = oracle_mod.Graph(n, s, d, lab)
+    for minsup in (1, 2):
+        assert g.fpm(4, minsup, "shapes") == g.fpm(4, minsup, "brute")
+
+
+def test_matches_matching_mni_l4(oracle_mod):
+    s, d = gg.rmat(7, 500, 0.45, 0.22, 0.22, 3)
+    lab = gg.labels(128, 2, 3)
+    g = oracle_mod.Graph(128, s, d, lab)
+    res = [r for r in g.fpm(4, 3) if r[0] == 4]
+    assert len(res) > 5
+    for ne, nv, labs, edges, sup, _ in res:
+        assert g.pattern_mni(nv, list(edges), list(labs)) == sup
