@@ -545,6 +545,8 @@ __global__ void seg_popc_kernel(const uint32_t *buf, uint64_t lo, uint64_t shard
   }
 }
 
+#include "fpm4_device.cuh"
+
 inline unsigned g1d(uint64_t n) {
   const uint64_t b = (n + 255) / 256;
   return (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(b, 148u * 32u));
@@ -865,6 +867,344 @@ struct PoolBuf {
   ~PoolBuf() { reset(); }
 };
 
+
+// ---- level 4 (4-edge patterns, Opt 3 out-of-core aggregation), host side ----------
+// Canonical-code table of <= 5-vertex, <= 4-edge patterns (reading R7), by enumeration
+// of the 120 orders sigma of the sorted positions (sigma[c] = sorted position placed at
+// canonical position c; valid iff it only permutes positions of equal labels): entry
+// (M << 4 | tie) = {smallest sorted pair-index key of the edge mask M under sigma,
+// the first minimizing sigma (3 bits per position) | the orbit representative of every
+// canonical position under Aut_L of the canonical pattern << 15}.  The orbit of c is
+// {c' : some minimizing sigma places at c' what the first one places at c}.
+static void fpm_canon5_table(std::vector<uint2> &tab) {
+  for (uint32_t x = 0; x < 3125; x++) {   // the sorting network, checked exhaustively
+    uint32_t d[5], t = x;
+    for (int i = 0; i < 5; i++) { d[i] = t % 5; t /= 5; }
+    sort5(d[0], d[1], d[2], d[3], d[4]);
+    for (int i = 0; i < 4; i++)
+      GAMMA_REQUIRE(d[i] <= d[i + 1], GAMMA_E_CUDA, "gamma_fpm: 5-element sorting network is wrong");
+  }
+  std::vector<std::array<uint32_t, 5>> perms;
+  std::array<uint32_t, 5> p{0, 1, 2, 3, 4};
+  do perms.push_back(p);
+  while (std::next_permutation(p.begin(), p.end()));
+  tab.assign(kCanon5Entries, make_uint2(0, 0));
+  for (uint32_t M = 0; M < 1024; M++) {
+    if (__builtin_popcount(M) > 4) continue;
+    for (uint32_t tie = 0; tie < 16; tie++) {
+      uint32_t grp[5] = {0, 0, 0, 0, 0};
+      for (int i = 0; i < 4; i++) grp[i + 1] = grp[i] + (((tie >> i) & 1) ? 0 : 1);
+      uint32_t best = 0xffffffffu;
+      std::vector<int> mins;
+      for (int r = 0; r < 120; r++) {
+        const auto &sg = perms[r];
+        bool ok = true;
+        for (int c = 0; c < 5; c++) ok = ok && grp[sg[c]] == grp[c];
+        if (!ok) continue;
+        uint32_t inv[5];
+        for (uint32_t c = 0; c < 5; c++) inv[sg[c]] = c;
+        uint32_t idx[4] = {15, 15, 15, 15}, ne = 0;
+        for (uint32_t i = 0; i < 10; i++)
+          if ((M >> i) & 1u) idx[ne++] = pid5u(inv[(kA5 >> (3 * i)) & 7u], inv[(kB5 >> (3 * i)) & 7u]);
+        std::sort(idx, idx + ne);
+        const uint32_t key = idx[0] << 12 | idx[1] << 8 | idx[2] << 4 | idx[3];
+        if (key < best) {
+          best = key;
+          mins.assign(1, r);
+        } else if (key == best) {
+          mins.push_back(r);
+        }
+      }
+      const auto &s0 = perms[mins[0]];
+      uint32_t y = 0;
+      for (uint32_t c = 0; c < 5; c++) {
+        y |= s0[c] << (3 * c);
+        uint32_t rep = c;
+        for (int r : mins)
+          for (uint32_t c2 = 0; c2 < 5; c2++)
+            if (perms[r][c2] == s0[c] && c2 < rep) rep = c2;
+        y |= rep << (15 + 3 * c);
+      }
+      tab[(M << 4) | tie] = make_uint2(best, y);
+    }
+  }
+}
+
+static gamma_fpm_pattern decode_pattern5(uint64_t key, uint64_t support, uint64_t instances) {
+  gamma_fpm_pattern p{};
+  p.nv = key5_nv(key);
+  p.ne = key5_ne(key);
+  const uint32_t ek = key5_edges(key);
+  for (uint32_t i = 0; i < p.nv; i++) p.labels[i] = key5_label(key, i);
+  for (uint32_t e = 0; e < p.ne; e++) {
+    const uint32_t id = (ek >> (4 * (3 - e))) & 15u;
+    p.edges[e][0] = (kA5 >> (3 * id)) & 7u;
+    p.edges[e][1] = (kB5 >> (3 * id)) & 7u;
+  }
+  p.support = support;
+  p.instances = instances;
+  return p;
+}
+
+// Sort + unique of n tuples in the double buffer db (result at db.Current()); returns
+// the unique count.
+static uint64_t sort_unique(gamma_ctx *ctx, cub::DoubleBuffer<unsigned long long> &db, uint64_t n, int end_bit,
+                            DevBuf<uint8_t> &tmp, unsigned long long *nsel) {
+  if (n == 0) return 0;
+  size_t t1 = 0, t2 = 0;
+  GAMMA_CUDA(cub::DeviceRadixSort::SortKeys(nullptr, t1, db, n, 0, end_bit, ctx->stream));
+  GAMMA_CUDA(cub::DeviceSelect::Unique(nullptr, t2, db.Current(), db.Alternate(), nsel, n, ctx->stream));
+  if (std::max(t1, t2) > tmp.n) tmp = DevBuf<uint8_t>(ctx, std::max(t1, t2));
+  ctx->launch(KC_FPM_SUPPORT, [&] {
+    GAMMA_CUDA(cub::DeviceRadixSort::SortKeys(tmp.p, t1, db, n, 0, end_bit, ctx->stream));
+  });
+  ctx->cub_sort_launched(KC_FPM_SUPPORT, n, end_bit);
+  ctx->launch(KC_FPM_SUPPORT, [&] {
+    GAMMA_CUDA(cub::DeviceSelect::Unique(tmp.p, t2, db.Current(), db.Alternate(), nsel, n, ctx->stream));
+  });
+  ctx->cub_select_launched(KC_FPM_SUPPORT);
+  db.selector ^= 1;
+  uint64_t r = 0;
+  GAMMA_CUDA(cudaMemcpyAsync(&r, nsel, 8, cudaMemcpyDeviceToHost, ctx->stream));
+  ctx->sync();
+  return r;
+}
+
+struct Run4 {
+  unsigned long long *dev = nullptr;   // in the device run area, or
+  unsigned long long *host = nullptr;  // spilled to pinned host memory
+  uint64_t len = 0;
+};
+
+// Level 4: passes of root-edge batches emit (slot, orbit, vertex) tuples; each pass's
+// tuples are segment-sorted and deduplicated into a run (Opt 3's segment sort); runs
+// live in an HBM run area and are spilled to pinned host memory when it fills; the runs
+// are then multi-merged by key range, each range's slice of every run located by its
+// matched index (Def. 5.1, Alg. 3), sorted, deduplicated and counted per
+// (slot, orbit); support = min over orbits (MNI).
+static void fpm_level4(gamma_graph *g, FpmArgs a, int grid4, uint64_t minsup, bool want_inst,
+                       std::vector<gamma_fpm_pattern> &out) {
+  gamma_ctx *ctx = g->ctx;
+  std::vector<uint2> htab5;
+  fpm_canon5_table(htab5);
+  DevBuf<uint2> tab5 = to_device(ctx, htab5.data(), htab5.size());
+  size_t fr = 0, tot = 0;
+  GAMMA_CUDA(cudaMemGetInfo(&fr, &tot));
+  const uint64_t budget = ctx->desc.hbm_budget_bytes ? ctx->desc.hbm_budget_bytes : (uint64_t)(fr * 0.8);
+  const uint64_t ndir = 2 * g->m;
+  const uint64_t nb_total = (ndir + 8 * (uint64_t)a.world - 1) / (8 * (uint64_t)a.world);
+  uint64_t cap4 = 1ull << 14;
+  while (cap4 < (1ull << 26) && cap4 * 48 * 8 < budget) cap4 <<= 1;   // table + counts <= 1/8 of the budget
+  // test knobs: a small tuple buffer / run area forces many passes, spilled runs and a
+  // multi-range merge (GAMMA_FPM4_TUPLES, GAMMA_FPM4_AREA, in tuples)
+  const char *env_t = getenv("GAMMA_FPM4_TUPLES"), *env_a = getenv("GAMMA_FPM4_AREA");
+  DevBuf<unsigned long long> flags(ctx, 4), nsel(ctx, 1);
+  for (int attempt = 0;; attempt++) {
+    GAMMA_REQUIRE(attempt < 4 && cap4 <= (1ull << 28), GAMMA_E_NOMEM, "gamma_fpm: level-4 pattern table overflow");
+    const uint64_t fixed = cap4 * (8 + 32 + 8 + (want_inst ? 16 : 0));
+    GAMMA_REQUIRE(fixed * 2 < budget, GAMMA_E_NOMEM, "gamma_fpm: level-4 pattern table exceeds the HBM budget");
+    // tuple buffers (double buffer for the sort) and the run area share the rest
+    const uint64_t rest = (budget - fixed) / 8;
+    uint64_t T = std::max<uint64_t>(1 << 16, (uint64_t)(rest * 0.22));
+    uint64_t Rcap = std::max<uint64_t>(1 << 16, rest - 2 * T - (rest / 16));   // keep slack for CUB temp
+    if (env_t && *env_t) T = std::max<uint64_t>(256, strtoull(env_t, nullptr, 10));
+    if (env_a && *env_a) Rcap = std::max<uint64_t>(256, strtoull(env_a, nullptr, 10));
+    DevBuf<unsigned long long> key4(ctx, cap4), inst4(ctx, want_inst ? cap4 : 1), inst_pass(ctx, want_inst ? cap4 : 1);
+    DevBuf<uint32_t> cnt(ctx, cap4 * 8);
+    DevBuf<unsigned long long> sup4(ctx, cap4);
+    DevBuf<unsigned long long> tA(ctx, T), tB(ctx, T), area(ctx, Rcap);
+    DevBuf<uint8_t> tmp;
+    GAMMA_CUDA(cudaMemsetAsync(key4.p, 0, cap4 * 8, ctx->stream));
+    GAMMA_CUDA(cudaMemsetAsync(cnt.p, 0, cap4 * 32, ctx->stream));
+    if (want_inst) GAMMA_CUDA(cudaMemsetAsync(inst4.p, 0, cap4 * 8, ctx->stream));
+    Fpm4Args b{};
+    b.tab5 = tab5.p;
+    b.key4 = key4.p;
+    b.inst4 = want_inst ? inst_pass.p : nullptr;
+    b.cap4 = cap4;
+    b.tup = tA.p;
+    b.tup_cap = T;
+    b.flags = flags.p;
+    int slot_bits = 0;
+    while ((1ull << slot_bits) < cap4) slot_bits++;
+    const int end_bit = 35 + slot_bits;
+    std::vector<Run4> runs;
+    std::vector<void *> pinned;
+    uint64_t area_top = 0, entries = 0;
+    bool full = false;
+    uint64_t b0 = 0, span = nb_total;
+    const auto spill_area = [&] {   // device runs -> pinned host memory
+      for (auto &r : runs) {
+        if (!r.dev) continue;
+        void *h = nullptr;
+        GAMMA_CUDA(cudaMallocHost(&h, std::max<uint64_t>(r.len, 1) * 8));
+        pinned.push_back(h);
+        GAMMA_CUDA(cudaMemcpyAsync(h, r.dev, r.len * 8, cudaMemcpyDeviceToHost, ctx->stream));
+        ctx->stats.spilled_bytes += r.len * 8;
+        r.host = (unsigned long long *)h;
+        r.dev = nullptr;
+      }
+      ctx->sync();
+      area_top = 0;
+    };
+    while (b0 < nb_total) {
+      const uint64_t b1 = std::min(nb_total, b0 + span);
+      b.b_begin = b0;
+      b.b_end = b1;
+      GAMMA_CUDA(cudaMemsetAsync(flags.p, 0, 32, ctx->stream));
+      GAMMA_CUDA(cudaMemsetAsync(ctx->ctrl + CTRL_WORK, 0, 8, ctx->stream));
+      if (want_inst) GAMMA_CUDA(cudaMemsetAsync(inst_pass.p, 0, cap4 * 8, ctx->stream));
+      ctx->launch(KC_FPM, [&] { fpm_enum4_kernel<<<grid4, kThreads, 0, ctx->stream>>>(a, b); });
+      uint64_t hf[4];
+      GAMMA_CUDA(cudaMemcpyAsync(hf, flags.p, 32, cudaMemcpyDeviceToHost, ctx->stream));
+      ctx->sync();
+      if (hf[2]) {
+        full = true;
+        break;
+      }
+      if (hf[1]) {   // the pass's tuples overflowed the buffer: halve the batch range
+        GAMMA_REQUIRE(span > 1, GAMMA_E_NOMEM, "gamma_fpm: one root-edge batch overflows the level-4 tuple buffer");
+        span = std::max<uint64_t>(1, span / 2);
+        ctx->stats.retries++;
+        continue;
+      }
+      entries += hf[3];
+      if (want_inst)
+        ctx->launch(KC_MISC, [&] { add_u64_kernel<<<g1d(cap4), 256, 0, ctx->stream>>>(inst4.p, inst_pass.p, cap4); });
+      cub::DoubleBuffer<unsigned long long> db(tA.p, tB.p);
+      const uint64_t r = sort_unique(ctx, db, hf[0], end_bit, tmp, nsel.p);
+      if (r) {
+        if (area_top + r > Rcap) spill_area();
+        if (r > Rcap) {   // a run larger than the area goes straight to the host
+          void *h = nullptr;
+          GAMMA_CUDA(cudaMallocHost(&h, r * 8));
+          pinned.push_back(h);
+          GAMMA_CUDA(cudaMemcpyAsync(h, db.Current(), r * 8, cudaMemcpyDeviceToHost, ctx->stream));
+          ctx->stats.spilled_bytes += r * 8;
+          runs.push_back(Run4{nullptr, (unsigned long long *)h, r});
+        } else {
+          GAMMA_CUDA(cudaMemcpyAsync(area.p + area_top, db.Current(), r * 8, cudaMemcpyDeviceToDevice, ctx->stream));
+          runs.push_back(Run4{area.p + area_top, nullptr, r});
+          area_top += r;
+        }
+      }
+      ctx->stats.chunks++;
+      b0 = b1;
+      if (hf[0] < T / 4 && span < nb_total) span *= 2;
+    }
+    if (full) {
+      ctx->sync();
+      for (void *h : pinned) cudaFreeHost(h);
+      ctx->stats.retries++;
+      cap4 *= 4;
+      continue;
+    }
+    ctx->stats.level_entries[4] = entries;
+    ctx->stats.alg_bytes[KC_FPM] += 40 * entries;   // <= 5 tuples of 8 B per level-4 embedding
+    // ---- multi-merge of the runs by key range (matched indices) + count ----
+    uint64_t total = 0;
+    for (auto &r : runs) total += r.len;
+    const uint64_t M = T;   // merge buffer: one tuple buffer (the other is the sort's alternate)
+    std::vector<unsigned long long> splits;   // range boundaries (exclusive upper bounds)
+    if (runs.size() == 1 && runs[0].dev) {
+      ctx->launch(KC_FPM_SUPPORT, [&] {
+        count_tuples_kernel<<<g1d((runs[0].len + 31) / 32), 256, 0, ctx->stream>>>(runs[0].dev, runs[0].len, cnt.p);
+      });
+    } else if (total) {
+      // splitters from a sample of every run
+      std::vector<unsigned long long> sample;
+      for (auto &r : runs) {
+        const uint64_t stride = std::max<uint64_t>(1, r.len / 256);
+        const uint64_t ns = (r.len + stride - 1) / stride;
+        std::vector<unsigned long long> s(ns);
+        if (r.dev)
+          GAMMA_CUDA(cudaMemcpy2DAsync(s.data(), 8, r.dev, stride * 8, 8, ns, cudaMemcpyDeviceToHost, ctx->stream));
+        else
+          for (uint64_t i = 0; i < ns; i++) s[i] = r.host[i * stride];
+        ctx->sync();
+        sample.insert(sample.end(), s.begin(), s.end());
+      }
+      std::sort(sample.begin(), sample.end());
+      const uint64_t nranges = std::max<uint64_t>(1, (2 * total + M - 1) / M);
+      for (uint64_t i = 1; i < nranges; i++) splits.push_back(sample[i * sample.size() / nranges]);
+      splits.push_back(~0ull);
+      std::sort(splits.begin(), splits.end());
+      splits.erase(std::unique(splits.begin(), splits.end()), splits.end());
+      DevBuf<unsigned long long> qk(ctx, 2);
+      DevBuf<uint64_t> qi(ctx, 2);
+      // matched index of `key` in run r (Def. 5.1: the first position holding a key >= it)
+      const auto matched = [&](const Run4 &r, unsigned long long lo, unsigned long long hi, uint64_t &ilo,
+                               uint64_t &ihi) {
+        if (r.host) {
+          ilo = std::lower_bound(r.host, r.host + r.len, lo) - r.host;
+          ihi = hi == ~0ull ? r.len : (uint64_t)(std::lower_bound(r.host, r.host + r.len, hi) - r.host);
+          return;
+        }
+        const unsigned long long k2[2] = {lo, hi};
+        GAMMA_CUDA(cudaMemcpyAsync(qk.p, k2, 16, cudaMemcpyHostToDevice, ctx->stream));
+        ctx->launch(KC_MISC, [&] { lower_bound_kernel<<<1, 32, 0, ctx->stream>>>(r.dev, r.len, qk.p, 2, qi.p); });
+        uint64_t h2[2];
+        GAMMA_CUDA(cudaMemcpyAsync(h2, qi.p, 16, cudaMemcpyDeviceToHost, ctx->stream));
+        ctx->sync();
+        ilo = h2[0];
+        ihi = hi == ~0ull ? r.len : h2[1];
+      };
+      std::vector<std::pair<unsigned long long, unsigned long long>> ranges;
+      unsigned long long lo = 0;
+      for (unsigned long long hi : splits) {
+        ranges.push_back({lo, hi});
+        lo = hi;
+      }
+      for (size_t qi_ = 0; qi_ < ranges.size(); qi_++) {
+        const unsigned long long rlo = ranges[qi_].first, rhi = ranges[qi_].second;
+        std::vector<std::pair<uint64_t, uint64_t>> sl(runs.size());
+        uint64_t need = 0;
+        for (size_t i = 0; i < runs.size(); i++) {
+          matched(runs[i], rlo, rhi, sl[i].first, sl[i].second);
+          need += sl[i].second - sl[i].first;
+        }
+        if (need > M) {   // the sample misjudged this range: split it at its key midpoint
+          GAMMA_REQUIRE(rhi - rlo > 1, GAMMA_E_NOMEM, "gamma_fpm: a level-4 merge range exceeds the buffer");
+          const unsigned long long mid = rlo + (rhi - rlo) / 2;
+          ranges.insert(ranges.begin() + qi_ + 1, {mid, rhi});
+          ranges[qi_].second = mid;
+          qi_--;
+          continue;
+        }
+        uint64_t at = 0;
+        for (size_t i = 0; i < runs.size(); i++) {
+          const uint64_t len = sl[i].second - sl[i].first;
+          if (!len) continue;
+          if (runs[i].dev)
+            GAMMA_CUDA(cudaMemcpyAsync(tA.p + at, runs[i].dev + sl[i].first, len * 8, cudaMemcpyDeviceToDevice,
+                                       ctx->stream));
+          else
+            GAMMA_CUDA(cudaMemcpyAsync(tA.p + at, runs[i].host + sl[i].first, len * 8, cudaMemcpyHostToDevice,
+                                       ctx->stream));
+          at += len;
+        }
+        cub::DoubleBuffer<unsigned long long> db(tA.p, tB.p);
+        const uint64_t u = sort_unique(ctx, db, at, end_bit, tmp, nsel.p);
+        if (u)
+          ctx->launch(KC_FPM_SUPPORT, [&] {
+            count_tuples_kernel<<<g1d((u + 31) / 32), 256, 0, ctx->stream>>>(db.Current(), u, cnt.p);
+          });
+        ctx->stats.chunks++;
+      }
+    }
+    ctx->launch(KC_FPM_SUPPORT, [&] { support4_kernel<<<g1d(cap4), 256, 0, ctx->stream>>>(key4.p, cap4, cnt.p, sup4.p); });
+    std::vector<unsigned long long> hk(cap4), hs(cap4), hi(want_inst ? cap4 : 0);
+    GAMMA_CUDA(cudaMemcpyAsync(hk.data(), key4.p, cap4 * 8, cudaMemcpyDeviceToHost, ctx->stream));
+    GAMMA_CUDA(cudaMemcpyAsync(hs.data(), sup4.p, cap4 * 8, cudaMemcpyDeviceToHost, ctx->stream));
+    if (want_inst) GAMMA_CUDA(cudaMemcpyAsync(hi.data(), inst4.p, cap4 * 8, cudaMemcpyDeviceToHost, ctx->stream));
+    ctx->sync();
+    for (void *h : pinned) cudaFreeHost(h);
+    for (uint64_t s = 0; s < cap4; s++)
+      if (hk[s] && hs[s] >= minsup) out.push_back(decode_pattern5(hk[s], hs[s], want_inst ? hi[s] : 0));
+    return;
+  }
+}
+
 static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::vector<gamma_fpm_pattern> &out) {
   gamma_ctx *ctx = g->ctx;
   const uint32_t n = g->n;
@@ -879,6 +1219,7 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
     GAMMA_CUDA(cudaMemcpyAsync(&ml, ctx->ctrl + CTRL_AUX1, 8, cudaMemcpyDeviceToHost, ctx->stream));
     ctx->sync();
     GAMMA_REQUIRE(ml < 4096, GAMMA_E_UNSUPPORTED, "gamma_fpm: labels must be < 4096");
+    GAMMA_REQUIRE(max_edges < 4 || ml < 256, GAMMA_E_UNSUPPORTED, "gamma_fpm: 4-edge patterns need labels < 256");
     nlab = (uint32_t)ml + 1;
   }
   DevBuf<uint32_t> csize(ctx, nlab), lrank(ctx, n);
@@ -979,7 +1320,8 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
     a.T = Table{slots.p, sup.p, freq.p, cap, pool.p, pool_words, pcur.p, want_inst ? inst.p : nullptr};
     bool full = false;
     found_last.clear();
-    for (uint32_t l = 1; l <= max_edges && !full; l++) {
+    const uint32_t lmax3 = std::min<uint32_t>(max_edges, 3);   // level 4: fpm_level4 (Opt 3)
+    for (uint32_t l = 1; l <= lmax3 && !full; l++) {
       if (dist && l == max_edges) {
         full = !fpm_dist_level(ctx, a, grid_enum, l, minsup, hsize, cap, slots.p, pool.p, pool_words, pcur.p,
                                found_last);
@@ -1086,6 +1428,24 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
     ctx->stats.retries++;   // sizes are only known after the fact: grow and redo
     cap *= 4;
   }
+  // ---- level 4: out-of-core aggregation of (slot, orbit, vertex) tuples ----
+  std::vector<gamma_fpm_pattern> found4;
+  if (max_edges >= 4) {
+    pool.reset();   // the level <= 3 MNI domains are dead (freq flags stay in the table)
+    FpmArgs a4 = a;
+    a4.level = 4;
+    a4.claim_only = 0;
+    a4.carve_below = 0xffffffffu;
+    a4.walk_lo = 0;
+    a4.rank = 0;
+    a4.world = 1;   // replicated on every rank (the exchange of level-4 tuples is not implemented)
+    a4.T.pool = nullptr;
+    const int grid4 = ctx->num_sms * occupancy_blocks((const void *)fpm_enum4_kernel, kThreads, 0);
+    ctrl_reset(ctx);
+    fpm_level4(g, a4, grid4, minsup, want_inst, found4);
+    ctrl_fetch(ctx);
+    count_fpm_bytes(ctx);
+  }
   // ---- collect the frequent patterns ----
   std::vector<uint32_t> hfreq(cap);
   std::vector<unsigned long long> hkey, hsup(cap), hinst(want_inst ? cap : 0);
@@ -1100,6 +1460,7 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
     out.push_back(decode_pattern(hkey[s], hsup[s], want_inst ? hinst[s] : 0));
   }
   out.insert(out.end(), found_last.begin(), found_last.end());
+  out.insert(out.end(), found4.begin(), found4.end());
   std::sort(out.begin(), out.end(), [](const gamma_fpm_pattern &x, const gamma_fpm_pattern &y) {
     if (x.ne != y.ne) return x.ne < y.ne;
     if (x.nv != y.nv) return x.nv < y.nv;
@@ -1123,7 +1484,7 @@ extern "C" gamma_status gamma_fpm(gamma_graph *g, uint32_t max_edges, uint64_t m
     GAMMA_REQUIRE(g && out, GAMMA_E_INVAL, "gamma_fpm: NULL argument");
     GAMMA_REQUIRE(minsup >= 1, GAMMA_E_INVAL, "gamma_fpm: minsup must be >= 1");
     GAMMA_REQUIRE(max_edges >= 1, GAMMA_E_INVAL, "gamma_fpm: max_edges must be >= 1");
-    GAMMA_REQUIRE(max_edges <= 3, GAMMA_E_UNSUPPORTED, "gamma_fpm: max_edges > 3 not supported in v1");
+    GAMMA_REQUIRE(max_edges <= 4, GAMMA_E_UNSUPPORTED, "gamma_fpm: max_edges > 4 not supported");
     // the enumeration carries symmetric-CSR offsets (< 2m) as u32
     GAMMA_REQUIRE(2 * g->m < (1ull << 32), GAMMA_E_UNSUPPORTED, "gamma_fpm: graphs with 2m >= 2^32 unsupported");
     gamma_ctx *c = g->ctx;

@@ -104,7 +104,7 @@ def test_invalid(G, ctx):
     n, (s, d) = gg.complete(4)
     g = ctx.load_edges(n, s, d)
     with pytest.raises(G.GammaError) as e:
-        g.fpm(4, 1)
+        g.fpm(5, 1)
     assert e.value.status == -5
     with pytest.raises(G.GammaError):
         g.fpm(2, 0)
@@ -238,3 +238,72 @@ def test_c4_full_size_sampled(ctx, oracle_mod):
         assert sup < minsup, (pat, sup)
         cands += 1
     assert cands >= 100
+
+
+# ---- 4-edge patterns (FPM length 4, Opt 3 out-of-core aggregation) ----
+def test_l4_closed_forms(ctx):
+    """K_6: the five connected 4-edge shapes each with MNI 6; star K_{1,5}: the 4-star
+    with MNI 1; cycle C_7: the 4-path with MNI 7 (oracle-independent closed forms)."""
+    import brute
+
+    def shape(nv, edges):
+        (labs, es), _ = brute.canon(nv, list(range(nv)), edges, [0] * nv)
+        return (4, nv, labs, es)
+    c4, paw = shape(4, [(0, 1), (1, 2), (2, 3), (3, 0)]), shape(4, [(0, 1), (0, 2), (1, 2), (2, 3)])
+    star4, path4 = shape(5, [(0, 1), (0, 2), (0, 3), (0, 4)]), shape(5, [(0, 1), (1, 2), (2, 3), (3, 4)])
+    fork = shape(5, [(0, 1), (1, 2), (0, 3), (0, 4)])
+    n, (s, d) = gg.complete(6)
+    res = {r[:4]: r[4] for r in ctx.load_edges(n, s, d).fpm(4, 1) if r[0] == 4}
+    assert res == {c4: 6, paw: 6, star4: 6, path4: 6, fork: 6}
+    n, (s, d) = gg.star(5)
+    assert {r[:4]: r[4] for r in ctx.load_edges(n, s, d).fpm(4, 1) if r[0] == 4} == {star4: 1}
+    n, (s, d) = gg.cycle(7)
+    assert {r[:4]: r[4] for r in ctx.load_edges(n, s, d).fpm(4, 1) if r[0] == 4} == {path4: 7}
+
+
+@pytest.mark.parametrize("seed", [1, 2, 3])
+@pytest.mark.parametrize("L", [1, 3])
+def test_l4_er_vs_oracle(G, oracle_mod, seed, L):
+    """Every (pattern, MNI support, instance count) of 1..4 edges against the oracle,
+    at several thresholds (Alg. 2 pruning of 3-edge prefixes included)."""
+    n = 60
+    s, d = gg.er(n, 140, seed)
+    lab = gg.labels(n, L, seed) if L > 1 else None
+    c = G.Context(flags=G._native.GAMMA_FLAG_FPM_INSTANCES)
+    g = c.load_edges(n, s, d, lab)
+    o = oracle_mod.Graph(n, s, d, lab)
+    for minsup in (1, 2, 4):
+        want = [r[:6] for r in o.fpm(4, minsup, pattern_cap=1 << 20)]
+        assert g.fpm(4, minsup, instances=True) == want, minsup
+        if minsup == 1:   # every connected 4-edge set enumerated exactly once
+            assert c.stats()["level_entries"][4] == sum(r[5] for r in want if r[0] == 4)
+
+
+def test_l4_rmat_vs_oracle(ctx, oracle_mod):
+    """configs[3]'s generator at scale 8 (5.6M connected 4-edge sets), 4 labels."""
+    n, s, d, lab = gg.config_graph("c4", seed=1, scale=8)
+    lab = gg.labels(n, 4, 1)
+    g = ctx.load_edges(n, s, d, lab)
+    o = oracle_mod.Graph(n, s, d, lab)
+    assert g.fpm(4, 10) == oracle_set(o, 4, 10)
+
+
+@pytest.mark.parametrize("tuples,area", [(1 << 14, 1 << 30), (1 << 14, 20000), (1 << 15, 4096)])
+def test_l4_out_of_core(G, oracle_mod, monkeypatch, tuples, area):
+    """Opt 3 paths forced by small buffers: many passes (tuple buffer overflow halves the
+    batch range), runs spilled to pinned host memory when the HBM run area fills, and a
+    multi-range merge located by matched indices -- same result as the oracle."""
+    monkeypatch.setenv("GAMMA_FPM4_TUPLES", str(tuples))
+    monkeypatch.setenv("GAMMA_FPM4_AREA", str(area))
+    n = 300
+    s, d = gg.er(n, 900, 3)
+    lab = gg.labels(n, 3, 3)
+    c = G.Context(flags=G._native.GAMMA_FLAG_FPM_INSTANCES)
+    g = c.load_edges(n, s, d, lab)
+    o = oracle_mod.Graph(n, s, d, lab)
+    want = [r[:6] for r in o.fpm(4, 2, pattern_cap=1 << 20)]
+    assert g.fpm(4, 2, instances=True) == want
+    st = c.stats()
+    assert st["chunks"] > 3
+    if area < 1 << 30:
+        assert st["spilled_bytes"] > 0
