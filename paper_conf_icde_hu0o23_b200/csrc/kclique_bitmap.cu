@@ -390,15 +390,31 @@ __device__ __forceinline__ uint64_t gdfs_count(const uint32_t *B, uint32_t BS, u
   return cnt;
 }
 
-// Item q -> this lane's word of the candidates of the triangle (v, R[j1], R[j2]).
-__device__ __forceinline__ uint32_t group_item_cur(const uint32_t *B, const uint32_t *P, uint32_t L, uint32_t W,
-                                                   uint32_t BS, uint32_t q, const LaneGroup &g) {
-  uint32_t lo = 0, hi = L;   // j1 = last row with P[j1] <= q
-  while (hi - lo > 1) {
-    const uint32_t mid = (lo + hi) >> 1;
-    if (P[mid] <= q) lo = mid; else hi = mid;
+// j1 = the last row with P[j1] <= q, found from the previous item's row (a caller's
+// items only move forward): a short forward scan, then a binary search over the rest
+// (the per-item binary search from row 0 was ~12 % of the CTA-team kernel's
+// instructions, ncu heavy r02).
+__device__ __forceinline__ uint32_t advance_row(const uint32_t *P, uint32_t L, uint32_t q, uint32_t j1) {
+#pragma unroll
+  for (int s = 0; s < 4; s++)
+    if (j1 + 1 < L && P[j1 + 1] <= q) j1++;
+  if (j1 + 1 < L && P[j1 + 1] <= q) {
+    uint32_t lo = j1 + 1, hi = L;
+    while (hi - lo > 1) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if (P[mid] <= q) lo = mid; else hi = mid;
+    }
+    j1 = lo;
   }
-  const uint32_t j1 = lo, r = q - P[j1];
+  return j1;
+}
+
+// Item q -> this lane's word of the candidates of the triangle (v, R[j1], R[j2]); j1
+// carries the row of the caller's previous item (0 for the first).
+__device__ __forceinline__ uint32_t group_item_cur(const uint32_t *B, const uint32_t *P, uint32_t L, uint32_t W,
+                                                   uint32_t BS, uint32_t q, const LaneGroup &g, uint32_t &j1) {
+  j1 = advance_row(P, L, q, j1);
+  const uint32_t r = q - P[j1];
   const uint32_t w1 = g.gl < (int)W ? B[j1 * BS + g.gl] : 0u;
   // the r-th set bit of row j1: inclusive scan of the word popcounts over the group
   const uint32_t pc = __popc(w1);
@@ -483,7 +499,7 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
     const uint32_t x = R[i];
     uint32_t h = (x * 0x9E3779B1u) >> (32 - hbits);
     if (Hv) {
-      h &= ~1u;   // probing starts at an even slot: a lookup reads the slot pair in one load
+      h &= ~3u;   // probing starts at a 4-slot bucket: a lookup reads the bucket in one load
       while (atomicCAS(&Hv[h], kEmptyId, x) != kEmptyId) h = (h + 1) & hmask;
       H[h] = (unsigned short)i;
     } else {
@@ -540,16 +556,17 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
       for (int u = 0; u < kTiles; u++) {
         const uint32_t yy = y[u];
         if (Hv) {
-          // one 8-byte load of the even slot pair where y's probe sequence starts;
-          // both compares are predicated, and only a full pair without y (rare at
-          // load <= 1/4) continues the linear probe
+          // one 16-byte load of the 4-slot bucket where y's probe sequence starts; the
+          // compares are predicated, and only a full bucket without y (rare at load
+          // <= 1/4: the pair-slot probe this replaced sent 87 % of warps into the chain
+          // loop, ncu heavy r02) continues the linear probe
           const bool inr = yy >= rmin && yy <= rmax;   // (the padding 0xffffffff is above every rmax < n)
-          const uint32_t h0 = ((yy * 0x9E3779B1u) >> (32 - hbits)) & ~1u;
-          const uint2 vv = *reinterpret_cast<const uint2 *>(Hv + h0);
-          bool hit = inr && (vv.x == yy || vv.y == yy);
-          uint32_t hh = vv.x == yy ? h0 : h0 + 1;
-          if (inr && vv.x != yy && vv.y != yy && vv.x != kEmptyId && vv.y != kEmptyId) {
-            for (uint32_t h = (h0 + 2) & hmask;; h = (h + 1) & hmask) {
+          const uint32_t h0 = ((yy * 0x9E3779B1u) >> (32 - hbits)) & ~3u;
+          const uint4 vv = *reinterpret_cast<const uint4 *>(Hv + h0);
+          bool hit = inr && (vv.x == yy || vv.y == yy || vv.z == yy || vv.w == yy);
+          uint32_t hh = vv.x == yy ? h0 : vv.y == yy ? h0 + 1 : vv.z == yy ? h0 + 2 : h0 + 3;
+          if (inr && !hit && vv.w != kEmptyId && vv.x != kEmptyId && vv.y != kEmptyId && vv.z != kEmptyId) {
+            for (uint32_t h = (h0 + 4) & hmask;; h = (h + 1) & hmask) {
               const uint32_t vh = Hv[h];
               if (vh == yy) {
                 hit = true;
@@ -620,16 +637,12 @@ __device__ void scan_rows(const TeamMem<TW> &m, uint32_t L, int tid, int lane) {
   team_sync<TEAM_WARPS>();
 }
 
-// Item q -> candidates of the triangle (v, R[j1], R[j2]).
+// Item q -> candidates of the triangle (v, R[j1], R[j2]); j1 carries the row of the
+// caller's previous item (0 for the first).
 template <int TW>
 __device__ __forceinline__ void item_cur(const TeamMem<TW> &m, uint32_t L, uint32_t W, uint32_t BS, uint32_t q,
-                                         uint32_t (&cur)[TW]) {
-  uint32_t lo = 0, hi = L;   // j1 = last row with P[j1] <= q
-  while (hi - lo > 1) {
-    const uint32_t mid = (lo + hi) >> 1;
-    if (m.P[mid] <= q) lo = mid; else hi = mid;
-  }
-  const uint32_t j1 = lo;
+                                         uint32_t (&cur)[TW], uint32_t &j1) {
+  j1 = advance_row(m.P, L, q, j1);
   uint32_t r = q - m.P[j1], j2 = 0;
   for (uint32_t w = 0; w < W; w++) {
     const uint32_t word = m.B[j1 * BS + w];
@@ -728,9 +741,10 @@ __global__ void GAMMA_BM_BOUNDS(KM) kcl_bitmap_kernel(BmArgs a) {
       bool deferred = false;
       if (a.heavy_cut) {   // hub splitting: estimate the DFS by the 4-clique count
         uint64_t est = 0;
+        uint32_t jr = 0;
         for (uint32_t q = tid; q < items; q += kTeamThreads) {
           uint32_t cur[TW];
-          item_cur<TW>(m, L, W, BS, q, cur);
+          item_cur<TW>(m, L, W, BS, q, cur, jr);
           uint32_t c = 0;
 #pragma unroll
           for (int w = 0; w < TW; w++) c += __popc(cur[w]);
@@ -767,10 +781,11 @@ __global__ void GAMMA_BM_BOUNDS(KM) kcl_bitmap_kernel(BmArgs a) {
           team_sync<TEAM_WARPS>();
         }
       }
+      uint32_t jr = 0;
       if (TEAM_WARPS == 1 && !deferred)
         for (uint32_t q = tid; q < items; q += kTeamThreads) {
           uint32_t cur[TW];
-          item_cur<TW>(m, L, W, BS, q, cur);
+          item_cur<TW>(m, L, W, BS, q, cur, jr);
           if constexpr (TEAM_WARPS == 1) {   // register-resident nested loops
             if (a.multi) {
               mc[3] += 1;   // the item is one triangle
@@ -784,8 +799,9 @@ __global__ void GAMMA_BM_BOUNDS(KM) kcl_bitmap_kernel(BmArgs a) {
         if (!deferred) {
           const LaneGroup g = lane_group(lane);
           constexpr uint32_t kGroups = kTeamThreads / kGroup;
+          uint32_t jg = 0;
           for (uint32_t q = tid / kGroup; q < items; q += kGroups) {
-            const uint32_t curw = group_item_cur(m.B, m.P, L, W, BS, q, g);
+            const uint32_t curw = group_item_cur(m.B, m.P, L, W, BS, q, g, jg);
             if (a.multi) {
               if (g.gl == 0) mc[3] += 1;   // the item is one triangle
               gdfs_multi<3, KM, kMaxStack + 3>(m.B, BS, W, curw, a.k, mc, g);
@@ -853,8 +869,9 @@ __global__ void GAMMA_BM_BOUNDS(KM) kcl_bitmap_parts_kernel(BmArgs a) {
     uint64_t cnt = 0;
     const LaneGroup g = lane_group(lane);
     constexpr uint32_t kGroups = 256 / kGroup;
+    uint32_t jg = 0;
     for (uint32_t q = part + (tid / kGroup) * nparts; q < items; q += kGroups * nparts) {
-      const uint32_t curw = group_item_cur(m.B, m.P, L, W, BS, q, g);
+      const uint32_t curw = group_item_cur(m.B, m.P, L, W, BS, q, g, jg);
       if (a.multi) {
         if (g.gl == 0) mc[3] += 1;
         gdfs_multi<3, KM, kMaxStack + 3>(m.B, BS, W, curw, a.k, mc, g);
