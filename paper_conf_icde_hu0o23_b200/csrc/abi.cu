@@ -295,6 +295,7 @@ void gamma_graph_free(gamma_graph *g) {
     c->free(g->dag_col);
     c->free(g->labels);
     c->free(g->root_order);
+    c->free(g->rank_of);
     try {
       c->keep_release();   // kept SM tables were sized for this graph
     } catch (...) {
@@ -323,11 +324,14 @@ gamma_status gamma_graph_copy_csr(const gamma_graph *g, int which, uint64_t *row
     GAMMA_REQUIRE(which == 0 || which == 1, GAMMA_E_INVAL, "which must be 0 (symmetric) or 1 (DAG)");
     gamma_ctx *c = g->ctx;
     GAMMA_CUDA(cudaSetDevice(c->device));
-    const uint64_t *rp = which ? g->dag_ptr : g->row_ptr;
-    const uint32_t *cl = which ? g->dag_col : g->col;
-    uint64_t ne = which ? g->m : 2 * g->m;
-    GAMMA_CUDA(cudaMemcpyAsync(row_ptr, rp, ((size_t)g->n + 1) * sizeof(uint64_t), cudaMemcpyDefault, c->stream));
-    if (ne) GAMMA_CUDA(cudaMemcpyAsync(col, cl, ne * sizeof(uint32_t), cudaMemcpyDefault, c->stream));
+    if (which == 1) {   // the kCL DAG lives in rank space: export it in id space
+      export_dag_ids(const_cast<gamma_graph *>(g), row_ptr, col);
+      return;
+    }
+    const uint64_t ne = 2 * g->m;
+    GAMMA_CUDA(cudaMemcpyAsync(row_ptr, g->row_ptr, ((size_t)g->n + 1) * sizeof(uint64_t), cudaMemcpyDefault,
+                               c->stream));
+    if (ne) GAMMA_CUDA(cudaMemcpyAsync(col, g->col, ne * sizeof(uint32_t), cudaMemcpyDefault, c->stream));
     c->sync();
   });
 }
@@ -394,6 +398,7 @@ gamma_status gamma_kclique_roots(gamma_graph *g, uint32_t k, uint64_t nroots, co
     c->keep_release();   // kCL sizes its levels from free HBM
     if (nroots == 0) return;
     DevBuf<uint32_t> r = to_device(c, roots, nroots);
+    to_rank_space(g, r.p, nroots);   // the kCL DAG is in rank space (graph.cu rank_dag)
     DevBuf<uint64_t> out(c, nroots);
     GAMMA_CUDA(cudaMemsetAsync(out.p, 0, nroots * sizeof(uint64_t), c->stream));
     kclique_count(g, k, r.p, nroots, out.p);

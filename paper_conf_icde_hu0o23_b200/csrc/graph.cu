@@ -250,6 +250,65 @@ __global__ void dag_write_kernel(const uint64_t *__restrict__ row_ptr, const uin
   }
 }
 
+// ---- rank-space DAG (kCL): vertices relabelled by their rank in the (degree, id)
+// order, so that a DAG list sorted ascending is sorted by rank and every out-neighbour
+// has a larger id than its tail; the kCL kernels then trim a child's list at the
+// largest rank of the root's run (everything above cannot be in it) ----
+__global__ void rank_keys_kernel(const uint64_t *__restrict__ row_ptr, uint32_t n, uint64_t *__restrict__ keys) {
+  for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x)
+    keys[v] = ((row_ptr[v + 1] - row_ptr[v]) << 32) | v;
+}
+
+__global__ void rank_scatter_kernel(const uint64_t *__restrict__ sorted, uint32_t n, uint32_t *__restrict__ rank_of) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+    rank_of[(uint32_t)sorted[i]] = (uint32_t)i;
+}
+
+// one warp per id-space DAG row u: key of every edge u -> x in rank space
+__global__ void dag_rank_keys_kernel(const uint64_t *__restrict__ dag_ptr, const uint32_t *__restrict__ dag_col,
+                                     const uint32_t *__restrict__ rank_of, uint32_t n, uint32_t b,
+                                     uint64_t *__restrict__ keys) {
+  const int lane = threadIdx.x & 31;
+  for (uint64_t u = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5; u < n;
+       u += ((uint64_t)gridDim.x * blockDim.x) >> 5) {
+    const uint64_t ru = (uint64_t)rank_of[u] << b;
+    for (uint64_t e = dag_ptr[u] + lane; e < dag_ptr[u + 1]; e += 32) keys[e] = ru | rank_of[dag_col[e]];
+  }
+}
+
+// id-space DAG (export): d+ of id u, then the sym row of u filtered by rank
+__global__ void dag_id_count_kernel(const uint64_t *__restrict__ rdag_ptr, const uint32_t *__restrict__ rank_of,
+                                    uint32_t n, uint64_t *__restrict__ cnt) {
+  for (uint64_t u = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; u < n; u += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t r = rank_of[u];
+    cnt[u] = rdag_ptr[r + 1] - rdag_ptr[r];
+  }
+}
+
+__global__ void dag_id_write_kernel(const uint64_t *__restrict__ row_ptr, const uint32_t *__restrict__ col,
+                                    const uint32_t *__restrict__ rank_of, uint32_t n,
+                                    const uint64_t *__restrict__ dag_ptr, uint32_t *__restrict__ dag_col) {
+  const int lane = threadIdx.x & 31;
+  const uint32_t below = (1u << lane) - 1u;
+  for (uint64_t v = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5; v < n;
+       v += ((uint64_t)gridDim.x * blockDim.x) >> 5) {
+    const uint32_t rv = rank_of[v];
+    uint64_t w = dag_ptr[v];
+    for (uint64_t i0 = row_ptr[v]; i0 < row_ptr[v + 1]; i0 += 32) {
+      const uint64_t i = i0 + lane;
+      uint32_t x = 0;
+      bool keep = false;
+      if (i < row_ptr[v + 1]) {
+        x = col[i];
+        keep = rank_of[x] > rv;
+      }
+      const uint32_t bal = __ballot_sync(0xffffffffu, keep);
+      if (keep) dag_col[w + __popc(bal & below)] = x;
+      w += __popc(bal);
+    }
+  }
+}
+
 uint32_t bit_width(uint32_t n) {  // bits to represent n itself
   uint32_t b = 0;
   while (b < 32 && (uint64_t(1) << b) <= n) b++;
@@ -341,6 +400,80 @@ void build_dag(gamma_graph *g, uint64_t *keys, uint64_t M) {
   g->dag_col = dc.release();
   g->device_bytes += ((uint64_t)g->n + 1) * 8 + mdag * 4;
   g->max_out_degree = max_degree(ctx, g->dag_ptr, g->n);
+}
+
+// Relabel the DAG built in id space (g->dag_ptr/dag_col) into rank space (see
+// rank_keys_kernel): rank_of by one sort of (degree, id) keys, the edges re-keyed and
+// sorted into a rank-space CSR; the id-space DAG is freed.
+void rank_dag(gamma_graph *g) {
+  gamma_ctx *ctx = g->ctx;
+  const uint32_t n = g->n, b = g->bits;
+  const uint64_t m = g->m;
+  DevBuf<uint32_t> rank_of(ctx, n);
+  {
+    DevBuf<uint64_t> k0(ctx, n), k1(ctx, n);
+    ctx->launch(KC_BUILD, [&] { rank_keys_kernel<<<grid_for(n), kThreads, 0, ctx->stream>>>(g->row_ptr, n, k0.p); });
+    int endbit = 32;
+    while (endbit < 64 && (1ull << (endbit - 32)) <= g->max_degree) endbit++;
+    sort_keys(ctx, k0.p, k1.p, n, endbit);
+    ctx->launch(KC_BUILD, [&] { rank_scatter_kernel<<<grid_for(n), kThreads, 0, ctx->stream>>>(k1.p, n, rank_of.p); });
+  }
+  if (m) {
+    DevBuf<uint64_t> k0(ctx, m), k1(ctx, m);
+    ctx->launch(KC_BUILD, [&] {
+      dag_rank_keys_kernel<<<grid_for((uint64_t)n * 32), kThreads, 0, ctx->stream>>>(g->dag_ptr, g->dag_col,
+                                                                                     rank_of.p, n, b, k0.p);
+    });
+    sort_keys(ctx, k0.p, k1.p, m, 2 * b);
+    ctx->launch(KC_BUILD, [&] {
+      csr_from_keys_kernel<<<grid_for(m), kThreads, 0, ctx->stream>>>(k1.p, m, n, b, g->dag_ptr, g->dag_col);
+    });
+  }
+  g->rank_of = rank_of.release();
+  g->device_bytes += (uint64_t)n * 4;
+}
+
+namespace {
+__global__ void to_rank_kernel(uint32_t *v, uint64_t nv, const uint32_t *rank_of, uint32_t n) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < nv; i += (uint64_t)gridDim.x * blockDim.x)
+    if (v[i] < n) v[i] = rank_of[v[i]];   // ids >= n stay invalid
+}
+}  // namespace
+
+void to_rank_space(gamma_graph *g, uint32_t *ids, uint64_t nids) {
+  if (!nids) return;
+  gamma_ctx *ctx = g->ctx;
+  ctx->launch(KC_ROOTS, [&] {
+    to_rank_kernel<<<grid_for(nids), kThreads, 0, ctx->stream>>>(ids, nids, g->rank_of, g->n);
+  });
+}
+
+// The id-space DAG (gamma_graph_copy_csr(which = 1)): out-lists of every vertex id,
+// ascending by id, oriented by the (degree, id) order.
+void export_dag_ids(gamma_graph *g, uint64_t *dag_ptr_out, uint32_t *dag_col_out) {
+  gamma_ctx *ctx = g->ctx;
+  const uint32_t n = g->n;
+  DevBuf<uint64_t> cnt(ctx, (size_t)n + 1), dp(ctx, (size_t)n + 1);
+  DevBuf<uint32_t> dc(ctx, g->m ? g->m : 1);
+  GAMMA_CUDA(cudaMemsetAsync(cnt.p + n, 0, 8, ctx->stream));
+  ctx->launch(KC_MISC, [&] {
+    dag_id_count_kernel<<<grid_for(n), kThreads, 0, ctx->stream>>>(g->dag_ptr, g->rank_of, n, cnt.p);
+  });
+  size_t tmp = 0;
+  GAMMA_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tmp, cnt.p, dp.p, (int64_t)n + 1, ctx->stream));
+  {
+    DevBuf<uint8_t> t(ctx, tmp);
+    ctx->launch(KC_MISC, [&] {
+      GAMMA_CUDA(cub::DeviceScan::ExclusiveSum(t.p, tmp, cnt.p, dp.p, (int64_t)n + 1, ctx->stream));
+    });
+  }
+  ctx->launch(KC_MISC, [&] {
+    dag_id_write_kernel<<<grid_for((uint64_t)n * 32), kThreads, 0, ctx->stream>>>(g->row_ptr, g->col, g->rank_of, n,
+                                                                                  dp.p, dc.p);
+  });
+  GAMMA_CUDA(cudaMemcpyAsync(dag_ptr_out, dp.p, ((size_t)n + 1) * 8, cudaMemcpyDefault, ctx->stream));
+  if (g->m) GAMMA_CUDA(cudaMemcpyAsync(dag_col_out, dc.p, g->m * 4, cudaMemcpyDefault, ctx->stream));
+  ctx->sync();
 }
 
 namespace {
@@ -461,6 +594,7 @@ void build_from_edges(gamma_graph *g, const uint32_t *src, const uint32_t *dst, 
   }
   if (m && 2 * m < (1ull << 31) && (ctx->desc.flags & GAMMA_FLAG_COUNT_SORT_BUILD) != 0) {
     build_counting(g, src, dst, m);
+    rank_dag(g);
     g->build_ms = timer.stop();
     return;
   }
@@ -514,6 +648,7 @@ void build_from_edges(gamma_graph *g, const uint32_t *src, const uint32_t *dst, 
   g->device_bytes += ((uint64_t)n + 1) * 8 + M * 4;
   g->max_degree = max_degree(ctx, g->row_ptr, n);
   build_dag(g, uniq.p, M);
+  rank_dag(g);
   g->build_ms = timer.stop();
 }
 
@@ -558,6 +693,7 @@ void build_from_csr(gamma_graph *g, const uint64_t *row_ptr, const uint32_t *col
   g->device_bytes += ((uint64_t)n + 1) * 8 + M * 4;
   g->max_degree = max_degree(ctx, g->row_ptr, n);
   build_dag(g, keys.p, M);
+  rank_dag(g);
   g->build_ms = timer.stop();
 }
 

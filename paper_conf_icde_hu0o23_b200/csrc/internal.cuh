@@ -168,8 +168,11 @@ struct gamma_graph {
   uint32_t bits = 1;             // bits needed for a vertex id (ids < 2^bits)
   uint64_t *row_ptr = nullptr;   // n+1
   uint32_t *col = nullptr;       // 2m
+  // kCL DAG in RANK space (graph.cu rank_dag): vertex r = the r-th vertex in the
+  // (degree, id) order; lists ascending (= by rank); rank_of maps an id to its rank
   uint64_t *dag_ptr = nullptr;   // n+1
   uint32_t *dag_col = nullptr;   // m
+  uint32_t *rank_of = nullptr;   // n
   uint32_t *labels = nullptr;    // n (nullptr: unlabeled, all 0)
   uint32_t max_degree = 0, max_out_degree = 0;
   uint64_t device_bytes = 0;
@@ -238,6 +241,9 @@ void build_from_edges(gamma_graph *g, const uint32_t *src, const uint32_t *dst, 
                       bool src_on_device);
 void build_from_csr(gamma_graph *g, const uint64_t *row_ptr, const uint32_t *col);
 void build_dag(gamma_graph *g, uint64_t *sorted_keys_dev, uint64_t nkeys);
+void rank_dag(gamma_graph *g);                       // id-space DAG -> rank space (+ rank_of)
+void export_dag_ids(gamma_graph *g, uint64_t *dag_ptr_out, uint32_t *dag_col_out);
+void to_rank_space(gamma_graph *g, uint32_t *ids_dev, uint64_t nids);   // in place, on the stream
 
 // kCL (kclique.cu)
 uint64_t kclique_count(gamma_graph *g, uint32_t k, const uint32_t *roots_dev, uint64_t nroots,

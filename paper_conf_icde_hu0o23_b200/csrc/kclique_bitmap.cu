@@ -517,6 +517,17 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
       const uint64_t cb = a.dag_ptr[c];
       dl = (uint32_t)(a.dag_ptr[c + 1] - cb);
       beg = (uint32_t)cb;
+      // rank space: lists ascend by rank, so the part of N+(c) above the run's largest
+      // rank cannot meet the run -- trim it (one binary search; ~19 % of the C2 row-build
+      // elements, scratch/rank_cut.py)
+      if (dl && __ldg(a.dag_col + cb + dl - 1) > rmax) {
+        uint32_t lo = 0, hi = dl - 1;   // first index with dag_col > rmax, in [0, dl - 1]
+        while (lo < hi) {
+          const uint32_t mid = (lo + hi) >> 1;
+          if (__ldg(a.dag_col + cb + mid) > rmax) hi = mid; else lo = mid + 1;
+        }
+        dl = lo;
+      }
     }
     elems += dl;
     // compact the children with non-empty lists to lanes 0..nnz-1 (every list then
