@@ -342,11 +342,54 @@ __device__ __forceinline__ uint32_t group_leaf_sum_w(const uint32_t *B, uint32_t
   return acc;
 }
 
+// Balanced variant: the group's set bits of cur are dealt to its lanes by rank (bit r
+// to lane r mod 16), each lane summing whole rows -- the per-word walk above gives a
+// lane the bits of its own word, and with the run sorted by rank the candidates of a
+// deep node crowd into its last words (ncu c2 r02: 2.4 threads per instruction on the
+// leaf loop of the CTA-team kernel).
+template <int WW>
+__device__ __forceinline__ uint32_t group_leaf_sum_bal(const uint32_t *B, uint32_t BS, uint32_t W, uint32_t curw,
+                                                       const LaneGroup &g) {
+  uint32_t s = __popc(curw);
+#pragma unroll
+  for (int o = 1; o < kGroup; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(g.mask, s, o);
+    if (g.gl >= o) s += y;
+  }
+  uint32_t cur[WW], inc[WW];
+#pragma unroll
+  for (int w = 0; w < WW; w++) {
+    cur[w] = __shfl_sync(g.mask, curw, g.base + w);
+    inc[w] = __shfl_sync(g.mask, s, g.base + w);   // bits in words 0..w (W <= WW: the rest are 0)
+  }
+  const uint32_t total = inc[WW - 1];
+  uint32_t acc = 0;
+  for (uint32_t r = g.gl; r < total; r += kGroup) {
+    uint32_t wsel = 0, before = 0;
+#pragma unroll
+    for (int w = 0; w < WW; w++)
+      if (inc[w] <= r) {
+        wsel = w + 1;
+        before = inc[w];
+      }
+    uint32_t word = 0;
+#pragma unroll
+    for (int w = 0; w < WW; w++)
+      if (w == (int)wsel) word = cur[w];
+    const uint32_t j = wsel * 32 + __fns(word, 0, r - before + 1);
+    const uint32_t *row = B + j * BS;
+#pragma unroll
+    for (int w = 0; w < WW; w++)
+      if (w < (int)W) acc += __popc(cur[w] & row[w]);
+  }
+  return acc;
+}
+
 __device__ __forceinline__ uint32_t group_leaf_sum(const uint32_t *B, uint32_t BS, uint32_t W, uint32_t curw,
                                                    const LaneGroup &g) {
-  if (W <= 4) return group_leaf_sum_w<4>(B, BS, W, curw, g);
-  if (W <= 8) return group_leaf_sum_w<8>(B, BS, W, curw, g);
-  return group_leaf_sum_w<kGroup>(B, BS, W, curw, g);
+  if (W <= 4) return group_leaf_sum_bal<4>(B, BS, W, curw, g);
+  if (W <= 8) return group_leaf_sum_bal<8>(B, BS, W, curw, g);
+  return group_leaf_sum_bal<kGroup>(B, BS, W, curw, g);
 }
 
 template <int S, int SM, int N>
@@ -1237,7 +1280,10 @@ uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint6
   a.multi = multi_out != nullptr;
   a.kmin = std::max<uint32_t>(3, std::min(kmin, k));
   // hub splitting only pays when the DFS below a triangle is deep (k >= 6)
-  const bool split = k >= 6 && (ctx->desc.flags & GAMMA_FLAG_NO_SPLIT) == 0;
+  // (GAMMA_KCL_SPLIT_MINK: the smallest k that splits, default 6)
+  const char *mk_env = getenv("GAMMA_KCL_SPLIT_MINK");
+  const uint32_t split_mink = mk_env && *mk_env ? (uint32_t)std::max(3ul, strtoul(mk_env, nullptr, 10)) : 6u;
+  const bool split = k >= split_mink && (ctx->desc.flags & GAMMA_FLAG_NO_SPLIT) == 0;
   DevBuf<uint2> parts;
   if (split) {
     // GAMMA_KCL_PARTS_CAP (tests): a small part list forces the "list full, expand
