@@ -793,7 +793,9 @@ __global__ void GAMMA_BM_BOUNDS(KM) kcl_bitmap_kernel(BmArgs a) {
       scan_rows<TEAM_WARPS, TW>(m, L, tid, lane);
       const uint32_t items = m.P[L];
       bool deferred = false;
-      if (a.heavy_cut) {   // hub splitting: estimate the DFS by the 4-clique count
+      // hub splitting: estimate the DFS by the 4-clique count (skipped when even
+      // items x |R| -- an upper bound of it -- is below the cut: most roots)
+      if (a.heavy_cut && (uint64_t)items * L > a.heavy_cut) {
         uint64_t est = 0;
         uint32_t jr = 0;
         for (uint32_t q = tid; q < items; q += kTeamThreads) {
