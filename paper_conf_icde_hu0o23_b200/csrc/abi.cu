@@ -296,6 +296,7 @@ void gamma_graph_free(gamma_graph *g) {
     c->free(g->labels);
     c->free(g->root_order);
     c->free(g->rank_of);
+    c->free(g->ldeg);
     try {
       c->keep_release();   // kept SM tables were sized for this graph
     } catch (...) {

@@ -173,6 +173,10 @@ struct gamma_graph {
   uint64_t *dag_ptr = nullptr;   // n+1
   uint32_t *dag_col = nullptr;   // m
   uint32_t *rank_of = nullptr;   // n
+  // SM filters: label << 24 | min(degree, 2^24 - 1) per vertex, built on the first
+  // gamma_match when every label is < 256 (ldeg_state: -1 not yet, 0 unusable, 1 built)
+  uint32_t *ldeg = nullptr;
+  int32_t ldeg_state = -1;
   uint32_t *labels = nullptr;    // n (nullptr: unlabeled, all 0)
   uint32_t max_degree = 0, max_out_degree = 0;
   uint64_t device_bytes = 0;

@@ -75,6 +75,8 @@ struct SmArgs {
   const uint64_t *rp;
   const uint32_t *col;
   const uint32_t *lab;      // nullable (unlabeled graph: all 0)
+  const uint32_t *ldeg;     // nullable: label << 24 | min(degree, 2^24 - 1) per vertex (labels < 256):
+                            // one 4-byte gather for the label and degree filters
   SmPlan P;
   uint32_t d;               // children are at position d; extend to q = d+1
   const uint32_t *vid_in;
@@ -97,6 +99,7 @@ struct SmArgs {
   uint32_t lm_cap, out_cap; // shared-memory staging per warp (u32 entries)
   uint32_t slice;           // children per group descriptor of the next level
   uint32_t long_ratio;      // last level: child lists > long_ratio * |L_m| are probed from L_m (0: off)
+  uint32_t short_lm;        // last level: |L_m| <= short_lm uses the (child, L_m element) pair probes
 };
 
 __device__ __forceinline__ uint32_t gdeg(const SmArgs &a, uint32_t v) {
@@ -116,7 +119,12 @@ struct Bounds {
 __device__ __forceinline__ bool sm_filter(const SmArgs &a, uint32_t q, uint32_t x, const Bounds &b,
                                           const uint32_t *phi, bool last, bool staged = false) {
   if ((int64_t)x <= b.lo || x >= b.hi) return false;
-  if (a.P.labeled && !staged) {
+  const bool need_deg = !last && !staged && a.P.mindeg[q] > 1;
+  uint32_t ld = 0;
+  if (a.ldeg && !staged && (a.P.labeled || need_deg)) {
+    ld = __ldg(a.ldeg + x);
+    if (a.P.labeled && (ld >> 24) != a.P.label[q]) return false;
+  } else if (a.P.labeled && !staged) {
     const uint32_t lx = a.lab ? a.lab[x] : 0u;
     if (lx != a.P.label[q]) return false;
   }
@@ -126,7 +134,7 @@ __device__ __forceinline__ bool sm_filter(const SmArgs &a, uint32_t q, uint32_t 
     m &= m - 1;
     if (phi[j] == x) return false;
   }
-  if (!last && !staged && a.P.mindeg[q] > 1 && gdeg(a, x) < a.P.mindeg[q]) return false;
+  if (need_deg && (a.ldeg ? (ld & 0xffffffu) : gdeg(a, x)) < a.P.mindeg[q]) return false;
   m = b.anti;   // induced: anti-edge checks, one binary search per non-neighbour
   while (m) {
     const int j = __ffs(m) - 1;
@@ -316,7 +324,7 @@ __global__ void __launch_bounds__(kThreads, 5) sm_kernel(SmArgs a) {
             if (inj_d && (int64_t)c > lo && c < hi && cnt && sorted_contains(lm, lm_len, c)) cnt--;
             part += cnt;
           }
-        } else if (lm_len > 32) {
+        } else if (lm_len > a.short_lm) {
           // cand(c) = L_m ∩ N(c) ∩ window with a long L_m: stream the children's lists
           // N(c) in flattened windows of 32 children (one element per lane per step,
           // child found by an OR-reduction of the window's start offsets) and probe L_m
@@ -543,6 +551,24 @@ struct RootOk {
   }
 };
 
+__global__ void sm_max_label(const uint32_t *lab, uint32_t n, unsigned long long *out) {
+  unsigned long long mx = 0;
+  for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x)
+    mx = lab[v] > mx ? lab[v] : mx;
+  for (int o = 16; o > 0; o >>= 1) {
+    const unsigned long long y = __shfl_down_sync(0xffffffffu, mx, o);
+    mx = y > mx ? y : mx;
+  }
+  if ((threadIdx.x & 31) == 0 && mx) atomicMax(out, mx);
+}
+
+__global__ void sm_ldeg(const uint64_t *rp, const uint32_t *lab, uint32_t n, uint32_t *ldeg) {
+  for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x) {
+    const uint64_t d = rp[v + 1] - rp[v];
+    ldeg[v] = ((lab ? lab[v] : 0u) << 24) | (uint32_t)(d < 0xffffffull ? d : 0xffffffull);
+  }
+}
+
 __global__ void sm_iota(uint32_t *p, uint32_t n) {
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
     p[i] = (uint32_t)i;
@@ -591,6 +617,10 @@ static uint32_t sm_out_cap() {
 }
 static uint32_t sm_long_ratio() {
   static const uint32_t v = env_u32("GAMMA_SM_LONGRATIO", kLongRatio, 0, 1u << 20);
+  return v;
+}
+static uint32_t sm_short_lm() {   // GAMMA_SM_SHORTLM: r01 behaviour was 32
+  static const uint32_t v = env_u32("GAMMA_SM_SHORTLM", 0, 0, 4096);
   return v;
 }
 static uint32_t sm_batch() {   // groups per work-queue atomic below the roots
@@ -761,6 +791,7 @@ struct SmRun {
     a.rp = g->row_ptr;
     a.col = g->col;
     a.lab = g->labels;
+    a.ldeg = g->ldeg;
     a.P = P;
     a.d = d;
     a.vid_in = lv[d].vid.p;
@@ -778,6 +809,7 @@ struct SmRun {
     a.lm_cap = sm_lm_cap();
     a.out_cap = sm_out_cap();
     a.long_ratio = sm_long_ratio();
+    a.short_lm = sm_short_lm();
     a.slice = sm_slice(d + 2 >= P.nv - 1);   // the groups written here are consumed at depth d+1
     return a;
   }
@@ -904,8 +936,30 @@ struct SmRun {
   }
 };
 
+static void ensure_ldeg(gamma_graph *g) {
+  if (g->ldeg_state >= 0) return;
+  gamma_ctx *ctx = g->ctx;
+  uint64_t ml = 0;
+  if (g->labels) {
+    GAMMA_CUDA(cudaMemsetAsync(ctx->ctrl + CTRL_AUX0, 0, 8, ctx->stream));
+    ctx->launch(KC_ROOTS, [&] {
+      sm_max_label<<<g1d(g->n), 256, 0, ctx->stream>>>(g->labels, g->n, (unsigned long long *)ctx->ctrl + CTRL_AUX0);
+    });
+    GAMMA_CUDA(cudaMemcpyAsync(&ml, ctx->ctrl + CTRL_AUX0, 8, cudaMemcpyDeviceToHost, ctx->stream));
+    ctx->sync();
+  }
+  g->ldeg_state = 0;
+  if (ml >= 256) return;
+  DevBuf<uint32_t> ld(ctx, g->n);
+  ctx->launch(KC_ROOTS, [&] { sm_ldeg<<<g1d(g->n), 256, 0, ctx->stream>>>(g->row_ptr, g->labels, g->n, ld.p); });
+  g->ldeg = ld.release();
+  g->device_bytes += (uint64_t)g->n * 4;
+  g->ldeg_state = 1;
+}
+
 static uint64_t match_count(gamma_graph *g, const SmPlan &P) {
   gamma_ctx *ctx = g->ctx;
+  ensure_ldeg(g);
   SmRun R;
   R.g = g;
   R.ctx = ctx;
