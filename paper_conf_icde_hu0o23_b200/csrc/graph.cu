@@ -254,6 +254,11 @@ __global__ void dag_write_kernel(const uint64_t *__restrict__ row_ptr, const uin
 // order, so that a DAG list sorted ascending is sorted by rank and every out-neighbour
 // has a larger id than its tail; the kCL kernels then trim a child's list at the
 // largest rank of the root's run (everything above cannot be in it) ----
+__global__ void iota_u32_kernel(uint32_t *p, uint32_t n) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+    p[i] = (uint32_t)i;
+}
+
 __global__ void rank_keys_kernel(const uint64_t *__restrict__ row_ptr, uint32_t n, uint64_t *__restrict__ keys) {
   for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x)
     keys[v] = ((row_ptr[v + 1] - row_ptr[v]) << 32) | v;
@@ -277,22 +282,29 @@ __global__ void dag_rank_keys_kernel(const uint64_t *__restrict__ dag_ptr, const
 }
 
 // id-space DAG (export): d+ of id u, then the sym row of u filtered by rank
-__global__ void dag_id_count_kernel(const uint64_t *__restrict__ rdag_ptr, const uint32_t *__restrict__ rank_of,
+__device__ __forceinline__ bool dag_before(const uint64_t *row_ptr, uint32_t v, uint32_t x) {   // (deg, id) order
+  const uint64_t dv = row_ptr[v + 1] - row_ptr[v], dx = row_ptr[x + 1] - row_ptr[x];
+  return dv < dx || (dv == dx && v < x);
+}
+
+__global__ void dag_id_count_kernel(const uint64_t *__restrict__ row_ptr, const uint32_t *__restrict__ col,
                                     uint32_t n, uint64_t *__restrict__ cnt) {
-  for (uint64_t u = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; u < n; u += (uint64_t)gridDim.x * blockDim.x) {
-    const uint32_t r = rank_of[u];
-    cnt[u] = rdag_ptr[r + 1] - rdag_ptr[r];
+  const int lane = threadIdx.x & 31;
+  for (uint64_t v = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5; v < n;
+       v += ((uint64_t)gridDim.x * blockDim.x) >> 5) {
+    uint32_t c = 0;
+    for (uint64_t i = row_ptr[v] + lane; i < row_ptr[v + 1]; i += 32) c += dag_before(row_ptr, (uint32_t)v, col[i]);
+    for (int o = 16; o > 0; o >>= 1) c += __shfl_down_sync(0xffffffffu, c, o);
+    if (lane == 0) cnt[v] = c;
   }
 }
 
 __global__ void dag_id_write_kernel(const uint64_t *__restrict__ row_ptr, const uint32_t *__restrict__ col,
-                                    const uint32_t *__restrict__ rank_of, uint32_t n,
-                                    const uint64_t *__restrict__ dag_ptr, uint32_t *__restrict__ dag_col) {
+                                    uint32_t n, const uint64_t *__restrict__ dag_ptr, uint32_t *__restrict__ dag_col) {
   const int lane = threadIdx.x & 31;
   const uint32_t below = (1u << lane) - 1u;
   for (uint64_t v = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5; v < n;
        v += ((uint64_t)gridDim.x * blockDim.x) >> 5) {
-    const uint32_t rv = rank_of[v];
     uint64_t w = dag_ptr[v];
     for (uint64_t i0 = row_ptr[v]; i0 < row_ptr[v + 1]; i0 += 32) {
       const uint64_t i = i0 + lane;
@@ -300,7 +312,7 @@ __global__ void dag_id_write_kernel(const uint64_t *__restrict__ row_ptr, const 
       bool keep = false;
       if (i < row_ptr[v + 1]) {
         x = col[i];
-        keep = rank_of[x] > rv;
+        keep = dag_before(row_ptr, (uint32_t)v, x);
       }
       const uint32_t bal = __ballot_sync(0xffffffffu, keep);
       if (keep) dag_col[w + __popc(bal & below)] = x;
@@ -410,6 +422,13 @@ void rank_dag(gamma_graph *g) {
   const uint32_t n = g->n, b = g->bits;
   const uint64_t m = g->m;
   DevBuf<uint32_t> rank_of(ctx, n);
+  const char *off_env = getenv("GAMMA_NO_RANK_DAG");   // ablation: keep the id-space DAG
+  if (off_env && *off_env && *off_env != '0') {
+    ctx->launch(KC_BUILD, [&] { iota_u32_kernel<<<grid_for(n), kThreads, 0, ctx->stream>>>(rank_of.p, n); });
+    g->rank_of = rank_of.release();
+    g->device_bytes += (uint64_t)n * 4;
+    return;
+  }
   {
     DevBuf<uint64_t> k0(ctx, n), k1(ctx, n);
     ctx->launch(KC_BUILD, [&] { rank_keys_kernel<<<grid_for(n), kThreads, 0, ctx->stream>>>(g->row_ptr, n, k0.p); });
@@ -457,7 +476,7 @@ void export_dag_ids(gamma_graph *g, uint64_t *dag_ptr_out, uint32_t *dag_col_out
   DevBuf<uint32_t> dc(ctx, g->m ? g->m : 1);
   GAMMA_CUDA(cudaMemsetAsync(cnt.p + n, 0, 8, ctx->stream));
   ctx->launch(KC_MISC, [&] {
-    dag_id_count_kernel<<<grid_for(n), kThreads, 0, ctx->stream>>>(g->dag_ptr, g->rank_of, n, cnt.p);
+    dag_id_count_kernel<<<grid_for((uint64_t)n * 32), kThreads, 0, ctx->stream>>>(g->row_ptr, g->col, n, cnt.p);
   });
   size_t tmp = 0;
   GAMMA_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tmp, cnt.p, dp.p, (int64_t)n + 1, ctx->stream));
@@ -468,8 +487,8 @@ void export_dag_ids(gamma_graph *g, uint64_t *dag_ptr_out, uint32_t *dag_col_out
     });
   }
   ctx->launch(KC_MISC, [&] {
-    dag_id_write_kernel<<<grid_for((uint64_t)n * 32), kThreads, 0, ctx->stream>>>(g->row_ptr, g->col, g->rank_of, n,
-                                                                                  dp.p, dc.p);
+    dag_id_write_kernel<<<grid_for((uint64_t)n * 32), kThreads, 0, ctx->stream>>>(g->row_ptr, g->col, n, dp.p,
+                                                                                  dc.p);
   });
   GAMMA_CUDA(cudaMemcpyAsync(dag_ptr_out, dp.p, ((size_t)n + 1) * 8, cudaMemcpyDefault, ctx->stream));
   if (g->m) GAMMA_CUDA(cudaMemcpyAsync(dag_col_out, dc.p, g->m * 4, cudaMemcpyDefault, ctx->stream));

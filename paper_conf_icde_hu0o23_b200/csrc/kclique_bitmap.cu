@@ -58,6 +58,7 @@ struct BmArgs {
   uint64_t root_base;         // index of roots[0] in the full root list (parts are absolute)
   uint32_t multi;             // count every clique size kmin..k at once (gamma_kclique_multi)
   uint32_t kmin;              // multi: smallest size asked for (>= 3); shorter runs are skipped
+  uint32_t trim;              // trim each child's list at the run's largest id (GAMMA_KCL_NO_TRIM: off)
   uint32_t *wide_rows;        // wide runs: per-CTA global row scratch (wide_stride words each)
   uint64_t wide_stride;
 };
@@ -563,7 +564,7 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
       // rank space: lists ascend by rank, so the part of N+(c) above the run's largest
       // rank cannot meet the run -- trim it (one binary search; ~19 % of the C2 row-build
       // elements, scratch/rank_cut.py)
-      if (dl && __ldg(a.dag_col + cb + dl - 1) > rmax) {
+      if (a.trim && dl && __ldg(a.dag_col + cb + dl - 1) > rmax) {
         uint32_t lo = 0, hi = dl - 1;   // first index with dag_col > rmax, in [0, dl - 1]
         while (lo < hi) {
           const uint32_t mid = (lo + hi) >> 1;
@@ -1281,6 +1282,10 @@ uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint6
   a.per_root = per_root;
   a.multi = multi_out != nullptr;
   a.kmin = std::max<uint32_t>(3, std::min(kmin, k));
+  {
+    const char *e = getenv("GAMMA_KCL_NO_TRIM");
+    a.trim = !(e && *e && *e != '0');
+  }
   // hub splitting only pays when the DFS below a triangle is deep (k >= 6)
   // (GAMMA_KCL_SPLIT_MINK: the smallest k that splits, default 6)
   const char *mk_env = getenv("GAMMA_KCL_SPLIT_MINK");

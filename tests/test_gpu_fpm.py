@@ -288,7 +288,7 @@ def test_l4_rmat_vs_oracle(ctx, oracle_mod):
     assert g.fpm(4, 10) == oracle_set(o, 4, 10)
 
 
-@pytest.mark.parametrize("tuples,area", [(1 << 14, 1 << 30), (1 << 14, 20000), (1 << 15, 4096)])
+@pytest.mark.parametrize("tuples,area", [(1 << 16, 1 << 30), (1 << 16, 20000), (1 << 17, 4096)])
 def test_l4_out_of_core(G, oracle_mod, monkeypatch, tuples, area):
     """Opt 3 paths forced by small buffers: many passes (tuple buffer overflow halves the
     batch range), runs spilled to pinned host memory when the HBM run area fills, and a
