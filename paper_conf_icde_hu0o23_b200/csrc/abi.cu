@@ -208,6 +208,7 @@ void gamma_ctx_destroy(gamma_ctx *ctx) {
   if (ctx->ctrl) cudaFree(ctx->ctrl);
   if (ctx->ctrl_host) cudaFreeHost(ctx->ctrl_host);
   if (ctx->spill_host) cudaFreeHost(ctx->spill_host);
+  if (ctx->copy_stream) cudaStreamDestroy(ctx->copy_stream);
   for (auto e : ctx->ev_pool) cudaEventDestroy(e);
   if (ctx->own_stream && ctx->stream) cudaStreamDestroy(ctx->stream);
   cudaGetLastError();

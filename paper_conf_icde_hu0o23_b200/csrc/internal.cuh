@@ -91,6 +91,12 @@ struct gamma_ctx {
   // pinned host arena for spilled ET levels (GAMMA_FLAG_SPILL), used as a stack
   uint8_t *spill_host = nullptr;
   size_t spill_cap = 0, spill_top = 0;
+  // second stream for the spill copies (created on first use, non-blocking)
+  cudaStream_t copy_stream = nullptr;
+  cudaStream_t copy_stream_get() {
+    if (!copy_stream) GAMMA_CUDA(cudaStreamCreateWithFlags(&copy_stream, cudaStreamNonBlocking));
+    return copy_stream;
+  }
   // stats of the last call
   gamma_run_stats stats;
   // event pool for kernel timing

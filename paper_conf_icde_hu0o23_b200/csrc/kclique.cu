@@ -573,21 +573,62 @@ struct KclRun {
   // GAMMA_FLAG_SPILL: BFS with a host-resident next level (the ET "should
   // be resident in host memory ... we keep a buffer on the device to write extension
   // results ... and flush them to host memory").  Level d+1 is produced in slabs that
-  // fit the device buffer, each slab is parked in pinned host memory, and the slabs
-  // are streamed back one at a time for the next extension.
+  // fit the device buffer and parked in pinned host memory; the slabs are then streamed
+  // back one at a time for the next extension.  Two device buffers alternate (the
+  // level's own and a spare of the same size) and every copy runs on the context's copy
+  // stream, fenced by events: the D2H of slab i overlaps the extension writing slab
+  // i + 1, and the H2D of slab i + 1 overlaps the processing of slab i.
+  struct SpillBufs {
+    Level spare;
+    cudaEvent_t free_ev[2] = {nullptr, nullptr};   // buffer b may be overwritten (copy done / use done)
+    cudaEvent_t ready_ev[2] = {nullptr, nullptr};  // buffer b holds its data (produced / copied in)
+    ~SpillBufs() {
+      for (int i = 0; i < 2; i++) {
+        if (free_ev[i]) cudaEventDestroy(free_ev[i]);
+        if (ready_ev[i]) cudaEventDestroy(ready_ev[i]);
+      }
+    }
+  };
+
   void process_spill(uint32_t d, uint64_t g0, uint64_t g1) {
     const uint32_t nd = d + 1;
     struct Slab { size_t off; uint64_t nv, ng; };
     std::vector<Slab> slabs;
     const size_t top0 = ctx->spill_top;
+    if (ctx->spill_host == nullptr) {
+      ctx->spill_cap = ctx->desc.host_spill_bytes;
+      GAMMA_CUDA(cudaMallocHost(&ctx->spill_host, ctx->spill_cap));
+    }
+    cudaStream_t cs = ctx->copy_stream_get();
+    SpillBufs sb;
+    for (int i = 0; i < 2; i++) {
+      GAMMA_CUDA(cudaEventCreateWithFlags(&sb.free_ev[i], cudaEventDisableTiming));
+      GAMMA_CUDA(cudaEventCreateWithFlags(&sb.ready_ev[i], cudaEventDisableTiming));
+    }
+    Level *buf[2] = {&levels[nd], &sb.spare};
+    {   // the spare has the level's capacity
+      Level &S = sb.spare;
+      S.vid = DevBuf<uint32_t>(ctx, buf[0]->cap_v);
+      S.grp = DevBuf<uint2>(ctx, buf[0]->cap_g);
+      if (per_root) S.groot = DevBuf<uint32_t>(ctx, buf[0]->cap_g);
+      S.cap_v = buf[0]->cap_v;
+      S.cap_g = buf[0]->cap_g;
+    }
+    const auto slab_bytes = [&](const Slab &s) { return s.nv * 4 + s.ng * 8 + (per_root ? s.ng * 4 : 0); };
+    // ---- produce: extension into buffer cur, D2H of the previous slab overlapping it ----
+    int cur = 0;
+    bool pending[2] = {false, false};
     std::vector<std::pair<uint64_t, uint64_t>> todo{{g0, g1}};
     while (!todo.empty()) {
       const auto r = todo.back();
       todo.pop_back();
-      Level &L = levels[nd];
+      Level &L = *buf[cur];
+      if (pending[cur]) GAMMA_CUDA(cudaStreamWaitEvent(ctx->stream, sb.free_ev[cur], 0));   // its D2H is done
+      if (cur) std::swap(levels[nd], L);   // the kernels write levels[nd]
       KclArgs a = args_for(d, r.first, r.second);
       set_output(a, nd);
-      launch<MODE_EXTEND>(a, d, L.cap_v);
+      launch<MODE_EXTEND>(a, d, levels[nd].cap_v);
+      if (cur) std::swap(levels[nd], L);
       const uint64_t *h = ctx->ctrl_host;
       if (h[CTRL_OVF]) {
         ctx->stats.retries++;
@@ -602,36 +643,51 @@ struct KclRun {
       ctx->stats.chunks++;
       ctx->stats.level_entries[nd + 1] += h[CTRL_ENTRIES];
       Slab s{0, std::min<uint64_t>(h[CTRL_VCUR], L.cap_v), std::min<uint64_t>(h[CTRL_GCUR], L.cap_g)};
-      const size_t bytes = s.nv * 4 + s.ng * 8 + (per_root ? s.ng * 4 : 0);
-      if (ctx->spill_host == nullptr) {
-        ctx->spill_cap = ctx->desc.host_spill_bytes;
-        GAMMA_CUDA(cudaMallocHost(&ctx->spill_host, ctx->spill_cap));
-      }
+      const size_t bytes = slab_bytes(s);
       GAMMA_REQUIRE(ctx->spill_top + bytes <= ctx->spill_cap, GAMMA_E_NOMEM,
                     "host spill budget exhausted (raise host_spill_bytes)");
       s.off = ctx->spill_top;
       uint8_t *dst = ctx->spill_host + s.off;
-      GAMMA_CUDA(cudaMemcpyAsync(dst, L.vid.p, s.nv * 4, cudaMemcpyDeviceToHost, ctx->stream));
-      GAMMA_CUDA(cudaMemcpyAsync(dst + s.nv * 4, L.grp.p, s.ng * 8, cudaMemcpyDeviceToHost, ctx->stream));
+      GAMMA_CUDA(cudaEventRecord(sb.ready_ev[cur], ctx->stream));
+      GAMMA_CUDA(cudaStreamWaitEvent(cs, sb.ready_ev[cur], 0));
+      GAMMA_CUDA(cudaMemcpyAsync(dst, L.vid.p, s.nv * 4, cudaMemcpyDeviceToHost, cs));
+      GAMMA_CUDA(cudaMemcpyAsync(dst + s.nv * 4, L.grp.p, s.ng * 8, cudaMemcpyDeviceToHost, cs));
       if (per_root)
-        GAMMA_CUDA(cudaMemcpyAsync(dst + s.nv * 4 + s.ng * 8, L.groot.p, s.ng * 4, cudaMemcpyDeviceToHost,
-                                   ctx->stream));
-      ctx->sync();
+        GAMMA_CUDA(cudaMemcpyAsync(dst + s.nv * 4 + s.ng * 8, L.groot.p, s.ng * 4, cudaMemcpyDeviceToHost, cs));
+      GAMMA_CUDA(cudaEventRecord(sb.free_ev[cur], cs));
+      pending[cur] = true;
       ctx->spill_top += bytes;
       ctx->stats.spilled_bytes += bytes;
       slabs.push_back(s);
+      cur ^= 1;
     }
-    for (const Slab &s : slabs) {
-      Level &L = levels[nd];
+    GAMMA_CUDA(cudaStreamSynchronize(cs));   // every slab is on the host
+    // ---- consume: slab i processed from one buffer while slab i + 1 is copied in ----
+    const auto fetch = [&](size_t i, int b) {
+      const Slab &s = slabs[i];
+      Level &L = *buf[b];
+      GAMMA_CUDA(cudaStreamWaitEvent(cs, sb.free_ev[b], 0));   // the previous user is done
       const uint8_t *src = ctx->spill_host + s.off;
-      GAMMA_CUDA(cudaMemcpyAsync(L.vid.p, src, s.nv * 4, cudaMemcpyHostToDevice, ctx->stream));
-      GAMMA_CUDA(cudaMemcpyAsync(L.grp.p, src + s.nv * 4, s.ng * 8, cudaMemcpyHostToDevice, ctx->stream));
+      GAMMA_CUDA(cudaMemcpyAsync(L.vid.p, src, s.nv * 4, cudaMemcpyHostToDevice, cs));
+      GAMMA_CUDA(cudaMemcpyAsync(L.grp.p, src + s.nv * 4, s.ng * 8, cudaMemcpyHostToDevice, cs));
       if (per_root)
-        GAMMA_CUDA(cudaMemcpyAsync(L.groot.p, src + s.nv * 4 + s.ng * 8, s.ng * 4, cudaMemcpyHostToDevice,
-                                   ctx->stream));
-      ctx->stats.spilled_bytes += s.nv * 4 + s.ng * 8 + (per_root ? s.ng * 4 : 0);
-      process(nd, 0, s.ng);
+        GAMMA_CUDA(cudaMemcpyAsync(L.groot.p, src + s.nv * 4 + s.ng * 8, s.ng * 4, cudaMemcpyHostToDevice, cs));
+      GAMMA_CUDA(cudaEventRecord(sb.ready_ev[b], cs));
+      ctx->stats.spilled_bytes += slab_bytes(s);
+    };
+    for (int b = 0; b < 2; b++) GAMMA_CUDA(cudaEventRecord(sb.free_ev[b], ctx->stream));
+    if (!slabs.empty()) fetch(0, 0);
+    for (size_t i = 0; i < slabs.size(); i++) {
+      const int b = (int)(i & 1);
+      if (i + 1 < slabs.size()) fetch(i + 1, b ^ 1);
+      GAMMA_CUDA(cudaStreamWaitEvent(ctx->stream, sb.ready_ev[b], 0));
+      if (b) std::swap(levels[nd], *buf[b]);   // process() reads levels[nd]
+      process(nd, 0, slabs[i].ng);
+      if (b) std::swap(levels[nd], *buf[b]);
+      GAMMA_CUDA(cudaEventRecord(sb.free_ev[b], ctx->stream));
     }
+    ctx->sync();
+    GAMMA_CUDA(cudaStreamSynchronize(cs));
     ctx->spill_top = top0;
   }
 };

@@ -57,6 +57,10 @@ def kernel_ms(st):
     return sum(c["ms"] for k, c in st["classes"].items() if k in HOT)
 
 
+def class_ms(st):
+    return {k: round(c["ms"], 3) for k, c in st["classes"].items() if c["launches"]}
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("workload", choices=["c2", "heavy", "c3", "c5"])
@@ -77,6 +81,8 @@ def main():
         got = work(g1, args.workload)
         torch.cuda.synchronize()
         t1.append(kernel_ms(base.stats()) if args.workload != "c3" else None)
+    if args.workload != "c3":
+        print("world 1 classes", class_ms(base.stats()), flush=True)
     g1.free()
     per_rank, parts = [], []
     for r, c in enumerate(ctxs):
@@ -95,12 +101,14 @@ def main():
             else:
                 res = work(g, args.workload)
                 ms = kernel_ms(c.stats())
+                cls = class_ms(c.stats())
             torch.cuda.synchronize()
             times.append(ms)
         per_rank.append(min(times))
         parts.append(res)
         g.free()
-        print(f"rank {r}: kernel ms {min(times):.3f} partial {res}", flush=True)
+        print(f"rank {r}: kernel ms {min(times):.3f} partial {res} classes {cls if args.workload != 'c3' else ''}",
+              flush=True)
     tot = [sum(p[i] for p in parts) for i in range(len(want))]
     assert tot == want, (tot, want)
     mean = statistics.mean(per_rank)
