@@ -591,9 +591,17 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
     // before any probe, so each lane keeps several L2 gathers in flight
     constexpr int kTiles = 4;
     for (uint32_t t0 = 0; t0 < T; t0 += 32 * kTiles) {
+      // tiles that hold elements (warp-uniform): a short window runs 1-3 tiles, not 4
+      // (the padded tiles were ~half the row-build instructions on C2's small roots)
+      const uint32_t nt = (T - t0 + 31) >> 5;
       uint32_t y[kTiles], rj[kTiles];
 #pragma unroll
       for (int u = 0; u < kTiles; u++) {
+        if ((uint32_t)u >= nt) {
+          y[u] = 0xffffffffu;
+          rj[u] = 0;
+          continue;
+        }
         const uint32_t tb = t0 + 32 * u;
         const uint32_t t = tb + lane;
         // lane t's list = the last list starting at or before t: one OR-reduction of
@@ -609,6 +617,7 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
       }
 #pragma unroll
       for (int u = 0; u < kTiles; u++) {
+        if ((uint32_t)u >= nt) break;
         const uint32_t yy = y[u];
         if (Hv) {
           // one 16-byte load of the 4-slot bucket where y's probe sequence starts; the
