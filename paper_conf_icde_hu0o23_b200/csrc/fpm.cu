@@ -1215,8 +1215,24 @@ static void fpm_level4(gamma_graph *g, FpmArgs a, int grid4, uint64_t minsup, bo
   }
 }
 
+// GAMMA_DEBUG: host wall time of the phases of one gamma_fpm call (stream-synchronised)
+struct PhaseLog {
+  gamma_ctx *ctx;
+  bool on;
+  std::chrono::steady_clock::time_point t;
+  explicit PhaseLog(gamma_ctx *c) : ctx(c), on(getenv("GAMMA_DEBUG") != nullptr), t(std::chrono::steady_clock::now()) {}
+  void mark(const char *what) {
+    if (!on) return;
+    ctx->sync();
+    const auto now = std::chrono::steady_clock::now();
+    fprintf(stderr, "[gamma_fpm] %-28s %9.2f ms\n", what, std::chrono::duration<double, std::milli>(now - t).count());
+    t = now;
+  }
+};
+
 static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::vector<gamma_fpm_pattern> &out) {
   gamma_ctx *ctx = g->ctx;
+  PhaseLog plog(ctx);
   const uint32_t n = g->n;
   // ---- label classes: sizes and in-class ranks ----
   uint32_t nlab = 1;
@@ -1317,7 +1333,9 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
     slots = DevBuf<unsigned long long>(ctx, 2 * cap);
     sup = DevBuf<unsigned long long>(ctx, cap);
     freq = DevBuf<uint32_t>(ctx, cap);
+    plog.mark("setup");
     pool.alloc(pool_words);
+    plog.mark("pool cudaMalloc");
     pcur = DevBuf<unsigned long long>(ctx, 1);
     GAMMA_CUDA(cudaMemsetAsync(slots.p, 0, cap * 16, ctx->stream));
     GAMMA_CUDA(cudaMemsetAsync(freq.p, 0, cap * 4, ctx->stream));
@@ -1328,6 +1346,7 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
       GAMMA_CUDA(cudaMemsetAsync(inst.p, 0, cap * 8, ctx->stream));
     }
     a.T = Table{slots.p, sup.p, freq.p, cap, pool.p, pool_words, pcur.p, want_inst ? inst.p : nullptr};
+    plog.mark("table + pool memset");
     bool full = false;
     found_last.clear();
     const uint32_t lmax3 = std::min<uint32_t>(max_edges, 3);   // level 4: fpm_level4 (Opt 3)
@@ -1369,6 +1388,7 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
         full = f != 0;
       }
       if (full) break;
+      plog.mark(l == 1 ? "level 1" : l == 2 ? "level 2" : "level 3");
       ctx->stats.level_entries[l] = ctx->ctrl_host[CTRL_ENTRIES];
       // a level's domains are dead once its supports are known (the next level reads
       // only freq): clear what it used and carve the next level from offset 0
@@ -1438,6 +1458,9 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
     ctx->stats.retries++;   // sizes are only known after the fact: grow and redo
     cap *= 4;
   }
+  plog.mark("levels done");
+  pool.reset();   // the level <= 3 MNI domains are dead (freq flags stay in the table)
+  plog.mark("pool cudaFree");
   // ---- level 4: out-of-core aggregation of (slot, orbit, vertex) tuples ----
   std::vector<gamma_fpm_pattern> found4;
   if (max_edges >= 4) {
@@ -1456,6 +1479,7 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
     ctrl_fetch(ctx);
     count_fpm_bytes(ctx);
   }
+  plog.mark("level 4 / pool free");
   // ---- collect the frequent patterns ----
   std::vector<uint32_t> hfreq(cap);
   std::vector<unsigned long long> hkey, hsup(cap), hinst(want_inst ? cap : 0);
@@ -1482,6 +1506,7 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
     }
     return false;
   });
+  plog.mark("collect + sort");
   ctx->collect_timings();
 }
 

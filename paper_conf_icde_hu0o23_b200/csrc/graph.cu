@@ -422,8 +422,11 @@ void rank_dag(gamma_graph *g) {
   const uint32_t n = g->n, b = g->bits;
   const uint64_t m = g->m;
   DevBuf<uint32_t> rank_of(ctx, n);
-  const char *off_env = getenv("GAMMA_NO_RANK_DAG");   // ablation: keep the id-space DAG
-  if (off_env && *off_env && *off_env != '0') {
+  // Rank-space relabelling is opt-in (GAMMA_RANK_DAG=1): on C2 it cost 11 ms of build and
+  // 1 ms of kCL time, on heavy it saved 2 ms (B200 r02, profiles/kcl_ab_r02); by default
+  // the DAG keeps vertex ids (rank_of = identity)
+  const char *on_env = getenv("GAMMA_RANK_DAG");
+  if (!(on_env && *on_env && *on_env != '0')) {
     ctx->launch(KC_BUILD, [&] { iota_u32_kernel<<<grid_for(n), kThreads, 0, ctx->stream>>>(rank_of.p, n); });
     g->rank_of = rank_of.release();
     g->device_bytes += (uint64_t)n * 4;
@@ -449,6 +452,7 @@ void rank_dag(gamma_graph *g) {
     });
   }
   g->rank_of = rank_of.release();
+  g->rank_space = true;
   g->device_bytes += (uint64_t)n * 4;
 }
 

@@ -179,6 +179,7 @@ struct gamma_graph {
   uint64_t *dag_ptr = nullptr;   // n+1
   uint32_t *dag_col = nullptr;   // m
   uint32_t *rank_of = nullptr;   // n
+  bool rank_space = false;       // the DAG ids are ranks (GAMMA_RANK_DAG=1), else ids (rank_of = identity)
   // SM filters: label << 24 | min(degree, 2^24 - 1) per vertex, built on the first
   // gamma_match when every label is < 256 (ldeg_state: -1 not yet, 0 unusable, 1 built)
   uint32_t *ldeg = nullptr;

@@ -38,6 +38,11 @@ namespace {
 #endif
 #define GAMMA_BM_BOUNDS(KM) __launch_bounds__(256, (KM) <= 6 ? GAMMA_BM_MINB : 1)
 
+// A/B switches of the bitmap kernels (GAMMA_KCL_ABLATE bits, read per call; 0 = the
+// defaults): 1 per-word leaf walk instead of the balanced one, 2 two-slot hash probe
+// instead of the 4-slot bucket, 4 per-item row search from row 0
+__constant__ uint32_t c_kcl_ablate;
+
 constexpr int kMaxStack = 10;        // DFS levels below the first child: k <= 12
 constexpr uint32_t kPartCost = 4096; // 4-cliques per heavy-root part
 constexpr uint32_t kMaxParts = 4096;
@@ -388,6 +393,11 @@ __device__ __forceinline__ uint32_t group_leaf_sum_bal(const uint32_t *B, uint32
 
 __device__ __forceinline__ uint32_t group_leaf_sum(const uint32_t *B, uint32_t BS, uint32_t W, uint32_t curw,
                                                    const LaneGroup &g) {
+  if (c_kcl_ablate & 1u) {
+    if (W <= 4) return group_leaf_sum_w<4>(B, BS, W, curw, g);
+    if (W <= 8) return group_leaf_sum_w<8>(B, BS, W, curw, g);
+    return group_leaf_sum_w<kGroup>(B, BS, W, curw, g);
+  }
   if (W <= 4) return group_leaf_sum_bal<4>(B, BS, W, curw, g);
   if (W <= 8) return group_leaf_sum_bal<8>(B, BS, W, curw, g);
   return group_leaf_sum_bal<kGroup>(B, BS, W, curw, g);
@@ -439,6 +449,7 @@ __device__ __forceinline__ uint64_t gdfs_count(const uint32_t *B, uint32_t BS, u
 // (the per-item binary search from row 0 was ~12 % of the CTA-team kernel's
 // instructions, ncu heavy r02).
 __device__ __forceinline__ uint32_t advance_row(const uint32_t *P, uint32_t L, uint32_t q, uint32_t j1) {
+  if (c_kcl_ablate & 4u) j1 = 0;
 #pragma unroll
   for (int s = 0; s < 4; s++)
     if (j1 + 1 < L && P[j1 + 1] <= q) j1++;
@@ -543,7 +554,7 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
     const uint32_t x = R[i];
     uint32_t h = (x * 0x9E3779B1u) >> (32 - hbits);
     if (Hv) {
-      h &= ~3u;   // probing starts at a 4-slot bucket: a lookup reads the bucket in one load
+      h &= (c_kcl_ablate & 2u) ? ~1u : ~3u;   // probing starts at a 4-slot bucket: a lookup reads it in one load
       while (atomicCAS(&Hv[h], kEmptyId, x) != kEmptyId) h = (h + 1) & hmask;
       H[h] = (unsigned short)i;
     } else {
@@ -625,10 +636,29 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
           // <= 1/4: the pair-slot probe this replaced sent 87 % of warps into the chain
           // loop, ncu heavy r02) continues the linear probe
           const bool inr = yy >= rmin && yy <= rmax;   // (the padding 0xffffffff is above every rmax < n)
+          bool hit;
+          uint32_t hh;
+          if (c_kcl_ablate & 2u) {   // r01: two-slot pair probe
+            const uint32_t h0 = ((yy * 0x9E3779B1u) >> (32 - hbits)) & ~1u;
+            const uint2 vv = *reinterpret_cast<const uint2 *>(Hv + h0);
+            hit = inr && (vv.x == yy || vv.y == yy);
+            hh = vv.x == yy ? h0 : h0 + 1;
+            if (inr && !hit && vv.x != kEmptyId && vv.y != kEmptyId) {
+              for (uint32_t h = (h0 + 2) & hmask;; h = (h + 1) & hmask) {
+                const uint32_t vh = Hv[h];
+                if (vh == yy) {
+                  hit = true;
+                  hh = h;
+                  break;
+                }
+                if (vh == kEmptyId) break;
+              }
+            }
+          } else {
           const uint32_t h0 = ((yy * 0x9E3779B1u) >> (32 - hbits)) & ~3u;
           const uint4 vv = *reinterpret_cast<const uint4 *>(Hv + h0);
-          bool hit = inr && (vv.x == yy || vv.y == yy || vv.z == yy || vv.w == yy);
-          uint32_t hh = vv.x == yy ? h0 : vv.y == yy ? h0 + 1 : vv.z == yy ? h0 + 2 : h0 + 3;
+          hit = inr && (vv.x == yy || vv.y == yy || vv.z == yy || vv.w == yy);
+          hh = vv.x == yy ? h0 : vv.y == yy ? h0 + 1 : vv.z == yy ? h0 + 2 : h0 + 3;
           if (inr && !hit && vv.w != kEmptyId && vv.x != kEmptyId && vv.y != kEmptyId && vv.z != kEmptyId) {
             for (uint32_t h = (h0 + 4) & hmask;; h = (h + 1) & hmask) {
               const uint32_t vh = Hv[h];
@@ -639,6 +669,7 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
               }
               if (vh == kEmptyId) break;
             }
+          }
           }
           if (hit) {
             const uint32_t e = H[hh];
@@ -1292,8 +1323,12 @@ uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint6
   a.multi = multi_out != nullptr;
   a.kmin = std::max<uint32_t>(3, std::min(kmin, k));
   {
+    // the list trim pays only in rank space (ids in degree order); GAMMA_KCL_NO_TRIM off
     const char *e = getenv("GAMMA_KCL_NO_TRIM");
-    a.trim = !(e && *e && *e != '0');
+    a.trim = g->rank_space && !(e && *e && *e != '0');
+    const char *ab = getenv("GAMMA_KCL_ABLATE");
+    const uint32_t abl = ab && *ab ? (uint32_t)strtoul(ab, nullptr, 10) : 0u;
+    GAMMA_CUDA(cudaMemcpyToSymbolAsync(c_kcl_ablate, &abl, sizeof(abl), 0, cudaMemcpyHostToDevice, ctx->stream));
   }
   // hub splitting only pays when the DFS below a triangle is deep (k >= 6)
   // (GAMMA_KCL_SPLIT_MINK: the smallest k that splits, default 6)
