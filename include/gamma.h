@@ -97,6 +97,9 @@ typedef struct {
                                           sort instead of the global key sort (2m' < 2^31
                                           only; same CSR; slower on hub-heavy graphs, where
                                           the hub rows fall to CUB's large-segment kernel) */
+#define GAMMA_FLAG_TWO_PASS     0x200u /* kCL ET path, ablation of Opt 1: each
+                                          extension counts its output, scans, then writes at
+                                          exact offsets (twice the intersections, no blocks)  */
 #define GAMMA_FLAG_FPM_INSTANCES 0x100u /* gamma_fpm: also count each pattern's instances
                                           (connected edge sets mapped to it; one atomic
                                           per embedding -- a parity check, not for timing) */

@@ -30,6 +30,7 @@
 //  * A8: DFS over (depth, group range), level buffers grow geometrically up to an
 //    equal share of the HBM budget; a range that still overflows is split in halves.
 #include <cub/device/device_radix_sort.cuh>
+#include <cub/device/device_scan.cuh>
 #include <cub/device/device_select.cuh>
 
 #include <algorithm>
@@ -72,6 +73,13 @@ struct KclArgs {
   uint32_t batch;
   uint32_t stage_cap;         // kRunCap (0: GAMMA_FLAG_DEBUG_NOSTAGE)
   uint32_t root_len_gt;       // depth 1: only roots with |N+(v)| > this (bitmap path took the rest)
+  // Opt 1 ablation (GAMMA_FLAG_TWO_PASS: the count-then-write scheme Opt 1
+  // replaces): pass 1 only counts each input group's output vids / groups into gcnt_v /
+  // gcnt_g; pass 2 writes them at the exclusive-scanned offsets goff_v / goff_g
+  // (indexed by gi - g_begin); 0 = Opt 1's single pass with warp memory blocks
+  uint32_t two_pass;
+  uint32_t *gcnt_v, *gcnt_g;
+  const uint64_t *goff_v, *goff_g;
 };
 
 struct Counters {
@@ -171,7 +179,8 @@ __device__ __forceinline__ uint64_t count_staged(const KclArgs &a, const uint32_
 // memory; EXTEND/FUSED write each kept child's run with a direct pool reservation.
 template <int MODE, bool PER_ROOT>
 __device__ bool process_unstaged(const KclArgs &a, const uint32_t *run, uint32_t len, uint32_t root_idx,
-                                 int lane, Counters &ct, WarpBlock &wg, uint64_t &gacc) {
+                                 int lane, Counters &ct, WarpBlock &wg, uint64_t &gacc, uint64_t gi,
+                                 uint32_t &tp_v, uint32_t &tp_g) {
   const BlockPool pv{&a.ctrl[CTRL_VCUR], &a.ctrl[CTRL_OVF], a.cap_v, kBlkV};
   const BlockPool pg{&a.ctrl[CTRL_GCUR], &a.ctrl[CTRL_OVF], a.cap_g, kBlkG};
   const uint32_t rmin = run[0], rmax = run[len - 1];
@@ -185,16 +194,27 @@ __device__ bool process_unstaged(const KclArgs &a, const uint32_t *run, uint32_t
     const uint32_t *lst = a.dag_col + lb;
     const uint32_t ub = min(dl, len);
     uint64_t pos = 0;
-    if (MODE != MODE_COUNT && !pool_reserve(pv, ub, lane, pos)) return false;
+    const bool tp_write = MODE == MODE_EXTEND && a.two_pass == 2;
+    if (tp_write) pos = a.goff_v[gi - a.g_begin] + tp_v;
+    else if (MODE != MODE_COUNT && !(MODE == MODE_EXTEND && a.two_pass == 1) && !pool_reserve(pv, ub, lane, pos))
+      return false;
+    // write pass of the two-pass ablation: a child's run is written only once its size
+    // says it is kept (its space was counted for kept children only), i.e. counted again
+    const int rounds = tp_write ? 2 : 1;
     uint32_t found = 0;
-    for (uint32_t j = 0; j < dl; j += 32) {
-      const uint32_t y = (j + lane < dl) ? __ldg(lst + j + lane) : 0xffffffffu;
-      bool hit = false;
-      if (y >= rmin && y <= rmax) hit = sorted_contains(run, len, y);
-      const uint32_t bal = __ballot_sync(0xffffffffu, hit);
-      if (MODE != MODE_COUNT && hit) a.vid_out[pos + found + __popc(bal & lanemask_lt())] = y;
-      found += __popc(bal);
-      if (__shfl_sync(0xffffffffu, y, 31) > rmax) break;
+    for (int rd = 0; rd < rounds; rd++) {
+      const bool write = MODE != MODE_COUNT && !(MODE == MODE_EXTEND && a.two_pass == 1) && (!tp_write || rd == 1);
+      if (rd == 1 && found < a.need_child) break;
+      found = 0;
+      for (uint32_t j = 0; j < dl; j += 32) {
+        const uint32_t y = (j + lane < dl) ? __ldg(lst + j + lane) : 0xffffffffu;
+        bool hit = false;
+        if (y >= rmin && y <= rmax) hit = sorted_contains(run, len, y);
+        const uint32_t bal = __ballot_sync(0xffffffffu, hit);
+        if (write && hit) a.vid_out[pos + found + __popc(bal & lanemask_lt())] = y;
+        found += __popc(bal);
+        if (__shfl_sync(0xffffffffu, y, 31) > rmax) break;
+      }
     }
     if (MODE == MODE_COUNT) {
       gacc += found;
@@ -202,7 +222,19 @@ __device__ bool process_unstaged(const KclArgs &a, const uint32_t *run, uint32_t
     }
     if (found < a.need_child) continue;
     uint64_t gpos;
-    if (!wb_reserve(wg, pg, 1, lane, gpos)) return false;
+    if (MODE == MODE_EXTEND && a.two_pass == 1) {
+      tp_v += found;
+      tp_g += 1;
+      ct.out_entries += (lane == 0) ? found : 0;
+      continue;
+    }
+    if (tp_write) {
+      gpos = a.goff_g[gi - a.g_begin] + tp_g;
+      tp_v += found;
+      tp_g += 1;
+    } else if (!wb_reserve(wg, pg, 1, lane, gpos)) {
+      return false;
+    }
     if (lane == 0) {
       a.grp_out[gpos] = make_uint2((uint32_t)pos, found);
       if (PER_ROOT) a.groot_out[gpos] = root_idx;
@@ -250,12 +282,15 @@ __global__ void __launch_bounds__(kThreads) kcl_kernel(KclArgs a) {
         run = a.vid_in + gd.x;
         if (PER_ROOT) root_idx = a.groot_in[gi];
       }
-      if (len < a.need_group) continue;
-      if (ROOT && len <= a.root_len_gt) continue;
+      if (len < a.need_group || (ROOT && len <= a.root_len_gt)) {
+        if (MODE == MODE_EXTEND && a.two_pass == 1 && lane == 0) a.gcnt_v[gi - a.g_begin] = a.gcnt_g[gi - a.g_begin] = 0;
+        continue;
+      }
       ct.in_entries += (lane == 0) ? len : 0;
       uint64_t gacc = 0;
+      uint32_t tp_v = 0, tp_g = 0;   // two-pass ablation: this group's output so far
       if (len > a.stage_cap) {
-        if (!process_unstaged<MODE, PER_ROOT>(a, run, len, root_idx, lane, ct, wg, gacc)) stop = true;
+        if (!process_unstaged<MODE, PER_ROOT>(a, run, len, root_idx, lane, ct, wg, gacc, gi, tp_v, tp_g)) stop = true;
       } else {
         for (uint32_t i = lane; i < len; i += 32) srun[i] = run[i];
         __syncwarp();
@@ -285,12 +320,23 @@ __global__ void __launch_bounds__(kThreads) kcl_kernel(KclArgs a) {
             const bool keep = active && cnt >= a.need_child;
             const uint32_t kbal = __ballot_sync(0xffffffffu, keep);
             if (MODE == MODE_EXTEND) {
-              if (kbal) {
+              if (kbal && a.two_pass == 1) {   // count pass: sizes only
+                tp_v += found;
+                tp_g += __popc(kbal);
+                ct.out_entries += (lane == 0) ? found : 0;
+              } else if (kbal) {
                 uint64_t pos = 0, gpos = 0;
+                if (a.two_pass == 2) {   // write pass: exact offsets from the count pass
+                  pos = a.goff_v[gi - a.g_begin] + tp_v;
+                  gpos = a.goff_g[gi - a.g_begin] + tp_g;
+                  tp_v += found;
+                  tp_g += __popc(kbal);
+                } else {
                 wb_retire_tail(wg, __popc(kbal), lane, [&](uint64_t s) { a.grp_out[s] = make_uint2(0, 0); });
                 if (!wb_reserve(wv, pv, found, lane, pos) || !wb_reserve(wg, pg, __popc(kbal), lane, gpos)) {
                   stop = true;
                   break;
+                }
                 }
                 for (uint32_t t = lane; t < found; t += 32) a.vid_out[pos + t] = sout[t];
                 if (keep) {
@@ -318,6 +364,10 @@ __global__ void __launch_bounds__(kThreads) kcl_kernel(KclArgs a) {
       }
       ct.acc += gacc;
       if (PER_ROOT && lane == 0 && gacc) atomicAdd(&a.per_root[root_idx], (unsigned long long)gacc);
+      if (MODE == MODE_EXTEND && a.two_pass == 1 && lane == 0) {
+        a.gcnt_v[gi - a.g_begin] = tp_v;
+        a.gcnt_g[gi - a.g_begin] = tp_g;
+      }
     }
   }
   // unused group slots of this warp's last block become empty groups
@@ -533,6 +583,10 @@ struct KclRun {
     }
     const bool fused = fuse && d == k - 3;
     const uint32_t nd = d + 1;
+    if (!fused && (ctx->desc.flags & GAMMA_FLAG_TWO_PASS)) {
+      process_two_pass(d, g0, g1);
+      return;
+    }
     for (;;) {
       Level &L = levels[nd];
       if (L.cap_v == 0)
@@ -568,6 +622,61 @@ struct KclRun {
       process(d, mid, g1);
       return;
     }
+  }
+
+  // Opt 1 ablation (GAMMA_FLAG_TWO_PASS): the count-then-write extension that Opt 1's
+  // warp memory blocks replace ("two-pass ... doubles the extension").
+  // Pass 1 counts every input group's output, an exclusive scan gives exact offsets,
+  // pass 2 recomputes the intersections and writes; no over-allocation, twice the work.
+  void process_two_pass(uint32_t d, uint64_t g0, uint64_t g1) {
+    const uint32_t nd = d + 1;
+    const uint64_t ng_in = g1 - g0;
+    Level &L = levels[nd];
+    if (L.cap_v == 0) grow_level(nd, std::max<uint64_t>(1ull << 24, 4ull * kBlkV * kWarps * (uint64_t)grid[MODE_EXTEND]));
+    DevBuf<uint32_t> cv(ctx, ng_in + 1), cg(ctx, ng_in + 1);
+    DevBuf<uint64_t> ov(ctx, ng_in + 1), og(ctx, ng_in + 1);
+    GAMMA_CUDA(cudaMemsetAsync(cv.p + ng_in, 0, 4, ctx->stream));
+    GAMMA_CUDA(cudaMemsetAsync(cg.p + ng_in, 0, 4, ctx->stream));
+    KclArgs a = args_for(d, g0, g1);
+    set_output(a, nd);
+    a.two_pass = 1;
+    a.gcnt_v = cv.p;
+    a.gcnt_g = cg.p;
+    launch<MODE_EXTEND>(a, d, L.cap_v);
+    account(KC_EXTEND, d, ctx->ctrl_host, true);
+    size_t tmp = 0;
+    GAMMA_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tmp, cv.p, ov.p, (int64_t)ng_in + 1, ctx->stream));
+    {
+      DevBuf<uint8_t> t(ctx, tmp);
+      ctx->launch(KC_MISC, [&] {
+        GAMMA_CUDA(cub::DeviceScan::ExclusiveSum(t.p, tmp, cv.p, ov.p, (int64_t)ng_in + 1, ctx->stream));
+      });
+      ctx->launch(KC_MISC, [&] {
+        GAMMA_CUDA(cub::DeviceScan::ExclusiveSum(t.p, tmp, cg.p, og.p, (int64_t)ng_in + 1, ctx->stream));
+      });
+    }
+    uint64_t tot[2];
+    GAMMA_CUDA(cudaMemcpyAsync(&tot[0], ov.p + ng_in, 8, cudaMemcpyDeviceToHost, ctx->stream));
+    GAMMA_CUDA(cudaMemcpyAsync(&tot[1], og.p + ng_in, 8, cudaMemcpyDeviceToHost, ctx->stream));
+    ctx->sync();
+    // exact sizes: grow once, or split the range when even the largest level share cannot hold them
+    if (tot[0] > L.cap_v || tot[1] > L.cap_g) grow_level(nd, std::max<uint64_t>(tot[0], 2 * tot[1]));
+    if (tot[0] > L.cap_v || tot[1] > L.cap_g) {
+      GAMMA_REQUIRE(ng_in > 1, GAMMA_E_NOMEM, "HBM budget too small for the children of a single embedding group");
+      ctx->stats.retries++;
+      const uint64_t mid = g0 + ng_in / 2;
+      process_two_pass(d, g0, mid);
+      process_two_pass(d, mid, g1);
+      return;
+    }
+    a.two_pass = 2;
+    a.goff_v = ov.p;
+    a.goff_g = og.p;
+    set_output(a, nd);
+    launch<MODE_EXTEND>(a, d, L.cap_v);
+    ctx->stats.chunks++;
+    ctx->stats.level_entries[nd + 1] += ctx->ctrl_host[CTRL_ENTRIES];
+    process(nd, 0, tot[1]);
   }
 
   // GAMMA_FLAG_SPILL: BFS with a host-resident next level (the ET "should

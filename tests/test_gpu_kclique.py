@@ -269,7 +269,7 @@ def test_wide_runs_closed_forms(ctx):
     assert g.kclique(3) == comb(8194, 3)
 
 
-@pytest.mark.parametrize("flags", [0, 0x10, 0x2 | 0x10, 0x20, 0x40])
+@pytest.mark.parametrize("flags", [0, 0x10, 0x2 | 0x10, 0x20, 0x40, 0x200 | 0x10, 0x200 | 0x10 | 0x2])
 def test_paths_agree(G, oracle_mod, flags):
     """Bitmap DFS (default), ET levels with the fused tail (NO_BITMAP), ET levels
     with every level materialised (NO_FUSE | NO_BITMAP), the bitmap path without hub

@@ -7,6 +7,8 @@ Variants of the same extension primitive, selected by ctx flags (include/gamma.h
        et_fused     list-based ET (Opt 1 per-warp blocks + Opt 2 grouping), last two
                     levels fused in shared memory              (GAMMA_FLAG_NO_BITMAP)
        et_levels    list-based ET, every level materialised    (NO_BITMAP | NO_FUSE)
+       et_two_pass  ... with the naive count-then-write extension instead of Opt 1's
+                    warp memory blocks (NO_BITMAP | NO_FUSE | TWO_PASS)
   SM   default      grouped extension, L_m staged once per group (Opt 2)
        no_group     L_m never staged: every child intersects all backward lists
                     (GAMMA_FLAG_DEBUG_NOSTAGE)
@@ -31,7 +33,7 @@ import torch  # noqa: E402
 import gamma_gen as gg  # noqa: E402
 import paper_conf_icde_hu0o23_b200 as G  # noqa: E402
 
-KCL = {"default": 0, "no_split": 0x20, "et_fused": 0x10, "et_levels": 0x10 | 0x2}
+KCL = {"default": 0, "no_split": 0x20, "et_fused": 0x10, "et_levels": 0x10 | 0x2, "et_two_pass": 0x10 | 0x2 | 0x200}
 SM = {"default": 0, "no_group": 0x8}
 
 
