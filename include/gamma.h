@@ -100,6 +100,10 @@ typedef struct {
 #define GAMMA_FLAG_TWO_PASS     0x200u /* kCL ET path, ablation of Opt 1: each
                                           extension counts its output, scans, then writes at
                                           exact offsets (twice the intersections, no blocks)  */
+#define GAMMA_FLAG_SM_EDGE_JOIN 0x400u /* gamma_match by edge extension ("binary join",
+                                          PAPER.md L141, L170): one pattern edge per ET step,
+                                          non-tree edges as separate filter passes; same
+                                          count, larger intermediate tables (ablation)   */
 #define GAMMA_FLAG_FPM_INSTANCES 0x100u /* gamma_fpm: also count each pattern's instances
                                           (connected edge sets mapped to it; one atomic
                                           per embedding -- a parity check, not for timing) */

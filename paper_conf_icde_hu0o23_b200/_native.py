@@ -28,6 +28,7 @@ GAMMA_FLAG_DEBUG_SPLIT_ALL = 0x40
 GAMMA_FLAG_COUNT_SORT_BUILD = 0x80
 GAMMA_FLAG_FPM_INSTANCES = 0x100
 GAMMA_FLAG_TWO_PASS = 0x200
+GAMMA_FLAG_SM_EDGE_JOIN = 0x400
 
 ALLOC_FN = C.CFUNCTYPE(C.c_void_p, C.c_size_t, C.c_void_p, C.c_void_p)
 FREE_FN = C.CFUNCTYPE(None, C.c_void_p, C.c_void_p)

@@ -166,6 +166,24 @@ __device__ __forceinline__ Bounds bounds_for(const SmArgs &a, uint32_t q, uint32
   return b;
 }
 
+// bounds_for over a plan (the join kernels have no SmArgs)
+__device__ __forceinline__ Bounds bounds_for_join(const SmPlan &P, uint32_t q, uint32_t avail, const uint32_t *phi) {
+  Bounds b{-1, 0xffffffffu, 0u, 0u};
+  uint32_t m = P.ltmask[q] & avail;
+  while (m) {
+    const int j = __ffs(m) - 1;
+    m &= m - 1;
+    b.lo = max(b.lo, (int64_t)phi[j]);
+  }
+  m = P.gtmask[q] & avail;
+  while (m) {
+    const int j = __ffs(m) - 1;
+    m &= m - 1;
+    b.hi = min(b.hi, phi[j]);
+  }
+  return b;
+}
+
 // Intersect the lists N(phi_j), j in `lists`, with filters; results (sorted) go to
 // out[] (if WRITE and they fit in cap) or are only counted.  The shortest list
 // drives; the others are probed by binary search.  Returns the number of results,
@@ -957,6 +975,237 @@ static void ensure_ldeg(gamma_graph *g) {
   g->ldeg_state = 1;
 }
 
+// ---- SM by edge extension ("binary join"):
+// the embedding table grows by ONE pattern edge per step instead of one vertex with all
+// its backward edges at once (Alg. 1's vertex extension, the path above): a tree edge
+// (the position's first backward neighbour b0) expands every row by the candidates in
+// N(phi(b0)) (label, degree, injectivity and symmetry-order filters), and every further
+// backward edge -- and, induced, every anti-edge -- is a separate pass that keeps the
+// rows whose pair is (resp. is not) adjacent.  Same constraints, same count; the
+// intermediate tables are what the vertex extension avoids (the ablation's point).
+// Rows are phi_0..phi_t (t+1 u32, row-major); root ranges are halved on overflow.
+struct JoinArgs {
+  const uint64_t *rp;
+  const uint32_t *col;
+  const uint32_t *ldeg;   // label << 24 | degree (nullable: labels / degrees gathered separately)
+  const uint32_t *lab;
+  SmPlan P;
+  const uint32_t *in;
+  uint64_t n_in;
+  uint32_t w_in;          // words per input row (= positions placed)
+  uint32_t *out;
+  uint64_t cap;           // output rows
+  unsigned long long *cursor, *ovf, *count;
+  uint32_t q;             // expand: the position being placed; check: its later endpoint
+  uint32_t b;             // expand: b0; check: the earlier endpoint
+  uint32_t anti;          // check: keep rows whose pair is NOT adjacent
+  uint32_t count_only;    // last step: count, do not write
+};
+
+// one warp per input row: lanes stream N(phi(b0)), survivors are compacted and appended
+__global__ void __launch_bounds__(256) sm_join_expand(JoinArgs a) {
+  const int lane = threadIdx.x & 31;
+  const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  const uint32_t q = a.q, placed = (1u << q) - 1u;
+  const bool last = q + 1 == a.P.nv;
+  unsigned long long cnt = 0;
+  for (uint64_t r = warp; r < a.n_in; r += nw) {
+    if (!a.count_only && *(volatile unsigned long long *)a.ovf) break;
+    const uint32_t *row = a.in + r * a.w_in;
+    uint32_t phi[kMaxV];
+#pragma unroll
+    for (int j = 0; j < kMaxV; j++) phi[j] = j < (int)a.w_in ? row[j] : 0u;
+    const Bounds bd = bounds_for_join(a.P, q, placed, phi);
+    const uint64_t s0 = a.rp[phi[a.b]];
+    const uint32_t dl = (uint32_t)(a.rp[phi[a.b] + 1] - s0);
+    for (uint32_t j0 = 0; j0 < dl; j0 += 32) {
+      const uint32_t jj = j0 + lane;
+      const uint32_t x = jj < dl ? a.col[s0 + jj] : 0xffffffffu;
+      bool ok = jj < dl && (int64_t)x > bd.lo && x < bd.hi;
+      if (ok && (a.P.labeled || (!last && a.P.mindeg[q] > 1))) {
+        uint32_t lx, dx;
+        if (a.ldeg) {
+          const uint32_t ld = a.ldeg[x];
+          lx = ld >> 24;
+          dx = ld & 0xffffffu;
+        } else {
+          lx = a.lab ? a.lab[x] : 0u;
+          dx = (uint32_t)(a.rp[x + 1] - a.rp[x]);
+        }
+        ok = (!a.P.labeled || lx == a.P.label[q]) && (last || dx >= a.P.mindeg[q]);
+      }
+#pragma unroll
+      for (int j = 0; j < kMaxV; j++)
+        if (ok && j < (int)q && phi[j] == x) ok = false;   // injective against every placed position
+      const uint32_t bal = __ballot_sync(0xffffffffu, ok);
+      if (!bal) continue;
+      if (a.count_only) {
+        cnt += (lane == 0) ? __popc(bal) : 0;
+        continue;
+      }
+      unsigned long long base = 0;
+      if (lane == 0) base = atomicAdd(a.cursor, (unsigned long long)__popc(bal));
+      base = __shfl_sync(0xffffffffu, base, 0);
+      if (base + __popc(bal) > a.cap) {
+        if (lane == 0) atomicExch(a.ovf, 1ull);
+        break;
+      }
+      if (ok) {
+        uint32_t *o = a.out + (base + __popc(bal & lanemask_lt())) * (a.w_in + 1);
+        for (uint32_t j = 0; j < a.w_in; j++) o[j] = phi[j];
+        o[a.w_in] = x;
+      }
+    }
+  }
+  if (a.count_only) {
+    for (int off = 16; off > 0; off >>= 1) cnt += __shfl_down_sync(0xffffffffu, cnt, off);
+    if (lane == 0 && cnt) atomicAdd(a.count, cnt);
+  }
+}
+
+// one thread per row: keep it iff phi(b) ~ phi(q) (anti: iff not); warp-aggregated append
+__global__ void __launch_bounds__(256) sm_join_check(JoinArgs a) {
+  const int lane = threadIdx.x & 31;
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  unsigned long long cnt = 0;
+  for (uint64_t r0 = blockIdx.x * (uint64_t)blockDim.x; r0 < a.n_in; r0 += stride) {
+    const uint64_t r = r0 + threadIdx.x;
+    bool ok = false;
+    if (r < a.n_in) {
+      const uint32_t *row = a.in + r * a.w_in;
+      const uint32_t u = row[a.b], x = row[a.q];
+      const uint64_t s0 = a.rp[u];
+      const uint32_t dl = (uint32_t)(a.rp[u + 1] - s0);
+      ok = (dl && sorted_contains(a.col + s0, dl, x)) != (a.anti != 0);
+    }
+    const uint32_t bal = __ballot_sync(0xffffffffu, ok);
+    if (a.count_only) {
+      cnt += (lane == 0) ? __popc(bal) : 0;
+      continue;
+    }
+    if (!bal) continue;
+    unsigned long long base = 0;
+    if (lane == 0) base = atomicAdd(a.cursor, (unsigned long long)__popc(bal));
+    base = __shfl_sync(0xffffffffu, base, 0);
+    if (base + __popc(bal) > a.cap) {   // cannot happen (a filter shrinks), kept for safety
+      if (lane == 0) atomicExch(a.ovf, 1ull);
+      break;
+    }
+    if (ok) {
+      const uint32_t *row = a.in + r * a.w_in;
+      uint32_t *o = a.out + (base + __popc(bal & lanemask_lt())) * a.w_in;
+      for (uint32_t j = 0; j < a.w_in; j++) o[j] = row[j];
+    }
+  }
+  if (a.count_only) {
+    for (int off = 16; off > 0; off >>= 1) cnt += __shfl_down_sync(0xffffffffu, cnt, off);
+    if (lane == 0 && cnt) atomicAdd(a.count, cnt);
+  }
+}
+
+struct JoinStep {
+  uint32_t kind;   // 0 expand, 1 check, 2 anti-check
+  uint32_t q, b;
+};
+
+static std::vector<JoinStep> join_steps(const SmPlan &P) {
+  std::vector<JoinStep> st;
+  for (uint32_t q = 1; q < P.nv; q++) {
+    const uint32_t b0 = (uint32_t)__builtin_ctz(P.bmask[q]);
+    st.push_back({0, q, b0});
+    for (uint32_t m = P.bmask[q] & ~(1u << b0); m; m &= m - 1) st.push_back({1, q, (uint32_t)__builtin_ctz(m)});
+    for (uint32_t m = P.antimask[q]; m; m &= m - 1) st.push_back({2, q, (uint32_t)__builtin_ctz(m)});
+  }
+  return st;
+}
+
+static uint64_t match_join(gamma_graph *g, const SmPlan &P, const uint32_t *roots, uint64_t nr,
+                           uint64_t level_share) {
+  gamma_ctx *ctx = g->ctx;
+  const std::vector<JoinStep> steps = join_steps(P);
+  const uint64_t cap = std::max<uint64_t>(1 << 16, level_share / 2 / (4ull * P.nv));   // rows per buffer
+  DevBuf<uint32_t> bufA(ctx, cap * P.nv), bufB(ctx, cap * P.nv);
+  DevBuf<unsigned long long> cur(ctx, 3);   // cursor, overflow, count
+  uint64_t total = 0;
+  std::vector<std::pair<uint64_t, uint64_t>> todo;
+  for (uint64_t r0 = nr; r0 > 0;) {   // chunks of <= cap roots, processed in root order
+    const uint64_t r1 = r0 > cap ? r0 - cap : 0;
+    todo.push_back({r1, r0});
+    r0 = r1;
+  }
+  while (!todo.empty()) {
+    const auto rg = todo.back();
+    todo.pop_back();
+    // the chunk's roots as 1-word rows
+    GAMMA_REQUIRE(rg.second - rg.first <= cap, GAMMA_E_NOMEM, "edge join: root chunk exceeds the row buffer");
+    GAMMA_CUDA(cudaMemcpyAsync(bufA.p, roots + rg.first, (rg.second - rg.first) * 4, cudaMemcpyDeviceToDevice,
+                               ctx->stream));
+    uint32_t *in = bufA.p, *out = bufB.p;
+    uint64_t n_in = rg.second - rg.first;
+    uint32_t w = 1;
+    bool ovf = false;
+    uint64_t chunk_count = 0;
+    for (size_t i = 0; i < steps.size() && n_in; i++) {
+      const JoinStep &stp = steps[i];
+      JoinArgs a{};
+      a.rp = g->row_ptr;
+      a.col = g->col;
+      a.ldeg = g->ldeg;
+      a.lab = g->labels;
+      a.P = P;
+      a.in = in;
+      a.n_in = n_in;
+      a.w_in = w;
+      a.out = out;
+      a.cap = cap;
+      a.cursor = cur.p;
+      a.ovf = cur.p + 1;
+      a.count = cur.p + 2;
+      a.q = stp.q;
+      a.b = stp.b;
+      a.anti = stp.kind == 2;
+      a.count_only = i + 1 == steps.size();
+      GAMMA_CUDA(cudaMemsetAsync(cur.p, 0, 24, ctx->stream));
+      const bool last = a.count_only;
+      const int kc = last ? KC_SM_COUNT : KC_SM_EXTEND;
+      if (stp.kind == 0)
+        ctx->launch(kc, [&] { sm_join_expand<<<g1d(n_in * 32), 256, 0, ctx->stream>>>(a); });
+      else
+        ctx->launch(kc, [&] { sm_join_check<<<g1d(n_in), 256, 0, ctx->stream>>>(a); });
+      uint64_t h[3];
+      GAMMA_CUDA(cudaMemcpyAsync(h, cur.p, 24, cudaMemcpyDeviceToHost, ctx->stream));
+      ctx->sync();
+      if (h[1]) {
+        ovf = true;
+        break;
+      }
+      if (last) {
+        chunk_count = h[2];
+        break;
+      }
+      n_in = h[0];
+      if (stp.kind == 0) w++;
+      std::swap(in, out);
+      ctx->stats.level_entries[w] += stp.kind == 0 ? n_in : 0;
+    }
+    if (ovf) {
+      ctx->stats.retries++;
+      GAMMA_REQUIRE(rg.second - rg.first > 1, GAMMA_E_NOMEM, "edge join: one root's rows exceed the buffer");
+      const uint64_t mid = rg.first + (rg.second - rg.first) / 2;
+      todo.push_back({mid, rg.second});
+      todo.push_back({rg.first, mid});
+      continue;
+    }
+    ctx->stats.chunks++;
+    total = checked_add(total, chunk_count);
+  }
+  ctx->stats.level_entries[P.nv] = total;
+  ctx->sync();
+  ctx->collect_timings();
+  return total;
+}
+
 static uint64_t match_count(gamma_graph *g, const SmPlan &P) {
   gamma_ctx *ctx = g->ctx;
   ensure_ldeg(g);
@@ -1039,6 +1288,7 @@ static uint64_t match_count(gamma_graph *g, const SmPlan &P) {
   }
   ctx->stats.level_entries[1] = nr;
   if (nr == 0) return 0;
+  if (ctx->desc.flags & GAMMA_FLAG_SM_EDGE_JOIN) return match_join(g, P, roots.p, nr, R.level_share);
   const uint64_t ngr = (nr + kRootChunk - 1) / kRootChunk;
   SmLevel &L0 = R.lv[0];
   L0.desc = DevBuf<uint32_t>(ctx, 2 * ngr);
