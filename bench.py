@@ -396,9 +396,10 @@ def run_gamma(args):
                     collect()
             emb = sum(results.values())
         else:
-            pats = g.fpm(w["l"], w["minsup"])
+            pats = g.fpm_array(w["l"], w["minsup"])   # the result records, no per-pattern Python objects
             st = collect() if coll else ctx.stats()
-            results = {f"frequent_l{l}": sum(1 for p in pats if p[0] == l) for l in range(1, w["l"] + 1)}
+            per = np.bincount(pats["ne"], minlength=w["l"] + 1) if len(pats) else np.zeros(w["l"] + 1, int)
+            results = {f"frequent_l{l}": int(per[l]) for l in range(1, w["l"] + 1)}
             emb = st["level_entries"][w["l"]]
             results["embeddings_per_level"] = st["level_entries"][1:w["l"] + 1]
             results["embeddings_l"] = emb

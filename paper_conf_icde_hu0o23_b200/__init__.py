@@ -358,10 +358,10 @@ class Graph:
             raise ValueError("motifs: k must be 3 or 4")
         return {name: self.match(k, e, induced=True)[0] for name, e in MOTIFS[k].items()}
 
-    def fpm(self, max_edges: int, minsup: int, instances: bool = False):
-        """Frequent patterns: sorted list of (ne, nv, labels, edges, support); with
-        ``instances`` (needs a Context created with GAMMA_FLAG_FPM_INSTANCES) each
-        tuple also carries the pattern's instance count (connected edge sets)."""
+    def fpm_array(self, max_edges: int, minsup: int) -> np.ndarray:
+        """Frequent patterns as a numpy structured array (fields nv, ne, labels[8],
+        edges[8][2], support, instances), one record per pattern in the library's order --
+        one copy of the result, no per-pattern Python objects."""
         t = self.ctx._torch
         if t is not None and t.cuda.is_available():
             # the MNI domain pool is sized from free HBM: return the context's kept
@@ -372,13 +372,27 @@ class Graph:
         r = C.POINTER(N.gamma_fpm_result)()
         _check(_lib.gamma_fpm(self._h, int(max_edges), int(minsup), C.byref(r)), "gamma_fpm")
         try:
-            out = []
             res = r.contents
-            for i in range(res.n):
-                pt = res.pats[i]
-                out.append((int(pt.ne), int(pt.nv), tuple(int(pt.labels[j]) for j in range(pt.nv)),
-                            tuple((int(pt.edges[e][0]), int(pt.edges[e][1])) for e in range(pt.ne)),
-                            int(pt.support)) + ((int(pt.instances),) if instances else ()))
-            return out
+            dt = np.dtype([("nv", np.uint32), ("ne", np.uint32), ("labels", np.uint32, 8),
+                           ("edges", np.uint8, (8, 2)), ("support", np.uint64), ("instances", np.uint64)],
+                          align=True)
+            assert dt.itemsize == C.sizeof(N.gamma_fpm_pattern)
+            if res.n == 0:
+                return np.zeros(0, dt)
+            buf = (C.c_char * (res.n * dt.itemsize)).from_address(C.addressof(res.pats.contents))
+            return np.frombuffer(buf, dtype=dt).copy()
         finally:
             _lib.gamma_fpm_result_free(r)
+
+    def fpm(self, max_edges: int, minsup: int, instances: bool = False):
+        """Frequent patterns: sorted list of (ne, nv, labels, edges, support); with
+        ``instances`` (needs a Context created with GAMMA_FLAG_FPM_INSTANCES) each
+        tuple also carries the pattern's instance count (connected edge sets)."""
+        arr = self.fpm_array(max_edges, minsup)
+        out = []
+        for pt in arr:
+            nv, ne = int(pt["nv"]), int(pt["ne"])
+            out.append((ne, nv, tuple(int(x) for x in pt["labels"][:nv]),
+                        tuple((int(pt["edges"][e][0]), int(pt["edges"][e][1])) for e in range(ne)),
+                        int(pt["support"])) + ((int(pt["instances"]),) if instances else ()))
+        return out

@@ -482,6 +482,22 @@ __global__ void fpm_support_kernel(FpmArgs a, uint32_t level, uint64_t minsup) {
   }
 }
 
+// frequent slots -> compact (key, support, instances) arrays; dist_level: slots of this
+// level come from the distributed path instead (skipped)
+__global__ void collect_kernel(const unsigned long long *slots, const unsigned long long *sup, const uint32_t *freq,
+                               const unsigned long long *inst, uint64_t cap, uint32_t dist_level,
+                               unsigned long long *ok, unsigned long long *os, unsigned long long *oi,
+                               unsigned long long *cursor) {
+  for (uint64_t s = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; s < cap; s += (uint64_t)gridDim.x * blockDim.x) {
+    const unsigned long long k = slots[2 * s];
+    if (k == 0 || !freq[s] || (dist_level && key_ne(k) == dist_level)) continue;
+    const unsigned long long i = atomicAdd(cursor, 1ull);
+    ok[i] = k;
+    os[i] = sup[s];
+    if (inst) oi[i] = inst[s];
+  }
+}
+
 __global__ void label_hist_kernel(const uint32_t *lab, uint32_t n, uint32_t *csize, uint32_t *lrank_tmp) {
   for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x)
     atomicAdd(&csize[lab ? lab[v] : 0u], 1u);
@@ -1480,32 +1496,43 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
     count_fpm_bytes(ctx);
   }
   plog.mark("level 4 / pool free");
-  // ---- collect the frequent patterns ----
-  std::vector<uint32_t> hfreq(cap);
-  std::vector<unsigned long long> hkey, hsup(cap), hinst(want_inst ? cap : 0);
-  GAMMA_CUDA(cudaMemcpyAsync(hfreq.data(), freq.p, cap * 4, cudaMemcpyDeviceToHost, ctx->stream));
-  if (want_inst) GAMMA_CUDA(cudaMemcpyAsync(hinst.data(), inst.p, cap * 8, cudaMemcpyDeviceToHost, ctx->stream));
-  slots_get(ctx, hkey, slots.p, cap, 0);
-  GAMMA_CUDA(cudaMemcpyAsync(hsup.data(), sup.p, cap * 8, cudaMemcpyDeviceToHost, ctx->stream));
+  // ---- collect the frequent patterns: compacted on the device (only frequent slots
+  // travel), ordered on the host by one packed key per pattern ----
+  uint64_t nf = 0;
+  DevBuf<unsigned long long> ck(ctx, cap), cs(ctx, cap), ci(ctx, want_inst ? cap : 1), ccur(ctx, 1);
+  GAMMA_CUDA(cudaMemsetAsync(ccur.p, 0, 8, ctx->stream));
+  ctx->launch(KC_MISC, [&] {
+    collect_kernel<<<g1d(cap), 256, 0, ctx->stream>>>(slots.p, sup.p, freq.p, want_inst ? inst.p : nullptr, cap,
+                                                       dist ? max_edges : 0u, ck.p, cs.p, ci.p, ccur.p);
+  });
+  GAMMA_CUDA(cudaMemcpyAsync(&nf, ccur.p, 8, cudaMemcpyDeviceToHost, ctx->stream));
   ctx->sync();
-  for (uint64_t s = 0; s < cap; s++) {
-    if (hkey[s] == 0 || !hfreq[s]) continue;
-    if (dist && key_ne(hkey[s]) == max_edges) continue;   // from found_last
-    out.push_back(decode_pattern(hkey[s], hsup[s], want_inst ? hinst[s] : 0));
+  std::vector<unsigned long long> hkey(nf), hsup(nf), hinst(want_inst ? nf : 0);
+  if (nf) {
+    GAMMA_CUDA(cudaMemcpyAsync(hkey.data(), ck.p, nf * 8, cudaMemcpyDeviceToHost, ctx->stream));
+    GAMMA_CUDA(cudaMemcpyAsync(hsup.data(), cs.p, nf * 8, cudaMemcpyDeviceToHost, ctx->stream));
+    if (want_inst) GAMMA_CUDA(cudaMemcpyAsync(hinst.data(), ci.p, nf * 8, cudaMemcpyDeviceToHost, ctx->stream));
+    ctx->sync();
   }
+  for (uint64_t i = 0; i < nf; i++) out.push_back(decode_pattern(hkey[i], hsup[i], want_inst ? hinst[i] : 0));
   out.insert(out.end(), found_last.begin(), found_last.end());
   out.insert(out.end(), found4.begin(), found4.end());
-  std::sort(out.begin(), out.end(), [](const gamma_fpm_pattern &x, const gamma_fpm_pattern &y) {
-    if (x.ne != y.ne) return x.ne < y.ne;
-    if (x.nv != y.nv) return x.nv < y.nv;
-    for (uint32_t i = 0; i < x.nv; i++)
-      if (x.labels[i] != y.labels[i]) return x.labels[i] < y.labels[i];
-    for (uint32_t e = 0; e < x.ne; e++) {
-      if (x.edges[e][0] != y.edges[e][0]) return x.edges[e][0] < y.edges[e][0];
-      if (x.edges[e][1] != y.edges[e][1]) return x.edges[e][1] < y.edges[e][1];
-    }
-    return false;
-  });
+  // sort key: (ne, nv, labels in canonical order, edge pairs) packed in 128 bits
+  std::vector<std::pair<std::pair<uint64_t, uint64_t>, uint32_t>> order(out.size());
+  for (size_t i = 0; i < out.size(); i++) {
+    const gamma_fpm_pattern &x = out[i];
+    uint64_t lab60 = 0;   // five 12-bit labels (labels < 4096), canonical order
+    for (uint32_t j = 0; j < 5; j++) lab60 = lab60 << 12 | (j < x.nv ? x.labels[j] & 0xfffu : 0u);
+    uint64_t ek = 0;      // four edges, 3 + 3 bits each
+    for (uint32_t e = 0; e < 4; e++) ek = ek << 6 | (e < x.ne ? (uint64_t)(x.edges[e][0] << 3 | x.edges[e][1]) : 0u);
+    const uint64_t hi = (uint64_t)x.ne << 61 | (uint64_t)x.nv << 58 | (lab60 >> 2);
+    const uint64_t lo = (lab60 & 3u) << 62 | ek;
+    order[i] = {{hi, lo}, (uint32_t)i};
+  }
+  std::sort(order.begin(), order.end());
+  std::vector<gamma_fpm_pattern> sorted(out.size());
+  for (size_t i = 0; i < out.size(); i++) sorted[i] = out[order[i].second];
+  out.swap(sorted);
   plog.mark("collect + sort");
   ctx->collect_timings();
 }

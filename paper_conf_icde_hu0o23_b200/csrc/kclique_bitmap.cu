@@ -40,7 +40,9 @@ namespace {
 
 // A/B switches of the bitmap kernels (GAMMA_KCL_ABLATE bits, read per call; 0 = the
 // defaults): 1 per-word leaf walk instead of the balanced one, 2 two-slot hash probe
-// instead of the 4-slot bucket, 4 per-item row search from row 0
+// instead of the 4-slot bucket, 4 per-item row search from row 0, 8 every window runs
+// all 4 tiles, 16 multi-k roots down to d+ = 2 (no kmin skip), 32 the hub estimate for
+// every root
 __constant__ uint32_t c_kcl_ablate;
 
 constexpr int kMaxStack = 10;        // DFS levels below the first child: k <= 12
@@ -604,7 +606,7 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
     for (uint32_t t0 = 0; t0 < T; t0 += 32 * kTiles) {
       // tiles that hold elements (warp-uniform): a short window runs 1-3 tiles, not 4
       // (the padded tiles were ~half the row-build instructions on C2's small roots)
-      const uint32_t nt = (T - t0 + 31) >> 5;
+      const uint32_t nt = (c_kcl_ablate & 8u) ? (uint32_t)kTiles : (T - t0 + 31) >> 5;
       uint32_t y[kTiles], rj[kTiles];
 #pragma unroll
       for (int u = 0; u < kTiles; u++) {
@@ -836,7 +838,7 @@ __global__ void GAMMA_BM_BOUNDS(KM) kcl_bitmap_kernel(BmArgs a) {
       bool deferred = false;
       // hub splitting: estimate the DFS by the 4-clique count (skipped when even
       // items x |R| -- an upper bound of it -- is below the cut: most roots)
-      if (a.heavy_cut && (uint64_t)items * L > a.heavy_cut) {
+      if (a.heavy_cut && ((c_kcl_ablate & 32u) || (uint64_t)items * L > a.heavy_cut)) {
         uint64_t est = 0;
         uint32_t jr = 0;
         for (uint32_t q = tid; q < items; q += kTeamThreads) {
