@@ -236,12 +236,13 @@ __device__ __forceinline__ uint32_t pick4(uint32_t i, uint32_t v0, uint32_t v1, 
 // parallelism (ncu c4s20 r02: 40 % of the kernel's stalls waited on these reads one by
 // one): the local vertices' in-class ranks are loaded before the slot lookup returns,
 // and all positions' domain words of one minimizing order are read before any atomic.
-__device__ void record(const FpmArgs &a, const uint2 *tab, const uint32_t *prm, uint32_t v0, uint32_t v1,
-                       uint32_t v2, uint32_t v3, uint32_t l0, uint32_t l1, uint32_t l2, uint32_t l3, uint32_t nv,
+// k0..k3: the in-class ranks (lrank) of the local vertices -- the enumeration loads the
+// root edge's once per edge, a prefix's third once per prefix, only a new fourth vertex
+// per embedding.
+__device__ void record(const FpmArgs &a, const uint2 *tab, const uint32_t *prm, uint32_t k0, uint32_t k1,
+                       uint32_t k2, uint32_t k3, uint32_t l0, uint32_t l1, uint32_t l2, uint32_t l3, uint32_t nv,
                        uint32_t em) {
   const Canon cn = canonical(tab, l0, l1, l2, l3, nv, em);
-  const uint32_t k0 = __ldg(a.lrank + v0), k1 = __ldg(a.lrank + v1);
-  const uint32_t k2 = nv > 2 ? __ldg(a.lrank + v2) : 0u, k3 = nv > 3 ? __ldg(a.lrank + v3) : 0u;
   unsigned long long d = 0;
   const int64_t s = table_slot(a, cn.key, true, d);
   if (s < 0) return;
@@ -337,9 +338,10 @@ __global__ void __launch_bounds__(kThreads) fpm_enum_kernel(FpmArgs a) {
       const uint64_t e1 = ekey(u, v);
       const uint32_t lu = labof(a, u), lv = labof(a, v);
       if (lu < a.walk_lo || lv < a.walk_lo) continue;   // uniform; 0 except in chunk passes
+      const uint32_t ku = __ldg(a.lrank + u), kv = __ldg(a.lrank + v);   // in-class ranks of the root edge
       if (a.level == 1) {
         if (lane == 0) {
-          record(a, s_tab, s_prm, u, v, 0u, 0u, lu, lv, 0u, 0u, 2, 1u << pid(0, 1));
+          record(a, s_tab, s_prm, ku, kv, 0u, 0u, lu, lv, 0u, 0u, 2, 1u << pid(0, 1));
           emb++;
         }
         continue;
@@ -368,7 +370,7 @@ __global__ void __launch_bounds__(kThreads) fpm_enum_kernel(FpmArgs a) {
         }
         if (valid) {
           if (a.level == 2) {
-            record(a, s_tab, s_prm, u, v, y, 0u, lu, lv, ly, 0u, 3, em2);
+            record(a, s_tab, s_prm, ku, kv, __ldg(a.lrank + y), 0u, lu, lv, ly, 0u, 3, em2);
             emb++;
             valid = false;
           } else {
@@ -382,10 +384,11 @@ __global__ void __launch_bounds__(kThreads) fpm_enum_kernel(FpmArgs a) {
         // OR-reduction of the start offsets), so a hub prefix does not serialise on
         // one lane.  N(u), N(v) are the same for every prefix of this e1.
         const uint32_t du = (uint32_t)nu, dv = (uint32_t)(ve - vs);
-        uint32_t by = 0, dy = 0;
+        uint32_t by = 0, dy = 0, ky = 0;
         if (valid) {
           by = (uint32_t)a.rp[y];
           dy = (uint32_t)(a.rp[y + 1] - by);
+          ky = __ldg(a.lrank + y);
         }
         const uint32_t tl = valid ? du + dv + dy : 0u;
         const uint32_t nz = __ballot_sync(0xffffffffu, tl > 0);
@@ -396,6 +399,7 @@ __global__ void __launch_bounds__(kThreads) fpm_enum_kernel(FpmArgs a) {
         const uint32_t cy = __shfl_sync(0xffffffffu, y, src);
         const uint32_t cl = __shfl_sync(0xffffffffu, ly | (em2 << 16), src);
         const uint32_t cby = __shfl_sync(0xffffffffu, by, src);
+        const uint32_t cky = __shfl_sync(0xffffffffu, ky, src);
         const uint32_t stl = __shfl_sync(0xffffffffu, tl, src);
         const uint32_t ctl = lane < (int)nnz ? stl : 0u;
         uint32_t sc = ctl;
@@ -418,6 +422,7 @@ __global__ void __launch_bounds__(kThreads) fpm_enum_kernel(FpmArgs a) {
           const uint32_t py = __shfl_sync(0xffffffffu, cy, j);
           const uint32_t pl = __shfl_sync(0xffffffffu, cl, j);
           const uint32_t pby = __shfl_sync(0xffffffffu, cby, j);
+          const uint32_t pky = __shfl_sync(0xffffffffu, cky, j);
           const uint32_t oj = __shfl_sync(0xffffffffu, ost, j);
           if (t >= T) continue;
           const uint32_t r = t - oj;
@@ -437,7 +442,8 @@ __global__ void __launch_bounds__(kThreads) fpm_enum_kernel(FpmArgs a) {
           const uint32_t em3 = (pl >> 16) | (1u << pid(lw, lz));
           const uint32_t l3 = lz == 3 ? labof(a, z) : 0u;
           if (lz == 3 && l3 < a.walk_lo) continue;
-          record(a, s_tab, s_prm, u, v, py, z, lu, lv, pl & 0xffffu, l3, lz == 3 ? 4 : 3, em3);
+          record(a, s_tab, s_prm, ku, kv, pky, lz == 3 ? __ldg(a.lrank + z) : 0u, lu, lv, pl & 0xffffu, l3,
+                 lz == 3 ? 4 : 3, em3);
           emb++;
         }
       }
