@@ -42,7 +42,7 @@ namespace {
 // defaults): 1 per-word leaf walk instead of the balanced one, 2 two-slot hash probe
 // instead of the 4-slot bucket, 4 per-item row search from row 0, 8 every window runs
 // all 4 tiles, 16 multi-k roots down to d+ = 2 (no kmin skip), 32 the hub estimate for
-// every root
+// every root, 64 short runs stream their lists (no pair probes)
 __constant__ uint32_t c_kcl_ablate;
 
 constexpr int kMaxStack = 10;        // DFS levels below the first child: k <= 12
@@ -541,6 +541,41 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
   constexpr int kTeamThreads = TEAM_WARPS * 32;
   const int wit = tid >> 5;
   const uint32_t W = stride;   // row stride in words (>= the row's (L + 31) / 32 words)
+  // Short runs (warp teams, |R| <= 32, one-word rows): probe the pairs instead of the
+  // lists.  Bit j of row i is R[j] in N+(R[i]): one binary search of R[j] in the child's
+  // sorted list per ordered pair -- |R|(|R|-1) probes where streaming the lists would
+  // probe sum |N+(c)| elements (C2, |R| <= 32: 1.2e8 pairs vs 5.7e8 elements,
+  // scratch/pair_cost.py) -- and no hash table.  The rows of 32 / |R|' consecutive
+  // lanes (|R|' = |R| rounded up to a power of two) are ORed with shuffles.
+  if (TEAM_WARPS == 1 && L <= 32 && !(c_kcl_ablate & 64u)) {
+    if (lane < (int)L) R[lane] = a.dag_col[b0 + lane];
+    __syncwarp();
+    const uint32_t lg = L <= 2 ? 1u : L <= 4 ? 2u : L <= 8 ? 3u : L <= 16 ? 4u : 5u;
+    const uint32_t j = lane & ((1u << lg) - 1u), rows_per = 32u >> lg;
+    const uint32_t rj = j < L ? R[j] : 0u;
+    uint64_t elems = 0;
+    for (uint32_t i0 = 0; i0 < L; i0 += rows_per) {
+      const uint32_t i = i0 + (lane >> lg);
+      bool hit = false;
+      if (i < L) {
+        const uint32_t c = R[i];
+        const uint64_t cb = a.dag_ptr[c];
+        const uint32_t dl = (uint32_t)(a.dag_ptr[c + 1] - cb);
+        if (j == 0) elems += dl;
+        hit = j < L && j != i && dl && sorted_contains(a.dag_col + cb, dl, rj);
+      }
+      uint32_t bits = hit ? 1u << j : 0u;
+      for (uint32_t o = 1; o < (1u << lg); o <<= 1) bits |= __shfl_xor_sync(0xffffffffu, bits, o);
+      if (j == 0 && i < L) {
+        B[i * W] = bits;
+#pragma unroll
+        for (uint32_t w = 1; w < 4; w++)
+          if (w < W) B[i * W + w] = 0u;
+      }
+    }
+    __syncwarp();
+    return elems;
+  }
   uint32_t hbits = 2;
   while ((1u << hbits) < 4 * L) hbits++;
   const uint32_t hmask = (1u << hbits) - 1u;
