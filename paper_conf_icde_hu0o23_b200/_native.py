@@ -9,7 +9,9 @@ import ctypes as C
 import os
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libgamma.so")
+# GAMMA_LIB_VARIANT=<tag>: an in-tree A/B build (build.py tag=...), libgamma_<tag>.so
+LIB_PATH = os.path.join(HERE, f"libgamma_{os.environ['GAMMA_LIB_VARIANT']}.so"
+                        if os.environ.get("GAMMA_LIB_VARIANT") else "libgamma.so")
 
 GAMMA_OK = 0
 GAMMA_E_INVAL = -1

@@ -990,10 +990,6 @@ bool kclique_multi(gamma_graph *g, uint32_t kmin, uint32_t kmax, uint64_t *multi
   GAMMA_REQUIRE(g->m < 0xFFFFFFFFull, GAMMA_E_UNSUPPORTED, "DAG with >= 2^32 edges");
   ensure_root_order(g);
   kmin = std::max<uint32_t>(3, std::min(kmin, kmax));
-  {
-    const char *ab = getenv("GAMMA_KCL_ABLATE");
-    if (ab && *ab && (strtoul(ab, nullptr, 10) & 16u)) kmin = 3;   // A/B: no kmin skip
-  }
   const uint64_t nroots = kmin - 1 < g->root_ge.size() ? g->root_ge[kmin - 1] : 0;   // d+ >= kmin - 1
   ctx->stats.level_entries[1] = nroots;
   for (uint32_t s = 0; s <= kmax; s++) multi_out[s] = 0;

@@ -38,12 +38,20 @@ namespace {
 #endif
 #define GAMMA_BM_BOUNDS(KM) __launch_bounds__(256, (KM) <= 6 ? GAMMA_BM_MINB : 1)
 
-// A/B switches of the bitmap kernels (GAMMA_KCL_ABLATE bits, read per call; 0 = the
-// defaults): 1 per-word leaf walk instead of the balanced one, 2 two-slot hash probe
-// instead of the 4-slot bucket, 4 per-item row search from row 0, 8 every window runs
-// all 4 tiles, 16 multi-k roots down to d+ = 2 (no kmin skip), 32 the hub estimate for
-// every root, 64 short runs stream their lists (no pair probes)
-__constant__ uint32_t c_kcl_ablate;
+// Compile-time variants (A/B builds, build.py tag=...; B200 r02 same-box A/B in
+// profiles/kcl_ab_r02.md): GAMMA_KCL_LEAF_BAL balanced lane-group leaf walk (default:
+// per-word walk -- faster with id-ordered runs, whose bits spread over the words),
+// GAMMA_KCL_BUCKET4 4-slot bucket hash probe (default: slot pair), GAMMA_KCL_NO_PAIRS
+// stream the lists of runs <= 32 too (default: pair probes there)
+#ifndef GAMMA_KCL_LEAF_BAL
+#define GAMMA_KCL_LEAF_BAL 0
+#endif
+#ifndef GAMMA_KCL_BUCKET4
+#define GAMMA_KCL_BUCKET4 0
+#endif
+#ifndef GAMMA_KCL_NO_PAIRS
+#define GAMMA_KCL_NO_PAIRS 0
+#endif
 
 constexpr int kMaxStack = 10;        // DFS levels below the first child: k <= 12
 constexpr uint32_t kPartCost = 4096; // 4-cliques per heavy-root part
@@ -395,7 +403,7 @@ __device__ __forceinline__ uint32_t group_leaf_sum_bal(const uint32_t *B, uint32
 
 __device__ __forceinline__ uint32_t group_leaf_sum(const uint32_t *B, uint32_t BS, uint32_t W, uint32_t curw,
                                                    const LaneGroup &g) {
-  if (c_kcl_ablate & 1u) {
+  if (!GAMMA_KCL_LEAF_BAL) {
     if (W <= 4) return group_leaf_sum_w<4>(B, BS, W, curw, g);
     if (W <= 8) return group_leaf_sum_w<8>(B, BS, W, curw, g);
     return group_leaf_sum_w<kGroup>(B, BS, W, curw, g);
@@ -451,7 +459,6 @@ __device__ __forceinline__ uint64_t gdfs_count(const uint32_t *B, uint32_t BS, u
 // (the per-item binary search from row 0 was ~12 % of the CTA-team kernel's
 // instructions, ncu heavy r02).
 __device__ __forceinline__ uint32_t advance_row(const uint32_t *P, uint32_t L, uint32_t q, uint32_t j1) {
-  if (c_kcl_ablate & 4u) j1 = 0;
 #pragma unroll
   for (int s = 0; s < 4; s++)
     if (j1 + 1 < L && P[j1 + 1] <= q) j1++;
@@ -547,7 +554,7 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
   // probe sum |N+(c)| elements (C2, |R| <= 32: 1.2e8 pairs vs 5.7e8 elements,
   // scratch/pair_cost.py) -- and no hash table.  The rows of 32 / |R|' consecutive
   // lanes (|R|' = |R| rounded up to a power of two) are ORed with shuffles.
-  if (TEAM_WARPS == 1 && L <= 32 && !(c_kcl_ablate & 64u)) {
+  if (TEAM_WARPS == 1 && L <= 32 && !GAMMA_KCL_NO_PAIRS) {
     if (lane < (int)L) R[lane] = a.dag_col[b0 + lane];
     __syncwarp();
     const uint32_t lg = L <= 2 ? 1u : L <= 4 ? 2u : L <= 8 ? 3u : L <= 16 ? 4u : 5u;
@@ -591,7 +598,7 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
     const uint32_t x = R[i];
     uint32_t h = (x * 0x9E3779B1u) >> (32 - hbits);
     if (Hv) {
-      h &= (c_kcl_ablate & 2u) ? ~1u : ~3u;   // probing starts at a 4-slot bucket: a lookup reads it in one load
+      h &= GAMMA_KCL_BUCKET4 ? ~3u : ~1u;   // probing starts at a bucket (pair / 4 slots) read in one load
       while (atomicCAS(&Hv[h], kEmptyId, x) != kEmptyId) h = (h + 1) & hmask;
       H[h] = (unsigned short)i;
     } else {
@@ -641,7 +648,7 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
     for (uint32_t t0 = 0; t0 < T; t0 += 32 * kTiles) {
       // tiles that hold elements (warp-uniform): a short window runs 1-3 tiles, not 4
       // (the padded tiles were ~half the row-build instructions on C2's small roots)
-      const uint32_t nt = (c_kcl_ablate & 8u) ? (uint32_t)kTiles : (T - t0 + 31) >> 5;
+      const uint32_t nt = (T - t0 + 31) >> 5;
       uint32_t y[kTiles], rj[kTiles];
 #pragma unroll
       for (int u = 0; u < kTiles; u++) {
@@ -675,7 +682,7 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
           const bool inr = yy >= rmin && yy <= rmax;   // (the padding 0xffffffff is above every rmax < n)
           bool hit;
           uint32_t hh;
-          if (c_kcl_ablate & 2u) {   // r01: two-slot pair probe
+          if (!GAMMA_KCL_BUCKET4) {   // two-slot pair probe
             const uint32_t h0 = ((yy * 0x9E3779B1u) >> (32 - hbits)) & ~1u;
             const uint2 vv = *reinterpret_cast<const uint2 *>(Hv + h0);
             hit = inr && (vv.x == yy || vv.y == yy);
@@ -873,7 +880,7 @@ __global__ void GAMMA_BM_BOUNDS(KM) kcl_bitmap_kernel(BmArgs a) {
       bool deferred = false;
       // hub splitting: estimate the DFS by the 4-clique count (skipped when even
       // items x |R| -- an upper bound of it -- is below the cut: most roots)
-      if (a.heavy_cut && ((c_kcl_ablate & 32u) || (uint64_t)items * L > a.heavy_cut)) {
+      if (a.heavy_cut && (uint64_t)items * L > a.heavy_cut) {
         uint64_t est = 0;
         uint32_t jr = 0;
         for (uint32_t q = tid; q < items; q += kTeamThreads) {
@@ -1363,9 +1370,6 @@ uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint6
     // the list trim pays only in rank space (ids in degree order); GAMMA_KCL_NO_TRIM off
     const char *e = getenv("GAMMA_KCL_NO_TRIM");
     a.trim = g->rank_space && !(e && *e && *e != '0');
-    const char *ab = getenv("GAMMA_KCL_ABLATE");
-    const uint32_t abl = ab && *ab ? (uint32_t)strtoul(ab, nullptr, 10) : 0u;
-    GAMMA_CUDA(cudaMemcpyToSymbolAsync(c_kcl_ablate, &abl, sizeof(abl), 0, cudaMemcpyHostToDevice, ctx->stream));
   }
   // hub splitting only pays when the DFS below a triangle is deep (k >= 6)
   // (GAMMA_KCL_SPLIT_MINK: the smallest k that splits, default 6)

@@ -1120,90 +1120,85 @@ static std::vector<JoinStep> join_steps(const SmPlan &P) {
   return st;
 }
 
+// DFS over (step, row range): step i turns its input rows into buffer i; a step whose
+// output overflows the buffer halves its input range (any step, not only the roots).
+struct JoinRun {
+  gamma_graph *g;
+  gamma_ctx *ctx;
+  SmPlan P;
+  std::vector<JoinStep> steps;
+  std::vector<DevBuf<uint32_t>> buf;   // one row buffer per step
+  uint64_t cap;                        // rows per buffer
+  DevBuf<unsigned long long> cur;      // cursor, overflow, count
+  uint64_t total = 0;
+
+  void run(size_t i, const uint32_t *in, uint64_t n_in, uint32_t w) {
+    if (n_in == 0) return;
+    const JoinStep &stp = steps[i];
+    JoinArgs a{};
+    a.rp = g->row_ptr;
+    a.col = g->col;
+    a.ldeg = g->ldeg;
+    a.lab = g->labels;
+    a.P = P;
+    a.in = in;
+    a.n_in = n_in;
+    a.w_in = w;
+    a.out = buf[i].p;
+    a.cap = cap;
+    a.cursor = cur.p;
+    a.ovf = cur.p + 1;
+    a.count = cur.p + 2;
+    a.q = stp.q;
+    a.b = stp.b;
+    a.anti = stp.kind == 2;
+    a.count_only = i + 1 == steps.size();
+    GAMMA_CUDA(cudaMemsetAsync(cur.p, 0, 24, ctx->stream));
+    const int kc = a.count_only ? KC_SM_COUNT : KC_SM_EXTEND;
+    if (stp.kind == 0)
+      ctx->launch(kc, [&] { sm_join_expand<<<g1d(n_in * 32), 256, 0, ctx->stream>>>(a); });
+    else
+      ctx->launch(kc, [&] { sm_join_check<<<g1d(n_in), 256, 0, ctx->stream>>>(a); });
+    uint64_t h[3];
+    GAMMA_CUDA(cudaMemcpyAsync(h, cur.p, 24, cudaMemcpyDeviceToHost, ctx->stream));
+    ctx->sync();
+    if (h[1]) {   // overflow: halve this step's input
+      ctx->stats.retries++;
+      GAMMA_REQUIRE(n_in > 1, GAMMA_E_NOMEM, "edge join: the rows of one embedding exceed the buffer");
+      const uint64_t half = n_in / 2;
+      run(i, in, half, w);
+      run(i, in + half * w, n_in - half, w);
+      return;
+    }
+    if (a.count_only) {
+      total = checked_add(total, h[2]);
+      ctx->stats.chunks++;
+      return;
+    }
+    const uint32_t w2 = stp.kind == 0 ? w + 1 : w;
+    if (stp.kind == 0) ctx->stats.level_entries[w2] += h[0];
+    run(i + 1, buf[i].p, h[0], w2);
+  }
+};
+
 static uint64_t match_join(gamma_graph *g, const SmPlan &P, const uint32_t *roots, uint64_t nr,
                            uint64_t level_share) {
   gamma_ctx *ctx = g->ctx;
-  const std::vector<JoinStep> steps = join_steps(P);
-  const uint64_t cap = std::max<uint64_t>(1 << 16, level_share / 2 / (4ull * P.nv));   // rows per buffer
-  DevBuf<uint32_t> bufA(ctx, cap * P.nv), bufB(ctx, cap * P.nv);
-  DevBuf<unsigned long long> cur(ctx, 3);   // cursor, overflow, count
-  uint64_t total = 0;
-  std::vector<std::pair<uint64_t, uint64_t>> todo;
-  for (uint64_t r0 = nr; r0 > 0;) {   // chunks of <= cap roots, processed in root order
-    const uint64_t r1 = r0 > cap ? r0 - cap : 0;
-    todo.push_back({r1, r0});
-    r0 = r1;
-  }
-  while (!todo.empty()) {
-    const auto rg = todo.back();
-    todo.pop_back();
-    // the chunk's roots as 1-word rows
-    GAMMA_REQUIRE(rg.second - rg.first <= cap, GAMMA_E_NOMEM, "edge join: root chunk exceeds the row buffer");
-    GAMMA_CUDA(cudaMemcpyAsync(bufA.p, roots + rg.first, (rg.second - rg.first) * 4, cudaMemcpyDeviceToDevice,
-                               ctx->stream));
-    uint32_t *in = bufA.p, *out = bufB.p;
-    uint64_t n_in = rg.second - rg.first;
-    uint32_t w = 1;
-    bool ovf = false;
-    uint64_t chunk_count = 0;
-    for (size_t i = 0; i < steps.size() && n_in; i++) {
-      const JoinStep &stp = steps[i];
-      JoinArgs a{};
-      a.rp = g->row_ptr;
-      a.col = g->col;
-      a.ldeg = g->ldeg;
-      a.lab = g->labels;
-      a.P = P;
-      a.in = in;
-      a.n_in = n_in;
-      a.w_in = w;
-      a.out = out;
-      a.cap = cap;
-      a.cursor = cur.p;
-      a.ovf = cur.p + 1;
-      a.count = cur.p + 2;
-      a.q = stp.q;
-      a.b = stp.b;
-      a.anti = stp.kind == 2;
-      a.count_only = i + 1 == steps.size();
-      GAMMA_CUDA(cudaMemsetAsync(cur.p, 0, 24, ctx->stream));
-      const bool last = a.count_only;
-      const int kc = last ? KC_SM_COUNT : KC_SM_EXTEND;
-      if (stp.kind == 0)
-        ctx->launch(kc, [&] { sm_join_expand<<<g1d(n_in * 32), 256, 0, ctx->stream>>>(a); });
-      else
-        ctx->launch(kc, [&] { sm_join_check<<<g1d(n_in), 256, 0, ctx->stream>>>(a); });
-      uint64_t h[3];
-      GAMMA_CUDA(cudaMemcpyAsync(h, cur.p, 24, cudaMemcpyDeviceToHost, ctx->stream));
-      ctx->sync();
-      if (h[1]) {
-        ovf = true;
-        break;
-      }
-      if (last) {
-        chunk_count = h[2];
-        break;
-      }
-      n_in = h[0];
-      if (stp.kind == 0) w++;
-      std::swap(in, out);
-      ctx->stats.level_entries[w] += stp.kind == 0 ? n_in : 0;
-    }
-    if (ovf) {
-      ctx->stats.retries++;
-      GAMMA_REQUIRE(rg.second - rg.first > 1, GAMMA_E_NOMEM, "edge join: one root's rows exceed the buffer");
-      const uint64_t mid = rg.first + (rg.second - rg.first) / 2;
-      todo.push_back({mid, rg.second});
-      todo.push_back({rg.first, mid});
-      continue;
-    }
-    ctx->stats.chunks++;
-    total = checked_add(total, chunk_count);
-  }
-  ctx->stats.level_entries[P.nv] = total;
+  JoinRun J;
+  J.g = g;
+  J.ctx = ctx;
+  J.P = P;
+  J.steps = join_steps(P);
+  const uint64_t nb = std::max<size_t>(1, J.steps.size() - 1);   // the last step only counts
+  J.cap = std::max<uint64_t>(1 << 12, level_share * std::max<uint32_t>(1, P.nv > 2 ? P.nv - 2 : 1) / nb /
+                                          (4ull * P.nv));
+  for (size_t i = 0; i < J.steps.size(); i++) J.buf.emplace_back(ctx, i + 1 < J.steps.size() ? J.cap * P.nv : 1);
+  J.cur = DevBuf<unsigned long long>(ctx, 3);
+  for (uint64_t r0 = 0; r0 < nr; r0 += J.cap) J.run(0, roots + r0, std::min<uint64_t>(J.cap, nr - r0), 1);
+  ctx->stats.level_entries[P.nv] = J.total;
   ctx->sync();
   ctx->collect_timings();
-  return total;
+  return J.total;
 }
 
 static uint64_t match_count(gamma_graph *g, const SmPlan &P) {

@@ -320,9 +320,9 @@ def test_edge_join_vs_oracle(G, oracle_mod, q, induced):
 
 
 def test_edge_join_small_buffer(G, oracle_mod):
-    """Root ranges halve when a step's rows overflow the row buffers (64 MiB budget)."""
+    """Row ranges halve at any step whose output overflows its row buffer (2 MiB budget)."""
     n, s, d, lab = gg.config_graph("c3", seed=1, scale=12)
-    c = G.Context(flags=G._native.GAMMA_FLAG_SM_EDGE_JOIN, hbm_budget_bytes=4 << 20)
+    c = G.Context(flags=G._native.GAMMA_FLAG_SM_EDGE_JOIN, hbm_budget_bytes=2 << 20)
     g = c.load_edges(n, s, d, lab)
     o = oracle_mod.Graph(n, s, d, lab)
     nv, e = Q["house"]
