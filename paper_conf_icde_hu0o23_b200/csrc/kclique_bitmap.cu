@@ -54,8 +54,10 @@ namespace {
 #endif
 
 constexpr int kMaxStack = 10;        // DFS levels below the first child: k <= 12
-constexpr uint32_t kPartCost = 4096; // 4-cliques per heavy-root part
+constexpr uint32_t kPartCost = 4096; // 4-cliques per heavy-root part (k >= 6; x4 at k = 5)
 constexpr uint32_t kMaxParts = 4096;
+constexpr uint32_t kSlotB = 520;     // root-rows slot: header 4 + P (<= 513) -> B at 520
+constexpr uint32_t kSlotWords = kSlotB + 512 * 17;
 
 struct BmArgs {
   const uint64_t *dag_ptr;
@@ -68,8 +70,13 @@ struct BmArgs {
   unsigned long long *per_root;
   // hub splitting (k >= 6): roots with more than heavy_cut 4-cliques are deferred
   uint64_t heavy_cut;         // 0: never defer
-  uint2 *parts;               // (absolute root index, part | nparts << 16)
+  uint2 *parts;               // (root-rows slot, part | nparts << 16)
   uint32_t parts_cap;
+  uint32_t part_cost;         // 4-cliques per part
+  // the deferred roots' rows, kept by the team that built them (the parts read them
+  // instead of rebuilding): slot = {L, W, BS, root index} + P[0..L] at 4 + B at kSlotB
+  uint32_t *root_rows;
+  uint32_t root_rows_cap;     // slots
   uint64_t root_base;         // index of roots[0] in the full root list (parts are absolute)
   uint32_t multi;             // count every clique size kmin..k at once (gamma_kclique_multi)
   uint32_t kmin;              // multi: smallest size asked for (>= 3); shorter runs are skipped
@@ -893,9 +900,30 @@ __global__ void GAMMA_BM_BOUNDS(KM) kcl_bitmap_kernel(BmArgs a) {
         }
         est = team_sum<TEAM_WARPS>(est, lane, m.slot);
         if (est > a.heavy_cut) {
-          const uint64_t want = est / kPartCost + 1;
+          const uint64_t want = est / a.part_cost + 1;
           const uint32_t nparts = want < kMaxParts ? (uint32_t)want : kMaxParts;
+          // keep the rows: one root-rows slot (none left: expand here)
           if (tid == 0) {
+            const unsigned long long sl = atomicAdd(&a.ctrl[CTRL_AUX2], 1ull);
+            m.slot[0] = sl < a.root_rows_cap ? (uint32_t)sl : 0xffffffffu;
+          }
+          team_sync<TEAM_WARPS>();
+          const uint32_t slot = m.slot[0];
+          team_sync<TEAM_WARPS>();
+          if (slot != 0xffffffffu) {
+            uint32_t *dst = a.root_rows + (uint64_t)slot * kSlotWords;
+            if (tid == 0) {
+              dst[0] = L;
+              dst[1] = W;
+              dst[2] = BS;
+              dst[3] = (uint32_t)(a.root_base + gi);
+            }
+            for (uint32_t i = tid; i <= L; i += kTeamThreads) dst[4 + i] = m.P[i];
+            for (uint32_t i = tid; i < L * BS; i += kTeamThreads) dst[kSlotB + i] = m.B[i];
+            __threadfence();
+            team_sync<TEAM_WARPS>();
+          }
+          if (tid == 0 && slot != 0xffffffffu) {
             // reserve [at, at + nparts) only if it fits: the cursor never passes
             // parts_cap, so every slot below it has been written by its reserver
             // (the parts kernel reads exactly [0, cursor))
@@ -910,12 +938,13 @@ __global__ void GAMMA_BM_BOUNDS(KM) kcl_bitmap_kernel(BmArgs a) {
               at = seen;
             }
             if (ok) {
-              for (uint32_t p = 0; p < nparts; p++)
-                a.parts[at + p] = make_uint2((uint32_t)(a.root_base + gi), p | (nparts << 16));
+              for (uint32_t p = 0; p < nparts; p++) a.parts[at + p] = make_uint2(slot, p | (nparts << 16));
               m.slot[0] = 1;
             } else {
               m.slot[0] = 0;   // list full: expand here
             }
+          } else if (tid == 0) {
+            m.slot[0] = 0;     // no root-rows slot: expand here
           }
           team_sync<TEAM_WARPS>();
           deferred = m.slot[0] == 1;
@@ -999,13 +1028,13 @@ __global__ void GAMMA_BM_BOUNDS(KM) kcl_bitmap_parts_kernel(BmArgs a) {
     __syncthreads();
     if (wi == 0xffffffffu) break;
     const uint2 pt = a.parts[wi];
-    const uint32_t gi = pt.x, part = pt.y & 0xffff, nparts = pt.y >> 16;
-    const uint32_t v = a.roots[gi];
-    const uint64_t b0 = a.dag_ptr[v];
-    const uint32_t L = (uint32_t)(a.dag_ptr[v + 1] - b0);
-    const uint32_t W = (L + 31) >> 5, BS = row_stride<8, TW>(L);
-    build_rows<8, TW>(a, m, b0, L, tid, lane);
-    scan_rows<8, TW>(m, L, tid, lane);
+    const uint32_t part = pt.y & 0xffff, nparts = pt.y >> 16;
+    // the root's rows as its team built them (no rebuild): one coalesced copy from L2
+    const uint32_t *src = a.root_rows + (uint64_t)pt.x * kSlotWords;
+    const uint32_t L = src[0], W = src[1], BS = src[2], gi = src[3];
+    for (uint32_t i = tid; i <= L; i += 256) m.P[i] = src[4 + i];
+    for (uint32_t i = tid; i < L * BS; i += 256) m.B[i] = src[kSlotB + i];
+    __syncthreads();
     const uint32_t items = m.P[L];
     uint64_t cnt = 0;
     const LaneGroup g = lane_group(lane);
@@ -1377,6 +1406,7 @@ uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint6
   const uint32_t split_mink = mk_env && *mk_env ? (uint32_t)std::max(3ul, strtoul(mk_env, nullptr, 10)) : 6u;
   const bool split = k >= split_mink && (ctx->desc.flags & GAMMA_FLAG_NO_SPLIT) == 0;
   DevBuf<uint2> parts;
+  DevBuf<uint32_t> root_rows;
   if (split) {
     // GAMMA_KCL_PARTS_CAP (tests): a small part list forces the "list full, expand
     // here" fallback
@@ -1385,7 +1415,11 @@ uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint6
                                       : 1u << 20;
     parts = DevBuf<uint2>(ctx, a.parts_cap);
     a.parts = parts.p;
-    a.heavy_cut = (ctx->desc.flags & GAMMA_FLAG_DEBUG_SPLIT_ALL) ? 1 : 4ull * kPartCost;
+    a.part_cost = k >= 6 ? kPartCost : 4 * kPartCost;
+    a.heavy_cut = (ctx->desc.flags & GAMMA_FLAG_DEBUG_SPLIT_ALL) ? 1 : 4ull * a.part_cost;
+    a.root_rows_cap = std::min<uint32_t>(a.parts_cap, 2048);
+    root_rows = DevBuf<uint32_t>(ctx, (uint64_t)a.root_rows_cap * kSlotWords);
+    a.root_rows = root_rows.p;
   }
   // Roots sorted by d+ descending fall into three contiguous classes: [0, n_long) ET
   // path, [n_long, n_mid) CTA teams, [n_mid, nroots) warp teams; each team kind runs
