@@ -335,7 +335,9 @@ def run_gamma(args):
     import paper_conf_icde_hu0o23_b200 as G
 
     n, s, d, lab, w = make_input(args.workload)
-    ctx = G.Context(device=dev, time_kernels=True)
+    hd = args.host_dag_cache_mb
+    ctx = G.Context(device=dev, time_kernels=True,
+                    **({"flags": G._native.GAMMA_FLAG_HOST_DAG, "dag_cache_bytes": int(hd * 2 ** 20)} if hd >= 0 else {}))
     stream = torch.cuda.current_stream()
     if isinstance(s, torch.Tensor):   # drawn on the device
         m_raw = s.numel()
@@ -526,6 +528,7 @@ def run_gamma(args):
                    **({"kcl_calls": "per-k gamma_kclique" if args.per_k else "one gamma_kclique_multi pass"}
                       if w["kind"] == "kcl" else {}),
                    "l2": "flushed between steps (256 MiB write)",
+                   **({"host_dag_cache_mb": args.host_dag_cache_mb} if args.host_dag_cache_mb >= 0 else {}),
                    "parallelism": f"root-partition dp{world} (CSR replicated)"},
         "roofline": roof,
         "cpu_baseline": cpu,
@@ -558,6 +561,9 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--per-k", action="store_true", help="kCL: one gamma_kclique call per k instead of one multi-k pass")
     ap.add_argument("--no-clocks", action="store_true", help="diagnostics only: skip nvidia-smi sampling")
+    ap.add_argument("--host-dag-cache-mb", type=float, default=-1,
+                    help="kCL with the DAG in pinned host memory and an HBM cache of this many MiB of its "
+                         "hottest pages (GAMMA_FLAG_HOST_DAG; SURVEY §8(f) rank 4); -1: DAG in HBM")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)

@@ -81,6 +81,9 @@ typedef struct {
      before the call; the callback returns once recv is complete.  NULL: gamma_fpm
      computes the whole result on every rank (replicas).                             */
   gamma_status (*alltoall_u32)(const uint32_t *send, uint32_t *recv, uint64_t n_per_rank, void *user);
+  /* GAMMA_FLAG_HOST_DAG: HBM bytes for the cache of the hottest DAG pages (the rest
+     stay in pinned host memory, read over the host link); 0: half of the DAG       */
+  uint64_t dag_cache_bytes;
 } gamma_ctx_desc;
 
 #define GAMMA_FLAG_TIME_KERNELS 0x1u   /* record per-launch CUDA-event times (stats) */
@@ -104,6 +107,12 @@ typedef struct {
                                           PAPER.md L141, L170): one pattern edge per ET step,
                                           non-tree edges as separate filter passes; same
                                           count, larger intermediate tables (ablation)   */
+#define GAMMA_FLAG_HOST_DAG      0x800u /* host-resident kCL DAG (the B200
+                                          analogue of the paper's host-memory graph):
+                                          the DAG columns live in pinned host memory, mapped into
+                                          the device address space, with an HBM cache of the
+                                          64 KiB pages ranked by heat (reads x elements, reads of
+                                          a list = 1 + its in-degree); bitmap kCL path only    */
 #define GAMMA_FLAG_FPM_INSTANCES 0x100u /* gamma_fpm: also count each pattern's instances
                                           (connected edge sets mapped to it; one atomic
                                           per embedding -- a parity check, not for timing) */

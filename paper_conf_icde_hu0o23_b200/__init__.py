@@ -179,7 +179,7 @@ class Context:
     def __init__(self, device: int = 0, rank: Optional[int] = None, world: Optional[int] = None,
                  use_torch: bool = True, hbm_budget_bytes: int = 0, host_spill_bytes: int = 0,
                  time_kernels: bool = False, flags: int = 0, reduce: bool = True,
-                 torch_alloc: Optional[bool] = None):
+                 torch_alloc: Optional[bool] = None, dag_cache_bytes: int = 0):
         self._keep = []
         if torch_alloc is None:   # GAMMA_ALLOC=native: the library's stream-ordered pool
             torch_alloc = os.environ.get("GAMMA_ALLOC", "torch") != "native"
@@ -228,6 +228,7 @@ class Context:
                 self._keep.append(fa2a)
         d.hbm_budget_bytes = hbm_budget_bytes
         d.host_spill_bytes = host_spill_bytes
+        d.dag_cache_bytes = dag_cache_bytes
         d.flags = flags | (N.GAMMA_FLAG_TIME_KERNELS if time_kernels else 0)
         self.desc = d
         h = C.c_void_p()

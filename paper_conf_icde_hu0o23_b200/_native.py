@@ -31,6 +31,7 @@ GAMMA_FLAG_COUNT_SORT_BUILD = 0x80
 GAMMA_FLAG_FPM_INSTANCES = 0x100
 GAMMA_FLAG_TWO_PASS = 0x200
 GAMMA_FLAG_SM_EDGE_JOIN = 0x400
+GAMMA_FLAG_HOST_DAG = 0x800
 
 ALLOC_FN = C.CFUNCTYPE(C.c_void_p, C.c_size_t, C.c_void_p, C.c_void_p)
 FREE_FN = C.CFUNCTYPE(None, C.c_void_p, C.c_void_p)
@@ -47,6 +48,7 @@ class gamma_ctx_desc(C.Structure):
         ("hbm_budget_bytes", C.c_uint64), ("host_spill_bytes", C.c_uint64),
         ("flags", C.c_uint32),
         ("alltoall_u32", ALLTOALL_FN),
+        ("dag_cache_bytes", C.c_uint64),
     ]
 
 

@@ -298,12 +298,15 @@ void gamma_graph_free(gamma_graph *g) {
     c->free(g->root_order);
     c->free(g->rank_of);
     c->free(g->ldeg);
+    c->free(g->dag_pages);
+    c->free(g->dag_cache);
     try {
       c->keep_release();   // kept SM tables were sized for this graph
     } catch (...) {
     }
     cudaStreamSynchronize(c->stream);
   }
+  if (g->dag_host) cudaFreeHost(g->dag_host);
   cudaGetLastError();
   delete g;
 }

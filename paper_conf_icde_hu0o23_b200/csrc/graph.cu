@@ -15,6 +15,9 @@
 #include <cub/device/device_segmented_sort.cuh>
 #include <cub/device/device_select.cuh>
 
+#include <algorithm>
+#include <vector>
+
 #include "internal.cuh"
 
 namespace gamma_impl {
@@ -321,6 +324,28 @@ __global__ void dag_id_write_kernel(const uint64_t *__restrict__ row_ptr, const 
   }
 }
 
+// ---- host-resident DAG (GAMMA_FLAG_HOST_DAG) ----
+__global__ void dag_indeg_kernel(const uint32_t *__restrict__ dag_col, uint64_t m, uint32_t *__restrict__ indeg) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < m; i += (uint64_t)gridDim.x * blockDim.x)
+    atomicAdd(&indeg[dag_col[i]], 1u);
+}
+
+// page heat: every list is read once as a root's run and once per parent (1 + its DAG
+// in-degree); a page's heat = the elements of it those reads fetch
+__global__ void dag_heat_kernel(const uint64_t *__restrict__ dag_ptr, const uint32_t *__restrict__ indeg, uint32_t n,
+                                unsigned long long *__restrict__ heat) {
+  for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x) {
+    const uint64_t b = dag_ptr[v], e = dag_ptr[v + 1];
+    if (b == e) continue;
+    const unsigned long long w = 1ull + indeg[v];
+    for (uint64_t p = b >> kDagPageShift; p <= (e - 1) >> kDagPageShift; p++) {
+      const uint64_t lo = b > (p << kDagPageShift) ? b : (p << kDagPageShift);
+      const uint64_t hi = e < ((p + 1) << kDagPageShift) ? e : ((p + 1) << kDagPageShift);
+      atomicAdd(&heat[p], w * (hi - lo));
+    }
+  }
+}
+
 uint32_t bit_width(uint32_t n) {  // bits to represent n itself
   uint32_t b = 0;
   while (b < 32 && (uint64_t(1) << b) <= n) b++;
@@ -471,6 +496,60 @@ void to_rank_space(gamma_graph *g, uint32_t *ids, uint64_t nids) {
   });
 }
 
+// Move the kCL DAG columns to pinned, mapped host memory and keep the hottest pages in
+// an HBM cache of cache_bytes (0: half of the DAG); the page table replaces dag_col.
+void host_dag(gamma_graph *g, uint64_t cache_bytes) {
+  gamma_ctx *ctx = g->ctx;
+  const uint64_t m = g->m;
+  if (m == 0) return;
+  const uint64_t page = 1ull << kDagPageShift;
+  const uint64_t np = (m + page - 1) / page;
+  std::vector<unsigned long long> heat(np);
+  {
+    DevBuf<uint32_t> indeg(ctx, g->n);
+    DevBuf<unsigned long long> dh(ctx, np);
+    GAMMA_CUDA(cudaMemsetAsync(indeg.p, 0, (size_t)g->n * 4, ctx->stream));
+    GAMMA_CUDA(cudaMemsetAsync(dh.p, 0, np * 8, ctx->stream));
+    ctx->launch(KC_BUILD, [&] { dag_indeg_kernel<<<grid_for(m), kThreads, 0, ctx->stream>>>(g->dag_col, m, indeg.p); });
+    ctx->launch(KC_BUILD, [&] {
+      dag_heat_kernel<<<grid_for(g->n), kThreads, 0, ctx->stream>>>(g->dag_ptr, indeg.p, g->n, dh.p);
+    });
+    GAMMA_CUDA(cudaMemcpyAsync(heat.data(), dh.p, np * 8, cudaMemcpyDeviceToHost, ctx->stream));
+    ctx->sync();
+  }
+  GAMMA_CUDA(cudaHostAlloc((void **)&g->dag_host, m * 4, cudaHostAllocMapped));
+  GAMMA_CUDA(cudaMemcpyAsync(g->dag_host, g->dag_col, m * 4, cudaMemcpyDeviceToHost, ctx->stream));
+  uint32_t *host_dev = nullptr;
+  GAMMA_CUDA(cudaHostGetDevicePointer((void **)&host_dev, g->dag_host, 0));
+  const uint64_t want = cache_bytes ? cache_bytes : m * 2;
+  const uint64_t k = std::min<uint64_t>(np, want / (page * 4));
+  std::vector<uint64_t> order(np);
+  for (uint64_t p = 0; p < np; p++) order[p] = p;
+  std::stable_sort(order.begin(), order.end(), [&](uint64_t x, uint64_t y) { return heat[x] > heat[y]; });
+  std::vector<uint64_t> table(np);
+  for (uint64_t p = 0; p < np; p++) table[p] = (uint64_t)(uintptr_t)(host_dev + p * page);
+  if (k) {
+    DevBuf<uint32_t> cache(ctx, k * page);
+    for (uint64_t i = 0; i < k; i++) {
+      const uint64_t p = order[i];
+      const uint64_t len = std::min<uint64_t>(page, m - p * page);
+      GAMMA_CUDA(cudaMemcpyAsync(cache.p + i * page, g->dag_col + p * page, len * 4, cudaMemcpyDeviceToDevice,
+                                 ctx->stream));
+      table[p] = (uint64_t)(uintptr_t)(cache.p + i * page);
+    }
+    g->dag_cache = cache.release();
+  }
+  DevBuf<uint64_t> pt = to_device(ctx, table.data(), np);
+  ctx->sync();
+  g->dag_pages = pt.release();
+  g->dag_npages = np;
+  g->dag_cached = k;
+  ctx->free(g->dag_col);
+  g->dag_col = nullptr;
+  g->device_bytes += np * 8 + k * page * 4;
+  g->device_bytes -= m * 4;
+}
+
 // The id-space DAG (gamma_graph_copy_csr(which = 1)): out-lists of every vertex id,
 // ascending by id, oriented by the (degree, id) order.
 void export_dag_ids(gamma_graph *g, uint64_t *dag_ptr_out, uint32_t *dag_col_out) {
@@ -618,6 +697,7 @@ void build_from_edges(gamma_graph *g, const uint32_t *src, const uint32_t *dst, 
   if (m && 2 * m < (1ull << 31) && (ctx->desc.flags & GAMMA_FLAG_COUNT_SORT_BUILD) != 0) {
     build_counting(g, src, dst, m);
     rank_dag(g);
+    if (ctx->desc.flags & GAMMA_FLAG_HOST_DAG) host_dag(g, ctx->desc.dag_cache_bytes);
     g->build_ms = timer.stop();
     return;
   }
@@ -672,6 +752,7 @@ void build_from_edges(gamma_graph *g, const uint32_t *src, const uint32_t *dst, 
   g->max_degree = max_degree(ctx, g->row_ptr, n);
   build_dag(g, uniq.p, M);
   rank_dag(g);
+  if (ctx->desc.flags & GAMMA_FLAG_HOST_DAG) host_dag(g, ctx->desc.dag_cache_bytes);
   g->build_ms = timer.stop();
 }
 
@@ -717,6 +798,7 @@ void build_from_csr(gamma_graph *g, const uint64_t *row_ptr, const uint32_t *col
   g->max_degree = max_degree(ctx, g->row_ptr, n);
   build_dag(g, keys.p, M);
   rank_dag(g);
+  if (ctx->desc.flags & GAMMA_FLAG_HOST_DAG) host_dag(g, ctx->desc.dag_cache_bytes);
   g->build_ms = timer.stop();
 }
 

@@ -185,6 +185,12 @@ struct gamma_graph {
   // gamma_match when every label is < 256 (ldeg_state: -1 not yet, 0 unusable, 1 built)
   uint32_t *ldeg = nullptr;
   int32_t ldeg_state = -1;
+  // GAMMA_FLAG_HOST_DAG (graph.cu host_dag): dag_col is freed; its 2^kDagPageShift-entry
+  // pages live in pinned host memory (dag_host, mapped) or in the HBM cache
+  // (dag_cache); dag_pages[p] = the device address of page p's first entry
+  uint64_t *dag_pages = nullptr;
+  uint32_t *dag_host = nullptr, *dag_cache = nullptr;
+  uint64_t dag_npages = 0, dag_cached = 0;
   uint32_t *labels = nullptr;    // n (nullptr: unlabeled, all 0)
   uint32_t max_degree = 0, max_out_degree = 0;
   uint64_t device_bytes = 0;
@@ -256,6 +262,8 @@ void build_dag(gamma_graph *g, uint64_t *sorted_keys_dev, uint64_t nkeys);
 void rank_dag(gamma_graph *g);                       // id-space DAG -> rank space (+ rank_of)
 void export_dag_ids(gamma_graph *g, uint64_t *dag_ptr_out, uint32_t *dag_col_out);
 void to_rank_space(gamma_graph *g, uint32_t *ids_dev, uint64_t nids);   // in place, on the stream
+constexpr uint32_t kDagPageShift = 14;   // 64 KiB pages of the host-resident DAG
+void host_dag(gamma_graph *g, uint64_t cache_bytes);   // GAMMA_FLAG_HOST_DAG (graph.cu)
 
 // kCL (kclique.cu)
 uint64_t kclique_count(gamma_graph *g, uint32_t k, const uint32_t *roots_dev, uint64_t nroots,

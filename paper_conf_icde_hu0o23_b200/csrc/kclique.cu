@@ -916,6 +916,10 @@ uint64_t kclique_count(gamma_graph *g, uint32_t k, const uint32_t *roots_dev, ui
   if (!per_root && ctx->desc.world <= 1 && k <= 2) return k == 1 ? g->n : g->m;
   GAMMA_REQUIRE(g->m < 0xFFFFFFFFull, GAMMA_E_UNSUPPORTED, "DAG with >= 2^32 edges");
   KclRun R;
+  if (g->dag_pages)   // host-resident DAG: the bitmap path only (runs <= kWideMaxRun, k <= 12)
+    GAMMA_REQUIRE((ctx->desc.flags & GAMMA_FLAG_NO_BITMAP) == 0 && k <= kBitmapMaxK &&
+                      g->max_out_degree <= kWideMaxRun, GAMMA_E_UNSUPPORTED,
+                  "GAMMA_FLAG_HOST_DAG: only the bitmap kCL path reads the paged DAG");
   R.g = g;
   R.ctx = ctx;
   R.k = k;

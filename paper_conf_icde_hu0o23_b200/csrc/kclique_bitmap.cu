@@ -59,9 +59,32 @@ constexpr uint32_t kMaxParts = 4096;
 constexpr uint32_t kSlotB = 520;     // root-rows slot: header 4 + P (<= 513) -> B at 520
 constexpr uint32_t kSlotWords = kSlotB + 512 * 17;
 
+// The DAG columns: HBM-resident (base) or, GAMMA_FLAG_HOST_DAG, paged (pages[p] = the
+// device address of page p: an HBM cache frame or mapped pinned host memory)
+struct DagCol {
+  const uint32_t *base;
+  const uint64_t *pages;
+  __device__ __forceinline__ uint32_t operator[](uint64_t i) const {
+    if (pages)
+      return __ldg(reinterpret_cast<const uint32_t *>(pages[i >> kDagPageShift]) + (i & ((1u << kDagPageShift) - 1u)));
+    return __ldg(base + i);
+  }
+};
+
+// lower-bound membership of y in col[b, b + len) (len >= 1)
+__device__ __forceinline__ bool col_contains(const DagCol &col, uint64_t b, uint32_t len, uint32_t y) {
+  uint32_t base = 0, n = len;
+  while (n > 1) {
+    const uint32_t half = n >> 1;
+    base = (col[b + base + half] <= y) ? base + half : base;
+    n -= half;
+  }
+  return col[b + base] == y;
+}
+
 struct BmArgs {
   const uint64_t *dag_ptr;
-  const uint32_t *dag_col;
+  DagCol dag_col;
   const uint32_t *roots;
   uint64_t nroots;
   uint32_t k;
@@ -576,7 +599,7 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
         const uint64_t cb = a.dag_ptr[c];
         const uint32_t dl = (uint32_t)(a.dag_ptr[c + 1] - cb);
         if (j == 0) elems += dl;
-        hit = j < L && j != i && dl && sorted_contains(a.dag_col + cb, dl, rj);
+        hit = j < L && j != i && dl && col_contains(a.dag_col, cb, dl, rj);
       }
       uint32_t bits = hit ? 1u << j : 0u;
       for (uint32_t o = 1; o < (1u << lg); o <<= 1) bits |= __shfl_xor_sync(0xffffffffu, bits, o);
@@ -626,11 +649,11 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
       // rank space: lists ascend by rank, so the part of N+(c) above the run's largest
       // rank cannot meet the run -- trim it (one binary search; ~19 % of the C2 row-build
       // elements, scratch/rank_cut.py)
-      if (a.trim && dl && __ldg(a.dag_col + cb + dl - 1) > rmax) {
+      if (a.trim && dl && a.dag_col[cb + dl - 1] > rmax) {
         uint32_t lo = 0, hi = dl - 1;   // first index with dag_col > rmax, in [0, dl - 1]
         while (lo < hi) {
           const uint32_t mid = (lo + hi) >> 1;
-          if (__ldg(a.dag_col + cb + mid) > rmax) hi = mid; else lo = mid + 1;
+          if (a.dag_col[cb + mid] > rmax) hi = mid; else lo = mid + 1;
         }
         dl = lo;
       }
@@ -675,7 +698,7 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
         const uint32_t bj = __shfl_sync(0xffffffffu, cbeg, j & 31);
         const uint32_t oj = __shfl_sync(0xffffffffu, o, j & 31);
         rj[u] = __shfl_sync(0xffffffffu, crow, j & 31);
-        y[u] = t < T ? __ldg(a.dag_col + bj + (t - oj)) : 0xffffffffu;
+        y[u] = t < T ? a.dag_col[(uint64_t)bj + (t - oj)] : 0xffffffffu;
       }
 #pragma unroll
       for (int u = 0; u < kTiles; u++) {
@@ -1387,7 +1410,7 @@ uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint6
   gamma_ctx *ctx = g->ctx;
   BmArgs a{};
   a.dag_ptr = g->dag_ptr;
-  a.dag_col = g->dag_col;
+  a.dag_col = DagCol{g->dag_col, g->dag_pages};
   a.roots = roots;
   a.nroots = nroots;
   a.k = k;

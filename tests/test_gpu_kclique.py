@@ -394,3 +394,20 @@ def test_c2_full_size_spill(G):
     for k in (5, 6):
         assert g.kclique(k) == gold["counts"][str(k)], k
         assert c.stats()["spilled_bytes"] > 0, k
+
+
+@pytest.mark.parametrize("cache_kb", [0, 64, 256, 1 << 20])
+def test_host_resident_dag(G, oracle_mod, cache_kb):
+    """GAMMA_FLAG_HOST_DAG: the DAG columns in pinned host memory
+    mapped into the device, the hottest 64 KiB pages cached in HBM (none / a few / all);
+    every count equals the oracle's, per root too."""
+    n, s, d, _ = gg.config_graph("c1", seed=3, scale=14)
+    c = G.Context(flags=G._native.GAMMA_FLAG_HOST_DAG, dag_cache_bytes=cache_kb << 10)
+    g = c.load_edges(n, s, d)
+    o = oracle_mod.Graph(n, s, d)
+    assert g.kclique_multi([3, 4, 5, 6]) == [o.kclique(k) for k in (3, 4, 5, 6)]
+    assert g.kclique(5) == o.kclique(5)
+    roots = np.arange(0, n, 7, dtype=np.uint32)
+    assert np.array_equal(g.kclique_roots(4, roots), o.kclique_roots(4, roots))
+    rp, col = g.csr("dag")   # export still in id space
+    assert int(rp[-1]) == g.info()["m"]
