@@ -41,13 +41,13 @@ namespace {
 // Compile-time variants (A/B builds, build.py tag=...; B200 r02 same-box A/B in
 // profiles/kcl_ab_r02.md): GAMMA_KCL_LEAF_BAL balanced lane-group leaf walk (default:
 // per-word walk -- faster with id-ordered runs, whose bits spread over the words),
-// GAMMA_KCL_BUCKET4 4-slot bucket hash probe (default: slot pair), GAMMA_KCL_NO_PAIRS
+// GAMMA_KCL_BUCKET4 4-slot bucket hash probe (default; 0: slot pair), GAMMA_KCL_NO_PAIRS
 // stream the lists of runs <= 32 too (default: pair probes there)
 #ifndef GAMMA_KCL_LEAF_BAL
 #define GAMMA_KCL_LEAF_BAL 0
 #endif
 #ifndef GAMMA_KCL_BUCKET4
-#define GAMMA_KCL_BUCKET4 0
+#define GAMMA_KCL_BUCKET4 1
 #endif
 #ifndef GAMMA_KCL_NO_PAIRS
 #define GAMMA_KCL_NO_PAIRS 0
