@@ -487,13 +487,26 @@ def run_gamma(args):
         launches = max(1, cand[dom]["launches"])
         per_launch_ms = cand[dom]["ms"] / launches
         kernel_bytes = cand[dom]["alg_bytes"] / launches   # the kernel's own counters
-        ab = load_alg_bytes(args.workload) if w["kind"] == "kcl" and not args.per_k else None
-        if ab and ab["kmax"] == max(w["ks"]):
-            # the method's bytes per step (oracle-counted), spread over the
-            # dominant class's launches of one step (at N > 1 this rank's 1/N share)
-            per_launch_bytes = ab["bytes_per_step"] / world * args.steps / launches
+        ab = load_alg_bytes(args.workload) if not args.per_k else None
+        step_bytes = None
+        if ab and w["kind"] == "kcl" and ab.get("kmax") == max(w["ks"]):
+            step_bytes = ab["bytes_per_step"]
             bytes_src = "SURVEY §8(d) B_l summed over the step's extension levels, counted over the oracle's " \
                         "enumeration (profiles/alg_bytes.json, tools/alg_bytes.py)"
+        elif ab and w["kind"] == "sm" and dom in ab.get("class_bytes_per_step", {}):
+            step_bytes = ab["class_bytes_per_step"][dom]
+            bytes_src = ("SURVEY §8(d) B_t of the " + dom + " steps of the 8 (query, labeling) runs, counted by the "
+                         "oracle's O-2b (og_match_levels) in the method's order and constraints (DESIGN R21; "
+                         "profiles/alg_bytes.json, tools/alg_bytes.py)")
+        elif ab and w["kind"] == "fpm" and ab.get("l") == w["l"]:
+            step_bytes = ab["bytes_per_step"]
+            bytes_src = ("FPM bytes per step (DESIGN §6): 4 B per adjacency element the extensions read + 32 B per "
+                         "recorded embedding, levels 1..l, from closed forms over the oracle's CSR and triangle "
+                         "count at minsup = 1 (an upper bound at the bench's minsup; profiles/alg_bytes.json)")
+        if step_bytes:
+            # the method's bytes per step (oracle-counted), spread over the dominant class's
+            # launches of one step (at N > 1 this rank's 1/N share)
+            per_launch_bytes = step_bytes / world * args.steps / launches
         else:
             per_launch_bytes = kernel_bytes
             bytes_src = "SURVEY §8(d) B_l from the kernel's own counters (list elements read, entries in/out)"

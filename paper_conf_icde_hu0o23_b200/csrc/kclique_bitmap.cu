@@ -61,25 +61,29 @@ constexpr uint32_t kSlotWords = kSlotB + 512 * 17;
 
 // The DAG columns: HBM-resident (base) or, GAMMA_FLAG_HOST_DAG, paged (pages[p] = the
 // device address of page p: an HBM cache frame or mapped pinned host memory)
+// (PAGED is a kernel template parameter: the HBM path pays nothing for the host mode)
 struct DagCol {
   const uint32_t *base;
   const uint64_t *pages;
-  __device__ __forceinline__ uint32_t operator[](uint64_t i) const {
-    if (pages)
+  template <bool PAGED>
+  __device__ __forceinline__ uint32_t at(uint64_t i) const {
+    if constexpr (PAGED)
       return __ldg(reinterpret_cast<const uint32_t *>(pages[i >> kDagPageShift]) + (i & ((1u << kDagPageShift) - 1u)));
-    return __ldg(base + i);
+    else
+      return __ldg(base + i);
   }
 };
 
 // lower-bound membership of y in col[b, b + len) (len >= 1)
+template <bool PAGED>
 __device__ __forceinline__ bool col_contains(const DagCol &col, uint64_t b, uint32_t len, uint32_t y) {
   uint32_t base = 0, n = len;
   while (n > 1) {
     const uint32_t half = n >> 1;
-    base = (col[b + base + half] <= y) ? base + half : base;
+    base = (col.at<PAGED>(b + base + half) <= y) ? base + half : base;
     n -= half;
   }
-  return col[b + base] == y;
+  return col.at<PAGED>(b + base) == y;
 }
 
 struct BmArgs {
@@ -572,7 +576,7 @@ struct TeamMem {
 // (wide runs, whose tables would not fit) the position table alone is probed.
 constexpr uint32_t kEmptyId = 0xffffffffu;   // vertex ids are < n <= 2^32 - 1
 
-template <int TEAM_WARPS>
+template <int TEAM_WARPS, bool PAGED>
 __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H, uint32_t *B, uint64_t b0,
                                  uint32_t L, int tid, int lane, uint32_t stride, uint32_t *Hv = nullptr) {
   constexpr int kTeamThreads = TEAM_WARPS * 32;
@@ -585,7 +589,7 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
   // scratch/pair_cost.py) -- and no hash table.  The rows of 32 / |R|' consecutive
   // lanes (|R|' = |R| rounded up to a power of two) are ORed with shuffles.
   if (TEAM_WARPS == 1 && L <= 32 && !GAMMA_KCL_NO_PAIRS) {
-    if (lane < (int)L) R[lane] = a.dag_col[b0 + lane];
+    if (lane < (int)L) R[lane] = a.dag_col.at<PAGED>(b0 + lane);
     __syncwarp();
     const uint32_t lg = L <= 2 ? 1u : L <= 4 ? 2u : L <= 8 ? 3u : L <= 16 ? 4u : 5u;
     const uint32_t j = lane & ((1u << lg) - 1u), rows_per = 32u >> lg;
@@ -599,7 +603,7 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
         const uint64_t cb = a.dag_ptr[c];
         const uint32_t dl = (uint32_t)(a.dag_ptr[c + 1] - cb);
         if (j == 0) elems += dl;
-        hit = j < L && j != i && dl && col_contains(a.dag_col, cb, dl, rj);
+        hit = j < L && j != i && dl && col_contains<PAGED>(a.dag_col, cb, dl, rj);
       }
       uint32_t bits = hit ? 1u << j : 0u;
       for (uint32_t o = 1; o < (1u << lg); o <<= 1) bits |= __shfl_xor_sync(0xffffffffu, bits, o);
@@ -616,7 +620,7 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
   uint32_t hbits = 2;
   while ((1u << hbits) < 4 * L) hbits++;
   const uint32_t hmask = (1u << hbits) - 1u;
-  for (uint32_t i = tid; i < L; i += kTeamThreads) R[i] = a.dag_col[b0 + i];
+  for (uint32_t i = tid; i < L; i += kTeamThreads) R[i] = a.dag_col.at<PAGED>(b0 + i);
   for (uint32_t i = tid; i < L * W; i += kTeamThreads) B[i] = 0u;
   if (Hv) {
     for (uint32_t i = tid; i <= hmask; i += kTeamThreads) Hv[i] = kEmptyId;
@@ -649,11 +653,11 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
       // rank space: lists ascend by rank, so the part of N+(c) above the run's largest
       // rank cannot meet the run -- trim it (one binary search; ~19 % of the C2 row-build
       // elements, scratch/rank_cut.py)
-      if (a.trim && dl && a.dag_col[cb + dl - 1] > rmax) {
+      if (a.trim && dl && a.dag_col.at<PAGED>(cb + dl - 1) > rmax) {
         uint32_t lo = 0, hi = dl - 1;   // first index with dag_col > rmax, in [0, dl - 1]
         while (lo < hi) {
           const uint32_t mid = (lo + hi) >> 1;
-          if (a.dag_col[cb + mid] > rmax) hi = mid; else lo = mid + 1;
+          if (a.dag_col.at<PAGED>(cb + mid) > rmax) hi = mid; else lo = mid + 1;
         }
         dl = lo;
       }
@@ -698,7 +702,7 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
         const uint32_t bj = __shfl_sync(0xffffffffu, cbeg, j & 31);
         const uint32_t oj = __shfl_sync(0xffffffffu, o, j & 31);
         rj[u] = __shfl_sync(0xffffffffu, crow, j & 31);
-        y[u] = t < T ? a.dag_col[(uint64_t)bj + (t - oj)] : 0xffffffffu;
+        y[u] = t < T ? a.dag_col.at<PAGED>((uint64_t)bj + (t - oj)) : 0xffffffffu;
       }
 #pragma unroll
       for (int u = 0; u < kTiles; u++) {
@@ -779,10 +783,10 @@ __device__ __forceinline__ uint32_t row_stride(uint32_t L) {
   return TEAM_WARPS == 1 ? (uint32_t)TW : (((L + 31) >> 5) | 1u);
 }
 
-template <int TEAM_WARPS, int TW>
+template <int TEAM_WARPS, int TW, bool PAGED>
 __device__ __forceinline__ uint64_t build_rows(const BmArgs &a, const TeamMem<TW> &m, uint64_t b0, uint32_t L,
                                                int tid, int lane) {
-  return build_rows_p<TEAM_WARPS>(a, m.R, m.H, m.B, b0, L, tid, lane, row_stride<TEAM_WARPS, TW>(L), m.Hv);
+  return build_rows_p<TEAM_WARPS, PAGED>(a, m.R, m.H, m.B, b0, L, tid, lane, row_stride<TEAM_WARPS, TW>(L), m.Hv);
 }
 
 // P[r] = exclusive scan of the row popcounts (the triangle items), P[L] = total.
@@ -855,7 +859,7 @@ __device__ __forceinline__ void flush_multi(uint64_t (&mc)[kMaxStack + 3], const
 
 // KM: compile-time bound on k for the register-resident DFS of warp teams (6 or 12;
 // the deeper instantiation needs more registers, so k <= 6 gets its own kernel).
-template <int TEAM_WARPS, int TW, bool PER_ROOT, int KM>
+template <int TEAM_WARPS, int TW, bool PER_ROOT, int KM, bool PAGED>
 __global__ void GAMMA_BM_BOUNDS(KM) kcl_bitmap_kernel(BmArgs a) {
   extern __shared__ uint32_t smem[];
   constexpr int kTeamThreads = TEAM_WARPS * 32;
@@ -893,7 +897,7 @@ __global__ void GAMMA_BM_BOUNDS(KM) kcl_bitmap_kernel(BmArgs a) {
     if (L <= a.len_lo || L > a.len_hi || L < (a.multi ? a.kmin - 1 : a.k - 1)) continue;   // uniform across the team
     const uint32_t W = (L + 31) >> 5, BS = row_stride<TEAM_WARPS, TW>(L);
     if (tid == 0) entries += L;
-    elems += build_rows<TEAM_WARPS, TW>(a, m, b0, L, tid, lane);
+    elems += build_rows<TEAM_WARPS, TW, PAGED>(a, m, b0, L, tid, lane);
     // ---- deeper extensions: bitmap DFS.  k = 3: one row per thread (its popcount).
     // k >= 4: the work items are the triangles (v, R[j1], R[j2]), j2 in row j1 ----
     uint64_t cnt = 0;
@@ -1214,7 +1218,7 @@ __device__ __forceinline__ uint64_t wdfs_count(const uint32_t *B, uint32_t W, co
   return cnt;
 }
 
-template <int WL, bool PER_ROOT, int KM>
+template <int WL, bool PER_ROOT, int KM, bool PAGED>
 __global__ void __launch_bounds__(kWideThreads) kcl_wide_kernel(BmArgs a) {
   extern __shared__ uint32_t smem[];
   constexpr int kMaxL = 1024 * WL;
@@ -1243,7 +1247,7 @@ __global__ void __launch_bounds__(kWideThreads) kcl_wide_kernel(BmArgs a) {
     }
     const uint32_t W = (L + 31) >> 5;
     if (tid == 0) entries += L;
-    elems += build_rows_p<kWideThreads / 32>(a, R, H, B, b0, L, tid, lane, W);
+    elems += build_rows_p<kWideThreads / 32, PAGED>(a, R, H, B, b0, L, tid, lane, W);
     uint64_t cnt = 0;
     for (;;) {
       uint32_t i = 0;
@@ -1296,19 +1300,20 @@ constexpr size_t wide_smem() {
 }
 
 // rows scratch: grid x (run length x words) for the longest run of the launch
-template <int WL, int KM>
+template <int WL, int KM, bool PAGED>
 void enqueue_wide_km(gamma_ctx *ctx, BmArgs a, bool per_root, uint32_t max_len, DevBuf<uint32_t> &rows) {
   static bool attr = false;
   if (!attr) {
-    GAMMA_CUDA(cudaFuncSetAttribute(kcl_wide_kernel<WL, false, KM>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    GAMMA_CUDA(cudaFuncSetAttribute(kcl_wide_kernel<WL, false, KM, PAGED>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                     (int)wide_smem<WL>()));
-    GAMMA_CUDA(cudaFuncSetAttribute(kcl_wide_kernel<WL, true, KM>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    GAMMA_CUDA(cudaFuncSetAttribute(kcl_wide_kernel<WL, true, KM, PAGED>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                     (int)wide_smem<WL>()));
     attr = true;
   }
   static int grid = 0;
   if (!grid)
-    grid = ctx->num_sms * occupancy_blocks((const void *)kcl_wide_kernel<WL, false, KM>, kWideThreads, wide_smem<WL>());
+    grid = ctx->num_sms *
+           occupancy_blocks((const void *)kcl_wide_kernel<WL, false, KM, PAGED>, kWideThreads, wide_smem<WL>());
   const uint64_t L = std::min<uint64_t>(max_len, 1024u * WL);
   a.wide_stride = L * ((L + 31) / 32);
   const uint64_t g = std::min<uint64_t>(grid, a.nroots);
@@ -1317,18 +1322,22 @@ void enqueue_wide_km(gamma_ctx *ctx, BmArgs a, bool per_root, uint32_t max_len, 
   GAMMA_CUDA(cudaMemsetAsync(ctx->ctrl + CTRL_WORK, 0, sizeof(uint64_t), ctx->stream));
   ctx->launch(KC_BITMAP, [&] {
     if (per_root)
-      kcl_wide_kernel<WL, true, KM><<<(unsigned)g, kWideThreads, wide_smem<WL>(), ctx->stream>>>(a);
+      kcl_wide_kernel<WL, true, KM, PAGED><<<(unsigned)g, kWideThreads, wide_smem<WL>(), ctx->stream>>>(a);
     else
-      kcl_wide_kernel<WL, false, KM><<<(unsigned)g, kWideThreads, wide_smem<WL>(), ctx->stream>>>(a);
+      kcl_wide_kernel<WL, false, KM, PAGED><<<(unsigned)g, kWideThreads, wide_smem<WL>(), ctx->stream>>>(a);
   });
 }
 
 template <int WL>
 void enqueue_wide(gamma_ctx *ctx, BmArgs a, bool per_root, uint32_t max_len, DevBuf<uint32_t> &rows) {
-  if (a.k <= 6)
-    enqueue_wide_km<WL, 6>(ctx, a, per_root, max_len, rows);
-  else
-    enqueue_wide_km<WL, kBitmapMaxK>(ctx, a, per_root, max_len, rows);
+  const bool paged = a.dag_col.pages != nullptr;
+  if (a.k <= 6) {
+    if (paged) enqueue_wide_km<WL, 6, true>(ctx, a, per_root, max_len, rows);
+    else enqueue_wide_km<WL, 6, false>(ctx, a, per_root, max_len, rows);
+  } else {
+    if (paged) enqueue_wide_km<WL, kBitmapMaxK, true>(ctx, a, per_root, max_len, rows);
+    else enqueue_wide_km<WL, kBitmapMaxK, false>(ctx, a, per_root, max_len, rows);
+  }
 }
 
 template <int TEAM_WARPS, int TW>
@@ -1338,35 +1347,39 @@ constexpr size_t bm_smem() {
 
 // Enqueue one team kind over a root range (no host round trip: the work counter is
 // reset on the stream, the counts accumulate in ctrl and are read once at the end).
-template <int TEAM_WARPS, int TW, int KM>
+template <int TEAM_WARPS, int TW, int KM, bool PAGED>
 void enqueue_bitmap_km(gamma_ctx *ctx, const BmArgs &a0, bool per_root) {
   static bool attr = false;
   if (!attr) {
-    GAMMA_CUDA(cudaFuncSetAttribute(kcl_bitmap_kernel<TEAM_WARPS, TW, false, KM>,
+    GAMMA_CUDA(cudaFuncSetAttribute(kcl_bitmap_kernel<TEAM_WARPS, TW, false, KM, PAGED>,
                                     cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bm_smem<TEAM_WARPS, TW>()));
-    GAMMA_CUDA(cudaFuncSetAttribute(kcl_bitmap_kernel<TEAM_WARPS, TW, true, KM>,
+    GAMMA_CUDA(cudaFuncSetAttribute(kcl_bitmap_kernel<TEAM_WARPS, TW, true, KM, PAGED>,
                                     cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bm_smem<TEAM_WARPS, TW>()));
     attr = true;
   }
   const size_t smem = bm_smem<TEAM_WARPS, TW>();
   static int grid = 0;
   if (!grid)
-    grid = ctx->num_sms * occupancy_blocks((const void *)kcl_bitmap_kernel<TEAM_WARPS, TW, false, KM>, 256, smem);
+    grid = ctx->num_sms * occupancy_blocks((const void *)kcl_bitmap_kernel<TEAM_WARPS, TW, false, KM, PAGED>, 256, smem);
   GAMMA_CUDA(cudaMemsetAsync(ctx->ctrl + CTRL_WORK, 0, sizeof(uint64_t), ctx->stream));
   ctx->launch(KC_BITMAP, [&] {
     if (per_root)
-      kcl_bitmap_kernel<TEAM_WARPS, TW, true, KM><<<grid, 256, smem, ctx->stream>>>(a0);
+      kcl_bitmap_kernel<TEAM_WARPS, TW, true, KM, PAGED><<<grid, 256, smem, ctx->stream>>>(a0);
     else
-      kcl_bitmap_kernel<TEAM_WARPS, TW, false, KM><<<grid, 256, smem, ctx->stream>>>(a0);
+      kcl_bitmap_kernel<TEAM_WARPS, TW, false, KM, PAGED><<<grid, 256, smem, ctx->stream>>>(a0);
   });
 }
 
 template <int TEAM_WARPS, int TW>
 void enqueue_bitmap(gamma_ctx *ctx, const BmArgs &a0, bool per_root) {
-  if (a0.k <= 6)
-    enqueue_bitmap_km<TEAM_WARPS, TW, 6>(ctx, a0, per_root);
-  else
-    enqueue_bitmap_km<TEAM_WARPS, TW, kBitmapMaxK>(ctx, a0, per_root);
+  const bool paged = a0.dag_col.pages != nullptr;
+  if (a0.k <= 6) {
+    if (paged) enqueue_bitmap_km<TEAM_WARPS, TW, 6, true>(ctx, a0, per_root);
+    else enqueue_bitmap_km<TEAM_WARPS, TW, 6, false>(ctx, a0, per_root);
+  } else {
+    if (paged) enqueue_bitmap_km<TEAM_WARPS, TW, kBitmapMaxK, true>(ctx, a0, per_root);
+    else enqueue_bitmap_km<TEAM_WARPS, TW, kBitmapMaxK, false>(ctx, a0, per_root);
+  }
 }
 
 template <int KM>
@@ -1424,9 +1437,13 @@ uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint6
     a.trim = g->rank_space && !(e && *e && *e != '0');
   }
   // hub splitting only pays when the DFS below a triangle is deep (k >= 6)
-  // (GAMMA_KCL_SPLIT_MINK: the smallest k that splits, default 6)
+  // (GAMMA_KCL_SPLIT_MINK: the smallest k that splits; default 6 on one GPU, 5 with
+  // world > 1: a rank holds 1/world of the roots, so a hub's single CTA becomes the
+  // critical path -- heavy, simulated 8 ranks on B200: 17.8 -> 9.3 ms per rank, while
+  // at world 1 splitting k = 5 cost 13 %, profiles/sim_ranks_r02.jsonl)
   const char *mk_env = getenv("GAMMA_KCL_SPLIT_MINK");
-  const uint32_t split_mink = mk_env && *mk_env ? (uint32_t)std::max(3ul, strtoul(mk_env, nullptr, 10)) : 6u;
+  const uint32_t split_mink = mk_env && *mk_env ? (uint32_t)std::max(3ul, strtoul(mk_env, nullptr, 10))
+                                                : (ctx->desc.world > 1 ? 5u : 6u);
   const bool split = k >= split_mink && (ctx->desc.flags & GAMMA_FLAG_NO_SPLIT) == 0;
   DevBuf<uint2> parts;
   DevBuf<uint32_t> root_rows;
