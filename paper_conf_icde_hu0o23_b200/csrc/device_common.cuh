@@ -26,6 +26,30 @@ __device__ __forceinline__ bool sorted_contains(P s, uint32_t len, uint32_t y) {
   return s[base] == y;
 }
 
+// Copies of sorted_contains per global-memory call-site kind, so ncu's source page
+// attributes them separately: a hub child's list probed from the short side, and the
+// (child, L_m element) pair probes of a short L_m.
+template <class P>
+__device__ __forceinline__ bool contains_hub(P s, uint32_t len, uint32_t y) {
+  uint32_t base = 0, n = len;
+  while (n > 1) {
+    uint32_t half = n >> 1;
+    base = (s[base + half] <= y) ? base + half : base;
+    n -= half;
+  }
+  return s[base] == y;
+}
+template <class P>
+__device__ __forceinline__ bool contains_pair(P s, uint32_t len, uint32_t y) {
+  uint32_t base = 0, n = len;
+  while (n > 1) {
+    uint32_t half = n >> 1;
+    base = (s[base + half] <= y) ? base + half : base;
+    n -= half;
+  }
+  return s[base] == y;
+}
+
 // First index i in [0, len) with s[i] > y (upper bound), len if none.
 template <class P>
 __device__ __forceinline__ uint32_t upper_bound_idx(P s, uint32_t len, uint32_t y) {

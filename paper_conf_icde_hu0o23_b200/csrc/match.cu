@@ -381,7 +381,7 @@ __global__ void __launch_bounds__(kThreads, 5) sm_kernel(SmArgs a) {
                 bool ok = false;
                 if (t < a1) {
                   const uint32_t x = lm[t];
-                  ok = !(inj_d && x == cj) && sorted_contains(a.col + bj, dj, x);
+                  ok = !(inj_d && x == cj) && contains_hub(a.col + bj, dj, x);
                 }
                 part += __popc(__ballot_sync(0xffffffffu, ok)) * (lane == 0);
               }
@@ -439,7 +439,7 @@ __global__ void __launch_bounds__(kThreads, 5) sm_kernel(SmArgs a) {
               if (ok) {
                 const uint64_t s0 = a.rp[c];
                 const uint32_t dl = (uint32_t)(a.rp[c + 1] - s0);
-                ok = dl > 0 && sorted_contains(a.col + s0, dl, x);
+                ok = dl > 0 && contains_pair(a.col + s0, dl, x);
               }
             }
             part += __popc(__ballot_sync(0xffffffffu, ok)) * (lane == 0);
