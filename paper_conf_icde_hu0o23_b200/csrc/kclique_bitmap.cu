@@ -587,7 +587,7 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
   // sorted list per ordered pair -- |R|(|R|-1) probes where streaming the lists would
   // probe sum |N+(c)| elements (C2, |R| <= 32: 1.2e8 pairs vs 5.7e8 elements,
   // scratch/pair_cost.py) -- and no hash table.  The rows of 32 / |R|' consecutive
-  // lanes (|R|' = |R| rounded up to a power of two) are ORed with shuffles.
+  // lanes (|R|' = |R| rounded up to a power of two) come out of one ballot.
   if (TEAM_WARPS == 1 && L <= 32 && !GAMMA_KCL_NO_PAIRS) {
     if (lane < (int)L) R[lane] = a.dag_col.at<PAGED>(b0 + lane);
     __syncwarp();
@@ -605,8 +605,9 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
         if (j == 0) elems += dl;
         hit = j < L && j != i && dl && col_contains<PAGED>(a.dag_col, cb, dl, rj);
       }
-      uint32_t bits = hit ? 1u << j : 0u;
-      for (uint32_t o = 1; o < (1u << lg); o <<= 1) bits |= __shfl_xor_sync(0xffffffffu, bits, o);
+      // one ballot holds every row of this iteration: row i's bits are its lane group's
+      const uint32_t bal = __ballot_sync(0xffffffffu, hit);
+      const uint32_t bits = lg == 5 ? bal : (bal >> (lane & ~((1u << lg) - 1u))) & ((1u << (1u << lg)) - 1u);
       if (j == 0 && i < L) {
         B[i * W] = bits;
 #pragma unroll
