@@ -337,28 +337,37 @@ __device__ __forceinline__ uint64_t rdfs_count(const uint32_t *B, const uint32_t
 // ---- lane-group DFS (CTA teams and heavy-root parts, rows of W <= 16 words) -------
 // A thread-per-item DFS over 16-word rows diverges badly (the subtree sizes of the
 // triangles of one hub differ by orders of magnitude; ncu: < 5 active threads per
-// warp instruction).  Here a group of kGroup = 16 aligned lanes walks one item, lane
-// gl holding word gl of every candidate bitmap: a node is one conflict-free row load,
-// an AND and a popcount per lane; the next child is one group ballot + shuffle.  The
-// counts stay per lane (summed by the final warp reduction).  Template recursion over
-// the number S of chosen vertices keeps every level in registers.
-constexpr int kGroup = 16;
+// warp instruction).  Here a group of aligned lanes walks one item, lane gl holding
+// word gl of every candidate bitmap: a node is one conflict-free row load, an AND and a
+// popcount per lane; the next child is one group ballot + shuffle.  The counts stay per
+// lane (summed by the final warp reduction).  Template recursion over the number S of
+// chosen vertices keeps every level in registers.  The group is 8 lanes for rows of
+// <= 8 words (|R| <= 256: C2's CTA teams have <= 6) and 16 above: a 16-lane group on
+// 6-word rows idled 10 lanes in every word-parallel step.
+constexpr int kGroup = 16;   // largest group
 
 struct LaneGroup {
   uint32_t mask;   // the group's lanes in the warp
   int base;        // first lane of the group
   int gl;          // this lane's index inside the group
   int lane;
+  int size;        // 8 or 16
 };
 
-__device__ __forceinline__ LaneGroup lane_group(int lane) {
+__device__ __forceinline__ LaneGroup lane_group(int lane, int size) {
   LaneGroup g;
-  g.base = lane & ~(kGroup - 1);
+  g.size = size;
+  g.base = lane & ~(size - 1);
   g.gl = lane - g.base;
-  g.mask = ((1u << kGroup) - 1u) << g.base;
+  g.mask = ((1u << size) - 1u) << g.base;
   g.lane = lane;
   return g;
 }
+
+#ifndef GAMMA_KCL_GROUP16   // A/B: always 16-lane groups (round 1)
+#define GAMMA_KCL_GROUP16 0
+#endif
+__device__ __forceinline__ int group_size_for(uint32_t W) { return (W <= 8 && !GAMMA_KCL_GROUP16) ? 8 : kGroup; }
 
 // next child of the group's remaining-bits word set (cleared), or -1
 __device__ __forceinline__ int group_next(const LaneGroup &g, uint32_t &rem) {
@@ -401,8 +410,7 @@ template <int WW>
 __device__ __forceinline__ uint32_t group_leaf_sum_bal(const uint32_t *B, uint32_t BS, uint32_t W, uint32_t curw,
                                                        const LaneGroup &g) {
   uint32_t s = __popc(curw);
-#pragma unroll
-  for (int o = 1; o < kGroup; o <<= 1) {
+  for (int o = 1; o < g.size; o <<= 1) {
     const uint32_t y = __shfl_up_sync(g.mask, s, o);
     if (g.gl >= o) s += y;
   }
@@ -414,7 +422,7 @@ __device__ __forceinline__ uint32_t group_leaf_sum_bal(const uint32_t *B, uint32
   }
   const uint32_t total = inc[WW - 1];
   uint32_t acc = 0;
-  for (uint32_t r = g.gl; r < total; r += kGroup) {
+  for (uint32_t r = g.gl; r < total; r += (uint32_t)g.size) {
     uint32_t wsel = 0, before = 0;
 #pragma unroll
     for (int w = 0; w < WW; w++)
@@ -517,8 +525,7 @@ __device__ __forceinline__ uint32_t group_item_cur(const uint32_t *B, const uint
   // the r-th set bit of row j1: inclusive scan of the word popcounts over the group
   const uint32_t pc = __popc(w1);
   uint32_t inc = pc;
-#pragma unroll
-  for (int o = 1; o < kGroup; o <<= 1) {
+  for (int o = 1; o < g.size; o <<= 1) {
     const uint32_t y = __shfl_up_sync(g.mask, inc, o);
     if (g.gl >= o) inc += y;
   }
@@ -995,10 +1002,11 @@ __global__ void GAMMA_BM_BOUNDS(KM) kcl_bitmap_kernel(BmArgs a) {
         }
       if constexpr (TEAM_WARPS > 1) {   // lane groups: one triangle item per 16-lane group
         if (!deferred) {
-          const LaneGroup g = lane_group(lane);
-          constexpr uint32_t kGroups = kTeamThreads / kGroup;
+          const int gsz = group_size_for(W);
+          const LaneGroup g = lane_group(lane, gsz);
+          const uint32_t ngroups = kTeamThreads / gsz;
           uint32_t jg = 0;
-          for (uint32_t q = tid / kGroup; q < items; q += kGroups) {
+          for (uint32_t q = tid / gsz; q < items; q += ngroups) {
             const uint32_t curw = group_item_cur(m.B, m.P, L, W, BS, q, g, jg);
             if (a.multi) {
               if (g.gl == 0) mc[3] += 1;   // the item is one triangle
@@ -1065,10 +1073,11 @@ __global__ void GAMMA_BM_BOUNDS(KM) kcl_bitmap_parts_kernel(BmArgs a) {
     __syncthreads();
     const uint32_t items = m.P[L];
     uint64_t cnt = 0;
-    const LaneGroup g = lane_group(lane);
-    constexpr uint32_t kGroups = 256 / kGroup;
+    const int gsz = group_size_for(W);
+    const LaneGroup g = lane_group(lane, gsz);
+    const uint32_t ngroups = 256 / gsz;
     uint32_t jg = 0;
-    for (uint32_t q = part + (tid / kGroup) * nparts; q < items; q += kGroups * nparts) {
+    for (uint32_t q = part + (tid / gsz) * nparts; q < items; q += ngroups * nparts) {
       const uint32_t curw = group_item_cur(m.B, m.P, L, W, BS, q, g, jg);
       if (a.multi) {
         if (g.gl == 0) mc[3] += 1;
