@@ -17,6 +17,8 @@ import ctypes as C
 import os
 import sys
 import weakref
+
+_is_finalizing = sys.is_finalizing   # bound now: module globals may be None at shutdown
 from typing import Optional
 
 import numpy as np
@@ -252,7 +254,7 @@ class Context:
     def __del__(self):
         # at interpreter shutdown the allocator callbacks (into torch) may already be
         # gone: leak instead of calling back into a half-finalised interpreter
-        if sys.is_finalizing():
+        if _is_finalizing():
             return
         try:
             self.close()
@@ -305,7 +307,7 @@ class Graph:
             self._h = None
 
     def __del__(self):
-        if sys.is_finalizing():
+        if _is_finalizing():
             return
         try:
             self.free()

@@ -411,3 +411,24 @@ def test_host_resident_dag(G, oracle_mod, cache_kb):
     assert np.array_equal(g.kclique_roots(4, roots), o.kclique_roots(4, roots))
     rp, col = g.csr("dag")   # export still in id space
     assert int(rp[-1]) == g.info()["m"]
+
+
+@pytest.mark.parametrize("scale,samples,world", [(16, 1_500_000, 8), (18, 6_000_000, 8), (18, 6_000_000, 3)])
+def test_simulated_ranks_wide_runs(G, scale, samples, world):
+    """The root partition on graphs whose runs reach the wide (|R| > 512) and CTA-team
+    paths (C5's shape family, a = 0.55 at small scale): the partial counts of the
+    `world` rank shares sum to the world-1 counts, for the multi-k pass (k = 3, 4, 5)
+    and per k (the C5 simulated-rank run of round 2 disagreed)."""
+    s, d = gg.rmat(scale, samples, 0.55, 0.20, 0.20, seed=1)
+    n = 1 << scale
+    g1 = G.Context().load_edges(n, s, d)
+    assert g1.info()["max_out_degree"] > 512
+    want = g1.kclique_multi([3, 4, 5])
+    want4 = g1.kclique(4)
+    tot, tot4 = [0, 0, 0], 0
+    for r in range(world):
+        g = G.Context(rank=r, world=world, reduce=False).load_edges(n, s, d)
+        tot = [x + y for x, y in zip(tot, g.kclique_multi([3, 4, 5]))]
+        tot4 += g.kclique(4)
+    assert tot4 == want4
+    assert tot == want
