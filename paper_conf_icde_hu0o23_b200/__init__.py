@@ -17,8 +17,6 @@ import ctypes as C
 import os
 import sys
 import weakref
-
-_is_finalizing = sys.is_finalizing   # bound now: module globals may be None at shutdown
 from typing import Optional
 
 import numpy as np
@@ -251,10 +249,10 @@ class Context:
             _lib.gamma_ctx_destroy(self._h)
             self._h = None
 
-    def __del__(self):
+    def __del__(self, _finalizing=sys.is_finalizing):   # bound at definition: globals may be gone
         # at interpreter shutdown the allocator callbacks (into torch) may already be
         # gone: leak instead of calling back into a half-finalised interpreter
-        if _is_finalizing():
+        if _finalizing():
             return
         try:
             self.close()
@@ -306,8 +304,8 @@ class Graph:
                 _lib.gamma_graph_free(self._h)
             self._h = None
 
-    def __del__(self):
-        if _is_finalizing():
+    def __del__(self, _finalizing=sys.is_finalizing):
+        if _finalizing():
             return
         try:
             self.free()
