@@ -1510,7 +1510,22 @@ uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint6
     a.roots = roots + (sorted ? n_mid : 0);
     a.root_base = sorted ? n_mid : 0;
     a.nroots = sorted ? nroots - n_mid : nroots;
-    enqueue_bitmap<1, 4>(ctx, a, per_root != nullptr);
+    const char *bands = getenv("GAMMA_KCL_BANDS");   // diagnostics: one warp-team launch per |R| band
+    if (sorted && bands && *bands && *bands != '0' && g->root_order == roots) {
+      const uint32_t thr[] = {129, 65, 33, 17, 9, 0};
+      for (int b = 0; b + 1 < 6; b++) {
+        const uint64_t lo = std::max<uint64_t>(n_mid, thr[b] < g->root_ge.size() ? g->root_ge[thr[b]] : 0);
+        const uint64_t hi = std::min<uint64_t>(nroots, thr[b + 1] < g->root_ge.size() ? g->root_ge[thr[b + 1]] : 0);
+        if (hi <= lo) continue;
+        BmArgs ab = a;
+        ab.roots = roots + lo;
+        ab.root_base = lo;
+        ab.nroots = hi - lo;
+        enqueue_bitmap<1, 4>(ctx, ab, per_root != nullptr);
+      }
+    } else {
+      enqueue_bitmap<1, 4>(ctx, a, per_root != nullptr);
+    }
   }
   if (split) {
     // parts carry absolute indices into the full root list
