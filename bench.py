@@ -392,8 +392,16 @@ def run_gamma(args):
                     collect()
             emb = sum(results.values())
         elif w["kind"] == "sm":
-            for (q, lname, nv, e, plab) in sm_runs():
-                results[f"{q}/{lname}"] = g.match(nv, e, plab)[0]
+            runs = sm_runs()
+            if args.sm_sequential:
+                for (q, lname, nv, e, plab) in runs:
+                    results[f"{q}/{lname}"] = g.match(nv, e, plab)[0]
+                    if coll:
+                        collect()
+            else:   # one gamma_match_batch: the eight level chains on concurrent streams
+                got = g.match_many([(nv, e, plab) for (q, lname, nv, e, plab) in runs])
+                for (q, lname, nv, e, plab), (cnt, _) in zip(runs, got):
+                    results[f"{q}/{lname}"] = cnt
                 if coll:
                     collect()
             emb = sum(results.values())
@@ -573,6 +581,8 @@ def main():
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--per-k", action="store_true", help="kCL: one gamma_kclique call per k instead of one multi-k pass")
+    ap.add_argument("--sm-sequential", action="store_true",
+                    help="SM: one gamma_match call per (query, labeling) instead of one gamma_match_batch")
     ap.add_argument("--no-clocks", action="store_true", help="diagnostics only: skip nvidia-smi sampling")
     ap.add_argument("--host-dag-cache-mb", type=float, default=-1,
                     help="kCL with the DAG in pinned host memory and an HBM cache of this many MiB of its "

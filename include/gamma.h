@@ -212,6 +212,14 @@ gamma_status gamma_pattern_plan(const gamma_pattern *p, gamma_plan_info *out);
 gamma_status gamma_match(gamma_graph *g, const gamma_pattern *p, uint64_t *count,
                          uint64_t *mappings);
 
+/* n queries at once (the same results as n gamma_match calls, in order): every query's
+ * roots first, then the level chains on separate streams of the context, so the tails of
+ * one query's launches overlap the others' (C3's eight (query, labeling) runs).
+ * counts[n] (and mappings[n], nullable) are written on GAMMA_OK; n <= 16 run
+ * concurrently, the rest sequentially.  Errors as gamma_match.                     */
+gamma_status gamma_match_batch(gamma_graph *g, uint32_t n, const gamma_pattern *patterns, uint64_t *counts,
+                               uint64_t *mappings);
+
 /* ---- Frequent pattern mining (Alg. 2) ------------------------------------------ */
 typedef struct {
   uint32_t nv, ne;

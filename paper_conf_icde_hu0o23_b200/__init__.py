@@ -352,6 +352,28 @@ class Graph:
         _check(_lib.gamma_match(self._h, C.byref(p), C.byref(c), C.byref(mp)), "gamma_match")
         return int(c.value), int(mp.value)
 
+    def match_many(self, queries) -> list:
+        """Several queries in one call (gamma_match_batch: level chains on concurrent
+        streams): queries = [(nv, edges, labels or None, induced), ...] ->
+        [(count, mappings), ...] in order."""
+        qs = list(queries)
+        if not qs:
+            return []
+        arr = (N.gamma_pattern * len(qs))()
+        keep = []
+        for i, q in enumerate(qs):
+            nv, e = q[0], q[1]
+            lab = q[2] if len(q) > 2 else None
+            ind = bool(q[3]) if len(q) > 3 else False
+            p, k = _pattern(nv, e, lab, ind)
+            arr[i] = p
+            keep.append(k)
+        counts = np.zeros(len(qs), np.uint64)
+        maps = np.zeros(len(qs), np.uint64)
+        _check(_lib.gamma_match_batch(self._h, len(qs), arr, counts.ctypes.data, maps.ctypes.data),
+               "gamma_match_batch")
+        return [(int(c), int(m)) for c, m in zip(counts, maps)]
+
     def motifs(self, k: int) -> dict:
         """Motif counts: induced counts of every connected unlabeled k-vertex pattern
         (k = 3, 4), one gamma_match(induced=1) call each."""

@@ -114,6 +114,8 @@ SIGNATURES = [
     ("gamma_pattern_plan", C.c_int32, [C.POINTER(gamma_pattern), C.POINTER(gamma_plan_info)]),
     ("gamma_match", C.c_int32, [C.c_void_p, C.POINTER(gamma_pattern), C.POINTER(C.c_uint64),
                                 C.POINTER(C.c_uint64)]),
+    ("gamma_match_batch", C.c_int32, [C.c_void_p, C.c_uint32, C.POINTER(gamma_pattern), C.c_void_p,
+                                      C.c_void_p]),
     ("gamma_fpm", C.c_int32, [C.c_void_p, C.c_uint32, C.c_uint64, C.POINTER(C.POINTER(gamma_fpm_result))]),
     ("gamma_fpm_result_free", None, [C.POINTER(gamma_fpm_result)]),
     ("gamma_get_stats", C.c_int32, [C.c_void_p, C.POINTER(gamma_run_stats)]),

@@ -112,6 +112,18 @@ void gamma_ctx::free(void *p) {
   else cudaFreeAsync(p, stream);
 }
 
+void gamma_ctx::side_init() {
+  if (!side_ctrl) {
+    GAMMA_CUDA(cudaMalloc(&side_ctrl, kMaxBatch * CTRL_WORDS * sizeof(uint64_t)));
+    GAMMA_CUDA(cudaMallocHost(&side_ctrl_host, kMaxBatch * CTRL_WORDS * sizeof(uint64_t)));
+  }
+  while (side_streams.size() < (size_t)kMaxBatch) {
+    cudaStream_t st;
+    GAMMA_CUDA(cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking));
+    side_streams.push_back(st);
+  }
+}
+
 void gamma_ctx::reset_stats() {
   pending.clear();
   ev_next = 0;
@@ -209,6 +221,9 @@ void gamma_ctx_destroy(gamma_ctx *ctx) {
   if (ctx->ctrl_host) cudaFreeHost(ctx->ctrl_host);
   if (ctx->spill_host) cudaFreeHost(ctx->spill_host);
   if (ctx->copy_stream) cudaStreamDestroy(ctx->copy_stream);
+  for (auto st : ctx->side_streams) cudaStreamDestroy(st);
+  if (ctx->side_ctrl) cudaFree(ctx->side_ctrl);
+  if (ctx->side_ctrl_host) cudaFreeHost(ctx->side_ctrl_host);
   for (auto e : ctx->ev_pool) cudaEventDestroy(e);
   if (ctx->own_stream && ctx->stream) cudaStreamDestroy(ctx->stream);
   cudaGetLastError();

@@ -116,22 +116,32 @@ struct gamma_ctx {
   // Launch helper: brackets the launch with events when timing is on.
   template <class F>
   void launch(int kc, F &&f) {
+    launch_on(kc, stream, f);
+  }
+  // the same on another stream of this context (batched SM queries)
+  template <class F>
+  void launch_on(int kc, cudaStream_t s, F &&f) {
     cudaEvent_t a = nullptr, b = nullptr;
     bool timing = (desc.flags & GAMMA_FLAG_TIME_KERNELS) != 0;
     if (timing) {
       a = next_event();
       b = next_event();
-      cudaEventRecord(a, stream);
+      cudaEventRecord(a, s);
     }
     f();
     GAMMA_CUDA(cudaGetLastError());
     if (timing) {
-      cudaEventRecord(b, stream);
+      cudaEventRecord(b, s);
       pending.push_back({kc, {a, b}});
     }
     stats.launches[kc]++;
     stats.total_launches++;
   }
+  // side streams and pinned control mirrors for batched queries (created on first use)
+  std::vector<cudaStream_t> side_streams;
+  uint64_t *side_ctrl = nullptr, *side_ctrl_host = nullptr;   // kMaxBatch x CTRL_WORDS
+  static constexpr int kMaxBatch = 16;
+  void side_init();
   // Library calls (CUB) that launch several kernels inside one ctx->launch(): add the
   // kernels beyond the first so total_launches matches the launch list.
   void extra_launches(int kc, uint64_t n) {

@@ -31,6 +31,7 @@
 #include <algorithm>
 #include <cstdlib>
 #include <cstring>
+#include <memory>
 #include <vector>
 
 #include "device_common.cuh"
@@ -860,12 +861,18 @@ struct SmRun {
   // shared overflow word makes every later level exit at once.  Returns false (nothing
   // recorded) when some level overflowed its table; the caller then runs the careful
   // per-level path (process), which grows tables and halves group ranges.
+  // chain_enqueue + chain_collect on the context's own stream and control block
   bool chain(uint64_t ngroups) {
+    chain_enqueue(ngroups, ctx->stream, (unsigned long long *)ctx->ctrl, ctx->ctrl_host);
+    ctx->sync();
+    return chain_collect(ctx->ctrl_host);
+  }
+
+  void chain_enqueue(uint64_t ngroups, cudaStream_t st, unsigned long long *ctrl, uint64_t *host) {
     const uint32_t nl = P.nv - 1;   // launches: d = 0 .. nv-2
     for (uint32_t q = 1; q < nl; q++)
       if (lv[q].cap_v == 0) grow(q, std::max<uint64_t>(1ull << 24, 4ull * kBlkV * kWarps * (uint64_t)grid));
-    unsigned long long *ctrl = (unsigned long long *)ctx->ctrl;
-    ctrl_reset(ctx);
+    GAMMA_CUDA(cudaMemsetAsync(ctrl, 0, CTRL_WORDS * sizeof(uint64_t), st));
     for (uint32_t d = 0; d < nl; d++) {
       const uint32_t q = d + 1;
       const bool last = q == P.nv - 1;
@@ -885,10 +892,14 @@ struct SmRun {
       }
       const int gr = grid_for(last, last ? 0 : lv[q].cap_v);
       const int kc = last ? KC_SM_COUNT : KC_SM_EXTEND;
-      ctx->launch(kc, [&] { sm_kernel<<<gr, kThreads, sm_smem(), ctx->stream>>>(a); });
+      ctx->launch_on(kc, st, [&] { sm_kernel<<<gr, kThreads, sm_smem(), st>>>(a); });
     }
-    ctrl_fetch(ctx);
-    const uint64_t *h = ctx->ctrl_host;
+    GAMMA_CUDA(cudaMemcpyAsync(host, ctrl, CTRL_WORDS * sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+  }
+
+  // after the stream of chain_enqueue completed: false (nothing recorded) on an overflow
+  bool chain_collect(const uint64_t *h) {
+    const uint32_t nl = P.nv - 1;
     if (h[CTRL_OVF]) {
       // hint for the careful path: grow the tables that ran out
       for (uint32_t d = 0; d + 1 < nl; d++) {
@@ -1201,10 +1212,13 @@ static uint64_t match_join(gamma_graph *g, const SmPlan &P, const uint32_t *root
   return J.total;
 }
 
-static uint64_t match_count(gamma_graph *g, const SmPlan &P) {
+// Roots, group table and staging scratch of one query (everything before the level
+// chain).  Returns true with `count` set when the query is already answered (nv = 1,
+// no roots, or the edge-join variant); else ngroups = the depth-0 groups.
+static bool match_prepare(gamma_graph *g, const SmPlan &P, SmRun &R, uint64_t &count, uint64_t &ngroups,
+                          uint32_t batch = 1) {
   gamma_ctx *ctx = g->ctx;
   ensure_ldeg(g);
-  SmRun R;
   R.g = g;
   R.ctx = ctx;
   R.P = P;
@@ -1214,7 +1228,7 @@ static uint64_t match_count(gamma_graph *g, const SmPlan &P) {
     size_t fr = 0, tot = 0;
     GAMMA_CUDA(cudaMemGetInfo(&fr, &tot));
     const uint64_t budget = ctx->desc.hbm_budget_bytes ? ctx->desc.hbm_budget_bytes : (uint64_t)(fr * 0.8);
-    R.level_share = budget / std::max<uint32_t>(1, P.nv > 2 ? P.nv - 2 : 1);
+    R.level_share = budget / batch / std::max<uint32_t>(1, P.nv > 2 ? P.nv - 2 : 1);
   }
   // ---- roots (position 0) ----
   const uint32_t n = g->n;
@@ -1242,9 +1256,11 @@ static uint64_t match_count(gamma_graph *g, const SmPlan &P) {
         const uint64_t x = i % (2 * w);
         mine += (x == r || x == 2 * w - 1 - r);
       }
-      return mine;
+      count = mine;
+      return true;
     }
-    return nr;
+    count = nr;
+    return true;
   }
   DevBuf<uint32_t> roots(ctx, nr ? nr : 1);
   if (nr) {
@@ -1282,8 +1298,14 @@ static uint64_t match_count(gamma_graph *g, const SmPlan &P) {
     roots = std::move(mine);
   }
   ctx->stats.level_entries[1] = nr;
-  if (nr == 0) return 0;
-  if (ctx->desc.flags & GAMMA_FLAG_SM_EDGE_JOIN) return match_join(g, P, roots.p, nr, R.level_share);
+  if (nr == 0) {
+    count = 0;
+    return true;
+  }
+  if (ctx->desc.flags & GAMMA_FLAG_SM_EDGE_JOIN) {
+    count = match_join(g, P, roots.p, nr, R.level_share);
+    return true;
+  }
   const uint64_t ngr = (nr + kRootChunk - 1) / kRootChunk;
   SmLevel &L0 = R.lv[0];
   L0.desc = DevBuf<uint32_t>(ctx, 2 * ngr);
@@ -1302,10 +1324,23 @@ static uint64_t match_count(gamma_graph *g, const SmPlan &P) {
     R.lm_scratch_cap = std::min<uint32_t>(g->max_degree, 1u << 16);
     R.lm_scratch = DevBuf<uint32_t>(ctx, (uint64_t)R.grid * kWarps * R.lm_scratch_cap, true);
   }
+  ngroups = ngr;
+  return false;
+}
+
+static bool sm_fast_ok(gamma_ctx *ctx, const SmPlan &P) {
+  return (ctx->desc.flags & GAMMA_FLAG_SPILL) == 0 && P.nv >= 2 && P.nv - 1 <= 12 &&
+         getenv("GAMMA_SM_NO_CHAIN") == nullptr;
+}
+
+static uint64_t match_count(gamma_graph *g, const SmPlan &P) {
+  gamma_ctx *ctx = g->ctx;
+  SmRun R;
+  uint64_t count = 0, ngr = 0;
+  if (match_prepare(g, P, R, count, ngr)) return count;
   // fast path: the whole level chain with one read-back; on a table overflow, the
   // careful per-level path (DFS over group ranges with table growth and halving)
-  const bool fast = (ctx->desc.flags & GAMMA_FLAG_SPILL) == 0 && P.nv >= 2 && P.nv - 1 <= 12 &&
-                    getenv("GAMMA_SM_NO_CHAIN") == nullptr;
+  const bool fast = sm_fast_ok(ctx, P);
   if (!fast || !R.chain(ngr)) {
     if (fast) ctx->stats.retries++;
     R.process(0, 0, ngr);
@@ -1313,6 +1348,54 @@ static uint64_t match_count(gamma_graph *g, const SmPlan &P) {
   ctx->sync();
   ctx->collect_timings();
   return R.total;
+}
+
+// Several queries at once (gamma_match_batch): roots of every query first, then every
+// level chain on its own side stream (a chain's kernels run back to back, the chains
+// overlap each other's tails), one wait; an overflowing chain reruns alone on the
+// careful path.
+static void match_batch(gamma_graph *g, const std::vector<SmPlan> &Ps, std::vector<uint64_t> &counts) {
+  gamma_ctx *ctx = g->ctx;
+  const size_t nq = Ps.size();
+  counts.assign(nq, 0);
+  std::vector<std::unique_ptr<SmRun>> runs(nq);
+  std::vector<uint64_t> ngr(nq, 0);
+  std::vector<bool> done(nq, false);
+  for (size_t i = 0; i < nq; i++) {
+    runs[i].reset(new SmRun());
+    uint64_t c = 0;
+    done[i] = match_prepare(g, Ps[i], *runs[i], c, ngr[i], (uint32_t)std::min<size_t>(nq, gamma_ctx::kMaxBatch));
+    if (done[i]) counts[i] = c;
+  }
+  ctx->side_init();
+  cudaEvent_t ready;
+  GAMMA_CUDA(cudaEventCreateWithFlags(&ready, cudaEventDisableTiming));
+  GAMMA_CUDA(cudaEventRecord(ready, ctx->stream));   // roots and tables are on ctx->stream
+  std::vector<int> slot(nq, -1);
+  int used = 0;
+  for (size_t i = 0; i < nq; i++) {
+    if (done[i] || !sm_fast_ok(ctx, Ps[i]) || used >= gamma_ctx::kMaxBatch) continue;
+    const int sl = used++;
+    slot[i] = sl;
+    cudaStream_t st = ctx->side_streams[sl];
+    GAMMA_CUDA(cudaStreamWaitEvent(st, ready, 0));
+    runs[i]->chain_enqueue(ngr[i], st, (unsigned long long *)(ctx->side_ctrl + (size_t)sl * CTRL_WORDS),
+                           ctx->side_ctrl_host + (size_t)sl * CTRL_WORDS);
+  }
+  for (int sl = 0; sl < used; sl++) GAMMA_CUDA(cudaStreamSynchronize(ctx->side_streams[sl]));
+  cudaEventDestroy(ready);
+  for (size_t i = 0; i < nq; i++) {
+    if (done[i]) continue;
+    SmRun &R = *runs[i];
+    bool ok = slot[i] >= 0 && R.chain_collect(ctx->side_ctrl_host + (size_t)slot[i] * CTRL_WORDS);
+    if (!ok) {
+      if (slot[i] >= 0) ctx->stats.retries++;
+      R.process(0, 0, ngr[i]);
+    }
+    counts[i] = R.total;
+  }
+  ctx->sync();
+  ctx->collect_timings();
 }
 
 }  // namespace gamma_impl
@@ -1332,6 +1415,34 @@ extern "C" gamma_status gamma_pattern_plan(const gamma_pattern *p, gamma_plan_in
       out->backward_mask[i] = P.bmask[i];
       out->less_mask[i] = P.ltmask[i];
       out->greater_mask[i] = P.gtmask[i];
+    }
+  });
+}
+
+extern "C" gamma_status gamma_match_batch(gamma_graph *g, uint32_t n, const gamma_pattern *ps, uint64_t *counts,
+                                          uint64_t *mappings) {
+  return guarded([&] {
+    GAMMA_REQUIRE(g && (n == 0 || (ps && counts)), GAMMA_E_INVAL, "gamma_match_batch: NULL argument");
+    GAMMA_REQUIRE(2 * g->m < (1ull << 32), GAMMA_E_UNSUPPORTED,
+                  "gamma_match_batch: graphs with 2m >= 2^32 unsupported");
+    std::vector<SmPlan> Ps(n);
+    for (uint32_t i = 0; i < n; i++) plan_pattern(ps + i, Ps[i]);
+    gamma_ctx *c = g->ctx;
+    GAMMA_CUDA(cudaSetDevice(c->device));
+    c->reset_stats();
+    std::vector<uint64_t> r;
+    match_batch(g, Ps, r);
+    if (c->desc.world > 1 && c->desc.allreduce_sum_u64 && n) {
+      gamma_status st = c->desc.allreduce_sum_u64(r.data(), n, c->desc.coll_user);
+      GAMMA_REQUIRE(st == GAMMA_OK, st, "allreduce_sum_u64 callback failed");
+    }
+    for (uint32_t i = 0; i < n; i++) {
+      counts[i] = r[i];
+      if (mappings) {
+        uint64_t mp;
+        GAMMA_REQUIRE(!__builtin_mul_overflow(r[i], Ps[i].aut, &mp), GAMMA_E_OVERFLOW, "mappings overflow uint64");
+        mappings[i] = mp;
+      }
     }
   });
 }

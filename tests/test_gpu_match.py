@@ -217,12 +217,16 @@ def test_c3_full_size(ctx):
     n, s, d, lab = gg.config_graph("c3", seed=1)
     g = ctx.load_edges(n, s, d, lab)
     assert g.info()["m"] == gold["m"]
+    batch = []
     for key, want in gold["counts"].items():
         parts = key.split("/")
         q, lname, ind = parts[0], parts[1], len(parts) > 2
         nv, e = Q[q]
         plab = [0] * nv if lname == "all0" else [i % 8 for i in range(nv)]
         assert g.match(nv, e, plab, induced=ind)[0] == want, key
+        batch.append(((nv, e, plab, ind), want))
+    # the bench's configuration: all runs in one gamma_match_batch (concurrent chains)
+    assert [c for c, _ in g.match_many([b[0] for b in batch])] == [b[1] for b in batch]
 
 
 def test_motifs(ctx, oracle_mod):
@@ -328,3 +332,19 @@ def test_edge_join_small_buffer(G, oracle_mod):
     nv, e = Q["house"]
     assert g.match(nv, e)[0] == o.match(nv, e)[0]
     assert c.stats()["chunks"] > 1
+
+
+def test_match_many(G, oracle_mod):
+    """gamma_match_batch: the same counts and mappings as one gamma_match per query,
+    in order, with tables small enough that some chains overflow and rerun alone."""
+    n, s, d, lab = gg.config_graph("c3", seed=3, scale=12)
+    o = oracle_mod.Graph(n, s, d, lab)
+    qs = []
+    for q in ("c4", "diamond", "tailed_triangle", "house"):
+        nv, e = Q[q]
+        qs += [(nv, e, [0] * nv, False), (nv, e, [i % 8 for i in range(nv)], False), (nv, e, None, True)]
+    want = [o.match(nv, e, pl, induced=ind)[:2] for nv, e, pl, ind in qs]
+    for c in (G.Context(), G.Context(hbm_budget_bytes=16 << 20)):
+        g = c.load_edges(n, s, d, lab)
+        assert g.match_many(qs) == want
+        assert g.match_many([]) == []
