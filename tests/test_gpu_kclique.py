@@ -413,8 +413,9 @@ def test_host_resident_dag(G, oracle_mod, cache_kb):
     assert int(rp[-1]) == g.info()["m"]
 
 
-@pytest.mark.parametrize("scale,samples,world", [(16, 1_500_000, 8), (18, 6_000_000, 8), (18, 6_000_000, 3)])
-def test_simulated_ranks_wide_runs(G, scale, samples, world):
+@pytest.mark.parametrize("scale,samples,world,min_dplus", [(16, 6_000_000, 8, 512), (16, 6_000_000, 3, 512),
+                                                            (18, 6_000_000, 8, 128)])
+def test_simulated_ranks_wide_runs(G, scale, samples, world, min_dplus):
     """The root partition on graphs whose runs reach the wide (|R| > 512) and CTA-team
     paths (C5's shape family, a = 0.55 at small scale): the partial counts of the
     `world` rank shares sum to the world-1 counts, for the multi-k pass (k = 3, 4, 5)
@@ -422,7 +423,7 @@ def test_simulated_ranks_wide_runs(G, scale, samples, world):
     s, d = gg.rmat(scale, samples, 0.55, 0.20, 0.20, seed=1)
     n = 1 << scale
     g1 = G.Context().load_edges(n, s, d)
-    assert g1.info()["max_out_degree"] > 512
+    assert g1.info()["max_out_degree"] > min_dplus   # (scale 16, 6M: 651; scale 18: 464)
     want = g1.kclique_multi([3, 4, 5])
     want4 = g1.kclique(4)
     tot, tot4 = [0, 0, 0], 0
