@@ -41,13 +41,13 @@ namespace {
 // Compile-time variants (A/B builds, build.py tag=...; B200 r02 same-box A/B in
 // profiles/kcl_ab_r02.md): GAMMA_KCL_LEAF_BAL balanced lane-group leaf walk (default:
 // per-word walk -- faster with id-ordered runs, whose bits spread over the words),
-// GAMMA_KCL_BUCKET4 4-slot bucket hash probe (default; 0: slot pair), GAMMA_KCL_NO_PAIRS
-// stream the lists of runs <= 32 too (default: pair probes there)
+// GAMMA_KCL_NO_PAIRS stream the lists of runs <= 32 too (default: pair probes there).
+// (The slot-pair hash probe lost to the 4-slot bucket, session g, and was removed.)
 #ifndef GAMMA_KCL_LEAF_BAL
 #define GAMMA_KCL_LEAF_BAL 0
 #endif
-#ifndef GAMMA_KCL_BUCKET4
-#define GAMMA_KCL_BUCKET4 1
+#ifndef GAMMA_KCL_SM_DFS   // warp teams, k <= 6: state-machine DFS (0: nested loops per item)
+#define GAMMA_KCL_SM_DFS 1
 #endif
 #ifndef GAMMA_KCL_NO_PAIRS
 #define GAMMA_KCL_NO_PAIRS 0
@@ -538,6 +538,111 @@ __device__ __forceinline__ uint32_t group_item_cur(const uint32_t *B, const uint
   return w1 & w2;
 }
 
+// ---- warp teams, k <= 6: the DFS as a per-lane state machine ----------------------
+// The nested-loop DFS (rdfs_*) gives each lane whole triangle items, and the subtrees
+// below the triangles of one root differ by orders of magnitude: ncu c2 r02b put the
+// DFS at 7.1 active threads per warp instruction.  Here every lane does exactly one
+// node per step -- the next child of its deepest open node, else a fresh triangle item
+// -- so the warp stays converged until the root's items run out.  Below a triangle
+// (S = 3 chosen vertices, candidates X) the open nodes are X (S = 3) and Y (S = 4):
+// a step pops a child j of Y (leaf: popc(Y & B[j]) (S+2)-cliques), else of X (node
+// Y = X & B[j]), else takes an item (X = B[j1] & B[j2]).  Items come from a per-warp
+// queue refilled 32 at a time (one item -> (j1, j2) mapping per lane).
+// Counts per size: multi (kmin..kmax, kmax <= 6) adds popc of every node; single k
+// adds only size k and prunes nodes that cannot reach it (as rdfs_count).
+__device__ __forceinline__ bool any4(const uint32_t (&x)[4]) { return (x[0] | x[1] | x[2] | x[3]) != 0u; }
+
+template <bool MULTI>
+__device__ __forceinline__ void warp_dfs_sm(const uint32_t *B, const uint32_t *P, uint32_t L, uint32_t W,
+                                            uint32_t items, uint32_t k, int lane, uint32_t *Q,
+                                            uint64_t &c3, uint64_t &c4, uint64_t &c5, uint64_t &c6, uint64_t &cnt) {
+  constexpr uint32_t kFull = 0xffffffffu;
+  const uint32_t lt = (1u << lane) - 1u;
+  uint32_t X[4] = {0, 0, 0, 0}, rX[4] = {0, 0, 0, 0}, Y[4] = {0, 0, 0, 0}, rY[4] = {0, 0, 0, 0};
+  uint32_t filled = 0, taken = 0, jq = 0;
+  uint32_t a3 = 0, a4 = 0, a5 = 0, a6 = 0;   // this root's counts (< 2^32 for |R| <= 128)
+  // expand a node of S chosen vertices (children add size S + 2 below it)?
+  const bool exp3 = MULTI ? k > 4 : k > 4, exp4 = MULTI ? k > 5 : k > 5;
+  for (;;) {
+    const bool useY = any4(rY), useX = !useY && any4(rX);
+    const bool busy = useY || useX;
+    const uint32_t need = __ballot_sync(kFull, !busy);
+    const uint32_t nneed = __popc(need);
+    if (filled < items && filled - taken < nneed) {   // warp-uniform refill
+      const uint32_t q = filled + lane;
+      if (q < items) {
+        jq = advance_row(P, L, q, jq);
+        uint32_t r = q - P[jq], j2 = 0;
+#pragma unroll
+        for (uint32_t w = 0; w < 4; w++) {
+          const uint32_t word = w < W ? B[jq * 4 + w] : 0u;
+          const uint32_t pc = __popc(word);
+          if (r < pc) {
+            j2 = w * 32 + __fns(word, 0, r + 1);
+            r = 0xffffffffu;   // found: no later word matches (r < pc fails)
+          } else if (r != 0xffffffffu) {
+            r -= pc;
+          }
+        }
+        Q[q & 63] = (jq << 16) | j2;
+      }
+      filled = min(items, filled + 32);
+      __syncwarp();
+    }
+    const uint32_t avail = filled - taken, rank = __popc(need & lt);
+    const bool got = !busy && rank < avail;
+    const uint32_t it = got ? Q[(taken + rank) & 63] : 0u;
+    taken += min(nneed, avail);
+    if (!__any_sync(kFull, busy || got)) break;
+    // the node of this step: its parent's candidates (src) and the child row j
+    uint32_t src[4], j = 0;
+    if (busy) {
+      uint32_t rr[4];
+#pragma unroll
+      for (int w = 0; w < 4; w++) rr[w] = useY ? rY[w] : rX[w];
+      const int wi = rr[0] ? 0 : rr[1] ? 1 : rr[2] ? 2 : 3;
+      const uint32_t word = wi == 0 ? rr[0] : wi == 1 ? rr[1] : wi == 2 ? rr[2] : rr[3];
+      j = (uint32_t)wi * 32 + __ffs(word) - 1;
+      const uint32_t nw = word & (word - 1u);
+#pragma unroll
+      for (int w = 0; w < 4; w++) {
+        if (w == wi) {
+          if (useY) rY[w] = nw; else rX[w] = nw;
+        }
+        src[w] = useY ? Y[w] : X[w];
+      }
+    } else if (got) {
+      j = it & 0xffffu;
+      const uint4 r1 = *reinterpret_cast<const uint4 *>(B + (it >> 16) * 4);
+      src[0] = r1.x; src[1] = r1.y; src[2] = r1.z; src[3] = r1.w;
+    } else {
+      src[0] = src[1] = src[2] = src[3] = 0u;
+    }
+    const uint4 rj = *reinterpret_cast<const uint4 *>(B + j * 4);
+    const uint32_t n0 = src[0] & rj.x, n1 = src[1] & rj.y, n2 = src[2] & rj.z, n3 = src[3] & rj.w;
+    const uint32_t c = __popc(n0) + __popc(n1) + __popc(n2) + __popc(n3);
+    if (useY) {            // leaf below Y: (S = 5)-node, c = (S + 1 = 6)-cliques
+      a6 += c;
+    } else if (useX) {     // Y = X & B[j]: S = 4 node, c = 5-cliques
+      a5 += c;
+      const bool e = exp4 && (MULTI || c >= k - 4);
+      Y[0] = n0; Y[1] = n1; Y[2] = n2; Y[3] = n3;
+      rY[0] = e ? n0 : 0u; rY[1] = e ? n1 : 0u; rY[2] = e ? n2 : 0u; rY[3] = e ? n3 : 0u;
+    } else if (got) {      // X = B[j1] & B[j2]: S = 3 node (a triangle), c = 4-cliques
+      a3 += 1;
+      a4 += c;
+      const bool e = exp3 && (MULTI || c >= k - 3);
+      X[0] = n0; X[1] = n1; X[2] = n2; X[3] = n3;
+      rX[0] = e ? n0 : 0u; rX[1] = e ? n1 : 0u; rX[2] = e ? n2 : 0u; rX[3] = e ? n3 : 0u;
+    }
+  }
+  if (MULTI) {
+    c3 += a3; c4 += a4; c5 += a5; c6 += a6;
+  } else {
+    cnt += k == 4 ? a4 : k == 5 ? a5 : a6;
+  }
+}
+
 template <int TEAM_WARPS>
 __device__ __forceinline__ void team_sync() {
   if (TEAM_WARPS == 1) __syncwarp();
@@ -640,7 +745,7 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
     const uint32_t x = R[i];
     uint32_t h = (x * 0x9E3779B1u) >> (32 - hbits);
     if (Hv) {
-      h &= GAMMA_KCL_BUCKET4 ? ~3u : ~1u;   // probing starts at a bucket (pair / 4 slots) read in one load
+      h &= ~3u;   // probing starts at a 4-slot bucket read in one load
       while (atomicCAS(&Hv[h], kEmptyId, x) != kEmptyId) h = (h + 1) & hmask;
       H[h] = (unsigned short)i;
     } else {
@@ -683,6 +788,9 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
     uint32_t T;
     const uint32_t o = excl_scan32(cdl, lane, T);
     const uint32_t upto = lane == 31 ? 0xffffffffu : ((2u << lane) - 1u);
+    // element t of the window (t in list i: o_i <= t < o_i + len_i) is
+    // dag_col[cofs_i + t] with cofs_i = beg_i - o_i (mod 2^32; offsets < m < 2^32)
+    const uint32_t cofs = cbeg - o;
     uint32_t nb = 0;   // lists that started before this tile
     // kTiles tiles of 32 elements per step: their loads are issued back to back
     // before any probe, so each lane keeps several L2 gathers in flight
@@ -695,75 +803,56 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
 #pragma unroll
       for (int u = 0; u < kTiles; u++) {
         if ((uint32_t)u >= nt) {
-          y[u] = 0xffffffffu;
+          y[u] = kEmptyId;
           rj[u] = 0;
           continue;
         }
         const uint32_t tb = t0 + 32 * u;
         const uint32_t t = tb + lane;
         // lane t's list = the last list starting at or before t: one OR-reduction of
-        // the start offsets that fall in this tile
-        const uint32_t mine = (lane < (int)nnz && o >= tb && o < tb + 32) ? (1u << (o - tb)) : 0u;
-        const uint32_t S = __reduce_or_sync(0xffffffffu, mine);
-        const int j = (int)(nb + __popc(S & upto)) - 1;
+        // the start offsets that fall in this tile (lanes past the compacted lists hold
+        // o = T: a bit at or above every valid t, so it moves no valid lane's list)
+        const uint32_t d = o - tb;
+        const uint32_t S = __reduce_or_sync(0xffffffffu, d < 32u ? 1u << d : 0u);
+        const uint32_t j = (nb + __popc(S & upto) - 1u) & 31u;
         nb += __popc(S);
-        const uint32_t bj = __shfl_sync(0xffffffffu, cbeg, j & 31);
-        const uint32_t oj = __shfl_sync(0xffffffffu, o, j & 31);
-        rj[u] = __shfl_sync(0xffffffffu, crow, j & 31);
-        y[u] = t < T ? a.dag_col.at<PAGED>((uint64_t)bj + (t - oj)) : 0xffffffffu;
+        const uint32_t off = __shfl_sync(0xffffffffu, cofs, j);
+        rj[u] = __shfl_sync(0xffffffffu, crow, j);
+        y[u] = t < T ? a.dag_col.at<PAGED>((uint64_t)(uint32_t)(off + t)) : kEmptyId;
       }
 #pragma unroll
       for (int u = 0; u < kTiles; u++) {
         if ((uint32_t)u >= nt) break;
         const uint32_t yy = y[u];
         if (Hv) {
-          // one 16-byte load of the 4-slot bucket where y's probe sequence starts; the
-          // compares are predicated, and only a full bucket without y (rare at load
-          // <= 1/4: the pair-slot probe this replaced sent 87 % of warps into the chain
-          // loop, ncu heavy r02) continues the linear probe
-          const bool inr = yy >= rmin && yy <= rmax;   // (the padding 0xffffffff is above every rmax < n)
-          bool hit;
-          uint32_t hh;
-          if (!GAMMA_KCL_BUCKET4) {   // two-slot pair probe
-            const uint32_t h0 = ((yy * 0x9E3779B1u) >> (32 - hbits)) & ~1u;
-            const uint2 vv = *reinterpret_cast<const uint2 *>(Hv + h0);
-            hit = inr && (vv.x == yy || vv.y == yy);
-            hh = vv.x == yy ? h0 : h0 + 1;
-            if (inr && !hit && vv.x != kEmptyId && vv.y != kEmptyId) {
-              for (uint32_t h = (h0 + 2) & hmask;; h = (h + 1) & hmask) {
-                const uint32_t vh = Hv[h];
-                if (vh == yy) {
-                  hit = true;
-                  hh = h;
-                  break;
-                }
-                if (vh == kEmptyId) break;
-              }
-            }
-          } else {
+          // one 16-byte load of the 4-slot bucket where y's probe sequence starts.  The
+          // slots of a bucket are claimed in order (every insertion enters a bucket at
+          // its first slot and moves on only past a taken one), so a free last slot
+          // ends the probe; only a full bucket without y (rare at load <= 1/4) walks on.
+          // The padding id kEmptyId matches the free slots: it is excluded by yy != kEmptyId.
           const uint32_t h0 = ((yy * 0x9E3779B1u) >> (32 - hbits)) & ~3u;
           const uint4 vv = *reinterpret_cast<const uint4 *>(Hv + h0);
-          hit = inr && (vv.x == yy || vv.y == yy || vv.z == yy || vv.w == yy);
-          hh = vv.x == yy ? h0 : vv.y == yy ? h0 + 1 : vv.z == yy ? h0 + 2 : h0 + 3;
-          if (inr && !hit && vv.w != kEmptyId && vv.x != kEmptyId && vv.y != kEmptyId && vv.z != kEmptyId) {
+          bool hit = (vv.x == yy || vv.y == yy || vv.z == yy || vv.w == yy) && yy != kEmptyId;
+          uint32_t hw = 0;   // slot found by the walk
+          if (!hit && vv.w != kEmptyId && yy != kEmptyId) {
             for (uint32_t h = (h0 + 4) & hmask;; h = (h + 1) & hmask) {
               const uint32_t vh = Hv[h];
               if (vh == yy) {
                 hit = true;
-                hh = h;
+                hw = h;
                 break;
               }
               if (vh == kEmptyId) break;
             }
           }
-          }
           if (hit) {
+            const uint32_t hh = vv.x == yy ? h0 : vv.y == yy ? h0 + 1 : vv.z == yy ? h0 + 2 : vv.w == yy ? h0 + 3 : hw;
             const uint32_t e = H[hh];
             atomicOr(&B[rj[u] * W + (e >> 5)], 1u << (e & 31));
           }
           continue;
         }
-        if (yy >= rmin && yy <= rmax) {   // (the padding 0xffffffff is above every rmax < n)
+        if (yy >= rmin && yy <= rmax) {   // (the padding kEmptyId is above every rmax < n)
           uint32_t h = (yy * 0x9E3779B1u) >> (32 - hbits);
           for (;;) {
             const uint32_t e = H[h];
@@ -987,7 +1076,14 @@ __global__ void GAMMA_BM_BOUNDS(KM) kcl_bitmap_kernel(BmArgs a) {
         }
       }
       uint32_t jr = 0;
-      if (TEAM_WARPS == 1 && !deferred)
+      if constexpr (TEAM_WARPS == 1 && KM == 6 && GAMMA_KCL_SM_DFS) {   // state-machine DFS
+        if (!deferred) {
+          if (a.multi)
+            warp_dfs_sm<true>(m.B, m.P, L, W, items, a.k, lane, m.Hv, mc[3], mc[4], mc[5], mc[6], cnt);
+          else
+            warp_dfs_sm<false>(m.B, m.P, L, W, items, a.k, lane, m.Hv, mc[3], mc[4], mc[5], mc[6], cnt);
+        }
+      } else if (TEAM_WARPS == 1 && !deferred)
         for (uint32_t q = tid; q < items; q += kTeamThreads) {
           uint32_t cur[TW];
           item_cur<TW>(m, L, W, BS, q, cur, jr);
