@@ -28,13 +28,13 @@ namespace gamma_impl {
 
 namespace {
 
-// Min resident CTAs per SM for the team kernels with k <= 6 (KM = 6): a register cap
-// (64 -> 51 registers at 5) that trades a few bytes of spill for 40 instead of 32
-// resident warps; measured on B200: C2 -6 %, heavy -18 %.  The k <= 12
-// instances keep 64 registers (their register-resident DFS would spill ~800 B).
+// Min resident CTAs per SM for the team kernels with k <= 6 (KM = 6).  Shared memory
+// (8 warp teams x 6.2 KB, or one CTA team) already limits residency to 4 CTAs, so 4
+// leaves the registers uncapped (64); round 1's 5 (51 registers) predates the 4-slot
+// bucket table and now only spilled (C2 same box: 7.48 ms at 5, 6.46 at 4).
 // Tuning knob: nvcc -DGAMMA_BM_MINB=n.
 #ifndef GAMMA_BM_MINB
-#define GAMMA_BM_MINB 5
+#define GAMMA_BM_MINB 4
 #endif
 #define GAMMA_BM_BOUNDS(KM) __launch_bounds__(256, (KM) <= 6 ? GAMMA_BM_MINB : 1)
 
@@ -45,6 +45,9 @@ namespace {
 // (The slot-pair hash probe lost to the 4-slot bucket, session g, and was removed.)
 #ifndef GAMMA_KCL_LEAF_BAL
 #define GAMMA_KCL_LEAF_BAL 0
+#endif
+#ifndef GAMMA_KCL_PAIR_U   // rows per lane group whose pair searches run in lock step
+#define GAMMA_KCL_PAIR_U 2
 #endif
 #ifndef GAMMA_KCL_SM_DFS   // warp teams, k <= 6: state-machine DFS (0: nested loops per item)
 #define GAMMA_KCL_SM_DFS 1
@@ -707,24 +710,55 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
     const uint32_t j = lane & ((1u << lg) - 1u), rows_per = 32u >> lg;
     const uint32_t rj = j < L ? R[j] : 0u;
     uint64_t elems = 0;
-    for (uint32_t i0 = 0; i0 < L; i0 += rows_per) {
-      const uint32_t i = i0 + (lane >> lg);
-      bool hit = false;
-      if (i < L) {
-        const uint32_t c = R[i];
-        const uint64_t cb = a.dag_ptr[c];
-        const uint32_t dl = (uint32_t)(a.dag_ptr[c + 1] - cb);
-        if (j == 0) elems += dl;
-        hit = j < L && j != i && dl && col_contains<PAGED>(a.dag_col, cb, dl, rj);
-      }
-      // one ballot holds every row of this iteration: row i's bits are its lane group's
-      const uint32_t bal = __ballot_sync(0xffffffffu, hit);
-      const uint32_t bits = lg == 5 ? bal : (bal >> (lane & ~((1u << lg) - 1u))) & ((1u << (1u << lg)) - 1u);
-      if (j == 0 && i < L) {
-        B[i * W] = bits;
+    // kU rows per lane group at once: their binary searches advance in lock step, so a
+    // lane keeps kU independent L2 loads in flight (a run of 17..32 took |R| rounds of
+    // ~log2 d+ dependent loads one row at a time; C2 same box: kU = 1 6.57 ms/step,
+    // 2 6.12, 4 6.44 -- more rows in flight cost registers the DFS needs)
+    constexpr int kU = GAMMA_KCL_PAIR_U;
+    for (uint32_t i0 = 0; i0 < L; i0 += rows_per * kU) {
+      uint64_t cb[kU];
+      uint32_t base[kU], len[kU];
 #pragma unroll
-        for (uint32_t w = 1; w < 4; w++)
-          if (w < W) B[i * W + w] = 0u;
+      for (int u = 0; u < kU; u++) {
+        const uint32_t i = i0 + (u * rows_per) + (lane >> lg);
+        cb[u] = 0;
+        len[u] = 0;
+        base[u] = 0;
+        if (i < L) {
+          const uint32_t c = R[i];
+          cb[u] = a.dag_ptr[c];
+          const uint32_t dl = (uint32_t)(a.dag_ptr[c + 1] - cb[u]);
+          if (j == 0) elems += dl;
+          len[u] = (j < L && j != i) ? dl : 0u;
+        }
+      }
+      // lower-bound search of rj in each list (len 0: no search, no hit)
+      for (;;) {
+        bool more = false;
+#pragma unroll
+        for (int u = 0; u < kU; u++) {
+          if (len[u] > 1) {
+            const uint32_t half = len[u] >> 1;
+            base[u] = a.dag_col.at<PAGED>(cb[u] + base[u] + half) <= rj ? base[u] + half : base[u];
+            len[u] -= half;
+            more |= len[u] > 1;
+          }
+        }
+        if (!__any_sync(0xffffffffu, more)) break;
+      }
+#pragma unroll
+      for (int u = 0; u < kU; u++) {
+        const uint32_t i = i0 + (u * rows_per) + (lane >> lg);
+        const bool hit = len[u] == 1 && a.dag_col.at<PAGED>(cb[u] + base[u]) == rj;
+        // one ballot holds every row of this step: row i's bits are its lane group's
+        const uint32_t bal = __ballot_sync(0xffffffffu, hit);
+        const uint32_t bits = lg == 5 ? bal : (bal >> (lane & ~((1u << lg) - 1u))) & ((1u << (1u << lg)) - 1u);
+        if (j == 0 && i < L) {
+          B[i * W] = bits;
+#pragma unroll
+          for (uint32_t w = 1; w < 4; w++)   // the state-machine DFS reads whole 4-word rows
+            if (w < W) B[i * W + w] = 0u;
+        }
       }
     }
     __syncwarp();
@@ -971,12 +1005,21 @@ __global__ void GAMMA_BM_BOUNDS(KM) kcl_bitmap_kernel(BmArgs a) {
   // root at a time (their roots are the long, costly ones)
   constexpr unsigned long long kBatch = TEAM_WARPS == 1 ? 4 : 1;
   unsigned long long next = 0, end = 0;
+  // warp teams: lane t < kBatch holds root base + t of the batch and its DAG offsets,
+  // all loaded when the batch is taken (one round trip chain per batch, not per root)
+  uint32_t bv = 0;
+  uint64_t bb0 = 0, bb1 = 0;
   for (;;) {
     if (next == end) {
       unsigned long long base = 0;
       if (tid == 0) base = atomicAdd(&a.ctrl[CTRL_WORK], kBatch);
       if (TEAM_WARPS == 1) {
         base = __shfl_sync(0xffffffffu, base, 0);
+        if ((unsigned long long)lane < kBatch && base + lane < a.nroots) {
+          bv = a.roots[base + lane];
+          bb0 = a.dag_ptr[bv];
+          bb1 = a.dag_ptr[bv + 1];
+        }
       } else {
         if (tid == 0) m.slot[0] = base < 0xffffffffull ? (uint32_t)base : 0xffffffffu;
         __syncthreads();
@@ -988,9 +1031,19 @@ __global__ void GAMMA_BM_BOUNDS(KM) kcl_bitmap_kernel(BmArgs a) {
     }
     if (next >= a.nroots) break;
     const unsigned long long gi = next++;
-    const uint32_t v = a.roots[gi];
-    const uint64_t b0 = a.dag_ptr[v];
-    const uint32_t L = (uint32_t)(a.dag_ptr[v + 1] - b0);
+    uint32_t v;
+    uint64_t b0;
+    uint32_t L;
+    if (TEAM_WARPS == 1) {
+      const int t = (int)(gi - (end - kBatch));
+      v = __shfl_sync(0xffffffffu, bv, t);
+      b0 = __shfl_sync(0xffffffffu, bb0, t);
+      L = (uint32_t)(__shfl_sync(0xffffffffu, bb1, t) - b0);
+    } else {
+      v = a.roots[gi];
+      b0 = a.dag_ptr[v];
+      L = (uint32_t)(a.dag_ptr[v + 1] - b0);
+    }
     if (L <= a.len_lo || L > a.len_hi || L < (a.multi ? a.kmin - 1 : a.k - 1)) continue;   // uniform across the team
     const uint32_t W = (L + 31) >> 5, BS = row_stride<TEAM_WARPS, TW>(L);
     if (tid == 0) entries += L;

@@ -25,3 +25,13 @@ for r in rows:
         if "kcl" in d["Kernel Name"]: out.append(d["Metric Value"])
 print("bands (CTA, 65-128, 33-64, 17-32, 9-16, 0-8, parts) ns:", out[-7:])
 PY
+# optional A/B variant library (build.py tag): GAMMA_LIB_VARIANT=$2
+if [ -n "$2" ]; then
+  GAMMA_LIB_VARIANT=$2 timeout 300 python bench.py --no-cpu-baseline --steps 10 > gpurun_out/${TAG}_c2_$2.json 2>/dev/null
+  GAMMA_LIB_VARIANT=$2 timeout 300 python bench.py --no-cpu-baseline --workload heavy --steps 5 > gpurun_out/${TAG}_heavy_$2.json 2>/dev/null
+  python -c "
+import json
+for f in ['gpurun_out/${TAG}_c2_$2.json','gpurun_out/${TAG}_heavy_$2.json']:
+    d=json.load(open(f)); print(f, round(d['ms_per_step'],3), {k:round(v['ms'],2) for k,v in d['kernels'].items()})
+"
+fi
