@@ -81,7 +81,10 @@ def peaks():
 
 
 class ClockSampler:
-    """nvidia-smi clocks + throttle reasons sampled every 200 ms during the timed region."""
+    """nvidia-smi clocks + throttle reasons sampled every 200 ms during the timed region
+    (the profiling recipe's query).  Note: the polling itself stalls host threads that
+    wait on the driver -- C3's batched step (kernel time constant to 0.5 %) took 100-190 ms
+    stalls in some steps with it and none without (--no-clocks, profiles/sm_r02b)."""
     Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
          "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
          "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
@@ -360,6 +363,9 @@ def run_gamma(args):
     lab_pin = None if lab is None else torch.from_numpy(lab.view(np.int32)).pin_memory()
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
     agg = {"_total_launches": {"n": 0}}
+    sm_retries = []   # SM: careful-path reruns per timed step (a chain overflowed its tables)
+    kern_ms = []      # event-timed compute-kernel ms per collect() (diagnostics: GPU vs host time)
+    host_ms = []      # host wall time of each timed step's work() call (diagnostics)
 
     def collect():
         st = ctx.stats()
@@ -368,6 +374,7 @@ def run_gamma(args):
             for key in a:
                 a[key] += c[key]
         agg["_total_launches"]["n"] += st["total_launches"]
+        kern_ms.append(sum(c["ms"] for name, c in st["classes"].items() if name in COMPUTE_CLASSES))
         return st
 
     def build(src, dst, labels, coll):
@@ -407,7 +414,8 @@ def run_gamma(args):
                 for (q, lname, nv, e, plab), (cnt, _) in zip(runs, got):
                     results[f"{q}/{lname}"] = cnt
                 if coll:
-                    collect()
+                    st = collect()
+                    sm_retries.append(st.get("retries"))
             emb = sum(results.values())
         else:
             pats = g.fpm_array(w["l"], w["minsup"])   # the result records, no per-pattern Python objects
@@ -456,7 +464,9 @@ def run_gamma(args):
         torch.cuda.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
+        h0 = time.perf_counter()
         emb, results = work(g, True)
+        host_ms.append(1e3 * (time.perf_counter() - h0))
         e1.record(stream)
         torch.cuda.synchronize()
         barrier()
@@ -576,6 +586,9 @@ def run_gamma(args):
                         "samples in HBM runs before each step, untimed (build_ms_per_step), then L2 is flushed; "
                         "e2e includes H2D + build",
         "step_ms": [round(x, 3) for x in times],
+        **({"sm_retries_per_step": sm_retries} if sm_retries else {}),
+        "step_kernel_ms": [round(x, 3) for x in kern_ms if x > 0],
+        "step_host_ms": [round(x, 3) for x in host_ms],
         "rank_time_max_over_mean": imbalance,
         "e2e_step_ms": [round(x, 3) for x in e2e_times],
     }

@@ -87,14 +87,15 @@ void *gamma_ctx::keep_take(size_t bytes, size_t &got) {
   return alloc(bytes);
 }
 
-// Kept bytes are capped (kKeepCap): beyond it a returned buffer is freed instead.
-static constexpr size_t kKeepCap = 8ull << 30;
-
+// Kept bytes are capped at a quarter of the device memory: beyond it a returned buffer
+// is freed instead.  (Round 1's 8 GiB held a fraction of a batched SM call's tables --
+// eight level chains of up to three levels -- so every C3 step re-allocated most of
+// them through the caching allocator.)
 void gamma_ctx::keep_give(void *p, size_t bytes) {
   if (!p) return;
   size_t held = 0;
   for (auto &b : kept) held += b.second;
-  if (held + bytes > kKeepCap) {
+  if (held + bytes > mem_total / 4) {
     free(p);
     return;
   }
@@ -104,6 +105,14 @@ void gamma_ctx::keep_give(void *p, size_t bytes) {
 void gamma_ctx::keep_release() {
   for (auto &b : kept) free(b.first);
   kept.clear();
+}
+
+// Before a graph build: release the kept buffers only when less than half of the
+// device memory is free (the build's scratch scales with the input).
+void gamma_ctx::keep_release_if_tight() {
+  if (kept.empty()) return;
+  size_t fr = 0, tot = 0;
+  if (cudaMemGetInfo(&fr, &tot) != cudaSuccess || fr < tot / 2) keep_release();
 }
 
 void gamma_ctx::free(void *p) {
@@ -185,6 +194,7 @@ gamma_status gamma_ctx_create(const gamma_ctx_desc *desc, gamma_ctx **out) {
       cudaDeviceProp prop;
       GAMMA_CUDA(cudaGetDeviceProperties(&prop, c->device));
       c->num_sms = prop.multiProcessorCount;
+      c->mem_total = prop.totalGlobalMem;
       c->smem_optin = prop.sharedMemPerBlockOptin;
       if (desc->stream) {
         c->stream = (cudaStream_t)desc->stream;
@@ -255,7 +265,7 @@ gamma_status gamma_load_edges(gamma_ctx *ctx, uint32_t n, const uint32_t *src, c
     GAMMA_REQUIRE(n < 0xFFFFFFFFu, GAMMA_E_INVAL, "gamma_load_edges: n too large");
     GAMMA_CUDA(cudaSetDevice(ctx->device));
     ctx->reset_stats();
-    ctx->keep_release();   // the build's scratch is sized from the input, not from kept buffers
+    ctx->keep_release_if_tight();   // the build needs room; kept SM tables only when it is there
     auto *g = new gamma_graph();
     g->ctx = ctx;
     g->n = n;
@@ -281,7 +291,7 @@ gamma_status gamma_load_csr(gamma_ctx *ctx, uint32_t n, const uint64_t *row_ptr,
     GAMMA_REQUIRE(n > 0 && n < 0xFFFFFFFFu, GAMMA_E_INVAL, "gamma_load_csr: bad n");
     GAMMA_CUDA(cudaSetDevice(ctx->device));
     ctx->reset_stats();
-    ctx->keep_release();
+    ctx->keep_release_if_tight();
     auto *g = new gamma_graph();
     g->ctx = ctx;
     g->n = n;
@@ -315,10 +325,9 @@ void gamma_graph_free(gamma_graph *g) {
     c->free(g->ldeg);
     c->free(g->dag_pages);
     c->free(g->dag_cache);
-    try {
-      c->keep_release();   // kept SM tables were sized for this graph
-    } catch (...) {
-    }
+    // (kept SM tables stay with the context: their sizes come from the budget and the
+    // level caps, not from this graph, and the next graph's SM calls take them back
+    // without an allocator round trip)
     cudaStreamSynchronize(c->stream);
   }
   if (g->dag_host) cudaFreeHost(g->dag_host);

@@ -82,6 +82,7 @@ struct gamma_ctx {
   gamma_ctx_desc desc;
   int device = 0;
   int num_sms = 148;
+  size_t mem_total = 0;   // device memory (bytes), read once at creation
   size_t smem_optin = 0;
   cudaStream_t stream = nullptr;
   bool own_stream = false;
@@ -112,6 +113,7 @@ struct gamma_ctx {
   void *keep_take(size_t bytes, size_t &got);   // smallest kept buffer >= bytes, else alloc
   void keep_give(void *p, size_t bytes);
   void keep_release();                          // free every kept buffer
+  void keep_release_if_tight();                 // ... when less than half the HBM is free
   void reset_stats();
   // Launch helper: brackets the launch with events when timing is on.
   template <class F>

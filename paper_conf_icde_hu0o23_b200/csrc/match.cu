@@ -29,6 +29,8 @@
 #include <cub/device/device_select.cuh>
 
 #include <algorithm>
+#include <chrono>
+#include <cstdio>
 #include <cstdlib>
 #include <cstring>
 #include <memory>
@@ -50,6 +52,9 @@ constexpr uint32_t kOutCap = 512;    // default staged child run per warp (u32);
 // sets the CTAs per SM; GAMMA_SM_LMCAP / GAMMA_SM_OUTCAP override them for tuning;
 // C3 sweep on B200: 512/512 233 ms, 256/256 243, 1024/512 272, 2048/512 338 per step)
 constexpr uint32_t kLongRatio = 1;   // see SmArgs::long_ratio (GAMMA_SM_LONGRATIO overrides; 0 = off)
+#ifndef GAMMA_SM_CAP_LOG2   // first entry-table size of an SM level (log2 slots)
+#define GAMMA_SM_CAP_LOG2 27
+#endif
 constexpr uint32_t kBlkV = 4096;
 constexpr uint32_t kBlkG = 256;      // descriptors per warp block
 constexpr uint32_t kSlice = 64;      // children per group descriptor when the count level consumes them
@@ -97,6 +102,8 @@ struct SmArgs {
   uint32_t stage;           // 0: never stage L_m (debug)
   uint32_t *lm_scratch;     // per-warp global L_m slices for hub prefixes (nullable)
   uint32_t lm_scratch_cap;  // entries per warp slice
+  uint32_t *big_scratch;    // per-warp global slices for child runs above out_cap (nullable)
+  uint32_t big_scratch_cap; // entries per warp slice
   uint32_t lm_cap, out_cap; // shared-memory staging per warp (u32 entries)
   uint32_t slice;           // children per group descriptor of the next level
   uint32_t long_ratio;      // last level: child lists > long_ratio * |L_m| are probed from L_m (0: off)
@@ -467,14 +474,18 @@ __global__ void __launch_bounds__(kThreads, 5) sm_kernel(SmArgs a) {
                                      staged ? (1u << d) : (prefix_mask | (1u << d)));
         uint32_t found;
         uint64_t pos = 0;
-        bool big = false;
+        bool big = false, via_scratch = false;
+        uint32_t *const bsc =
+            a.big_scratch ? a.big_scratch + (uint64_t)(blockIdx.x * kWarps + wid) * a.big_scratch_cap : nullptr;
         if (staged && !child_in_b) {
           // candidates = L_m minus position-d filters (all prefix filters applied); a
-          // run longer than the staging buffer is written straight to the level
+          // run longer than the staging buffer goes to the warp's global slice (or,
+          // without one, straight to lm_len reserved slots of the level)
           found = 0;
           big = !last && lm_len > a.out_cap;
-          if (big && !pool_reserve(pv, lm_len, lane, pos)) { stop = true; break; }
-          uint32_t *dst = big ? a.vid_out + pos : sout;
+          via_scratch = big && bsc && lm_len <= a.big_scratch_cap;
+          if (big && !via_scratch && !pool_reserve(pv, lm_len, lane, pos)) { stop = true; break; }
+          uint32_t *dst = via_scratch ? bsc : big ? a.vid_out + pos : sout;
           const uint64_t cs = a.rp[c];
           const uint32_t cl = anti_d ? (uint32_t)(a.rp[c + 1] - cs) : 0u;
           for (uint32_t j0 = 0; j0 < lm_len; j0 += 32) {
@@ -499,13 +510,17 @@ __global__ void __launch_bounds__(kThreads, 5) sm_kernel(SmArgs a) {
               ub = min(ub, gdeg(a, phi[j]));
             }
             big = ub > a.out_cap;
-            if (big && !pool_reserve(pv, ub, lane, pos)) { stop = true; break; }
+            // a run that may not fit the staging buffer goes to the warp's global slice
+            // (then exactly `found` pool slots); without one, to ub reserved pool slots
+            via_scratch = big && a.big_scratch && ub <= a.big_scratch_cap;
+            if (big && !via_scratch && !pool_reserve(pv, ub, lane, pos)) { stop = true; break; }
           }
           if (last)
             found = sm_intersect<false>(a, q, lists, phi, bc, last, staged ? lm : nullptr, lm_len, nullptr, 0, lane);
           else
             found = sm_intersect<true>(a, q, lists, phi, bc, last, staged ? lm : nullptr, lm_len,
-                                       big ? a.vid_out + pos : sout, big ? 0xffffffffu : a.out_cap, lane);
+                                       via_scratch ? bsc : big ? a.vid_out + pos : sout,
+                                       big ? 0xffffffffu : a.out_cap, lane);
         }
         if (last) {
           acc += found;
@@ -513,12 +528,30 @@ __global__ void __launch_bounds__(kThreads, 5) sm_kernel(SmArgs a) {
         }
         if (found == 0) continue;
         __syncwarp();
-        if (!big) {
-          if (!wb_reserve(wv, pv, found, lane, pos)) { stop = true; break; }
-          for (uint32_t t = lane; t < found; t += 32) a.vid_out[pos + t] = sout[t];
+        if (via_scratch) {   // exactly the survivors into the pool (one coalesced copy)
+          if (!pool_reserve(pv, found, lane, pos)) { stop = true; break; }
+          for (uint32_t t = lane; t < found; t += 32) a.vid_out[pos + t] = bsc[t];
         }
         // descriptors: slices of kSlice children, each carrying the prefix + c
         const uint32_t slice = a.slice;
+        // the run may split at a slice boundary: whole slices fill the rest of the warp's
+        // block (pos), the others go to a fresh one (pos2) -- abandoning the rest instead
+        // wasted up to a run per block (C3: 7x the entries written, GAMMA_DEBUG)
+        uint32_t first = found;
+        uint64_t pos2 = 0;
+        if (!big) {
+          const uint64_t rest = wv.e - wv.b;
+          first = (uint32_t)(rest / slice * slice < found ? rest / slice * slice : found);
+          if (first == found) {
+            pos = wv.b;
+            wv.b += found;
+          } else {
+            pos = wv.b;
+            wv.b += first;
+            if (!wb_reserve(wv, pv, found - first, lane, pos2)) { stop = true; break; }
+          }
+          for (uint32_t t = lane; t < found; t += 32) a.vid_out[t < first ? pos + t : pos2 + (t - first)] = sout[t];
+        }
         const uint32_t ns = (found + slice - 1) / slice;
         uint64_t gpos;
         if (ns <= kBlkG)
@@ -529,7 +562,7 @@ __global__ void __launch_bounds__(kThreads, 5) sm_kernel(SmArgs a) {
           uint32_t *o = a.desc_out + (gpos + s) * a.dw_out;
           if (lane < (int)a.dw_out) {
             uint32_t val;
-            if (lane == 0) val = (uint32_t)(pos + s * slice);
+            if (lane == 0) val = (uint32_t)(s * slice < first ? pos + s * slice : pos2 + (s * slice - first));
             else if (lane == 1) val = min(slice, found - s * slice);
             else val = phi[0];
 #pragma unroll
@@ -781,16 +814,39 @@ struct SmRun {
   uint32_t stage = 1;
   DevBuf<uint32_t> lm_scratch;       // per-warp global L_m slices (hub prefixes)
   uint32_t lm_scratch_cap = 0;
+  DevBuf<uint32_t> big_scratch;      // per-warp global slices for child runs above out_cap
+  uint32_t big_scratch_cap = 0;
 
-  bool grow(uint32_t d, uint64_t want_v) {
+  // First table size of a level (grow caps it at the level's share of the HBM budget):
+  // 2^29 entry slots, 2^26 group descriptors.  Slots run well ahead of the entries
+  // written: a child whose run may exceed the warp's staging buffer reserves its upper
+  // bound (the shortest list involved) and keeps what survives (C3, 4-cycle, labels
+  // i mod 8, GAMMA_DEBUG: the pool cursor at 2.8e8 slots for 5.1e7 entries).  Round 1's
+  // 2^24 overflowed there in every call, so the one-read-back chain was thrown away and
+  // the query rerun on the careful per-level path.
+  uint64_t initial_cap() const {
+    return std::max<uint64_t>(1ull << GAMMA_SM_CAP_LOG2, 4ull * kBlkV * kWarps * (uint64_t)grid);
+  }
+
+  // Tables of level d for want_v entries and want_g group descriptors (0: cap_v / 8),
+  // never smaller than they are, scaled down together to the level's share of the HBM
+  // budget.  Returns false when nothing grew.
+  bool grow(uint32_t d, uint64_t want_v, uint64_t want_g = 0) {
     SmLevel &L = lv[d];
     const uint32_t dw = 2 + d;
-    const uint64_t per_slot = 4 + (uint64_t)dw * 4 / 8;   // cap_g = cap_v / 8
-    uint64_t cv = std::max<uint64_t>(want_v, 1ull << 16);
-    cv = std::min<uint64_t>(cv, level_share / per_slot);
+    uint64_t cv = std::max<uint64_t>(std::max<uint64_t>(want_v, 1ull << 16), L.cap_v);
+    uint64_t cg = std::max<uint64_t>(std::max<uint64_t>(cv / 8, want_g), L.cap_g);
+    const double bytes = 4.0 * cv + 4.0 * dw * cg;
+    if (bytes > (double)level_share) {
+      const double f = (double)level_share / bytes;
+      cv = (uint64_t)(cv * f);
+      cg = (uint64_t)(cg * f);
+    }
     cv = std::min<uint64_t>(cv, 0xFFFFFFFFull - kBlkV);
-    if (cv <= L.cap_v) return false;
-    const uint64_t cg = cv / 8 + 2 * kBlkG;
+    cg = std::max<uint64_t>(cg, 2 * kBlkG);
+    if (cv <= L.cap_v && cg <= L.cap_g) return false;
+    cv = std::max<uint64_t>(cv, L.cap_v);
+    cg = std::max<uint64_t>(cg, L.cap_g);
     // the superseded (smaller) tables are freed, not kept: keeping them would hold
     // ~1/3 more than level_share per level and shrink later budgets
     L.vid.kept = false;
@@ -825,6 +881,8 @@ struct SmRun {
     a.stage = stage;
     a.lm_scratch = lm_scratch.p;
     a.lm_scratch_cap = lm_scratch_cap;
+    a.big_scratch = big_scratch.p;
+    a.big_scratch_cap = big_scratch_cap;
     a.lm_cap = sm_lm_cap();
     a.out_cap = sm_out_cap();
     a.long_ratio = sm_long_ratio();
@@ -871,7 +929,7 @@ struct SmRun {
   void chain_enqueue(uint64_t ngroups, cudaStream_t st, unsigned long long *ctrl, uint64_t *host) {
     const uint32_t nl = P.nv - 1;   // launches: d = 0 .. nv-2
     for (uint32_t q = 1; q < nl; q++)
-      if (lv[q].cap_v == 0) grow(q, std::max<uint64_t>(1ull << 24, 4ull * kBlkV * kWarps * (uint64_t)grid));
+      if (lv[q].cap_v == 0) grow(q, initial_cap(), 1ull << 26);
     GAMMA_CUDA(cudaMemsetAsync(ctrl, 0, CTRL_WORDS * sizeof(uint64_t), st));
     for (uint32_t d = 0; d < nl; d++) {
       const uint32_t q = d + 1;
@@ -904,7 +962,14 @@ struct SmRun {
       // hint for the careful path: grow the tables that ran out
       for (uint32_t d = 0; d + 1 < nl; d++) {
         const uint64_t *b = h + CTRL_LEVELS + CTRL_LSTRIDE * d;
-        if (b[CTRL_VCUR] > lv[d + 1].cap_v) grow(d + 1, b[CTRL_VCUR]);
+        // (a cursor past its capacity: that pool ran out -- entries or group descriptors)
+        const bool ov = b[CTRL_VCUR] > lv[d + 1].cap_v, og = b[CTRL_GCUR] > lv[d + 1].cap_g;
+        if (getenv("GAMMA_DEBUG"))
+          fprintf(stderr, "[gamma sm chain] nv %u level %u: entries %llu / %llu, groups %llu / %llu, share %llu\n",
+                  P.nv, d + 1, (unsigned long long)b[CTRL_VCUR], (unsigned long long)lv[d + 1].cap_v,
+                  (unsigned long long)b[CTRL_GCUR], (unsigned long long)lv[d + 1].cap_g,
+                  (unsigned long long)level_share);
+        if (ov || og) grow(d + 1, ov ? 2 * b[CTRL_VCUR] : 0, og ? 2 * b[CTRL_GCUR] : 0);
       }
       return false;
     }
@@ -939,7 +1004,7 @@ struct SmRun {
     }
     for (;;) {
       SmLevel &L = lv[q];
-      if (L.cap_v == 0) grow(q, std::max<uint64_t>(1ull << 24, 4ull * kBlkV * kWarps * (uint64_t)grid));
+      if (L.cap_v == 0) grow(q, initial_cap(), 1ull << 26);
       SmArgs a = args(d, g0, g1);
       a.vid_out = L.vid.p;
       a.desc_out = L.desc.p;
@@ -955,7 +1020,8 @@ struct SmRun {
         return;
       }
       ctx->stats.retries++;
-      if (grow(q, std::max<uint64_t>(h[CTRL_VCUR], L.cap_v) * 4)) continue;
+      if (grow(q, std::max<uint64_t>(h[CTRL_VCUR], L.cap_v) * 4, std::max<uint64_t>(h[CTRL_GCUR], L.cap_g) * 4))
+        continue;
       GAMMA_REQUIRE(g1 - g0 > 1, GAMMA_E_NOMEM, "HBM budget too small for one embedding group (SM)");
       const uint64_t mid = g0 + (g1 - g0) / 2;
       process(d, g0, mid);
@@ -1324,6 +1390,13 @@ static bool match_prepare(gamma_graph *g, const SmPlan &P, SmRun &R, uint64_t &c
     R.lm_scratch_cap = std::min<uint32_t>(g->max_degree, 1u << 16);
     R.lm_scratch = DevBuf<uint32_t>(ctx, (uint64_t)R.grid * kWarps * R.lm_scratch_cap, true);
   }
+  if (P.nv > 2 && g->max_degree > sm_out_cap()) {
+    // a child run above the staging buffer is bounded by a list length (<= max degree):
+    // kept in the warp's slice, then copied to exactly `found` pool slots (reserving the
+    // bound in the pool ran its cursor 5x past the entries written on C3)
+    R.big_scratch_cap = std::min<uint32_t>(g->max_degree, 1u << 16);
+    R.big_scratch = DevBuf<uint32_t>(ctx, (uint64_t)R.grid * kWarps * R.big_scratch_cap, true);
+  }
   ngroups = ngr;
   return false;
 }
@@ -1361,12 +1434,22 @@ static void match_batch(gamma_graph *g, const std::vector<SmPlan> &Ps, std::vect
   std::vector<std::unique_ptr<SmRun>> runs(nq);
   std::vector<uint64_t> ngr(nq, 0);
   std::vector<bool> done(nq, false);
+  const bool dbg = getenv("GAMMA_DEBUG") != nullptr;   // host wall time of the phases
+  auto now = [] { return std::chrono::steady_clock::now(); };
+  auto ms = [](std::chrono::steady_clock::time_point a, std::chrono::steady_clock::time_point b) {
+    return std::chrono::duration<double, std::milli>(b - a).count();
+  };
+  const auto t0 = now();
+  std::vector<double> tprep(nq, 0.0);
   for (size_t i = 0; i < nq; i++) {
+    const auto ti = now();
     runs[i].reset(new SmRun());
     uint64_t c = 0;
     done[i] = match_prepare(g, Ps[i], *runs[i], c, ngr[i], (uint32_t)std::min<size_t>(nq, gamma_ctx::kMaxBatch));
     if (done[i]) counts[i] = c;
+    tprep[i] = ms(ti, now());
   }
+  const auto t1 = now();
   ctx->side_init();
   cudaEvent_t ready;
   GAMMA_CUDA(cudaEventCreateWithFlags(&ready, cudaEventDisableTiming));
@@ -1382,7 +1465,9 @@ static void match_batch(gamma_graph *g, const std::vector<SmPlan> &Ps, std::vect
     runs[i]->chain_enqueue(ngr[i], st, (unsigned long long *)(ctx->side_ctrl + (size_t)sl * CTRL_WORDS),
                            ctx->side_ctrl_host + (size_t)sl * CTRL_WORDS);
   }
+  const auto t2 = now();
   for (int sl = 0; sl < used; sl++) GAMMA_CUDA(cudaStreamSynchronize(ctx->side_streams[sl]));
+  const auto t3 = now();
   cudaEventDestroy(ready);
   for (size_t i = 0; i < nq; i++) {
     if (done[i]) continue;
@@ -1396,6 +1481,11 @@ static void match_batch(gamma_graph *g, const std::vector<SmPlan> &Ps, std::vect
   }
   ctx->sync();
   ctx->collect_timings();
+  if (dbg) {
+    fprintf(stderr, "[gamma sm batch] prepare %.2f ms (", ms(t0, t1));
+    for (size_t i = 0; i < nq; i++) fprintf(stderr, "%s%.2f", i ? " " : "", tprep[i]);
+    fprintf(stderr, "), enqueue %.2f, wait %.2f, collect %.2f ms\n", ms(t1, t2), ms(t2, t3), ms(t3, now()));
+  }
 }
 
 }  // namespace gamma_impl
@@ -1431,7 +1521,11 @@ extern "C" gamma_status gamma_match_batch(gamma_graph *g, uint32_t n, const gamm
     GAMMA_CUDA(cudaSetDevice(c->device));
     c->reset_stats();
     std::vector<uint64_t> r;
+    const auto tb = std::chrono::steady_clock::now();
     match_batch(g, Ps, r);
+    if (getenv("GAMMA_DEBUG"))
+      fprintf(stderr, "[gamma sm batch] call %.2f ms (incl. table release)\n",
+              std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - tb).count());
     if (c->desc.world > 1 && c->desc.allreduce_sum_u64 && n) {
       gamma_status st = c->desc.allreduce_sum_u64(r.data(), n, c->desc.coll_user);
       GAMMA_REQUIRE(st == GAMMA_OK, st, "allreduce_sum_u64 callback failed");
