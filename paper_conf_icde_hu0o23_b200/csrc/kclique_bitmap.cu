@@ -49,6 +49,12 @@ namespace {
 #ifndef GAMMA_KCL_PAIR_U   // rows per lane group whose pair searches run in lock step
 #define GAMMA_KCL_PAIR_U 2
 #endif
+// GAMMA_KCL_PAIR_SORT: runs <= 32 sorted by (degree, id) in the warp, only the pairs above
+// the diagonal searched (half the searches, one more gather round trip and the sort;
+// C2 same box 6.20 vs 6.14 ms/step, heavy 40.2 vs 40.5: off)
+#ifndef GAMMA_KCL_PAIR_SORT
+#define GAMMA_KCL_PAIR_SORT 0
+#endif
 #ifndef GAMMA_KCL_SM_DFS   // warp teams, k <= 6: state-machine DFS (0: nested loops per item)
 #define GAMMA_KCL_SM_DFS 1
 #endif
@@ -113,6 +119,8 @@ struct BmArgs {
   uint32_t trim;              // trim each child's list at the run's largest id (GAMMA_KCL_NO_TRIM: off)
   uint32_t *wide_rows;        // wide runs: per-CTA global row scratch (wide_stride words each)
   uint64_t wide_stride;
+  const uint64_t *row_ptr;    // symmetric CSR offsets (degrees of the orientation order);
+                              // nullptr in rank space, where the id order is that order
 };
 
 __device__ __forceinline__ uint32_t excl_scan32(uint32_t x, int lane, uint32_t &total) {
@@ -703,6 +711,105 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
   // probe sum |N+(c)| elements (C2, |R| <= 32: 1.2e8 pairs vs 5.7e8 elements,
   // scratch/pair_cost.py) -- and no hash table.  The rows of 32 / |R|' consecutive
   // lanes (|R|' = |R| rounded up to a power of two) come out of one ballot.
+  if (GAMMA_KCL_PAIR_SORT && TEAM_WARPS == 1 && L <= 32 && !GAMMA_KCL_NO_PAIRS) {
+    // The run sorted by the orientation order (degree, id) first (a warp bitonic sort
+    // of 64-bit keys): then bit j of row i can only be set for j > i, so only the
+    // |R|(|R|-1)/2 pairs above the diagonal are searched -- rows i and |R|-2-i share a
+    // lane group (their |R|-1-i and i+1 candidates fill |R| lanes).  The DFS does not
+    // care how R is ordered.
+    constexpr uint32_t kFull = 0xffffffffu;
+    uint32_t x = kEmptyId, dlx = 0, dgx = 0;
+    uint64_t cbx = 0;
+    if (lane < (int)L) x = a.dag_col.at<PAGED>(b0 + lane);
+    if (lane < (int)L) {
+      cbx = a.dag_ptr[x];
+      dlx = (uint32_t)(a.dag_ptr[x + 1] - cbx);
+      if (a.row_ptr) dgx = (uint32_t)(a.row_ptr[x + 1] - a.row_ptr[x]);
+    }
+    uint64_t key = lane < (int)L ? ((uint64_t)dgx << 32 | x) : ~0ull;
+    uint32_t src = lane;
+#pragma unroll
+    for (uint32_t k = 2; k <= 32; k <<= 1)
+#pragma unroll
+      for (uint32_t jj = k >> 1; jj > 0; jj >>= 1) {
+        const uint64_t ok = __shfl_xor_sync(kFull, key, jj);
+        const uint32_t os = __shfl_xor_sync(kFull, src, jj);
+        const bool keep_min = ((lane & k) == 0) == ((lane & jj) == 0);
+        if (keep_min ? ok < key : ok > key) {
+          key = ok;
+          src = os;
+        }
+      }
+    const uint64_t cbs = __shfl_sync(kFull, cbx, src);
+    const uint32_t dls = __shfl_sync(kFull, dlx, src);
+    const uint32_t xs = (uint32_t)key;   // lane p: the p-th vertex of the sorted run
+    if (lane < (int)L) R[lane] = xs;
+    uint64_t elems = lane < (int)L ? dls : 0u;
+    const uint32_t lg = L <= 2 ? 1u : L <= 4 ? 2u : L <= 8 ? 3u : L <= 16 ? 4u : 5u;
+    const uint32_t t = lane & ((1u << lg) - 1u), groups = 32u >> lg, gbase = lane & ~((1u << lg) - 1u);
+    const uint32_t npairs = L / 2;   // row pairs (p, |R|-2-p); row |R|-1 has no candidate
+    constexpr int kU = GAMMA_KCL_PAIR_U;
+    for (uint32_t p0 = 0; p0 < npairs; p0 += groups * kU) {
+      uint64_t cb[kU];
+      uint32_t base[kU], len[kU], yv[kU];
+#pragma unroll
+      for (int u = 0; u < kU; u++) {
+        const uint32_t pp = p0 + u * groups + (lane >> lg);
+        const uint32_t first = L - 1 - pp;   // candidates of row pp (j = pp + 1 + t)
+        const uint32_t r = t < first ? pp : L - 2 - pp;
+        const uint32_t j = t < first ? pp + 1 + t : t;
+        const bool on = pp < npairs && t < L && (t < first || r != pp);
+        const uint64_t cr = __shfl_sync(kFull, cbs, r & 31);
+        const uint32_t dr = __shfl_sync(kFull, dls, r & 31);
+        yv[u] = __shfl_sync(kFull, xs, j & 31);
+        cb[u] = cr;
+        base[u] = 0;
+        len[u] = on ? dr : 0u;
+      }
+      for (;;) {
+        bool more = false;
+#pragma unroll
+        for (int u = 0; u < kU; u++) {
+          if (len[u] > 1) {
+            const uint32_t half = len[u] >> 1;
+            base[u] = a.dag_col.at<PAGED>(cb[u] + base[u] + half) <= yv[u] ? base[u] + half : base[u];
+            len[u] -= half;
+            more |= len[u] > 1;
+          }
+        }
+        if (!__any_sync(kFull, more)) break;
+      }
+#pragma unroll
+      for (int u = 0; u < kU; u++) {
+        const uint32_t pp = p0 + u * groups + (lane >> lg);
+        const bool hit = len[u] == 1 && a.dag_col.at<PAGED>(cb[u] + base[u]) == yv[u];
+        const uint32_t bal = __ballot_sync(kFull, hit);
+        const uint32_t gb = lg == 5 ? bal : (bal >> gbase) & ((1u << (1u << lg)) - 1u);
+        if (t == 0 && pp < npairs) {
+          const uint32_t first = L - 1 - pp, r = L - 2 - pp;
+          const uint32_t lowm = (1u << first) - 1u;
+          B[pp * W] = (gb & lowm) << (pp + 1);
+          if (r != pp) B[r * W] = gb & ~lowm;
+#pragma unroll
+          for (uint32_t w = 1; w < 4; w++)   // the state-machine DFS reads whole 4-word rows
+            if (w < W) {
+              B[pp * W + w] = 0u;
+              B[r * W + w] = 0u;
+            }
+        }
+      }
+    }
+    if (lane == 0) {   // the last row: no candidate after it
+      B[(L - 1) * W] = 0u;
+#pragma unroll
+      for (uint32_t w = 1; w < 4; w++)
+        if (w < W) B[(L - 1) * W + w] = 0u;
+    }
+    __syncwarp();
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) elems += __shfl_down_sync(kFull, elems, off);
+    return lane == 0 ? elems : 0u;
+  }
   if (TEAM_WARPS == 1 && L <= 32 && !GAMMA_KCL_NO_PAIRS) {
     if (lane < (int)L) R[lane] = a.dag_col.at<PAGED>(b0 + lane);
     __syncwarp();
@@ -1582,6 +1689,7 @@ uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint6
   gamma_ctx *ctx = g->ctx;
   BmArgs a{};
   a.dag_ptr = g->dag_ptr;
+  a.row_ptr = g->rank_space ? nullptr : g->row_ptr;
   a.dag_col = DagCol{g->dag_col, g->dag_pages};
   a.roots = roots;
   a.nroots = nroots;
