@@ -170,30 +170,41 @@ def load_traffic(workload: str, kernel_class: str):
 
 def issue_roofline(workload: str, kernel_class: str, ms_per_launch: float, clk: dict):
     """The ceiling that binds an L2-resident, integer path: instruction issue.  Warp
-    instructions per launch (committed ncu --set full summary of this workload's
-    dominant class, profiles/ncu_<workload>_<class>.json: smsp__inst_executed.sum over
-    the class's launches of one step, averaged) / (148 SMs x 4 schedulers x SM clock x
-    the live event-timed ms per launch).  1.0 = every scheduler issues every cycle."""
-    p = os.path.join(ROOT, "profiles", f"ncu_{workload}_{kernel_class}.json")
-    if not os.path.exists(p):
+    instructions per launch (committed ncu --set full summaries of this workload's
+    dominant class, profiles/ncu_<workload>_<class>[_*].json -- e.g. the kCL hub-part
+    kernel is summarised apart from the team kernels but is a launch of the same class:
+    smsp__inst_executed.sum over the captured launches of one step / their number) /
+    (148 SMs x 4 schedulers x SM clock x the live event-timed ms per launch).  1.0 =
+    every scheduler issues every cycle."""
+    import glob
+    files = sorted(glob.glob(os.path.join(ROOT, "profiles", f"ncu_{workload}_{kernel_class}.json")) +
+                   glob.glob(os.path.join(ROOT, "profiles", f"ncu_{workload}_{kernel_class}_*.json")))
+    inst_total, launches, thr_w, srcs = 0.0, 0, 0.0, []
+    for p in files:
+        try:
+            j = json.load(open(p))
+        except (OSError, ValueError):
+            continue
+        inst, nl = j.get("inst_executed_per_launch"), j.get("launches_captured") or 0
+        if not inst or not nl:
+            continue
+        inst_total += inst * nl
+        launches += nl
+        thr_w += (j.get("threads_per_warp_inst") or 0) * inst * nl
+        srcs.append(os.path.relpath(p, ROOT))
+    if not launches:
         return None
-    try:
-        j = json.load(open(p))
-    except (OSError, ValueError):
-        return None
-    inst = j.get("inst_executed_per_launch")
-    if not inst:
-        return None
+    inst = inst_total / launches
     mhz = (clk or {}).get("sm_mhz") or (clk or {}).get("sm_max_mhz") or 1965.0
     peak = 148 * 4 * mhz * 1e6                     # warp instructions / s
     achieved = inst / (ms_per_launch / 1000.0)
     if achieved > peak:   # the committed summary predates the kernel that ran: no claim
         return {"bound": "issue", "achieved": None, "peak": peak, "unit": "warp-inst/s", "frac": None,
-                "stale": f"{os.path.relpath(p, ROOT)} counts more instructions than this launch time can issue; "
-                         "re-capture it for this build"}
+                "stale": f"{srcs} count more instructions than this launch time can issue; "
+                         "re-capture them for this build"}
     return {"bound": "issue", "achieved": achieved, "peak": peak, "unit": "warp-inst/s", "frac": achieved / peak,
-            "inst_per_launch": inst, "sm_mhz": mhz, "threads_per_inst": j.get("threads_per_warp_inst"),
-            "source": os.path.relpath(p, ROOT)}
+            "inst_per_launch": inst, "sm_mhz": mhz, "threads_per_inst": thr_w / inst_total if inst_total else None,
+            "source": srcs}
 
 
 def load_alg_bytes(workload: str):

@@ -49,6 +49,9 @@ namespace gamma_impl {
 namespace {
 
 constexpr int kThreads = 256;
+#ifndef GAMMA_FPM_MEMO   // level-3 per-warp memo of (prefix, edge mask, new label) -> domains (0: off)
+#define GAMMA_FPM_MEMO 1
+#endif
 
 // Pattern code packed in one word (0 = empty slot):
 //   bits 0..47 four 12-bit labels (canonical order), 48..50 nv, 51..52 ne,
@@ -239,24 +242,11 @@ __device__ __forceinline__ uint32_t pick4(uint32_t i, uint32_t v0, uint32_t v1, 
 // k0..k3: the in-class ranks (lrank) of the local vertices -- the enumeration loads the
 // root edge's once per edge, a prefix's third once per prefix, only a new fourth vertex
 // per embedding.
-__device__ void record(const FpmArgs &a, const uint2 *tab, const uint32_t *prm, uint32_t k0, uint32_t k1,
-                       uint32_t k2, uint32_t k3, uint32_t l0, uint32_t l1, uint32_t l2, uint32_t l3, uint32_t nv,
-                       uint32_t em) {
-  const Canon cn = canonical(tab, l0, l1, l2, l3, nv, em);
-  unsigned long long d = 0;
-  const int64_t s = table_slot(a, cn.key, true, d);
-  if (s < 0) return;
-  // the claimer may still be carving this slot's domains (a few instructions away);
-  // the wait yields with nanosleep so a claiming lane of the same warp progresses.
-  // (No fence: the pool words were zeroed before the launch; the claimer only
-  // publishes an offset.)
-  while (d == 0) {
-    __nanosleep(32);
-    d = __ldcg(&a.T.slots[2 * s + 1]);
-  }
-  if (d == ~0ull) return;   // no domains in this pass (pool exhausted / another chunk)
-  // instances: counted in the one pass that carves the slot's domains
-  if (a.T.inst) atomicAdd(&a.T.inst[s], 1ull);
+// OR the bits of the local vertices in `only` (bit i: local vertex i) into the domains
+// (base offset d) at every position a minimizing order gives them.
+__device__ __forceinline__ void record_bits(const FpmArgs &a, const uint32_t *prm, const Canon &cn,
+                                            unsigned long long d, uint32_t k0, uint32_t k1, uint32_t k2, uint32_t k3,
+                                            uint32_t nv, uint32_t only) {
   uint64_t off[4];
   off[0] = d - 1;
   off[1] = off[0] + __ldg(a.cwords + key_label(cn.key, 0));
@@ -269,19 +259,62 @@ __device__ void record(const FpmArgs &a, const uint2 *tab, const uint32_t *prm, 
     const uint32_t sg = prm[r];
     uint32_t *w[4];
     uint32_t bb[4], x[4];
+    bool on[4];
 #pragma unroll
     for (uint32_t c = 0; c < 4; c++) {
       const uint32_t sp = (sg >> (2 * c)) & 3u;            // sorted position placed at canonical c
-      const uint32_t bit = pick4((cn.ordw >> (2 * sp)) & 3u, k0, k1, k2, k3);
+      const uint32_t lv = (cn.ordw >> (2 * sp)) & 3u;      // its local vertex
+      const uint32_t bit = pick4(lv, k0, k1, k2, k3);
       w[c] = a.T.pool + off[c] + (bit >> 5);
       bb[c] = 1u << (bit & 31);
+      on[c] = c < nv && ((only >> lv) & 1u);
     }
 #pragma unroll
-    for (uint32_t c = 0; c < 4; c++) x[c] = c < nv ? __ldcg(w[c]) : ~0u;
+    for (uint32_t c = 0; c < 4; c++) x[c] = on[c] ? __ldcg(w[c]) : ~0u;
 #pragma unroll
     for (uint32_t c = 0; c < 4; c++)
       if (!(x[c] & bb[c])) atomicOr(w[c], bb[c]);
   }
+}
+
+// Record one embedding: its canonical code, the pattern slot (claimed on first sight),
+// then the domain bits of every local vertex.  Returns the slot's domain offset d
+// (0: no slot, the table is full; ~0: no domains in this pass).
+__device__ unsigned long long record(const FpmArgs &a, const uint2 *tab, const uint32_t *prm, uint32_t k0,
+                                     uint32_t k1, uint32_t k2, uint32_t k3, uint32_t l0, uint32_t l1, uint32_t l2,
+                                     uint32_t l3, uint32_t nv, uint32_t em) {
+  const Canon cn = canonical(tab, l0, l1, l2, l3, nv, em);
+  unsigned long long d = 0;
+  const int64_t s = table_slot(a, cn.key, true, d);
+  if (s < 0) return 0;
+  // the claimer may still be carving this slot's domains (a few instructions away);
+  // the wait yields with nanosleep so a claiming lane of the same warp progresses.
+  // (No fence: the pool words were zeroed before the launch; the claimer only
+  // publishes an offset.)
+  while (d == 0) {
+    __nanosleep(32);
+    d = __ldcg(&a.T.slots[2 * s + 1]);
+  }
+  if (d == ~0ull) return d;   // no domains in this pass (pool exhausted / another chunk)
+  // instances: counted in the one pass that carves the slot's domains
+  if (a.T.inst) atomicAdd(&a.T.inst[s], 1ull);
+  record_bits(a, prm, cn, d, k0, k1, k2, k3, nv, 0xfu);
+  return d;
+}
+
+// Level-3 memo (per warp, per window of prefixes): (prefix j, edge mask, label of the
+// new vertex) -> the slot's domain offset.  Two embeddings with the same key have the
+// same labels and edges, hence the same canonical code, slot and minimizing orders:
+// the prefix's vertices u, v, y land on the same positions, so the later one only adds
+// its new vertex z -- no slot lookup and three of four domain words skipped (a hub
+// prefix has hundreds of z, its labels repeat).  Entry: key << 40 | d (d < 2^40; the
+// all-ones low part stands for "no domains in this pass"); one 64-bit word, so a
+// concurrent overwrite by a colliding key never tears.
+constexpr int kMemoBits = 7;   // 128 entries (1 KB) per warp
+constexpr uint64_t kMemoD = (1ull << 40) - 1;
+
+__device__ __forceinline__ uint32_t memo_key(uint32_t j, uint32_t em, uint32_t l3) {
+  return 1u | (j << 1) | (em << 6) | (l3 << 12);   // 24 bits (labels < 4096, em < 64, j < 32)
 }
 
 // Is the pattern of this (prefix) edge set frequent?  (Alg. 2 line 4 pruning)
@@ -304,10 +337,13 @@ __device__ __forceinline__ bool frequent(const FpmArgs &a, const uint2 *tab, uin
 __global__ void __launch_bounds__(kThreads) fpm_enum_kernel(FpmArgs a) {
   __shared__ uint2 s_tab[kCanonEntries];
   __shared__ uint32_t s_prm[24];
+  __shared__ unsigned long long s_memo[kThreads / 32][1 << kMemoBits];
   for (int i = threadIdx.x; i < kCanonEntries; i += blockDim.x) s_tab[i] = a.canon_tab[i];
   if (threadIdx.x < 24) s_prm[threadIdx.x] = a.perm_tab[threadIdx.x];
   __syncthreads();
   const int lane = threadIdx.x & 31;
+  unsigned long long *memo = s_memo[threadIdx.x >> 5];
+  const bool use_memo = a.level == 3 && a.T.inst == nullptr && GAMMA_FPM_MEMO;   // (instance counts need every record)
   uint64_t emb = 0, elems = 0;       // embeddings recorded; adjacency elements streamed (lane 0)
   const uint64_t ndir = a.rp[a.n];   // directed edges: the roots are the (u, v > u) ones
   constexpr uint64_t kBatch = 8;
@@ -352,6 +388,12 @@ __global__ void __launch_bounds__(kThreads) fpm_enum_kernel(FpmArgs a) {
       const uint64_t nu = ue - us, ncand = nu + (ve - vs);
       if (lane == 0) elems += ncand;
       for (uint64_t c0 = 0; c0 < ncand; c0 += 32) {
+        if (use_memo) {   // the memo's prefix indices are this window's
+          __syncwarp();   // every lane is done with the previous window's entries
+#pragma unroll
+          for (int q = 0; q < (1 << kMemoBits) / 32; q++) memo[lane + 32 * q] = 0ull;
+          __syncwarp();
+        }
         const uint64_t ci = c0 + lane;
         // lane's second edge e2 = (x, y), x in {u, v}: a candidate prefix {e1, e2}
         bool valid = ci < ncand;
@@ -442,9 +484,25 @@ __global__ void __launch_bounds__(kThreads) fpm_enum_kernel(FpmArgs a) {
           const uint32_t em3 = (pl >> 16) | (1u << pid(lw, lz));
           const uint32_t l3 = lz == 3 ? labof(a, z) : 0u;
           if (lz == 3 && l3 < a.walk_lo) continue;
-          record(a, s_tab, s_prm, ku, kv, pky, lz == 3 ? __ldg(a.lrank + z) : 0u, lu, lv, pl & 0xffffu, l3,
-                 lz == 3 ? 4 : 3, em3);
+          const uint32_t kz = lz == 3 ? __ldg(a.lrank + z) : 0u;
           emb++;
+          if (use_memo) {
+            const uint32_t mk = memo_key((uint32_t)j, em3, l3);
+            const uint32_t mh = (mk * 0x9E3779B1u) >> (32 - kMemoBits);
+            const unsigned long long me = memo[mh];
+            if ((uint32_t)(me >> 40) == mk) {   // seen: only the new vertex's bits
+              const unsigned long long dd = me & kMemoD;
+              if (dd != kMemoD && lz == 3)
+                record_bits(a, s_prm, canonical(s_tab, lu, lv, pl & 0xffffu, l3, 4, em3), dd, 0u, 0u, 0u, kz, 4,
+                            0x8u);
+              continue;
+            }
+            const unsigned long long dd = record(a, s_tab, s_prm, ku, kv, pky, kz, lu, lv, pl & 0xffffu, l3,
+                                                 lz == 3 ? 4 : 3, em3);
+            if (dd) memo[mh] = ((unsigned long long)mk << 40) | (dd == ~0ull ? kMemoD : dd);
+            continue;
+          }
+          record(a, s_tab, s_prm, ku, kv, pky, kz, lu, lv, pl & 0xffffu, l3, lz == 3 ? 4 : 3, em3);
         }
       }
     }
