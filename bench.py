@@ -520,7 +520,7 @@ def run_gamma(args):
         launches = max(1, cand[dom]["launches"])
         per_launch_ms = cand[dom]["ms"] / launches
         summed_ms = sum(v["ms"] for v in cand.values())
-        concurrent = summed_ms > total_ms * 1.02   # SM batch: level chains overlap on side streams
+        concurrent = summed_ms > total_ms * 1.02   # SM batch chains / kCL team launches overlap on side streams
         if concurrent:
             # overlapping launches each see part of the GPU, so their event durations
             # overstate the time the class holds it: charge the class its share of the
@@ -558,7 +558,7 @@ def run_gamma(args):
                 "kernel_counted_bytes_per_launch": kernel_bytes,
                 "ms_per_launch": per_launch_ms, "launches_per_step": launches / args.steps,
                 "share_of_step": cand[dom]["ms"] / (summed_ms if concurrent else total_ms),
-                **({"timing_basis": "concurrent launches (SM batch side streams): ms_per_launch = step time x the "
+                **({"timing_basis": "concurrent launches (side streams: SM batch chains, kCL warp and CTA teams): ms_per_launch = step time x the "
                                     "class's share of the summed kernel time / its launches"} if concurrent else {}),
                 "traffic_source": traffic_src,
                 "issue": issue_roofline(args.workload, dom, per_launch_ms, clk)}

@@ -174,6 +174,7 @@ enum {
   CTRL_AUX0 = 8,
   CTRL_AUX1 = 9,
   CTRL_AUX2 = 10,
+  CTRL_WORK2 = 11,    // a second work counter (a launch running concurrently with another)
   CTRL_MULTI = 16,    // CTRL_MULTI + s: number of s-cliques (gamma_kclique_multi), s <= 32
   CTRL_LEVELS = 64,   // CTRL_LEVELS + CTRL_LSTRIDE * d: a per-level control block (same word
   CTRL_LSTRIDE = 16,  // offsets as above) for launch chains read back once (match.cu)

@@ -121,6 +121,7 @@ struct BmArgs {
   uint64_t wide_stride;
   const uint64_t *row_ptr;    // symmetric CSR offsets (degrees of the orientation order);
                               // nullptr in rank space, where the id order is that order
+  unsigned long long *work;   // this launch's work cursor (its own word when launches run concurrently)
 };
 
 __device__ __forceinline__ uint32_t excl_scan32(uint32_t x, int lane, uint32_t &total) {
@@ -1119,7 +1120,7 @@ __global__ void GAMMA_BM_BOUNDS(KM) kcl_bitmap_kernel(BmArgs a) {
   for (;;) {
     if (next == end) {
       unsigned long long base = 0;
-      if (tid == 0) base = atomicAdd(&a.ctrl[CTRL_WORK], kBatch);
+      if (tid == 0) base = atomicAdd(a.work, kBatch);
       if (TEAM_WARPS == 1) {
         base = __shfl_sync(0xffffffffu, base, 0);
         if ((unsigned long long)lane < kBatch && base + lane < a.nroots) {
@@ -1312,7 +1313,7 @@ __global__ void GAMMA_BM_BOUNDS(KM) kcl_bitmap_parts_kernel(BmArgs a) {
       // the part list was filled by the previous launch; its length (<= parts_cap,
       // every slot below it written) sits in ctrl
       const unsigned long long nparts_total = *(volatile unsigned long long *)&a.ctrl[CTRL_AUX1];
-      const unsigned long long w = atomicAdd(&a.ctrl[CTRL_WORK], 1ull);
+      const unsigned long long w = atomicAdd(a.work, 1ull);
       m.slot[0] = w < nparts_total ? (uint32_t)w : 0xffffffffu;
     }
     __syncthreads();
@@ -1497,7 +1498,7 @@ __global__ void __launch_bounds__(kWideThreads) kcl_wide_kernel(BmArgs a) {
   uint64_t mc[kMaxStack + 3] = {};
   for (;;) {
     if (tid == 0) {
-      const unsigned long long w = atomicAdd(&a.ctrl[CTRL_WORK], 1ull);
+      const unsigned long long w = atomicAdd(a.work, 1ull);
       slot[0] = w < a.nroots ? (uint32_t)w : 0xffffffffu;
       slot[1] = 0;   // row cursor
     }
@@ -1585,7 +1586,7 @@ void enqueue_wide_km(gamma_ctx *ctx, BmArgs a, bool per_root, uint32_t max_len, 
   const uint64_t g = std::min<uint64_t>(grid, a.nroots);
   rows = DevBuf<uint32_t>(ctx, g * a.wide_stride);
   a.wide_rows = rows.p;
-  GAMMA_CUDA(cudaMemsetAsync(ctx->ctrl + CTRL_WORK, 0, sizeof(uint64_t), ctx->stream));
+  GAMMA_CUDA(cudaMemsetAsync(a.work, 0, sizeof(uint64_t), ctx->stream));
   ctx->launch(KC_BITMAP, [&] {
     if (per_root)
       kcl_wide_kernel<WL, true, KM, PAGED><<<(unsigned)g, kWideThreads, wide_smem<WL>(), ctx->stream>>>(a);
@@ -1614,7 +1615,7 @@ constexpr size_t bm_smem() {
 // Enqueue one team kind over a root range (no host round trip: the work counter is
 // reset on the stream, the counts accumulate in ctrl and are read once at the end).
 template <int TEAM_WARPS, int TW, int KM, bool PAGED>
-void enqueue_bitmap_km(gamma_ctx *ctx, const BmArgs &a0, bool per_root) {
+void enqueue_bitmap_km(gamma_ctx *ctx, const BmArgs &a0, bool per_root, cudaStream_t st) {
   static bool attr = false;
   if (!attr) {
     GAMMA_CUDA(cudaFuncSetAttribute(kcl_bitmap_kernel<TEAM_WARPS, TW, false, KM, PAGED>,
@@ -1627,24 +1628,24 @@ void enqueue_bitmap_km(gamma_ctx *ctx, const BmArgs &a0, bool per_root) {
   static int grid = 0;
   if (!grid)
     grid = ctx->num_sms * occupancy_blocks((const void *)kcl_bitmap_kernel<TEAM_WARPS, TW, false, KM, PAGED>, 256, smem);
-  GAMMA_CUDA(cudaMemsetAsync(ctx->ctrl + CTRL_WORK, 0, sizeof(uint64_t), ctx->stream));
-  ctx->launch(KC_BITMAP, [&] {
+  GAMMA_CUDA(cudaMemsetAsync(a0.work, 0, sizeof(uint64_t), st));
+  ctx->launch_on(KC_BITMAP, st, [&] {
     if (per_root)
-      kcl_bitmap_kernel<TEAM_WARPS, TW, true, KM, PAGED><<<grid, 256, smem, ctx->stream>>>(a0);
+      kcl_bitmap_kernel<TEAM_WARPS, TW, true, KM, PAGED><<<grid, 256, smem, st>>>(a0);
     else
-      kcl_bitmap_kernel<TEAM_WARPS, TW, false, KM, PAGED><<<grid, 256, smem, ctx->stream>>>(a0);
+      kcl_bitmap_kernel<TEAM_WARPS, TW, false, KM, PAGED><<<grid, 256, smem, st>>>(a0);
   });
 }
 
 template <int TEAM_WARPS, int TW>
-void enqueue_bitmap(gamma_ctx *ctx, const BmArgs &a0, bool per_root) {
+void enqueue_bitmap(gamma_ctx *ctx, const BmArgs &a0, bool per_root, cudaStream_t st) {
   const bool paged = a0.dag_col.pages != nullptr;
   if (a0.k <= 6) {
-    if (paged) enqueue_bitmap_km<TEAM_WARPS, TW, 6, true>(ctx, a0, per_root);
-    else enqueue_bitmap_km<TEAM_WARPS, TW, 6, false>(ctx, a0, per_root);
+    if (paged) enqueue_bitmap_km<TEAM_WARPS, TW, 6, true>(ctx, a0, per_root, st);
+    else enqueue_bitmap_km<TEAM_WARPS, TW, 6, false>(ctx, a0, per_root, st);
   } else {
-    if (paged) enqueue_bitmap_km<TEAM_WARPS, TW, kBitmapMaxK, true>(ctx, a0, per_root);
-    else enqueue_bitmap_km<TEAM_WARPS, TW, kBitmapMaxK, false>(ctx, a0, per_root);
+    if (paged) enqueue_bitmap_km<TEAM_WARPS, TW, kBitmapMaxK, true>(ctx, a0, per_root, st);
+    else enqueue_bitmap_km<TEAM_WARPS, TW, kBitmapMaxK, false>(ctx, a0, per_root, st);
   }
 }
 
@@ -1661,7 +1662,7 @@ void enqueue_parts_km(gamma_ctx *ctx, const BmArgs &a0, bool per_root) {
   static int pgrid = 0;
   if (!pgrid)
     pgrid = ctx->num_sms * occupancy_blocks((const void *)kcl_bitmap_parts_kernel<false, KM>, 256, bm_smem<8, 16>());
-  GAMMA_CUDA(cudaMemsetAsync(ctx->ctrl + CTRL_WORK, 0, sizeof(uint64_t), ctx->stream));
+  GAMMA_CUDA(cudaMemsetAsync(a0.work, 0, sizeof(uint64_t), ctx->stream));
   ctx->launch(KC_BITMAP, [&] {
     if (per_root)
       kcl_bitmap_parts_kernel<true, KM><<<pgrid, 256, bm_smem<8, 16>(), ctx->stream>>>(a0);
@@ -1737,6 +1738,30 @@ uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint6
     n_mid = std::min(n_mid, nroots);
   }
   ctrl_reset(ctx);
+  a.work = reinterpret_cast<unsigned long long *>(ctx->ctrl) + CTRL_WORK;
+  const bool cta = g->max_out_degree > 128 && (!sorted || n_mid > n_long);
+  const bool warp = !sorted || nroots > n_mid;
+  const char *bands = getenv("GAMMA_KCL_BANDS");   // diagnostics: one warp-team launch per |R| band
+  const bool banded = sorted && bands && *bands && *bands != '0' && g->root_order == roots;
+  // The warp-team launch runs on a side stream beside the CTA-team launch (their tails
+  // overlap), taking its roots from its own work cursor; the hub parts follow both.
+  // (GAMMA_KCL_SERIAL=1: one stream.  Warp teams expanding their heavy roots themselves
+  // so that the parts could overlap them too cost C2 6.1 -> 9.2 ms/step.)
+  static const bool serial_env = [] {
+    const char *e = getenv("GAMMA_KCL_SERIAL");
+    return e && *e && *e != '0';
+  }();
+  const bool conc = cta && warp && !banded && !serial_env;
+  cudaEvent_t fork = nullptr, join = nullptr;
+  cudaStream_t wst = ctx->stream;
+  if (conc) {
+    ctx->side_init();
+    wst = ctx->side_streams[0];
+    GAMMA_CUDA(cudaEventCreateWithFlags(&fork, cudaEventDisableTiming));
+    GAMMA_CUDA(cudaEventCreateWithFlags(&join, cudaEventDisableTiming));
+    GAMMA_CUDA(cudaEventRecord(fork, ctx->stream));   // after the control block reset
+    GAMMA_CUDA(cudaStreamWaitEvent(wst, fork, 0));
+  }
   // wide runs, [n_xl, n_long): 512 < |R| <= 2048 with 2 words per lane, longer with 8
   DevBuf<uint32_t> rows_a, rows_b;
   if (g->max_out_degree > kBitmapMaxRun && (!sorted || n_long > n_xl)) {
@@ -1755,34 +1780,41 @@ uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint6
   }
   a.len_lo = 128;
   a.len_hi = 512;
-  if (g->max_out_degree > 128 && (!sorted || n_mid > n_long)) {
+  if (cta) {
     a.roots = roots + (sorted ? n_long : 0);
     a.root_base = sorted ? n_long : 0;
     a.nroots = sorted ? n_mid - n_long : nroots;
-    enqueue_bitmap<8, 16>(ctx, a, per_root != nullptr);
+    enqueue_bitmap<8, 16>(ctx, a, per_root != nullptr, ctx->stream);
   }
   a.len_lo = 0;
   a.len_hi = 128;
-  if (!sorted || nroots > n_mid) {
-    a.roots = roots + (sorted ? n_mid : 0);
-    a.root_base = sorted ? n_mid : 0;
-    a.nroots = sorted ? nroots - n_mid : nroots;
-    const char *bands = getenv("GAMMA_KCL_BANDS");   // diagnostics: one warp-team launch per |R| band
-    if (sorted && bands && *bands && *bands != '0' && g->root_order == roots) {
+  if (warp) {
+    BmArgs aw = a;
+    aw.roots = roots + (sorted ? n_mid : 0);
+    aw.root_base = sorted ? n_mid : 0;
+    aw.nroots = sorted ? nroots - n_mid : nroots;
+    if (conc) aw.work = reinterpret_cast<unsigned long long *>(ctx->ctrl) + CTRL_WORK2;
+    if (banded) {
       const uint32_t thr[] = {129, 65, 33, 17, 9, 0};
       for (int b = 0; b + 1 < 6; b++) {
         const uint64_t lo = std::max<uint64_t>(n_mid, thr[b] < g->root_ge.size() ? g->root_ge[thr[b]] : 0);
         const uint64_t hi = std::min<uint64_t>(nroots, thr[b + 1] < g->root_ge.size() ? g->root_ge[thr[b + 1]] : 0);
         if (hi <= lo) continue;
-        BmArgs ab = a;
+        BmArgs ab = aw;
         ab.roots = roots + lo;
         ab.root_base = lo;
         ab.nroots = hi - lo;
-        enqueue_bitmap<1, 4>(ctx, ab, per_root != nullptr);
+        enqueue_bitmap<1, 4>(ctx, ab, per_root != nullptr, ctx->stream);
       }
     } else {
-      enqueue_bitmap<1, 4>(ctx, a, per_root != nullptr);
+      enqueue_bitmap<1, 4>(ctx, aw, per_root != nullptr, wst);
     }
+  }
+  if (conc) {   // join: the parts read the part lists of both team launches
+    GAMMA_CUDA(cudaEventRecord(join, wst));
+    GAMMA_CUDA(cudaStreamWaitEvent(ctx->stream, join, 0));
+    cudaEventDestroy(fork);
+    cudaEventDestroy(join);
   }
   if (split) {
     // parts carry absolute indices into the full root list
