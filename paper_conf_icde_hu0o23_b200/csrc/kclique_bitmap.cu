@@ -1746,7 +1746,9 @@ uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint6
   // The warp-team launch runs on a side stream beside the CTA-team launch (their tails
   // overlap), taking its roots from its own work cursor; the hub parts follow both.
   // (GAMMA_KCL_SERIAL=1: one stream.  Warp teams expanding their heavy roots themselves
-  // so that the parts could overlap them too cost C2 6.1 -> 9.2 ms/step.)
+  // so that the parts could overlap them too cost C2 6.1 -> 9.2 ms/step; a separate
+  // launch for runs of 65..128, so that the parts could overlap the runs <= 64, 7.15:
+  // the light runs no longer filled the heavy runs' tail.)
   static const bool serial_env = [] {
     const char *e = getenv("GAMMA_KCL_SERIAL");
     return e && *e && *e != '0';
