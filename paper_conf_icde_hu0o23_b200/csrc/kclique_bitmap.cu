@@ -1724,6 +1724,10 @@ uint64_t kclique_bitmap(gamma_graph *g, uint32_t k, const uint32_t *roots, uint6
     parts = DevBuf<uint2>(ctx, a.parts_cap);
     a.parts = parts.p;
     a.part_cost = k >= 6 ? kPartCost : 4 * kPartCost;
+    {   // GAMMA_KCL_PART_COST: 4-cliques per hub part (A/B knob)
+      const char *pc = getenv("GAMMA_KCL_PART_COST");
+      if (pc && *pc) a.part_cost = (uint32_t)std::max(64ul, std::min(strtoul(pc, nullptr, 10), 1ul << 24));
+    }
     a.heavy_cut = (ctx->desc.flags & GAMMA_FLAG_DEBUG_SPLIT_ALL) ? 1 : 4ull * a.part_cost;
     a.root_rows_cap = std::min<uint32_t>(a.parts_cap, 2048);
     root_rows = DevBuf<uint32_t>(ctx, (uint64_t)a.root_rows_cap * kSlotWords);
