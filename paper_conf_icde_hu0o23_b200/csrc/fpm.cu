@@ -33,6 +33,7 @@
 #include <cub/device/device_select.cuh>
 
 #include <algorithm>
+#include <thread>
 #include <cstdio>
 #include <cstdlib>
 #include <array>
@@ -701,6 +702,52 @@ static void slots_get(gamma_ctx *ctx, std::vector<unsigned long long> &h, const 
 static void slots_put(gamma_ctx *ctx, unsigned long long *slots, const std::vector<unsigned long long> &h,
                       uint64_t cap, int colm) {
   GAMMA_CUDA(cudaMemcpy2DAsync(slots + colm, 16, h.data(), 8, 8, cap, cudaMemcpyHostToDevice, ctx->stream));
+}
+
+// Host-side parallel helpers for the result (C4: 1.2e6 patterns; one thread took 280 ms
+// to decode and sort them).  f(i0, i1) over [0, n) in contiguous chunks.
+static unsigned host_threads(size_t n) {
+  const unsigned hw = std::max(1u, std::thread::hardware_concurrency());
+  return n < (1u << 15) ? 1u : std::min(16u, hw);
+}
+
+template <class F>
+static void par_for(size_t n, F &&f) {
+  const unsigned T = host_threads(n);
+  if (T <= 1) {
+    f(0, n);
+    return;
+  }
+  std::vector<std::thread> th;
+  for (unsigned t = 0; t < T; t++) th.emplace_back([&, t] { f(n * t / T, n * (t + 1) / T); });
+  for (auto &x : th) x.join();
+}
+
+// sort = chunk sorts on host threads, then pairwise merges
+template <class V>
+static void par_sort(V &v) {
+  const size_t n = v.size();
+  unsigned P = 1;
+  while (P * 2 <= host_threads(n)) P *= 2;
+  if (P <= 1) {
+    std::sort(v.begin(), v.end());
+    return;
+  }
+  std::vector<size_t> b(P + 1);
+  for (unsigned i = 0; i <= P; i++) b[i] = n * i / P;
+  {
+    std::vector<std::thread> th;
+    for (unsigned i = 0; i < P; i++) th.emplace_back([&, i] { std::sort(v.begin() + b[i], v.begin() + b[i + 1]); });
+    for (auto &x : th) x.join();
+  }
+  for (unsigned w = 1; w < P; w *= 2) {
+    std::vector<std::thread> th;
+    for (unsigned i = 0; i + w < P; i += 2 * w)
+      th.emplace_back([&, i, w] {
+        std::inplace_merge(v.begin() + b[i], v.begin() + b[i + w], v.begin() + b[std::min(i + 2 * w, P)]);
+      });
+    for (auto &x : th) x.join();
+  }
 }
 
 static gamma_fpm_pattern decode_pattern(uint64_t key, uint64_t support, uint64_t instances = 0) {
@@ -1578,24 +1625,36 @@ static void fpm_run(gamma_graph *g, uint32_t max_edges, uint64_t minsup, std::ve
     if (want_inst) GAMMA_CUDA(cudaMemcpyAsync(hinst.data(), ci.p, nf * 8, cudaMemcpyDeviceToHost, ctx->stream));
     ctx->sync();
   }
-  for (uint64_t i = 0; i < nf; i++) out.push_back(decode_pattern(hkey[i], hsup[i], want_inst ? hinst[i] : 0));
+  {   // decode (parallel over host threads: 1.2e6 patterns on C4)
+    const size_t base = out.size();
+    out.resize(base + nf);
+    par_for(nf, [&](size_t i0, size_t i1) {
+      for (size_t i = i0; i < i1; i++) out[base + i] = decode_pattern(hkey[i], hsup[i], want_inst ? hinst[i] : 0);
+    });
+  }
   out.insert(out.end(), found_last.begin(), found_last.end());
   out.insert(out.end(), found4.begin(), found4.end());
-  // sort key: (ne, nv, labels in canonical order, edge pairs) packed in 128 bits
+  // sort key: (ne, nv, labels in canonical order, edge pairs) packed in 128 bits (unique
+  // per pattern, so any sort gives the same order)
   std::vector<std::pair<std::pair<uint64_t, uint64_t>, uint32_t>> order(out.size());
-  for (size_t i = 0; i < out.size(); i++) {
-    const gamma_fpm_pattern &x = out[i];
-    uint64_t lab60 = 0;   // five 12-bit labels (labels < 4096), canonical order
-    for (uint32_t j = 0; j < 5; j++) lab60 = lab60 << 12 | (j < x.nv ? x.labels[j] & 0xfffu : 0u);
-    uint64_t ek = 0;      // four edges, 3 + 3 bits each
-    for (uint32_t e = 0; e < 4; e++) ek = ek << 6 | (e < x.ne ? (uint64_t)(x.edges[e][0] << 3 | x.edges[e][1]) : 0u);
-    const uint64_t hi = (uint64_t)x.ne << 61 | (uint64_t)x.nv << 58 | (lab60 >> 2);
-    const uint64_t lo = (lab60 & 3u) << 62 | ek;
-    order[i] = {{hi, lo}, (uint32_t)i};
-  }
-  std::sort(order.begin(), order.end());
+  par_for(out.size(), [&](size_t i0, size_t i1) {
+    for (size_t i = i0; i < i1; i++) {
+      const gamma_fpm_pattern &x = out[i];
+      uint64_t lab60 = 0;   // five 12-bit labels (labels < 4096), canonical order
+      for (uint32_t j = 0; j < 5; j++) lab60 = lab60 << 12 | (j < x.nv ? x.labels[j] & 0xfffu : 0u);
+      uint64_t ek = 0;      // four edges, 3 + 3 bits each
+      for (uint32_t e = 0; e < 4; e++)
+        ek = ek << 6 | (e < x.ne ? (uint64_t)(x.edges[e][0] << 3 | x.edges[e][1]) : 0u);
+      const uint64_t hi = (uint64_t)x.ne << 61 | (uint64_t)x.nv << 58 | (lab60 >> 2);
+      const uint64_t lo = (lab60 & 3u) << 62 | ek;
+      order[i] = {{hi, lo}, (uint32_t)i};
+    }
+  });
+  par_sort(order);
   std::vector<gamma_fpm_pattern> sorted(out.size());
-  for (size_t i = 0; i < out.size(); i++) sorted[i] = out[order[i].second];
+  par_for(out.size(), [&](size_t i0, size_t i1) {
+    for (size_t i = i0; i < i1; i++) sorted[i] = out[order[i].second];
+  });
   out.swap(sorted);
   plog.mark("collect + sort");
   ctx->collect_timings();
