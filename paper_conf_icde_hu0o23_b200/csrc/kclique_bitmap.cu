@@ -46,6 +46,10 @@ namespace {
 #ifndef GAMMA_KCL_LEAF_BAL
 #define GAMMA_KCL_LEAF_BAL 0
 #endif
+#ifndef GAMMA_KCL_TILES   // streamed row build: 32-element tiles whose loads are in flight together
+                          // (C2 same box: 2 tiles 5.65 ms/step, 4 5.59, 8 5.83)
+#define GAMMA_KCL_TILES 4
+#endif
 #ifndef GAMMA_KCL_PAIR_U   // rows per lane group whose pair searches run in lock step
 #define GAMMA_KCL_PAIR_U 2
 #endif
@@ -936,7 +940,7 @@ __device__ uint64_t build_rows_p(const BmArgs &a, uint32_t *R, unsigned short *H
     uint32_t nb = 0;   // lists that started before this tile
     // kTiles tiles of 32 elements per step: their loads are issued back to back
     // before any probe, so each lane keeps several L2 gathers in flight
-    constexpr int kTiles = 4;
+    constexpr int kTiles = GAMMA_KCL_TILES;
     for (uint32_t t0 = 0; t0 < T; t0 += 32 * kTiles) {
       // tiles that hold elements (warp-uniform): a short window runs 1-3 tiles, not 4
       // (the padded tiles were ~half the row-build instructions on C2's small roots)
