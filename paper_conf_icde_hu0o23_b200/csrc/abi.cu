@@ -87,15 +87,15 @@ void *gamma_ctx::keep_take(size_t bytes, size_t &got) {
   return alloc(bytes);
 }
 
-// Kept bytes are capped at a quarter of the device memory: beyond it a returned buffer
-// is freed instead.  (Round 1's 8 GiB held a fraction of a batched SM call's tables --
+// Kept bytes are capped at an eighth of the device memory: beyond it a returned buffer
+// is freed instead (an idle context must not starve other processes on the GPU).  (Round 1's 8 GiB held a fraction of a batched SM call's tables --
 // eight level chains of up to three levels -- so every C3 step re-allocated most of
 // them through the caching allocator.)
 void gamma_ctx::keep_give(void *p, size_t bytes) {
   if (!p) return;
   size_t held = 0;
   for (auto &b : kept) held += b.second;
-  if (held + bytes > mem_total / 4) {
+  if (held + bytes > mem_total / 8) {
     free(p);
     return;
   }

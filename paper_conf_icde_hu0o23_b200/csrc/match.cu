@@ -818,12 +818,10 @@ struct SmRun {
   uint32_t big_scratch_cap = 0;
 
   // First table size of a level (grow caps it at the level's share of the HBM budget):
-  // 2^29 entry slots, 2^26 group descriptors.  Slots run well ahead of the entries
-  // written: a child whose run may exceed the warp's staging buffer reserves its upper
-  // bound (the shortest list involved) and keeps what survives (C3, 4-cycle, labels
-  // i mod 8, GAMMA_DEBUG: the pool cursor at 2.8e8 slots for 5.1e7 entries).  Round 1's
-  // 2^24 overflowed there in every call, so the one-read-back chain was thrown away and
-  // the query rerun on the careful per-level path.
+  // 2^27 entry slots and 2^23 group descriptors (C3's widest level: 5.1e7 entries, under
+  // 2e6 groups).  Round 1's 2^24 overflowed on C3's 4-cycle in every call (the pool cursor
+  // ran to 2.8e8 slots while runs reserved upper bounds and abandoned block tails), so
+  // the one-read-back chain was thrown away and the query rerun on the careful path.
   uint64_t initial_cap() const {
     return std::max<uint64_t>(1ull << GAMMA_SM_CAP_LOG2, 4ull * kBlkV * kWarps * (uint64_t)grid);
   }
@@ -929,7 +927,7 @@ struct SmRun {
   void chain_enqueue(uint64_t ngroups, cudaStream_t st, unsigned long long *ctrl, uint64_t *host) {
     const uint32_t nl = P.nv - 1;   // launches: d = 0 .. nv-2
     for (uint32_t q = 1; q < nl; q++)
-      if (lv[q].cap_v == 0) grow(q, initial_cap(), 1ull << 26);
+      if (lv[q].cap_v == 0) grow(q, initial_cap(), 1ull << 23);
     GAMMA_CUDA(cudaMemsetAsync(ctrl, 0, CTRL_WORDS * sizeof(uint64_t), st));
     for (uint32_t d = 0; d < nl; d++) {
       const uint32_t q = d + 1;
@@ -1004,7 +1002,7 @@ struct SmRun {
     }
     for (;;) {
       SmLevel &L = lv[q];
-      if (L.cap_v == 0) grow(q, initial_cap(), 1ull << 26);
+      if (L.cap_v == 0) grow(q, initial_cap(), 1ull << 23);
       SmArgs a = args(d, g0, g1);
       a.vid_out = L.vid.p;
       a.desc_out = L.desc.p;
@@ -1293,7 +1291,11 @@ static bool match_prepare(gamma_graph *g, const SmPlan &P, SmRun &R, uint64_t &c
   {
     size_t fr = 0, tot = 0;
     GAMMA_CUDA(cudaMemGetInfo(&fr, &tot));
-    const uint64_t budget = ctx->desc.hbm_budget_bytes ? ctx->desc.hbm_budget_bytes : (uint64_t)(fr * 0.8);
+    // (the context's kept buffers count as free: this call's tables take them back)
+    size_t kept = 0;
+    for (const auto &b : ctx->kept) kept += b.second;
+    const uint64_t budget =
+        ctx->desc.hbm_budget_bytes ? ctx->desc.hbm_budget_bytes : (uint64_t)((double)(fr + kept) * 0.8);
     R.level_share = budget / batch / std::max<uint32_t>(1, P.nv > 2 ? P.nv - 2 : 1);
   }
   // ---- roots (position 0) ----

@@ -46,7 +46,15 @@ def _worker(rank, world, port, q, budget):
 
 @pytest.mark.parametrize("budget", [0, 100 << 10])
 def test_two_ranks_gloo(oracle_mod, budget):
+    import gc
+
+    import torch
     import torch.multiprocessing as mp
+    # the two rank processes share this GPU and size FPM pools from its free memory:
+    # hand back what earlier tests of this process hold (contexts of finished modules,
+    # the caching allocator's idle blocks)
+    gc.collect()
+    torch.cuda.empty_cache()
     world = 2
     port = _free_port()
     ctx = mp.get_context("spawn")
